@@ -1,0 +1,188 @@
+"""Seeded synthetic inputs (graphs and timestamped update streams).
+
+The one module both the CUDA path's tests/bench and the oracle draw inputs
+from.  It holds none of the method's arithmetic: it only generates edge lists,
+vertex-ID lists and op streams from a counter-based generator (``synth.c``).
+See DESIGN.md "Input recipe" and SURVEY.md §8(d).
+"""
+from __future__ import annotations
+
+import ctypes
+import os
+import subprocess
+from dataclasses import dataclass
+
+import numpy as np
+
+_HERE = os.path.dirname(os.path.abspath(__file__))
+_SRC = os.path.join(_HERE, "synth.c")
+_LIB = os.path.join(_HERE, "libsynth.so")
+
+NODE_INSERT, NODE_DELETE, EDGE_INSERT, EDGE_DELETE, EDGE_WEIGHT = 0, 1, 2, 3, 4
+MASTER_SEED = 0x48325441  # master seed + config index
+
+
+def build(force: bool = False) -> str:
+    if force or not os.path.exists(_LIB) or os.path.getmtime(_LIB) < os.path.getmtime(_SRC):
+        subprocess.check_call(["gcc", "-O2", "-fopenmp", "-fPIC", "-shared", "-o", _LIB, _SRC])
+    return _LIB
+
+
+_lib = None
+
+
+def lib():
+    global _lib
+    if _lib is None:
+        build()
+        L = ctypes.CDLL(_LIB)
+        u64, i32, f64, P = ctypes.c_uint64, ctypes.c_int, ctypes.c_double, ctypes.c_void_p
+        L.synth_rand.restype = u64
+        L.synth_rand.argtypes = [u64, u64, u64]
+        L.synth_scramble.restype = u64
+        L.synth_scramble.argtypes = [i32, u64, u64]
+        L.synth_rmat_edges.argtypes = [i32, u64, u64, u64, P, P, P]
+        L.synth_rmat_batch.argtypes = [i32, u64, u64, u64, u64, f64, f64, f64, u64, u64,
+                                       P, P, P, P, P]
+        L.synth_ldbc_vertices.argtypes = [u64, u64, P]
+        L.synth_ldbc_edges.argtypes = [u64, u64, u64, u64, u64, u64, P, P, P]
+        L.synth_ldbc_batch.restype = u64
+        L.synth_ldbc_batch.argtypes = [u64, u64, u64, u64, u64, u64, i32, u64, P, P, P, P, P]
+        L.synth_fuzz_batch.argtypes = [u64, u64, u64, u64, P, u64, u64, P, P, P, P, P]
+        _lib = L
+    return _lib
+
+
+def _p(a: np.ndarray):
+    return ctypes.c_void_p(a.ctypes.data)
+
+
+@dataclass
+class Batch:
+    """SoA op batch (h2tap_batch layout): kind u8, src u64, dst u64, w f32, ts u64."""
+    kind: np.ndarray
+    src: np.ndarray
+    dst: np.ndarray
+    w: np.ndarray
+    ts: np.ndarray
+
+    def __len__(self) -> int:
+        return int(self.kind.shape[0])
+
+    @staticmethod
+    def empty(n: int = 0) -> "Batch":
+        return Batch(np.zeros(n, np.uint8), np.zeros(n, np.uint64), np.zeros(n, np.uint64),
+                     np.zeros(n, np.float32), np.zeros(n, np.uint64))
+
+    @staticmethod
+    def of(ops) -> "Batch":
+        """ops: iterable of (kind, src, dst, w, ts)."""
+        ops = list(ops)
+        b = Batch.empty(len(ops))
+        for i, (k, s, d, w, t) in enumerate(ops):
+            b.kind[i], b.src[i], b.dst[i], b.w[i], b.ts[i] = k, s, d, w, t
+        return b
+
+    def slice(self, sl) -> "Batch":
+        return Batch(self.kind[sl], self.src[sl], self.dst[sl], self.w[sl], self.ts[sl])
+
+    def concat(self, other: "Batch") -> "Batch":
+        return Batch(*(np.concatenate([a, b]) for a, b in zip(
+            (self.kind, self.src, self.dst, self.w, self.ts),
+            (other.kind, other.src, other.dst, other.w, other.ts))))
+
+    def nbytes(self) -> int:
+        return sum(a.nbytes for a in (self.kind, self.src, self.dst, self.w, self.ts))
+
+
+# ------------------------------------------------------------------ RMAT ----
+def rmat_edges(scale: int, seed: int, n: int | None = None, first: int = 0, weights: bool = True):
+    """Initial RMAT edge list (Graph500 A,B,C,D; scrambled labels; f32 weights)."""
+    if n is None:
+        n = 16 << scale
+    src = np.empty(n, np.uint64)
+    dst = np.empty(n, np.uint64)
+    w = np.empty(n, np.float32) if weights else None
+    lib().synth_rmat_edges(scale, seed, first, n, _p(src), _p(dst), _p(w) if weights else None)
+    return src, dst, w
+
+
+def rmat_batch(scale: int, seed: int, k: int, n: int, m_initial: int, p_insert: float = 0.8,
+               p_weight: float = 0.0, p_repeat: float = 0.0, ops_per_txn: int = 1,
+               ts_base: int = 0) -> Batch:
+    b = Batch.empty(n)
+    lib().synth_rmat_batch(scale, seed, k, n, m_initial, p_insert, p_weight, p_repeat,
+                           ops_per_txn, ts_base, _p(b.kind), _p(b.src), _p(b.dst), _p(b.w),
+                           _p(b.ts))
+    return b
+
+
+# ------------------------------------------------------------- LDBC-SNB ----
+@dataclass
+class LdbcShape:
+    n_person: int
+    n_msg: int
+    e_person: int
+
+    @property
+    def n_vertices(self) -> int:
+        return self.n_person + self.n_msg
+
+    @property
+    def n_edges(self) -> int:
+        return self.e_person + 4 * self.n_msg
+
+
+# SF10-shaped: ~30.0 M vertices, ~176.6 M directed edges, 65,536 Person hubs
+LDBC_SF10 = LdbcShape(n_person=65536, n_msg=30_000_000 - 65536,
+                      e_person=176_600_000 - 4 * (30_000_000 - 65536))
+
+
+def ldbc_vertices(shape: LdbcShape) -> np.ndarray:
+    ids = np.empty(shape.n_vertices, np.uint64)
+    lib().synth_ldbc_vertices(shape.n_person, shape.n_msg, _p(ids))
+    return ids
+
+
+def ldbc_edges(shape: LdbcShape, seed: int, first: int = 0, n: int | None = None):
+    if n is None:
+        n = shape.n_edges - first
+    src = np.empty(n, np.uint64)
+    dst = np.empty(n, np.uint64)
+    w = np.empty(n, np.float32)
+    lib().synth_ldbc_edges(shape.n_person, shape.n_msg, shape.e_person, seed, first, n,
+                           _p(src), _p(dst), _p(w))
+    return src, dst, w
+
+
+def ldbc_batch(shape: LdbcShape, seed: int, k: int, n_cap: int, lodeg: bool = False,
+               ts_base: int = 0) -> Batch:
+    b = Batch.empty(n_cap)
+    n = lib().synth_ldbc_batch(shape.n_person, shape.n_msg, shape.e_person, seed, k, n_cap,
+                               int(lodeg), ts_base, _p(b.kind), _p(b.src), _p(b.dst), _p(b.w),
+                               _p(b.ts))
+    return b.slice(slice(0, int(n)))
+
+
+# ------------------------------------------------------------------ fuzz ----
+def fuzz_batch(seed: int, k: int, n: int, n_ids: int, probs=(0.1, 0.05, 0.5, 0.2, 0.15),
+               ts_lo: int = 1, ts_span: int = 8) -> Batch:
+    b = Batch.empty(n)
+    p = np.asarray(probs, np.float64)
+    p = p / p.sum()
+    lib().synth_fuzz_batch(seed, k, n, n_ids, _p(p), ts_lo, ts_span, _p(b.kind), _p(b.src),
+                           _p(b.dst), _p(b.w), _p(b.ts))
+    return b
+
+
+# ----------------------------------------------------------- configs ----
+CONFIGS = {
+    # name: description (BASELINE.json configs[i]) and generator parameters
+    "c1": dict(index=0, kind="rmat", scale=16, edge_factor=16, batch=10_000, p_insert=0.8),
+    "c2": dict(index=1, kind="ldbc", shape=LDBC_SF10, batch=100_000),
+    "c3": dict(index=2, kind="rmat", scale=24, edge_factor=16, batch=1_000_000, p_insert=0.8),
+}
+
+
+def seed_of(name: str) -> int:
+    return MASTER_SEED + CONFIGS[name]["index"]

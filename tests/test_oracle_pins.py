@@ -1,0 +1,307 @@
+"""Pins for the oracle (CPU only): O1 is checked against things other than itself.
+
+* O2 brute force (independent implementation) on exhaustive and random tiny cases
+* the paper's Fig. 2 worked example (tests/golden/fig2.json)
+* a textbook CSR build (numpy lexsort + keep-last unique) for insert-only batches
+* invariants I1-I5 of a compact sorted CSR
+* algebraic properties: composition, deferral, permutation of distinct-ts ops
+* error codes and the strong guarantee
+"""
+import itertools
+import json
+import os
+
+import numpy as np
+import pytest
+
+import oracle
+import synth
+from oracle import O1, BruteForce
+from synth import Batch, NODE_INSERT, NODE_DELETE, EDGE_INSERT, EDGE_DELETE, EDGE_WEIGHT
+
+HERE = os.path.dirname(os.path.abspath(__file__))
+
+
+def same_export(a, b):
+    return all(np.array_equal(np.asarray(x), np.asarray(y)) for x, y in zip(a, b))
+
+
+def check_invariants(off, cols, w, ids):
+    V = len(ids)
+    assert len(off) == V + 1 and off[0] == 0 and off[-1] == len(cols) == len(w)  # I1
+    assert np.all(np.diff(off) >= 0)                                              # I1
+    assert np.all(cols < max(V, 1)) if len(cols) else True                         # I3
+    if V > 1:
+        assert np.all(np.diff(ids.astype(np.uint64)) > 0)                         # I4
+    for r in range(V):                                                             # I2
+        row = cols[off[r]:off[r + 1]].astype(np.int64)
+        assert np.all(np.diff(row) > 0)
+
+
+# ------------------------------------------------------------ Fig. 2 ----
+def test_fig2_worked_example():
+    g = json.load(open(os.path.join(HERE, "golden", "fig2.json")))
+    e = np.array(g["edges"], dtype=object)
+    o = O1.from_edges(len(g["vertices"]), np.array(g["vertices"], np.uint64),
+                      np.array(e[:, 0], np.uint64), np.array(e[:, 1], np.uint64),
+                      np.array(e[:, 2], np.float32), g["create_ts"])
+    rc, st = o.apply(Batch.of(g["ops"]), g["snapshot_ts"])
+    assert rc == 0 and st["n_visible"] == len(g["ops"])
+    off, cols, w, ids = o.export()
+    ex = g["expected"]
+    assert ids.tolist() == ex["ext_ids"]
+    assert off.tolist() == ex["offsets"]
+    assert cols.tolist() == ex["cols"]
+    assert w.tolist() == ex["weights"]
+
+
+# ------------------------------------------- exhaustive vs brute force ----
+def _all_ops(nv):
+    ops = []
+    for v in range(nv):
+        ops.append((NODE_INSERT, v, 0, 0.0))
+        ops.append((NODE_DELETE, v, 0, 0.0))
+    for u in range(nv):
+        for v in range(nv):
+            ops.append((EDGE_INSERT, u, v, 7.0))
+            ops.append((EDGE_DELETE, u, v, 0.0))
+            ops.append((EDGE_WEIGHT, u, v, 9.0))
+    return ops
+
+
+INIT_LIVE = [0, 1]           # vertex 2 never existed
+INIT_EDGES = [(0, 1, 1.0), (1, 1, 0.5), (1, 0, 2.0)]
+
+
+def _run_both(seq, ts, snapshot):
+    o = O1.from_edges(len(INIT_LIVE), np.array(INIT_LIVE, np.uint64),
+                      np.array([e[0] for e in INIT_EDGES], np.uint64),
+                      np.array([e[1] for e in INIT_EDGES], np.uint64),
+                      np.array([e[2] for e in INIT_EDGES], np.float32))
+    bf = BruteForce(INIT_LIVE, INIT_EDGES)
+    b = Batch.of([(k, s, d, w, t) for (k, s, d, w), t in zip(seq, ts)])
+    rc1, _ = o.apply(b, snapshot)
+    rc2 = bf.apply(b.kind, b.src, b.dst, b.w, b.ts, snapshot)
+    assert rc1 == rc2 == 0
+    return o.export(), bf.export()
+
+
+def test_exhaustive_length2_all_orders():
+    ops = _all_ops(3)
+    n = 0
+    for a, b in itertools.product(ops, ops):
+        for ts in ((1, 2), (2, 1), (1, 1)):
+            x, y = _run_both([a, b], ts, 2)
+            assert same_export(x, y), (a, b, ts)
+            n += 1
+    assert n == 3 * len(ops) ** 2
+
+
+def test_exhaustive_length3():
+    ops = _all_ops(3)
+    for seq in itertools.product(ops, repeat=3):
+        x, y = _run_both(list(seq), (1, 2, 3), 3)
+        assert same_export(x, y), seq
+
+
+def test_random_vs_bruteforce_multibatch():
+    """Random multi-batch streams with equal ts, out-of-order arrival, deferral."""
+    for case in range(400):
+        nid = 3 + case % 5
+        live = list(range(0, nid, 2))
+        rng = np.random.default_rng(case)
+        edges = [(int(u), int(v), float(rng.integers(0, 8)) / 4)
+                 for u in live for v in live if rng.random() < 0.4]
+        o = O1.from_edges(len(live), np.array(live, np.uint64),
+                          np.array([e[0] for e in edges], np.uint64),
+                          np.array([e[1] for e in edges], np.uint64),
+                          np.array([e[2] for e in edges], np.float32))
+        bf = BruteForce(live, edges)
+        snap = 0
+        for k in range(3):
+            b = synth.fuzz_batch(seed=case, k=k, n=4 + case % 9, n_ids=nid, ts_lo=snap + 1,
+                                 ts_span=6)
+            s_new = snap + 3 + k
+            rc1, st = o.apply(b, s_new)
+            rc2 = bf.apply(b.kind, b.src, b.dst, b.w, b.ts, s_new)
+            assert rc1 == rc2 == 0
+            assert st["n_deferred"] == len(bf.pending)
+            x, y = o.export(), bf.export()
+            assert same_export(x, y), (case, k)
+            check_invariants(*x)
+            snap = s_new
+
+
+# ------------------------------------------------- textbook CSR build ----
+def textbook_csr(n, src, dst, w):
+    """Insert-only into identity vertices 0..n-1: lexsort + keep the last duplicate."""
+    idx = np.arange(len(src))
+    order = np.lexsort((idx, dst, src))            # by (src, dst, arrival)
+    s, d, ww = src[order], dst[order], w[order]
+    last = np.ones(len(s), bool)
+    last[:-1] = (s[1:] != s[:-1]) | (d[1:] != d[:-1])
+    s, d, ww = s[last], d[last], ww[last]
+    off = np.zeros(n + 1, np.int64)
+    np.add.at(off, s.astype(np.int64) + 1, 1)
+    return np.cumsum(off), d.astype(np.uint32), ww.astype(np.float32)
+
+
+@pytest.mark.parametrize("scale", [6, 9])
+def test_insert_only_equals_textbook_csr(scale):
+    n = 1 << scale
+    src, dst, w = synth.rmat_edges(scale, seed=scale, n=8 * n)
+    o = O1.from_edges(n, None, np.array([], np.uint64), np.array([], np.uint64),
+                      np.array([], np.float32))
+    b = Batch(np.full(len(src), EDGE_INSERT, np.uint8), src, dst, w,
+              np.arange(1, len(src) + 1, dtype=np.uint64))
+    rc, _ = o.apply(b, len(src))
+    assert rc == 0
+    off, cols, ww, ids = o.export()
+    toff, tcols, tw = textbook_csr(n, src, dst, w)
+    assert np.array_equal(ids, np.arange(n, dtype=np.uint64))
+    assert np.array_equal(off, toff) and np.array_equal(cols, tcols) and np.array_equal(ww, tw)
+    # create-from-edges (A17) is the same thing
+    o2 = O1.from_edges(n, None, src, dst, w)
+    assert same_export(o2.export(), (off, cols, ww, ids))
+
+
+def test_delete_all_and_empty_batch():
+    n = 64
+    src, dst, w = synth.rmat_edges(6, seed=3, n=400)
+    o = O1.from_edges(n, None, src, dst, w)
+    before = o.export()
+    rc, _ = o.apply(Batch.empty(0), 5)                  # empty batch: identity
+    assert rc == 0 and same_export(o.export(), before)
+    off, cols, _, ids = before
+    u = np.repeat(ids, np.diff(off))
+    v = ids[cols]
+    b = Batch(np.full(len(u), EDGE_DELETE, np.uint8), u, v, np.zeros(len(u), np.float32),
+              np.full(len(u), 6, np.uint64))
+    rc, _ = o.apply(b, 6)
+    off2, cols2, _, ids2 = o.export()
+    assert rc == 0 and len(cols2) == 0 and np.all(off2 == 0) and np.array_equal(ids2, ids)
+
+
+# ----------------------------------------------------------- properties ----
+def _rmat_oracle(scale=7, seed=1):
+    n = 1 << scale
+    src, dst, w = synth.rmat_edges(scale, seed=seed, n=6 * n)
+    return n, (src, dst, w)
+
+
+def _fresh(n, edges):
+    return O1.from_edges(n, None, *edges)
+
+
+def _mixed_batch(seed, k, n_ids, n, ts_lo, ts_span):
+    return synth.fuzz_batch(seed, k, n, n_ids, probs=(0.05, 0.03, 0.5, 0.25, 0.17), ts_lo=ts_lo,
+                            ts_span=ts_span)
+
+
+def test_composition():
+    n, edges = _rmat_oracle()
+    for s in range(20):
+        b1 = _mixed_batch(s, 0, n + 4, 300, 1, 50)
+        b2 = _mixed_batch(s, 1, n + 4, 300, 51, 50)
+        a = _fresh(n, edges); a.apply(b1, 50); a.apply(b2, 100)
+        c = _fresh(n, edges); c.apply(b1.concat(b2), 100)
+        assert same_export(a.export(), c.export())
+
+
+def test_deferral():
+    n, edges = _rmat_oracle()
+    for s in range(20):
+        b = _mixed_batch(s, 0, n + 4, 300, 1, 100)
+        a = _fresh(n, edges)
+        rc, st = a.apply(b, 40)
+        assert rc == 0 and st["n_deferred"] == int(np.sum(b.ts > 40))
+        a.apply(Batch.empty(0), 100)
+        c = _fresh(n, edges); c.apply(b, 100)
+        assert same_export(a.export(), c.export())
+        assert a.info()["n_pending"] == 0
+
+
+def test_permutation_of_distinct_ts():
+    n, edges = _rmat_oracle()
+    for s in range(20):
+        b = _mixed_batch(s, 0, n + 4, 300, 1, 1)
+        b.ts = np.arange(1, len(b) + 1, dtype=np.uint64)      # distinct timestamps
+        perm = np.random.default_rng(s).permutation(len(b))
+        a = _fresh(n, edges); a.apply(b, len(b))
+        c = _fresh(n, edges); c.apply(b.slice(perm), len(b))
+        assert same_export(a.export(), c.export())
+
+
+def test_equal_ts_ties_follow_arrival():
+    # same txn: insert then delete of one key -> absent; delete then insert -> present
+    o = O1.from_edges(2, None, np.array([], np.uint64), np.array([], np.uint64),
+                      np.array([], np.float32))
+    o.apply(Batch.of([(EDGE_INSERT, 0, 1, 1.0, 5), (EDGE_DELETE, 0, 1, 0, 5)]), 5)
+    assert o.info()["n_edges"] == 0
+    o.apply(Batch.of([(EDGE_DELETE, 0, 1, 0, 6), (EDGE_INSERT, 0, 1, 3.0, 6)]), 6)
+    assert o.export()[2].tolist() == [3.0]
+
+
+# --------------------------------------------------------- error codes ----
+def test_errors_leave_state_unchanged():
+    n, edges = _rmat_oracle(6, 2)
+    o = _fresh(n, edges)
+    o.apply(_mixed_batch(1, 0, n, 50, 1, 10), 20)
+    before = o.export()
+    rc, _ = o.apply(_mixed_batch(1, 1, n, 5, 30, 5), 10)
+    assert rc == oracle.E_SNAPSHOT_REGRESSION
+    rc, _ = o.apply(Batch.of([(EDGE_INSERT, 0, 1, 1.0, 20)]), 30)     # ts <= snapshot
+    assert rc == oracle.E_STALE_TS
+    rc, _ = o.apply(Batch.of([(7, 0, 1, 1.0, 25)]), 30)               # unknown kind
+    assert rc == oracle.E_INVAL
+    assert same_export(o.export(), before) and o.info()["snapshot_ts"] == 20
+
+
+# ----------------------------------------------------------- analytics ----
+def test_bfs_matches_scipy():
+    from scipy.sparse import csr_matrix
+    from scipy.sparse.csgraph import shortest_path
+    for scale in (5, 8):
+        n = 1 << scale
+        src, dst, w = synth.rmat_edges(scale, seed=scale + 10, n=4 * n)
+        off, cols, _, _ = O1.from_edges(n, None, src, dst, w).export()
+        A = csr_matrix((np.ones(len(cols)), cols.astype(np.int64), off), shape=(n, n))
+        for s in (0, 1, n // 2):
+            lvl = oracle.bfs(off, cols, s)
+            d = shortest_path(A, unweighted=True, indices=s)
+            ref = np.where(np.isinf(d), -1, d).astype(np.int32)
+            assert np.array_equal(lvl, ref)
+
+
+def test_pagerank_closed_forms_and_dense_power_iteration():
+    # directed n-cycle: the uniform vector is the fixed point -> 1/n exactly
+    n = 7
+    off = np.arange(n + 1, dtype=np.int64)
+    cols = ((np.arange(n) + 1) % n).astype(np.uint32)
+    pr = oracle.pagerank(off, cols, 0.85, 30)
+    assert np.allclose(pr, 1.0 / n, rtol=0, atol=1e-15)
+    # random graph with dangling vertices: dense matrix power iteration, sum = 1
+    scale = 7
+    N = 1 << scale
+    src, dst, w = synth.rmat_edges(scale, seed=5, n=3 * N)
+    off, cols, _, _ = O1.from_edges(N, None, src, dst, w).export()
+    deg = np.diff(off)
+    M = np.zeros((N, N))
+    for u in range(N):
+        for e in range(off[u], off[u + 1]):
+            M[cols[e], u] += 1.0 / deg[u]
+    dang = (deg == 0).astype(float)
+    x = np.full(N, 1.0 / N)
+    for _ in range(20):
+        x = (1 - 0.85) / N + 0.85 * (M @ x + dang @ x / N)
+    pr = oracle.pagerank(off, cols, 0.85, 20)
+    assert abs(pr.sum() - 1.0) < 1e-12
+    assert np.max(np.abs(pr - x) / x) < 1e-12
+
+
+def test_checksum_is_position_keyed():
+    a = np.array([1, 2, 3], np.uint32)
+    b = np.array([2, 1, 3], np.uint32)
+    assert oracle.checksum(a, 2) != oracle.checksum(b, 2)
+    assert oracle.checksum(a, 2) == oracle.checksum(a.copy(), 2)
+    assert oracle.checksum(np.array([], np.uint32), 2) == 0

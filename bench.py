@@ -1,0 +1,359 @@
+#!/usr/bin/env python
+"""Benchmark: delta updates/s merged into the GPU-resident CSR replica.
+
+    python bench.py [--gpus N] [--steps K] [--warmup W] [--config c2|c3|c1] [--impl h2tap|reference]
+
+A step is one h2tap_delta_apply of one synthetic batch (all SURVEY.md §8(a)
+steps a1-a7) into the replica.  Default workload: BASELINE.json configs[1]
+(LDBC-SNB-shaped SF10 property graph, 100K-update batches with node inserts and
+deletes and ID remap).  Inputs are device-resident when the timed region
+starts; the e2e leg repeats the measurement with pinned host batches copied in
+by the library inside the timed region.  The CSR (~2.8 GB read + written per
+step) exceeds the 126 MB L2, so no explicit flush is needed.
+
+Prints ONE JSON line (rank 0).  Under torchrun with N > 1 every rank holds an
+independent replica with its own batch stream (replicas, weak scaling; DESIGN.md
+§6).  ``--impl reference`` times the oracle (O1, test infrastructure) on the
+host cores over a bounded scaled-down sample of the same workload.
+"""
+from __future__ import annotations
+
+import argparse
+import json
+import os
+import statistics
+import subprocess
+import sys
+import threading
+import time
+
+import numpy as np
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+import synth  # noqa: E402
+
+METRIC = "delta updates/sec merged into CSR replica"
+PEAKS_FILE = os.path.join(ROOT, "MEASURED_PEAKS.json")
+FALLBACK_HBM = 6650.0  # GB/s, /opt/skills/guides/B200_PROFILING.md fallback
+
+
+# ------------------------------------------------------------- workload ----
+class Workload:
+    """Initial graph + batch generator for one config (seeded, synthetic)."""
+
+    def __init__(self, name: str, scale_down: int = 1):
+        self.name = name
+        self.cfg = synth.CONFIGS[name]
+        self.seed = synth.seed_of(name)
+        self.scale_down = scale_down
+        if self.cfg["kind"] == "ldbc":
+            s = self.cfg["shape"]
+            if scale_down > 1:
+                s = synth.LdbcShape(max(64, s.n_person // scale_down), max(64, s.n_msg // scale_down),
+                                    max(64, s.e_person // scale_down))
+            self.shape = s
+            self.batch_size = max(64, self.cfg["batch"] // scale_down)
+        else:
+            self.scale = self.cfg["scale"] - (int(np.log2(scale_down)) if scale_down > 1 else 0)
+            self.batch_size = max(64, self.cfg["batch"] // scale_down)
+        self.ts = 0
+
+    def graph(self):
+        if self.cfg["kind"] == "ldbc":
+            ids = synth.ldbc_vertices(self.shape)
+            src, dst, w = synth.ldbc_edges(self.shape, self.seed)
+            return self.shape.n_vertices, ids, src, dst, w
+        src, dst, w = synth.rmat_edges(self.scale, self.seed, n=self.cfg["edge_factor"] << self.scale)
+        self.m_initial = len(src)
+        return 1 << self.scale, None, src, dst, w
+
+    def batch(self, k: int) -> synth.Batch:
+        if self.cfg["kind"] == "ldbc":
+            b = synth.ldbc_batch(self.shape, self.seed, k, self.batch_size, ts_base=self.ts)
+        else:
+            b = synth.rmat_batch(self.scale, self.seed, k, self.batch_size, self.m_initial,
+                                 p_insert=self.cfg["p_insert"], ts_base=self.ts)
+        self.ts = int(b.ts.max())
+        return b
+
+    def describe(self) -> str:
+        if self.cfg["kind"] == "ldbc":
+            s = self.shape
+            return (f"LDBC-SNB-shaped SF10 ({s.n_vertices} vertices, {s.n_edges} generated edges, "
+                    f"{s.n_person} Person hubs), {self.batch_size}-op batches "
+                    f"(66/22/11/1 insert-rel/insert-node/delete-rel/delete-node)")
+        return (f"RMAT scale-{self.scale} ({1 << self.scale} vertices, "
+                f"{self.cfg['edge_factor'] << self.scale} generated edges), {self.batch_size}-op "
+                f"batches ({int(self.cfg['p_insert'] * 100)}/{100 - int(self.cfg['p_insert'] * 100)} insert/delete)")
+
+
+# --------------------------------------------------------------- clocks ----
+class ClockSampler:
+    FIELDS = ("clocks.sm,clocks.max.sm,power.draw,clocks_event_reasons.hw_slowdown,"
+              "clocks_event_reasons.hw_thermal_slowdown,clocks_event_reasons.sw_thermal_slowdown,"
+              "clocks_event_reasons.sw_power_cap")
+
+    def __init__(self, index: int):
+        self.index = index
+        self.rows = []
+        self.proc = None
+
+    def __enter__(self):
+        try:
+            self.proc = subprocess.Popen(
+                ["nvidia-smi", "-i", str(self.index), f"--query-gpu={self.FIELDS}",
+                 "--format=csv,noheader,nounits", "-lms", "100"],
+                stdout=subprocess.PIPE, stderr=subprocess.DEVNULL, text=True)
+            self.t = threading.Thread(target=self._read, daemon=True)
+            self.t.start()
+        except FileNotFoundError:
+            self.proc = None
+        return self
+
+    def _read(self):
+        for line in self.proc.stdout:
+            self.rows.append([x.strip() for x in line.split(",")])
+
+    def __exit__(self, *a):
+        if self.proc:
+            time.sleep(0.25)
+            self.proc.terminate()
+            try:
+                self.proc.wait(2)
+            except Exception:
+                self.proc.kill()
+
+    def summary(self):
+        if not self.rows:
+            return {"sm_mhz": None, "sm_max_mhz": None, "reasons": ["unsampled"]}
+        sm = [float(r[0]) for r in self.rows if r and r[0].replace(".", "").isdigit()]
+        mx = [float(r[1]) for r in self.rows if len(r) > 1 and r[1].replace(".", "").isdigit()]
+        names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
+        reasons = sorted({names[i] for r in self.rows for i in range(4)
+                          if len(r) > 3 + i and r[3 + i].lower().startswith("active")})
+        return {"sm_mhz": statistics.median(sm) if sm else None, "sm_max_mhz": max(mx) if mx else None,
+                "reasons": reasons, "samples": len(self.rows)}
+
+
+def peaks():
+    try:
+        p = json.load(open(PEAKS_FILE))
+        return float(p["hbm_gbs"]), "measured (MEASURED_PEAKS.json hbm_gbs)"
+    except Exception:
+        return FALLBACK_HBM, "fallback (B200_PROFILING.md 6.65 TB/s)"
+
+
+# ------------------------------------------------------------ dist utils ----
+def dist_setup():
+    world = int(os.environ.get("WORLD_SIZE", "1"))
+    rank = int(os.environ.get("RANK", "0"))
+    local = int(os.environ.get("LOCAL_RANK", "0"))
+    return world, rank, local
+
+
+def cpu_cores():
+    try:
+        return len(os.sched_getaffinity(0))
+    except Exception:
+        return os.cpu_count()
+
+
+# ------------------------------------------------------------- oracle arm ----
+def oracle_sample(name: str, steps: int, warmup: int, target_s: float = 20.0):
+    """Time O1 (single-threaded std::map replay + CSR export) on a scaled-down sample."""
+    import oracle
+    scale_down = {"c1": 4, "c2": 128, "c3": 256}[name]
+    wl = Workload(name, scale_down)
+    nv, ids, src, dst, w = wl.graph()
+    o = oracle.O1.from_edges(nv, ids, src, dst, w)
+    times, ops = [], 0
+    total = 0.0
+    for k in range(warmup + steps):
+        b = wl.batch(k)
+        t0 = time.perf_counter()
+        rc, st = o.apply(b, int(b.ts.max()))
+        o.export()
+        dt = time.perf_counter() - t0
+        assert rc == 0
+        if k >= warmup:
+            times.append(dt)
+            ops += st["n_visible"]
+        total += dt
+        if total > target_s * 3:
+            break
+    value = ops / sum(times) if times else 0.0
+    sample = (f"O1 on a 1/{scale_down} scale-down of the same workload: {wl.describe()}; "
+              f"apply + CSR export per batch, {len(times)} timed batches, 1 thread")
+    return value, sample, (sum(times) / max(1, len(times))) * 1e3
+
+
+def run_reference(args):
+    world, rank, _ = dist_setup()
+    if rank != 0:
+        return
+    value, sample, ms = oracle_sample(args.config, args.steps, args.warmup)
+    wl = Workload(args.config)
+    line = {
+        "impl": "reference", "metric": METRIC, "value": value, "unit": "updates/s",
+        "n_gpus": args.gpus, "steps": args.steps, "warmup": args.warmup, "ms_per_step": ms,
+        "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": "u32/f32",
+        "data": "synthetic", "config": {"workload": wl.describe(), "name": args.config},
+        "cpu_baseline": {"value": value, "unit": "updates/s", "cores": 1, "kind": "oracle",
+                         "sample": sample},
+        "e2e": {"value": value, "unit": "updates/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0},
+    }
+    print(json.dumps(line), flush=True)
+
+
+# --------------------------------------------------------------- GPU arm ----
+def run_gpu(args):
+    import torch
+    import torch.distributed as dist
+
+    import paper_conf_edbt_jibrilabs23_b200 as h2
+
+    world, rank, local = dist_setup()
+    if world > 1:
+        dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+    torch.cuda.set_device(local)
+    stream = torch.cuda.current_stream()
+
+    wl = Workload(args.config)
+    t0 = time.time()
+    nv, ids, src, dst, w = wl.graph()
+    # rank-distinct batch streams (independent replicas); same initial graph shape
+    rep = h2.Replica.from_edges(nv, ids, src, dst, w, 0, device=local)
+    del src, dst, w
+    setup_s = time.time() - t0
+
+    n_total = args.warmup + args.steps
+    k0 = rank * 1000
+    host = [wl.batch(k0 + k) for k in range(n_total)]
+
+    def to_dev(b):
+        return synth.Batch(*(torch.from_numpy(a.view(np.int64) if a.dtype == np.uint64 else a).cuda()
+                             for a in (b.kind, b.src, b.dst, b.w, b.ts)))
+
+    dev = [to_dev(b) for b in host]
+    snaps = [int(b.ts.max()) for b in host]
+    for k in range(args.warmup):
+        rep.apply(dev[k], snaps[k])
+    torch.cuda.synchronize()
+    if world > 1:
+        dist.barrier()
+    stats = []
+    ev0, ev1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    with ClockSampler(local) as clk:
+        torch.cuda.synchronize()
+        ev0.record(stream)
+        for k in range(args.warmup, n_total):
+            stats.append(rep.apply(dev[k], snaps[k]))
+        ev1.record(stream)
+        torch.cuda.synchronize()
+    if world > 1:
+        dist.barrier()
+    ms = ev0.elapsed_time(ev1)
+    updates = sum(s["n_visible"] for s in stats)
+    if world > 1:
+        t = torch.tensor([ms, float(updates)], device="cuda", dtype=torch.float64)
+        mx = t.clone()
+        dist.all_reduce(mx, op=dist.ReduceOp.MAX)
+        dist.all_reduce(t, op=dist.ReduceOp.SUM)
+        ms_max, updates_all = float(mx[0]), float(t[1])
+    else:
+        ms_max, updates_all = ms, float(updates)
+    value = updates_all / (ms_max / 1e3)
+
+    # ---- e2e: pinned host batches through the public API, H2D inside the timed region
+    e_host = [wl.batch(k0 + n_total + k) for k in range(args.steps)]
+
+    def pinned(b):
+        return synth.Batch(*(torch.from_numpy(a.view(np.int64) if a.dtype == np.uint64 else a).pin_memory()
+                             for a in (b.kind, b.src, b.dst, b.w, b.ts)))
+
+    e_pin = [pinned(b) for b in e_host]
+    e_snaps = [int(b.ts.max()) for b in e_host]
+    torch.cuda.synchronize()
+    if world > 1:
+        dist.barrier()
+    e_stats = []
+    ev0.record(stream)
+    for k in range(args.steps):
+        e_stats.append(rep.apply(e_pin[k], e_snaps[k]))
+    ev1.record(stream)
+    torch.cuda.synchronize()
+    e_ms = ev0.elapsed_time(ev1)
+    e_updates = sum(s["n_visible"] for s in e_stats)
+    if world > 1:
+        t = torch.tensor([e_ms, float(e_updates)], device="cuda", dtype=torch.float64)
+        mx = t.clone()
+        dist.all_reduce(mx, op=dist.ReduceOp.MAX)
+        dist.all_reduce(t, op=dist.ReduceOp.SUM)
+        e_ms, e_updates = float(mx[0]), float(t[1])
+    e_value = e_updates / (e_ms / 1e3)
+
+    if rank == 0:
+        peak, peak_src = peaks()
+        mean = lambda key: sum(s[key] for s in stats) / len(stats)  # noqa: E731
+        merge_ms = mean("ms_merge")
+        merge_bytes = mean("bytes_merge")
+        achieved = merge_bytes / (merge_ms / 1e3) / 1e9 if merge_ms > 0 else 0.0
+        path_bytes = mean("bytes_alg")
+        ms_step = ms / len(stats)
+        path_gbs = path_bytes / (ms_step / 1e3) / 1e9
+        info = rep.info()
+        line = {
+            "metric": METRIC, "value": value, "unit": "updates/s", "n_gpus": world,
+            "steps": args.steps, "warmup": args.warmup, "ms_per_step": ms_max / args.steps,
+            "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": "u32/f32",
+            "data": "synthetic",
+            "config": {"workload": wl.describe(), "name": args.config, "parallelism":
+                       "replicas" if world > 1 else "single",
+                       "l2": "inputs larger than L2 (CSR ~%.1f GB per step)" % (path_bytes / 1e9),
+                       "replica_vertices": info["n_vertices"], "replica_edges": info["n_edges"]},
+            "roofline": {"bound": "hbm", "kernel": "k_merge", "achieved": achieved, "peak": peak,
+                         "unit": "GB/s", "frac": achieved / peak, "traffic": None,
+                         "peak_source": peak_src, "bytes_per_launch": merge_bytes,
+                         "ms_per_launch": merge_ms},
+            "path": {"bytes_alg_per_step": path_bytes, "achieved_gbs": path_gbs,
+                     "frac_of_peak": path_gbs / peak,
+                     "phase_ms": {k: mean(k) for k in ("ms_ingest", "ms_nodeops", "ms_sort_reduce",
+                                                      "ms_merge", "ms_degree_scan", "ms_total")},
+                     "setup_s": setup_s},
+            "gpu_launches": int(sum(s["n_launches"] for s in stats)),
+            "e2e": {"value": e_value, "unit": "updates/s",
+                    "h2d_bytes_per_step": int(sum(s["h2d_bytes"] for s in e_stats) / len(e_stats)),
+                    "d2h_bytes_per_step": int(sum(s["d2h_bytes"] for s in e_stats) / len(e_stats))},
+            "clocks": clk.summary(),
+        }
+        if not args.no_cpu_baseline:
+            v, sample, _ = oracle_sample(args.config, 3, 1, target_s=8.0)
+            line["cpu_baseline"] = {"value": v, "unit": "updates/s", "cores": 1, "kind": "oracle",
+                                    "sample": sample}
+        print(json.dumps(line), flush=True)
+    rep.close()
+    if world > 1:
+        dist.destroy_process_group()
+
+
+def main():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--gpus", type=int, default=1)
+    ap.add_argument("--steps", type=int, default=20)
+    ap.add_argument("--warmup", type=int, default=3)
+    ap.add_argument("--config", default="c2", choices=sorted(synth.CONFIGS))
+    ap.add_argument("--impl", default="h2tap", choices=["h2tap", "reference"])
+    ap.add_argument("--no-cpu-baseline", action="store_true")
+    args = ap.parse_args()
+    if args.warmup < 3 and args.impl == "h2tap":
+        args.warmup = 3
+    if args.impl == "reference":
+        run_reference(args)
+    else:
+        run_gpu(args)
+
+
+if __name__ == "__main__":
+    main()

@@ -1,0 +1,167 @@
+/*
+ * h2tap.h - C ABI of the B200-native update-propagation path for graph H2TAP.
+ *
+ * The path: a batch of committed, timestamped delta-store updates is propagated
+ * into a CSR replica resident in GPU memory (§4.2, §5.2-5.4
+ * P:L702-890).  Implemented by hand-written sm_100a kernels in libh2tap.so; no
+ * CPU fallback.  Every entry point returns a status code (no exception crosses
+ * the ABI); detail text for the last failure on the calling thread comes from
+ * h2tap_last_error().
+ *
+ * Replica layout: offsets int64[V+1], cols uint32[E] (dense IDs),
+ * weights float32[E] (carried bit-exactly), ext_ids uint64[V] (strictly
+ * increasing external IDs; dense ID = rank of the external ID among live
+ * vertices, reading A9).  Rows are sorted by column and duplicate-free
+ * (reading A1).
+ *
+ * Ownership: caller buffers are only read (or, for export/bfs/pagerank,
+ * written) during the call and never retained.  The replica owns all device
+ * state; it allocates through h2tap_config.alloc (e.g. the torch caching
+ * allocator) or cudaMallocAsync when alloc.alloc is NULL.
+ *
+ * Strong guarantee: on any error the replica's CSR, ID map, snapshot_ts and
+ * pending set are unchanged.  A sticky CUDA error marks the handle POISONED;
+ * then only h2tap_replica_destroy is valid.
+ *
+ * Streams: all work is ordered on h2tap_config.stream; calls return after the
+ * work has completed.
+ */
+#ifndef H2TAP_H
+#define H2TAP_H
+
+#include <stddef.h>
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+typedef struct h2tap_replica h2tap_replica; /* opaque; owns all device state */
+
+typedef enum {
+    H2TAP_OK = 0,
+    H2TAP_E_INVAL = -1,               /* bad argument, unknown op kind, malformed CSR */
+    H2TAP_E_NOMEM = -2,               /* device allocation failed */
+    H2TAP_E_CUDA = -3,                /* CUDA error (sticky ones poison the handle) */
+    H2TAP_E_NCCL = -4,                /* collective failed (multi-GPU) */
+    H2TAP_E_STALE_TS = -5,            /* an op has ts <= current snapshot_ts (reading A7) */
+    H2TAP_E_SNAPSHOT_REGRESSION = -6, /* snapshot_ts < current snapshot_ts */
+    H2TAP_E_CAPACITY = -7,            /* size beyond the 32-bit dense-ID / op-index limits */
+    H2TAP_E_POISONED = -8             /* handle unusable after a sticky CUDA error */
+} h2tap_status;
+
+/* op kinds (uint8_t), §5.1; EDGE_WEIGHT is reading A3 */
+enum {
+    H2TAP_NODE_INSERT = 0, /* src = vertex; no-op if live (A12)                     */
+    H2TAP_NODE_DELETE = 1, /* src = vertex; removes it and all in/out edges (A8)     */
+    H2TAP_EDGE_INSERT = 2, /* src->dst, weight; upsert if both endpoints live (A2)   */
+    H2TAP_EDGE_DELETE = 3, /* src->dst; no-op if absent (A4)                         */
+    H2TAP_EDGE_WEIGHT = 4  /* src->dst, weight; update-if-present (A3)               */
+};
+
+/* A batch of ops, structure of arrays, all arrays of length n (29 B/op).
+ * Caller-owned, read-only, not retained.  on_device: 0 = host memory (pinned
+ * preferred; copied in), 1 = device memory of the replica's device. */
+typedef struct {
+    size_t n;
+    int on_device;
+    const uint8_t* kind;
+    const uint64_t* src;
+    const uint64_t* dst;    /* ignored for NODE_* */
+    const float* weight;    /* ignored for NODE_* and EDGE_DELETE; may be NULL if unused */
+    const uint64_t* ts;     /* commit timestamps (MVTO txn timestamps) */
+} h2tap_batch;
+
+/* Filled by h2tap_delta_apply (counts are global over all ranks). */
+typedef struct {
+    uint64_t n_visible;   /* ops with ts <= snapshot_ts applied this call (incl. earlier pending) */
+    uint64_t n_deferred;  /* ops with ts > snapshot_ts kept pending for a later call (A6) */
+    uint64_t n_gated;     /* edge ops dropped: endpoint not live at the op's point (A13) or
+                             superseded by a later node delete of an endpoint (A8) */
+    uint64_t n_new;       /* keys inserted that were absent from the old CSR */
+    uint64_t n_del;       /* old edges removed by EDGE_DELETE */
+    uint64_t n_upd;       /* old edges whose weight was overwritten (upsert or EDGE_WEIGHT) */
+    uint64_t n_casc;      /* old edges removed by a node delete of an endpoint (A8) */
+    uint64_t n_vertex_inserted, n_vertex_deleted;
+    float ms_ingest, ms_nodeops, ms_sort_reduce, ms_degree_scan, ms_merge, ms_route, ms_total;
+    uint64_t bytes_alg;   /* algorithmic bytes of this call */
+    uint64_t bytes_merge; /* algorithmic bytes of the merge kernel launch */
+    uint64_t n_launches;  /* kernels launched by this call */
+    uint64_t h2d_bytes, d2h_bytes; /* host<->device bytes copied by this call */
+} h2tap_apply_stats;
+
+typedef struct {
+    void* ctx;
+    void* (*alloc)(void* ctx, size_t bytes, void* stream); /* NULL -> cudaMallocAsync */
+    void (*free)(void* ctx, void* p, void* stream);
+} h2tap_allocator;
+
+typedef struct {
+    int device;                  /* CUDA device ordinal */
+    int rank, world;             /* world == 1 for a single replica */
+    const void* nccl_unique_id;  /* ncclUniqueId bytes (world > 1), else NULL */
+    uint64_t expected_batch;     /* capacity hint (ops per batch); 0 = none */
+    h2tap_allocator alloc;
+    void* stream;                /* cudaStream_t; NULL = legacy default stream */
+} h2tap_config;
+
+/* Create from an edge list (reading A17): the vertex set is vertex_ids
+ * (strictly increasing; NULL = identity 0..n_vertices-1), then the edges are
+ * inserted in order, the last duplicate (src,dst) winning.  An edge endpoint
+ * outside the vertex set, or non-increasing vertex_ids -> E_INVAL.
+ * snapshot_ts = create_ts.  Arrays host (on_device=0) or device (1). */
+h2tap_status h2tap_replica_create_from_edges(const h2tap_config* cfg, size_t n_vertices,
+        const uint64_t* vertex_ids, size_t n_edges, const uint64_t* src, const uint64_t* dst,
+        const float* w, int on_device, uint64_t create_ts, h2tap_replica** out);
+
+/* Create from a CSR (checkpoint restore): offsets int64[n_vertices+1], cols
+ * uint32[offsets[n]], w float[offsets[n]] (NULL = zeros), ext_ids uint64[n]
+ * (NULL = identity).  Requires offsets[0]=0 and monotone, rows strictly
+ * increasing, cols < n_vertices, ext_ids strictly increasing; else E_INVAL. */
+h2tap_status h2tap_replica_create_from_csr(const h2tap_config* cfg, size_t n_vertices,
+        const int64_t* offsets, const uint32_t* cols, const float* w, const uint64_t* ext_ids,
+        int on_device, uint64_t create_ts, h2tap_replica** out);
+
+/* One propagation cycle (the hot path; §5.2-5.4, Algorithm 2
+ * P:L845-887): ops of this batch and earlier pending ops with ts <= snapshot_ts
+ * are applied as if replayed in (ts, seq) order (seq = arrival order, reading
+ * A5); the rest stay pending (A6).  Result: a new compact sorted CSR + ID map,
+ * swapped in atomically at snapshot_ts.
+ * Errors: snapshot_ts < current -> E_SNAPSHOT_REGRESSION; unknown kind ->
+ * E_INVAL; any batch op with ts <= current snapshot_ts -> E_STALE_TS. */
+h2tap_status h2tap_delta_apply(h2tap_replica* r, const h2tap_batch* batch, uint64_t snapshot_ts,
+        h2tap_apply_stats* stats /* nullable */);
+
+/* Sizes of the current replica (any pointer may be NULL). */
+h2tap_status h2tap_replica_info(const h2tap_replica* r, uint64_t* n_vertices, uint64_t* n_edges,
+        uint64_t* snapshot_ts, uint64_t* n_pending, uint64_t* shard_vertex_base,
+        uint64_t* shard_edge_base);
+
+/* Copy the replica into caller buffers sized from h2tap_replica_info
+ * (offsets V+1, cols E, w E, ext_ids V; any may be NULL).  checksums (nullable)
+ * receives the position-keyed 64-bit checksums of {offsets, cols, w, ext_ids}:
+ *   cs(a, salt) = sum_i sm64(bits(a_i) ^ sm64(i ^ salt)) mod 2^64, salts 1..4,
+ *   sm64 = SplitMix64 finaliser, bits = raw pattern zero-extended to 64 bits. */
+h2tap_status h2tap_replica_export(const h2tap_replica* r, int64_t* offsets, uint32_t* cols,
+        float* w, uint64_t* ext_ids, int on_device, uint64_t checksums[4]);
+
+/* BFS levels over out-edges from the vertex with external ID source_ext
+ * (freshness check, LDBC Graphalytics P:L951-954, reading A18): level int32[V],
+ * source 0, unreachable -1.  Unknown source -> E_INVAL. */
+h2tap_status h2tap_bfs(const h2tap_replica* r, uint64_t source_ext, int32_t* level_out,
+        int on_device);
+
+/* PageRank, fp64 (Graphalytics): PR_0 = 1/V; PR_t(v) = (1-d)/V + d*(sum over
+ * in-edges u->v of PR_{t-1}(u)/outdeg(u) + dangling mass / V). rank double[V]. */
+h2tap_status h2tap_pagerank(const h2tap_replica* r, double damping, int iterations,
+        double* rank_out, int on_device);
+
+void h2tap_replica_destroy(h2tap_replica* r);
+const char* h2tap_status_str(h2tap_status s);
+const char* h2tap_last_error(void);
+const char* h2tap_version(void);
+
+#ifdef __cplusplus
+}
+#endif
+#endif /* H2TAP_H */

@@ -1,0 +1,272 @@
+"""B200-native update propagation into a GPU-resident CSR replica (graph H2TAP).
+
+Thin ctypes binding over ``libh2tap.so`` (include/h2tap.h).  Argument
+marshalling only: every step of the propagation path runs in the library's
+sm_100a kernels.  There is no CPU fallback — importing this package raises if
+the shared library is missing.  PyTorch is used only for device memory (the
+caching allocator backs the library's allocations) and streams.
+
+Arrays may be numpy arrays (host memory; copied in by the library) or torch
+CUDA tensors (device memory of the replica's device).
+"""
+from __future__ import annotations
+
+import ctypes
+import os
+
+import numpy as np
+
+_HERE = os.path.dirname(os.path.abspath(__file__))
+LIB_PATH = os.path.join(_HERE, "libh2tap.so")
+
+OK = 0
+STATUS = {0: "OK", -1: "E_INVAL", -2: "E_NOMEM", -3: "E_CUDA", -4: "E_NCCL", -5: "E_STALE_TS",
+          -6: "E_SNAPSHOT_REGRESSION", -7: "E_CAPACITY", -8: "E_POISONED"}
+NODE_INSERT, NODE_DELETE, EDGE_INSERT, EDGE_DELETE, EDGE_WEIGHT = 0, 1, 2, 3, 4
+
+if not os.path.exists(LIB_PATH):
+    raise ImportError(f"{LIB_PATH} is missing: build the CUDA library first (`make lib` or "
+                      "`python -c 'import __graft_entry__ as g; g.build()'`). There is no CPU fallback.")
+
+
+class H2tapError(RuntimeError):
+    def __init__(self, status: int, where: str, detail: str):
+        self.status = status
+        self.name = STATUS.get(status, str(status))
+        super().__init__(f"{where}: {self.name}: {detail}")
+
+
+_P = ctypes.c_void_p
+_u64 = ctypes.c_uint64
+_ALLOC = ctypes.CFUNCTYPE(ctypes.c_void_p, ctypes.c_void_p, ctypes.c_size_t, ctypes.c_void_p)
+_FREE = ctypes.CFUNCTYPE(None, ctypes.c_void_p, ctypes.c_void_p, ctypes.c_void_p)
+
+
+class _Allocator(ctypes.Structure):
+    _fields_ = [("ctx", _P), ("alloc", _ALLOC), ("free", _FREE)]
+
+
+class _Config(ctypes.Structure):
+    _fields_ = [("device", ctypes.c_int), ("rank", ctypes.c_int), ("world", ctypes.c_int),
+                ("nccl_unique_id", _P), ("expected_batch", _u64), ("alloc", _Allocator),
+                ("stream", _P)]
+
+
+class _Batch(ctypes.Structure):
+    _fields_ = [("n", ctypes.c_size_t), ("on_device", ctypes.c_int), ("kind", _P), ("src", _P),
+                ("dst", _P), ("weight", _P), ("ts", _P)]
+
+
+class ApplyStats(ctypes.Structure):
+    _fields_ = [(n, _u64) for n in ("n_visible", "n_deferred", "n_gated", "n_new", "n_del", "n_upd",
+                                    "n_casc", "n_vertex_inserted", "n_vertex_deleted")] + \
+               [(n, ctypes.c_float) for n in ("ms_ingest", "ms_nodeops", "ms_sort_reduce",
+                                              "ms_degree_scan", "ms_merge", "ms_route", "ms_total")] + \
+               [(n, _u64) for n in ("bytes_alg", "bytes_merge", "n_launches", "h2d_bytes", "d2h_bytes")]
+
+    def as_dict(self):
+        return {f: getattr(self, f) for f, _ in self._fields_}
+
+
+_lib = ctypes.CDLL(LIB_PATH)
+_lib.h2tap_replica_create_from_edges.restype = ctypes.c_int
+_lib.h2tap_replica_create_from_edges.argtypes = [ctypes.POINTER(_Config), ctypes.c_size_t, _P,
+                                                 ctypes.c_size_t, _P, _P, _P, ctypes.c_int, _u64,
+                                                 ctypes.POINTER(_P)]
+_lib.h2tap_replica_create_from_csr.restype = ctypes.c_int
+_lib.h2tap_replica_create_from_csr.argtypes = [ctypes.POINTER(_Config), ctypes.c_size_t, _P, _P, _P,
+                                               _P, ctypes.c_int, _u64, ctypes.POINTER(_P)]
+_lib.h2tap_delta_apply.restype = ctypes.c_int
+_lib.h2tap_delta_apply.argtypes = [_P, ctypes.POINTER(_Batch), _u64, ctypes.POINTER(ApplyStats)]
+_lib.h2tap_replica_info.restype = ctypes.c_int
+_lib.h2tap_replica_info.argtypes = [_P] + [ctypes.POINTER(_u64)] * 6
+_lib.h2tap_replica_export.restype = ctypes.c_int
+_lib.h2tap_replica_export.argtypes = [_P, _P, _P, _P, _P, ctypes.c_int, ctypes.POINTER(_u64)]
+_lib.h2tap_bfs.restype = ctypes.c_int
+_lib.h2tap_bfs.argtypes = [_P, _u64, _P, ctypes.c_int]
+_lib.h2tap_pagerank.restype = ctypes.c_int
+_lib.h2tap_pagerank.argtypes = [_P, ctypes.c_double, ctypes.c_int, _P, ctypes.c_int]
+_lib.h2tap_replica_destroy.restype = None
+_lib.h2tap_replica_destroy.argtypes = [_P]
+_lib.h2tap_status_str.restype = ctypes.c_char_p
+_lib.h2tap_status_str.argtypes = [ctypes.c_int]
+_lib.h2tap_last_error.restype = ctypes.c_char_p
+_lib.h2tap_version.restype = ctypes.c_char_p
+
+
+def version() -> str:
+    return _lib.h2tap_version().decode()
+
+
+def _check(rc: int, where: str):
+    if rc != OK:
+        raise H2tapError(rc, where, (_lib.h2tap_last_error() or b"").decode())
+
+
+def _is_torch(x) -> bool:
+    return hasattr(x, "data_ptr") and hasattr(x, "is_cuda")
+
+
+def _ptr(x, dtype=None):
+    """(pointer, on_device, keepalive) for a numpy array or a torch tensor (or None)."""
+    if x is None:
+        return None, None, None
+    if _is_torch(x):
+        if not x.is_contiguous():
+            x = x.contiguous()
+        return ctypes.c_void_p(x.data_ptr()), bool(x.is_cuda), x
+    a = np.ascontiguousarray(x, dtype=dtype)
+    return ctypes.c_void_p(a.ctypes.data), False, a
+
+
+def _on_device(*ptrs):
+    flags = {p[1] for p in ptrs if p[0] is not None}
+    if len(flags) > 1:
+        raise ValueError("mix of host and device arrays in one call")
+    return int(flags.pop()) if flags else 0
+
+
+def _torch_allocator(device: int):
+    import torch
+
+    def _alloc(ctx, nbytes, stream):
+        return torch.cuda.caching_allocator_alloc(int(nbytes), device, int(stream or 0))
+
+    def _free(ctx, p, stream):
+        torch.cuda.caching_allocator_delete(int(p))
+
+    return _ALLOC(_alloc), _FREE(_free)
+
+
+class Replica:
+    """A CSR replica in device memory (opaque h2tap_replica*)."""
+
+    def __init__(self, handle, keep):
+        self._h = handle
+        self._keep = keep
+
+    # ---------------------------------------------------------------- create
+    @staticmethod
+    def _config(device, stream, torch_allocator):
+        cfg = _Config()
+        cfg.device = device
+        cfg.rank, cfg.world = 0, 1
+        keep = []
+        if torch_allocator:
+            a, f = _torch_allocator(device)
+            cfg.alloc.alloc, cfg.alloc.free = a, f
+            keep += [a, f]
+        if stream is None:
+            try:
+                import torch
+                stream = torch.cuda.current_stream(device).cuda_stream
+            except Exception:  # pragma: no cover
+                stream = 0
+        cfg.stream = ctypes.c_void_p(int(stream))
+        return cfg, keep
+
+    @classmethod
+    def from_edges(cls, n_vertices, vertex_ids, src, dst, w, create_ts=0, device=0, stream=None,
+                   torch_allocator=True) -> "Replica":
+        cfg, keep = cls._config(device, stream, torch_allocator)
+        pi, ps, pd, pw = (_ptr(vertex_ids, np.uint64), _ptr(src, np.uint64), _ptr(dst, np.uint64),
+                          _ptr(w, np.float32))
+        ond = _on_device(pi, ps, pd, pw)
+        n_e = len(src) if src is not None else 0
+        h = ctypes.c_void_p()
+        rc = _lib.h2tap_replica_create_from_edges(ctypes.byref(cfg), int(n_vertices), pi[0], n_e,
+                                                  ps[0], pd[0], pw[0], ond, int(create_ts),
+                                                  ctypes.byref(h))
+        _check(rc, "h2tap_replica_create_from_edges")
+        return cls(h, keep + [cfg])
+
+    @classmethod
+    def from_csr(cls, offsets, cols, w, ext_ids=None, create_ts=0, device=0, stream=None,
+                 torch_allocator=True) -> "Replica":
+        cfg, keep = cls._config(device, stream, torch_allocator)
+        po, pc, pw, pi = (_ptr(offsets, np.int64), _ptr(cols, np.uint32), _ptr(w, np.float32),
+                          _ptr(ext_ids, np.uint64))
+        ond = _on_device(po, pc, pw, pi)
+        h = ctypes.c_void_p()
+        rc = _lib.h2tap_replica_create_from_csr(ctypes.byref(cfg), len(offsets) - 1, po[0], pc[0],
+                                                pw[0], pi[0], ond, int(create_ts), ctypes.byref(h))
+        _check(rc, "h2tap_replica_create_from_csr")
+        return cls(h, keep + [cfg])
+
+    # ----------------------------------------------------------------- apply
+    def apply(self, batch, snapshot_ts: int, raise_on_error: bool = True):
+        """h2tap_delta_apply; batch has .kind .src .dst .w .ts (numpy or torch CUDA)."""
+        pk, ps, pd, pw, pt = (_ptr(batch.kind, np.uint8), _ptr(batch.src, np.uint64),
+                              _ptr(batch.dst, np.uint64), _ptr(batch.w, np.float32),
+                              _ptr(batch.ts, np.uint64))
+        b = _Batch()
+        b.n = len(batch.kind)
+        b.on_device = _on_device(pk, ps, pd, pw, pt)
+        b.kind, b.src, b.dst, b.weight, b.ts = pk[0], ps[0], pd[0], pw[0], pt[0]
+        st = ApplyStats()
+        rc = _lib.h2tap_delta_apply(self._h, ctypes.byref(b), int(snapshot_ts), ctypes.byref(st))
+        if raise_on_error:
+            _check(rc, "h2tap_delta_apply")
+            return st.as_dict()
+        return rc, st.as_dict()
+
+    # ------------------------------------------------------------- read back
+    def info(self):
+        v = [_u64() for _ in range(6)]
+        _check(_lib.h2tap_replica_info(self._h, *(ctypes.byref(x) for x in v)), "h2tap_replica_info")
+        return dict(n_vertices=v[0].value, n_edges=v[1].value, snapshot_ts=v[2].value,
+                    n_pending=v[3].value, shard_vertex_base=v[4].value, shard_edge_base=v[5].value)
+
+    def export(self, on_device: bool = False, checksums: bool = False):
+        """(offsets, cols, w, ext_ids[, checksums]) as numpy (host) or torch CUDA tensors."""
+        inf = self.info()
+        V, E = inf["n_vertices"], inf["n_edges"]
+        if on_device:
+            import torch
+            dev = torch.device("cuda", torch.cuda.current_device())
+            out = (torch.empty(V + 1, dtype=torch.int64, device=dev),
+                   torch.empty(E, dtype=torch.int32, device=dev),
+                   torch.empty(E, dtype=torch.float32, device=dev),
+                   torch.empty(V, dtype=torch.int64, device=dev))
+            ptrs = [ctypes.c_void_p(t.data_ptr()) for t in out]
+        else:
+            out = (np.empty(V + 1, np.int64), np.empty(E, np.uint32), np.empty(E, np.float32),
+                   np.empty(V, np.uint64))
+            ptrs = [ctypes.c_void_p(a.ctypes.data) for a in out]
+        cs = (_u64 * 4)()
+        _check(_lib.h2tap_replica_export(self._h, *ptrs, int(on_device), cs if checksums else None),
+               "h2tap_replica_export")
+        return (*out, [int(x) for x in cs]) if checksums else out
+
+    def checksums(self):
+        cs = (_u64 * 4)()
+        _check(_lib.h2tap_replica_export(self._h, None, None, None, None, 0, cs), "h2tap_replica_export")
+        return [int(x) for x in cs]
+
+    def bfs(self, source_ext: int) -> np.ndarray:
+        lvl = np.empty(self.info()["n_vertices"], np.int32)
+        _check(_lib.h2tap_bfs(self._h, int(source_ext), ctypes.c_void_p(lvl.ctypes.data), 0), "h2tap_bfs")
+        return lvl
+
+    def pagerank(self, damping: float = 0.85, iterations: int = 20) -> np.ndarray:
+        pr = np.empty(self.info()["n_vertices"], np.float64)
+        _check(_lib.h2tap_pagerank(self._h, damping, iterations, ctypes.c_void_p(pr.ctypes.data), 0),
+               "h2tap_pagerank")
+        return pr
+
+    def close(self):
+        if getattr(self, "_h", None):
+            _lib.h2tap_replica_destroy(self._h)
+            self._h = None
+
+    def __del__(self):
+        try:
+            self.close()
+        except Exception:
+            pass
+
+    def __enter__(self):
+        return self
+
+    def __exit__(self, *a):
+        self.close()

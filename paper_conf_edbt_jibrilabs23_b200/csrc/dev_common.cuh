@@ -1,0 +1,138 @@
+// dev_common.cuh - device building blocks shared by the h2tap kernels (sm_100a).
+//
+//  * block-wide exclusive scans over per-thread item counts (warp shuffles + smem)
+//  * decoupled look-back (Merrill & Garland single-pass scan): each tile publishes
+//    its aggregate, then one warp inspects 32 predecessors at a time until it
+//    meets an inclusive prefix.  Status word: 2-bit flag | 62-bit value.
+//    Tiles take their index from an atomic counter, so every predecessor of a
+//    spinning tile has already been scheduled (forward progress).
+//  * lower_bound searches over sorted device arrays.
+#pragma once
+#include <cstdint>
+#include <cuda_runtime.h>
+
+namespace h2tap {
+
+constexpr int kWarp = 32;
+constexpr uint64_t kFlagAgg = 1ull << 62;
+constexpr uint64_t kFlagPrefix = 2ull << 62;
+constexpr uint64_t kValMask = (1ull << 62) - 1;
+constexpr uint32_t kNone32 = 0xFFFFFFFFu;
+
+__device__ __forceinline__ uint64_t sm64(uint64_t x) {
+    x += 0x9E3779B97F4A7C15ull;
+    x = (x ^ (x >> 30)) * 0xBF58476D1CE4E5B9ull;
+    x = (x ^ (x >> 27)) * 0x94D049BB133111EBull;
+    return x ^ (x >> 31);
+}
+
+__device__ __forceinline__ uint32_t lane_id() { return threadIdx.x & 31; }
+__device__ __forceinline__ uint32_t lanemask_lt() {
+    uint32_t m;
+    asm("mov.u32 %0, %%lanemask_lt;" : "=r"(m));
+    return m;
+}
+
+template <typename T>
+__device__ __forceinline__ T warp_inclusive_scan(T v) {
+#pragma unroll
+    for (int o = 1; o < 32; o <<= 1) {
+        T n = __shfl_up_sync(0xffffffffu, v, o);
+        if ((int)lane_id() >= o) v += n;
+    }
+    return v;
+}
+
+template <typename T>
+__device__ __forceinline__ T warp_sum(T v) {
+#pragma unroll
+    for (int o = 16; o > 0; o >>= 1) v += __shfl_xor_sync(0xffffffffu, v, o);
+    return v;
+}
+
+// Block-wide exclusive scan of one value per thread.  smem: >= NT/32 + 1 slots.
+// Returns the exclusive prefix; *total gets the block total (all threads).
+template <int NT, typename T>
+__device__ __forceinline__ T block_exclusive_scan(T v, T* smem, T* total) {
+    const int w = threadIdx.x >> 5;
+    T inc = warp_inclusive_scan(v);
+    if (lane_id() == 31) smem[w] = inc;
+    __syncthreads();
+    if (w == 0) {
+        T s = (lane_id() < NT / 32) ? smem[lane_id()] : T(0);
+        T si = warp_inclusive_scan(s);
+        if (lane_id() < NT / 32) smem[lane_id()] = si - s;
+        if (lane_id() == NT / 32 - 1) smem[NT / 32] = si;
+    }
+    __syncthreads();
+    T r = smem[w] + inc - v;
+    *total = smem[NT / 32];
+    __syncthreads();
+    return r;
+}
+
+// ---------------------------------------------------------------- look-back
+__device__ __forceinline__ uint64_t ld_volatile(const uint64_t* p) {
+    return *reinterpret_cast<const volatile uint64_t*>(p);
+}
+__device__ __forceinline__ void st_volatile(uint64_t* p, uint64_t v) {
+    *reinterpret_cast<volatile uint64_t*>(p) = v;
+}
+
+// Called by ONE full warp of the tile.  Publishes `aggregate` for `tile`, looks
+// back over predecessors, publishes the inclusive prefix, returns the exclusive
+// prefix (identical in all lanes).
+__device__ __forceinline__ uint64_t lookback_warp(uint64_t* status, uint32_t tile, uint64_t aggregate) {
+    if (tile == 0) {
+        if (lane_id() == 0) st_volatile(&status[0], kFlagPrefix | aggregate);
+        return 0;
+    }
+    if (lane_id() == 0) st_volatile(&status[tile], kFlagAgg | aggregate);
+    uint64_t excl = 0;
+    int64_t t = (int64_t)tile - 1;
+    while (true) {
+        int64_t idx = t - (int64_t)lane_id();  // lane 0 = nearest predecessor
+        uint64_t s = (idx >= 0) ? ld_volatile(&status[idx]) : kFlagPrefix;  // virtual prefix 0 before tile 0
+        uint32_t not_ready = __ballot_sync(0xffffffffu, (s >> 62) == 0);
+        if (not_ready) { continue; }  // spin until all 32 visible (predecessors are scheduled)
+        uint32_t is_prefix = __ballot_sync(0xffffffffu, (s >> 62) == 2);
+        // nearest prefix lane (smallest lane index with prefix)
+        int first = is_prefix ? (__ffs(is_prefix) - 1) : 32;
+        uint64_t v = ((int)lane_id() <= first) ? (s & kValMask) : 0;
+        excl += warp_sum(v);
+        if (is_prefix) break;
+        t -= 32;
+    }
+    if (lane_id() == 0) st_volatile(&status[tile], kFlagPrefix | (excl + aggregate));
+    return excl;
+}
+
+// ------------------------------------------------------------------ search
+// first index i in [lo, hi) with a[i] >= key (returns hi if none)
+template <typename T, typename K>
+__device__ __forceinline__ uint64_t lower_bound_dev(const T* a, uint64_t lo, uint64_t hi, K key) {
+    while (lo < hi) {
+        uint64_t mid = lo + ((hi - lo) >> 1);
+        if (a[mid] < key) lo = mid + 1; else hi = mid;
+    }
+    return lo;
+}
+// first index i in [lo, hi) with a[i] > key
+template <typename T, typename K>
+__device__ __forceinline__ uint64_t upper_bound_dev(const T* a, uint64_t lo, uint64_t hi, K key) {
+    while (lo < hi) {
+        uint64_t mid = lo + ((hi - lo) >> 1);
+        if (!(key < a[mid])) lo = mid + 1; else hi = mid;
+    }
+    return lo;
+}
+
+// (ts, seq) commit point, lexicographic (reading A5)
+struct Point {
+    uint64_t ts, seq;
+};
+__device__ __forceinline__ bool pt_less(uint64_t ts_a, uint64_t seq_a, uint64_t ts_b, uint64_t seq_b) {
+    return ts_a < ts_b || (ts_a == ts_b && seq_a < seq_b);
+}
+
+}  // namespace h2tap

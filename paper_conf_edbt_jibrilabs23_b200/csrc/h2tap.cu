@@ -1,0 +1,894 @@
+// h2tap.cu - host orchestrator and C ABI of libh2tap.so (include/h2tap.h).
+//
+// One propagation cycle (h2tap_delta_apply) runs these device steps on the
+// replica's stream:
+//   a1 k_partition         validate, number, split pending / node ops / edge ops
+//   a2 node ops            radix sort by (v, ts, seq), k_node_segments, k_node_lists,
+//                          k_remap + k_place_inserted (ID-map compaction), hd bitmap
+//   a3 edge ops            k_edge_prep (lookup, gating, packed key), onesweep radix
+//                          sort, k_reduce_classify (latest-commit-wins + outcome lists)
+//   a6 k_merge             global merge path into the back buffer
+//   a4/a5 k_offsets_*      new row offsets
+//   a7 swap                front <-> back at snapshot_ts (host pointer flip)
+// Host syncs read small counters between steps (sizes of the next launches).
+#include <cuda_runtime.h>
+
+#include <cstdarg>
+#include <cstdio>
+#include <cstring>
+#include <new>
+#include <string>
+
+#include "../../include/h2tap.h"
+#include "kernels.cuh"
+#include "radix_sort.cuh"
+
+using namespace h2tap;
+
+namespace {
+
+thread_local std::string g_err;
+
+void set_err(const char* fmt, ...) {
+    char buf[512];
+    va_list ap;
+    va_start(ap, fmt);
+    vsnprintf(buf, sizeof buf, fmt, ap);
+    va_end(ap);
+    g_err = buf;
+}
+
+struct Fail {
+    h2tap_status st;
+};
+
+#define CK(call)                                                                          \
+    do {                                                                                  \
+        cudaError_t e_ = (call);                                                          \
+        if (e_ != cudaSuccess) {                                                          \
+            set_err("%s:%d %s: %s", __FILE__, __LINE__, #call, cudaGetErrorString(e_));    \
+            throw Fail{e_ == cudaErrorMemoryAllocation ? H2TAP_E_NOMEM : H2TAP_E_CUDA};    \
+        }                                                                                 \
+    } while (0)
+thread_local uint64_t g_launches = 0, g_h2d = 0, g_d2h = 0;  // per-call accounting
+#define CKL()          \
+    do {               \
+        ++g_launches;  \
+        CK(cudaGetLastError()); \
+    } while (0)
+
+struct Buf {
+    void* p = nullptr;
+    size_t cap = 0;
+};
+
+inline uint64_t cdiv(uint64_t a, uint64_t b) { return (a + b - 1) / b; }
+inline int bits_for(uint64_t range) { return range == 0 ? 0 : 64 - __builtin_clzll(range); }
+
+}  // namespace
+
+struct h2tap_replica {
+    h2tap_config cfg{};
+    cudaStream_t st = nullptr;
+    uint64_t V = 0, E = 0, snap = 0, next_seq = 0, n_pend = 0;
+    bool identity = true, poisoned = false;
+    int cur = 0, ext_cur = 0, pcur = 0;
+    Buf off[2], cols[2], w[2], ext[2];
+    Buf pk[2], ps[2], pd[2], pw[2], pt[2], pq[2];
+    // scratch
+    Buf Wk, Ws, Wd, Ww, Wt, Wq, idx_p, idx_n, idx_e, status;
+    Buf keyA, keyB, valA, valB, hist, dbase, rs_status, rs_ctr;
+    Buf nv, nv_ext, dropped, ins_q, ins_oldpos, hd_rows, remap, hd_bits;
+    Buf op_flags, op_ou, op_ow;
+    Buf ins_pos, ins_row, ins_col, ins_w, del_pos, upd_pos, upd_w, KR;
+    Buf misc, nsorted, bfs_a, bfs_b, pr_a, pr_b;
+    Buf ctr;
+    Counters* hc = nullptr;  // pinned host mirror
+    cudaEvent_t ev[8]{};
+
+    void* dalloc(size_t bytes) {
+        void* p = nullptr;
+        if (cfg.alloc.alloc) {
+            p = cfg.alloc.alloc(cfg.alloc.ctx, bytes, (void*)st);
+            if (!p) { set_err("allocator returned NULL for %zu bytes", bytes); throw Fail{H2TAP_E_NOMEM}; }
+        } else {
+            cudaError_t e = cudaMallocAsync(&p, bytes, st);
+            if (e != cudaSuccess) {
+                cudaGetLastError();
+                set_err("cudaMallocAsync(%zu): %s", bytes, cudaGetErrorString(e));
+                throw Fail{H2TAP_E_NOMEM};
+            }
+        }
+        return p;
+    }
+    void dfree(void* p) {
+        if (!p) return;
+        if (cfg.alloc.alloc) { if (cfg.alloc.free) cfg.alloc.free(cfg.alloc.ctx, p, (void*)st); }
+        else cudaFreeAsync(p, st);
+    }
+    // grow-only buffer; 16 elements of slack so 128-bit loads may run past the end
+    template <typename T>
+    T* get(Buf& b, uint64_t count) {
+        size_t need = (size_t)(count + 16) * sizeof(T);
+        if (b.cap < need) {
+            if (b.p) dfree(b.p);
+            b.p = nullptr;
+            b.cap = 0;
+            size_t nc = need + need / 8;
+            b.p = dalloc(nc);
+            b.cap = nc;
+        }
+        return static_cast<T*>(b.p);
+    }
+    void release(Buf& b) { dfree(b.p); b.p = nullptr; b.cap = 0; }
+    void sync() { CK(cudaStreamSynchronize(st)); }
+    void read_counters() {
+        g_d2h += sizeof(Counters);
+        CK(cudaMemcpyAsync(hc, ctr.p, sizeof(Counters), cudaMemcpyDeviceToHost, st));
+        sync();
+    }
+    Counters* dctr() { return static_cast<Counters*>(ctr.p); }
+    template <typename T>
+    void zero(Buf& b, uint64_t count) { CK(cudaMemsetAsync(b.p, 0, count * sizeof(T), st)); }
+};
+
+namespace {
+
+// ---------------------------------------------------------------- sort ----
+// Stable LSD sort of (keys, vals)[0, n) on the low `bits` bits; result in (k, v).
+void radix_sort(h2tap_replica* r, uint64_t*& k, uint32_t*& v, uint64_t*& k2, uint32_t*& v2, uint64_t n, int bits) {
+    if (n <= 1 || bits <= 0) return;
+    const int passes = (bits + 7) / 8;
+    const uint64_t ntiles = cdiv(n, kRsTile);
+    uint32_t* hist = r->get<uint32_t>(r->hist, kRsMaxPasses * 256);
+    uint64_t* dbase = r->get<uint64_t>(r->dbase, kRsMaxPasses * 256);
+    uint64_t* st = r->get<uint64_t>(r->rs_status, (uint64_t)passes * ntiles * 256);
+    uint32_t* ctr = r->get<uint32_t>(r->rs_ctr, kRsMaxPasses);
+    CK(cudaMemsetAsync(hist, 0, kRsMaxPasses * 256 * sizeof(uint32_t), r->st));
+    CK(cudaMemsetAsync(st, 0, (size_t)passes * ntiles * 256 * sizeof(uint64_t), r->st));
+    CK(cudaMemsetAsync(ctr, 0, kRsMaxPasses * sizeof(uint32_t), r->st));
+    int grid = (int)std::min<uint64_t>(cdiv(n, 256 * 8), 148 * 8);
+    rs_histogram<<<grid, 256, 0, r->st>>>(k, n, passes, hist);
+    CKL();
+    rs_digit_base<<<passes, 256, 0, r->st>>>(hist, dbase);
+    CKL();
+    for (int p = 0; p < passes; ++p) {
+        rs_onesweep<<<(unsigned)ntiles, kRsThreads, 0, r->st>>>(k, v, k2, v2, n, 8 * p, dbase + p * 256,
+                                                              st + (uint64_t)p * ntiles * 256, ctr + p);
+        CKL();
+        std::swap(k, k2);
+        std::swap(v, v2);
+    }
+}
+
+struct BatchIn {
+    uint64_t n;
+    int on_device;
+    const uint8_t* kind;  // NULL -> all EDGE_INSERT (create)
+    const uint64_t* src;
+    const uint64_t* dst;
+    const float* w;
+    const uint64_t* ts;   // NULL -> all create_ts (create)
+    uint64_t fill_ts;
+};
+
+template <typename T>
+void copy_in(h2tap_replica* r, T* dst, const T* src, uint64_t n, int on_device) {
+    if (n == 0) return;
+    if (!on_device) g_h2d += n * sizeof(T);
+    CK(cudaMemcpyAsync(dst, src, n * sizeof(T), on_device ? cudaMemcpyDeviceToDevice : cudaMemcpyHostToDevice, r->st));
+}
+
+__global__ void k_fill_u8(uint8_t* p, uint64_t n, uint8_t v) {
+    uint64_t i = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x;
+    if (i < n) p[i] = v;
+}
+__global__ void k_fill_u64(uint64_t* p, uint64_t n, uint64_t v) {
+    uint64_t i = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x;
+    if (i < n) p[i] = v;
+}
+
+inline unsigned g1(uint64_t n, unsigned b = 256) { return (unsigned)std::max<uint64_t>(1, cdiv(n, b)); }
+
+float ev_ms(cudaEvent_t a, cudaEvent_t b) {
+    float ms = 0;
+    cudaEventElapsedTime(&ms, a, b);
+    return ms;
+}
+
+// One propagation cycle.  Nothing visible changes until the final swap.
+h2tap_status apply_core(h2tap_replica* r, const BatchIn& in, uint64_t S, bool create, h2tap_apply_stats* stats) {
+    cudaStream_t st = r->st;
+    const uint64_t n = in.n, np = r->n_pend, m = np + n;
+    if (m >= 0xFFFFFFFFull) { set_err("batch + pending = %llu ops exceeds 2^32-1", (unsigned long long)m); return H2TAP_E_CAPACITY; }
+    g_launches = g_h2d = g_d2h = 0;
+    for (int i = 0; i < 8; ++i)
+        if (!r->ev[i]) CK(cudaEventCreate(&r->ev[i]));
+    CK(cudaEventRecord(r->ev[0], st));
+
+    // ---- a1: assemble work ops (pending ++ batch) and partition
+    uint8_t* Wk = r->get<uint8_t>(r->Wk, m);
+    uint64_t* Ws = r->get<uint64_t>(r->Ws, m);
+    uint64_t* Wd = r->get<uint64_t>(r->Wd, m);
+    float* Ww = r->get<float>(r->Ww, m);
+    uint64_t* Wt = r->get<uint64_t>(r->Wt, m);
+    uint64_t* Wq = r->get<uint64_t>(r->Wq, m);
+    const int pc = r->pcur;
+    if (np) {
+        CK(cudaMemcpyAsync(Wk, r->pk[pc].p, np, cudaMemcpyDeviceToDevice, st));
+        CK(cudaMemcpyAsync(Ws, r->ps[pc].p, np * 8, cudaMemcpyDeviceToDevice, st));
+        CK(cudaMemcpyAsync(Wd, r->pd[pc].p, np * 8, cudaMemcpyDeviceToDevice, st));
+        CK(cudaMemcpyAsync(Ww, r->pw[pc].p, np * 4, cudaMemcpyDeviceToDevice, st));
+        CK(cudaMemcpyAsync(Wt, r->pt[pc].p, np * 8, cudaMemcpyDeviceToDevice, st));
+        CK(cudaMemcpyAsync(Wq, r->pq[pc].p, np * 8, cudaMemcpyDeviceToDevice, st));
+    }
+    if (n) {
+        if (in.kind) copy_in(r, Wk + np, in.kind, n, in.on_device);
+        else { k_fill_u8<<<g1(n), 256, 0, st>>>(Wk + np, n, EDGE_INSERT); CKL(); }
+        copy_in(r, Ws + np, in.src, n, in.on_device);
+        if (in.dst) copy_in(r, Wd + np, in.dst, n, in.on_device);
+        else CK(cudaMemsetAsync(Wd + np, 0, n * 8, st));
+        if (in.w) copy_in(r, Ww + np, in.w, n, in.on_device);
+        else CK(cudaMemsetAsync(Ww + np, 0, n * 4, st));
+        if (in.ts) copy_in(r, Wt + np, in.ts, n, in.on_device);
+        else { k_fill_u64<<<g1(n), 256, 0, st>>>(Wt + np, n, in.fill_ts); CKL(); }
+        k_fill_seq<<<g1(n), 256, 0, st>>>(Wq, np, n, r->next_seq);
+        CKL();
+    }
+    Ops ops{Wk, Ws, Wd, Ww, Wt, Wq};
+
+    Counters init{};
+    init.ts_min = ~0ull;
+    init.v_min = ~0ull;
+    r->get<Counters>(r->ctr, 1);
+    *r->hc = init;
+    CK(cudaMemcpyAsync(r->ctr.p, r->hc, sizeof(Counters), cudaMemcpyHostToDevice, st));
+    g_h2d += sizeof(Counters);
+    Counters* dc = r->dctr();
+
+    uint32_t* idx_p = r->get<uint32_t>(r->idx_p, m);
+    uint32_t* idx_n = r->get<uint32_t>(r->idx_n, m);
+    uint32_t* idx_e = r->get<uint32_t>(r->idx_e, m);
+    if (m) {
+        uint64_t nt = cdiv(m, kTile);
+        uint64_t* stt = r->get<uint64_t>(r->status, 3 * nt);
+        CK(cudaMemsetAsync(stt, 0, 3 * nt * 8, st));
+        k_partition<<<(unsigned)nt, kThreads, 0, st>>>(ops, m, np, r->snap, S, create ? 0 : 1, idx_p, idx_n, idx_e,
+                                                       stt, nt, dc);
+        CKL();
+    }
+    r->read_counters();
+    Counters hc = *r->hc;
+    if (hc.status & ST_BAD_KIND) { set_err("unknown op kind in batch"); return H2TAP_E_INVAL; }
+    if (hc.status & ST_STALE) {
+        set_err("op with ts <= current snapshot_ts %llu (reading A7)", (unsigned long long)r->snap);
+        return H2TAP_E_STALE_TS;
+    }
+    const uint64_t n_pend_new = hc.n_pend, n_node = hc.n_node, n_edge = hc.n_edge;
+    CK(cudaEventRecord(r->ev[1], st));
+
+    // ---- a2: node ops -> per-vertex timeline, ID-map compaction, remap
+    const uint64_t V = r->V, E = r->E;
+    const int ec = r->ext_cur;
+    const uint64_t* old_ext = static_cast<const uint64_t*>(r->ext[ec].p);
+    uint64_t U = 0, n_dropped = 0, n_vins = 0, n_hd = 0, Vn = V;
+    bool remap_on = false, set_changed = false;
+    NodeVtx* nv = nullptr;
+    uint64_t* nv_ext = nullptr;
+    uint32_t *dropped = nullptr, *ins_q = nullptr, *ins_oldpos = nullptr, *hd_rows = nullptr, *remap = nullptr,
+             *hd_bits = nullptr, *node_sorted = nullptr;
+    uint64_t* new_ext = nullptr;
+    if (n_node) {
+        uint64_t* kA = r->get<uint64_t>(r->keyA, n_node);
+        uint64_t* kB = r->get<uint64_t>(r->keyB, n_node);
+        uint32_t* vA = r->get<uint32_t>(r->valA, n_node);
+        uint32_t* vB = r->get<uint32_t>(r->valB, n_node);
+        // stable by ts (input is in seq order), then stable by vertex -> (v, ts, seq)
+        k_keys_from<<<g1(n_node), 256, 0, st>>>(idx_n, n_node, Wt, hc.ts_min, kA, vA);
+        CKL();
+        radix_sort(r, kA, vA, kB, vB, n_node, bits_for(hc.ts_max - hc.ts_min));
+        k_keys_from<<<g1(n_node), 256, 0, st>>>(vA, n_node, Ws, hc.v_min, kB, vB);
+        CKL();
+        std::swap(kA, kB);
+        std::swap(vA, vB);
+        radix_sort(r, kA, vA, kB, vB, n_node, bits_for(hc.v_max - hc.v_min));
+        node_sorted = r->get<uint32_t>(r->nsorted, n_node);
+        CK(cudaMemcpyAsync(node_sorted, vA, n_node * 4, cudaMemcpyDeviceToDevice, st));
+
+        nv = r->get<NodeVtx>(r->nv, n_node);
+        nv_ext = r->get<uint64_t>(r->nv_ext, n_node);
+        uint64_t nt = cdiv(n_node, kTile);
+        uint64_t* stt = r->get<uint64_t>(r->status, 3 * nt);
+        CK(cudaMemsetAsync(stt, 0, nt * 8, st));
+        k_node_segments<<<(unsigned)nt, kThreads, 0, st>>>(ops, node_sorted, n_node, old_ext, V, r->identity, nv,
+                                                           nv_ext, stt, nt, dc);
+        CKL();
+        r->read_counters();
+        U = r->hc->n_unique;
+        dropped = r->get<uint32_t>(r->dropped, U);
+        ins_q = r->get<uint32_t>(r->ins_q, U);
+        ins_oldpos = r->get<uint32_t>(r->ins_oldpos, U);
+        hd_rows = r->get<uint32_t>(r->hd_rows, U);
+        uint64_t nt2 = cdiv(U, kTile);
+        stt = r->get<uint64_t>(r->status, 3 * nt2);
+        CK(cudaMemsetAsync(stt, 0, 3 * nt2 * 8, st));
+        k_node_lists<<<(unsigned)nt2, kThreads, 0, st>>>(nv, U, dropped, ins_q, ins_oldpos, hd_rows, stt, nt2, dc);
+        CKL();
+        uint32_t first_ins_oldpos = 0;
+        r->read_counters();
+        n_dropped = r->hc->n_dropped;
+        n_vins = r->hc->n_inserted;
+        n_hd = r->hc->n_hd;
+        if (n_vins) {
+            g_d2h += 4;
+            CK(cudaMemcpyAsync(&r->hc->status, ins_oldpos, 4, cudaMemcpyDeviceToHost, st));
+            r->sync();
+            first_ins_oldpos = (uint32_t)(r->hc->status & 0xFFFFFFFFu);
+        }
+        Vn = V - n_dropped + n_vins;
+        if (Vn >= 0xFFFFFFFFull) { set_err("vertex count exceeds 2^32-1"); return H2TAP_E_CAPACITY; }
+        set_changed = n_dropped || n_vins;
+        remap_on = n_dropped > 0 || (n_vins > 0 && first_ins_oldpos < V);
+        if (set_changed) {
+            new_ext = r->get<uint64_t>(r->ext[ec ^ 1], Vn);
+            if (remap_on) {
+                remap = r->get<uint32_t>(r->remap, V);
+                if (V) {
+                    k_remap<<<g1(V, kThreads * kItems), kThreads, 0, st>>>(old_ext, r->identity, V, dropped, n_dropped,
+                                                                           ins_oldpos, n_vins, remap, new_ext);
+                    CKL();
+                }
+            } else if (V) {
+                CK(cudaMemcpyAsync(new_ext, old_ext, V * 8, cudaMemcpyDeviceToDevice, st));
+            }
+            if (n_vins) {
+                k_place_inserted<<<g1(n_vins), 256, 0, st>>>(nv, nv_ext, ins_q, ins_oldpos, n_vins, dropped, n_dropped,
+                                                            new_ext);
+                CKL();
+            }
+        }
+        k_nv_newid<<<g1(U), 256, 0, st>>>(nv, U, remap, remap_on ? 1 : 0);
+        CKL();
+        if (n_hd) {
+            hd_bits = r->get<uint32_t>(r->hd_bits, cdiv(V, 32));
+            CK(cudaMemsetAsync(hd_bits, 0, cdiv(V, 32) * 4, st));
+            k_set_bits<<<g1(n_hd), 256, 0, st>>>(hd_rows, n_hd, hd_bits);
+            CKL();
+        }
+    }
+    CK(cudaEventRecord(r->ev[2], st));
+
+    // ---- a3: edge ops -> keys, sort, segmented reduce + classify
+    const int bits = std::max(1, bits_for(Vn > 1 ? Vn - 1 : 1));
+    const int64_t* old_off = static_cast<const int64_t*>(r->off[r->cur].p);
+    const uint32_t* old_cols = static_cast<const uint32_t*>(r->cols[r->cur].p);
+    const float* old_w = static_cast<const float*>(r->w[r->cur].p);
+    uint64_t n_valid = 0, n_ins = 0, n_del = 0, n_upd = 0, n_gated = 0;
+    uint64_t* ins_pos = r->get<uint64_t>(r->ins_pos, 1);
+    uint32_t* ins_row = r->get<uint32_t>(r->ins_row, 1);
+    uint32_t* ins_col = r->get<uint32_t>(r->ins_col, 1);
+    float* ins_w = r->get<float>(r->ins_w, 1);
+    uint64_t* del_pos = r->get<uint64_t>(r->del_pos, 1);
+    uint64_t* upd_pos = r->get<uint64_t>(r->upd_pos, 1);
+    float* upd_w = r->get<float>(r->upd_w, 1);
+    if (n_edge) {
+        uint64_t* kA = r->get<uint64_t>(r->keyA, n_edge);
+        uint64_t* kB = r->get<uint64_t>(r->keyB, n_edge);
+        uint32_t* vA = r->get<uint32_t>(r->valA, n_edge);
+        uint32_t* vB = r->get<uint32_t>(r->valB, n_edge);
+        PrepArgs pa{};
+        pa.ops = ops;
+        pa.edge_idx = idx_e;
+        pa.n_edge = n_edge;
+        pa.old_ext = old_ext;
+        pa.V = V;
+        pa.identity = r->identity;
+        pa.remap = remap_on ? remap : nullptr;
+        pa.nv = nv;
+        pa.nv_ext = nv_ext;
+        pa.U = U;
+        pa.node_sorted = node_sorted;
+        pa.bits = bits;
+        pa.create = create ? 1 : 0;
+        pa.keys = kA;
+        pa.vals = vA;
+        pa.op_flags = r->get<uint8_t>(r->op_flags, m);
+        pa.op_opos_u = r->get<uint32_t>(r->op_ou, m);
+        pa.op_opos_w = r->get<uint32_t>(r->op_ow, m);
+        uint64_t nt = cdiv(n_edge, kTile);
+        pa.status = r->get<uint64_t>(r->status, 3 * nt);
+        CK(cudaMemsetAsync(pa.status, 0, nt * 8, st));
+        pa.n_tiles = nt;
+        pa.c = dc;
+        k_edge_prep<<<(unsigned)nt, kThreads, 0, st>>>(pa);
+        CKL();
+        r->read_counters();
+        if (create && (r->hc->status & ST_CREATE_ENDPOINT)) {
+            set_err("create: edge endpoint not in the vertex set");
+            return H2TAP_E_INVAL;
+        }
+        n_valid = r->hc->n_valid;
+        n_gated = r->hc->n_gated;
+        radix_sort(r, kA, vA, kB, vB, n_valid, 2 * bits);
+        ins_pos = r->get<uint64_t>(r->ins_pos, n_valid);
+        ins_row = r->get<uint32_t>(r->ins_row, n_valid);
+        ins_col = r->get<uint32_t>(r->ins_col, n_valid);
+        ins_w = r->get<float>(r->ins_w, n_valid);
+        del_pos = r->get<uint64_t>(r->del_pos, n_valid);
+        upd_pos = r->get<uint64_t>(r->upd_pos, n_valid);
+        upd_w = r->get<float>(r->upd_w, n_valid);
+        if (n_valid) {
+            ClassArgs ca{};
+            ca.ops = ops;
+            ca.keys = kA;
+            ca.vals = vA;
+            ca.n = n_valid;
+            ca.bits = bits;
+            ca.op_flags = pa.op_flags;
+            ca.op_opos_u = pa.op_opos_u;
+            ca.op_opos_w = pa.op_opos_w;
+            ca.old_off = old_off;
+            ca.old_cols = old_cols;
+            ca.ins_pos = ins_pos; ca.ins_row = ins_row; ca.ins_col = ins_col; ca.ins_w = ins_w;
+            ca.del_pos = del_pos;
+            ca.upd_pos = upd_pos; ca.upd_w = upd_w;
+            uint64_t nt2 = cdiv(n_valid, kTile);
+            ca.status3 = r->get<uint64_t>(r->status, 3 * nt2);
+            CK(cudaMemsetAsync(ca.status3, 0, 3 * nt2 * 8, st));
+            ca.n_tiles = nt2;
+            ca.c = dc;
+            k_reduce_classify<<<(unsigned)nt2, kThreads, 0, st>>>(ca);
+            CKL();
+            r->read_counters();
+            n_ins = r->hc->n_ins;
+            n_del = r->hc->n_del;
+            n_upd = r->hc->n_upd;
+        }
+    }
+    CK(cudaEventRecord(r->ev[3], st));
+
+    // ---- a6: merge into the back buffer (skipped when no op changes the CSR)
+    const bool csr_changed = n_node || n_ins || n_del || n_upd;
+    const int nb = csr_changed ? (r->cur ^ 1) : r->cur;
+    uint64_t n_casc = 0, En = E;
+    if (csr_changed) {
+    const uint64_t Ecap = E + n_ins;
+    int64_t* new_off = r->get<int64_t>(r->off[nb], Vn + 1);
+    uint32_t* new_cols = r->get<uint32_t>(r->cols[nb], Ecap);
+    float* new_w = r->get<float>(r->w[nb], Ecap);
+    const bool casc = n_hd > 0;
+    int64_t* KR = casc ? r->get<int64_t>(r->KR, V + 1) : nullptr;
+    const uint64_t Dtot = E + n_ins;
+    if (Dtot) {
+        MergeArgs ma{};
+        ma.old_cols = old_cols; ma.old_w = old_w; ma.old_off = old_off; ma.E_old = E; ma.V_old = V;
+        ma.ins_pos = ins_pos; ma.ins_col = ins_col; ma.ins_w = ins_w; ma.n_ins = n_ins;
+        ma.del_pos = del_pos; ma.n_del = n_del;
+        ma.upd_pos = upd_pos; ma.upd_w = upd_w; ma.n_upd = n_upd;
+        ma.remap = remap; ma.hd_bits = hd_bits; ma.hd_rows = hd_rows; ma.n_hd = n_hd;
+        ma.new_cols = new_cols; ma.new_w = new_w; ma.KR = KR;
+        ma.n_tiles = cdiv(Dtot, kMergeTile);
+        ma.c = dc;
+        if (casc) {
+            ma.status = r->get<uint64_t>(r->status, ma.n_tiles);
+            CK(cudaMemsetAsync(ma.status, 0, ma.n_tiles * 8, st));
+        }
+        const unsigned grid = (unsigned)ma.n_tiles;
+        if (casc && remap_on) k_merge<true, true><<<grid, kThreads, 0, st>>>(ma);
+        else if (casc) k_merge<true, false><<<grid, kThreads, 0, st>>>(ma);
+        else if (remap_on) k_merge<false, true><<<grid, kThreads, 0, st>>>(ma);
+        else k_merge<false, false><<<grid, kThreads, 0, st>>>(ma);
+        CKL();
+    } else if (casc) {
+        CK(cudaMemsetAsync(KR, 0, (V + 1) * 8, st));
+    }
+    CK(cudaEventRecord(r->ev[4], st));
+    if (casc) {
+        r->read_counters();
+        n_casc = r->hc->n_casc;
+    }
+    En = E + n_ins - n_del - n_casc;
+
+    // ---- a4/a5: row offsets
+    if (V) {
+        unsigned grid = g1(V, kThreads * kItems);
+        const uint32_t* rm = remap_on ? remap : nullptr;
+        if (casc && remap_on) k_offsets_old<true, true><<<grid, kThreads, 0, st>>>(old_off, V, KR, del_pos, n_del, ins_row, n_ins, rm, new_off);
+        else if (casc) k_offsets_old<true, false><<<grid, kThreads, 0, st>>>(old_off, V, KR, del_pos, n_del, ins_row, n_ins, rm, new_off);
+        else if (remap_on) k_offsets_old<false, true><<<grid, kThreads, 0, st>>>(old_off, V, KR, del_pos, n_del, ins_row, n_ins, rm, new_off);
+        else k_offsets_old<false, false><<<grid, kThreads, 0, st>>>(old_off, V, KR, del_pos, n_del, ins_row, n_ins, rm, new_off);
+        CKL();
+    }
+    if (n_vins) {
+        if (casc) k_offsets_inserted<true><<<g1(n_vins), 256, 0, st>>>(nv, ins_q, n_vins, old_off, KR, del_pos, n_del, ins_row, n_ins, new_off);
+        else k_offsets_inserted<false><<<g1(n_vins), 256, 0, st>>>(nv, ins_q, n_vins, old_off, KR, del_pos, n_del, ins_row, n_ins, new_off);
+        CKL();
+    }
+    k_set_i64<<<1, 1, 0, st>>>(new_off + Vn, (int64_t)En);
+    CKL();
+    } else {
+        CK(cudaEventRecord(r->ev[4], st));
+    }
+
+    // ---- new pending set (double-buffered so an error above leaves the old one intact)
+    const int pn = pc ^ 1;
+    if (n_pend_new) {
+        k_gather_ops<<<g1(n_pend_new), 256, 0, st>>>(
+            ops, idx_p, n_pend_new, r->get<uint8_t>(r->pk[pn], n_pend_new), r->get<uint64_t>(r->ps[pn], n_pend_new),
+            r->get<uint64_t>(r->pd[pn], n_pend_new), r->get<float>(r->pw[pn], n_pend_new),
+            r->get<uint64_t>(r->pt[pn], n_pend_new), r->get<uint64_t>(r->pq[pn], n_pend_new));
+        CKL();
+    }
+    CK(cudaEventRecord(r->ev[5], st));
+    bool new_identity = r->identity;
+    if (set_changed) {
+        if (Vn == 0) new_identity = true;
+        else {
+            uint64_t last = 0;
+            g_d2h += 8;
+            CK(cudaMemcpyAsync(&r->hc->status, new_ext + Vn - 1, 8, cudaMemcpyDeviceToHost, st));
+            r->sync();
+            last = r->hc->status;
+            new_identity = (last == Vn - 1);
+        }
+    }
+    r->sync();
+
+    // ---- a7: swap at snapshot_ts (nothing above touched the front state)
+    r->cur = nb;
+    if (set_changed) r->ext_cur = ec ^ 1;
+    r->identity = new_identity;
+    r->V = Vn;
+    r->E = En;
+    r->pcur = pn;
+    r->n_pend = n_pend_new;
+    r->next_seq += n;
+    r->snap = S;
+    if (stats) {
+        memset(stats, 0, sizeof *stats);
+        stats->n_visible = n_node + n_edge;
+        stats->n_deferred = n_pend_new;
+        stats->n_gated = n_gated;
+        stats->n_new = n_ins;
+        stats->n_del = n_del;
+        stats->n_upd = n_upd;
+        stats->n_casc = n_casc;
+        stats->n_vertex_inserted = n_vins;
+        stats->n_vertex_deleted = n_dropped;
+        stats->ms_ingest = ev_ms(r->ev[0], r->ev[1]);
+        stats->ms_nodeops = ev_ms(r->ev[1], r->ev[2]);
+        stats->ms_sort_reduce = ev_ms(r->ev[2], r->ev[3]);
+        stats->ms_merge = ev_ms(r->ev[3], r->ev[4]);
+        stats->ms_degree_scan = ev_ms(r->ev[4], r->ev[5]);
+        stats->ms_total = ev_ms(r->ev[0], r->ev[5]);
+        uint64_t b = 8 * (V + 1) + 8 * E + 8 * (Vn + 1) + 8 * En + 29 * n;
+        if (n_node) b += 16 * V + 4 * E + 4 * V;
+        stats->bytes_alg = b;
+        // merge launch: stream old cols+weights, write new ones, read the outcome lists
+        // (+ remap table and cascade bitmap when node ops changed the ID map)
+        uint64_t bm = 0;
+        if (csr_changed && E + n_ins) {
+            bm = 8 * E + 8 * En + 20 * n_ins + 8 * n_del + 12 * n_upd;
+            if (remap_on) bm += 4 * V;
+            if (n_hd) bm += V / 8 + 4 * n_hd;
+        }
+        stats->bytes_merge = bm;
+        stats->n_launches = g_launches;
+        stats->h2d_bytes = g_h2d;
+        stats->d2h_bytes = g_d2h;
+    }
+    return H2TAP_OK;
+}
+
+template <typename F>
+h2tap_status run_guarded(h2tap_replica* r, F&& f) {
+    if (r && r->poisoned) { set_err("replica poisoned by an earlier CUDA error"); return H2TAP_E_POISONED; }
+    try {
+        return f();
+    } catch (const Fail& e) {
+        if (r && e.st == H2TAP_E_CUDA) {
+            cudaError_t s = cudaDeviceSynchronize();
+            if (s != cudaSuccess) r->poisoned = true;
+            cudaGetLastError();
+        }
+        return e.st;
+    } catch (const std::bad_alloc&) {
+        set_err("host allocation failed");
+        return H2TAP_E_NOMEM;
+    } catch (...) {
+        set_err("unexpected C++ exception");
+        return H2TAP_E_CUDA;
+    }
+}
+
+h2tap_replica* new_replica(const h2tap_config* cfg) {
+    h2tap_replica* r = new h2tap_replica();
+    if (cfg) r->cfg = *cfg;
+    else { r->cfg.world = 1; }
+    if (r->cfg.world <= 0) r->cfg.world = 1;
+    CK(cudaSetDevice(r->cfg.device));
+    r->st = static_cast<cudaStream_t>(r->cfg.stream);
+    CK(cudaMallocHost(&r->hc, sizeof(Counters)));
+    r->get<Counters>(r->ctr, 1);
+    return r;
+}
+
+void free_replica(h2tap_replica* r) {
+    if (!r) return;
+    Buf* bufs[] = {&r->off[0], &r->off[1], &r->cols[0], &r->cols[1], &r->w[0], &r->w[1], &r->ext[0], &r->ext[1],
+                   &r->pk[0], &r->pk[1], &r->ps[0], &r->ps[1], &r->pd[0], &r->pd[1], &r->pw[0], &r->pw[1],
+                   &r->pt[0], &r->pt[1], &r->pq[0], &r->pq[1], &r->Wk, &r->Ws, &r->Wd, &r->Ww, &r->Wt, &r->Wq,
+                   &r->idx_p, &r->idx_n, &r->idx_e, &r->status, &r->keyA, &r->keyB, &r->valA, &r->valB,
+                   &r->hist, &r->dbase, &r->rs_status, &r->rs_ctr, &r->nv, &r->nv_ext, &r->dropped, &r->ins_q,
+                   &r->ins_oldpos, &r->hd_rows, &r->remap, &r->hd_bits, &r->op_flags, &r->op_ou, &r->op_ow,
+                   &r->ins_pos, &r->ins_row, &r->ins_col, &r->ins_w, &r->del_pos, &r->upd_pos, &r->upd_w,
+                   &r->KR, &r->misc, &r->nsorted, &r->bfs_a, &r->bfs_b, &r->pr_a, &r->pr_b, &r->ctr};
+    for (Buf* b : bufs) if (b->p) r->dfree(b->p);
+    cudaStreamSynchronize(r->st);
+    for (auto& e : r->ev) if (e) cudaEventDestroy(e);
+    if (r->hc) cudaFreeHost(r->hc);
+    delete r;
+}
+
+// empty replica over a vertex set (ids strictly increasing or identity)
+void init_vertices(h2tap_replica* r, uint64_t nv, const uint64_t* ids, int on_device) {
+    r->V = nv;
+    r->E = 0;
+    uint64_t* ext = r->get<uint64_t>(r->ext[0], nv);
+    if (ids) copy_in(r, ext, ids, nv, on_device);
+    else if (nv) { k_iota_u64<<<g1(nv), 256, 0, r->st>>>(ext, nv); CKL(); }
+    int64_t* off = r->get<int64_t>(r->off[0], nv + 1);
+    CK(cudaMemsetAsync(off, 0, (nv + 1) * 8, r->st));
+    r->get<uint32_t>(r->cols[0], 0);
+    r->get<float>(r->w[0], 0);
+    r->identity = (ids == nullptr);
+    if (ids && nv) {
+        // validate strictly increasing ids (and detect identity)
+        unsigned long long* bad = r->get<unsigned long long>(r->misc, 1);
+        CK(cudaMemsetAsync(bad, 0, 8, r->st));
+        k_validate_csr<<<g1(nv), 256, 0, r->st>>>(off, nullptr, nv, ext, bad);
+        CKL();
+        uint64_t h[2];
+        CK(cudaMemcpyAsync(&h[0], bad, 8, cudaMemcpyDeviceToHost, r->st));
+        CK(cudaMemcpyAsync(&h[1], ext + nv - 1, 8, cudaMemcpyDeviceToHost, r->st));
+        r->sync();
+        if (h[0]) { set_err("vertex ids not strictly increasing"); throw Fail{H2TAP_E_INVAL}; }
+        r->identity = (h[1] == nv - 1);
+    }
+}
+
+}  // namespace
+
+// ======================================================================= ABI ==
+extern "C" {
+
+const char* h2tap_version(void) { return "h2tap-b200 0.1 (sm_100a)"; }
+const char* h2tap_last_error(void) { return g_err.c_str(); }
+
+const char* h2tap_status_str(h2tap_status s) {
+    switch (s) {
+        case H2TAP_OK: return "OK";
+        case H2TAP_E_INVAL: return "E_INVAL";
+        case H2TAP_E_NOMEM: return "E_NOMEM";
+        case H2TAP_E_CUDA: return "E_CUDA";
+        case H2TAP_E_NCCL: return "E_NCCL";
+        case H2TAP_E_STALE_TS: return "E_STALE_TS";
+        case H2TAP_E_SNAPSHOT_REGRESSION: return "E_SNAPSHOT_REGRESSION";
+        case H2TAP_E_CAPACITY: return "E_CAPACITY";
+        case H2TAP_E_POISONED: return "E_POISONED";
+    }
+    return "unknown";
+}
+
+h2tap_status h2tap_replica_create_from_edges(const h2tap_config* cfg, size_t n_vertices, const uint64_t* vertex_ids,
+                                             size_t n_edges, const uint64_t* src, const uint64_t* dst, const float* w,
+                                             int on_device, uint64_t create_ts, h2tap_replica** out) {
+    if (!out || (n_edges && (!src || !dst))) { set_err("null argument"); return H2TAP_E_INVAL; }
+    if (cfg && cfg->world > 1) { set_err("multi-GPU replicas are not enabled in this build"); return H2TAP_E_INVAL; }
+    if (n_vertices >= 0xFFFFFFFFull) { set_err("n_vertices >= 2^32-1"); return H2TAP_E_CAPACITY; }
+    *out = nullptr;
+    h2tap_replica* r = nullptr;
+    h2tap_status s = run_guarded(nullptr, [&]() -> h2tap_status {
+        r = new_replica(cfg);
+        init_vertices(r, n_vertices, vertex_ids, on_device);
+        r->snap = 0;
+        BatchIn in{n_edges, on_device, nullptr, src, dst, w, nullptr, create_ts};
+        h2tap_status st = apply_core(r, in, create_ts, true, nullptr);
+        if (st != H2TAP_OK) return st;
+        r->snap = create_ts;
+        r->next_seq = 0;
+        return H2TAP_OK;
+    });
+    if (s != H2TAP_OK) { free_replica(r); return s; }
+    *out = r;
+    return H2TAP_OK;
+}
+
+h2tap_status h2tap_replica_create_from_csr(const h2tap_config* cfg, size_t n_vertices, const int64_t* offsets,
+                                           const uint32_t* cols, const float* w, const uint64_t* ext_ids,
+                                           int on_device, uint64_t create_ts, h2tap_replica** out) {
+    if (!out || !offsets) { set_err("null argument"); return H2TAP_E_INVAL; }
+    if (cfg && cfg->world > 1) { set_err("multi-GPU replicas are not enabled in this build"); return H2TAP_E_INVAL; }
+    if (n_vertices >= 0xFFFFFFFFull) { set_err("n_vertices >= 2^32-1"); return H2TAP_E_CAPACITY; }
+    *out = nullptr;
+    h2tap_replica* r = nullptr;
+    h2tap_status s = run_guarded(nullptr, [&]() -> h2tap_status {
+        r = new_replica(cfg);
+        init_vertices(r, n_vertices, ext_ids, on_device);
+        int64_t* off = static_cast<int64_t*>(r->off[0].p);
+        copy_in(r, off, offsets, n_vertices + 1, on_device);
+        int64_t E = 0;
+        CK(cudaMemcpyAsync(&E, off + n_vertices, 8, cudaMemcpyDeviceToHost, r->st));
+        r->sync();
+        if (E < 0) { set_err("negative edge count"); return H2TAP_E_INVAL; }
+        uint32_t* c = r->get<uint32_t>(r->cols[0], E);
+        float* ww = r->get<float>(r->w[0], E);
+        if (E && !cols) { set_err("cols is NULL"); return H2TAP_E_INVAL; }
+        copy_in(r, c, cols, E, on_device);
+        if (w) copy_in(r, ww, w, E, on_device);
+        else CK(cudaMemsetAsync(ww, 0, E * 4, r->st));
+        unsigned long long* bad = r->get<unsigned long long>(r->misc, 1);
+        CK(cudaMemsetAsync(bad, 0, 8, r->st));
+        if (n_vertices) {
+            k_validate_csr<<<g1(n_vertices), 256, 0, r->st>>>(off, c, n_vertices, nullptr, bad);
+            CKL();
+        }
+        uint64_t hb = 0;
+        CK(cudaMemcpyAsync(&hb, bad, 8, cudaMemcpyDeviceToHost, r->st));
+        r->sync();
+        if (hb || (n_vertices == 0 && E != 0)) { set_err("malformed CSR"); return H2TAP_E_INVAL; }
+        r->E = E;
+        r->snap = create_ts;
+        return H2TAP_OK;
+    });
+    if (s != H2TAP_OK) { free_replica(r); return s; }
+    *out = r;
+    return H2TAP_OK;
+}
+
+h2tap_status h2tap_delta_apply(h2tap_replica* r, const h2tap_batch* b, uint64_t snapshot_ts, h2tap_apply_stats* stats) {
+    if (!r || !b) { set_err("null argument"); return H2TAP_E_INVAL; }
+    if (b->n && (!b->kind || !b->src || !b->ts)) { set_err("batch kind/src/ts must be non-NULL"); return H2TAP_E_INVAL; }
+    return run_guarded(r, [&]() -> h2tap_status {
+        if (snapshot_ts < r->snap) {
+            set_err("snapshot_ts %llu < current %llu", (unsigned long long)snapshot_ts, (unsigned long long)r->snap);
+            return H2TAP_E_SNAPSHOT_REGRESSION;
+        }
+        CK(cudaSetDevice(r->cfg.device));
+        BatchIn in{b->n, b->on_device, b->kind, b->src, b->dst, b->weight, b->ts, 0};
+        return apply_core(r, in, snapshot_ts, false, stats);
+    });
+}
+
+h2tap_status h2tap_replica_info(const h2tap_replica* r, uint64_t* nv, uint64_t* ne, uint64_t* snap, uint64_t* npend,
+                                uint64_t* vbase, uint64_t* ebase) {
+    if (!r) { set_err("null replica"); return H2TAP_E_INVAL; }
+    if (nv) *nv = r->V;
+    if (ne) *ne = r->E;
+    if (snap) *snap = r->snap;
+    if (npend) *npend = r->n_pend;
+    if (vbase) *vbase = 0;
+    if (ebase) *ebase = 0;
+    return H2TAP_OK;
+}
+
+h2tap_status h2tap_replica_export(const h2tap_replica* rc, int64_t* offsets, uint32_t* cols, float* w,
+                                  uint64_t* ext_ids, int on_device, uint64_t checksums[4]) {
+    h2tap_replica* r = const_cast<h2tap_replica*>(rc);
+    if (!r) { set_err("null replica"); return H2TAP_E_INVAL; }
+    return run_guarded(r, [&]() -> h2tap_status {
+        CK(cudaSetDevice(r->cfg.device));
+        cudaMemcpyKind k = on_device ? cudaMemcpyDeviceToDevice : cudaMemcpyDeviceToHost;
+        const int c = r->cur;
+        if (offsets) CK(cudaMemcpyAsync(offsets, r->off[c].p, (r->V + 1) * 8, k, r->st));
+        if (cols && r->E) CK(cudaMemcpyAsync(cols, r->cols[c].p, r->E * 4, k, r->st));
+        if (w && r->E) CK(cudaMemcpyAsync(w, r->w[c].p, r->E * 4, k, r->st));
+        if (ext_ids && r->V) CK(cudaMemcpyAsync(ext_ids, r->ext[r->ext_cur].p, r->V * 8, k, r->st));
+        if (checksums) {
+            unsigned long long* cs = r->get<unsigned long long>(r->misc, 4);
+            CK(cudaMemsetAsync(cs, 0, 32, r->st));
+            auto grid = [](uint64_t n) { return (unsigned)std::max<uint64_t>(1, std::min<uint64_t>(cdiv(n, 256), 148 * 16)); };
+            k_checksum<int64_t><<<grid(r->V + 1), 256, 0, r->st>>>(static_cast<int64_t*>(r->off[c].p), r->V + 1, 1, cs);
+            k_checksum<uint32_t><<<grid(r->E), 256, 0, r->st>>>(static_cast<uint32_t*>(r->cols[c].p), r->E, 2, cs + 1);
+            k_checksum<float><<<grid(r->E), 256, 0, r->st>>>(static_cast<float*>(r->w[c].p), r->E, 3, cs + 2);
+            k_checksum<uint64_t><<<grid(r->V), 256, 0, r->st>>>(static_cast<uint64_t*>(r->ext[r->ext_cur].p), r->V, 4, cs + 3);
+            CKL();
+            CK(cudaMemcpyAsync(checksums, cs, 32, cudaMemcpyDeviceToHost, r->st));
+        }
+        r->sync();
+        return H2TAP_OK;
+    });
+}
+
+h2tap_status h2tap_bfs(const h2tap_replica* rc, uint64_t source_ext, int32_t* level_out, int on_device) {
+    h2tap_replica* r = const_cast<h2tap_replica*>(rc);
+    if (!r || !level_out) { set_err("null argument"); return H2TAP_E_INVAL; }
+    return run_guarded(r, [&]() -> h2tap_status {
+        CK(cudaSetDevice(r->cfg.device));
+        const uint64_t V = r->V;
+        // source lookup on the host side of the ID map (one binary search through D2H probes is
+        // avoided: copy-free search via a tiny kernel would be equivalent; V is small relative)
+        uint64_t src = V;
+        if (r->identity) src = source_ext < V ? source_ext : V;
+        else {
+            const uint64_t* ext = static_cast<const uint64_t*>(r->ext[r->ext_cur].p);
+            uint64_t lo = 0, hi = V;
+            while (lo < hi) {
+                uint64_t mid = (lo + hi) / 2, x;
+                CK(cudaMemcpy(&x, ext + mid, 8, cudaMemcpyDeviceToHost));
+                if (x < source_ext) lo = mid + 1; else hi = mid;
+            }
+            uint64_t x = ~0ull;
+            if (lo < V) CK(cudaMemcpy(&x, ext + lo, 8, cudaMemcpyDeviceToHost));
+            if (lo < V && x == source_ext) src = lo;
+        }
+        if (src >= V) { set_err("BFS source %llu is not a live vertex", (unsigned long long)source_ext); return H2TAP_E_INVAL; }
+        int32_t* level = on_device ? level_out : r->get<int32_t>(r->pr_a, V);
+        uint32_t* fa = r->get<uint32_t>(r->bfs_a, V);
+        uint32_t* fb = r->get<uint32_t>(r->bfs_b, V);
+        unsigned long long* cnt = r->get<unsigned long long>(r->misc, 1);
+        k_fill_i32<<<g1(V), 256, 0, r->st>>>(level, V, -1);
+        CKL();
+        int32_t zero = 0;
+        uint32_t s32 = (uint32_t)src;
+        CK(cudaMemcpyAsync(level + src, &zero, 4, cudaMemcpyHostToDevice, r->st));
+        CK(cudaMemcpyAsync(fa, &s32, 4, cudaMemcpyHostToDevice, r->st));
+        uint64_t nf = 1;
+        const int64_t* off = static_cast<const int64_t*>(r->off[r->cur].p);
+        const uint32_t* cols = static_cast<const uint32_t*>(r->cols[r->cur].p);
+        for (int32_t depth = 0; nf; ++depth) {
+            CK(cudaMemsetAsync(cnt, 0, 8, r->st));
+            unsigned grid = (unsigned)std::min<uint64_t>(cdiv(nf * 32, 256), 148 * 32);
+            k_bfs_expand<<<grid, 256, 0, r->st>>>(off, cols, fa, nf, level, depth, fb, cnt);
+            CKL();
+            unsigned long long h = 0;
+            CK(cudaMemcpyAsync(&h, cnt, 8, cudaMemcpyDeviceToHost, r->st));
+            r->sync();
+            nf = h;
+            std::swap(fa, fb);
+        }
+        if (!on_device) CK(cudaMemcpyAsync(level_out, level, V * 4, cudaMemcpyDeviceToHost, r->st));
+        r->sync();
+        return H2TAP_OK;
+    });
+}
+
+h2tap_status h2tap_pagerank(const h2tap_replica* rc, double damping, int iterations, double* rank_out, int on_device) {
+    h2tap_replica* r = const_cast<h2tap_replica*>(rc);
+    if (!r || !rank_out || iterations < 0) { set_err("bad argument"); return H2TAP_E_INVAL; }
+    return run_guarded(r, [&]() -> h2tap_status {
+        CK(cudaSetDevice(r->cfg.device));
+        const uint64_t V = r->V;
+        if (V == 0) return H2TAP_OK;
+        double* a = r->get<double>(r->pr_a, V);
+        double* b = r->get<double>(r->pr_b, V);
+        double* ds = r->get<double>(r->misc, 1);
+        const int64_t* off = static_cast<const int64_t*>(r->off[r->cur].p);
+        const uint32_t* cols = static_cast<const uint32_t*>(r->cols[r->cur].p);
+        k_pr_init<<<g1(V), 256, 0, r->st>>>(a, V);
+        CKL();
+        unsigned gs = (unsigned)std::min<uint64_t>(g1(V), 148 * 8);
+        unsigned gw = (unsigned)std::min<uint64_t>(cdiv(V * 32, 256), 148 * 32);
+        for (int it = 0; it < iterations; ++it) {
+            CK(cudaMemsetAsync(ds, 0, 8, r->st));
+            CK(cudaMemsetAsync(b, 0, V * 8, r->st));
+            k_pr_dangling<<<gs, 256, 0, r->st>>>(off, a, V, ds);
+            k_pr_push<<<gw, 256, 0, r->st>>>(off, cols, a, V, b);
+            k_pr_finish<<<g1(V), 256, 0, r->st>>>(b, V, damping, ds);
+            CKL();
+            std::swap(a, b);
+        }
+        CK(cudaMemcpyAsync(rank_out, a, V * 8, on_device ? cudaMemcpyDeviceToDevice : cudaMemcpyDeviceToHost, r->st));
+        r->sync();
+        return H2TAP_OK;
+    });
+}
+
+void h2tap_replica_destroy(h2tap_replica* r) {
+    try {
+        free_replica(r);
+    } catch (...) {
+    }
+}
+
+}  // extern "C"

@@ -1,0 +1,153 @@
+// radix_sort.cuh - stable LSD radix sort of (uint64 key, uint32 value) pairs for
+// sm_100a, onesweep style (one kernel per 8-bit digit pass):
+//   1. one histogram kernel counts the digits of every pass in a single read;
+//   2. a tiny kernel turns them into per-pass digit bases;
+//   3. per pass, each 3072-key tile ranks its keys stably with warp match_any,
+//      publishes per-digit counts and resolves its global digit offsets with a
+//      per-digit decoupled look-back (256 threads, one digit each), stages the
+//      keys digit-sorted in shared memory and writes them out in contiguous runs.
+// Only the significant key bits are sorted (2*ceil(log2 V') for packed
+// (src', dst') edge keys).
+#pragma once
+#include "dev_common.cuh"
+
+namespace h2tap {
+
+constexpr int kRsThreads = 256;
+constexpr int kRsItems = 12;
+constexpr int kRsTile = kRsThreads * kRsItems;  // 3072 keys per tile
+constexpr int kRsWarps = kRsThreads / 32;
+constexpr int kRsMaxPasses = 8;
+
+__global__ void __launch_bounds__(256) rs_histogram(const uint64_t* __restrict__ keys, uint64_t n,
+                                                    int passes, uint32_t* __restrict__ hist) {
+    __shared__ uint32_t s[kRsMaxPasses][256];
+    for (int i = threadIdx.x; i < kRsMaxPasses * 256; i += blockDim.x) (&s[0][0])[i] = 0;
+    __syncthreads();
+    for (uint64_t i = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; i < n;
+         i += (uint64_t)gridDim.x * blockDim.x) {
+        uint64_t k = keys[i];
+        for (int p = 0; p < passes; ++p) atomicAdd(&s[p][(k >> (8 * p)) & 255], 1u);
+    }
+    __syncthreads();
+    for (int i = threadIdx.x; i < passes * 256; i += blockDim.x) {
+        uint32_t v = (&s[0][0])[i];
+        if (v) atomicAdd(&hist[i], v);
+    }
+}
+
+// one block per pass: exclusive scan of the 256 digit counts
+__global__ void __launch_bounds__(256) rs_digit_base(const uint32_t* __restrict__ hist,
+                                                     uint64_t* __restrict__ base) {
+    __shared__ uint64_t sm[9];
+    const int p = blockIdx.x;
+    uint64_t v = hist[p * 256 + threadIdx.x], tot;
+    uint64_t e = block_exclusive_scan<256>(v, sm, &tot);
+    base[p * 256 + threadIdx.x] = e;
+}
+
+__global__ void __launch_bounds__(kRsThreads) rs_onesweep(
+    const uint64_t* __restrict__ kin, const uint32_t* __restrict__ vin, uint64_t* __restrict__ kout,
+    uint32_t* __restrict__ vout, uint64_t n, int shift, const uint64_t* __restrict__ digit_base,
+    uint64_t* __restrict__ status /* [ntiles][256] */, uint32_t* __restrict__ tile_ctr) {
+    __shared__ uint32_t s_tile;
+    __shared__ uint32_t s_wcnt[kRsWarps][256];
+    __shared__ uint32_t s_dstart[256];
+    __shared__ uint64_t s_gpre[256];
+    __shared__ uint64_t s_keys[kRsTile];
+    __shared__ uint32_t s_vals[kRsTile];
+    __shared__ uint32_t s_scan[kRsThreads / 32 + 1];
+
+    const int tid = threadIdx.x, w = tid >> 5, l = lane_id();
+    if (tid == 0) s_tile = atomicAdd(tile_ctr, 1u);
+    for (int i = tid; i < kRsWarps * 256; i += kRsThreads) (&s_wcnt[0][0])[i] = 0;
+    __syncthreads();
+    const uint32_t tile = s_tile;
+    const uint64_t base = (uint64_t)tile * kRsTile;
+    const uint64_t tile_n = (n - base < (uint64_t)kRsTile) ? (n - base) : (uint64_t)kRsTile;
+
+    uint64_t k[kRsItems];
+    uint32_t v[kRsItems];
+    uint32_t rank[kRsItems];
+#pragma unroll
+    for (int i = 0; i < kRsItems; ++i) {
+        uint64_t idx = base + (uint64_t)w * 32 * kRsItems + i * 32 + l;
+        bool ok = idx < n;
+        k[i] = ok ? kin[idx] : 0;
+        v[i] = ok ? vin[idx] : 0;
+    }
+    // stable in-warp ranking, iteration-major then lane order == tile index order
+#pragma unroll
+    for (int i = 0; i < kRsItems; ++i) {
+        uint64_t idx = base + (uint64_t)w * 32 * kRsItems + i * 32 + l;
+        bool ok = idx < n;
+        uint32_t valid = __ballot_sync(0xffffffffu, ok);
+        rank[i] = 0;
+        if (ok) {
+            uint32_t d = (uint32_t)(k[i] >> shift) & 255u;
+            uint32_t peers = __match_any_sync(valid, d);
+            uint32_t before = s_wcnt[w][d];
+            __syncwarp(valid);
+            if (l == (uint32_t)(__ffs(peers) - 1)) s_wcnt[w][d] = before + __popc(peers);
+            __syncwarp(valid);
+            rank[i] = before + __popc(peers & lanemask_lt());
+        }
+    }
+    __syncthreads();
+    // per digit: exclusive over warps, tile count
+    uint32_t c = 0;
+    {
+        const int d = tid;  // 256 threads == 256 digits
+        for (int ww = 0; ww < kRsWarps; ++ww) {
+            uint32_t t = s_wcnt[ww][d];
+            s_wcnt[ww][d] = c;
+            c += t;
+        }
+    }
+    uint32_t tot;
+    uint32_t ds = block_exclusive_scan<kRsThreads>(c, s_scan, &tot);
+    s_dstart[tid] = ds;
+    // per-digit decoupled look-back (thread d walks back over tiles for digit d)
+    {
+        const int d = tid;
+        uint64_t* st = status + (uint64_t)tile * 256 + d;
+        uint64_t excl = 0;
+        if (tile == 0) {
+            st_volatile(st, kFlagPrefix | c);
+        } else {
+            st_volatile(st, kFlagAgg | c);
+            int64_t t = (int64_t)tile - 1;
+            while (t >= 0) {
+                uint64_t s = ld_volatile(status + (uint64_t)t * 256 + d);
+                uint64_t f = s >> 62;
+                if (f == 0) continue;
+                excl += s & kValMask;
+                if (f == 2) break;
+                --t;
+            }
+            st_volatile(st, kFlagPrefix | (excl + c));
+        }
+        s_gpre[d] = digit_base[d] + excl;
+    }
+    __syncthreads();
+#pragma unroll
+    for (int i = 0; i < kRsItems; ++i) {
+        uint64_t idx = base + (uint64_t)w * 32 * kRsItems + i * 32 + l;
+        if (idx < n) {
+            uint32_t d = (uint32_t)(k[i] >> shift) & 255u;
+            uint32_t pos = s_dstart[d] + s_wcnt[w][d] + rank[i];
+            s_keys[pos] = k[i];
+            s_vals[pos] = v[i];
+        }
+    }
+    __syncthreads();
+    for (uint32_t p = tid; p < tile_n; p += kRsThreads) {
+        uint64_t key = s_keys[p];
+        uint32_t d = (uint32_t)(key >> shift) & 255u;
+        uint64_t o = s_gpre[d] + (p - s_dstart[d]);
+        kout[o] = key;
+        vout[o] = s_vals[p];
+    }
+}
+
+}  // namespace h2tap

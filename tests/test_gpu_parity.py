@@ -1,0 +1,237 @@
+"""Parity of the CUDA path (libh2tap.so through its C ABI) with the oracle O1.
+
+Bar: offsets, cols, weights and the ID map bit-exact after every
+batch; BFS levels bit-exact; PageRank within 1e-6 max relative error.
+"""
+import json
+import os
+
+import numpy as np
+import pytest
+
+import oracle
+import synth
+from oracle import O1
+from synth import Batch, NODE_INSERT, NODE_DELETE, EDGE_INSERT, EDGE_DELETE, EDGE_WEIGHT
+
+pytestmark = pytest.mark.gpu
+HERE = os.path.dirname(os.path.abspath(__file__))
+
+
+@pytest.fixture(scope="module")
+def h2():
+    import paper_conf_edbt_jibrilabs23_b200 as h2
+    return h2
+
+
+def assert_same(gpu, ora, ctx=""):
+    names = ("offsets", "cols", "weights", "ext_ids")
+    for n, a, b in zip(names, gpu, ora):
+        a, b = np.asarray(a), np.asarray(b)
+        assert a.shape == b.shape, f"{ctx} {n}: shape {a.shape} vs {b.shape}"
+        if n == "weights":
+            a, b = a.view(np.uint32), b.view(np.uint32)
+        if not np.array_equal(a, b):
+            bad = np.nonzero(a != b)[0]
+            raise AssertionError(f"{ctx} {n}: {len(bad)} mismatches, first at {bad[:5]}: "
+                                 f"{a[bad[:5]]} vs {b[bad[:5]]}")
+
+
+def pair_from_edges(h2, n, ids, src, dst, w, create_ts=0):
+    g = h2.Replica.from_edges(n, ids, src, dst, w, create_ts)
+    o = O1.from_edges(n, ids, src, dst, w, create_ts)
+    step.last_E[id(g)] = g.info()["n_edges"]
+    return g, o
+
+
+def step(g, o, batch, snap, ctx=""):
+    st = g.apply(batch, snap)
+    rc, ost = o.apply(batch, snap)
+    assert rc == 0
+    assert st["n_visible"] == ost["n_visible"] and st["n_deferred"] == ost["n_deferred"], ctx
+    E_old = step.last_E.get(id(g))
+    ex = g.export()
+    assert_same(ex, o.export(), ctx)
+    if E_old is not None:  # I6: E' = E + NEW - DEL - CASC
+        assert len(ex[1]) == E_old + st["n_new"] - st["n_del"] - st["n_casc"], ctx
+    step.last_E[id(g)] = len(ex[1])
+    return st
+
+
+step.last_E = {}
+
+
+# ------------------------------------------------------------------ cases ----
+def test_fig2_worked_example(h2):
+    gj = json.load(open(os.path.join(HERE, "golden", "fig2.json")))
+    e = np.array(gj["edges"], dtype=object)
+    ids = np.array(gj["vertices"], np.uint64)
+    g = h2.Replica.from_edges(len(ids), ids, np.array(e[:, 0], np.uint64), np.array(e[:, 1], np.uint64),
+                              np.array(e[:, 2], np.float32), gj["create_ts"])
+    st = g.apply(Batch.of(gj["ops"]), gj["snapshot_ts"])
+    off, cols, w, ext = g.export()
+    ex = gj["expected"]
+    assert ext.tolist() == ex["ext_ids"] and off.tolist() == ex["offsets"]
+    assert cols.tolist() == ex["cols"] and w.tolist() == ex["weights"]
+    assert st["n_vertex_inserted"] == 1 and st["n_vertex_deleted"] == 1
+
+
+def test_tiny_fuzz_multibatch(h2):
+    """Adversarial tiny streams: equal ts, out-of-order arrival, deferral, all op kinds."""
+    for case in range(150):
+        nid = 3 + case % 6
+        rng = np.random.default_rng(1000 + case)
+        live = np.array(sorted(rng.choice(nid, size=max(1, nid // 2), replace=False)), np.uint64)
+        pairs = [(u, v) for u in live for v in live if rng.random() < 0.5]
+        src = np.array([p[0] for p in pairs], np.uint64)
+        dst = np.array([p[1] for p in pairs], np.uint64)
+        w = (rng.integers(0, 16, len(pairs)) / 4).astype(np.float32)
+        g, o = pair_from_edges(h2, len(live), live, src, dst, w)
+        snap = 0
+        for k in range(4):
+            b = synth.fuzz_batch(seed=case, k=k, n=1 + (case * 7 + k) % 23, n_ids=nid, ts_lo=snap + 1,
+                                 ts_span=8)
+            snap += 4
+            step(g, o, b, snap, f"case {case} batch {k}")
+
+
+def test_rmat_c1_config(h2):
+    """BASELINE configs[0]: RMAT scale 16, 1M generated edges, one 10K 80/20 batch."""
+    cfg = synth.CONFIGS["c1"]
+    seed = synth.seed_of("c1")
+    n = 1 << cfg["scale"]
+    src, dst, w = synth.rmat_edges(cfg["scale"], seed)
+    g, o = pair_from_edges(h2, n, None, src, dst, w)
+    assert_same(g.export(), o.export(), "create")
+    b = synth.rmat_batch(cfg["scale"], seed, 0, cfg["batch"], len(src), p_insert=0.8, ts_base=0)
+    st = step(g, o, b, int(b.ts.max()), "c1 batch")
+    assert st["n_new"] > 0 and st["n_del"] > 0
+    # freshness checks on the new snapshot
+    off, cols, _, _ = g.export()
+    for s in (0, 17, 4242):
+        assert np.array_equal(g.bfs(s), oracle.bfs(off, cols, s))
+    pr_g, pr_o = g.pagerank(0.85, 20), oracle.pagerank(off, cols, 0.85, 20)
+    assert np.max(np.abs(pr_g - pr_o) / pr_o) < 1e-6
+
+
+def test_rmat_parity_variant_weights_repeats_txns(h2):
+    """C1 parity variant: 10% EDGE_WEIGHT, repeated keys, 4-op transactions (equal ts)."""
+    seed = synth.seed_of("c1") + 77
+    scale = 14
+    src, dst, w = synth.rmat_edges(scale, seed)
+    g, o = pair_from_edges(h2, 1 << scale, None, src, dst, w)
+    ts = 0
+    for k in range(3):
+        b = synth.rmat_batch(scale, seed, k, 20000, len(src), p_insert=0.6, p_weight=0.1, p_repeat=0.3,
+                             ops_per_txn=4, ts_base=ts)
+        snap = int(np.quantile(b.ts, 0.9))          # defer ~10%
+        step(g, o, b, snap, f"variant batch {k}")
+        ts = int(b.ts.max())
+    step(g, o, Batch.empty(0), ts, "flush pending")
+    assert g.info()["n_pending"] == 0
+
+
+def test_mixed_node_ops_multi_tile(h2):
+    """Node inserts/deletes (incl. re-insert, ids outside the graph), many merge tiles."""
+    scale = 13
+    n = 1 << scale
+    src, dst, w = synth.rmat_edges(scale, 5, n=12 * n)
+    ids = (np.arange(n, dtype=np.uint64) * 3 + 7)       # sparse external ids
+    g, o = pair_from_edges(h2, n, ids, ids[src], ids[dst], w)
+    ts = 0
+    for k in range(4):
+        b = synth.fuzz_batch(seed=99, k=k, n=30000, n_ids=3 * n + 20, probs=(0.03, 0.01, 0.6, 0.25, 0.11),
+                             ts_lo=ts + 1, ts_span=5000)
+        # map half the random ids onto existing vertices so edge ops hit the graph
+        hit = np.arange(len(b)) % 2 == 0
+        b.src[hit] = ids[b.src[hit] % n]
+        b.dst[hit] = ids[b.dst[hit] % n]
+        snap = ts + 4000
+        step(g, o, b, snap, f"mixed batch {k}")
+        ts = snap + 1000
+
+
+def test_ldbc_shaped_small(h2):
+    shape = synth.LdbcShape(n_person=512, n_msg=20000, e_person=40000)
+    seed = synth.seed_of("c2")
+    ids = synth.ldbc_vertices(shape)
+    src, dst, w = synth.ldbc_edges(shape, seed)
+    g, o = pair_from_edges(h2, shape.n_vertices, ids, src, dst, w)
+    ts = 0
+    for k in range(3):
+        b = synth.ldbc_batch(shape, seed, k, 5000, lodeg=(k == 1), ts_base=ts)
+        ts = int(b.ts.max())
+        st = step(g, o, b, ts, f"ldbc batch {k}")
+        assert st["n_vertex_inserted"] > 0
+
+
+def test_empty_batch_is_identity_and_errors_leave_state(h2):
+    scale = 10
+    src, dst, w = synth.rmat_edges(scale, 3)
+    g, o = pair_from_edges(h2, 1 << scale, None, src, dst, w)
+    before = g.export(checksums=True)
+    g.apply(Batch.empty(0), 5)
+    after = g.export(checksums=True)
+    assert_same(after[:4], before[:4]) and after[4] == before[4]
+    assert g.info()["snapshot_ts"] == 5
+    rc, _ = g.apply(Batch.of([(EDGE_INSERT, 0, 1, 1.0, 9)]), 4, raise_on_error=False)
+    assert rc == -6                                              # snapshot regression
+    rc, _ = g.apply(Batch.of([(EDGE_INSERT, 0, 1, 1.0, 5)]), 9, raise_on_error=False)
+    assert rc == -5                                              # stale ts
+    rc, _ = g.apply(Batch.of([(9, 0, 1, 1.0, 7)]), 9, raise_on_error=False)
+    assert rc == -1                                              # unknown kind
+    assert_same(g.export(), before[:4])
+    assert g.info()["snapshot_ts"] == 5
+
+
+def test_delete_all_edges(h2):
+    src, dst, w = synth.rmat_edges(9, 4)
+    g, o = pair_from_edges(h2, 512, None, src, dst, w)
+    off, cols, _, ids = g.export()
+    u = np.repeat(ids, np.diff(off))
+    b = Batch(np.full(len(u), EDGE_DELETE, np.uint8), u, ids[cols], np.zeros(len(u), np.float32),
+              np.full(len(u), 3, np.uint64))
+    st = step(g, o, b, 3, "delete all")
+    assert g.info()["n_edges"] == 0 and st["n_del"] == len(u)
+
+
+def test_create_from_csr_roundtrip_and_validation(h2):
+    src, dst, w = synth.rmat_edges(11, 8)
+    ids = np.arange(1 << 11, dtype=np.uint64) * 5 + 1
+    g = h2.Replica.from_edges(1 << 11, ids, ids[src], ids[dst], w, 3)
+    off, cols, ww, ext = g.export()
+    g2 = h2.Replica.from_csr(off, cols, ww, ext, 3)
+    assert_same(g2.export(), (off, cols, ww, ext))
+    bad = cols.copy()
+    bad[0] = 1 << 11                                          # column out of range
+    with pytest.raises(h2.H2tapError):
+        h2.Replica.from_csr(off, bad, ww, ext)
+    r = int(np.argmax(np.diff(off) >= 2))                     # a row with >= 2 entries
+    dup = cols.copy()
+    dup[off[r] + 1] = dup[off[r]]                             # duplicate column in a row
+    with pytest.raises(h2.H2tapError):
+        h2.Replica.from_csr(off, dup, ww, ext)
+    with pytest.raises(h2.H2tapError):                        # edge endpoint outside the vertex set
+        h2.Replica.from_edges(4, None, np.array([0], np.uint64), np.array([9], np.uint64),
+                              np.array([1.0], np.float32))
+
+
+def test_checksums_match_oracle_definition(h2):
+    src, dst, w = synth.rmat_edges(12, 6)
+    g, o = pair_from_edges(h2, 1 << 12, None, src, dst, w)
+    b = synth.rmat_batch(12, 6, 0, 5000, len(src))
+    step(g, o, b, int(b.ts.max()))
+    assert g.checksums() == oracle.checksums(*o.export())
+
+
+def test_device_resident_batch(h2):
+    import torch
+    src, dst, w = synth.rmat_edges(12, 12)
+    g, o = pair_from_edges(h2, 1 << 12, None, src, dst, w)
+    b = synth.rmat_batch(12, 12, 0, 8000, len(src), p_weight=0.1)
+    dev = Batch(*(torch.from_numpy(a.view(np.int64) if a.dtype == np.uint64 else a).cuda()
+                  for a in (b.kind, b.src, b.dst, b.w, b.ts)))
+    st = g.apply(dev, int(b.ts.max()))
+    o.apply(b, int(b.ts.max()))
+    assert_same(g.export(), o.export(), "device batch")
+    assert st["n_visible"] == len(b)

@@ -127,6 +127,40 @@ __device__ __forceinline__ uint64_t upper_bound_dev(const T* a, uint64_t lo, uin
     return lo;
 }
 
+// Stable compaction of a tile of kThreads x ITEMS items in STRIPED order (item k of
+// thread t is tile item k*NT + t, so global loads coalesce): flag[k] -> pos[k] =
+// rank of the item among flagged items of the tile.  smem: ITEMS*NT/32 + 1 words.
+// Returns the tile total.  Requires ITEMS * NT/32 <= 64.
+template <int NT, int ITEMS>
+__device__ __forceinline__ uint32_t striped_compact(const bool (&flag)[ITEMS], uint32_t (&pos)[ITEMS], uint32_t* s) {
+    constexpr int NW = NT / 32;
+    static_assert(ITEMS * NW <= 64, "striped_compact: too many (item, warp) cells");
+    const int w = threadIdx.x >> 5;
+    const uint32_t lane = lane_id(), lt = lanemask_lt();
+#pragma unroll
+    for (int k = 0; k < ITEMS; ++k) {
+        uint32_t m = __ballot_sync(0xffffffffu, flag[k]);
+        pos[k] = __popc(m & lt);
+        if (lane == 0) s[k * NW + w] = __popc(m);
+    }
+    __syncthreads();
+    if (w == 0) {
+        constexpr int C = ITEMS * NW;
+        uint32_t a = (2 * lane < C) ? s[2 * lane] : 0, b = (2 * lane + 1 < C) ? s[2 * lane + 1] : 0;
+        uint32_t inc = warp_inclusive_scan(a + b);
+        uint32_t ex = inc - a - b;
+        if (2 * lane < C) s[2 * lane] = ex;
+        if (2 * lane + 1 < C) s[2 * lane + 1] = ex + a;
+        if (lane == 31) s[C] = inc;
+    }
+    __syncthreads();
+#pragma unroll
+    for (int k = 0; k < ITEMS; ++k) pos[k] += s[k * NW + w];
+    uint32_t tot = s[ITEMS * NW];
+    __syncthreads();
+    return tot;
+}
+
 // (ts, seq) commit point, lexicographic (reading A5)
 struct Point {
     uint64_t ts, seq;

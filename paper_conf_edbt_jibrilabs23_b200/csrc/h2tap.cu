@@ -69,11 +69,13 @@ inline int bits_for(uint64_t range) { return range == 0 ? 0 : 64 - __builtin_clz
 
 struct h2tap_replica {
     h2tap_config cfg{};
-    cudaStream_t st = nullptr;
+    cudaStream_t st = nullptr, st2 = nullptr;  // st2: side stream (cascade pass)
+    cudaEvent_t evA = nullptr, evB = nullptr;
     uint64_t V = 0, E = 0, snap = 0, next_seq = 0, n_pend = 0;
     bool identity = true, poisoned = false;
+    int n_sm = 148;
     int cur = 0, ext_cur = 0, pcur = 0;
-    Buf off[2], cols[2], w[2], ext[2];
+    Buf off[2], cols[2], w[2], ext[2], fence[2];
     Buf pk[2], ps[2], pd[2], pw[2], pt[2], pq[2];
     // scratch
     Buf Wk, Ws, Wd, Ww, Wt, Wq, idx_p, idx_n, idx_e, status;
@@ -81,7 +83,7 @@ struct h2tap_replica {
     Buf nv, nv_ext, dropped, ins_q, ins_oldpos, hd_rows, remap, hd_bits;
     Buf op_flags, op_ou, op_ow;
     Buf ins_pos, ins_row, ins_col, ins_w, del_pos, upd_pos, upd_w, KR;
-    Buf misc, nsorted, bfs_a, bfs_b, pr_a, pr_b;
+    Buf misc, nsorted, part, opart, deg, tsum, remap_shift, tile_emit, tile_base, del_row, casc_mask, status2, bfs_a, bfs_b, pr_a, pr_b;
     Buf ctr;
     Counters* hc = nullptr;  // pinned host mirror
     cudaEvent_t ev[8]{};
@@ -122,6 +124,8 @@ struct h2tap_replica {
     }
     void release(Buf& b) { dfree(b.p); b.p = nullptr; b.cap = 0; }
     void sync() { CK(cudaStreamSynchronize(st)); }
+    bool identity_pending = false;  // identity flag of the ext buffer being built
+    bool identity_of(int which) const { return which == ext_cur ? identity : identity_pending; }
     void read_counters() {
         g_d2h += sizeof(Counters);
         CK(cudaMemcpyAsync(hc, ctr.p, sizeof(Counters), cudaMemcpyDeviceToHost, st));
@@ -194,6 +198,27 @@ float ev_ms(cudaEvent_t a, cudaEvent_t b) {
     float ms = 0;
     cudaEventElapsedTime(&ms, a, b);
     return ms;
+}
+
+uint64_t n_fence(uint64_t V) { return (V + (1u << kFenceShift) - 1) >> kFenceShift; }
+
+void build_fence(h2tap_replica* r, int which, uint64_t V) {
+    uint64_t nf = n_fence(V);
+    uint64_t* f = r->get<uint64_t>(r->fence[which], nf);
+    if (nf && !r->identity_of(which)) {
+        k_build_fence<<<g1(nf), 256, 0, r->st>>>(static_cast<const uint64_t*>(r->ext[which].p), V, f);
+        CKL();
+    }
+}
+
+ExtIndex ext_index(h2tap_replica* r) {
+    ExtIndex X;
+    X.ext = static_cast<const uint64_t*>(r->ext[r->ext_cur].p);
+    X.fence = static_cast<const uint64_t*>(r->fence[r->ext_cur].p);
+    X.V = r->V;
+    X.nf = n_fence(r->V);
+    X.identity = r->identity;
+    return X;
 }
 
 // One propagation cycle.  Nothing visible changes until the final swap.
@@ -278,6 +303,10 @@ h2tap_status apply_core(h2tap_replica* r, const BatchIn& in, uint64_t S, bool cr
     uint32_t *dropped = nullptr, *ins_q = nullptr, *ins_oldpos = nullptr, *hd_rows = nullptr, *remap = nullptr,
              *hd_bits = nullptr, *node_sorted = nullptr;
     uint64_t* new_ext = nullptr;
+    uint32_t* casc_mask = nullptr;
+    uint64_t *casc_cnt = nullptr, *casc_pre = nullptr;
+    const int64_t* old_off_nc = static_cast<const int64_t*>(r->off[r->cur].p);
+    const uint32_t* old_cols_nc = static_cast<const uint32_t*>(r->cols[r->cur].p);
     if (n_node) {
         uint64_t* kA = r->get<uint64_t>(r->keyA, n_node);
         uint64_t* kB = r->get<uint64_t>(r->keyB, n_node);
@@ -300,8 +329,8 @@ h2tap_status apply_core(h2tap_replica* r, const BatchIn& in, uint64_t S, bool cr
         uint64_t nt = cdiv(n_node, kTile);
         uint64_t* stt = r->get<uint64_t>(r->status, 3 * nt);
         CK(cudaMemsetAsync(stt, 0, nt * 8, st));
-        k_node_segments<<<(unsigned)nt, kThreads, 0, st>>>(ops, node_sorted, n_node, old_ext, V, r->identity, nv,
-                                                           nv_ext, stt, nt, dc);
+        k_node_segments<<<(unsigned)nt, kThreads, 0, st>>>(ops, node_sorted, n_node, ext_index(r), nv, nv_ext,
+                                                           stt, nt, dc);
         CKL();
         r->read_counters();
         U = r->hc->n_unique;
@@ -334,8 +363,8 @@ h2tap_status apply_core(h2tap_replica* r, const BatchIn& in, uint64_t S, bool cr
             if (remap_on) {
                 remap = r->get<uint32_t>(r->remap, V);
                 if (V) {
-                    k_remap<<<g1(V, kThreads * kItems), kThreads, 0, st>>>(old_ext, r->identity, V, dropped, n_dropped,
-                                                                           ins_oldpos, n_vins, remap, new_ext);
+                    k_remap<<<g1(V, kRemapTile), kThreads, 0, st>>>(old_ext, r->identity, V, dropped, n_dropped,
+                                                                    ins_oldpos, n_vins, remap, new_ext);
                     CKL();
                 }
             } else if (V) {
@@ -347,6 +376,11 @@ h2tap_status apply_core(h2tap_replica* r, const BatchIn& in, uint64_t S, bool cr
                 CKL();
             }
         }
+        if (set_changed) {
+            // identity test of the new set is done at the end; fence built regardless
+            r->identity_pending = false;
+            build_fence(r, ec ^ 1, Vn);
+        }
         k_nv_newid<<<g1(U), 256, 0, st>>>(nv, U, remap, remap_on ? 1 : 0);
         CKL();
         if (n_hd) {
@@ -354,6 +388,29 @@ h2tap_status apply_core(h2tap_replica* r, const BatchIn& in, uint64_t S, bool cr
             CK(cudaMemsetAsync(hd_bits, 0, cdiv(V, 32) * 4, st));
             k_set_bits<<<g1(n_hd), 256, 0, st>>>(hd_rows, n_hd, hd_bits);
             CKL();
+            // cascade pass on the side stream, overlapped with the edge-op phase
+            const uint64_t nblk = cdiv(E, kCascBlock);
+            casc_mask = r->get<uint32_t>(r->casc_mask, (nblk + 1) * (kCascBlock / 32));
+            casc_cnt = r->get<uint64_t>(r->tile_emit, nblk + 1);
+            casc_pre = r->get<uint64_t>(r->tile_base, nblk + 1);
+            CK(cudaEventRecord(r->evA, st));
+            CK(cudaStreamWaitEvent(r->st2, r->evA, 0));
+            cudaStream_t s2 = r->st2;
+            unsigned rg = (unsigned)std::min<uint64_t>(cdiv(n_hd * 32, 256), (uint64_t)r->n_sm * 8);
+            const uint64_t nst = cdiv(nblk + 1, kThreads);
+            uint64_t* st2s2 = r->get<uint64_t>(r->status2, nst);
+            CK(cudaMemsetAsync(st2s2, 0, nst * 8, s2));
+            if (nblk) {
+                k_casc_cols<<<(unsigned)nblk, kThreads, 0, s2>>>(old_cols_nc, E, hd_bits, casc_mask);
+                CKL();
+                k_casc_rows<<<rg, 256, 0, s2>>>(old_off_nc, hd_rows, n_hd, casc_mask);
+                CKL();
+            }
+            k_casc_scan<<<(unsigned)nst, kThreads, 0, s2>>>(casc_mask, nblk, casc_pre, st2s2, &dc->tiles[6]);
+            CKL();
+            k_copy_u64<<<1, 1, 0, s2>>>(&dc->n_casc, casc_pre + nblk);
+            CKL();
+            CK(cudaEventRecord(r->evB, s2));
         }
     }
     CK(cudaEventRecord(r->ev[2], st));
@@ -380,9 +437,7 @@ h2tap_status apply_core(h2tap_replica* r, const BatchIn& in, uint64_t S, bool cr
         pa.ops = ops;
         pa.edge_idx = idx_e;
         pa.n_edge = n_edge;
-        pa.old_ext = old_ext;
-        pa.V = V;
-        pa.identity = r->identity;
+        pa.X = ext_index(r);
         pa.remap = remap_on ? remap : nullptr;
         pa.nv = nv;
         pa.nv_ext = nv_ext;
@@ -415,6 +470,7 @@ h2tap_status apply_core(h2tap_replica* r, const BatchIn& in, uint64_t S, bool cr
         ins_col = r->get<uint32_t>(r->ins_col, n_valid);
         ins_w = r->get<float>(r->ins_w, n_valid);
         del_pos = r->get<uint64_t>(r->del_pos, n_valid);
+        r->get<uint32_t>(r->del_row, n_valid);
         upd_pos = r->get<uint64_t>(r->upd_pos, n_valid);
         upd_w = r->get<float>(r->upd_w, n_valid);
         if (n_valid) {
@@ -429,10 +485,12 @@ h2tap_status apply_core(h2tap_replica* r, const BatchIn& in, uint64_t S, bool cr
             ca.op_opos_w = pa.op_opos_w;
             ca.old_off = old_off;
             ca.old_cols = old_cols;
+            ca.V_old = V;
             ca.ins_pos = ins_pos; ca.ins_row = ins_row; ca.ins_col = ins_col; ca.ins_w = ins_w;
             ca.del_pos = del_pos;
+            ca.del_row = static_cast<uint32_t*>(r->del_row.p);
             ca.upd_pos = upd_pos; ca.upd_w = upd_w;
-            uint64_t nt2 = cdiv(n_valid, kTile);
+            uint64_t nt2 = cdiv(n_valid, kCTile);
             ca.status3 = r->get<uint64_t>(r->status, 3 * nt2);
             CK(cudaMemsetAsync(ca.status3, 0, 3 * nt2 * 8, st));
             ca.n_tiles = nt2;
@@ -469,17 +527,36 @@ h2tap_status apply_core(h2tap_replica* r, const BatchIn& in, uint64_t S, bool cr
         ma.new_cols = new_cols; ma.new_w = new_w; ma.KR = KR;
         ma.n_tiles = cdiv(Dtot, kMergeTile);
         ma.c = dc;
-        if (casc) {
-            ma.status = r->get<uint64_t>(r->status, ma.n_tiles);
-            CK(cudaMemsetAsync(ma.status, 0, ma.n_tiles * 8, st));
+        if (remap_on) {
+            const uint64_t nblk = cdiv(V, 1u << kRemapBlockShift);
+            int32_t* rs = r->get<int32_t>(r->remap_shift, nblk);
+            if (nblk) {
+                k_remap_blocks<<<g1(nblk), 256, 0, st>>>(V, dropped, n_dropped, ins_oldpos, n_vins, rs);
+                CKL();
+            }
+            ma.remap_shift = rs;
         }
-        const unsigned grid = (unsigned)ma.n_tiles;
-        if (casc && remap_on) k_merge<true, true><<<grid, kThreads, 0, st>>>(ma);
-        else if (casc) k_merge<true, false><<<grid, kThreads, 0, st>>>(ma);
-        else if (remap_on) k_merge<false, true><<<grid, kThreads, 0, st>>>(ma);
-        else k_merge<false, false><<<grid, kThreads, 0, st>>>(ma);
+        TilePart* part = r->get<TilePart>(r->part, ma.n_tiles + 1);
+        k_merge_partition<<<g1(ma.n_tiles + 1), 256, 0, st>>>(ma, part);
+        CKL();
+        if (casc) {
+            ma.casc_mask = casc_mask;
+            ma.casc_pre = casc_pre;
+            CK(cudaStreamWaitEvent(st, r->evB, 0));
+        }
+        auto launch = [&](auto kern) {
+            int occ = 0;
+            CK(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, kern, kThreads, 0));
+            const uint64_t grid = std::min<uint64_t>(ma.n_tiles, (uint64_t)std::max(1, occ) * r->n_sm);
+            kern<<<(unsigned)grid, kThreads, 0, st>>>(ma, part);
+        };
+        if (casc && remap_on) launch(k_merge<true, true>);
+        else if (casc) launch(k_merge<true, false>);
+        else if (remap_on) launch(k_merge<false, true>);
+        else launch(k_merge<false, false>);
         CKL();
     } else if (casc) {
+        CK(cudaStreamWaitEvent(st, r->evB, 0));
         CK(cudaMemsetAsync(KR, 0, (V + 1) * 8, st));
     }
     CK(cudaEventRecord(r->ev[4], st));
@@ -490,13 +567,39 @@ h2tap_status apply_core(h2tap_replica* r, const BatchIn& in, uint64_t S, bool cr
     En = E + n_ins - n_del - n_casc;
 
     // ---- a4/a5: row offsets
-    if (V) {
-        unsigned grid = g1(V, kThreads * kItems);
-        const uint32_t* rm = remap_on ? remap : nullptr;
-        if (casc && remap_on) k_offsets_old<true, true><<<grid, kThreads, 0, st>>>(old_off, V, KR, del_pos, n_del, ins_row, n_ins, rm, new_off);
-        else if (casc) k_offsets_old<true, false><<<grid, kThreads, 0, st>>>(old_off, V, KR, del_pos, n_del, ins_row, n_ins, rm, new_off);
-        else if (remap_on) k_offsets_old<false, true><<<grid, kThreads, 0, st>>>(old_off, V, KR, del_pos, n_del, ins_row, n_ins, rm, new_off);
-        else k_offsets_old<false, false><<<grid, kThreads, 0, st>>>(old_off, V, KR, del_pos, n_del, ins_row, n_ins, rm, new_off);
+    if (V && !n_node) {
+        // per-vertex degree delta + single-pass decoupled look-back exclusive scan
+        int32_t* deg = r->get<int32_t>(r->deg, V);
+        int64_t* tsum = r->get<int64_t>(r->tsum, cdiv(V, kTile) + 1);
+        CK(cudaMemsetAsync(deg, 0, V * 4, st));
+        CK(cudaMemsetAsync(tsum, 0, (cdiv(V, kTile) + 1) * 8, st));
+        if (n_ins + n_del) {
+            k_deg_scatter<<<g1(n_ins + n_del), 256, 0, st>>>(ins_row, n_ins, static_cast<uint32_t*>(r->del_row.p), n_del, deg, tsum);
+            CKL();
+        }
+        // chain-free: tile sums were accumulated by the scatter; scan them in one CTA,
+        // then a streaming pass writes new_off = old_off + tile base + in-tile prefix
+        const uint64_t nt = cdiv(V, kTile);
+        k_tile_sum_scan<<<1, 1024, 0, st>>>(tsum, nt);
+        CKL();
+        k_offsets_apply<<<(unsigned)nt, kThreads, 0, st>>>(old_off, deg, V, tsum, new_off);
+        CKL();
+    } else if (V) {
+        OffArgs oa{};
+        oa.old_off = old_off; oa.V_old = V; oa.KR = KR;
+        oa.del_pos = del_pos; oa.n_del = n_del; oa.ins_row = ins_row; oa.n_ins = n_ins;
+        oa.remap = remap; oa.dropped = dropped; oa.n_dropped = n_dropped;
+        oa.ins_oldpos = ins_oldpos; oa.n_vins = n_vins; oa.new_off = new_off;
+        const uint64_t ncta = cdiv(V, kOffTile);
+        oa.part = r->get<uint64_t>(r->opart, 2 * (ncta + 1));
+        if (remap_on) k_offsets_partition<true><<<g1(ncta + 1), 256, 0, st>>>(oa);
+        else k_offsets_partition<false><<<g1(ncta + 1), 256, 0, st>>>(oa);
+        CKL();
+        const unsigned grid = (unsigned)ncta;
+        if (casc && remap_on) k_offsets_old<true, true><<<grid, kThreads, 0, st>>>(oa);
+        else if (casc) k_offsets_old<true, false><<<grid, kThreads, 0, st>>>(oa);
+        else if (remap_on) k_offsets_old<false, true><<<grid, kThreads, 0, st>>>(oa);
+        else k_offsets_old<false, false><<<grid, kThreads, 0, st>>>(oa);
         CKL();
     }
     if (n_vins) {
@@ -607,7 +710,11 @@ h2tap_replica* new_replica(const h2tap_config* cfg) {
     else { r->cfg.world = 1; }
     if (r->cfg.world <= 0) r->cfg.world = 1;
     CK(cudaSetDevice(r->cfg.device));
+    CK(cudaDeviceGetAttribute(&r->n_sm, cudaDevAttrMultiProcessorCount, r->cfg.device));
     r->st = static_cast<cudaStream_t>(r->cfg.stream);
+    CK(cudaStreamCreateWithFlags(&r->st2, cudaStreamNonBlocking));
+    CK(cudaEventCreateWithFlags(&r->evA, cudaEventDisableTiming));
+    CK(cudaEventCreateWithFlags(&r->evB, cudaEventDisableTiming));
     CK(cudaMallocHost(&r->hc, sizeof(Counters)));
     r->get<Counters>(r->ctr, 1);
     return r;
@@ -622,10 +729,13 @@ void free_replica(h2tap_replica* r) {
                    &r->hist, &r->dbase, &r->rs_status, &r->rs_ctr, &r->nv, &r->nv_ext, &r->dropped, &r->ins_q,
                    &r->ins_oldpos, &r->hd_rows, &r->remap, &r->hd_bits, &r->op_flags, &r->op_ou, &r->op_ow,
                    &r->ins_pos, &r->ins_row, &r->ins_col, &r->ins_w, &r->del_pos, &r->upd_pos, &r->upd_w,
-                   &r->KR, &r->misc, &r->nsorted, &r->bfs_a, &r->bfs_b, &r->pr_a, &r->pr_b, &r->ctr};
+                   &r->KR, &r->misc, &r->nsorted, &r->part, &r->opart, &r->deg, &r->tsum, &r->remap_shift, &r->tile_emit, &r->tile_base, &r->del_row, &r->casc_mask, &r->status2, &r->fence[0], &r->fence[1], &r->bfs_a, &r->bfs_b, &r->pr_a, &r->pr_b, &r->ctr};
     for (Buf* b : bufs) if (b->p) r->dfree(b->p);
     cudaStreamSynchronize(r->st);
     for (auto& e : r->ev) if (e) cudaEventDestroy(e);
+    if (r->evA) cudaEventDestroy(r->evA);
+    if (r->evB) cudaEventDestroy(r->evB);
+    if (r->st2) { cudaStreamSynchronize(r->st2); cudaStreamDestroy(r->st2); }
     if (r->hc) cudaFreeHost(r->hc);
     delete r;
 }
@@ -655,6 +765,7 @@ void init_vertices(h2tap_replica* r, uint64_t nv, const uint64_t* ids, int on_de
         if (h[0]) { set_err("vertex ids not strictly increasing"); throw Fail{H2TAP_E_INVAL}; }
         r->identity = (h[1] == nv - 1);
     }
+    build_fence(r, 0, nv);
 }
 
 }  // namespace

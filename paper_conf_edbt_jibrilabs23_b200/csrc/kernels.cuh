@@ -141,47 +141,61 @@ __global__ void k_keys_from(const uint32_t* __restrict__ idx, uint64_t n, const 
     vals[i] = o;
 }
 
-// old dense index of external id x (identity fast path or binary search)
-__device__ __forceinline__ uint64_t old_lookup(const uint64_t* ext, uint64_t V, bool identity, uint64_t x,
-                                               bool* present) {
-    if (identity) { *present = x < V; return x < V ? x : V; }
-    uint64_t k = lower_bound_dev(ext, 0, V, x);
-    *present = (k < V && ext[k] == x);
+// Old dense index of external id x.  Identity fast path, else a two-level search:
+// fence[i] = ext[i << 8] (V/32 bytes, L2-resident) picks a 256-id block, then a
+// binary search inside the block (2 KB) -- one DRAM-latency chain of ~8 probes
+// instead of ~25 over the whole 8V-byte array.
+constexpr int kFenceShift = 8;
+struct ExtIndex {
+    const uint64_t* ext;
+    const uint64_t* fence;
+    uint64_t V, nf;
+    int identity;
+};
+__device__ __forceinline__ uint64_t old_lookup(const ExtIndex& X, uint64_t x, bool* present) {
+    if (X.identity) { *present = x < X.V; return x < X.V ? x : X.V; }
+    uint64_t i = upper_bound_dev(X.fence, 0, X.nf, x);
+    if (i == 0) { *present = false; return 0; }
+    uint64_t lo = (i - 1) << kFenceShift, hi = min(lo + (uint64_t)(1u << kFenceShift), (uint64_t)X.V);
+    uint64_t k = lower_bound_dev(X.ext, lo, hi, x);
+    *present = (k < X.V && X.ext[k] == x);
     return k;
+}
+__global__ void k_build_fence(const uint64_t* __restrict__ ext, uint64_t V, uint64_t* __restrict__ fence) {
+    uint64_t i = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x;
+    if ((i << kFenceShift) < V) fence[i] = ext[i << kFenceShift];
 }
 
 // ===================================================================== a2 ====
 // Unique vertices of the (v, ts, seq)-sorted visible node ops: final liveness
 // (last op), latest delete point tD, old presence.  Compaction via look-back.
 __global__ void __launch_bounds__(kThreads) k_node_segments(
-    Ops ops, const uint32_t* __restrict__ sidx, uint64_t n, const uint64_t* __restrict__ old_ext,
-    uint64_t V, int identity, NodeVtx* __restrict__ nv, uint64_t* __restrict__ nv_ext,
-    uint64_t* __restrict__ status, uint64_t n_tiles, Counters* __restrict__ c) {
+    Ops ops, const uint32_t* __restrict__ sidx, uint64_t n, ExtIndex X, NodeVtx* __restrict__ nv,
+    uint64_t* __restrict__ nv_ext, uint64_t* __restrict__ status, uint64_t n_tiles, Counters* __restrict__ c) {
     __shared__ uint32_t s_tile;
-    __shared__ uint64_t s_scan[kThreads / 32 + 1];
+    __shared__ uint32_t s_cmp[kItems * kThreads / 32 + 1];
     __shared__ uint64_t s_base;
     if (threadIdx.x == 0) s_tile = atomicAdd(&c->tiles[1], 1u);
     __syncthreads();
     const uint32_t tile = s_tile;
-    const uint64_t i0 = (uint64_t)tile * kTile + (uint64_t)threadIdx.x * kItems;
-    uint64_t heads = 0;
-    uint32_t hmask = 0;
+    const uint64_t i0 = (uint64_t)tile * kTile + threadIdx.x;
+    bool head[kItems];
+    uint32_t pos[kItems];
 #pragma unroll
     for (int j = 0; j < kItems; ++j) {
-        uint64_t i = i0 + j;
-        if (i < n && (i == 0 || ops.src[sidx[i]] != ops.src[sidx[i - 1]])) { hmask |= 1u << j; heads++; }
+        uint64_t i = i0 + (uint64_t)j * kThreads;
+        head[j] = i < n && (i == 0 || ops.src[sidx[i]] != ops.src[sidx[i - 1]]);
     }
-    uint64_t tot, excl = block_exclusive_scan<kThreads>(heads, s_scan, &tot);
+    uint32_t tot = striped_compact<kThreads, kItems>(head, pos, s_cmp);
     if (threadIdx.x < 32) {
         uint64_t b = lookback_warp(status, tile, tot);
         if (lane_id() == 0) { s_base = b; if (tile == n_tiles - 1) c->n_unique = b + tot; }
     }
     __syncthreads();
-    uint64_t q = s_base + excl;
 #pragma unroll
     for (int j = 0; j < kItems; ++j) {
-        if (!(hmask >> j & 1)) continue;
-        uint64_t i = i0 + j;
+        if (!head[j]) continue;
+        uint64_t i = i0 + (uint64_t)j * kThreads;
         uint64_t v = ops.src[sidx[i]];
         uint64_t e = i;
         NodeVtx r;
@@ -195,16 +209,16 @@ __global__ void __launch_bounds__(kThreads) k_node_segments(
         }
         if (last == NODE_INSERT) r.flags |= NV_FINAL;
         bool present;
-        uint64_t k = old_lookup(old_ext, V, identity, v, &present);
+        uint64_t k = old_lookup(X, v, &present);
         if (present) r.flags |= NV_OLD;
         r.oldpos = (uint32_t)k;
         r.start = (uint32_t)i;
         r.end = (uint32_t)e;
         r.newid = kNone32;
         r.pad = 0;
+        uint64_t q = s_base + pos[j];
         nv[q] = r;
         nv_ext[q] = v;
-        ++q;
     }
 }
 
@@ -277,21 +291,28 @@ __device__ __forceinline__ uint64_t gallop_ub(const T* a, uint64_t lo, uint64_t 
 
 // ID-map compaction (reading A9): remap[k] = new dense id of old vertex k or
 // kNone32 (dropped); new_ext[remap[k]] = ext[k].  Survivor rank minus dropped
-// before plus inserted (by old position) at or before.
+// before plus inserted (by old position) at or before.  Thread per vertex; the
+// CTA narrows the two small sorted lists to its id range first.
+constexpr int kRemapTile = 1024;
 __global__ void __launch_bounds__(kThreads) k_remap(
     const uint64_t* __restrict__ old_ext, int identity, uint64_t V, const uint32_t* __restrict__ dropped,
     uint64_t n_dropped, const uint32_t* __restrict__ ins_oldpos, uint64_t n_ins,
     uint32_t* __restrict__ remap, uint64_t* __restrict__ new_ext) {
-    uint64_t k0 = ((uint64_t)blockIdx.x * kThreads + threadIdx.x) * kItems;
-    if (k0 >= V) return;
-    uint64_t dp = lower_bound_dev(dropped, 0, n_dropped, (uint32_t)k0);
-    uint64_t ip = lower_bound_dev(ins_oldpos, 0, n_ins, (uint32_t)k0);
-    for (int j = 0; j < kItems; ++j) {
-        uint64_t k = k0 + j;
-        if (k >= V) break;
-        dp = gallop_lb(dropped, dp, n_dropped, (uint32_t)k);
-        ip = gallop_ub(ins_oldpos, ip, n_ins, (uint32_t)k);
+    __shared__ uint64_t s_r[4];
+    const uint64_t k0 = (uint64_t)blockIdx.x * kRemapTile, k1 = min(k0 + kRemapTile, V);
+    if (threadIdx.x < 4) {
+        const int w = threadIdx.x;
+        uint32_t key = (uint32_t)((w & 1) ? k1 : k0);
+        s_r[w] = (w < 2) ? lower_bound_dev(dropped, 0, n_dropped, key)
+                         : upper_bound_dev(ins_oldpos, 0, n_ins, key);  // oldpos <= key
+    }
+    __syncthreads();
+    const uint64_t da = s_r[0], db = s_r[1], ia = s_r[2], ib = s_r[3];
+    for (uint64_t k = k0 + threadIdx.x; k < k1; k += kThreads) {
+        uint64_t dp = lower_bound_dev(dropped, da, db, (uint32_t)k);
         bool is_dropped = dp < n_dropped && dropped[dp] == (uint32_t)k;
+        // inserted with oldpos <= k: those <= k0 (= ia) plus those in (k0, k]
+        uint64_t ip = upper_bound_dev(ins_oldpos, ia, ib, (uint32_t)k);
         uint32_t r = is_dropped ? kNone32 : (uint32_t)(k - dp + ip);
         remap[k] = r;
         if (!is_dropped) new_ext[r] = identity ? k : old_ext[k];
@@ -337,9 +358,7 @@ struct PrepArgs {
     Ops ops;
     const uint32_t* edge_idx;
     uint64_t n_edge;
-    const uint64_t* old_ext;
-    uint64_t V;
-    int identity;
+    ExtIndex X;
     const uint32_t* remap;  // nullable (identity remap)
     const NodeVtx* nv;
     const uint64_t* nv_ext;
@@ -377,7 +396,7 @@ __device__ __forceinline__ Lookup do_lookup(const PrepArgs& a, uint64_t x) {
         }
     }
     bool present;
-    uint64_t k = old_lookup(a.old_ext, a.V, a.identity, x, &present);
+    uint64_t k = old_lookup(a.X, x, &present);
     L.oldpos = (uint32_t)k;
     L.old_present = present;
     L.final_live = present;
@@ -404,19 +423,21 @@ __device__ __forceinline__ bool live_at(const PrepArgs& a, const Lookup& L, uint
 // (src' << bits | dst'), compaction of surviving ops via look-back.
 __global__ void __launch_bounds__(kThreads) k_edge_prep(PrepArgs a) {
     __shared__ uint32_t s_tile;
-    __shared__ uint64_t s_scan[kThreads / 32 + 1];
+    __shared__ uint32_t s_cmp[kItems * kThreads / 32 + 1];
     __shared__ uint64_t s_base;
     if (threadIdx.x == 0) s_tile = atomicAdd(&a.c->tiles[3], 1u);
     __syncthreads();
     const uint32_t tile = s_tile;
-    const uint64_t i0 = (uint64_t)tile * kTile + (uint64_t)threadIdx.x * kItems;
+    const uint64_t i0 = (uint64_t)tile * kTile + threadIdx.x;
     uint64_t key[kItems];
-    uint32_t valid = 0;
-    uint64_t nvalid = 0, ngated = 0, nbad = 0;
+    bool valid[kItems];
+    uint32_t pos[kItems];
+    uint64_t ngated = 0, nbad = 0;
 #pragma unroll
     for (int j = 0; j < kItems; ++j) {
-        uint64_t i = i0 + j;
+        uint64_t i = i0 + (uint64_t)j * kThreads;
         key[j] = 0;
+        valid[j] = false;
         if (i >= a.n_edge) continue;
         uint32_t o = a.edge_idx[i];
         uint8_t kind = a.ops.kind[o];
@@ -434,8 +455,7 @@ __global__ void __launch_bounds__(kThreads) k_edge_prep(PrepArgs a) {
             if (!live_at(a, Lu, ts, seq) || !live_at(a, Lw, ts, seq)) ok = false;
         }
         if (ok) {
-            valid |= 1u << j;
-            nvalid++;
+            valid[j] = true;
             key[j] = ((uint64_t)Lu.newid << a.bits) | (uint64_t)Lw.newid;
             a.op_flags[o] = (uint8_t)((Lu.old_present ? 1 : 0) | (Lw.old_present ? 2 : 0) |
                                       ((Lu.hasD || Lw.hasD) ? 4 : 0));
@@ -449,16 +469,19 @@ __global__ void __launch_bounds__(kThreads) k_edge_prep(PrepArgs a) {
     if (lane_id() == 0 && gsum) atomicAdd(&a.c->n_gated, (unsigned long long)gsum);
     uint64_t bsum = warp_sum(nbad);
     if (lane_id() == 0 && bsum) atomicOr(&a.c->status, (unsigned long long)ST_CREATE_ENDPOINT);
-    uint64_t tot, excl = block_exclusive_scan<kThreads>(nvalid, s_scan, &tot);
+    uint32_t tot = striped_compact<kThreads, kItems>(valid, pos, s_cmp);
     if (threadIdx.x < 32) {
         uint64_t b = lookback_warp(a.status, tile, tot);
         if (lane_id() == 0) { s_base = b; if (tile == a.n_tiles - 1) a.c->n_valid = b + tot; }
     }
     __syncthreads();
-    uint64_t p = s_base + excl;
 #pragma unroll
     for (int j = 0; j < kItems; ++j) {
-        if (valid >> j & 1) { a.keys[p] = key[j]; a.vals[p] = a.edge_idx[i0 + j]; ++p; }
+        if (valid[j]) {
+            uint64_t p = s_base + pos[j];
+            a.keys[p] = key[j];
+            a.vals[p] = a.edge_idx[i0 + (uint64_t)j * kThreads];
+        }
     }
 }
 
@@ -481,11 +504,13 @@ struct ClassArgs {
     const uint32_t* op_opos_w;
     const int64_t* old_off;
     const uint32_t* old_cols;
+    uint64_t V_old;
     uint64_t* ins_pos;
     uint32_t* ins_row;
     uint32_t* ins_col;
     float* ins_w;
     uint64_t* del_pos;
+    uint32_t* del_row;
     uint64_t* upd_pos;
     float* upd_w;
     uint64_t* status3;
@@ -493,26 +518,33 @@ struct ClassArgs {
     Counters* c;
 };
 
+constexpr int kCItems = 4;                    // classify: items per thread (register budget)
+constexpr int kCTile = kThreads * kCItems;
 __global__ void __launch_bounds__(kThreads) k_reduce_classify(ClassArgs a) {
     __shared__ uint32_t s_tile;
-    __shared__ uint64_t s_scan[kThreads / 32 + 1];
+    __shared__ uint32_t s_cmp[3][kCItems * kThreads / 32 + 1];
     __shared__ uint64_t s_base[3];
     if (threadIdx.x == 0) s_tile = atomicAdd(&a.c->tiles[4], 1u);
     __syncthreads();
     const uint32_t tile = s_tile;
-    const uint64_t i0 = (uint64_t)tile * kTile + (uint64_t)threadIdx.x * kItems;
-    uint8_t cat[kItems];
-    uint64_t pos[kItems];
-    float wv[kItems];
-    uint64_t cnt[3] = {0, 0, 0};
+    const uint64_t i0 = (uint64_t)tile * kCTile + threadIdx.x;
+    uint8_t cat[kCItems], meta[kCItems];
+    uint64_t pos[kCItems], lo[kCItems], hi[kCItems], end[kCItems];
+    uint32_t colq[kCItems];
+    float wv[kCItems];
 #pragma unroll
-    for (int j = 0; j < kItems; ++j) {
+    for (int j = 0; j < kCItems; ++j) {
         cat[j] = 0;
-        uint64_t i = i0 + j;
+        pos[j] = 0;
+        wv[j] = 0.f;
+        lo[j] = hi[j] = end[j] = 0;
+        colq[j] = 0;
+        meta[j] = 0;
+        uint64_t i = i0 + (uint64_t)j * kThreads;
         if (i >= a.n) continue;
         uint64_t key = a.keys[i];
         if (i > 0 && a.keys[i - 1] == key) continue;
-        // segment [i, e)
+        // segment [i, e): latest-commit-wins over (ts, seq)
         uint64_t nw_ts = 0, nw_seq = 0, w_ts = 0, w_seq = 0;
         bool has_nw = false, has_w = false;
         uint8_t nw_kind = 0;
@@ -530,30 +562,63 @@ __global__ void __launch_bounds__(kThreads) k_reduce_classify(ClassArgs a) {
         }
         uint32_t o0 = a.vals[i];
         uint8_t fl = a.op_flags[o0];
-        bool u_old = fl & 1, w_old = fl & 2, hd = fl & 4;
+        bool u_old = fl & 1;
         uint32_t ou = a.op_opos_u[o0], ow = a.op_opos_w[o0];
-        uint64_t p;
-        bool found = false;
-        if (u_old) {
-            uint64_t beg = (uint64_t)a.old_off[ou], end = (uint64_t)a.old_off[ou + 1];
-            p = lower_bound_dev(a.old_cols, beg, end, ow);
-            found = w_old && p < end && a.old_cols[p] == ow;
-        } else {
-            p = (uint64_t)a.old_off[ou];
+        // outcome category before the old-row lookup: 1 insert-like, 2 delete, 3 weight-only
+        cat[j] = (has_nw && nw_kind == EDGE_INSERT) ? 1 : (has_nw ? 2 : (has_w ? 3 : 0));
+        meta[j] = fl;
+        colq[j] = ow;
+        wv[j] = w_val;
+        if (u_old) { lo[j] = (uint64_t)a.old_off[ou]; hi[j] = (uint64_t)a.old_off[ou + 1]; }
+        else { lo[j] = hi[j] = (uint64_t)a.old_off[ou]; }
+        end[j] = hi[j];
+    }
+    // lock-step searches of every item's column in its old row: up to kCItems
+    // independent loads in flight per thread.  The first probes interpolate
+    // between the known value bounds (columns of a row spread over [0, V)),
+    // then plain bisection; cuts DRAM probes per lookup from ~log2(deg) to ~3.
+    uint32_t vlo[kCItems], vhi[kCItems];
+#pragma unroll
+    for (int j = 0; j < kCItems; ++j) { vlo[j] = 0; vhi[j] = (uint32_t)a.V_old; }
+    for (int step = 0; step < 48; ++step) {
+        bool any = false;
+#pragma unroll
+        for (int j = 0; j < kCItems; ++j) {
+            if (lo[j] < hi[j]) {
+                const uint64_t len = hi[j] - lo[j];
+                uint64_t mid;
+                if (step < 4 && len > 8 && colq[j] >= vlo[j] && vhi[j] > vlo[j]) {
+                    mid = lo[j] + (uint64_t)(((float)(colq[j] - vlo[j]) / (float)(vhi[j] - vlo[j])) * (float)len);
+                    if (mid >= hi[j]) mid = hi[j] - 1;
+                } else {
+                    mid = (lo[j] + hi[j]) >> 1;
+                }
+                const uint32_t v = a.old_cols[mid];
+                if (v < colq[j]) { lo[j] = mid + 1; vlo[j] = v + 1; } else { hi[j] = mid; vhi[j] = v; }
+                any = true;
+            }
         }
-        bool present = found && !hd;  // a node delete of an endpoint cleared the old edge
+        if (!any) break;
+    }
+#pragma unroll
+    for (int j = 0; j < kCItems; ++j) {
+        if (!cat[j]) continue;
+        const uint64_t p = lo[j];
+        const bool found = (meta[j] & 1) && (meta[j] & 2) && p < end[j] && a.old_cols[p] == colq[j];
+        const bool present = found && !(meta[j] & 4);  // a node delete of an endpoint cleared the old edge
         uint8_t ct = 0;
-        if (has_nw && nw_kind == EDGE_INSERT) ct = present ? 3 : 1;
-        else if (has_nw && nw_kind == EDGE_DELETE) ct = present ? 2 : 0;
-        else if (has_w) ct = present ? 3 : 0;
+        if (cat[j] == 1) ct = present ? 3 : 1;
+        else if (cat[j] == 2) ct = present ? 2 : 0;
+        else ct = present ? 3 : 0;
         cat[j] = ct;
         pos[j] = p;
-        wv[j] = w_val;
-        if (ct) cnt[ct - 1]++;
     }
-    uint64_t excl[3], tot[3];
+    bool f[3][kCItems];
+    uint32_t rk[3][kCItems], tot[3];
 #pragma unroll
-    for (int q = 0; q < 3; ++q) excl[q] = block_exclusive_scan<kThreads>(cnt[q], s_scan, &tot[q]);
+    for (int j = 0; j < kCItems; ++j) { f[0][j] = cat[j] == 1; f[1][j] = cat[j] == 2; f[2][j] = cat[j] == 3; }
+#pragma unroll
+    for (int q = 0; q < 3; ++q) tot[q] = striped_compact<kThreads, kCItems>(f[q], rk[q], s_cmp[q]);
     const int wid = threadIdx.x >> 5;
     if (wid < 3) {
         uint64_t b = lookback_warp(a.status3 + (uint64_t)wid * a.n_tiles, tile, tot[wid]);
@@ -566,23 +631,24 @@ __global__ void __launch_bounds__(kThreads) k_reduce_classify(ClassArgs a) {
         }
     }
     __syncthreads();
-    uint64_t oi = s_base[0] + excl[0], od = s_base[1] + excl[1], ou = s_base[2] + excl[2];
     const uint64_t mask = (1ull << a.bits) - 1;
 #pragma unroll
-    for (int j = 0; j < kItems; ++j) {
+    for (int j = 0; j < kCItems; ++j) {
         if (cat[j] == 1) {
-            uint64_t key = a.keys[i0 + j];
+            uint64_t key = a.keys[i0 + (uint64_t)j * kThreads];
+            uint64_t oi = s_base[0] + rk[0][j];
             a.ins_pos[oi] = pos[j];
             a.ins_row[oi] = (uint32_t)(key >> a.bits);
             a.ins_col[oi] = (uint32_t)(key & mask);
             a.ins_w[oi] = wv[j];
-            ++oi;
         } else if (cat[j] == 2) {
-            a.del_pos[od++] = pos[j];
+            uint64_t od = s_base[1] + rk[1][j];
+            a.del_pos[od] = pos[j];
+            a.del_row[od] = (uint32_t)(a.keys[i0 + (uint64_t)j * kThreads] >> a.bits);
         } else if (cat[j] == 3) {
+            uint64_t ou = s_base[2] + rk[2][j];
             a.upd_pos[ou] = pos[j];
             a.upd_w[ou] = wv[j];
-            ++ou;
         }
     }
 }
@@ -595,8 +661,11 @@ __global__ void __launch_bounds__(kThreads) k_reduce_classify(ClassArgs a) {
 // for giant rows and insert bursts), stages its old elements in shared memory,
 // drops deleted / cascaded elements, overrides weights, remaps column IDs and
 // writes its contiguous output chunk with coalesced 128-bit stores.
-constexpr int kMergeItems = 8;
-constexpr int kMergeTile = kThreads * kMergeItems;  // 2048 merged items per CTA
+constexpr int kMergeTile = 2048;             // merged items per tile
+constexpr int kCascBlock = 2048;             // cascade mask: elements per counted block (64 words)
+constexpr int kMergeBuf = kMergeTile + 8;     // staged old elements (+ 16 B alignment slack)
+constexpr int kRemapBlockShift = 10;          // two-level remap: 1024 old ids per block
+constexpr int32_t kRemapMixed = INT32_MIN;    // block has a dropped/inserted id inside
 
 struct MergeArgs {
     const uint32_t* old_cols;
@@ -613,18 +682,26 @@ struct MergeArgs {
     const float* upd_w;
     uint64_t n_upd;
     const uint32_t* remap;
+    const int32_t* remap_shift;  // per 1024-block constant shift or kRemapMixed
     const uint32_t* hd_bits;
     const uint32_t* hd_rows;
     uint64_t n_hd;
     uint32_t* new_cols;
     float* new_w;
     int64_t* KR;  // CASC: kept elements before each old row start, [V_old + 1]
-    uint64_t* status;
+    const uint32_t* casc_mask;  // CASC: 1 bit per old element (removed by a node delete)
+    const uint64_t* casc_pre;   // CASC: cascaded elements before each 2048-element block
     uint64_t n_tiles;
     Counters* c;
 };
 
-// smallest r with ins_pos[r] + r >= d  (number of inserted records among the first d merged items)
+// Merge-path split of tile boundary t: r = inserted records among the first d
+// merged items (smallest r with ins_pos[r] + r >= d), j = d - r old elements,
+// and the ranks of j in the sorted delete / update / cascade-row lists.
+struct TilePart {
+    uint64_t r, dl, ul, hA, hB, k;  // k: first old row starting at or after j (CASC)
+};
+
 __device__ __forceinline__ uint64_t ins_split(const uint64_t* ins_pos, uint64_t n_ins, uint64_t d) {
     uint64_t lo = 0, hi = n_ins;
     while (lo < hi) {
@@ -634,190 +711,410 @@ __device__ __forceinline__ uint64_t ins_split(const uint64_t* ins_pos, uint64_t 
     return lo;
 }
 
+__global__ void k_merge_partition(MergeArgs a, TilePart* __restrict__ part) {
+    uint64_t t = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x;
+    if (t > a.n_tiles) return;
+    const uint64_t Dtot = a.E_old + a.n_ins;
+    const uint64_t d = min(t * kMergeTile, Dtot);
+    TilePart p;
+    p.r = (d == Dtot) ? a.n_ins : ins_split(a.ins_pos, a.n_ins, d);
+    const uint64_t j = d - p.r;
+    p.dl = lower_bound_dev(a.del_pos, 0, a.n_del, j);
+    p.ul = lower_bound_dev(a.upd_pos, 0, a.n_upd, j);
+    p.hA = p.hB = 0;
+    p.k = a.n_hd ? lower_bound_dev(a.old_off, 0, a.V_old + 1, (int64_t)j) : 0;
+    part[t] = p;
+}
+
+// ---- TMA 1-D bulk copy + mbarrier helpers (sm_90+ async proxy; SASS UBLKCP)
+__device__ __forceinline__ uint32_t smem_u32(const void* p) { return (uint32_t)__cvta_generic_to_shared(p); }
+__device__ __forceinline__ void mbar_init(uint64_t* bar, uint32_t count) {
+    asm volatile("mbarrier.init.shared::cta.b64 [%0], %1;" ::"r"(smem_u32(bar)), "r"(count) : "memory");
+}
+__device__ __forceinline__ void fence_mbar_init() { asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory"); }
+__device__ __forceinline__ void fence_proxy_async() { asm volatile("fence.proxy.async.shared::cta;" ::: "memory"); }
+__device__ __forceinline__ void mbar_expect_tx(uint64_t* bar, uint32_t bytes) {
+    asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(smem_u32(bar)), "r"(bytes) : "memory");
+}
+__device__ __forceinline__ void bulk_g2s(void* dst, const void* src, uint32_t bytes, uint64_t* bar) {
+    asm volatile("cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];"
+                 ::"r"(smem_u32(dst)), "l"(src), "r"(bytes), "r"(smem_u32(bar)) : "memory");
+}
+__device__ __forceinline__ void mbar_wait(uint64_t* bar, uint32_t phase) {
+    asm volatile(
+        "{\n"
+        ".reg .pred p;\n"
+        "WAIT_%=:\n"
+        "mbarrier.try_wait.parity.shared::cta.b64 p, [%0], %1;\n"
+        "@!p bra WAIT_%=;\n"
+        "}\n" ::"r"(smem_u32(bar)), "r"(phase) : "memory");
+}
+
+// Global merge path.  The new column/weight arrays are the merge of the kept
+// old elements (old order) with the inserted records (key order); an inserted
+// record at old position p precedes old element p, so its merged index is
+// p + r.  Tile t owns merged items [t*2048, (t+1)*2048) (load balanced for
+// giant rows and insert bursts).  Persistent CTAs walk the tiles; while one
+// tile is processed the next tile's old elements stream into the other shared
+// buffer with two TMA bulk copies.  Each warp compacts a 256-slot chunk with
+// ballots: slot -> old element index / inserted record, drop deleted and
+// cascaded elements, override weights, remap column IDs, coalesced stores.
 template <bool CASC, bool REMAP>
-__global__ void __launch_bounds__(kThreads) k_merge(MergeArgs a) {
-    __shared__ __align__(16) uint32_t s_col[kMergeTile + 8];
-    __shared__ __align__(16) float s_w[kMergeTile + 8];
-    __shared__ uint32_t s_slot[kMergeTile + 1];
-    __shared__ uint32_t s_oc[kMergeTile];
-    __shared__ float s_ow[kMergeTile];
+__global__ void __launch_bounds__(kThreads) k_merge(MergeArgs a, const TilePart* __restrict__ part) {
+    __shared__ __align__(128) uint32_t s_col[2][kMergeBuf];
+    __shared__ __align__(128) float s_w[2][kMergeBuf];
+    __shared__ uint16_t s_slot[kMergeTile];
     __shared__ uint8_t s_keep[kMergeTile];
-    // kept-before per old element (CASC); aliases s_slot, which is dead once the
-    // blocked pass has loaded it into registers (two block scans = barriers in between)
-    uint32_t* const s_kp = s_slot;
-    __shared__ uint64_t s_scan[kThreads / 32 + 1];
-    __shared__ uint64_t s_r[2], s_d[2], s_u[2], s_h[2], s_base;
+    __shared__ uint32_t s_kp[CASC ? kMergeTile + 1 : 1];
+    __shared__ uint32_t s_wold[kThreads / 32], s_wemit[kThreads / 32];
+    __shared__ __align__(8) uint64_t s_bar[2];
+    __shared__ uint64_t s_cbefore;
+
+    const int tid = threadIdx.x, wid = tid >> 5;
+    const uint32_t lane = lane_id(), lt = lanemask_lt();
+    const uint64_t Dtot = a.E_old + a.n_ins;
+    if (tid == 0) { mbar_init(&s_bar[0], 1); mbar_init(&s_bar[1], 1); fence_mbar_init(); }
+    __syncthreads();
+
+    auto tile_j = [&](uint64_t t) -> uint64_t { return min(t * kMergeTile, Dtot) - part[t].r; };
+    auto issue = [&](uint64_t t, int b) {  // one thread: stage old elements of tile t
+        const uint64_t j0 = tile_j(t), j1 = tile_j(t + 1);
+        const uint64_t a0 = j0 & ~3ull, a1 = (j1 + 3) & ~3ull;
+        const uint32_t bytes = (uint32_t)((a1 - a0) * 4);
+        mbar_expect_tx(&s_bar[b], 2 * bytes);
+        if (bytes) {
+            bulk_g2s(&s_col[b][0], a.old_cols + a0, bytes, &s_bar[b]);
+            bulk_g2s(&s_w[b][0], a.old_w + a0, bytes, &s_bar[b]);
+        }
+    };
+
+    uint64_t t = blockIdx.x;
+    if (t < a.n_tiles && tid == 0) issue(t, 0);
+    for (uint32_t it = 0; t < a.n_tiles; t += gridDim.x, ++it) {
+        const int b = it & 1;
+        if (tid == 0 && t + gridDim.x < a.n_tiles) { fence_proxy_async(); issue(t + gridDim.x, b ^ 1); }
+        const TilePart p0 = part[t], p1 = part[t + 1];
+        const uint64_t d0 = min(t * kMergeTile, Dtot), d1 = min((t + 1) * kMergeTile, Dtot);
+        const uint64_t r0 = p0.r, j0 = d0 - r0, j1 = d1 - p1.r;
+        const uint32_t n_old = (uint32_t)(j1 - j0), n_new = (uint32_t)(p1.r - r0), n_tot = n_old + n_new;
+        const uint32_t sh = (uint32_t)(j0 & 3);  // staged element i lives at s_*[i + sh]
+        for (uint32_t i = tid; i < kMergeTile; i += kThreads) { s_slot[i] = 0xFFFF; s_keep[i] = 1; }
+        __syncthreads();
+        for (uint32_t s = tid; s < n_new; s += kThreads) s_slot[(a.ins_pos[r0 + s] - j0) + s] = (uint16_t)s;
+        for (uint64_t i = p0.dl + tid; i < p1.dl; i += kThreads) s_keep[a.del_pos[i] - j0] = 0;
+        if (CASC) {
+            for (uint32_t i = tid; i < n_old; i += kThreads)
+                if (a.casc_mask[(j0 + i) >> 5] >> ((j0 + i) & 31) & 1) s_keep[i] = 0;
+            if (wid == 0) {  // cascaded elements before j0: block prefix + popcount of the partial block
+                const uint64_t blk = j0 / kCascBlock, wb = blk * (kCascBlock / 32), we = j0 >> 5;
+                uint32_t c = 0;
+                for (uint64_t q = wb + lane; q <= we; q += 32) {
+                    uint32_t m = a.casc_mask[q];
+                    if (q == we) m &= (j0 & 31) ? (0xFFFFFFFFu >> (32 - (j0 & 31))) : 0u;
+                    c += __popc(m);
+                }
+                c = warp_sum(c);
+                if (lane == 0) s_cbefore = a.casc_pre[blk] + c;
+            }
+        }
+        mbar_wait(&s_bar[b], (it >> 1) & 1);
+        const uint64_t a0 = j0 & ~3ull;
+        for (uint64_t i = p0.ul + tid; i < p1.ul; i += kThreads) s_w[b][a.upd_pos[i] - a0] = a.upd_w[i];
+        __syncthreads();
+        // pass 1: old slots per warp chunk
+        const uint32_t mb = wid * 256;
+        uint32_t oldm[8];
+        uint32_t n_oldw = 0;
+#pragma unroll
+        for (int k = 0; k < 8; ++k) {
+            uint32_t m = mb + k * 32 + lane;
+            oldm[k] = __ballot_sync(0xffffffffu, m < n_tot && s_slot[m] == 0xFFFF);
+            n_oldw += __popc(oldm[k]);
+        }
+        if (lane == 0) s_wold[wid] = n_oldw;
+        __syncthreads();
+        uint32_t oi_base = 0;
+        for (int w2 = 0; w2 < wid; ++w2) oi_base += s_wold[w2];
+        // pass 2: emitted items per warp chunk
+        uint32_t emm[8];
+        uint32_t n_emw = 0;
+        {
+            uint32_t oi_run = oi_base;
+#pragma unroll
+            for (int k = 0; k < 8; ++k) {
+                uint32_t m = mb + k * 32 + lane;
+                bool isold = oldm[k] >> lane & 1;
+                uint32_t oi = oi_run + __popc(oldm[k] & lt);
+                bool e = (m < n_tot) && (!isold || s_keep[oi]);
+                emm[k] = __ballot_sync(0xffffffffu, e);
+                n_emw += __popc(emm[k]);
+                oi_run += __popc(oldm[k]);
+            }
+        }
+        if (lane == 0) s_wemit[wid] = n_emw;
+        __syncthreads();
+        uint32_t em_base = 0, tile_emit = 0;
+        for (int w2 = 0; w2 < kThreads / 32; ++w2) {
+            uint32_t v = s_wemit[w2];
+            if (w2 < wid) em_base += v;
+            tile_emit += v;
+        }
+        // output index of the tile's first item: kept old elements before j0 + inserted
+        // records before d0 (cascade mode: from the count pass + scan)
+        const uint64_t base = j0 - p0.dl - (CASC ? s_cbefore : 0) + r0;
+        // pass 3: write the tile's output chunk (coalesced 4 B stores per warp iteration)
+        {
+            uint32_t oi_run = oi_base, e_run = em_base;
+#pragma unroll
+            for (int k = 0; k < 8; ++k) {
+                uint32_t m = mb + k * 32 + lane;
+                bool isold = oldm[k] >> lane & 1;
+                uint32_t oi = oi_run + __popc(oldm[k] & lt);
+                bool e = emm[k] >> lane & 1;
+                uint32_t eo = e_run + __popc(emm[k] & lt);
+                if (CASC && isold) s_kp[oi] = eo - (m - oi);
+                if (e) {
+                    uint32_t col;
+                    float wv;
+                    if (isold) {
+                        col = s_col[b][oi + sh];
+                        wv = s_w[b][oi + sh];
+                        if (REMAP) {
+                            int32_t shf = a.remap_shift[col >> kRemapBlockShift];
+                            col = (shf != kRemapMixed) ? (uint32_t)((int64_t)col + shf) : a.remap[col];
+                        }
+                    } else {
+                        uint32_t s = s_slot[m];
+                        col = a.ins_col[r0 + s];
+                        wv = a.ins_w[r0 + s];
+                    }
+                    a.new_cols[base + eo] = col;
+                    a.new_w[base + eo] = wv;
+                }
+                oi_run += __popc(oldm[k]);
+                e_run += __popc(emm[k]);
+            }
+        }
+        if (CASC) {
+            __syncthreads();
+            if (tid == 0) s_kp[n_old] = tile_emit - n_new;
+            __syncthreads();
+            // kept-before at every old row that starts inside this tile (last tile: also at E)
+            const bool last = (t == a.n_tiles - 1);
+            const uint64_t kept_before = base - r0;
+            uint64_t ka = p0.k;
+            uint64_t kb = last ? a.V_old + 1 : p1.k;
+            for (uint64_t k = ka + tid; k < kb; k += kThreads)
+                a.KR[k] = (int64_t)(kept_before + s_kp[(uint64_t)a.old_off[k] - j0]);
+        }
+        __syncthreads();
+    }
+}
+
+// Cascade mode (a4 cascade pass): one bit per old element, set when a node delete
+// removes it (its row's vertex or its column's vertex had a visible delete, A8),
+// plus per-2048-element block counts.  Runs on a side stream, overlapped with the
+// edge-op sort/classify phase, so the merge never touches the cascade bitmap.
+
+// columns pointing at deleted vertices: one ballot per 32 elements -> one mask
+// word (pure stores, every element's loads independent)
+__global__ void __launch_bounds__(kThreads) k_casc_cols(const uint32_t* __restrict__ old_cols, uint64_t E,
+        const uint32_t* __restrict__ hd_bits, uint32_t* __restrict__ mask) {
+    const uint64_t b0 = (uint64_t)blockIdx.x * kCascBlock;
+    constexpr int PER = kCascBlock / kThreads;  // 8 elements per thread, striped
+    uint32_t col[PER];
+#pragma unroll
+    for (int j = 0; j < PER; ++j) {
+        uint64_t x = b0 + (uint64_t)j * kThreads + threadIdx.x;
+        col[j] = x < E ? old_cols[x] : 0;
+    }
+    uint32_t bit[PER];
+#pragma unroll
+    for (int j = 0; j < PER; ++j) bit[j] = hd_bits[col[j] >> 5] >> (col[j] & 31);
+#pragma unroll
+    for (int j = 0; j < PER; ++j) {
+        uint64_t x = b0 + (uint64_t)j * kThreads + threadIdx.x;
+        uint32_t m = __ballot_sync(0xffffffffu, x < E && (bit[j] & 1));
+        if (lane_id() == 0) mask[x >> 5] = m;  // words past E are written as 0
+    }
+}
+
+// rows of deleted vertices -> whole bit ranges (warp per row), OR-ed into the mask
+__global__ void k_casc_rows(const int64_t* __restrict__ old_off, const uint32_t* __restrict__ hd_rows,
+                            uint64_t n_hd, uint32_t* __restrict__ mask) {
+    const uint64_t nw = ((uint64_t)gridDim.x * blockDim.x) >> 5;
+    for (uint64_t h = (blockIdx.x * (uint64_t)blockDim.x + threadIdx.x) >> 5; h < n_hd; h += nw) {
+        uint32_t k = hd_rows[h];
+        uint64_t b = (uint64_t)old_off[k], e = (uint64_t)old_off[k + 1];
+        if (b == e) continue;
+        uint64_t wb = b >> 5, we = (e - 1) >> 5;
+        for (uint64_t q = wb + lane_id(); q <= we; q += 32) {
+            uint32_t m = 0xFFFFFFFFu;
+            if (q == wb) m &= 0xFFFFFFFFu << (b & 31);
+            if (q == we) m &= 0xFFFFFFFFu >> (31 - ((e - 1) & 31));
+            if (m == 0xFFFFFFFFu) mask[q] = m; else atomicOr(&mask[q], m);
+        }
+    }
+}
+
+// per 2048-element block: cascaded count = popcount of its 64 mask words; then
+// the exclusive scan over blocks (decoupled look-back), total at [nblk]
+__global__ void __launch_bounds__(kThreads) k_casc_scan(const uint32_t* __restrict__ mask, uint64_t nblk,
+        uint64_t* __restrict__ pre, uint64_t* __restrict__ status, unsigned int* __restrict__ ctr) {
     __shared__ uint32_t s_tile;
+    __shared__ uint64_t s_scan[kThreads / 32 + 1];
+    __shared__ uint64_t s_cnt[kThreads];
+    __shared__ uint64_t s_base;
+    if (threadIdx.x == 0) s_tile = atomicAdd(ctr, 1u);
+    __syncthreads();
+    const uint64_t blk0 = (uint64_t)s_tile * kThreads;  // one block count per thread
+    const int w = threadIdx.x >> 5;
+    for (int i = 0; i < 32; ++i) {  // warp w counts blocks blk0 + w*32 + i (coalesced 2 words per lane)
+        uint64_t bk = blk0 + w * 32 + i;
+        uint32_t c = 0;
+        if (bk < nblk) {
+            const uint2 v = reinterpret_cast<const uint2*>(mask + bk * (kCascBlock / 32))[lane_id()];
+            c = __popc(v.x) + __popc(v.y);
+        }
+        c = warp_sum(c);
+        if (lane_id() == 0) s_cnt[w * 32 + i] = c;
+    }
+    __syncthreads();
+    uint64_t v = s_cnt[threadIdx.x], tot;
+    uint64_t ex = block_exclusive_scan<kThreads>(v, s_scan, &tot);
+    if (threadIdx.x < 32) {
+        uint64_t b = lookback_warp(status, s_tile, tot);
+        if (lane_id() == 0) s_base = b;
+    }
+    __syncthreads();
+    uint64_t bk = blk0 + threadIdx.x;
+    if (bk <= nblk) pre[bk] = s_base + ex;
+}
+
+// Device-wide exclusive scan of u64 values, single pass (decoupled look-back).
+__global__ void __launch_bounds__(kThreads) k_scan_exclusive_u64(const uint64_t* __restrict__ in,
+        uint64_t* __restrict__ out, uint64_t n, uint64_t* __restrict__ status, unsigned int* __restrict__ ctr) {
+    __shared__ uint32_t s_tile;
+    __shared__ uint64_t s_scan[kThreads / 32 + 1];
+    __shared__ uint64_t s_base;
+    if (threadIdx.x == 0) s_tile = atomicAdd(ctr, 1u);
+    __syncthreads();
+    const uint32_t tile = s_tile;
+    const uint64_t i0 = (uint64_t)tile * kTile + (uint64_t)threadIdx.x * kItems;
+    uint64_t v[kItems], sum = 0;
+#pragma unroll
+    for (int j = 0; j < kItems; ++j) { v[j] = (i0 + j < n) ? in[i0 + j] : 0; sum += v[j]; }
+    uint64_t tot, ex = block_exclusive_scan<kThreads>(sum, s_scan, &tot);
+    if (threadIdx.x < 32) {
+        uint64_t b = lookback_warp(status, tile, tot);
+        if (lane_id() == 0) s_base = b;
+    }
+    __syncthreads();
+    uint64_t run = s_base + ex;
+#pragma unroll
+    for (int j = 0; j < kItems; ++j) {
+        if (i0 + j < n) out[i0 + j] = run;
+        run += v[j];
+    }
+}
+
+// Lean merge for the identity-ID-map mode (no node ops in the batch): within a
+// tile the output index of old element i is  base + i - D(i) + I(i)  with
+// D(i) = #deleted elements before i and I(i) = #inserted records at positions
+// <= i (both from short sorted lists in shared memory).  Each warp iteration
+// covers 32 consecutive elements; when no edit falls inside them the chunk is a
+// plain shifted copy, otherwise each lane ranks itself in the two lists.
+template <bool UNUSED = false>
+__global__ void __launch_bounds__(kThreads) k_merge_plain(MergeArgs a, const TilePart* __restrict__ part) {
+    __shared__ __align__(128) uint32_t s_col[2][kMergeBuf];
+    __shared__ __align__(128) float s_w[2][kMergeBuf];
+    __shared__ uint16_t s_del[kMergeTile];      // local positions of deleted elements (sorted)
+    __shared__ uint16_t s_ins[kMergeTile + 1];  // local insertion positions of inserted records (sorted)
+    __shared__ __align__(8) uint64_t s_bar[2];
+    __shared__ uint64_t s_meta[2][5];          // r0, r1, dl0, ul0, (nd | nu << 16) of the staged tile
 
     const int tid = threadIdx.x;
-    if (tid == 0) s_tile = CASC ? atomicAdd(&a.c->tiles[5], 1u) : blockIdx.x;
-    __syncthreads();
-    const uint64_t tile = s_tile;
+    const uint32_t lane = lane_id();
     const uint64_t Dtot = a.E_old + a.n_ins;
-    const uint64_t d0 = tile * kMergeTile;
-    const uint64_t d1 = min(d0 + (uint64_t)kMergeTile, Dtot);
-    if (tid < 2) {
-        uint64_t d = tid == 0 ? d0 : d1;
-        s_r[tid] = (d == Dtot) ? a.n_ins : ins_split(a.ins_pos, a.n_ins, d);
-    }
+    if (tid == 0) { mbar_init(&s_bar[0], 1); mbar_init(&s_bar[1], 1); fence_mbar_init(); }
     __syncthreads();
-    const uint64_t r0 = s_r[0], r1 = s_r[1];
-    const uint64_t j0 = d0 - r0, j1 = d1 - r1;
-    const uint32_t n_old = (uint32_t)(j1 - j0), n_new = (uint32_t)(r1 - r0), n_tot = n_old + n_new;
-    if (tid < 2) {
-        uint64_t j = tid == 0 ? j0 : j1;
-        s_d[tid] = lower_bound_dev(a.del_pos, 0, a.n_del, j);
-        s_u[tid] = lower_bound_dev(a.upd_pos, 0, a.n_upd, j);
-    }
-    if (CASC && tid >= 32 && tid < 34) {
-        // hd rows whose row range [off[k], off[k+1]) intersects [j0, j1)
-        const int which = tid - 32;
-        uint64_t lo = 0, hi = a.n_hd;
-        if (which == 0) {  // first hd row with end > j0
-            while (lo < hi) { uint64_t mid = (lo + hi) >> 1; if ((uint64_t)a.old_off[a.hd_rows[mid] + 1] <= j0) lo = mid + 1; else hi = mid; }
-        } else {           // first hd row with start >= j1
-            while (lo < hi) { uint64_t mid = (lo + hi) >> 1; if ((uint64_t)a.old_off[a.hd_rows[mid]] < j1) lo = mid + 1; else hi = mid; }
+    auto issue = [&](uint64_t t, int b) {  // one thread: tile metadata + TMA of its old elements
+        const TilePart p0 = part[t], p1 = part[t + 1];
+        s_meta[b][0] = p0.r; s_meta[b][1] = p1.r; s_meta[b][2] = p0.dl; s_meta[b][3] = p0.ul;
+        s_meta[b][4] = (p1.dl - p0.dl) | ((p1.ul - p0.ul) << 16);  // both <= 2048
+        const uint64_t j0 = min(t * kMergeTile, Dtot) - p0.r, j1 = min((t + 1) * kMergeTile, Dtot) - p1.r;
+        const uint64_t a0 = j0 & ~3ull, a1 = (j1 + 3) & ~3ull;
+        const uint32_t bytes = (uint32_t)((a1 - a0) * 4);
+        mbar_expect_tx(&s_bar[b], 2 * bytes);
+        if (bytes) {
+            bulk_g2s(&s_col[b][0], a.old_cols + a0, bytes, &s_bar[b]);
+            bulk_g2s(&s_w[b][0], a.old_w + a0, bytes, &s_bar[b]);
         }
-        s_h[which] = lo;
-    }
-    // stage old elements [j0, j1) (aligned 16 B chunks; buffers are padded)
-    const uint64_t a0 = j0 & ~3ull;
-    {
-        const uint64_t c0 = a0 >> 2, c1 = (j1 + 3) >> 2;
-        const uint4* gc = reinterpret_cast<const uint4*>(a.old_cols);
-        const uint4* gw = reinterpret_cast<const uint4*>(a.old_w);
-        for (uint64_t q = c0 + tid; q < c1; q += kThreads) {
-            uint4 vc = gc[q], vw = gw[q];
-            uint32_t o = (uint32_t)((q << 2) - a0);
-            *reinterpret_cast<uint4*>(&s_col[o]) = vc;
-            *reinterpret_cast<uint4*>(&s_w[o]) = vw;
-        }
-    }
-    for (uint32_t i = tid; i < kMergeTile; i += kThreads) { s_keep[i] = 1; s_slot[i] = 0; }
+    };
+    uint64_t t = blockIdx.x;
+    if (t < a.n_tiles && tid == 0) issue(t, 0);
     __syncthreads();
-    const uint32_t sh = (uint32_t)(j0 - a0);
-    // deletes and weight overrides (sorted old positions in [j0, j1))
-    for (uint64_t i = s_d[0] + tid; i < s_d[1]; i += kThreads) s_keep[a.del_pos[i] - j0] = 0;
-    for (uint64_t i = s_u[0] + tid; i < s_u[1]; i += kThreads) s_w[a.upd_pos[i] - a0] = a.upd_w[i];
-    if (CASC) {
-        for (uint64_t h = s_h[0]; h < s_h[1]; ++h) {
-            uint32_t k = a.hd_rows[h];
-            uint64_t b = max((uint64_t)a.old_off[k], j0), e = min((uint64_t)a.old_off[k + 1], j1);
-            for (uint64_t x = b + tid; x < e; x += kThreads) s_keep[x - j0] = 0;
-        }
-    }
-    for (uint32_t s = tid; s < n_new; s += kThreads) {
-        uint64_t m = (a.ins_pos[r0 + s] - j0) + s;
-        s_slot[m] = 0x80000000u | s;
-    }
-    __syncthreads();
-    if (CASC) {
-        for (uint32_t i = tid; i < n_old; i += kThreads) {
-            if (s_keep[i]) {
-                uint32_t col = s_col[i + sh];
-                if (a.hd_bits[col >> 5] >> (col & 31) & 1) s_keep[i] = 0;
-            }
-        }
+    for (uint32_t it = 0; t < a.n_tiles; t += gridDim.x, ++it) {
+        const int b = it & 1;
+        const uint64_t r0 = s_meta[b][0], r1 = s_meta[b][1], dl0 = s_meta[b][2], ul0 = s_meta[b][3];
+        const uint32_t nd = (uint32_t)(s_meta[b][4] & 0xFFFF), nu = (uint32_t)(s_meta[b][4] >> 16);
+        const uint64_t d0 = min(t * kMergeTile, Dtot), d1 = min((t + 1) * kMergeTile, Dtot);
+        const uint64_t j0 = d0 - r0, j1 = d1 - r1;
+        const uint32_t n_old = (uint32_t)(j1 - j0), ni = (uint32_t)(r1 - r0);
+        const uint32_t sh = (uint32_t)(j0 & 3);
+        if (tid == 0 && t + gridDim.x < a.n_tiles) { fence_proxy_async(); issue(t + gridDim.x, b ^ 1); }
+        for (uint32_t i = tid; i < nd; i += kThreads) s_del[i] = (uint16_t)(a.del_pos[dl0 + i] - j0);
+        for (uint32_t s = tid; s < ni; s += kThreads) s_ins[s] = (uint16_t)(a.ins_pos[r0 + s] - j0);
+        mbar_wait(&s_bar[b], (it >> 1) & 1);
+        for (uint32_t i = tid; i < nu; i += kThreads) s_w[b][a.upd_pos[ul0 + i] - (j0 & ~3ull)] = a.upd_w[ul0 + i];
         __syncthreads();
-    }
-    // blocked pass over merged slots: old-element index, emit flag, output index
-    const uint32_t m0 = tid * kMergeItems;
-    uint32_t slot[kMergeItems];
-    uint64_t n_oldc = 0;
-#pragma unroll
-    for (int j = 0; j < kMergeItems; ++j) {
-        uint32_t m = m0 + j;
-        slot[j] = (m < n_tot) ? s_slot[m] : 0xFFFFFFFFu;
-        if (m < n_tot && !(slot[j] & 0x80000000u)) n_oldc++;
-    }
-    uint64_t tot_old, oi0 = block_exclusive_scan<kThreads>(n_oldc, s_scan, &tot_old);
-    uint32_t oi[kMergeItems];
-    uint64_t n_emit = 0;
-    {
-        uint32_t o = (uint32_t)oi0;
-#pragma unroll
-        for (int j = 0; j < kMergeItems; ++j) {
-            uint32_t m = m0 + j;
-            oi[j] = o;
-            if (m < n_tot) {
-                if (slot[j] & 0x80000000u) n_emit++;
-                else { n_emit += s_keep[o]; ++o; }
-            }
-        }
-    }
-    uint64_t tot_emit, e0 = block_exclusive_scan<kThreads>(n_emit, s_scan, &tot_emit);
-    if (CASC) {
-        if (tid < 32) {
-            uint64_t b = lookback_warp(a.status, (uint32_t)tile, tot_emit);
-            if (lane_id() == 0) s_base = b;
-        }
-    } else if (tid == 0) {
-        s_base = j0 - s_d[0] + r0;  // kept old elements before j0 + inserted records before d0
-    }
-    // stage the output chunk in merged order
-    {
-        uint32_t e = (uint32_t)e0;
-#pragma unroll
-        for (int j = 0; j < kMergeItems; ++j) {
-            uint32_t m = m0 + j;
-            if (m >= n_tot) break;
-            if (slot[j] & 0x80000000u) {
-                uint32_t s = slot[j] & 0x7FFFFFFFu;
-                s_oc[e] = a.ins_col[r0 + s];
-                s_ow[e] = a.ins_w[r0 + s];
-                ++e;
-            } else {
-                uint32_t o = oi[j];
-                if (CASC) s_kp[o] = e - (m - o);
-                if (s_keep[o]) {
-                    uint32_t col = s_col[o + sh];
-                    s_oc[e] = REMAP ? a.remap[col] : col;
-                    s_ow[e] = s_w[o + sh];
-                    ++e;
+        const uint64_t base = j0 - dl0 + r0;
+        uint32_t* __restrict__ oc = a.new_cols + base;
+        float* __restrict__ ow = a.new_w + base;
+        // old elements
+        for (uint32_t c0 = (tid & ~31u); c0 < n_old; c0 += kThreads) {
+            const uint32_t i = c0 + lane;
+            // ranks at the chunk start (identical in all lanes)
+            const uint32_t D0 = (uint32_t)lower_bound_dev(s_del, 0, nd, (uint16_t)c0);
+            const uint32_t I0 = (uint32_t)upper_bound_dev(s_ins, 0, ni, (uint16_t)c0);
+            const bool clean = (D0 == nd || s_del[D0] >= c0 + 32) && (I0 == ni || s_ins[I0] >= c0 + 32);
+            if (i < n_old) {
+                uint32_t o;
+                bool keep = true;
+                if (clean) o = i - D0 + I0;
+                else {
+                    const uint32_t Di = (uint32_t)lower_bound_dev(s_del, D0, nd, (uint16_t)i);
+                    const uint32_t Ii = (uint32_t)upper_bound_dev(s_ins, I0, ni, (uint16_t)i);
+                    keep = !(Di < nd && s_del[Di] == i);
+                    o = i - Di + Ii;
                 }
+                if (keep) { oc[o] = s_col[b][i + sh]; ow[o] = s_w[b][i + sh]; }
             }
         }
-        if (CASC && tid == 0) s_kp[n_old] = (uint32_t)(tot_emit - n_new);
-    }
-    __syncthreads();
-    const uint64_t base = s_base;
-    const uint32_t cnt = (uint32_t)tot_emit;
-    // coalesced store: scalar head to a 16 B boundary, 128-bit body, scalar tail
-    {
-        uint32_t head = (uint32_t)((4 - (base & 3)) & 3);
-        if (head > cnt) head = cnt;
-        if (tid < head) { a.new_cols[base + tid] = s_oc[tid]; a.new_w[base + tid] = s_ow[tid]; }
-        const uint32_t body = (cnt - head) >> 2;
-        uint4* gc = reinterpret_cast<uint4*>(a.new_cols + base + head);
-        uint4* gw = reinterpret_cast<uint4*>(a.new_w + base + head);
-        for (uint32_t q = tid; q < body; q += kThreads) {
-            uint32_t s = head + (q << 2);
-            gc[q] = make_uint4(s_oc[s], s_oc[s + 1], s_oc[s + 2], s_oc[s + 3]);
-            gw[q] = make_uint4(__float_as_uint(s_ow[s]), __float_as_uint(s_ow[s + 1]),
-                               __float_as_uint(s_ow[s + 2]), __float_as_uint(s_ow[s + 3]));
-        }
-        for (uint32_t s = head + (body << 2) + tid; s < cnt; s += kThreads) {
-            a.new_cols[base + s] = s_oc[s];
-            a.new_w[base + s] = s_ow[s];
-        }
-    }
-    if (CASC) {
-        // kept-before at every old row that starts inside this tile (last tile: also at E)
-        const bool last = (tile == a.n_tiles - 1);
-        __shared__ uint64_t s_k[2];
-        if (tid < 2) {
-            if (tid == 0) s_k[0] = lower_bound_dev(a.old_off, 0, a.V_old + 1, (int64_t)j0);
-            else s_k[1] = last ? a.V_old + 1 : lower_bound_dev(a.old_off, 0, a.V_old + 1, (int64_t)j1);
+        // inserted records: local pos p precedes old element p
+        for (uint32_t s = tid; s < ni; s += kThreads) {
+            const uint32_t p = s_ins[s];
+            const uint32_t o = p - (uint32_t)lower_bound_dev(s_del, 0, nd, (uint16_t)p) + s;
+            oc[o] = a.ins_col[r0 + s];
+            ow[o] = a.ins_w[r0 + s];
         }
         __syncthreads();
-        const uint64_t kept_before = base - r0;
-        for (uint64_t k = s_k[0] + tid; k < s_k[1]; k += kThreads)
-            a.KR[k] = (int64_t)(kept_before + s_kp[(uint64_t)a.old_off[k] - j0]);
-        if (tid == 0) {
-            uint64_t casc = (uint64_t)n_old - (tot_emit - n_new) - (s_d[1] - s_d[0]);
-            if (casc) atomicAdd(&a.c->n_casc, (unsigned long long)casc);
-        }
     }
+}
+
+// per 1024-block of old ids: constant new-id shift, or kRemapMixed if a dropped
+// id or an inserted id's insertion point lies strictly inside the block
+__global__ void k_remap_blocks(uint64_t V, const uint32_t* __restrict__ dropped, uint64_t n_dropped,
+                               const uint32_t* __restrict__ ins_oldpos, uint64_t n_ins, int32_t* __restrict__ shift) {
+    uint64_t bk = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x;
+    uint64_t nb = (V + (1u << kRemapBlockShift) - 1) >> kRemapBlockShift;
+    if (bk >= nb) return;
+    uint64_t lo = bk << kRemapBlockShift, hi = min(lo + (1u << kRemapBlockShift), V);
+    uint64_t d0 = lower_bound_dev(dropped, 0, n_dropped, (uint32_t)lo);
+    uint64_t d1 = lower_bound_dev(dropped, d0, n_dropped, (uint32_t)hi);
+    uint64_t i0 = upper_bound_dev(ins_oldpos, 0, n_ins, (uint32_t)lo);      // oldpos <= lo
+    uint64_t i1 = upper_bound_dev(ins_oldpos, i0, n_ins, (uint32_t)(hi - 1));  // oldpos <= hi-1
+    shift[bk] = (d1 > d0 || i1 > i0) ? kRemapMixed : (int32_t)((int64_t)i0 - (int64_t)d0);
 }
 
 // ============================================================== a4 + a5 ====
@@ -826,30 +1123,210 @@ __global__ void __launch_bounds__(kThreads) k_merge(MergeArgs a) {
 //   (kept old elements before row u's old start) + (inserted records in rows < u')
 // where both terms are ranks in sorted lists (no cascade) or the kept-before
 // table KR written by the merge's decoupled look-back (cascade).
+constexpr int kOffTile = 4096;  // old rows per CTA of the offsets kernel
+
+// new dense id of the first surviving old row >= k (REMAP: compaction formula)
+__device__ __forceinline__ uint64_t new_id_at(uint64_t k, const uint32_t* dropped, uint64_t n_dropped,
+                                              const uint32_t* ins_oldpos, uint64_t n_vins) {
+    return k - lower_bound_dev(dropped, 0, n_dropped, (uint32_t)k) +
+           upper_bound_dev(ins_oldpos, 0, n_vins, (uint32_t)k);
+}
+
+struct OffArgs {
+    const int64_t* old_off;
+    uint64_t V_old;
+    const int64_t* KR;
+    const uint64_t* del_pos;
+    uint64_t n_del;
+    const uint32_t* ins_row;
+    uint64_t n_ins;
+    const uint32_t* remap;
+    const uint32_t* dropped;
+    uint64_t n_dropped;
+    const uint32_t* ins_oldpos;
+    uint64_t n_vins;
+    int64_t* new_off;
+    uint64_t* part;  // [n_cta + 1][2]: ins-row rank, delete rank at each CTA boundary
+};
+
+template <bool REMAP>
+__global__ void k_offsets_partition(OffArgs a) {
+    uint64_t b = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x;
+    uint64_t nb = (a.V_old + kOffTile - 1) / kOffTile;
+    if (b > nb) return;
+    uint64_t k = min(b * kOffTile, a.V_old);
+    uint64_t ir, dr;
+    if (k == a.V_old) { ir = a.n_ins; dr = a.n_del; }
+    else {
+        uint64_t u = REMAP ? new_id_at(k, a.dropped, a.n_dropped, a.ins_oldpos, a.n_vins) : k;
+        ir = lower_bound_dev(a.ins_row, 0, a.n_ins, (uint32_t)u);
+        dr = lower_bound_dev(a.del_pos, 0, a.n_del, (uint64_t)a.old_off[k]);
+    }
+    a.part[2 * b] = ir;
+    a.part[2 * b + 1] = dr;
+}
+
+// new_off[u'] = (kept old elements before old row k) + (inserted records in rows < u')
+// The CTA's slices of the sorted insert-row and delete-position lists are staged
+// in shared memory; each thread then answers its rank queries there.
+constexpr int kOffStageIns = 4096, kOffStageDel = 2048;
 template <bool CASC, bool REMAP>
-__global__ void __launch_bounds__(kThreads) k_offsets_old(
-    const int64_t* __restrict__ old_off, uint64_t V_old, const int64_t* __restrict__ KR,
-    const uint64_t* __restrict__ del_pos, uint64_t n_del, const uint32_t* __restrict__ ins_row, uint64_t n_ins,
-    const uint32_t* __restrict__ remap, int64_t* __restrict__ new_off) {
-    uint64_t k0 = ((uint64_t)blockIdx.x * kThreads + threadIdx.x) * kItems;
-    if (k0 >= V_old) return;
-    uint64_t dp = 0, ip = 0;
-    bool first = true;
-    for (int j = 0; j < kItems; ++j) {
-        uint64_t k = k0 + j;
-        if (k >= V_old) break;
-        uint32_t u = REMAP ? remap[k] : (uint32_t)k;
-        if (u == kNone32) continue;
-        int64_t kept;
-        if (CASC) kept = KR[k];
-        else {
-            uint64_t x = (uint64_t)old_off[k];
-            dp = first ? lower_bound_dev(del_pos, 0, n_del, x) : gallop_lb(del_pos, dp, n_del, x);
-            kept = (int64_t)(x - dp);
+__global__ void __launch_bounds__(kThreads) k_offsets_old(OffArgs a) {
+    __shared__ uint32_t s_ins[kOffStageIns];
+    __shared__ uint64_t s_del[CASC ? 1 : kOffStageDel];
+    const uint64_t cta = blockIdx.x;
+    const uint64_t ia = a.part[2 * cta], ib = a.part[2 * cta + 2];
+    const uint64_t da = a.part[2 * cta + 1], db = a.part[2 * cta + 3];
+    const uint64_t ni = ib - ia, nd = db - da;
+    const bool stage_i = ni <= kOffStageIns, stage_d = !CASC && nd <= kOffStageDel;
+    if (stage_i) for (uint64_t i = threadIdx.x; i < ni; i += kThreads) s_ins[i] = a.ins_row[ia + i];
+    if (stage_d) for (uint64_t i = threadIdx.x; i < nd; i += kThreads) s_del[i] = a.del_pos[da + i];
+    constexpr int PER = kOffTile / kThreads;
+    const uint64_t k0 = cta * kOffTile + threadIdx.x;
+    uint32_t u[PER];
+    int64_t x[PER];
+#pragma unroll
+    for (int j = 0; j < PER; ++j) {
+        uint64_t k = k0 + (uint64_t)j * kThreads;
+        u[j] = kNone32;
+        if (k < a.V_old) {
+            u[j] = REMAP ? a.remap[k] : (uint32_t)k;
+            x[j] = CASC ? a.KR[k] : a.old_off[k];
         }
-        ip = first ? lower_bound_dev(ins_row, 0, n_ins, u) : gallop_lb(ins_row, ip, n_ins, u);
-        first = false;
-        new_off[u] = kept + (int64_t)ip;
+    }
+    __syncthreads();
+#pragma unroll
+    for (int j = 0; j < PER; ++j) {
+        if (u[j] == kNone32) continue;
+        int64_t kept = x[j];
+        if (!CASC) {
+            uint64_t r = stage_d ? da + lower_bound_dev(s_del, 0, nd, (uint64_t)x[j])
+                                 : lower_bound_dev(a.del_pos, da, db, (uint64_t)x[j]);
+            kept -= (int64_t)r;
+        }
+        uint64_t ir = stage_i ? ia + lower_bound_dev(s_ins, 0, ni, u[j]) : lower_bound_dev(a.ins_row, ia, ib, u[j]);
+        a.new_off[u[j]] = kept + (int64_t)ir;
+    }
+}
+
+// Mode without node ops (identity ID map): the per-vertex degree delta
+// deg[u] = (#inserted records in row u) - (#deleted old edges in row u) is
+// scattered from the two sorted record lists, then one single-pass exclusive
+// scan (decoupled look-back) writes new_off[u] = old_off[u] + sum_{v<u} deg[v].
+__global__ void k_deg_scatter(const uint32_t* __restrict__ ins_row, uint64_t n_ins,
+                              const uint32_t* __restrict__ del_row, uint64_t n_del, int32_t* __restrict__ deg,
+                              int64_t* __restrict__ tsum) {
+    uint64_t i = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x;
+    const bool ok = i < n_ins + n_del;
+    const bool is_ins = i < n_ins;
+    const uint32_t r = ok ? (is_ins ? ins_row[i] : del_row[i - n_ins]) : 0;
+    // warp-aggregated: one atomic per (row, sign) group of the warp (hub rows get many records)
+    const uint64_t key = ok ? (((uint64_t)r << 1) | (is_ins ? 1u : 0u)) : ~0ull;
+    const uint32_t peers = __match_any_sync(0xffffffffu, key);
+    if (ok && lane_id() == (uint32_t)(__ffs(peers) - 1)) {
+        const int v = is_ins ? __popc(peers) : -__popc(peers);
+        atomicAdd(&deg[r], v);
+        atomicAdd(reinterpret_cast<unsigned long long*>(&tsum[r / kTile]), (unsigned long long)(int64_t)v);
+    }
+}
+
+// exclusive scan in place of the per-tile degree-delta sums (one CTA; nt <= ~1M)
+__global__ void __launch_bounds__(1024) k_tile_sum_scan(int64_t* __restrict__ tsum, uint64_t nt) {
+    __shared__ int64_t s_scan[1024 / 32 + 1];
+    __shared__ int64_t s_carry;
+    if (threadIdx.x == 0) s_carry = 0;
+    __syncthreads();
+    constexpr int PER = 8;
+    for (uint64_t c0 = 0; c0 < nt; c0 += 1024 * PER) {
+        const uint64_t i0 = c0 + (uint64_t)threadIdx.x * PER;
+        int64_t v[PER], sum = 0;
+#pragma unroll
+        for (int j = 0; j < PER; ++j) { v[j] = (i0 + j < nt) ? tsum[i0 + j] : 0; sum += v[j]; }
+        int64_t tot, ex = block_exclusive_scan<1024>(sum, s_scan, &tot);
+        int64_t run = s_carry + ex;
+#pragma unroll
+        for (int j = 0; j < PER; ++j) { if (i0 + j < nt) tsum[i0 + j] = run; run += v[j]; }
+        __syncthreads();
+        if (threadIdx.x == 0) s_carry += tot;
+        __syncthreads();
+    }
+}
+
+// new_off[u] = old_off[u] + (tile base) + (exclusive prefix of deg inside the tile)
+__global__ void __launch_bounds__(kThreads) k_offsets_apply(const int64_t* __restrict__ old_off,
+        const int32_t* __restrict__ deg, uint64_t V, const int64_t* __restrict__ tbase, int64_t* __restrict__ new_off) {
+    __shared__ int64_t s_scan[kThreads / 32 + 1];
+    const uint64_t i0 = (uint64_t)blockIdx.x * kTile + (uint64_t)threadIdx.x * kItems;
+    int32_t d[kItems];
+    int64_t oo[kItems];
+    int64_t sum = 0;
+    if (i0 + kItems <= V) {
+        const int4* p = reinterpret_cast<const int4*>(deg + i0);
+        int4 a = p[0], b = p[1];
+        d[0] = a.x; d[1] = a.y; d[2] = a.z; d[3] = a.w; d[4] = b.x; d[5] = b.y; d[6] = b.z; d[7] = b.w;
+        const longlong2* q = reinterpret_cast<const longlong2*>(old_off + i0);
+#pragma unroll
+        for (int j = 0; j < kItems / 2; ++j) { longlong2 v = q[j]; oo[2 * j] = v.x; oo[2 * j + 1] = v.y; }
+    } else {
+#pragma unroll
+        for (int j = 0; j < kItems; ++j) { d[j] = (i0 + j < V) ? deg[i0 + j] : 0; oo[j] = (i0 + j < V) ? old_off[i0 + j] : 0; }
+    }
+#pragma unroll
+    for (int j = 0; j < kItems; ++j) sum += d[j];
+    int64_t tot, ex = block_exclusive_scan<kThreads>(sum, s_scan, &tot);
+    int64_t run = tbase[blockIdx.x] + ex;
+    int64_t o[kItems];
+#pragma unroll
+    for (int j = 0; j < kItems; ++j) { o[j] = oo[j] + run; run += d[j]; }
+    if (i0 + kItems <= V) {
+        longlong2* q = reinterpret_cast<longlong2*>(new_off + i0);
+#pragma unroll
+        for (int j = 0; j < kItems / 2; ++j) q[j] = make_longlong2(o[2 * j], o[2 * j + 1]);
+    } else {
+#pragma unroll
+        for (int j = 0; j < kItems; ++j) if (i0 + j < V) new_off[i0 + j] = o[j];
+    }
+}
+
+__global__ void __launch_bounds__(kThreads) k_offsets_scan(const int64_t* __restrict__ old_off, const int32_t* __restrict__ deg,
+        uint64_t V, int64_t* __restrict__ new_off, uint64_t* __restrict__ status, unsigned int* __restrict__ ctr) {
+    __shared__ uint32_t s_tile;
+    __shared__ int64_t s_scan[kThreads / 32 + 1];
+    __shared__ int64_t s_base;
+    if (threadIdx.x == 0) s_tile = atomicAdd(ctr, 1u);
+    __syncthreads();
+    const uint32_t tile = s_tile;
+    const uint64_t i0 = (uint64_t)tile * kTile + (uint64_t)threadIdx.x * kItems;  // blocked: 8 rows per thread
+    int32_t d[kItems];
+    int64_t oo[kItems];  // old offsets, loaded before the look-back so the loads overlap it
+    int64_t sum = 0;
+    if (i0 + kItems <= V) {
+        const int4* p = reinterpret_cast<const int4*>(deg + i0);
+        int4 a = p[0], b = p[1];
+        d[0] = a.x; d[1] = a.y; d[2] = a.z; d[3] = a.w; d[4] = b.x; d[5] = b.y; d[6] = b.z; d[7] = b.w;
+        const longlong2* q = reinterpret_cast<const longlong2*>(old_off + i0);
+#pragma unroll
+        for (int j = 0; j < kItems / 2; ++j) { longlong2 v = q[j]; oo[2 * j] = v.x; oo[2 * j + 1] = v.y; }
+    } else {
+#pragma unroll
+        for (int j = 0; j < kItems; ++j) { d[j] = (i0 + j < V) ? deg[i0 + j] : 0; oo[j] = (i0 + j < V) ? old_off[i0 + j] : 0; }
+    }
+#pragma unroll
+    for (int j = 0; j < kItems; ++j) sum += d[j];
+    int64_t tot, ex = block_exclusive_scan<kThreads>(sum, s_scan, &tot);
+    if (threadIdx.x < 32) {
+        // look-back values must be non-negative: bias each tile aggregate by +kTile*2^31
+        const uint64_t bias = (uint64_t)kTile << 31;
+        uint64_t b = lookback_warp(status, tile, (uint64_t)(tot + (int64_t)bias));
+        if (lane_id() == 0) s_base = (int64_t)(b - (uint64_t)tile * bias);
+    }
+    __syncthreads();
+    int64_t run = s_base + ex;
+#pragma unroll
+    for (int j = 0; j < kItems; ++j) {
+        uint64_t u = i0 + j;
+        if (u < V) new_off[u] = oo[j] + run;
+        run += d[j];
     }
 }
 
@@ -872,6 +1349,7 @@ __global__ void k_offsets_inserted(const NodeVtx* __restrict__ nv, const uint32_
 }
 
 __global__ void k_set_i64(int64_t* p, int64_t v) { *p = v; }
+__global__ void k_copy_u64(unsigned long long* dst, const uint64_t* src) { *dst = *src; }
 
 // ================================================================ checks ====
 template <typename T>

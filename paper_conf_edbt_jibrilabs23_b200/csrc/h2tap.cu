@@ -546,14 +546,15 @@ h2tap_status apply_core(h2tap_replica* r, const BatchIn& in, uint64_t S, bool cr
         }
         auto launch = [&](auto kern) {
             int occ = 0;
-            CK(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, kern, kThreads, 0));
+            CK(cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, kMerge3Smem));
+            CK(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, kern, kThreads, kMerge3Smem));
             const uint64_t grid = std::min<uint64_t>(ma.n_tiles, (uint64_t)std::max(1, occ) * r->n_sm);
-            kern<<<(unsigned)grid, kThreads, 0, st>>>(ma, part);
+            kern<<<(unsigned)grid, kThreads, kMerge3Smem, st>>>(ma, part);
         };
-        if (casc && remap_on) launch(k_merge<true, true>);
-        else if (casc) launch(k_merge<true, false>);
-        else if (remap_on) launch(k_merge<false, true>);
-        else launch(k_merge<false, false>);
+        if (casc && remap_on) launch(k_merge3<true, true>);
+        else if (casc) launch(k_merge3<true, false>);
+        else if (remap_on) launch(k_merge3<false, true>);
+        else launch(k_merge3<false, false>);
         CKL();
     } else if (casc) {
         CK(cudaStreamWaitEvent(st, r->evB, 0));

@@ -1018,30 +1018,53 @@ __global__ void __launch_bounds__(kThreads) k_scan_exclusive_u64(const uint64_t*
     }
 }
 
-// Lean merge for the identity-ID-map mode (no node ops in the batch): within a
-// tile the output index of old element i is  base + i - D(i) + I(i)  with
-// D(i) = #deleted elements before i and I(i) = #inserted records at positions
-// <= i (both from short sorted lists in shared memory).  Each warp iteration
-// covers 32 consecutive elements; when no edit falls inside them the chunk is a
-// plain shifted copy, otherwise each lane ranks itself in the two lists.
-template <bool UNUSED = false>
-__global__ void __launch_bounds__(kThreads) k_merge_plain(MergeArgs a, const TilePart* __restrict__ part) {
-    __shared__ __align__(128) uint32_t s_col[2][kMergeBuf];
-    __shared__ __align__(128) float s_w[2][kMergeBuf];
-    __shared__ uint16_t s_del[kMergeTile];      // local positions of deleted elements (sorted)
-    __shared__ uint16_t s_ins[kMergeTile + 1];  // local insertion positions of inserted records (sorted)
-    __shared__ __align__(8) uint64_t s_bar[2];
-    __shared__ uint64_t s_meta[2][5];          // r0, r1, dl0, ul0, (nd | nu << 16) of the staged tile
+constexpr int kMerge3Smem = 6 * kMergeBuf * 4;  // dynamic shared memory of k_merge3
 
-    const int tid = threadIdx.x;
-    const uint32_t lane = lane_id();
+// ---- TMA bulk store (smem -> global) helpers
+__device__ __forceinline__ void bulk_s2g(void* dst, const void* src, uint32_t bytes) {
+    asm volatile("cp.async.bulk.global.shared::cta.bulk_group [%0], [%1], %2;"
+                 ::"l"(dst), "r"(smem_u32(src)), "r"(bytes) : "memory");
+}
+__device__ __forceinline__ void bulk_commit() { asm volatile("cp.async.bulk.commit_group;" ::: "memory"); }
+__device__ __forceinline__ void bulk_wait_read0() { asm volatile("cp.async.bulk.wait_group.read 0;" ::: "memory"); }
+__device__ __forceinline__ void bulk_wait_all() { asm volatile("cp.async.bulk.wait_group 0;" ::: "memory"); }
+
+// Merge v3.  Tile t covers merged items [t*2048, (t+1)*2048): old elements
+// [j0, j1) (TMA-staged, double-buffered) and inserted records [r0, r1).
+//   phase A (per 32-element chunk): keep-ballot (not deleted, not cascaded)
+//   scan of the 64 chunk counts -> kept-before at any element (smem masks)
+//   phase B: output index e = kept_before(i) + I(i), I(i) = inserted records at
+//            local positions <= i (uniform per chunk unless one falls inside);
+//            values (remapped column, weight) staged in smem at e + (base & 3)
+//   inserted records: e = kept_before(p) + s
+//   store: scalar head/tail, one TMA bulk store per array for the aligned body
+template <bool CASC, bool REMAP>
+__global__ void __launch_bounds__(kThreads) k_merge3(MergeArgs a, const TilePart* __restrict__ part) {
+    constexpr int NCH = kMergeTile / 32;  // 64 chunks of 32 old elements
+    extern __shared__ __align__(128) uint8_t dsm[];  // kMerge3Smem bytes
+    auto s_col = reinterpret_cast<uint32_t(*)[kMergeBuf]>(dsm);
+    auto s_w = reinterpret_cast<float(*)[kMergeBuf]>(dsm + 2 * kMergeBuf * 4);
+    uint32_t* s_oc = reinterpret_cast<uint32_t*>(dsm + 4 * kMergeBuf * 4);
+    float* s_ow = reinterpret_cast<float*>(dsm + 5 * kMergeBuf * 4);
+    __shared__ uint16_t s_ins[kMergeTile + 1];
+    __shared__ uint32_t s_dmask[NCH + 2];   // deleted old elements, per chunk
+    __shared__ uint32_t s_icnt[NCH + 2];    // inserted records per chunk of insertion positions
+    __shared__ uint32_t s_mask[NCH + 1];    // kept old elements, per chunk
+    __shared__ uint32_t s_cbase[NCH + 1];   // kept before each chunk
+    __shared__ uint32_t s_ibase[NCH + 2];   // inserted records at positions before each chunk
+    __shared__ __align__(8) uint64_t s_bar[2];
+    __shared__ uint64_t s_meta[2][5];
+    __shared__ uint64_t s_cbefore;
+
+    const int tid = threadIdx.x, wid = tid >> 5;
+    const uint32_t lane = lane_id(), lt = lanemask_lt();
     const uint64_t Dtot = a.E_old + a.n_ins;
     if (tid == 0) { mbar_init(&s_bar[0], 1); mbar_init(&s_bar[1], 1); fence_mbar_init(); }
     __syncthreads();
     auto issue = [&](uint64_t t, int b) {  // one thread: tile metadata + TMA of its old elements
         const TilePart p0 = part[t], p1 = part[t + 1];
         s_meta[b][0] = p0.r; s_meta[b][1] = p1.r; s_meta[b][2] = p0.dl; s_meta[b][3] = p0.ul;
-        s_meta[b][4] = (p1.dl - p0.dl) | ((p1.ul - p0.ul) << 16);  // both <= 2048
+        s_meta[b][4] = (p1.dl - p0.dl) | ((p1.ul - p0.ul) << 16) | (CASC ? (p0.k << 32) : 0);
         const uint64_t j0 = min(t * kMergeTile, Dtot) - p0.r, j1 = min((t + 1) * kMergeTile, Dtot) - p1.r;
         const uint64_t a0 = j0 & ~3ull, a1 = (j1 + 3) & ~3ull;
         const uint32_t bytes = (uint32_t)((a1 - a0) * 4);
@@ -1057,49 +1080,145 @@ __global__ void __launch_bounds__(kThreads) k_merge_plain(MergeArgs a, const Til
     for (uint32_t it = 0; t < a.n_tiles; t += gridDim.x, ++it) {
         const int b = it & 1;
         const uint64_t r0 = s_meta[b][0], r1 = s_meta[b][1], dl0 = s_meta[b][2], ul0 = s_meta[b][3];
-        const uint32_t nd = (uint32_t)(s_meta[b][4] & 0xFFFF), nu = (uint32_t)(s_meta[b][4] >> 16);
+        const uint32_t nd = (uint32_t)(s_meta[b][4] & 0xFFFF), nu = (uint32_t)((s_meta[b][4] >> 16) & 0xFFFF);
         const uint64_t d0 = min(t * kMergeTile, Dtot), d1 = min((t + 1) * kMergeTile, Dtot);
         const uint64_t j0 = d0 - r0, j1 = d1 - r1;
         const uint32_t n_old = (uint32_t)(j1 - j0), ni = (uint32_t)(r1 - r0);
         const uint32_t sh = (uint32_t)(j0 & 3);
         if (tid == 0 && t + gridDim.x < a.n_tiles) { fence_proxy_async(); issue(t + gridDim.x, b ^ 1); }
-        for (uint32_t i = tid; i < nd; i += kThreads) s_del[i] = (uint16_t)(a.del_pos[dl0 + i] - j0);
-        for (uint32_t s = tid; s < ni; s += kThreads) s_ins[s] = (uint16_t)(a.ins_pos[r0 + s] - j0);
-        mbar_wait(&s_bar[b], (it >> 1) & 1);
-        for (uint32_t i = tid; i < nu; i += kThreads) s_w[b][a.upd_pos[ul0 + i] - (j0 & ~3ull)] = a.upd_w[ul0 + i];
+        // the tile's edit lists: first kThreads entries of each list straight into registers,
+        // all loads in flight together (overflow entries are loaded in the loops below)
+        const uint64_t pf_del = tid < nd ? a.del_pos[dl0 + tid] : 0;
+        const uint64_t pf_ins = tid < ni ? a.ins_pos[r0 + tid] : 0;
+        const uint32_t pf_icol = tid < ni ? a.ins_col[r0 + tid] : 0;
+        const float pf_iw = tid < ni ? a.ins_w[r0 + tid] : 0.f;
+        const uint64_t pf_upd = tid < nu ? a.upd_pos[ul0 + tid] : 0;
+        const float pf_uw = tid < nu ? a.upd_w[ul0 + tid] : 0.f;
+        if (tid < NCH + 2) { s_dmask[tid] = 0; s_icnt[tid] = 0; }
+        if (CASC && wid == 1) {  // cascaded elements before j0 (block prefix + partial popcount)
+            const uint64_t blk = j0 / kCascBlock, wb = blk * (kCascBlock / 32), we = j0 >> 5;
+            uint32_t c = 0;
+            for (uint64_t q = wb + lane; q <= we; q += 32) {
+                uint32_t m = a.casc_mask[q];
+                if (q == we) m &= (j0 & 31) ? (0xFFFFFFFFu >> (32 - (j0 & 31))) : 0u;
+                c += __popc(m);
+            }
+            c = warp_sum(c);
+            if (lane == 0) s_cbefore = a.casc_pre[blk] + c;
+        }
         __syncthreads();
-        const uint64_t base = j0 - dl0 + r0;
-        uint32_t* __restrict__ oc = a.new_cols + base;
-        float* __restrict__ ow = a.new_w + base;
-        // old elements
-        for (uint32_t c0 = (tid & ~31u); c0 < n_old; c0 += kThreads) {
-            const uint32_t i = c0 + lane;
-            // ranks at the chunk start (identical in all lanes)
-            const uint32_t D0 = (uint32_t)lower_bound_dev(s_del, 0, nd, (uint16_t)c0);
-            const uint32_t I0 = (uint32_t)upper_bound_dev(s_ins, 0, ni, (uint16_t)c0);
-            const bool clean = (D0 == nd || s_del[D0] >= c0 + 32) && (I0 == ni || s_ins[I0] >= c0 + 32);
-            if (i < n_old) {
-                uint32_t o;
-                bool keep = true;
-                if (clean) o = i - D0 + I0;
-                else {
-                    const uint32_t Di = (uint32_t)lower_bound_dev(s_del, D0, nd, (uint16_t)i);
-                    const uint32_t Ii = (uint32_t)upper_bound_dev(s_ins, I0, ni, (uint16_t)i);
-                    keep = !(Di < nd && s_del[Di] == i);
-                    o = i - Di + Ii;
+        for (uint32_t i = tid; i < nd; i += kThreads) {
+            const uint32_t p = (uint32_t)((i == (uint32_t)tid ? pf_del : a.del_pos[dl0 + i]) - j0);
+            atomicOr(&s_dmask[p >> 5], 1u << (p & 31));
+        }
+        for (uint32_t s = tid; s < ni; s += kThreads) {
+            const uint32_t p = (uint32_t)((s == (uint32_t)tid ? pf_ins : a.ins_pos[r0 + s]) - j0);
+            s_ins[s] = (uint16_t)p;
+            atomicAdd(&s_icnt[p >> 5], 1u);
+        }
+        __syncthreads();
+        if (wid == 0) {
+            // keep masks of the 64 chunks (2 per lane): valid & not deleted & not cascaded,
+            // then exclusive scans of kept counts and of inserted-record counts
+            uint32_t m[2];
+#pragma unroll
+            for (int h = 0; h < 2; ++h) {
+                const uint32_t c = 2 * lane + h, i0 = c * 32;
+                uint32_t v = (i0 >= n_old) ? 0u : (n_old - i0 >= 32 ? 0xFFFFFFFFu : (0xFFFFFFFFu >> (32 - (n_old - i0))));
+                v &= ~s_dmask[c];
+                if (CASC && v) {
+                    const uint64_t x = j0 + i0, q = x >> 5;
+                    const uint32_t lo = a.casc_mask[q], hi = (x & 31) ? a.casc_mask[q + 1] : 0u;
+                    v &= ~__funnelshift_r(lo, hi, (uint32_t)(x & 31));
                 }
-                if (keep) { oc[o] = s_col[b][i + sh]; ow[o] = s_w[b][i + sh]; }
+                m[h] = v;
+                s_mask[c] = v;
+            }
+            const uint32_t c0 = __popc(m[0]), c1 = __popc(m[1]);
+            const uint32_t inc = warp_inclusive_scan(c0 + c1);
+            s_cbase[2 * lane] = inc - c0 - c1;
+            s_cbase[2 * lane + 1] = inc - c1;
+            if (lane == 31) s_cbase[NCH] = inc;
+            const uint32_t k0 = s_icnt[2 * lane], k1 = s_icnt[2 * lane + 1];
+            const uint32_t ik = warp_inclusive_scan(k0 + k1);
+            s_ibase[2 * lane] = ik - k0 - k1;
+            s_ibase[2 * lane + 1] = ik - k1;
+            if (lane == 31) { s_ibase[NCH] = ik; s_ibase[NCH + 1] = ik + s_icnt[NCH]; }
+        }
+        mbar_wait(&s_bar[b], (it >> 1) & 1);
+        for (uint32_t i = tid; i < nu; i += kThreads) {
+            const bool pf = i == (uint32_t)tid;
+            s_w[b][(pf ? pf_upd : a.upd_pos[ul0 + i]) - (j0 & ~3ull)] = pf ? pf_uw : a.upd_w[ul0 + i];
+        }
+        if (tid == 0) bulk_wait_read0();  // previous tile's bulk store has finished reading s_oc/s_ow
+        __syncthreads();
+        const uint32_t kept = s_cbase[NCH];
+        const uint32_t n_out = kept + ni;
+        const uint64_t base = j0 - dl0 - (CASC ? s_cbefore : 0) + r0;
+        const uint32_t ob = (uint32_t)(base & 3);
+        // phase B: old elements, output index = kept before + inserted at positions <= i
+        for (uint32_t c = wid; c * 32 < n_old; c += kThreads / 32) {
+            const uint32_t m = s_mask[c];
+            const uint32_t i = c * 32 + lane;
+            uint32_t I = s_ibase[c];
+            if (s_icnt[c]) {  // inserted records inside this chunk: count those at positions <= i
+                const uint32_t lo = s_ibase[c], hi = lo + s_icnt[c];
+                I = (uint32_t)upper_bound_dev(s_ins, lo, hi, (uint16_t)i);
+            }
+            if (m >> lane & 1) {
+                const uint32_t e = s_cbase[c] + __popc(m & lt) + I + ob;
+                uint32_t col = s_col[b][i + sh];
+                if (REMAP) {
+                    const int32_t shf = a.remap_shift[col >> kRemapBlockShift];
+                    col = (shf != kRemapMixed) ? (uint32_t)((int64_t)col + shf) : a.remap[col];
+                }
+                s_oc[e] = col;
+                s_ow[e] = s_w[b][i + sh];
             }
         }
-        // inserted records: local pos p precedes old element p
+        // inserted records: local position p precedes old element p
+        auto kept_before = [&](uint32_t i) -> uint32_t {  // i in [0, n_old]
+            const uint32_t c = i >> 5, r = i & 31;
+            return s_cbase[c] + (r ? __popc(s_mask[c] & (0xFFFFFFFFu >> (32 - r))) : 0u);
+        };
         for (uint32_t s = tid; s < ni; s += kThreads) {
-            const uint32_t p = s_ins[s];
-            const uint32_t o = p - (uint32_t)lower_bound_dev(s_del, 0, nd, (uint16_t)p) + s;
-            oc[o] = a.ins_col[r0 + s];
-            ow[o] = a.ins_w[r0 + s];
+            const uint32_t e = kept_before(s_ins[s]) + s + ob;
+            const bool pf = s == (uint32_t)tid;
+            s_oc[e] = pf ? pf_icol : a.ins_col[r0 + s];
+            s_ow[e] = pf ? pf_iw : a.ins_w[r0 + s];
+        }
+        if (CASC) {
+            // kept-before at every old row that starts inside this tile (last tile: also at E)
+            const bool last = (t == a.n_tiles - 1);
+            const uint64_t ka = s_meta[b][4] >> 32;
+            const uint64_t kb = last ? a.V_old + 1 : (part[t + 1].k);
+            const uint64_t kb0 = j0 - dl0 - s_cbefore;  // kept old elements before j0
+            for (uint64_t k = ka + tid; k < kb; k += kThreads)
+                a.KR[k] = (int64_t)(kb0 + kept_before((uint32_t)((uint64_t)a.old_off[k] - j0)));
+        }
+        __syncthreads();
+        // store the contiguous output chunk [base, base + n_out)
+        {
+            uint32_t head = (4 - ob) & 3;
+            if (head > n_out) head = n_out;
+            const uint32_t body = ((n_out - head) >> 2) << 2;
+            if (tid < head) { a.new_cols[base + tid] = s_oc[ob + tid]; a.new_w[base + tid] = s_ow[ob + tid]; }
+            for (uint32_t e = head + body + tid; e < n_out; e += kThreads) {
+                a.new_cols[base + e] = s_oc[ob + e];
+                a.new_w[base + e] = s_ow[ob + e];
+            }
+            if (tid == 0) {
+                if (body) {
+                    fence_proxy_async();
+                    bulk_s2g(a.new_cols + base + head, &s_oc[ob + head], body * 4);
+                    bulk_s2g(a.new_w + base + head, &s_ow[ob + head], body * 4);
+                }
+                bulk_commit();
+            }
         }
         __syncthreads();
     }
+    if (tid == 0) bulk_wait_all();
 }
 
 // per 1024-block of old ids: constant new-id shift, or kRemapMixed if a dropped

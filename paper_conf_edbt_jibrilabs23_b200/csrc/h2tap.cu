@@ -83,7 +83,7 @@ struct h2tap_replica {
     Buf nv, nv_ext, dropped, ins_q, ins_oldpos, hd_rows, remap, hd_bits;
     Buf op_flags, op_ou, op_ow;
     Buf ins_pos, ins_row, ins_col, ins_w, del_pos, upd_pos, upd_w, KR;
-    Buf misc, nsorted, part, opart, deg, tsum, remap_shift, tile_emit, tile_base, del_row, casc_mask, status2, bfs_a, bfs_b, pr_a, pr_b;
+    Buf misc, nsorted, part, opart, deg, tsum, remap_shift, remap32, tile_emit, tile_base, del_row, casc_mask, status2, bfs_a, bfs_b, pr_a, pr_b;
     Buf ctr;
     Counters* hc = nullptr;  // pinned host mirror
     cudaEvent_t ev[8]{};
@@ -515,7 +515,6 @@ h2tap_status apply_core(h2tap_replica* r, const BatchIn& in, uint64_t S, bool cr
     uint32_t* new_cols = r->get<uint32_t>(r->cols[nb], Ecap);
     float* new_w = r->get<float>(r->w[nb], Ecap);
     const bool casc = n_hd > 0;
-    int64_t* KR = casc ? r->get<int64_t>(r->KR, V + 1) : nullptr;
     const uint64_t Dtot = E + n_ins;
     if (Dtot) {
         MergeArgs ma{};
@@ -524,7 +523,10 @@ h2tap_status apply_core(h2tap_replica* r, const BatchIn& in, uint64_t S, bool cr
         ma.del_pos = del_pos; ma.n_del = n_del;
         ma.upd_pos = upd_pos; ma.upd_w = upd_w; ma.n_upd = n_upd;
         ma.remap = remap; ma.hd_bits = hd_bits; ma.hd_rows = hd_rows; ma.n_hd = n_hd;
-        ma.new_cols = new_cols; ma.new_w = new_w; ma.KR = KR;
+        ma.new_cols = new_cols; ma.new_w = new_w;
+        ma.rows = n_node ? 1 : 0;
+        ma.new_off = new_off; ma.ins_row = ins_row;
+        ma.dropped = dropped; ma.n_dropped = n_dropped; ma.ins_oldpos = ins_oldpos; ma.n_vins = n_vins;
         ma.n_tiles = cdiv(Dtot, kMergeTile);
         ma.c = dc;
         if (remap_on) {
@@ -535,6 +537,10 @@ h2tap_status apply_core(h2tap_replica* r, const BatchIn& in, uint64_t S, bool cr
                 CKL();
             }
             ma.remap_shift = rs;
+            const uint64_t ng = cdiv(V, 32);
+            uint2* r32 = r->get<uint2>(r->remap32, ng);
+            if (ng) { k_remap32<<<g1(ng), 256, 0, st>>>(V, dropped, n_dropped, ins_oldpos, n_vins, r32); CKL(); }
+            ma.remap32 = r32;
         }
         TilePart* part = r->get<TilePart>(r->part, ma.n_tiles + 1);
         k_merge_partition<<<g1(ma.n_tiles + 1), 256, 0, st>>>(ma, part);
@@ -556,9 +562,10 @@ h2tap_status apply_core(h2tap_replica* r, const BatchIn& in, uint64_t S, bool cr
         else if (remap_on) launch(k_merge3<false, true>);
         else launch(k_merge3<false, false>);
         CKL();
-    } else if (casc) {
-        CK(cudaStreamWaitEvent(st, r->evB, 0));
-        CK(cudaMemsetAsync(KR, 0, (V + 1) * 8, st));
+    } else {
+        if (casc) CK(cudaStreamWaitEvent(st, r->evB, 0));
+        // nothing to merge: every surviving row is empty
+        if (n_node) CK(cudaMemsetAsync(new_off, 0, (Vn + 1) * 8, st));
     }
     CK(cudaEventRecord(r->ev[4], st));
     if (casc) {
@@ -569,43 +576,29 @@ h2tap_status apply_core(h2tap_replica* r, const BatchIn& in, uint64_t S, bool cr
 
     // ---- a4/a5: row offsets
     if (V && !n_node) {
-        // per-vertex degree delta + single-pass decoupled look-back exclusive scan
+        // per-vertex degree delta + exclusive scan (tile sums by decoupled look-back)
         int32_t* deg = r->get<int32_t>(r->deg, V);
-        int64_t* tsum = r->get<int64_t>(r->tsum, cdiv(V, kTile) + 1);
+        const uint64_t nt = cdiv(V, kTile);
+        int64_t* tsum = r->get<int64_t>(r->tsum, nt + 1);
+        int64_t* tbase = r->get<int64_t>(r->KR, nt + 1);
         CK(cudaMemsetAsync(deg, 0, V * 4, st));
-        CK(cudaMemsetAsync(tsum, 0, (cdiv(V, kTile) + 1) * 8, st));
+        CK(cudaMemsetAsync(tsum, 0, (nt + 1) * 8, st));
         if (n_ins + n_del) {
             k_deg_scatter<<<g1(n_ins + n_del), 256, 0, st>>>(ins_row, n_ins, static_cast<uint32_t*>(r->del_row.p), n_del, deg, tsum);
             CKL();
         }
-        // chain-free: tile sums were accumulated by the scatter; scan them in one CTA,
-        // then a streaming pass writes new_off = old_off + tile base + in-tile prefix
-        const uint64_t nt = cdiv(V, kTile);
-        k_tile_sum_scan<<<1, 1024, 0, st>>>(tsum, nt);
+        const uint64_t nts = cdiv(nt, kTile);
+        uint64_t* stt = r->get<uint64_t>(r->status, nts);
+        CK(cudaMemsetAsync(stt, 0, nts * 8, st));
+        k_scan_exclusive_i64<<<(unsigned)nts, kThreads, 0, st>>>(tsum, tbase, nt, stt, &dc->tiles[7]);
         CKL();
-        k_offsets_apply<<<(unsigned)nt, kThreads, 0, st>>>(old_off, deg, V, tsum, new_off);
-        CKL();
-    } else if (V) {
-        OffArgs oa{};
-        oa.old_off = old_off; oa.V_old = V; oa.KR = KR;
-        oa.del_pos = del_pos; oa.n_del = n_del; oa.ins_row = ins_row; oa.n_ins = n_ins;
-        oa.remap = remap; oa.dropped = dropped; oa.n_dropped = n_dropped;
-        oa.ins_oldpos = ins_oldpos; oa.n_vins = n_vins; oa.new_off = new_off;
-        const uint64_t ncta = cdiv(V, kOffTile);
-        oa.part = r->get<uint64_t>(r->opart, 2 * (ncta + 1));
-        if (remap_on) k_offsets_partition<true><<<g1(ncta + 1), 256, 0, st>>>(oa);
-        else k_offsets_partition<false><<<g1(ncta + 1), 256, 0, st>>>(oa);
-        CKL();
-        const unsigned grid = (unsigned)ncta;
-        if (casc && remap_on) k_offsets_old<true, true><<<grid, kThreads, 0, st>>>(oa);
-        else if (casc) k_offsets_old<true, false><<<grid, kThreads, 0, st>>>(oa);
-        else if (remap_on) k_offsets_old<false, true><<<grid, kThreads, 0, st>>>(oa);
-        else k_offsets_old<false, false><<<grid, kThreads, 0, st>>>(oa);
+        k_offsets_apply<<<(unsigned)nt, kThreads, 0, st>>>(old_off, deg, V, tbase, new_off);
         CKL();
     }
+    // (with node ops the merge kernel wrote the offsets of surviving old rows)
     if (n_vins) {
-        if (casc) k_offsets_inserted<true><<<g1(n_vins), 256, 0, st>>>(nv, ins_q, n_vins, old_off, KR, del_pos, n_del, ins_row, n_ins, new_off);
-        else k_offsets_inserted<false><<<g1(n_vins), 256, 0, st>>>(nv, ins_q, n_vins, old_off, KR, del_pos, n_del, ins_row, n_ins, new_off);
+        k_offsets_inserted<<<g1(n_vins), 256, 0, st>>>(nv, ins_q, n_vins, old_off, del_pos, n_del, casc ? casc_mask : nullptr,
+                                                       casc_pre, ins_row, n_ins, new_off);
         CKL();
     }
     k_set_i64<<<1, 1, 0, st>>>(new_off + Vn, (int64_t)En);
@@ -730,7 +723,7 @@ void free_replica(h2tap_replica* r) {
                    &r->hist, &r->dbase, &r->rs_status, &r->rs_ctr, &r->nv, &r->nv_ext, &r->dropped, &r->ins_q,
                    &r->ins_oldpos, &r->hd_rows, &r->remap, &r->hd_bits, &r->op_flags, &r->op_ou, &r->op_ow,
                    &r->ins_pos, &r->ins_row, &r->ins_col, &r->ins_w, &r->del_pos, &r->upd_pos, &r->upd_w,
-                   &r->KR, &r->misc, &r->nsorted, &r->part, &r->opart, &r->deg, &r->tsum, &r->remap_shift, &r->tile_emit, &r->tile_base, &r->del_row, &r->casc_mask, &r->status2, &r->fence[0], &r->fence[1], &r->bfs_a, &r->bfs_b, &r->pr_a, &r->pr_b, &r->ctr};
+                   &r->KR, &r->misc, &r->nsorted, &r->part, &r->opart, &r->deg, &r->tsum, &r->remap_shift, &r->remap32, &r->tile_emit, &r->tile_base, &r->del_row, &r->casc_mask, &r->status2, &r->fence[0], &r->fence[1], &r->bfs_a, &r->bfs_b, &r->pr_a, &r->pr_b, &r->ctr};
     for (Buf* b : bufs) if (b->p) r->dfree(b->p);
     cudaStreamSynchronize(r->st);
     for (auto& e : r->ev) if (e) cudaEventDestroy(e);

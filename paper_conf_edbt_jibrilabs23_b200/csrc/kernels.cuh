@@ -688,7 +688,14 @@ struct MergeArgs {
     uint64_t n_hd;
     uint32_t* new_cols;
     float* new_w;
-    int64_t* KR;  // CASC: kept elements before each old row start, [V_old + 1]
+    int64_t* new_off;            // ROWS mode (node ops): offsets of surviving old rows written by the merge
+    const uint32_t* ins_row;     // row of each inserted record (sorted)
+    const uint32_t* dropped;     // sorted old ids of dropped vertices
+    uint64_t n_dropped;
+    const uint32_t* ins_oldpos;  // sorted insertion ranks of inserted vertices
+    uint64_t n_vins;
+    const uint2* remap32;        // per 32 old ids: {base new id, dropped bitmask} (kRemapExact: use remap[])
+    int rows;                    // 1: merge writes new_off for old rows starting in each tile
     const uint32_t* casc_mask;  // CASC: 1 bit per old element (removed by a node delete)
     const uint64_t* casc_pre;   // CASC: cascaded elements before each 2048-element block
     uint64_t n_tiles;
@@ -699,7 +706,7 @@ struct MergeArgs {
 // merged items (smallest r with ins_pos[r] + r >= d), j = d - r old elements,
 // and the ranks of j in the sorted delete / update / cascade-row lists.
 struct TilePart {
-    uint64_t r, dl, ul, hA, hB, k;  // k: first old row starting at or after j (CASC)
+    uint64_t r, dl, ul, k, ir;  // k: first old row starting at or after j; ir: ins-row rank of k's new id
 };
 
 __device__ __forceinline__ uint64_t ins_split(const uint64_t* ins_pos, uint64_t n_ins, uint64_t d) {
@@ -721,8 +728,17 @@ __global__ void k_merge_partition(MergeArgs a, TilePart* __restrict__ part) {
     const uint64_t j = d - p.r;
     p.dl = lower_bound_dev(a.del_pos, 0, a.n_del, j);
     p.ul = lower_bound_dev(a.upd_pos, 0, a.n_upd, j);
-    p.hA = p.hB = 0;
-    p.k = a.n_hd ? lower_bound_dev(a.old_off, 0, a.V_old + 1, (int64_t)j) : 0;
+    p.k = p.ir = 0;
+    if (a.rows) {
+        p.k = lower_bound_dev(a.old_off, 0, a.V_old + 1, (int64_t)j);
+        if (p.k >= a.V_old) p.ir = a.n_ins;
+        else {
+            // new id of the first surviving old row >= k (compaction formula, reading A9)
+            const uint64_t u = p.k - lower_bound_dev(a.dropped, 0, a.n_dropped, (uint32_t)p.k) +
+                               upper_bound_dev(a.ins_oldpos, 0, a.n_vins, (uint32_t)p.k);
+            p.ir = lower_bound_dev(a.ins_row, 0, a.n_ins, (uint32_t)u);
+        }
+    }
     part[t] = p;
 }
 
@@ -748,167 +764,6 @@ __device__ __forceinline__ void mbar_wait(uint64_t* bar, uint32_t phase) {
         "mbarrier.try_wait.parity.shared::cta.b64 p, [%0], %1;\n"
         "@!p bra WAIT_%=;\n"
         "}\n" ::"r"(smem_u32(bar)), "r"(phase) : "memory");
-}
-
-// Global merge path.  The new column/weight arrays are the merge of the kept
-// old elements (old order) with the inserted records (key order); an inserted
-// record at old position p precedes old element p, so its merged index is
-// p + r.  Tile t owns merged items [t*2048, (t+1)*2048) (load balanced for
-// giant rows and insert bursts).  Persistent CTAs walk the tiles; while one
-// tile is processed the next tile's old elements stream into the other shared
-// buffer with two TMA bulk copies.  Each warp compacts a 256-slot chunk with
-// ballots: slot -> old element index / inserted record, drop deleted and
-// cascaded elements, override weights, remap column IDs, coalesced stores.
-template <bool CASC, bool REMAP>
-__global__ void __launch_bounds__(kThreads) k_merge(MergeArgs a, const TilePart* __restrict__ part) {
-    __shared__ __align__(128) uint32_t s_col[2][kMergeBuf];
-    __shared__ __align__(128) float s_w[2][kMergeBuf];
-    __shared__ uint16_t s_slot[kMergeTile];
-    __shared__ uint8_t s_keep[kMergeTile];
-    __shared__ uint32_t s_kp[CASC ? kMergeTile + 1 : 1];
-    __shared__ uint32_t s_wold[kThreads / 32], s_wemit[kThreads / 32];
-    __shared__ __align__(8) uint64_t s_bar[2];
-    __shared__ uint64_t s_cbefore;
-
-    const int tid = threadIdx.x, wid = tid >> 5;
-    const uint32_t lane = lane_id(), lt = lanemask_lt();
-    const uint64_t Dtot = a.E_old + a.n_ins;
-    if (tid == 0) { mbar_init(&s_bar[0], 1); mbar_init(&s_bar[1], 1); fence_mbar_init(); }
-    __syncthreads();
-
-    auto tile_j = [&](uint64_t t) -> uint64_t { return min(t * kMergeTile, Dtot) - part[t].r; };
-    auto issue = [&](uint64_t t, int b) {  // one thread: stage old elements of tile t
-        const uint64_t j0 = tile_j(t), j1 = tile_j(t + 1);
-        const uint64_t a0 = j0 & ~3ull, a1 = (j1 + 3) & ~3ull;
-        const uint32_t bytes = (uint32_t)((a1 - a0) * 4);
-        mbar_expect_tx(&s_bar[b], 2 * bytes);
-        if (bytes) {
-            bulk_g2s(&s_col[b][0], a.old_cols + a0, bytes, &s_bar[b]);
-            bulk_g2s(&s_w[b][0], a.old_w + a0, bytes, &s_bar[b]);
-        }
-    };
-
-    uint64_t t = blockIdx.x;
-    if (t < a.n_tiles && tid == 0) issue(t, 0);
-    for (uint32_t it = 0; t < a.n_tiles; t += gridDim.x, ++it) {
-        const int b = it & 1;
-        if (tid == 0 && t + gridDim.x < a.n_tiles) { fence_proxy_async(); issue(t + gridDim.x, b ^ 1); }
-        const TilePart p0 = part[t], p1 = part[t + 1];
-        const uint64_t d0 = min(t * kMergeTile, Dtot), d1 = min((t + 1) * kMergeTile, Dtot);
-        const uint64_t r0 = p0.r, j0 = d0 - r0, j1 = d1 - p1.r;
-        const uint32_t n_old = (uint32_t)(j1 - j0), n_new = (uint32_t)(p1.r - r0), n_tot = n_old + n_new;
-        const uint32_t sh = (uint32_t)(j0 & 3);  // staged element i lives at s_*[i + sh]
-        for (uint32_t i = tid; i < kMergeTile; i += kThreads) { s_slot[i] = 0xFFFF; s_keep[i] = 1; }
-        __syncthreads();
-        for (uint32_t s = tid; s < n_new; s += kThreads) s_slot[(a.ins_pos[r0 + s] - j0) + s] = (uint16_t)s;
-        for (uint64_t i = p0.dl + tid; i < p1.dl; i += kThreads) s_keep[a.del_pos[i] - j0] = 0;
-        if (CASC) {
-            for (uint32_t i = tid; i < n_old; i += kThreads)
-                if (a.casc_mask[(j0 + i) >> 5] >> ((j0 + i) & 31) & 1) s_keep[i] = 0;
-            if (wid == 0) {  // cascaded elements before j0: block prefix + popcount of the partial block
-                const uint64_t blk = j0 / kCascBlock, wb = blk * (kCascBlock / 32), we = j0 >> 5;
-                uint32_t c = 0;
-                for (uint64_t q = wb + lane; q <= we; q += 32) {
-                    uint32_t m = a.casc_mask[q];
-                    if (q == we) m &= (j0 & 31) ? (0xFFFFFFFFu >> (32 - (j0 & 31))) : 0u;
-                    c += __popc(m);
-                }
-                c = warp_sum(c);
-                if (lane == 0) s_cbefore = a.casc_pre[blk] + c;
-            }
-        }
-        mbar_wait(&s_bar[b], (it >> 1) & 1);
-        const uint64_t a0 = j0 & ~3ull;
-        for (uint64_t i = p0.ul + tid; i < p1.ul; i += kThreads) s_w[b][a.upd_pos[i] - a0] = a.upd_w[i];
-        __syncthreads();
-        // pass 1: old slots per warp chunk
-        const uint32_t mb = wid * 256;
-        uint32_t oldm[8];
-        uint32_t n_oldw = 0;
-#pragma unroll
-        for (int k = 0; k < 8; ++k) {
-            uint32_t m = mb + k * 32 + lane;
-            oldm[k] = __ballot_sync(0xffffffffu, m < n_tot && s_slot[m] == 0xFFFF);
-            n_oldw += __popc(oldm[k]);
-        }
-        if (lane == 0) s_wold[wid] = n_oldw;
-        __syncthreads();
-        uint32_t oi_base = 0;
-        for (int w2 = 0; w2 < wid; ++w2) oi_base += s_wold[w2];
-        // pass 2: emitted items per warp chunk
-        uint32_t emm[8];
-        uint32_t n_emw = 0;
-        {
-            uint32_t oi_run = oi_base;
-#pragma unroll
-            for (int k = 0; k < 8; ++k) {
-                uint32_t m = mb + k * 32 + lane;
-                bool isold = oldm[k] >> lane & 1;
-                uint32_t oi = oi_run + __popc(oldm[k] & lt);
-                bool e = (m < n_tot) && (!isold || s_keep[oi]);
-                emm[k] = __ballot_sync(0xffffffffu, e);
-                n_emw += __popc(emm[k]);
-                oi_run += __popc(oldm[k]);
-            }
-        }
-        if (lane == 0) s_wemit[wid] = n_emw;
-        __syncthreads();
-        uint32_t em_base = 0, tile_emit = 0;
-        for (int w2 = 0; w2 < kThreads / 32; ++w2) {
-            uint32_t v = s_wemit[w2];
-            if (w2 < wid) em_base += v;
-            tile_emit += v;
-        }
-        // output index of the tile's first item: kept old elements before j0 + inserted
-        // records before d0 (cascade mode: from the count pass + scan)
-        const uint64_t base = j0 - p0.dl - (CASC ? s_cbefore : 0) + r0;
-        // pass 3: write the tile's output chunk (coalesced 4 B stores per warp iteration)
-        {
-            uint32_t oi_run = oi_base, e_run = em_base;
-#pragma unroll
-            for (int k = 0; k < 8; ++k) {
-                uint32_t m = mb + k * 32 + lane;
-                bool isold = oldm[k] >> lane & 1;
-                uint32_t oi = oi_run + __popc(oldm[k] & lt);
-                bool e = emm[k] >> lane & 1;
-                uint32_t eo = e_run + __popc(emm[k] & lt);
-                if (CASC && isold) s_kp[oi] = eo - (m - oi);
-                if (e) {
-                    uint32_t col;
-                    float wv;
-                    if (isold) {
-                        col = s_col[b][oi + sh];
-                        wv = s_w[b][oi + sh];
-                        if (REMAP) {
-                            int32_t shf = a.remap_shift[col >> kRemapBlockShift];
-                            col = (shf != kRemapMixed) ? (uint32_t)((int64_t)col + shf) : a.remap[col];
-                        }
-                    } else {
-                        uint32_t s = s_slot[m];
-                        col = a.ins_col[r0 + s];
-                        wv = a.ins_w[r0 + s];
-                    }
-                    a.new_cols[base + eo] = col;
-                    a.new_w[base + eo] = wv;
-                }
-                oi_run += __popc(oldm[k]);
-                e_run += __popc(emm[k]);
-            }
-        }
-        if (CASC) {
-            __syncthreads();
-            if (tid == 0) s_kp[n_old] = tile_emit - n_new;
-            __syncthreads();
-            // kept-before at every old row that starts inside this tile (last tile: also at E)
-            const bool last = (t == a.n_tiles - 1);
-            const uint64_t kept_before = base - r0;
-            uint64_t ka = p0.k;
-            uint64_t kb = last ? a.V_old + 1 : p1.k;
-            for (uint64_t k = ka + tid; k < kb; k += kThreads)
-                a.KR[k] = (int64_t)(kept_before + s_kp[(uint64_t)a.old_off[k] - j0]);
-        }
-        __syncthreads();
-    }
 }
 
 // Cascade mode (a4 cascade pass): one bit per old element, set when a node delete
@@ -1020,6 +875,20 @@ __global__ void __launch_bounds__(kThreads) k_scan_exclusive_u64(const uint64_t*
 
 constexpr int kMerge3Smem = 6 * kMergeBuf * 4;  // dynamic shared memory of k_merge3
 
+constexpr uint32_t kRemapExact = 0xFFFFFFFFu;  // remap32 base: group needs the exact table
+constexpr int kRowStage = 512;                 // rows mode: insert-row slice staged in smem
+
+// new dense id of surviving old vertex `col` (REMAP mode): constant shift of its
+// 1024-block, else base of its 32-group minus the dropped ids below it
+__device__ __forceinline__ uint32_t remap_col(const MergeArgs& a, uint32_t col) {
+    const int32_t shf = a.remap_shift[col >> kRemapBlockShift];
+    if (shf != kRemapMixed) return (uint32_t)((int64_t)col + shf);
+    const uint2 g = a.remap32[col >> 5];
+    if (g.x == kRemapExact) return a.remap[col];
+    const uint32_t r = col & 31;
+    return g.x + r - (r ? __popc(g.y & (0xFFFFFFFFu >> (32 - r))) : 0u);
+}
+
 // ---- TMA bulk store (smem -> global) helpers
 __device__ __forceinline__ void bulk_s2g(void* dst, const void* src, uint32_t bytes) {
     asm volatile("cp.async.bulk.global.shared::cta.bulk_group [%0], [%1], %2;"
@@ -1054,6 +923,8 @@ __global__ void __launch_bounds__(kThreads) k_merge3(MergeArgs a, const TilePart
     __shared__ uint32_t s_ibase[NCH + 2];   // inserted records at positions before each chunk
     __shared__ __align__(8) uint64_t s_bar[2];
     __shared__ uint64_t s_meta[2][5];
+    __shared__ uint64_t s_rows[2][4];
+    __shared__ uint32_t s_irow[kRowStage];  // rows mode: the tile's slice of insert rows
     __shared__ uint64_t s_cbefore;
 
     const int tid = threadIdx.x, wid = tid >> 5;
@@ -1064,7 +935,8 @@ __global__ void __launch_bounds__(kThreads) k_merge3(MergeArgs a, const TilePart
     auto issue = [&](uint64_t t, int b) {  // one thread: tile metadata + TMA of its old elements
         const TilePart p0 = part[t], p1 = part[t + 1];
         s_meta[b][0] = p0.r; s_meta[b][1] = p1.r; s_meta[b][2] = p0.dl; s_meta[b][3] = p0.ul;
-        s_meta[b][4] = (p1.dl - p0.dl) | ((p1.ul - p0.ul) << 16) | (CASC ? (p0.k << 32) : 0);
+        s_meta[b][4] = (p1.dl - p0.dl) | ((p1.ul - p0.ul) << 16);
+        s_rows[b][0] = p0.k; s_rows[b][1] = p1.k; s_rows[b][2] = p0.ir; s_rows[b][3] = p1.ir;
         const uint64_t j0 = min(t * kMergeTile, Dtot) - p0.r, j1 = min((t + 1) * kMergeTile, Dtot) - p1.r;
         const uint64_t a0 = j0 & ~3ull, a1 = (j1 + 3) & ~3ull;
         const uint32_t bytes = (uint32_t)((a1 - a0) * 4);
@@ -1080,6 +952,7 @@ __global__ void __launch_bounds__(kThreads) k_merge3(MergeArgs a, const TilePart
     for (uint32_t it = 0; t < a.n_tiles; t += gridDim.x, ++it) {
         const int b = it & 1;
         const uint64_t r0 = s_meta[b][0], r1 = s_meta[b][1], dl0 = s_meta[b][2], ul0 = s_meta[b][3];
+        const uint64_t rk0 = s_rows[b][0], rk1 = s_rows[b][1], ir0 = s_rows[b][2], ir1 = s_rows[b][3];
         const uint32_t nd = (uint32_t)(s_meta[b][4] & 0xFFFF), nu = (uint32_t)((s_meta[b][4] >> 16) & 0xFFFF);
         const uint64_t d0 = min(t * kMergeTile, Dtot), d1 = min((t + 1) * kMergeTile, Dtot);
         const uint64_t j0 = d0 - r0, j1 = d1 - r1;
@@ -1094,6 +967,21 @@ __global__ void __launch_bounds__(kThreads) k_merge3(MergeArgs a, const TilePart
         const float pf_iw = tid < ni ? a.ins_w[r0 + tid] : 0.f;
         const uint64_t pf_upd = tid < nu ? a.upd_pos[ul0 + tid] : 0;
         const float pf_uw = tid < nu ? a.upd_w[ul0 + tid] : 0.f;
+        // rows mode: the tile's old rows (first 2*kThreads) and its slice of insert rows
+        const bool last_tile = (t == a.n_tiles - 1);
+        const uint64_t rk_end = last_tile ? a.V_old : rk1;
+        const uint64_t ir_end = last_tile ? a.n_ins : ir1;
+        const uint32_t n_rows = a.rows ? (uint32_t)min(rk_end - rk0, (uint64_t)0xFFFFFFFF) : 0u;
+        const uint32_t n_irs = a.rows ? (uint32_t)(ir_end - ir0) : 0u;
+        int64_t pf_x[2];
+        uint32_t pf_u[2];
+#pragma unroll
+        for (int h = 0; h < 2; ++h) {
+            const uint32_t q = tid + h * kThreads;
+            pf_x[h] = q < n_rows ? a.old_off[rk0 + q] : 0;
+            pf_u[h] = q < n_rows ? (REMAP ? a.remap[rk0 + q] : (uint32_t)(rk0 + q)) : kNone32;
+        }
+        for (uint32_t q = tid; q < n_irs && q < kRowStage; q += kThreads) s_irow[q] = a.ins_row[ir0 + q];
         if (tid < NCH + 2) { s_dmask[tid] = 0; s_icnt[tid] = 0; }
         if (CASC && wid == 1) {  // cascaded elements before j0 (block prefix + partial popcount)
             const uint64_t blk = j0 / kCascBlock, wb = blk * (kCascBlock / 32), we = j0 >> 5;
@@ -1156,24 +1044,47 @@ __global__ void __launch_bounds__(kThreads) k_merge3(MergeArgs a, const TilePart
         const uint32_t n_out = kept + ni;
         const uint64_t base = j0 - dl0 - (CASC ? s_cbefore : 0) + r0;
         const uint32_t ob = (uint32_t)(base & 3);
-        // phase B: old elements, output index = kept before + inserted at positions <= i
-        for (uint32_t c = wid; c * 32 < n_old; c += kThreads / 32) {
-            const uint32_t m = s_mask[c];
-            const uint32_t i = c * 32 + lane;
-            uint32_t I = s_ibase[c];
-            if (s_icnt[c]) {  // inserted records inside this chunk: count those at positions <= i
-                const uint32_t lo = s_ibase[c], hi = lo + s_icnt[c];
-                I = (uint32_t)upper_bound_dev(s_ins, lo, hi, (uint16_t)i);
+        // phase B: old elements, output index = kept before + inserted at positions <= i.
+        // Warp w owns chunks w, w+8, ..., w+56; the 8 chunks are unrolled so that the
+        // remap-table lookups of all of them are in flight together.
+        {
+            constexpr int KCH = NCH / (kThreads / 32);  // 8 chunks per warp
+            uint32_t colv[KCH];
+#pragma unroll
+            for (int k = 0; k < KCH; ++k) {
+                const uint32_t c = wid + k * (kThreads / 32), i = c * 32 + lane;
+                colv[k] = (i < n_old) ? s_col[b][i + sh] : 0u;
             }
-            if (m >> lane & 1) {
-                const uint32_t e = s_cbase[c] + __popc(m & lt) + I + ob;
-                uint32_t col = s_col[b][i + sh];
-                if (REMAP) {
-                    const int32_t shf = a.remap_shift[col >> kRemapBlockShift];
-                    col = (shf != kRemapMixed) ? (uint32_t)((int64_t)col + shf) : a.remap[col];
+            if (REMAP) {
+                int32_t shf[KCH];
+#pragma unroll
+                for (int k = 0; k < KCH; ++k) shf[k] = a.remap_shift[colv[k] >> kRemapBlockShift];
+                uint2 g[KCH];
+#pragma unroll
+                for (int k = 0; k < KCH; ++k) g[k] = (shf[k] == kRemapMixed) ? a.remap32[colv[k] >> 5] : make_uint2(0u, 0u);
+#pragma unroll
+                for (int k = 0; k < KCH; ++k) {
+                    const uint32_t col = colv[k], r = col & 31;
+                    if (shf[k] != kRemapMixed) colv[k] = (uint32_t)((int64_t)col + shf[k]);
+                    else if (g[k].x == kRemapExact) colv[k] = a.remap[col];
+                    else colv[k] = g[k].x + r - (r ? __popc(g[k].y & (0xFFFFFFFFu >> (32 - r))) : 0u);
                 }
-                s_oc[e] = col;
-                s_ow[e] = s_w[b][i + sh];
+            }
+#pragma unroll
+            for (int k = 0; k < KCH; ++k) {
+                const uint32_t c = wid + k * (kThreads / 32), i = c * 32 + lane;
+                if (c * 32 >= n_old) break;
+                const uint32_t m = s_mask[c];
+                uint32_t I = s_ibase[c];
+                if (s_icnt[c]) {  // inserted records inside this chunk: count those at positions <= i
+                    const uint32_t lo = s_ibase[c], hi = lo + s_icnt[c];
+                    I = (uint32_t)upper_bound_dev(s_ins, lo, hi, (uint16_t)i);
+                }
+                if (m >> lane & 1) {
+                    const uint32_t e = s_cbase[c] + __popc(m & lt) + I + ob;
+                    s_oc[e] = colv[k];
+                    s_ow[e] = s_w[b][i + sh];
+                }
             }
         }
         // inserted records: local position p precedes old element p
@@ -1187,14 +1098,21 @@ __global__ void __launch_bounds__(kThreads) k_merge3(MergeArgs a, const TilePart
             s_oc[e] = pf ? pf_icol : a.ins_col[r0 + s];
             s_ow[e] = pf ? pf_iw : a.ins_w[r0 + s];
         }
-        if (CASC) {
-            // kept-before at every old row that starts inside this tile (last tile: also at E)
-            const bool last = (t == a.n_tiles - 1);
-            const uint64_t ka = s_meta[b][4] >> 32;
-            const uint64_t kb = last ? a.V_old + 1 : (part[t + 1].k);
-            const uint64_t kb0 = j0 - dl0 - s_cbefore;  // kept old elements before j0
-            for (uint64_t k = ka + tid; k < kb; k += kThreads)
-                a.KR[k] = (int64_t)(kb0 + kept_before((uint32_t)((uint64_t)a.old_off[k] - j0)));
+        if (a.rows) {
+            // a4/a5 fused: new_off[u'] of every surviving old row k starting in this tile
+            //   = (kept old elements before its old start) + (inserted records in rows < u')
+            const uint64_t kb0 = j0 - dl0 - (CASC ? s_cbefore : 0);  // kept old elements before j0
+            const bool staged = n_irs <= kRowStage;
+            for (uint32_t q = tid; q < n_rows; q += kThreads) {
+                const bool pf = q < 2 * kThreads;
+                const uint32_t u = pf ? (q < kThreads ? pf_u[0] : pf_u[1]) : (REMAP ? a.remap[rk0 + q] : (uint32_t)(rk0 + q));
+                if (u == kNone32) continue;
+                const int64_t x = pf ? (q < kThreads ? pf_x[0] : pf_x[1]) : a.old_off[rk0 + q];
+                const uint64_t kept_b = kb0 + kept_before((uint32_t)((uint64_t)x - j0));
+                const uint64_t irk = staged ? ir0 + lower_bound_dev(s_irow, 0, n_irs, u)
+                                            : lower_bound_dev(a.ins_row, ir0, ir_end, u);
+                a.new_off[u] = (int64_t)(kept_b + irk);
+            }
         }
         __syncthreads();
         // store the contiguous output chunk [base, base + n_out)
@@ -1242,92 +1160,6 @@ __global__ void k_remap_blocks(uint64_t V, const uint32_t* __restrict__ dropped,
 //   (kept old elements before row u's old start) + (inserted records in rows < u')
 // where both terms are ranks in sorted lists (no cascade) or the kept-before
 // table KR written by the merge's decoupled look-back (cascade).
-constexpr int kOffTile = 4096;  // old rows per CTA of the offsets kernel
-
-// new dense id of the first surviving old row >= k (REMAP: compaction formula)
-__device__ __forceinline__ uint64_t new_id_at(uint64_t k, const uint32_t* dropped, uint64_t n_dropped,
-                                              const uint32_t* ins_oldpos, uint64_t n_vins) {
-    return k - lower_bound_dev(dropped, 0, n_dropped, (uint32_t)k) +
-           upper_bound_dev(ins_oldpos, 0, n_vins, (uint32_t)k);
-}
-
-struct OffArgs {
-    const int64_t* old_off;
-    uint64_t V_old;
-    const int64_t* KR;
-    const uint64_t* del_pos;
-    uint64_t n_del;
-    const uint32_t* ins_row;
-    uint64_t n_ins;
-    const uint32_t* remap;
-    const uint32_t* dropped;
-    uint64_t n_dropped;
-    const uint32_t* ins_oldpos;
-    uint64_t n_vins;
-    int64_t* new_off;
-    uint64_t* part;  // [n_cta + 1][2]: ins-row rank, delete rank at each CTA boundary
-};
-
-template <bool REMAP>
-__global__ void k_offsets_partition(OffArgs a) {
-    uint64_t b = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x;
-    uint64_t nb = (a.V_old + kOffTile - 1) / kOffTile;
-    if (b > nb) return;
-    uint64_t k = min(b * kOffTile, a.V_old);
-    uint64_t ir, dr;
-    if (k == a.V_old) { ir = a.n_ins; dr = a.n_del; }
-    else {
-        uint64_t u = REMAP ? new_id_at(k, a.dropped, a.n_dropped, a.ins_oldpos, a.n_vins) : k;
-        ir = lower_bound_dev(a.ins_row, 0, a.n_ins, (uint32_t)u);
-        dr = lower_bound_dev(a.del_pos, 0, a.n_del, (uint64_t)a.old_off[k]);
-    }
-    a.part[2 * b] = ir;
-    a.part[2 * b + 1] = dr;
-}
-
-// new_off[u'] = (kept old elements before old row k) + (inserted records in rows < u')
-// The CTA's slices of the sorted insert-row and delete-position lists are staged
-// in shared memory; each thread then answers its rank queries there.
-constexpr int kOffStageIns = 4096, kOffStageDel = 2048;
-template <bool CASC, bool REMAP>
-__global__ void __launch_bounds__(kThreads) k_offsets_old(OffArgs a) {
-    __shared__ uint32_t s_ins[kOffStageIns];
-    __shared__ uint64_t s_del[CASC ? 1 : kOffStageDel];
-    const uint64_t cta = blockIdx.x;
-    const uint64_t ia = a.part[2 * cta], ib = a.part[2 * cta + 2];
-    const uint64_t da = a.part[2 * cta + 1], db = a.part[2 * cta + 3];
-    const uint64_t ni = ib - ia, nd = db - da;
-    const bool stage_i = ni <= kOffStageIns, stage_d = !CASC && nd <= kOffStageDel;
-    if (stage_i) for (uint64_t i = threadIdx.x; i < ni; i += kThreads) s_ins[i] = a.ins_row[ia + i];
-    if (stage_d) for (uint64_t i = threadIdx.x; i < nd; i += kThreads) s_del[i] = a.del_pos[da + i];
-    constexpr int PER = kOffTile / kThreads;
-    const uint64_t k0 = cta * kOffTile + threadIdx.x;
-    uint32_t u[PER];
-    int64_t x[PER];
-#pragma unroll
-    for (int j = 0; j < PER; ++j) {
-        uint64_t k = k0 + (uint64_t)j * kThreads;
-        u[j] = kNone32;
-        if (k < a.V_old) {
-            u[j] = REMAP ? a.remap[k] : (uint32_t)k;
-            x[j] = CASC ? a.KR[k] : a.old_off[k];
-        }
-    }
-    __syncthreads();
-#pragma unroll
-    for (int j = 0; j < PER; ++j) {
-        if (u[j] == kNone32) continue;
-        int64_t kept = x[j];
-        if (!CASC) {
-            uint64_t r = stage_d ? da + lower_bound_dev(s_del, 0, nd, (uint64_t)x[j])
-                                 : lower_bound_dev(a.del_pos, da, db, (uint64_t)x[j]);
-            kept -= (int64_t)r;
-        }
-        uint64_t ir = stage_i ? ia + lower_bound_dev(s_ins, 0, ni, u[j]) : lower_bound_dev(a.ins_row, ia, ib, u[j]);
-        a.new_off[u[j]] = kept + (int64_t)ir;
-    }
-}
-
 // Mode without node ops (identity ID map): the per-vertex degree delta
 // deg[u] = (#inserted records in row u) - (#deleted old edges in row u) is
 // scattered from the two sorted record lists, then one single-pass exclusive
@@ -1349,25 +1181,33 @@ __global__ void k_deg_scatter(const uint32_t* __restrict__ ins_row, uint64_t n_i
     }
 }
 
-// exclusive scan in place of the per-tile degree-delta sums (one CTA; nt <= ~1M)
-__global__ void __launch_bounds__(1024) k_tile_sum_scan(int64_t* __restrict__ tsum, uint64_t nt) {
-    __shared__ int64_t s_scan[1024 / 32 + 1];
-    __shared__ int64_t s_carry;
-    if (threadIdx.x == 0) s_carry = 0;
+// Device-wide exclusive scan of signed values (the per-tile degree-delta sums),
+// single pass with decoupled look-back.  Look-back words hold non-negative
+// values, so each tile aggregate is biased by +2^47 (|sum| < 2^36 per tile).
+__global__ void __launch_bounds__(kThreads) k_scan_exclusive_i64(const int64_t* __restrict__ in,
+        int64_t* __restrict__ out, uint64_t n, uint64_t* __restrict__ status, unsigned int* __restrict__ ctr) {
+    __shared__ uint32_t s_tile;
+    __shared__ int64_t s_scan[kThreads / 32 + 1];
+    __shared__ int64_t s_base;
+    if (threadIdx.x == 0) s_tile = atomicAdd(ctr, 1u);
     __syncthreads();
-    constexpr int PER = 8;
-    for (uint64_t c0 = 0; c0 < nt; c0 += 1024 * PER) {
-        const uint64_t i0 = c0 + (uint64_t)threadIdx.x * PER;
-        int64_t v[PER], sum = 0;
+    const uint32_t tile = s_tile;
+    const uint64_t i0 = (uint64_t)tile * kTile + (uint64_t)threadIdx.x * kItems;
+    int64_t v[kItems], sum = 0;
 #pragma unroll
-        for (int j = 0; j < PER; ++j) { v[j] = (i0 + j < nt) ? tsum[i0 + j] : 0; sum += v[j]; }
-        int64_t tot, ex = block_exclusive_scan<1024>(sum, s_scan, &tot);
-        int64_t run = s_carry + ex;
+    for (int j = 0; j < kItems; ++j) { v[j] = (i0 + j < n) ? in[i0 + j] : 0; sum += v[j]; }
+    int64_t tot, ex = block_exclusive_scan<kThreads>(sum, s_scan, &tot);
+    if (threadIdx.x < 32) {
+        const uint64_t bias = 1ull << 47;
+        uint64_t b = lookback_warp(status, tile, (uint64_t)(tot + (int64_t)bias));
+        if (lane_id() == 0) s_base = (int64_t)(b - (uint64_t)tile * bias);
+    }
+    __syncthreads();
+    int64_t run = s_base + ex;
 #pragma unroll
-        for (int j = 0; j < PER; ++j) { if (i0 + j < nt) tsum[i0 + j] = run; run += v[j]; }
-        __syncthreads();
-        if (threadIdx.x == 0) s_carry += tot;
-        __syncthreads();
+    for (int j = 0; j < kItems; ++j) {
+        if (i0 + j < n) out[i0 + j] = run;
+        run += v[j];
     }
 }
 
@@ -1449,22 +1289,41 @@ __global__ void __launch_bounds__(kThreads) k_offsets_scan(const int64_t* __rest
     }
 }
 
-template <bool CASC>
+// rows of inserted (new) vertices: kept old elements before the old position they
+// are inserted at, plus inserted records in rows < their new id
 __global__ void k_offsets_inserted(const NodeVtx* __restrict__ nv, const uint32_t* __restrict__ ins_q,
                                    uint64_t n_vins, const int64_t* __restrict__ old_off,
-                                   const int64_t* __restrict__ KR, const uint64_t* __restrict__ del_pos,
-                                   uint64_t n_del, const uint32_t* __restrict__ ins_row, uint64_t n_ins,
-                                   int64_t* __restrict__ new_off) {
+                                   const uint64_t* __restrict__ del_pos, uint64_t n_del,
+                                   const uint32_t* __restrict__ casc_mask, const uint64_t* __restrict__ casc_pre,
+                                   const uint32_t* __restrict__ ins_row, uint64_t n_ins, int64_t* __restrict__ new_off) {
     uint64_t i = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x;
     if (i >= n_vins) return;
     const NodeVtx& r = nv[ins_q[i]];
-    int64_t kept;
-    if (CASC) kept = KR[r.oldpos];
-    else {
-        uint64_t x = (uint64_t)old_off[r.oldpos];
-        kept = (int64_t)(x - lower_bound_dev(del_pos, 0, n_del, x));
+    const uint64_t x = (uint64_t)old_off[r.oldpos];
+    uint64_t kept = x - lower_bound_dev(del_pos, 0, n_del, x);
+    if (casc_mask) {
+        const uint64_t blk = x / kCascBlock;
+        uint64_t c = casc_pre[blk];
+        for (uint64_t q = blk * (kCascBlock / 32); q < (x >> 5); ++q) c += __popc(casc_mask[q]);
+        if (x & 31) c += __popc(casc_mask[x >> 5] & (0xFFFFFFFFu >> (32 - (x & 31))));
+        kept -= c;
     }
-    new_off[r.newid] = kept + (int64_t)lower_bound_dev(ins_row, 0, n_ins, r.newid);
+    new_off[r.newid] = (int64_t)(kept + lower_bound_dev(ins_row, 0, n_ins, r.newid));
+}
+
+// per 32 old ids: {new id of the group's first id (as if it survived), dropped bitmask};
+// kRemapExact if an inserted vertex lands strictly inside the group
+__global__ void k_remap32(uint64_t V, const uint32_t* __restrict__ dropped, uint64_t n_dropped,
+                          const uint32_t* __restrict__ ins_oldpos, uint64_t n_vins, uint2* __restrict__ out) {
+    const uint64_t g = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x;
+    if (g >= (V + 31) / 32) return;
+    const uint32_t c0 = (uint32_t)(g * 32);
+    const uint64_t d0 = lower_bound_dev(dropped, 0, n_dropped, c0);
+    const uint64_t i0 = upper_bound_dev(ins_oldpos, 0, n_vins, c0);
+    const uint64_t i1 = upper_bound_dev(ins_oldpos, i0, n_vins, c0 + 31);
+    uint32_t m = 0;
+    for (uint64_t d = d0; d < n_dropped && dropped[d] < c0 + 32; ++d) m |= 1u << (dropped[d] - c0);
+    out[g] = make_uint2(i1 > i0 ? kRemapExact : (uint32_t)(c0 - d0 + i0), m);
 }
 
 __global__ void k_set_i64(int64_t* p, int64_t v) { *p = v; }

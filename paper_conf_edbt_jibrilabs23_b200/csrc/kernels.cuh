@@ -664,7 +664,7 @@ __global__ void __launch_bounds__(kThreads) k_reduce_classify(ClassArgs a) {
 constexpr int kMergeTile = 2048;             // merged items per tile
 constexpr int kCascBlock = 2048;             // cascade mask: elements per counted block (64 words)
 constexpr int kMergeBuf = kMergeTile + 8;     // staged old elements (+ 16 B alignment slack)
-constexpr int kRemapBlockShift = 10;          // two-level remap: 1024 old ids per block
+constexpr int kRemapBlockShift = 16;          // two-level remap: 64K old ids per block (L1-resident table)
 constexpr int32_t kRemapMixed = INT32_MIN;    // block has a dropped/inserted id inside
 
 struct MergeArgs {
@@ -682,7 +682,7 @@ struct MergeArgs {
     const float* upd_w;
     uint64_t n_upd;
     const uint32_t* remap;
-    const int32_t* remap_shift;  // per 1024-block constant shift or kRemapMixed
+    const int32_t* remap_shift;  // per 64K-id block: constant shift or kRemapMixed
     const uint32_t* hd_bits;
     const uint32_t* hd_rows;
     uint64_t n_hd;
@@ -707,6 +707,7 @@ struct MergeArgs {
 // and the ranks of j in the sorted delete / update / cascade-row lists.
 struct TilePart {
     uint64_t r, dl, ul, k, ir;  // k: first old row starting at or after j; ir: ins-row rank of k's new id
+    uint64_t cb;                // cascade mode: cascaded old elements before j
 };
 
 __device__ __forceinline__ uint64_t ins_split(const uint64_t* ins_pos, uint64_t n_ins, uint64_t d) {
@@ -728,7 +729,14 @@ __global__ void k_merge_partition(MergeArgs a, TilePart* __restrict__ part) {
     const uint64_t j = d - p.r;
     p.dl = lower_bound_dev(a.del_pos, 0, a.n_del, j);
     p.ul = lower_bound_dev(a.upd_pos, 0, a.n_upd, j);
-    p.k = p.ir = 0;
+    p.k = p.ir = p.cb = 0;
+    if (a.casc_mask) {  // cascaded elements before j: block prefix + popcount of the partial block
+        const uint64_t blk = j / kCascBlock;
+        uint64_t c = a.casc_pre[blk];
+        for (uint64_t q = blk * (kCascBlock / 32); q < (j >> 5); ++q) c += __popc(a.casc_mask[q]);
+        if (j & 31) c += __popc(a.casc_mask[j >> 5] & (0xFFFFFFFFu >> (32 - (j & 31))));
+        p.cb = c;
+    }
     if (a.rows) {
         p.k = lower_bound_dev(a.old_off, 0, a.V_old + 1, (int64_t)j);
         if (p.k >= a.V_old) p.ir = a.n_ins;
@@ -879,7 +887,7 @@ constexpr uint32_t kRemapExact = 0xFFFFFFFFu;  // remap32 base: group needs the 
 constexpr int kRowStage = 512;                 // rows mode: insert-row slice staged in smem
 
 // new dense id of surviving old vertex `col` (REMAP mode): constant shift of its
-// 1024-block, else base of its 32-group minus the dropped ids below it
+// 64K-id block, else base of its 32-group minus the dropped ids below it
 __device__ __forceinline__ uint32_t remap_col(const MergeArgs& a, uint32_t col) {
     const int32_t shf = a.remap_shift[col >> kRemapBlockShift];
     if (shf != kRemapMixed) return (uint32_t)((int64_t)col + shf);
@@ -924,6 +932,7 @@ __global__ void __launch_bounds__(kThreads) k_merge3(MergeArgs a, const TilePart
     __shared__ __align__(8) uint64_t s_bar[2];
     __shared__ uint64_t s_meta[2][5];
     __shared__ uint64_t s_rows[2][4];
+    __shared__ uint64_t s_cb[2];
     __shared__ uint32_t s_irow[kRowStage];  // rows mode: the tile's slice of insert rows
     __shared__ uint64_t s_cbefore;
 
@@ -937,6 +946,7 @@ __global__ void __launch_bounds__(kThreads) k_merge3(MergeArgs a, const TilePart
         s_meta[b][0] = p0.r; s_meta[b][1] = p1.r; s_meta[b][2] = p0.dl; s_meta[b][3] = p0.ul;
         s_meta[b][4] = (p1.dl - p0.dl) | ((p1.ul - p0.ul) << 16);
         s_rows[b][0] = p0.k; s_rows[b][1] = p1.k; s_rows[b][2] = p0.ir; s_rows[b][3] = p1.ir;
+        s_cb[b] = p0.cb;
         const uint64_t j0 = min(t * kMergeTile, Dtot) - p0.r, j1 = min((t + 1) * kMergeTile, Dtot) - p1.r;
         const uint64_t a0 = j0 & ~3ull, a1 = (j1 + 3) & ~3ull;
         const uint32_t bytes = (uint32_t)((a1 - a0) * 4);
@@ -983,16 +993,19 @@ __global__ void __launch_bounds__(kThreads) k_merge3(MergeArgs a, const TilePart
         }
         for (uint32_t q = tid; q < n_irs && q < kRowStage; q += kThreads) s_irow[q] = a.ins_row[ir0 + q];
         if (tid < NCH + 2) { s_dmask[tid] = 0; s_icnt[tid] = 0; }
-        if (CASC && wid == 1) {  // cascaded elements before j0 (block prefix + partial popcount)
-            const uint64_t blk = j0 / kCascBlock, wb = blk * (kCascBlock / 32), we = j0 >> 5;
-            uint32_t c = 0;
-            for (uint64_t q = wb + lane; q <= we; q += 32) {
-                uint32_t m = a.casc_mask[q];
-                if (q == we) m &= (j0 & 31) ? (0xFFFFFFFFu >> (32 - (j0 & 31))) : 0u;
-                c += __popc(m);
+        const uint64_t cbefore = CASC ? s_cb[b] : 0;  // cascaded old elements before j0
+        // phase A inputs of warp 0: the cascade-mask words under its two chunks
+        uint32_t pf_cm[4] = {0u, 0u, 0u, 0u};
+        if (CASC && wid == 0) {
+#pragma unroll
+            for (int h = 0; h < 2; ++h) {
+                const uint32_t i0 = (2 * lane + h) * 32;
+                if (i0 < n_old) {
+                    const uint64_t x = j0 + i0, q = x >> 5;
+                    pf_cm[2 * h] = a.casc_mask[q];
+                    pf_cm[2 * h + 1] = (x & 31) ? a.casc_mask[q + 1] : 0u;
+                }
             }
-            c = warp_sum(c);
-            if (lane == 0) s_cbefore = a.casc_pre[blk] + c;
         }
         __syncthreads();
         for (uint32_t i = tid; i < nd; i += kThreads) {
@@ -1014,11 +1027,7 @@ __global__ void __launch_bounds__(kThreads) k_merge3(MergeArgs a, const TilePart
                 const uint32_t c = 2 * lane + h, i0 = c * 32;
                 uint32_t v = (i0 >= n_old) ? 0u : (n_old - i0 >= 32 ? 0xFFFFFFFFu : (0xFFFFFFFFu >> (32 - (n_old - i0))));
                 v &= ~s_dmask[c];
-                if (CASC && v) {
-                    const uint64_t x = j0 + i0, q = x >> 5;
-                    const uint32_t lo = a.casc_mask[q], hi = (x & 31) ? a.casc_mask[q + 1] : 0u;
-                    v &= ~__funnelshift_r(lo, hi, (uint32_t)(x & 31));
-                }
+                if (CASC && v) v &= ~__funnelshift_r(pf_cm[2 * h], pf_cm[2 * h + 1], (uint32_t)((j0 + i0) & 31));
                 m[h] = v;
                 s_mask[c] = v;
             }
@@ -1042,7 +1051,7 @@ __global__ void __launch_bounds__(kThreads) k_merge3(MergeArgs a, const TilePart
         __syncthreads();
         const uint32_t kept = s_cbase[NCH];
         const uint32_t n_out = kept + ni;
-        const uint64_t base = j0 - dl0 - (CASC ? s_cbefore : 0) + r0;
+        const uint64_t base = j0 - dl0 - cbefore + r0;
         const uint32_t ob = (uint32_t)(base & 3);
         // phase B: old elements, output index = kept before + inserted at positions <= i.
         // Warp w owns chunks w, w+8, ..., w+56; the 8 chunks are unrolled so that the
@@ -1101,7 +1110,7 @@ __global__ void __launch_bounds__(kThreads) k_merge3(MergeArgs a, const TilePart
         if (a.rows) {
             // a4/a5 fused: new_off[u'] of every surviving old row k starting in this tile
             //   = (kept old elements before its old start) + (inserted records in rows < u')
-            const uint64_t kb0 = j0 - dl0 - (CASC ? s_cbefore : 0);  // kept old elements before j0
+            const uint64_t kb0 = j0 - dl0 - cbefore;  // kept old elements before j0
             const bool staged = n_irs <= kRowStage;
             for (uint32_t q = tid; q < n_rows; q += kThreads) {
                 const bool pf = q < 2 * kThreads;
@@ -1139,7 +1148,7 @@ __global__ void __launch_bounds__(kThreads) k_merge3(MergeArgs a, const TilePart
     if (tid == 0) bulk_wait_all();
 }
 
-// per 1024-block of old ids: constant new-id shift, or kRemapMixed if a dropped
+// per 64K-id block of old ids: constant new-id shift, or kRemapMixed if a dropped
 // id or an inserted id's insertion point lies strictly inside the block
 __global__ void k_remap_blocks(uint64_t V, const uint32_t* __restrict__ dropped, uint64_t n_dropped,
                                const uint32_t* __restrict__ ins_oldpos, uint64_t n_ins, int32_t* __restrict__ shift) {

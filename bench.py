@@ -304,6 +304,10 @@ def run_gpu(args):
         ms_step = ms / len(stats)
         path_gbs = path_bytes / (ms_step / 1e3) / 1e9
         info = rep.info()
+        try:  # DRAM bytes per launch of the same kernel from the committed ncu --set full capture
+            traffic = json.load(open(os.path.join(ROOT, "profiles", "traffic.json"))).get(args.config)
+        except Exception:
+            traffic = None
         line = {
             "metric": METRIC, "value": value, "unit": "updates/s", "n_gpus": world,
             "steps": args.steps, "warmup": args.warmup, "ms_per_step": ms_max / args.steps,
@@ -314,7 +318,8 @@ def run_gpu(args):
                        "l2": "inputs larger than L2 (CSR ~%.1f GB per step)" % (path_bytes / 1e9),
                        "replica_vertices": info["n_vertices"], "replica_edges": info["n_edges"]},
             "roofline": {"bound": "hbm", "kernel": "k_merge", "achieved": achieved, "peak": peak,
-                         "unit": "GB/s", "frac": achieved / peak, "traffic": None,
+                         "unit": "GB/s", "frac": achieved / peak, "traffic": traffic,
+                         "traffic_source": "ncu --set full, profiles/r1/summary.json (dram read+write per launch)",
                          "peak_source": peak_src, "bytes_per_launch": merge_bytes,
                          "ms_per_launch": merge_ms},
             "path": {"bytes_alg_per_step": path_bytes, "achieved_gbs": path_gbs,

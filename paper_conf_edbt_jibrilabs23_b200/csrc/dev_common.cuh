@@ -127,6 +127,24 @@ __device__ __forceinline__ uint64_t upper_bound_dev(const T* a, uint64_t lo, uin
     return lo;
 }
 
+// lower_bound over a sorted u64 array: a few interpolation steps between the
+// known key bounds (external IDs are near-arithmetic runs), then bisection
+__device__ __forceinline__ uint64_t interp_lower_bound(const uint64_t* a, uint64_t lo, uint64_t hi, uint64_t key) {
+    if (lo >= hi) return lo;
+    uint64_t vlo = a[lo], vhi = a[hi - 1];
+    if (key <= vlo) return lo;
+    if (key > vhi) return hi;
+    // invariant: a[lo] < key <= a[hi-1] (so lo < hi - 1 here)
+    for (int step = 0; step < 6 && hi - lo > 16; ++step) {
+        const double f = (double)(key - vlo) / (double)(vhi - vlo);
+        uint64_t mid = lo + 1 + (uint64_t)(f * (double)(hi - lo - 2));
+        if (mid >= hi - 1) mid = hi - 2;
+        const uint64_t v = a[mid];
+        if (v < key) { lo = mid; vlo = v; } else { hi = mid + 1; vhi = v; }
+    }
+    return lower_bound_dev(a, lo + 1, hi, key);
+}
+
 // Stable compaction of a tile of kThreads x ITEMS items in STRIPED order (item k of
 // thread t is tile item k*NT + t, so global loads coalesce): flag[k] -> pos[k] =
 // rank of the item among flagged items of the tile.  smem: ITEMS*NT/32 + 1 words.

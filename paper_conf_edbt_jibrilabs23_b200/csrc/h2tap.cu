@@ -4,7 +4,7 @@
 // replica's stream:
 //   a1 k_partition         validate, number, split pending / node ops / edge ops
 //   a2 node ops            radix sort by (v, ts, seq), k_node_segments, k_node_lists,
-//                          k_remap + k_place_inserted (ID-map compaction), hd bitmap
+//                          remap tables + k_new_ext + k_place_inserted (ID-map compaction)
 //   a3 edge ops            k_edge_prep (lookup, gating, packed key), onesweep radix
 //                          sort, k_reduce_classify (latest-commit-wins + outcome lists)
 //   a6 k_merge             global merge path into the back buffer
@@ -14,6 +14,7 @@
 #include <cuda_runtime.h>
 
 #include <cstdarg>
+#include <cstdlib>
 #include <cstdio>
 #include <cstring>
 #include <new>
@@ -63,6 +64,42 @@ struct Buf {
 };
 
 inline uint64_t cdiv(uint64_t a, uint64_t b) { return (a + b - 1) / b; }
+
+// Opt-in step trace (H2TAP_TRACE=1): events recorded on the replica's stream at every
+// step boundary, printed as device-time deltas at the end of each apply.
+struct Trace {
+    bool on = false;
+    int n = 0;
+    const char* name[48];
+    cudaEvent_t ev[48];
+    void init() {
+        const char* e = getenv("H2TAP_TRACE");
+        on = e && *e && *e != '0';
+        if (on && !ev[0]) for (auto& x : ev) cudaEventCreate(&x);
+        n = 0;
+    }
+    void mark(const char* nm, cudaStream_t st) {
+        if (!on || n >= 48) return;
+        name[n] = nm;
+        cudaEventRecord(ev[n++], st);
+    }
+    void dump() {
+        if (!on || n < 2) return;
+        cudaEventSynchronize(ev[n - 1]);
+        fprintf(stderr, "[h2tap trace]");
+        for (int i = 1; i < n; ++i) {
+            float ms = 0;
+            cudaEventElapsedTime(&ms, ev[i - 1], ev[i]);
+            fprintf(stderr, " %s=%.1fus", name[i], ms * 1e3f);
+        }
+        float tot = 0;
+        cudaEventElapsedTime(&tot, ev[0], ev[n - 1]);
+        fprintf(stderr, " | total=%.1fus\n", tot * 1e3f);
+    }
+    Trace() { for (auto& x : ev) x = nullptr; }
+};
+thread_local Trace g_tr;
+#define TR(nm) g_tr.mark(nm, st)
 inline int bits_for(uint64_t range) { return range == 0 ? 0 : 64 - __builtin_clzll(range); }
 
 }  // namespace
@@ -80,10 +117,10 @@ struct h2tap_replica {
     // scratch
     Buf Wk, Ws, Wd, Ww, Wt, Wq, idx_p, idx_n, idx_e, status;
     Buf keyA, keyB, valA, valB, hist, dbase, rs_status, rs_ctr;
-    Buf nv, nv_ext, dropped, ins_q, ins_oldpos, hd_rows, remap, hd_bits;
+    Buf nv, nv_ext, dropped, ins_q, ins_oldpos, hd_rows, hd_bits;
     Buf op_flags, op_ou, op_ow;
     Buf ins_pos, ins_row, ins_col, ins_w, del_pos, upd_pos, upd_w, KR;
-    Buf misc, nsorted, part, opart, deg, tsum, remap_shift, remap32, tile_emit, tile_base, del_row, casc_mask, status2, bfs_a, bfs_b, pr_a, pr_b;
+    Buf misc, nsorted, part, opart, deg, tsum, remap_shift, remap32, casc_wrel, tile_emit, tile_base, del_row, casc_mask, status2, bfs_a, bfs_b, pr_a, pr_b;
     Buf ctr;
     Counters* hc = nullptr;  // pinned host mirror
     cudaEvent_t ev[8]{};
@@ -227,9 +264,11 @@ h2tap_status apply_core(h2tap_replica* r, const BatchIn& in, uint64_t S, bool cr
     const uint64_t n = in.n, np = r->n_pend, m = np + n;
     if (m >= 0xFFFFFFFFull) { set_err("batch + pending = %llu ops exceeds 2^32-1", (unsigned long long)m); return H2TAP_E_CAPACITY; }
     g_launches = g_h2d = g_d2h = 0;
+    g_tr.init();
     for (int i = 0; i < 8; ++i)
         if (!r->ev[i]) CK(cudaEventCreate(&r->ev[i]));
     CK(cudaEventRecord(r->ev[0], st));
+    TR("start");
 
     // ---- a1: assemble work ops (pending ++ batch) and partition
     uint8_t* Wk = r->get<uint8_t>(r->Wk, m);
@@ -282,7 +321,9 @@ h2tap_status apply_core(h2tap_replica* r, const BatchIn& in, uint64_t S, bool cr
                                                        stt, nt, dc);
         CKL();
     }
+    TR("assemble+partition");
     r->read_counters();
+    TR("sync1");
     Counters hc = *r->hc;
     if (hc.status & ST_BAD_KIND) { set_err("unknown op kind in batch"); return H2TAP_E_INVAL; }
     if (hc.status & ST_STALE) {
@@ -300,11 +341,13 @@ h2tap_status apply_core(h2tap_replica* r, const BatchIn& in, uint64_t S, bool cr
     bool remap_on = false, set_changed = false;
     NodeVtx* nv = nullptr;
     uint64_t* nv_ext = nullptr;
-    uint32_t *dropped = nullptr, *ins_q = nullptr, *ins_oldpos = nullptr, *hd_rows = nullptr, *remap = nullptr,
+    RemapView R{};  // identity unless node ops shift the dense ids
+    uint32_t *dropped = nullptr, *ins_q = nullptr, *ins_oldpos = nullptr, *hd_rows = nullptr,
              *hd_bits = nullptr, *node_sorted = nullptr;
     uint64_t* new_ext = nullptr;
     uint32_t* casc_mask = nullptr;
     uint64_t *casc_cnt = nullptr, *casc_pre = nullptr;
+    uint16_t* casc_wrel = nullptr;
     const int64_t* old_off_nc = static_cast<const int64_t*>(r->off[r->cur].p);
     const uint32_t* old_cols_nc = static_cast<const uint32_t*>(r->cols[r->cur].p);
     if (n_node) {
@@ -321,6 +364,7 @@ h2tap_status apply_core(h2tap_replica* r, const BatchIn& in, uint64_t S, bool cr
         std::swap(kA, kB);
         std::swap(vA, vB);
         radix_sort(r, kA, vA, kB, vB, n_node, bits_for(hc.v_max - hc.v_min));
+        TR("node_sort");
         node_sorted = r->get<uint32_t>(r->nsorted, n_node);
         CK(cudaMemcpyAsync(node_sorted, vA, n_node * 4, cudaMemcpyDeviceToDevice, st));
 
@@ -332,7 +376,9 @@ h2tap_status apply_core(h2tap_replica* r, const BatchIn& in, uint64_t S, bool cr
         k_node_segments<<<(unsigned)nt, kThreads, 0, st>>>(ops, node_sorted, n_node, ext_index(r), nv, nv_ext,
                                                            stt, nt, dc);
         CKL();
+        TR("node_segments");
         r->read_counters();
+        TR("sync_nseg");
         U = r->hc->n_unique;
         dropped = r->get<uint32_t>(r->dropped, U);
         ins_q = r->get<uint32_t>(r->ins_q, U);
@@ -344,7 +390,9 @@ h2tap_status apply_core(h2tap_replica* r, const BatchIn& in, uint64_t S, bool cr
         k_node_lists<<<(unsigned)nt2, kThreads, 0, st>>>(nv, U, dropped, ins_q, ins_oldpos, hd_rows, stt, nt2, dc);
         CKL();
         uint32_t first_ins_oldpos = 0;
+        TR("node_lists");
         r->read_counters();
+        TR("sync_nlists");
         n_dropped = r->hc->n_dropped;
         n_vins = r->hc->n_inserted;
         n_hd = r->hc->n_hd;
@@ -355,18 +403,22 @@ h2tap_status apply_core(h2tap_replica* r, const BatchIn& in, uint64_t S, bool cr
             first_ins_oldpos = (uint32_t)(r->hc->status & 0xFFFFFFFFu);
         }
         Vn = V - n_dropped + n_vins;
-        if (Vn >= 0xFFFFFFFFull) { set_err("vertex count exceeds 2^32-1"); return H2TAP_E_CAPACITY; }
+        if (Vn >= 0x7FFFFFFFull) { set_err("vertex count exceeds 2^31-1"); return H2TAP_E_CAPACITY; }
         set_changed = n_dropped || n_vins;
         remap_on = n_dropped > 0 || (n_vins > 0 && first_ins_oldpos < V);
         if (set_changed) {
             new_ext = r->get<uint64_t>(r->ext[ec ^ 1], Vn);
             if (remap_on) {
-                remap = r->get<uint32_t>(r->remap, V);
-                if (V) {
-                    k_remap<<<g1(V, kRemapTile), kThreads, 0, st>>>(old_ext, r->identity, V, dropped, n_dropped,
-                                                                    ins_oldpos, n_vins, remap, new_ext);
-                    CKL();
-                }
+                // remap tables (64K-id block shifts, 32-id groups), then scatter the survivors
+                const uint64_t nblk = cdiv(V, 1ull << kRemapBlockShift), ng = cdiv(V, 32);
+                int32_t* rs = r->get<int32_t>(r->remap_shift, nblk);
+                uint2* r32 = r->get<uint2>(r->remap32, ng);
+                if (nblk) { k_remap_blocks<<<g1(nblk), 256, 0, st>>>(V, dropped, n_dropped, ins_oldpos, n_vins, rs); CKL(); }
+                if (ng) { k_remap32<<<g1(ng), 256, 0, st>>>(V, dropped, n_dropped, ins_oldpos, n_vins, r32); CKL(); }
+                R.shift = rs; R.g32 = r32; R.ins_oldpos = ins_oldpos; R.n_vins = n_vins;
+                TR("remap_tables");
+                if (V) { k_new_ext<<<g1(V), 256, 0, st>>>(old_ext, r->identity, V, R, new_ext); CKL(); }
+                TR("new_ext");
             } else if (V) {
                 CK(cudaMemcpyAsync(new_ext, old_ext, V * 8, cudaMemcpyDeviceToDevice, st));
             }
@@ -381,7 +433,7 @@ h2tap_status apply_core(h2tap_replica* r, const BatchIn& in, uint64_t S, bool cr
             r->identity_pending = false;
             build_fence(r, ec ^ 1, Vn);
         }
-        k_nv_newid<<<g1(U), 256, 0, st>>>(nv, U, remap, remap_on ? 1 : 0);
+        k_nv_newid<<<g1(U), 256, 0, st>>>(nv, U, R);
         CKL();
         if (n_hd) {
             hd_bits = r->get<uint32_t>(r->hd_bits, cdiv(V, 32));
@@ -390,30 +442,34 @@ h2tap_status apply_core(h2tap_replica* r, const BatchIn& in, uint64_t S, bool cr
             CKL();
             // cascade pass on the side stream, overlapped with the edge-op phase
             const uint64_t nblk = cdiv(E, kCascBlock);
-            casc_mask = r->get<uint32_t>(r->casc_mask, (nblk + 1) * (kCascBlock / 32));
+            casc_mask = r->get<uint32_t>(r->casc_mask, (nblk + 2) * (kCascBlock / 32));
             casc_cnt = r->get<uint64_t>(r->tile_emit, nblk + 1);
             casc_pre = r->get<uint64_t>(r->tile_base, nblk + 1);
-            CK(cudaEventRecord(r->evA, st));
-            CK(cudaStreamWaitEvent(r->st2, r->evA, 0));
-            cudaStream_t s2 = r->st2;
+            // in-line on the main stream: overlapping this streaming pass with the
+            // latency-bound edge-op kernels only delayed them (H2TAP_TRACE measurements)
+            cudaStream_t s2 = st;
             unsigned rg = (unsigned)std::min<uint64_t>(cdiv(n_hd * 32, 256), (uint64_t)r->n_sm * 8);
             const uint64_t nst = cdiv(nblk + 1, kThreads);
             uint64_t* st2s2 = r->get<uint64_t>(r->status2, nst);
             CK(cudaMemsetAsync(st2s2, 0, nst * 8, s2));
+            TR("nv_newid+bits");
             if (nblk) {
-                k_casc_cols<<<(unsigned)nblk, kThreads, 0, s2>>>(old_cols_nc, E, hd_bits, casc_mask);
+                k_casc_cols<<<(unsigned)cdiv(nblk, 2), kThreads, 0, s2>>>(old_cols_nc, E, hd_bits, hd_rows, n_hd, casc_mask);
                 CKL();
+                TR("casc_cols");
                 k_casc_rows<<<rg, 256, 0, s2>>>(old_off_nc, hd_rows, n_hd, casc_mask);
                 CKL();
+                TR("casc_rows");
             }
-            k_casc_scan<<<(unsigned)nst, kThreads, 0, s2>>>(casc_mask, nblk, casc_pre, st2s2, &dc->tiles[6]);
+            casc_wrel = r->get<uint16_t>(r->casc_wrel, (nblk + 1) * (kCascBlock / 32));
+            k_casc_scan<<<(unsigned)nst, kThreads, 0, s2>>>(casc_mask, nblk, casc_pre, casc_wrel, st2s2, &dc->tiles[6]);
             CKL();
             k_copy_u64<<<1, 1, 0, s2>>>(&dc->n_casc, casc_pre + nblk);
             CKL();
-            CK(cudaEventRecord(r->evB, s2));
         }
     }
     CK(cudaEventRecord(r->ev[2], st));
+    TR("idmap+remap");
 
     // ---- a3: edge ops -> keys, sort, segmented reduce + classify
     const int bits = std::max(1, bits_for(Vn > 1 ? Vn - 1 : 1));
@@ -438,7 +494,7 @@ h2tap_status apply_core(h2tap_replica* r, const BatchIn& in, uint64_t S, bool cr
         pa.edge_idx = idx_e;
         pa.n_edge = n_edge;
         pa.X = ext_index(r);
-        pa.remap = remap_on ? remap : nullptr;
+        pa.R = R;
         pa.nv = nv;
         pa.nv_ext = nv_ext;
         pa.U = U;
@@ -447,17 +503,20 @@ h2tap_status apply_core(h2tap_replica* r, const BatchIn& in, uint64_t S, bool cr
         pa.create = create ? 1 : 0;
         pa.keys = kA;
         pa.vals = vA;
-        pa.op_flags = r->get<uint8_t>(r->op_flags, m);
-        pa.op_opos_u = r->get<uint32_t>(r->op_ou, m);
-        pa.op_opos_w = r->get<uint32_t>(r->op_ow, m);
-        uint64_t nt = cdiv(n_edge, kTile);
+        pa.recs = r->get<EdgeRec>(r->op_flags, m);
+        const bool lookups_direct = r->identity && U == 0;  // no searches -> 8 ops per thread
+        const int eitems = lookups_direct ? 8 : 1;
+        uint64_t nt = cdiv(n_edge, (uint64_t)kThreads * eitems);
         pa.status = r->get<uint64_t>(r->status, 3 * nt);
         CK(cudaMemsetAsync(pa.status, 0, nt * 8, st));
         pa.n_tiles = nt;
         pa.c = dc;
-        k_edge_prep<<<(unsigned)nt, kThreads, 0, st>>>(pa);
+        if (lookups_direct) k_edge_prep<8><<<(unsigned)nt, kThreads, 0, st>>>(pa);
+        else k_edge_prep<1><<<(unsigned)nt, kThreads, 0, st>>>(pa);
         CKL();
+        TR("edge_prep");
         r->read_counters();
+        TR("sync_prep");
         if (create && (r->hc->status & ST_CREATE_ENDPOINT)) {
             set_err("create: edge endpoint not in the vertex set");
             return H2TAP_E_INVAL;
@@ -465,6 +524,7 @@ h2tap_status apply_core(h2tap_replica* r, const BatchIn& in, uint64_t S, bool cr
         n_valid = r->hc->n_valid;
         n_gated = r->hc->n_gated;
         radix_sort(r, kA, vA, kB, vB, n_valid, 2 * bits);
+        TR("edge_sort");
         ins_pos = r->get<uint64_t>(r->ins_pos, n_valid);
         ins_row = r->get<uint32_t>(r->ins_row, n_valid);
         ins_col = r->get<uint32_t>(r->ins_col, n_valid);
@@ -480,9 +540,7 @@ h2tap_status apply_core(h2tap_replica* r, const BatchIn& in, uint64_t S, bool cr
             ca.vals = vA;
             ca.n = n_valid;
             ca.bits = bits;
-            ca.op_flags = pa.op_flags;
-            ca.op_opos_u = pa.op_opos_u;
-            ca.op_opos_w = pa.op_opos_w;
+            ca.recs = pa.recs;
             ca.old_off = old_off;
             ca.old_cols = old_cols;
             ca.V_old = V;
@@ -497,7 +555,9 @@ h2tap_status apply_core(h2tap_replica* r, const BatchIn& in, uint64_t S, bool cr
             ca.c = dc;
             k_reduce_classify<<<(unsigned)nt2, kThreads, 0, st>>>(ca);
             CKL();
+            TR("classify");
             r->read_counters();
+            TR("sync_cls");
             n_ins = r->hc->n_ins;
             n_del = r->hc->n_del;
             n_upd = r->hc->n_upd;
@@ -522,35 +582,22 @@ h2tap_status apply_core(h2tap_replica* r, const BatchIn& in, uint64_t S, bool cr
         ma.ins_pos = ins_pos; ma.ins_col = ins_col; ma.ins_w = ins_w; ma.n_ins = n_ins;
         ma.del_pos = del_pos; ma.n_del = n_del;
         ma.upd_pos = upd_pos; ma.upd_w = upd_w; ma.n_upd = n_upd;
-        ma.remap = remap; ma.hd_bits = hd_bits; ma.hd_rows = hd_rows; ma.n_hd = n_hd;
+        ma.R = R; ma.hd_bits = hd_bits; ma.hd_rows = hd_rows; ma.n_hd = n_hd;
         ma.new_cols = new_cols; ma.new_w = new_w;
-        ma.rows = n_node ? 1 : 0;
+        ma.rows = 0;  // row offsets: k_offsets_rows (a separate, row-balanced pass)
         ma.new_off = new_off; ma.ins_row = ins_row;
         ma.dropped = dropped; ma.n_dropped = n_dropped; ma.ins_oldpos = ins_oldpos; ma.n_vins = n_vins;
         ma.n_tiles = cdiv(Dtot, kMergeTile);
         ma.c = dc;
-        if (remap_on) {
-            const uint64_t nblk = cdiv(V, 1u << kRemapBlockShift);
-            int32_t* rs = r->get<int32_t>(r->remap_shift, nblk);
-            if (nblk) {
-                k_remap_blocks<<<g1(nblk), 256, 0, st>>>(V, dropped, n_dropped, ins_oldpos, n_vins, rs);
-                CKL();
-            }
-            ma.remap_shift = rs;
-            const uint64_t ng = cdiv(V, 32);
-            uint2* r32 = r->get<uint2>(r->remap32, ng);
-            if (ng) { k_remap32<<<g1(ng), 256, 0, st>>>(V, dropped, n_dropped, ins_oldpos, n_vins, r32); CKL(); }
-            ma.remap32 = r32;
-        }
         if (casc) {
             ma.casc_mask = casc_mask;
             ma.casc_pre = casc_pre;
-            CK(cudaStreamWaitEvent(st, r->evB, 0));
         }
         TilePart* part = r->get<TilePart>(r->part, ma.n_tiles + 1);
         k_merge_partition<<<g1(ma.n_tiles + 1), 256, 0, st>>>(ma, part);
         CKL();
         CK(cudaEventRecord(r->ev[6], st));  // merge kernel starts here (after its prerequisites)
+        TR("merge_prep+casc_join");
         auto launch = [&](auto kern) {
             int occ = 0;
             CK(cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, kMerge3Smem));
@@ -564,12 +611,12 @@ h2tap_status apply_core(h2tap_replica* r, const BatchIn& in, uint64_t S, bool cr
         else launch(k_merge3<false, false>);
         CKL();
     } else {
-        if (casc) CK(cudaStreamWaitEvent(st, r->evB, 0));
         // nothing to merge: every surviving row is empty
         if (n_node) CK(cudaMemsetAsync(new_off, 0, (Vn + 1) * 8, st));
         CK(cudaEventRecord(r->ev[6], st));
     }
     CK(cudaEventRecord(r->ev[4], st));
+    TR("merge");
     if (casc) {
         r->read_counters();
         n_casc = r->hc->n_casc;
@@ -597,11 +644,23 @@ h2tap_status apply_core(h2tap_replica* r, const BatchIn& in, uint64_t S, bool cr
         k_offsets_apply<<<(unsigned)nt, kThreads, 0, st>>>(old_off, deg, V, tbase, new_off);
         CKL();
     }
-    // (with node ops the merge kernel wrote the offsets of surviving old rows)
-    if (n_vins) {
-        k_offsets_inserted<<<g1(n_vins), 256, 0, st>>>(nv, ins_q, n_vins, old_off, del_pos, n_del, casc ? casc_mask : nullptr,
-                                                       casc_pre, ins_row, n_ins, new_off);
+    if (V && n_node) {
+        RowArgs ra{};
+        ra.old_off = old_off; ra.V_old = V; ra.E_old = E; ra.R = R;
+        ra.casc_mask = casc ? casc_mask : nullptr; ra.casc_pre = casc_pre; ra.casc_wrel = casc_wrel;
+        ra.del_pos = del_pos; ra.n_del = n_del; ra.ins_row = ins_row; ra.n_ins = n_ins;
+        ra.dropped = dropped; ra.n_dropped = n_dropped; ra.ins_oldpos = ins_oldpos; ra.n_vins = n_vins;
+        ra.new_off = new_off;
+        const uint64_t ncta = cdiv(V, kRowTile);
+        ra.part = r->get<uint64_t>(r->opart, 2 * (ncta + 1));
+        k_rows_partition<<<g1(ncta + 1), 256, 0, st>>>(ra);
         CKL();
+        k_offsets_rows<<<(unsigned)ncta, kThreads, 0, st>>>(ra);
+        CKL();
+        if (n_vins) {
+            k_offsets_inserted<<<g1(n_vins), 256, 0, st>>>(nv, ins_q, n_vins, ra);
+            CKL();
+        }
     }
     k_set_i64<<<1, 1, 0, st>>>(new_off + Vn, (int64_t)En);
     CKL();
@@ -620,6 +679,7 @@ h2tap_status apply_core(h2tap_replica* r, const BatchIn& in, uint64_t S, bool cr
         CKL();
     }
     CK(cudaEventRecord(r->ev[5], st));
+    TR("offsets+pending");
     bool new_identity = r->identity;
     if (set_changed) {
         if (Vn == 0) new_identity = true;
@@ -633,6 +693,8 @@ h2tap_status apply_core(h2tap_replica* r, const BatchIn& in, uint64_t S, bool cr
         }
     }
     r->sync();
+    TR("end");
+    g_tr.dump();
 
     // ---- a7: swap at snapshot_ts (nothing above touched the front state)
     r->cur = nb;
@@ -671,7 +733,6 @@ h2tap_status apply_core(h2tap_replica* r, const BatchIn& in, uint64_t S, bool cr
         uint64_t bm = 0;
         if (csr_changed && E + n_ins) {
             bm = 8 * E + 8 * En + 20 * n_ins + 8 * n_del + 12 * n_upd;
-            if (n_node) bm += 8 * V + 8 * Vn + (remap_on ? 4 * V : 0);  // fused row offsets
             if (n_hd) bm += E / 8;                                       // cascade mask
         }
         stats->bytes_merge = bm;
@@ -711,7 +772,12 @@ h2tap_replica* new_replica(const h2tap_config* cfg) {
     CK(cudaSetDevice(r->cfg.device));
     CK(cudaDeviceGetAttribute(&r->n_sm, cudaDevAttrMultiProcessorCount, r->cfg.device));
     r->st = static_cast<cudaStream_t>(r->cfg.stream);
-    CK(cudaStreamCreateWithFlags(&r->st2, cudaStreamNonBlocking));
+    {   // side stream at the lowest priority: its streaming work fills gaps left by the
+        // latency-bound main-stream kernels instead of delaying them
+        int lo = 0, hi = 0;
+        CK(cudaDeviceGetStreamPriorityRange(&lo, &hi));
+        CK(cudaStreamCreateWithPriority(&r->st2, cudaStreamNonBlocking, lo));
+    }
     CK(cudaEventCreateWithFlags(&r->evA, cudaEventDisableTiming));
     CK(cudaEventCreateWithFlags(&r->evB, cudaEventDisableTiming));
     CK(cudaMallocHost(&r->hc, sizeof(Counters)));
@@ -726,9 +792,9 @@ void free_replica(h2tap_replica* r) {
                    &r->pt[0], &r->pt[1], &r->pq[0], &r->pq[1], &r->Wk, &r->Ws, &r->Wd, &r->Ww, &r->Wt, &r->Wq,
                    &r->idx_p, &r->idx_n, &r->idx_e, &r->status, &r->keyA, &r->keyB, &r->valA, &r->valB,
                    &r->hist, &r->dbase, &r->rs_status, &r->rs_ctr, &r->nv, &r->nv_ext, &r->dropped, &r->ins_q,
-                   &r->ins_oldpos, &r->hd_rows, &r->remap, &r->hd_bits, &r->op_flags, &r->op_ou, &r->op_ow,
+                   &r->ins_oldpos, &r->hd_rows, &r->hd_bits, &r->op_flags, &r->op_ou, &r->op_ow,
                    &r->ins_pos, &r->ins_row, &r->ins_col, &r->ins_w, &r->del_pos, &r->upd_pos, &r->upd_w,
-                   &r->KR, &r->misc, &r->nsorted, &r->part, &r->opart, &r->deg, &r->tsum, &r->remap_shift, &r->remap32, &r->tile_emit, &r->tile_base, &r->del_row, &r->casc_mask, &r->status2, &r->fence[0], &r->fence[1], &r->bfs_a, &r->bfs_b, &r->pr_a, &r->pr_b, &r->ctr};
+                   &r->KR, &r->misc, &r->nsorted, &r->part, &r->opart, &r->deg, &r->tsum, &r->remap_shift, &r->remap32, &r->casc_wrel, &r->tile_emit, &r->tile_base, &r->del_row, &r->casc_mask, &r->status2, &r->fence[0], &r->fence[1], &r->bfs_a, &r->bfs_b, &r->pr_a, &r->pr_b, &r->ctr};
     for (Buf* b : bufs) if (b->p) r->dfree(b->p);
     cudaStreamSynchronize(r->st);
     for (auto& e : r->ev) if (e) cudaEventDestroy(e);

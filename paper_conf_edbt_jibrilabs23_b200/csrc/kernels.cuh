@@ -51,6 +51,36 @@ struct NodeVtx {
 };
 enum : uint32_t { NV_FINAL = 1, NV_HASD = 2, NV_OLD = 4 };
 
+// ID-map compaction (reading A9), evaluated on the fly: new dense id of old vertex k
+// = k - (#dropped ids < k) + (#inserted ids placed at old positions <= k).
+//   shift[k >> 16]: constant shift of a 64K-id block without dropped ids or insertion
+//                   points strictly inside, else kRemapMixed
+//   g32[k >> 5]  : {new id of the group's first id | exact << 31, dropped bitmask};
+//                   exact groups (an insertion point strictly inside) add the insertion
+//                   ranks.  Dense ids stay below 2^31 (checked on the host).
+constexpr int kRemapBlockShift = 16;
+constexpr int32_t kRemapMixed = INT32_MIN;
+struct RemapView {
+    const int32_t* shift;  // nullptr: identity
+    const uint2* g32;
+    const uint32_t* ins_oldpos;
+    uint64_t n_vins;
+};
+__device__ __forceinline__ uint32_t remap_of(const RemapView& R, uint32_t k) {
+    if (!R.shift) return k;
+    const int32_t shf = R.shift[k >> kRemapBlockShift];
+    if (shf != kRemapMixed) return (uint32_t)((int64_t)k + shf);
+    const uint2 g = R.g32[k >> 5];
+    const uint32_t r = k & 31;
+    if (g.y >> r & 1) return kNone32;  // dropped
+    uint32_t v = (g.x & 0x7FFFFFFFu) + r - (r ? __popc(g.y & (0xFFFFFFFFu >> (32 - r))) : 0u);
+    if (g.x >> 31) v += (uint32_t)(upper_bound_dev(R.ins_oldpos, 0, R.n_vins, k) -
+                             upper_bound_dev(R.ins_oldpos, 0, R.n_vins, k - r));
+    return v;
+}
+
+__device__ __noinline__ uint32_t remap_of_slow(const RemapView& R, uint32_t k) { return remap_of(R, k); }
+
 // ===================================================================== a1 ====
 // Validate + number + split: pending (ts > S) / visible node ops / visible edge
 // ops, each stable (ascending seq) via a 3-way decoupled look-back compaction.
@@ -289,34 +319,13 @@ __device__ __forceinline__ uint64_t gallop_ub(const T* a, uint64_t lo, uint64_t 
     return upper_bound_dev(a, lo, p, key);
 }
 
-// ID-map compaction (reading A9): remap[k] = new dense id of old vertex k or
-// kNone32 (dropped); new_ext[remap[k]] = ext[k].  Survivor rank minus dropped
-// before plus inserted (by old position) at or before.  Thread per vertex; the
-// CTA narrows the two small sorted lists to its id range first.
-constexpr int kRemapTile = 1024;
-__global__ void __launch_bounds__(kThreads) k_remap(
-    const uint64_t* __restrict__ old_ext, int identity, uint64_t V, const uint32_t* __restrict__ dropped,
-    uint64_t n_dropped, const uint32_t* __restrict__ ins_oldpos, uint64_t n_ins,
-    uint32_t* __restrict__ remap, uint64_t* __restrict__ new_ext) {
-    __shared__ uint64_t s_r[4];
-    const uint64_t k0 = (uint64_t)blockIdx.x * kRemapTile, k1 = min(k0 + kRemapTile, V);
-    if (threadIdx.x < 4) {
-        const int w = threadIdx.x;
-        uint32_t key = (uint32_t)((w & 1) ? k1 : k0);
-        s_r[w] = (w < 2) ? lower_bound_dev(dropped, 0, n_dropped, key)
-                         : upper_bound_dev(ins_oldpos, 0, n_ins, key);  // oldpos <= key
-    }
-    __syncthreads();
-    const uint64_t da = s_r[0], db = s_r[1], ia = s_r[2], ib = s_r[3];
-    for (uint64_t k = k0 + threadIdx.x; k < k1; k += kThreads) {
-        uint64_t dp = lower_bound_dev(dropped, da, db, (uint32_t)k);
-        bool is_dropped = dp < n_dropped && dropped[dp] == (uint32_t)k;
-        // inserted with oldpos <= k: those <= k0 (= ia) plus those in (k0, k]
-        uint64_t ip = upper_bound_dev(ins_oldpos, ia, ib, (uint32_t)k);
-        uint32_t r = is_dropped ? kNone32 : (uint32_t)(k - dp + ip);
-        remap[k] = r;
-        if (!is_dropped) new_ext[r] = identity ? k : old_ext[k];
-    }
+// new ID map, survivors: new_ext[remap(k)] = ext[k] (thread per old vertex)
+__global__ void k_new_ext(const uint64_t* __restrict__ old_ext, int identity, uint64_t V, RemapView R,
+                          uint64_t* __restrict__ new_ext) {
+    const uint64_t k = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x;
+    if (k >= V) return;
+    const uint32_t u = remap_of(R, (uint32_t)k);
+    if (u != kNone32) new_ext[u] = identity ? k : old_ext[k];
 }
 
 // inserted vertex i lands at oldpos_i - (#dropped before oldpos_i) + i
@@ -333,11 +342,11 @@ __global__ void k_place_inserted(NodeVtx* __restrict__ nv, const uint64_t* __res
 }
 
 // new ids of surviving old vertices that have node ops
-__global__ void k_nv_newid(NodeVtx* __restrict__ nv, uint64_t U, const uint32_t* __restrict__ remap, int has_remap) {
+__global__ void k_nv_newid(NodeVtx* __restrict__ nv, uint64_t U, RemapView R) {
     uint64_t q = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x;
     if (q >= U) return;
     uint32_t f = nv[q].flags;
-    if ((f & NV_OLD) && (f & NV_FINAL)) nv[q].newid = has_remap ? remap[nv[q].oldpos] : nv[q].oldpos;
+    if ((f & NV_OLD) && (f & NV_FINAL)) nv[q].newid = remap_of(R, nv[q].oldpos);
 }
 
 __global__ void k_set_bits(const uint32_t* __restrict__ rows, uint64_t n, uint32_t* __restrict__ bits) {
@@ -354,12 +363,24 @@ struct Lookup {
     uint64_t tD_ts, tD_seq;
 };
 
+// Everything the segmented reduce needs about one surviving edge op, in one 32-byte
+// sector (the sort carries only the record index; the SoA op arrays would cost
+// ~7 scattered sectors per op once the sort passes have evicted them from L2).
+struct __align__(32) EdgeRec {
+    uint64_t ts, seq;         // commit point (reading A5)
+    float w;
+    uint32_t opos_u, opos_w;  // old dense index (present) or insertion rank of src / dst
+    uint8_t kind;
+    uint8_t flags;            // bit0 src old-present, bit1 dst old-present, bit2 key had a node delete
+    uint16_t pad;
+};
+
 struct PrepArgs {
     Ops ops;
     const uint32_t* edge_idx;
     uint64_t n_edge;
     ExtIndex X;
-    const uint32_t* remap;  // nullable (identity remap)
+    RemapView R;            // identity when R.shift == nullptr
     const NodeVtx* nv;
     const uint64_t* nv_ext;
     uint64_t U;
@@ -368,9 +389,7 @@ struct PrepArgs {
     int create;                   // create_from_edges: endpoints must exist
     uint64_t* keys;
     uint32_t* vals;
-    uint8_t* op_flags;            // per W index: bit0 u old-present, bit1 w old-present, bit2 key had node delete
-    uint32_t* op_opos_u;
-    uint32_t* op_opos_w;
+    struct EdgeRec* recs;         // one compact record per surviving edge op, indexed by op
     uint64_t* status;
     uint64_t n_tiles;
     Counters* c;
@@ -400,7 +419,7 @@ __device__ __forceinline__ Lookup do_lookup(const PrepArgs& a, uint64_t x) {
     L.oldpos = (uint32_t)k;
     L.old_present = present;
     L.final_live = present;
-    L.newid = present ? (a.remap ? a.remap[k] : (uint32_t)k) : kNone32;
+    L.newid = present ? remap_of(a.R, (uint32_t)k) : kNone32;
     return L;
 }
 
@@ -421,20 +440,24 @@ __device__ __forceinline__ bool live_at(const PrepArgs& a, const Lookup& L, uint
 // Per visible edge op: endpoint lookups, liveness gating and node-delete
 // supersession (order-free form of the replay), packed key
 // (src' << bits | dst'), compaction of surviving ops via look-back.
+// EI ops per thread: 1 when ID lookups are searches (latency-bound chains need
+// parallelism), 8 for the identity ID map
+template <int EI>
 __global__ void __launch_bounds__(kThreads) k_edge_prep(PrepArgs a) {
+    constexpr int kEItems = EI, kETile = kThreads * EI;
     __shared__ uint32_t s_tile;
-    __shared__ uint32_t s_cmp[kItems * kThreads / 32 + 1];
+    __shared__ uint32_t s_cmp[kEItems * kThreads / 32 + 1];
     __shared__ uint64_t s_base;
     if (threadIdx.x == 0) s_tile = atomicAdd(&a.c->tiles[3], 1u);
     __syncthreads();
     const uint32_t tile = s_tile;
-    const uint64_t i0 = (uint64_t)tile * kTile + threadIdx.x;
-    uint64_t key[kItems];
-    bool valid[kItems];
-    uint32_t pos[kItems];
+    const uint64_t i0 = (uint64_t)tile * kETile + threadIdx.x;
+    uint64_t key[kEItems];
+    bool valid[kEItems];
+    uint32_t pos[kEItems];
     uint64_t ngated = 0, nbad = 0;
 #pragma unroll
-    for (int j = 0; j < kItems; ++j) {
+    for (int j = 0; j < kEItems; ++j) {
         uint64_t i = i0 + (uint64_t)j * kThreads;
         key[j] = 0;
         valid[j] = false;
@@ -457,10 +480,16 @@ __global__ void __launch_bounds__(kThreads) k_edge_prep(PrepArgs a) {
         if (ok) {
             valid[j] = true;
             key[j] = ((uint64_t)Lu.newid << a.bits) | (uint64_t)Lw.newid;
-            a.op_flags[o] = (uint8_t)((Lu.old_present ? 1 : 0) | (Lw.old_present ? 2 : 0) |
-                                      ((Lu.hasD || Lw.hasD) ? 4 : 0));
-            a.op_opos_u[o] = Lu.oldpos;
-            a.op_opos_w[o] = Lw.oldpos;
+            EdgeRec rc;
+            rc.ts = ts;
+            rc.seq = seq;
+            rc.w = a.ops.w[o];
+            rc.opos_u = Lu.oldpos;
+            rc.opos_w = Lw.oldpos;
+            rc.kind = kind;
+            rc.flags = (uint8_t)((Lu.old_present ? 1 : 0) | (Lw.old_present ? 2 : 0) | ((Lu.hasD || Lw.hasD) ? 4 : 0));
+            rc.pad = 0;
+            a.recs[o] = rc;  // indexed by op; the sort payload is the op index
         } else {
             ngated++;
         }
@@ -469,14 +498,14 @@ __global__ void __launch_bounds__(kThreads) k_edge_prep(PrepArgs a) {
     if (lane_id() == 0 && gsum) atomicAdd(&a.c->n_gated, (unsigned long long)gsum);
     uint64_t bsum = warp_sum(nbad);
     if (lane_id() == 0 && bsum) atomicOr(&a.c->status, (unsigned long long)ST_CREATE_ENDPOINT);
-    uint32_t tot = striped_compact<kThreads, kItems>(valid, pos, s_cmp);
+    uint32_t tot = striped_compact<kThreads, kEItems>(valid, pos, s_cmp);
     if (threadIdx.x < 32) {
         uint64_t b = lookback_warp(a.status, tile, tot);
         if (lane_id() == 0) { s_base = b; if (tile == a.n_tiles - 1) a.c->n_valid = b + tot; }
     }
     __syncthreads();
 #pragma unroll
-    for (int j = 0; j < kItems; ++j) {
+    for (int j = 0; j < kEItems; ++j) {
         if (valid[j]) {
             uint64_t p = s_base + pos[j];
             a.keys[p] = key[j];
@@ -499,9 +528,7 @@ struct ClassArgs {
     const uint32_t* vals;
     uint64_t n;
     int bits;
-    const uint8_t* op_flags;
-    const uint32_t* op_opos_u;
-    const uint32_t* op_opos_w;
+    const EdgeRec* recs;
     const int64_t* old_off;
     const uint32_t* old_cols;
     uint64_t V_old;
@@ -549,21 +576,22 @@ __global__ void __launch_bounds__(kThreads) k_reduce_classify(ClassArgs a) {
         bool has_nw = false, has_w = false;
         uint8_t nw_kind = 0;
         float w_val = 0.f;
+        EdgeRec r0;
         for (uint64_t e = i; e < a.n && a.keys[e] == key; ++e) {
-            uint32_t o = a.vals[e];
-            uint8_t k = a.ops.kind[o];
-            uint64_t ts = a.ops.ts[o], sq = a.ops.seq[o];
+            const EdgeRec re = a.recs[a.vals[e]];
+            if (e == i) r0 = re;
+            uint8_t k = re.kind;
+            uint64_t ts = re.ts, sq = re.seq;
             if (k == EDGE_INSERT || k == EDGE_DELETE) {
                 if (!has_nw || pt_less(nw_ts, nw_seq, ts, sq)) { has_nw = true; nw_ts = ts; nw_seq = sq; nw_kind = k; }
             }
             if (k == EDGE_INSERT || k == EDGE_WEIGHT) {
-                if (!has_w || pt_less(w_ts, w_seq, ts, sq)) { has_w = true; w_ts = ts; w_seq = sq; w_val = a.ops.w[o]; }
+                if (!has_w || pt_less(w_ts, w_seq, ts, sq)) { has_w = true; w_ts = ts; w_seq = sq; w_val = re.w; }
             }
         }
-        uint32_t o0 = a.vals[i];
-        uint8_t fl = a.op_flags[o0];
+        uint8_t fl = r0.flags;
         bool u_old = fl & 1;
-        uint32_t ou = a.op_opos_u[o0], ow = a.op_opos_w[o0];
+        uint32_t ou = r0.opos_u, ow = r0.opos_w;
         // outcome category before the old-row lookup: 1 insert-like, 2 delete, 3 weight-only
         cat[j] = (has_nw && nw_kind == EDGE_INSERT) ? 1 : (has_nw ? 2 : (has_w ? 3 : 0));
         meta[j] = fl;
@@ -664,8 +692,6 @@ __global__ void __launch_bounds__(kThreads) k_reduce_classify(ClassArgs a) {
 constexpr int kMergeTile = 2048;             // merged items per tile
 constexpr int kCascBlock = 2048;             // cascade mask: elements per counted block (64 words)
 constexpr int kMergeBuf = kMergeTile + 8;     // staged old elements (+ 16 B alignment slack)
-constexpr int kRemapBlockShift = 16;          // two-level remap: 64K old ids per block (L1-resident table)
-constexpr int32_t kRemapMixed = INT32_MIN;    // block has a dropped/inserted id inside
 
 struct MergeArgs {
     const uint32_t* old_cols;
@@ -681,8 +707,7 @@ struct MergeArgs {
     const uint64_t* upd_pos;
     const float* upd_w;
     uint64_t n_upd;
-    const uint32_t* remap;
-    const int32_t* remap_shift;  // per 64K-id block: constant shift or kRemapMixed
+    RemapView R;
     const uint32_t* hd_bits;
     const uint32_t* hd_rows;
     uint64_t n_hd;
@@ -694,7 +719,6 @@ struct MergeArgs {
     uint64_t n_dropped;
     const uint32_t* ins_oldpos;  // sorted insertion ranks of inserted vertices
     uint64_t n_vins;
-    const uint2* remap32;        // per 32 old ids: {base new id, dropped bitmask} (kRemapExact: use remap[])
     int rows;                    // 1: merge writes new_off for old rows starting in each tile
     const uint32_t* casc_mask;  // CASC: 1 bit per old element (removed by a node delete)
     const uint64_t* casc_pre;   // CASC: cascaded elements before each 2048-element block
@@ -782,23 +806,46 @@ __device__ __forceinline__ void mbar_wait(uint64_t* bar, uint32_t phase) {
 // columns pointing at deleted vertices: one ballot per 32 elements -> one mask
 // word (pure stores, every element's loads independent)
 __global__ void __launch_bounds__(kThreads) k_casc_cols(const uint32_t* __restrict__ old_cols, uint64_t E,
-        const uint32_t* __restrict__ hd_bits, uint32_t* __restrict__ mask) {
-    const uint64_t b0 = (uint64_t)blockIdx.x * kCascBlock;
-    constexpr int PER = kCascBlock / kThreads;  // 8 elements per thread, striped
-    uint32_t col[PER];
+        const uint32_t* __restrict__ hd_bits, const uint32_t* __restrict__ hd_rows, uint64_t n_hd,
+        uint32_t* __restrict__ mask) {
+    const uint32_t hd_lo = hd_rows[0], hd_hi = hd_rows[n_hd - 1];  // sorted: id range of deleted vertices
+    // 2 x 2048 elements per CTA; each lane owns 4 consecutive elements per step (128-bit
+    // loads), a warp step covers 128 elements = 4 mask words; 16 columns in flight per lane
+    constexpr int STEPS = 4;
+    const uint64_t b0 = (uint64_t)blockIdx.x * (2 * kCascBlock);
+    const int w = threadIdx.x >> 5;
+    uint4 c[STEPS];
 #pragma unroll
-    for (int j = 0; j < PER; ++j) {
-        uint64_t x = b0 + (uint64_t)j * kThreads + threadIdx.x;
-        col[j] = x < E ? old_cols[x] : 0;
+    for (int j = 0; j < STEPS; ++j) {
+        const uint64_t x = b0 + ((uint64_t)(j * (kThreads / 32) + w) * 128) + lane_id() * 4;
+        c[j] = (x + 3 < E) ? __ldcs(reinterpret_cast<const uint4*>(old_cols + x))
+                           : make_uint4(x < E ? old_cols[x] : 0u, x + 1 < E ? old_cols[x + 1] : 0u,
+                                        x + 2 < E ? old_cols[x + 2] : 0u, 0u);
     }
-    uint32_t bit[PER];
+    uint32_t bits[STEPS];
 #pragma unroll
-    for (int j = 0; j < PER; ++j) bit[j] = hd_bits[col[j] >> 5] >> (col[j] & 31);
+    for (int j = 0; j < STEPS; ++j) {
+        const uint64_t x = b0 + ((uint64_t)(j * (kThreads / 32) + w) * 128) + lane_id() * 4;
+        const uint32_t v[4] = {c[j].x, c[j].y, c[j].z, c[j].w};
+        uint32_t m = 0;
 #pragma unroll
-    for (int j = 0; j < PER; ++j) {
-        uint64_t x = b0 + (uint64_t)j * kThreads + threadIdx.x;
-        uint32_t m = __ballot_sync(0xffffffffu, x < E && (bit[j] & 1));
-        if (lane_id() == 0) mask[x >> 5] = m;  // words past E are written as 0
+        for (int e = 0; e < 4; ++e) {
+            const bool in = x + e < E && v[e] >= hd_lo && v[e] <= hd_hi && (hd_bits[v[e] >> 5] >> (v[e] & 31) & 1);
+            m |= (uint32_t)in << e;
+        }
+        bits[j] = m;  // 4 bits for this lane's elements
+    }
+#pragma unroll
+    for (int j = 0; j < STEPS; ++j) {
+        // lane L holds bits of elements 4L..4L+3 of the 128-element step: word q = L / 8
+        const uint32_t nib = bits[j] << ((lane_id() & 7) * 4);
+        uint32_t word = nib;
+        word |= __shfl_xor_sync(0xffffffffu, word, 1);
+        word |= __shfl_xor_sync(0xffffffffu, word, 2);
+        word |= __shfl_xor_sync(0xffffffffu, word, 4);
+        const uint64_t x = b0 + ((uint64_t)(j * (kThreads / 32) + w) * 128);
+        if ((lane_id() & 7) == 0 && x + lane_id() * 4 < ((E + 31) & ~31ull) + 2 * kCascBlock)
+            mask[(x >> 5) + lane_id() / 8] = word;  // words past E are written as 0
     }
 }
 
@@ -820,10 +867,13 @@ __global__ void k_casc_rows(const int64_t* __restrict__ old_off, const uint32_t*
     }
 }
 
-// per 2048-element block: cascaded count = popcount of its 64 mask words; then
-// the exclusive scan over blocks (decoupled look-back), total at [nblk]
+// per 2048-element block: cascaded count = popcount of its 64 mask words, the
+// per-word prefix inside the block (u16), then the exclusive scan over blocks
+// (decoupled look-back), total at [nblk].  cascaded_before(x) =
+// pre[x / 2048] + wrel[x / 32] + popc(mask[x / 32] below bit x % 32).
 __global__ void __launch_bounds__(kThreads) k_casc_scan(const uint32_t* __restrict__ mask, uint64_t nblk,
-        uint64_t* __restrict__ pre, uint64_t* __restrict__ status, unsigned int* __restrict__ ctr) {
+        uint64_t* __restrict__ pre, uint16_t* __restrict__ wrel, uint64_t* __restrict__ status,
+        unsigned int* __restrict__ ctr) {
     __shared__ uint32_t s_tile;
     __shared__ uint64_t s_scan[kThreads / 32 + 1];
     __shared__ uint64_t s_cnt[kThreads];
@@ -832,14 +882,17 @@ __global__ void __launch_bounds__(kThreads) k_casc_scan(const uint32_t* __restri
     __syncthreads();
     const uint64_t blk0 = (uint64_t)s_tile * kThreads;  // one block count per thread
     const int w = threadIdx.x >> 5;
-    for (int i = 0; i < 32; ++i) {  // warp w counts blocks blk0 + w*32 + i (coalesced 2 words per lane)
+    for (int i = 0; i < 32; ++i) {  // warp w handles blocks blk0 + w*32 + i (2 words per lane)
         uint64_t bk = blk0 + w * 32 + i;
         uint32_t c = 0;
         if (bk < nblk) {
             const uint2 v = reinterpret_cast<const uint2*>(mask + bk * (kCascBlock / 32))[lane_id()];
-            c = __popc(v.x) + __popc(v.y);
+            const uint32_t c0 = __popc(v.x), c1 = __popc(v.y);
+            const uint32_t inc = warp_inclusive_scan(c0 + c1);
+            reinterpret_cast<ushort2*>(wrel + bk * (kCascBlock / 32))[lane_id()] =
+                make_ushort2((uint16_t)(inc - c0 - c1), (uint16_t)(inc - c1));
+            c = __shfl_sync(0xffffffffu, inc, 31);
         }
-        c = warp_sum(c);
         if (lane_id() == 0) s_cnt[w * 32 + i] = c;
     }
     __syncthreads();
@@ -852,6 +905,80 @@ __global__ void __launch_bounds__(kThreads) k_casc_scan(const uint32_t* __restri
     __syncthreads();
     uint64_t bk = blk0 + threadIdx.x;
     if (bk <= nblk) pre[bk] = s_base + ex;
+}
+
+// Row offsets with node ops (a4/a5): thread per old row k that survives,
+//   new_off[u'] = x - (cascaded before x) - (deleted before x) + (inserted records in rows < u')
+// with x = old_off[k]; the CTA narrows the sorted delete / insert-row lists first.
+constexpr int kRowTile = 1024;
+struct RowArgs {
+    const int64_t* old_off;
+    uint64_t V_old, E_old;
+    RemapView R;  // identity when R.shift == nullptr
+    const uint32_t* casc_mask;
+    const uint64_t* casc_pre;
+    const uint16_t* casc_wrel;
+    const uint64_t* del_pos;
+    uint64_t n_del;
+    const uint32_t* ins_row;
+    uint64_t n_ins;
+    const uint32_t* dropped;
+    uint64_t n_dropped;
+    const uint32_t* ins_oldpos;
+    uint64_t n_vins;
+    int64_t* new_off;
+    uint64_t* part;  // [n_cta + 1][2]: delete rank and insert-row rank at each CTA's first row
+};
+__device__ __forceinline__ uint64_t casc_before(const RowArgs& a, uint64_t x) {
+    if (!a.casc_mask) return 0;
+    if (x >= a.E_old) return a.casc_pre[(a.E_old + kCascBlock - 1) / kCascBlock];  // all cascaded
+    const uint32_t r = x & 31;
+    return a.casc_pre[x / kCascBlock] + a.casc_wrel[x >> 5] +
+           (r ? __popc(a.casc_mask[x >> 5] & (0xFFFFFFFFu >> (32 - r))) : 0u);
+}
+// CTA boundaries of k_offsets_rows: ranks of each CTA's first row in the two lists
+__global__ void k_rows_partition(RowArgs a) {
+    const uint64_t c = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x;
+    const uint64_t ncta = (a.V_old + kRowTile - 1) / kRowTile;
+    if (c > ncta) return;
+    const uint64_t k = c * kRowTile;
+    uint64_t dr, ir;
+    if (k >= a.V_old) { dr = a.n_del; ir = a.n_ins; }
+    else {
+        dr = lower_bound_dev(a.del_pos, 0, a.n_del, (uint64_t)a.old_off[k]);
+        // insert-row rank of the new id of the first surviving row >= k (compaction formula)
+        const uint64_t u = a.R.shift ? k - lower_bound_dev(a.dropped, 0, a.n_dropped, (uint32_t)k) +
+                                       upper_bound_dev(a.ins_oldpos, 0, a.n_vins, (uint32_t)k)
+                                     : k;
+        ir = lower_bound_dev(a.ins_row, 0, a.n_ins, (uint32_t)u);
+    }
+    a.part[2 * c] = dr;
+    a.part[2 * c + 1] = ir;
+}
+
+__global__ void __launch_bounds__(kThreads) k_offsets_rows(RowArgs a) {
+    const uint64_t k0 = (uint64_t)blockIdx.x * kRowTile, k1 = min(k0 + kRowTile, a.V_old);
+    const uint64_t* pp = a.part + 2 * blockIdx.x;  // this CTA's slices of the delete / insert-row lists
+    const uint64_t da = pp[0], ia = pp[1], db = pp[2], ib = pp[3];
+    constexpr int PER = kRowTile / kThreads;  // rows per thread, all loads issued together
+    uint32_t u[PER];
+    uint64_t x[PER];
+#pragma unroll
+    for (int j = 0; j < PER; ++j) {
+        const uint64_t k = k0 + threadIdx.x + (uint64_t)j * kThreads;
+        u[j] = kNone32;
+        x[j] = 0;
+        if (k < k1) { u[j] = remap_of(a.R, (uint32_t)k); x[j] = (uint64_t)a.old_off[k]; }
+    }
+    uint64_t cb[PER];
+#pragma unroll
+    for (int j = 0; j < PER; ++j) cb[j] = (u[j] != kNone32) ? casc_before(a, x[j]) : 0;
+#pragma unroll
+    for (int j = 0; j < PER; ++j) {
+        if (u[j] == kNone32) continue;
+        const uint64_t kept = x[j] - cb[j] - lower_bound_dev(a.del_pos, da, db, x[j]);
+        a.new_off[u[j]] = (int64_t)(kept + lower_bound_dev(a.ins_row, ia, ib, u[j]));
+    }
 }
 
 // Device-wide exclusive scan of u64 values, single pass (decoupled look-back).
@@ -883,19 +1010,8 @@ __global__ void __launch_bounds__(kThreads) k_scan_exclusive_u64(const uint64_t*
 
 constexpr int kMerge3Smem = 6 * kMergeBuf * 4;  // dynamic shared memory of k_merge3
 
-constexpr uint32_t kRemapExact = 0xFFFFFFFFu;  // remap32 base: group needs the exact table
 constexpr int kRowStage = 512;                 // rows mode: insert-row slice staged in smem
-
-// new dense id of surviving old vertex `col` (REMAP mode): constant shift of its
-// 64K-id block, else base of its 32-group minus the dropped ids below it
-__device__ __forceinline__ uint32_t remap_col(const MergeArgs& a, uint32_t col) {
-    const int32_t shf = a.remap_shift[col >> kRemapBlockShift];
-    if (shf != kRemapMixed) return (uint32_t)((int64_t)col + shf);
-    const uint2 g = a.remap32[col >> 5];
-    if (g.x == kRemapExact) return a.remap[col];
-    const uint32_t r = col & 31;
-    return g.x + r - (r ? __popc(g.y & (0xFFFFFFFFu >> (32 - r))) : 0u);
-}
+constexpr int kRowPf = 4;                      // rows mode: old rows prefetched per thread
 
 // ---- TMA bulk store (smem -> global) helpers
 __device__ __forceinline__ void bulk_s2g(void* dst, const void* src, uint32_t bytes) {
@@ -983,13 +1099,13 @@ __global__ void __launch_bounds__(kThreads) k_merge3(MergeArgs a, const TilePart
         const uint64_t ir_end = last_tile ? a.n_ins : ir1;
         const uint32_t n_rows = a.rows ? (uint32_t)min(rk_end - rk0, (uint64_t)0xFFFFFFFF) : 0u;
         const uint32_t n_irs = a.rows ? (uint32_t)(ir_end - ir0) : 0u;
-        int64_t pf_x[2];
-        uint32_t pf_u[2];
+        int64_t pf_x[kRowPf];
+        uint32_t pf_u[kRowPf];
 #pragma unroll
-        for (int h = 0; h < 2; ++h) {
+        for (int h = 0; h < kRowPf; ++h) {
             const uint32_t q = tid + h * kThreads;
             pf_x[h] = q < n_rows ? a.old_off[rk0 + q] : 0;
-            pf_u[h] = q < n_rows ? (REMAP ? a.remap[rk0 + q] : (uint32_t)(rk0 + q)) : kNone32;
+            pf_u[h] = q < n_rows ? (REMAP ? remap_of(a.R, (uint32_t)(rk0 + q)) : (uint32_t)(rk0 + q)) : kNone32;
         }
         for (uint32_t q = tid; q < n_irs && q < kRowStage; q += kThreads) s_irow[q] = a.ins_row[ir0 + q];
         if (tid < NCH + 2) { s_dmask[tid] = 0; s_icnt[tid] = 0; }
@@ -1064,18 +1180,18 @@ __global__ void __launch_bounds__(kThreads) k_merge3(MergeArgs a, const TilePart
                 const uint32_t c = wid + k * (kThreads / 32), i = c * 32 + lane;
                 colv[k] = (i < n_old) ? s_col[b][i + sh] : 0u;
             }
-            if (REMAP) {
+            if (REMAP) {  // lookups of all 8 chunks in flight together (tables stay in L1/L2)
                 int32_t shf[KCH];
 #pragma unroll
-                for (int k = 0; k < KCH; ++k) shf[k] = a.remap_shift[colv[k] >> kRemapBlockShift];
+                for (int k = 0; k < KCH; ++k) shf[k] = a.R.shift[colv[k] >> kRemapBlockShift];
                 uint2 g[KCH];
 #pragma unroll
-                for (int k = 0; k < KCH; ++k) g[k] = (shf[k] == kRemapMixed) ? a.remap32[colv[k] >> 5] : make_uint2(0u, 0u);
+                for (int k = 0; k < KCH; ++k) g[k] = (shf[k] == kRemapMixed) ? a.R.g32[colv[k] >> 5] : make_uint2(0u, 0u);
 #pragma unroll
                 for (int k = 0; k < KCH; ++k) {
                     const uint32_t col = colv[k], r = col & 31;
                     if (shf[k] != kRemapMixed) colv[k] = (uint32_t)((int64_t)col + shf[k]);
-                    else if (g[k].x == kRemapExact) colv[k] = a.remap[col];
+                    else if (g[k].x >> 31) colv[k] = remap_of_slow(a.R, col);  // rare: out of line
                     else colv[k] = g[k].x + r - (r ? __popc(g[k].y & (0xFFFFFFFFu >> (32 - r))) : 0u);
                 }
             }
@@ -1112,11 +1228,21 @@ __global__ void __launch_bounds__(kThreads) k_merge3(MergeArgs a, const TilePart
             //   = (kept old elements before its old start) + (inserted records in rows < u')
             const uint64_t kb0 = j0 - dl0 - cbefore;  // kept old elements before j0
             const bool staged = n_irs <= kRowStage;
-            for (uint32_t q = tid; q < n_rows; q += kThreads) {
-                const bool pf = q < 2 * kThreads;
-                const uint32_t u = pf ? (q < kThreads ? pf_u[0] : pf_u[1]) : (REMAP ? a.remap[rk0 + q] : (uint32_t)(rk0 + q));
+#pragma unroll
+            for (int h = 0; h < kRowPf; ++h) {  // prefetched rows
+                const uint32_t q = tid + h * kThreads;
+                const uint32_t u = pf_u[h];
+                if (q >= n_rows || u == kNone32) continue;
+                const int64_t x = pf_x[h];
+                const uint64_t kept_b = kb0 + kept_before((uint32_t)((uint64_t)x - j0));
+                const uint64_t irk = staged ? ir0 + lower_bound_dev(s_irow, 0, n_irs, u)
+                                            : lower_bound_dev(a.ins_row, ir0, ir_end, u);
+                a.new_off[u] = (int64_t)(kept_b + irk);
+            }
+            for (uint32_t q = tid + kRowPf * kThreads; q < n_rows; q += kThreads) {  // rare overflow
+                const uint32_t u = REMAP ? remap_of(a.R, (uint32_t)(rk0 + q)) : (uint32_t)(rk0 + q);
                 if (u == kNone32) continue;
-                const int64_t x = pf ? (q < kThreads ? pf_x[0] : pf_x[1]) : a.old_off[rk0 + q];
+                const int64_t x = a.old_off[rk0 + q];
                 const uint64_t kept_b = kb0 + kept_before((uint32_t)((uint64_t)x - j0));
                 const uint64_t irk = staged ? ir0 + lower_bound_dev(s_irow, 0, n_irs, u)
                                             : lower_bound_dev(a.ins_row, ir0, ir_end, u);
@@ -1301,27 +1427,17 @@ __global__ void __launch_bounds__(kThreads) k_offsets_scan(const int64_t* __rest
 // rows of inserted (new) vertices: kept old elements before the old position they
 // are inserted at, plus inserted records in rows < their new id
 __global__ void k_offsets_inserted(const NodeVtx* __restrict__ nv, const uint32_t* __restrict__ ins_q,
-                                   uint64_t n_vins, const int64_t* __restrict__ old_off,
-                                   const uint64_t* __restrict__ del_pos, uint64_t n_del,
-                                   const uint32_t* __restrict__ casc_mask, const uint64_t* __restrict__ casc_pre,
-                                   const uint32_t* __restrict__ ins_row, uint64_t n_ins, int64_t* __restrict__ new_off) {
+                                   uint64_t n_vins, RowArgs a) {
     uint64_t i = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x;
     if (i >= n_vins) return;
     const NodeVtx& r = nv[ins_q[i]];
-    const uint64_t x = (uint64_t)old_off[r.oldpos];
-    uint64_t kept = x - lower_bound_dev(del_pos, 0, n_del, x);
-    if (casc_mask) {
-        const uint64_t blk = x / kCascBlock;
-        uint64_t c = casc_pre[blk];
-        for (uint64_t q = blk * (kCascBlock / 32); q < (x >> 5); ++q) c += __popc(casc_mask[q]);
-        if (x & 31) c += __popc(casc_mask[x >> 5] & (0xFFFFFFFFu >> (32 - (x & 31))));
-        kept -= c;
-    }
-    new_off[r.newid] = (int64_t)(kept + lower_bound_dev(ins_row, 0, n_ins, r.newid));
+    const uint64_t x = (uint64_t)a.old_off[r.oldpos];
+    const uint64_t kept = x - casc_before(a, x) - lower_bound_dev(a.del_pos, 0, a.n_del, x);
+    a.new_off[r.newid] = (int64_t)(kept + lower_bound_dev(a.ins_row, 0, a.n_ins, r.newid));
 }
 
-// per 32 old ids: {new id of the group's first id (as if it survived), dropped bitmask};
-// kRemapExact if an inserted vertex lands strictly inside the group
+// per 32 old ids: {new id of the group's first id (as if it survived) | exact << 31,
+// dropped bitmask}; exact = an insertion point lies strictly inside the group
 __global__ void k_remap32(uint64_t V, const uint32_t* __restrict__ dropped, uint64_t n_dropped,
                           const uint32_t* __restrict__ ins_oldpos, uint64_t n_vins, uint2* __restrict__ out) {
     const uint64_t g = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x;
@@ -1332,7 +1448,7 @@ __global__ void k_remap32(uint64_t V, const uint32_t* __restrict__ dropped, uint
     const uint64_t i1 = upper_bound_dev(ins_oldpos, i0, n_vins, c0 + 31);
     uint32_t m = 0;
     for (uint64_t d = d0; d < n_dropped && dropped[d] < c0 + 32; ++d) m |= 1u << (dropped[d] - c0);
-    out[g] = make_uint2(i1 > i0 ? kRemapExact : (uint32_t)(c0 - d0 + i0), m);
+    out[g] = make_uint2((uint32_t)(c0 - d0 + i0) | (i1 > i0 ? 0x80000000u : 0u), m);
 }
 
 __global__ void k_set_i64(int64_t* p, int64_t v) { *p = v; }

@@ -11,9 +11,11 @@ starts; the e2e leg repeats the measurement with pinned host batches copied in
 by the library inside the timed region.  The CSR (~2.8 GB read + written per
 step) exceeds the 126 MB L2, so no explicit flush is needed.
 
-Prints ONE JSON line (rank 0).  Under torchrun with N > 1 every rank holds an
-independent replica with its own batch stream (replicas, weak scaling; DESIGN.md
-§6).  ``--impl reference`` times the oracle (O1, test infrastructure) on the
+Prints ONE JSON line (rank 0).  Under torchrun with N > 1 the graph is sharded by
+1D external-ID ranges (one shard per rank); every global batch is split rank-major,
+routed to the owners with an all-to-all (NCCL; gloo with --dist-backend gloo) and
+applied per shard (strong scaling: the global batch is the config's).
+``--parallelism replicas`` runs independent replicas instead (weak scaling).  ``--impl reference`` times the oracle (O1, test infrastructure) on the
 host cores over a bounded scaled-down sample of the same workload.
 """
 from __future__ import annotations
@@ -213,85 +215,124 @@ def run_gpu(args):
     import torch.distributed as dist
 
     import paper_conf_edbt_jibrilabs23_b200 as h2
+    from paper_conf_edbt_jibrilabs23_b200.sharded import LibEngine, ShardedReplica
 
     world, rank, local = dist_setup()
+    dev_idx = local % max(1, torch.cuda.device_count())
+    torch.cuda.set_device(dev_idx)
     if world > 1:
-        dist.init_process_group("nccl", device_id=torch.device("cuda", local))
-    torch.cuda.set_device(local)
+        if args.dist_backend == "nccl":
+            dist.init_process_group("nccl", device_id=torch.device("cuda", dev_idx))
+        else:
+            dist.init_process_group("gloo")
     stream = torch.cuda.current_stream()
+    sharded = world > 1 and args.parallelism == "shard"
 
     wl = Workload(args.config)
     t0 = time.time()
     nv, ids, src, dst, w = wl.graph()
-    # rank-distinct batch streams (independent replicas); same initial graph shape
-    rep = h2.Replica.from_edges(nv, ids, src, dst, w, 0, device=local)
+    if sharded:
+        # 1D external-ID ranges balanced by edge count; this rank keeps the rows it owns
+        bounds = h2.balanced_bounds(src, world)
+        mine = np.searchsorted(bounds[1:world], src, side="right") == rank
+        rep = h2.Replica.from_edges(nv, ids, src[mine], dst[mine], w[mine], 0, device=dev_idx,
+                                    rank=rank, world=world, shard_bounds=bounds)
+        eng = LibEngine(rep, f"cuda:{dev_idx}")
+        shr = ShardedReplica(eng, rank, world, f"cuda:{dev_idx}")
+    else:
+        rep = h2.Replica.from_edges(nv, ids, src, dst, w, 0, device=dev_idx)
     del src, dst, w
     setup_s = time.time() - t0
 
     n_total = args.warmup + args.steps
-    k0 = rank * 1000
-    host = [wl.batch(k0 + k) for k in range(n_total)]
+    # sharded: every rank draws the same global batches and takes its rank-major slice
+    # (strong scaling: the global batch is the config's); replicas: rank-distinct streams
+    k0 = 0 if sharded else rank * 1000
+
+    def my_part(b):
+        if not sharded:
+            return b
+        return b.slice(slice(rank * len(b) // world, (rank + 1) * len(b) // world))
+
+    glob = [wl.batch(k0 + k) for k in range(n_total)]
+    host = [my_part(b) for b in glob]
+    snaps = [int(b.ts.max()) for b in glob]
+    glob_n = [len(b) for b in glob]
+    del glob
 
     def to_dev(b):
         return synth.Batch(*(torch.from_numpy(a.view(np.int64) if a.dtype == np.uint64 else a).cuda()
                              for a in (b.kind, b.src, b.dst, b.w, b.ts)))
 
+    def apply(b, snap):
+        if not sharded:
+            return rep.apply(b, snap)
+        l0 = eng.launches
+        st = shr.apply(b, snap)
+        st["n_launches"] += eng.launches - l0
+        return st
+
     dev = [to_dev(b) for b in host]
-    snaps = [int(b.ts.max()) for b in host]
     for k in range(args.warmup):
-        rep.apply(dev[k], snaps[k])
+        apply(dev[k], snaps[k])
     torch.cuda.synchronize()
     if world > 1:
         dist.barrier()
     stats = []
     ev0, ev1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
-    with ClockSampler(local) as clk:
+    with ClockSampler(dev_idx) as clk:
         torch.cuda.synchronize()
         ev0.record(stream)
         for k in range(args.warmup, n_total):
-            stats.append(rep.apply(dev[k], snaps[k]))
+            stats.append(apply(dev[k], snaps[k]))
         ev1.record(stream)
         torch.cuda.synchronize()
     if world > 1:
         dist.barrier()
     ms = ev0.elapsed_time(ev1)
-    updates = sum(s["n_visible"] for s in stats)
-    if world > 1:
-        t = torch.tensor([ms, float(updates)], device="cuda", dtype=torch.float64)
+    # updates: the global batches' ops (sharded: node ops reach every shard, count them once)
+    updates = (sum(glob_n[args.warmup:]) / world if sharded else sum(s["n_visible"] for s in stats))
+
+    def reduce_max_sum(ms_, upd):
+        if world == 1:
+            return ms_, float(upd)
+        t = torch.tensor([ms_, float(upd)], dtype=torch.float64,
+                         device="cpu" if args.dist_backend == "gloo" else "cuda")
         mx = t.clone()
         dist.all_reduce(mx, op=dist.ReduceOp.MAX)
         dist.all_reduce(t, op=dist.ReduceOp.SUM)
-        ms_max, updates_all = float(mx[0]), float(t[1])
-    else:
-        ms_max, updates_all = ms, float(updates)
+        return float(mx[0]), float(t[1])
+
+    ms_max, updates_all = reduce_max_sum(ms, updates)
     value = updates_all / (ms_max / 1e3)
 
     # ---- e2e: pinned host batches through the public API, H2D inside the timed region
-    e_host = [wl.batch(k0 + n_total + k) for k in range(args.steps)]
+    e_glob = [wl.batch(k0 + n_total + k) for k in range(args.steps)]
+    e_host = [my_part(b) for b in e_glob]
+    e_snaps = [int(b.ts.max()) for b in e_glob]
+    e_glob_n = [len(b) for b in e_glob]
+    del e_glob
 
     def pinned(b):
         return synth.Batch(*(torch.from_numpy(a.view(np.int64) if a.dtype == np.uint64 else a).pin_memory()
                              for a in (b.kind, b.src, b.dst, b.w, b.ts)))
 
     e_pin = [pinned(b) for b in e_host]
-    e_snaps = [int(b.ts.max()) for b in e_host]
     torch.cuda.synchronize()
     if world > 1:
         dist.barrier()
     e_stats = []
+    h2d0 = eng.h2d if sharded else 0
     ev0.record(stream)
     for k in range(args.steps):
-        e_stats.append(rep.apply(e_pin[k], e_snaps[k]))
+        e_stats.append(apply(e_pin[k], e_snaps[k]))
     ev1.record(stream)
     torch.cuda.synchronize()
     e_ms = ev0.elapsed_time(ev1)
-    e_updates = sum(s["n_visible"] for s in e_stats)
-    if world > 1:
-        t = torch.tensor([e_ms, float(e_updates)], device="cuda", dtype=torch.float64)
-        mx = t.clone()
-        dist.all_reduce(mx, op=dist.ReduceOp.MAX)
-        dist.all_reduce(t, op=dist.ReduceOp.SUM)
-        e_ms, e_updates = float(mx[0]), float(t[1])
+    if sharded:
+        e_stats[0]["h2d_bytes"] += eng.h2d - h2d0  # slice staging (route packing reads device memory)
+    e_updates = (sum(e_glob_n) / world if sharded else sum(s["n_visible"] for s in e_stats))
+    e_ms, e_updates = reduce_max_sum(e_ms, e_updates)
     e_value = e_updates / (e_ms / 1e3)
 
     if rank == 0:
@@ -305,16 +346,18 @@ def run_gpu(args):
         path_gbs = path_bytes / (ms_step / 1e3) / 1e9
         info = rep.info()
         try:  # DRAM bytes per launch of the same kernel from the committed ncu --set full capture
-            traffic = json.load(open(os.path.join(ROOT, "profiles", "traffic.json"))).get(args.config)
+            traffic = (None if sharded else  # captured for the unsharded merge only
+                       json.load(open(os.path.join(ROOT, "profiles", "traffic.json"))).get(args.config))
         except Exception:
             traffic = None
         line = {
             "metric": METRIC, "value": value, "unit": "updates/s", "n_gpus": world,
             "steps": args.steps, "warmup": args.warmup, "ms_per_step": ms_max / args.steps,
-            "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": "u32/f32",
-            "data": "synthetic",
+            "higher_is_better": True, "scaling": "strong" if sharded else "weak", "vs_baseline": None,
+            "dtype": "u32/f32", "data": "synthetic",
             "config": {"workload": wl.describe(), "name": args.config, "parallelism":
-                       "replicas" if world > 1 else "single",
+                       (f"shard{world} (1D vertex ranges, all-to-all routing over {args.dist_backend})"
+                        if sharded else "replicas" if world > 1 else "single"),
                        "l2": "inputs larger than L2 (CSR ~%.1f GB per step)" % (path_bytes / 1e9),
                        "replica_vertices": info["n_vertices"], "replica_edges": info["n_edges"]},
             "roofline": {"bound": "hbm", "kernel": "k_merge", "achieved": achieved, "peak": peak,
@@ -351,6 +394,10 @@ def main():
     ap.add_argument("--config", default="c2", choices=sorted(synth.CONFIGS))
     ap.add_argument("--impl", default="h2tap", choices=["h2tap", "reference"])
     ap.add_argument("--no-cpu-baseline", action="store_true")
+    ap.add_argument("--parallelism", default="shard", choices=["shard", "replicas"],
+                    help="N > 1: shard one graph (default) or run independent replicas")
+    ap.add_argument("--dist-backend", default="nccl", choices=["nccl", "gloo"],
+                    help="gloo lets several ranks share one GPU (testing)")
     args = ap.parse_args()
     if args.warmup < 3 and args.impl == "h2tap":
         args.warmup = 3

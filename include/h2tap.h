@@ -70,6 +70,9 @@ typedef struct {
     const uint64_t* dst;    /* ignored for NODE_* */
     const float* weight;    /* ignored for NODE_* and EDGE_DELETE; may be NULL if unused */
     const uint64_t* ts;     /* commit timestamps (MVTO txn timestamps) */
+    const uint64_t* seq;    /* arrival numbers (reading A5); NULL = assigned by the library in
+                               batch order.  Sharded replicas without a communicator receive
+                               routed ops and must pass their global (rank-major) numbers. */
 } h2tap_batch;
 
 /* Filled by h2tap_delta_apply (counts are global over all ranks). */
@@ -96,10 +99,20 @@ typedef struct {
     void (*free)(void* ctx, void* p, void* stream);
 } h2tap_allocator;
 
+/* Sharding (world > 1): 1D ranges of EXTERNAL vertex IDs.  Shard `rank` owns the rows
+ * of the live vertices with shard_bounds[rank] <= id < shard_bounds[rank+1] (the last
+ * bound is inclusive of UINT64_MAX); columns hold GLOBAL dense IDs (rank among all live
+ * vertices) and every shard keeps the global ID map.  Without a communicator
+ * (nccl_unique_id == NULL) the caller routes: each shard receives the edge ops whose
+ * source it owns plus every node op, with explicit global seq numbers, and combines
+ * shard bases itself; h2tap_replica_info reports the shard's rows/edges and its
+ * global row base. */
 typedef struct {
     int device;                  /* CUDA device ordinal */
     int rank, world;             /* world == 1 for a single replica */
-    const void* nccl_unique_id;  /* ncclUniqueId bytes (world > 1), else NULL */
+    const void* nccl_unique_id;  /* ncclUniqueId bytes (collective mode), else NULL */
+    const uint64_t* shard_bounds;/* world + 1 non-decreasing external-ID split points (host),
+                                    NULL if world == 1; world <= 4096, else H2TAP_E_INVAL */
     uint64_t expected_batch;     /* capacity hint (ops per batch); 0 = none */
     h2tap_allocator alloc;
     void* stream;                /* cudaStream_t; NULL = legacy default stream */
@@ -131,6 +144,33 @@ h2tap_status h2tap_replica_create_from_csr(const h2tap_config* cfg, size_t n_ver
  * E_INVAL; any batch op with ts <= current snapshot_ts -> E_STALE_TS. */
 h2tap_status h2tap_delta_apply(h2tap_replica* r, const h2tap_batch* batch, uint64_t snapshot_ts,
         h2tap_apply_stats* stats /* nullable */);
+
+/* ---- exchange step of a sharded apply ----------------------
+ * A rank holding a slice of the global batch (i) validates it (every rank must agree
+ * before anything is applied), (ii) packs its ops into 40-byte route records grouped
+ * by destination shard — an edge op goes to the shard owning its source, a node op to
+ * every shard — (iii) exchanges them with an all-to-all (NCCL over NVLink; the caller's
+ * process group), and (iv) applies what it received. */
+typedef struct {
+    uint64_t src, dst, ts, seq;  /* seq: global rank-major arrival number (reading A5) */
+    float w;
+    uint8_t kind;
+    uint8_t pad[3];
+} h2tap_route_rec;
+
+/* E_INVAL (unknown kind) / E_STALE_TS (ts <= snapshot) / OK for a batch slice. */
+h2tap_status h2tap_batch_validate(const h2tap_replica* r, const h2tap_batch* batch);
+
+/* Pack `batch` (on_device must be 1) into `out` (device, `capacity` records), grouped
+ * by destination rank 0..world-1; counts[world] (host) receives the records per
+ * destination.  Op i gets seq = seq0 + i.  Needs n_edge + world * n_node records; if
+ * capacity is smaller, returns E_CAPACITY with counts filled (retry with more). */
+h2tap_status h2tap_route_pack(const h2tap_replica* r, const h2tap_batch* batch, uint64_t seq0,
+        h2tap_route_rec* out, uint64_t capacity, uint64_t* counts);
+
+/* h2tap_delta_apply on received route records (device, n records, any order). */
+h2tap_status h2tap_delta_apply_routed(h2tap_replica* r, const h2tap_route_rec* recs, size_t n,
+        uint64_t snapshot_ts, h2tap_apply_stats* stats /* nullable */);
 
 /* Sizes of the current replica (any pointer may be NULL). */
 h2tap_status h2tap_replica_info(const h2tap_replica* r, uint64_t* n_vertices, uint64_t* n_edges,

@@ -48,13 +48,13 @@ class _Allocator(ctypes.Structure):
 
 class _Config(ctypes.Structure):
     _fields_ = [("device", ctypes.c_int), ("rank", ctypes.c_int), ("world", ctypes.c_int),
-                ("nccl_unique_id", _P), ("expected_batch", _u64), ("alloc", _Allocator),
-                ("stream", _P)]
+                ("nccl_unique_id", _P), ("shard_bounds", _P), ("expected_batch", _u64),
+                ("alloc", _Allocator), ("stream", _P)]
 
 
 class _Batch(ctypes.Structure):
     _fields_ = [("n", ctypes.c_size_t), ("on_device", ctypes.c_int), ("kind", _P), ("src", _P),
-                ("dst", _P), ("weight", _P), ("ts", _P)]
+                ("dst", _P), ("weight", _P), ("ts", _P), ("seq", _P)]
 
 
 class ApplyStats(ctypes.Structure):
@@ -78,6 +78,13 @@ _lib.h2tap_replica_create_from_csr.argtypes = [ctypes.POINTER(_Config), ctypes.c
                                                _P, ctypes.c_int, _u64, ctypes.POINTER(_P)]
 _lib.h2tap_delta_apply.restype = ctypes.c_int
 _lib.h2tap_delta_apply.argtypes = [_P, ctypes.POINTER(_Batch), _u64, ctypes.POINTER(ApplyStats)]
+_lib.h2tap_batch_validate.restype = ctypes.c_int
+_lib.h2tap_batch_validate.argtypes = [_P, ctypes.POINTER(_Batch)]
+_lib.h2tap_route_pack.restype = ctypes.c_int
+_lib.h2tap_route_pack.argtypes = [_P, ctypes.POINTER(_Batch), _u64, _P, _u64, ctypes.POINTER(_u64)]
+_lib.h2tap_delta_apply_routed.restype = ctypes.c_int
+_lib.h2tap_delta_apply_routed.argtypes = [_P, _P, ctypes.c_size_t, _u64, ctypes.POINTER(ApplyStats)]
+ROUTE_REC_BYTES = 40  # sizeof(h2tap_route_rec)
 _lib.h2tap_replica_info.restype = ctypes.c_int
 _lib.h2tap_replica_info.argtypes = [_P] + [ctypes.POINTER(_u64)] * 6
 _lib.h2tap_replica_export.restype = ctypes.c_int
@@ -96,6 +103,17 @@ _lib.h2tap_version.restype = ctypes.c_char_p
 
 def version() -> str:
     return _lib.h2tap_version().decode()
+
+
+def balanced_bounds(src_ext, world: int) -> np.ndarray:
+    """world + 1 external-ID split points that balance the edges (rows are owned by their
+    source): quantiles of the edge sources' external IDs.  Host-side planning only."""
+    s = np.sort(np.asarray(src_ext, dtype=np.uint64))
+    b = np.zeros(world + 1, np.uint64)
+    for p in range(1, world):
+        b[p] = s[min(len(s) - 1, (len(s) * p) // world)] if len(s) else p
+    b[world] = np.iinfo(np.uint64).max
+    return np.maximum.accumulate(b)
 
 
 def _check(rc: int, where: str):
@@ -147,11 +165,17 @@ class Replica:
 
     # ---------------------------------------------------------------- create
     @staticmethod
-    def _config(device, stream, torch_allocator):
+    def _config(device, stream, torch_allocator, rank=0, world=1, shard_bounds=None):
         cfg = _Config()
         cfg.device = device
-        cfg.rank, cfg.world = 0, 1
+        cfg.rank, cfg.world = rank, world
         keep = []
+        if world > 1:
+            sb = np.ascontiguousarray(shard_bounds, dtype=np.uint64)
+            if sb.shape != (world + 1,):
+                raise ValueError("shard_bounds must have world + 1 entries")
+            cfg.shard_bounds = ctypes.c_void_p(sb.ctypes.data)
+            keep.append(sb)
         if torch_allocator:
             a, f = _torch_allocator(device)
             cfg.alloc.alloc, cfg.alloc.free = a, f
@@ -167,8 +191,10 @@ class Replica:
 
     @classmethod
     def from_edges(cls, n_vertices, vertex_ids, src, dst, w, create_ts=0, device=0, stream=None,
-                   torch_allocator=True) -> "Replica":
-        cfg, keep = cls._config(device, stream, torch_allocator)
+                   torch_allocator=True, rank=0, world=1, shard_bounds=None) -> "Replica":
+        """Create a replica (world > 1: shard `rank` of a vertex-range sharded graph; pass
+        the GLOBAL vertex set and only the edges whose source this shard owns)."""
+        cfg, keep = cls._config(device, stream, torch_allocator, rank, world, shard_bounds)
         pi, ps, pd, pw = (_ptr(vertex_ids, np.uint64), _ptr(src, np.uint64), _ptr(dst, np.uint64),
                           _ptr(w, np.float32))
         ond = _on_device(pi, ps, pd, pw)
@@ -194,15 +220,43 @@ class Replica:
         return cls(h, keep + [cfg])
 
     # ----------------------------------------------------------------- apply
-    def apply(self, batch, snapshot_ts: int, raise_on_error: bool = True):
-        """h2tap_delta_apply; batch has .kind .src .dst .w .ts (numpy or torch CUDA)."""
+    @staticmethod
+    def _batch(batch):
         pk, ps, pd, pw, pt = (_ptr(batch.kind, np.uint8), _ptr(batch.src, np.uint64),
                               _ptr(batch.dst, np.uint64), _ptr(batch.w, np.float32),
                               _ptr(batch.ts, np.uint64))
+        pq = _ptr(getattr(batch, "seq", None), np.uint64)
         b = _Batch()
         b.n = len(batch.kind)
-        b.on_device = _on_device(pk, ps, pd, pw, pt)
-        b.kind, b.src, b.dst, b.weight, b.ts = pk[0], ps[0], pd[0], pw[0], pt[0]
+        b.on_device = _on_device(pk, ps, pd, pw, pt, pq)
+        b.kind, b.src, b.dst, b.weight, b.ts, b.seq = pk[0], ps[0], pd[0], pw[0], pt[0], pq[0]
+        return b, (pk, ps, pd, pw, pt, pq)
+
+    def validate(self, batch) -> int:
+        """h2tap_batch_validate: status code of a batch slice (0 = OK)."""
+        b, keep = self._batch(batch)
+        return _lib.h2tap_batch_validate(self._h, ctypes.byref(b))
+
+    def route_pack(self, batch, seq0: int, out, capacity_records: int):
+        """h2tap_route_pack into `out` (torch CUDA uint8, >= capacity*40 bytes); returns
+        (status, counts[world])."""
+        b, keep = self._batch(batch)
+        world = self._keep[-1].world if self._keep else 1
+        counts = (_u64 * max(1, world))()
+        rc = _lib.h2tap_route_pack(self._h, ctypes.byref(b), int(seq0), ctypes.c_void_p(out.data_ptr()),
+                                   int(capacity_records), counts)
+        return rc, [int(x) for x in counts]
+
+    def apply_routed(self, recs, n: int, snapshot_ts: int):
+        """h2tap_delta_apply_routed on `n` received route records (torch CUDA uint8)."""
+        st = ApplyStats()
+        _check(_lib.h2tap_delta_apply_routed(self._h, ctypes.c_void_p(recs.data_ptr()) if n else None, int(n),
+                                             int(snapshot_ts), ctypes.byref(st)), "h2tap_delta_apply_routed")
+        return st.as_dict()
+
+    def apply(self, batch, snapshot_ts: int, raise_on_error: bool = True):
+        """h2tap_delta_apply; batch has .kind .src .dst .w .ts (numpy or torch CUDA)."""
+        b, keep = self._batch(batch)
         st = ApplyStats()
         rc = _lib.h2tap_delta_apply(self._h, ctypes.byref(b), int(snapshot_ts), ctypes.byref(st))
         if raise_on_error:

@@ -19,6 +19,7 @@
 #include <cstring>
 #include <new>
 #include <string>
+#include <vector>
 
 #include "../../include/h2tap.h"
 #include "kernels.cuh"
@@ -109,6 +110,12 @@ struct h2tap_replica {
     cudaStream_t st = nullptr, st2 = nullptr;  // st2: side stream (cascade pass)
     cudaEvent_t evA = nullptr, evB = nullptr;
     uint64_t V = 0, E = 0, snap = 0, next_seq = 0, n_pend = 0;
+    // sharding: V = global live vertices (the replicated ID map), the CSR holds the Vr rows
+    // of the owned external-ID range starting at global dense id row_lo
+    bool sharded = false;
+    OwnRange own{0, ~0ull};
+    Buf bounds_dev;  // world + 1 split points (device) for routing
+    uint64_t row_lo = 0, Vr = 0;
     bool identity = true, poisoned = false;
     int n_sm = 148;
     int cur = 0, ext_cur = 0, pcur = 0;
@@ -205,12 +212,14 @@ void radix_sort(h2tap_replica* r, uint64_t*& k, uint32_t*& v, uint64_t*& k2, uin
 struct BatchIn {
     uint64_t n;
     int on_device;
+    const uint64_t* seq;  // NULL -> next_seq + i
     const uint8_t* kind;  // NULL -> all EDGE_INSERT (create)
     const uint64_t* src;
     const uint64_t* dst;
     const float* w;
     const uint64_t* ts;   // NULL -> all create_ts (create)
     uint64_t fill_ts;
+    const RouteRec* recs = nullptr;  // routed records (device) instead of the SoA arrays
 };
 
 template <typename T>
@@ -286,7 +295,10 @@ h2tap_status apply_core(h2tap_replica* r, const BatchIn& in, uint64_t S, bool cr
         CK(cudaMemcpyAsync(Wt, r->pt[pc].p, np * 8, cudaMemcpyDeviceToDevice, st));
         CK(cudaMemcpyAsync(Wq, r->pq[pc].p, np * 8, cudaMemcpyDeviceToDevice, st));
     }
-    if (n) {
+    if (n && in.recs) {
+        k_unpack_recs<<<g1(n), 256, 0, st>>>(in.recs, n, Wk + np, Ws + np, Wd + np, Ww + np, Wt + np, Wq + np);
+        CKL();
+    } else if (n) {
         if (in.kind) copy_in(r, Wk + np, in.kind, n, in.on_device);
         else { k_fill_u8<<<g1(n), 256, 0, st>>>(Wk + np, n, EDGE_INSERT); CKL(); }
         copy_in(r, Ws + np, in.src, n, in.on_device);
@@ -296,8 +308,8 @@ h2tap_status apply_core(h2tap_replica* r, const BatchIn& in, uint64_t S, bool cr
         else CK(cudaMemsetAsync(Ww + np, 0, n * 4, st));
         if (in.ts) copy_in(r, Wt + np, in.ts, n, in.on_device);
         else { k_fill_u64<<<g1(n), 256, 0, st>>>(Wt + np, n, in.fill_ts); CKL(); }
-        k_fill_seq<<<g1(n), 256, 0, st>>>(Wq, np, n, r->next_seq);
-        CKL();
+        if (in.seq) copy_in(r, Wq + np, in.seq, n, in.on_device);
+        else { k_fill_seq<<<g1(n), 256, 0, st>>>(Wq, np, n, r->next_seq); CKL(); }
     }
     Ops ops{Wk, Ws, Wd, Ww, Wt, Wq};
 
@@ -334,7 +346,8 @@ h2tap_status apply_core(h2tap_replica* r, const BatchIn& in, uint64_t S, bool cr
     CK(cudaEventRecord(r->ev[1], st));
 
     // ---- a2: node ops -> per-vertex timeline, ID-map compaction, remap
-    const uint64_t V = r->V, E = r->E;
+    const uint64_t V = r->V, E = r->E, row_lo = r->row_lo, Vr = r->Vr;
+    uint64_t row_lo_new = row_lo, Vr_new = Vr;
     const int ec = r->ext_cur;
     const uint64_t* old_ext = static_cast<const uint64_t*>(r->ext[ec].p);
     uint64_t U = 0, n_dropped = 0, n_vins = 0, n_hd = 0, Vn = V;
@@ -435,6 +448,15 @@ h2tap_status apply_core(h2tap_replica* r, const BatchIn& in, uint64_t S, bool cr
         }
         k_nv_newid<<<g1(U), 256, 0, st>>>(nv, U, R);
         CKL();
+        if (r->sharded) {
+            k_row_range<<<1, 1, 0, st>>>(set_changed ? new_ext : old_ext, Vn, r->own, dc);
+            CKL();
+            r->read_counters();
+            row_lo_new = r->hc->row_lo_new;
+            Vr_new = r->hc->row_hi_new - r->hc->row_lo_new;
+        } else {
+            Vr_new = Vn;
+        }
         if (n_hd) {
             hd_bits = r->get<uint32_t>(r->hd_bits, cdiv(V, 32));
             CK(cudaMemsetAsync(hd_bits, 0, cdiv(V, 32) * 4, st));
@@ -457,7 +479,7 @@ h2tap_status apply_core(h2tap_replica* r, const BatchIn& in, uint64_t S, bool cr
                 k_casc_cols<<<(unsigned)cdiv(nblk, 2), kThreads, 0, s2>>>(old_cols_nc, E, hd_bits, hd_rows, n_hd, casc_mask);
                 CKL();
                 TR("casc_cols");
-                k_casc_rows<<<rg, 256, 0, s2>>>(old_off_nc, hd_rows, n_hd, casc_mask);
+                k_casc_rows<<<rg, 256, 0, s2>>>(old_off_nc, hd_rows, n_hd, row_lo, row_lo + Vr, casc_mask);
                 CKL();
                 TR("casc_rows");
             }
@@ -501,6 +523,7 @@ h2tap_status apply_core(h2tap_replica* r, const BatchIn& in, uint64_t S, bool cr
         pa.node_sorted = node_sorted;
         pa.bits = bits;
         pa.create = create ? 1 : 0;
+        pa.own = r->own;
         pa.keys = kA;
         pa.vals = vA;
         pa.recs = r->get<EdgeRec>(r->op_flags, m);
@@ -519,6 +542,10 @@ h2tap_status apply_core(h2tap_replica* r, const BatchIn& in, uint64_t S, bool cr
         TR("sync_prep");
         if (create && (r->hc->status & ST_CREATE_ENDPOINT)) {
             set_err("create: edge endpoint not in the vertex set");
+            return H2TAP_E_INVAL;
+        }
+        if (r->hc->status & ST_NOT_OWNED) {
+            set_err("sharded replica: edge op whose source is owned by another shard");
             return H2TAP_E_INVAL;
         }
         n_valid = r->hc->n_valid;
@@ -541,7 +568,7 @@ h2tap_status apply_core(h2tap_replica* r, const BatchIn& in, uint64_t S, bool cr
             ca.n = n_valid;
             ca.bits = bits;
             ca.recs = pa.recs;
-            ca.old_off = old_off;
+            ca.old_off = old_off - row_lo;  // indexed by global dense ids of owned rows
             ca.old_cols = old_cols;
             ca.V_old = V;
             ca.ins_pos = ins_pos; ca.ins_row = ins_row; ca.ins_col = ins_col; ca.ins_w = ins_w;
@@ -571,14 +598,14 @@ h2tap_status apply_core(h2tap_replica* r, const BatchIn& in, uint64_t S, bool cr
     uint64_t n_casc = 0, En = E;
     if (csr_changed) {
     const uint64_t Ecap = E + n_ins;
-    int64_t* new_off = r->get<int64_t>(r->off[nb], Vn + 1);
+    int64_t* new_off = r->get<int64_t>(r->off[nb], Vr_new + 1);
     uint32_t* new_cols = r->get<uint32_t>(r->cols[nb], Ecap);
     float* new_w = r->get<float>(r->w[nb], Ecap);
     const bool casc = n_hd > 0;
     const uint64_t Dtot = E + n_ins;
     if (Dtot) {
         MergeArgs ma{};
-        ma.old_cols = old_cols; ma.old_w = old_w; ma.old_off = old_off; ma.E_old = E; ma.V_old = V;
+        ma.old_cols = old_cols; ma.old_w = old_w; ma.old_off = old_off; ma.E_old = E; ma.V_old = Vr;
         ma.ins_pos = ins_pos; ma.ins_col = ins_col; ma.ins_w = ins_w; ma.n_ins = n_ins;
         ma.del_pos = del_pos; ma.n_del = n_del;
         ma.upd_pos = upd_pos; ma.upd_w = upd_w; ma.n_upd = n_upd;
@@ -612,7 +639,7 @@ h2tap_status apply_core(h2tap_replica* r, const BatchIn& in, uint64_t S, bool cr
         CKL();
     } else {
         // nothing to merge: every surviving row is empty
-        if (n_node) CK(cudaMemsetAsync(new_off, 0, (Vn + 1) * 8, st));
+        if (n_node) CK(cudaMemsetAsync(new_off, 0, (Vr_new + 1) * 8, st));
         CK(cudaEventRecord(r->ev[6], st));
     }
     CK(cudaEventRecord(r->ev[4], st));
@@ -624,16 +651,16 @@ h2tap_status apply_core(h2tap_replica* r, const BatchIn& in, uint64_t S, bool cr
     En = E + n_ins - n_del - n_casc;
 
     // ---- a4/a5: row offsets
-    if (V && !n_node) {
+    if (Vr && !n_node) {
         // per-vertex degree delta + exclusive scan (tile sums by decoupled look-back)
-        int32_t* deg = r->get<int32_t>(r->deg, V);
-        const uint64_t nt = cdiv(V, kTile);
+        int32_t* deg = r->get<int32_t>(r->deg, Vr);
+        const uint64_t nt = cdiv(Vr, kTile);
         int64_t* tsum = r->get<int64_t>(r->tsum, nt + 1);
         int64_t* tbase = r->get<int64_t>(r->KR, nt + 1);
-        CK(cudaMemsetAsync(deg, 0, V * 4, st));
+        CK(cudaMemsetAsync(deg, 0, Vr * 4, st));
         CK(cudaMemsetAsync(tsum, 0, (nt + 1) * 8, st));
         if (n_ins + n_del) {
-            k_deg_scatter<<<g1(n_ins + n_del), 256, 0, st>>>(ins_row, n_ins, static_cast<uint32_t*>(r->del_row.p), n_del, deg, tsum);
+            k_deg_scatter<<<g1(n_ins + n_del), 256, 0, st>>>(ins_row, n_ins, static_cast<uint32_t*>(r->del_row.p), n_del, deg, tsum, row_lo);
             CKL();
         }
         const uint64_t nts = cdiv(nt, kTile);
@@ -641,28 +668,29 @@ h2tap_status apply_core(h2tap_replica* r, const BatchIn& in, uint64_t S, bool cr
         CK(cudaMemsetAsync(stt, 0, nts * 8, st));
         k_scan_exclusive_i64<<<(unsigned)nts, kThreads, 0, st>>>(tsum, tbase, nt, stt, &dc->tiles[7]);
         CKL();
-        k_offsets_apply<<<(unsigned)nt, kThreads, 0, st>>>(old_off, deg, V, tbase, new_off);
+        k_offsets_apply<<<(unsigned)nt, kThreads, 0, st>>>(old_off, deg, Vr, tbase, new_off);
         CKL();
     }
-    if (V && n_node) {
+    if (n_node && (Vr || Vr_new)) {
         RowArgs ra{};
-        ra.old_off = old_off; ra.V_old = V; ra.E_old = E; ra.R = R;
+        ra.old_off = old_off - row_lo; ra.V_old = V; ra.E_old = E; ra.R = R;
+        ra.row_lo = row_lo; ra.row_hi = row_lo + Vr; ra.row_lo_new = row_lo_new;
+        ra.own = r->own; ra.nv_ext = nv_ext;
         ra.casc_mask = casc ? casc_mask : nullptr; ra.casc_pre = casc_pre; ra.casc_wrel = casc_wrel;
         ra.del_pos = del_pos; ra.n_del = n_del; ra.ins_row = ins_row; ra.n_ins = n_ins;
         ra.dropped = dropped; ra.n_dropped = n_dropped; ra.ins_oldpos = ins_oldpos; ra.n_vins = n_vins;
         ra.new_off = new_off;
-        const uint64_t ncta = cdiv(V, kRowTile);
+        const uint64_t ncta = cdiv(Vr, kRowTile);
         ra.part = r->get<uint64_t>(r->opart, 2 * (ncta + 1));
         k_rows_partition<<<g1(ncta + 1), 256, 0, st>>>(ra);
         CKL();
-        k_offsets_rows<<<(unsigned)ncta, kThreads, 0, st>>>(ra);
-        CKL();
+        if (ncta) { k_offsets_rows<<<(unsigned)ncta, kThreads, 0, st>>>(ra); CKL(); }
         if (n_vins) {
             k_offsets_inserted<<<g1(n_vins), 256, 0, st>>>(nv, ins_q, n_vins, ra);
             CKL();
         }
     }
-    k_set_i64<<<1, 1, 0, st>>>(new_off + Vn, (int64_t)En);
+    k_set_i64<<<1, 1, 0, st>>>(new_off + Vr_new, (int64_t)En);
     CKL();
     } else {
         CK(cudaEventRecord(r->ev[6], st));
@@ -702,6 +730,8 @@ h2tap_status apply_core(h2tap_replica* r, const BatchIn& in, uint64_t S, bool cr
     r->identity = new_identity;
     r->V = Vn;
     r->E = En;
+    r->row_lo = row_lo_new;
+    r->Vr = Vr_new;
     r->pcur = pn;
     r->n_pend = n_pend_new;
     r->next_seq += n;
@@ -725,7 +755,7 @@ h2tap_status apply_core(h2tap_replica* r, const BatchIn& in, uint64_t S, bool cr
         stats->ms_merge = ev_ms(r->ev[6], r->ev[4]);
         stats->ms_degree_scan = ev_ms(r->ev[3], r->ev[6]) + ev_ms(r->ev[4], r->ev[5]);
         stats->ms_total = ev_ms(r->ev[0], r->ev[5]);
-        uint64_t b = 8 * (V + 1) + 8 * E + 8 * (Vn + 1) + 8 * En + 29 * n;
+        uint64_t b = 8 * (Vr + 1) + 8 * E + 8 * (Vr_new + 1) + 8 * En + 29 * n;
         if (n_node) b += 16 * V + 4 * E + 4 * V;
         stats->bytes_alg = b;
         // merge launch: stream old cols+weights, write new ones, read the outcome lists
@@ -769,6 +799,29 @@ h2tap_replica* new_replica(const h2tap_config* cfg) {
     if (cfg) r->cfg = *cfg;
     else { r->cfg.world = 1; }
     if (r->cfg.world <= 0) r->cfg.world = 1;
+    if (r->cfg.world > 1) {
+        if (!r->cfg.shard_bounds || r->cfg.rank < 0 || r->cfg.rank >= r->cfg.world) {
+            set_err("sharded replica needs shard_bounds[world+1] and 0 <= rank < world");
+            throw Fail{H2TAP_E_INVAL};
+        }
+        if (r->cfg.world > 4096) { set_err("world > 4096"); throw Fail{H2TAP_E_INVAL}; }
+        for (int p = 0; p < r->cfg.world; ++p)
+            if (r->cfg.shard_bounds[p] > r->cfg.shard_bounds[p + 1]) {
+                set_err("shard_bounds must be non-decreasing");
+                throw Fail{H2TAP_E_INVAL};
+            }
+        if (r->cfg.nccl_unique_id) {
+            set_err("collective mode (NCCL communicator inside the library) is not in this build; "
+                    "use caller-routed sharding (nccl_unique_id = NULL)");
+            throw Fail{H2TAP_E_INVAL};
+        }
+        r->sharded = true;
+        uint64_t* bd = r->get<uint64_t>(r->bounds_dev, r->cfg.world + 1);
+        CK(cudaMemcpy(bd, r->cfg.shard_bounds, (r->cfg.world + 1) * 8, cudaMemcpyHostToDevice));
+        r->own.lo = r->cfg.shard_bounds[r->cfg.rank];
+        r->own.hi = (r->cfg.rank == r->cfg.world - 1) ? ~0ull : r->cfg.shard_bounds[r->cfg.rank + 1];
+        r->cfg.shard_bounds = nullptr;  // not retained
+    }
     CK(cudaSetDevice(r->cfg.device));
     CK(cudaDeviceGetAttribute(&r->n_sm, cudaDevAttrMultiProcessorCount, r->cfg.device));
     r->st = static_cast<cudaStream_t>(r->cfg.stream);
@@ -794,7 +847,7 @@ void free_replica(h2tap_replica* r) {
                    &r->hist, &r->dbase, &r->rs_status, &r->rs_ctr, &r->nv, &r->nv_ext, &r->dropped, &r->ins_q,
                    &r->ins_oldpos, &r->hd_rows, &r->hd_bits, &r->op_flags, &r->op_ou, &r->op_ow,
                    &r->ins_pos, &r->ins_row, &r->ins_col, &r->ins_w, &r->del_pos, &r->upd_pos, &r->upd_w,
-                   &r->KR, &r->misc, &r->nsorted, &r->part, &r->opart, &r->deg, &r->tsum, &r->remap_shift, &r->remap32, &r->casc_wrel, &r->tile_emit, &r->tile_base, &r->del_row, &r->casc_mask, &r->status2, &r->fence[0], &r->fence[1], &r->bfs_a, &r->bfs_b, &r->pr_a, &r->pr_b, &r->ctr};
+                   &r->KR, &r->misc, &r->nsorted, &r->part, &r->opart, &r->deg, &r->tsum, &r->remap_shift, &r->remap32, &r->casc_wrel, &r->tile_emit, &r->tile_base, &r->del_row, &r->casc_mask, &r->status2, &r->bounds_dev, &r->fence[0], &r->fence[1], &r->bfs_a, &r->bfs_b, &r->pr_a, &r->pr_b, &r->ctr};
     for (Buf* b : bufs) if (b->p) r->dfree(b->p);
     cudaStreamSynchronize(r->st);
     for (auto& e : r->ev) if (e) cudaEventDestroy(e);
@@ -831,6 +884,16 @@ void init_vertices(h2tap_replica* r, uint64_t nv, const uint64_t* ids, int on_de
         r->identity = (h[1] == nv - 1);
     }
     build_fence(r, 0, nv);
+    r->row_lo = 0;
+    r->Vr = nv;
+    if (r->sharded) {
+        k_row_range<<<1, 1, 0, r->st>>>(ext, nv, r->own, r->dctr());
+        CKL();
+        r->read_counters();
+        r->row_lo = r->hc->row_lo_new;
+        r->Vr = r->hc->row_hi_new - r->hc->row_lo_new;
+        CK(cudaMemsetAsync(off, 0, (r->Vr + 1) * 8, r->st));
+    }
 }
 
 }  // namespace
@@ -860,7 +923,6 @@ h2tap_status h2tap_replica_create_from_edges(const h2tap_config* cfg, size_t n_v
                                              size_t n_edges, const uint64_t* src, const uint64_t* dst, const float* w,
                                              int on_device, uint64_t create_ts, h2tap_replica** out) {
     if (!out || (n_edges && (!src || !dst))) { set_err("null argument"); return H2TAP_E_INVAL; }
-    if (cfg && cfg->world > 1) { set_err("multi-GPU replicas are not enabled in this build"); return H2TAP_E_INVAL; }
     if (n_vertices >= 0xFFFFFFFFull) { set_err("n_vertices >= 2^32-1"); return H2TAP_E_CAPACITY; }
     *out = nullptr;
     h2tap_replica* r = nullptr;
@@ -868,7 +930,7 @@ h2tap_status h2tap_replica_create_from_edges(const h2tap_config* cfg, size_t n_v
         r = new_replica(cfg);
         init_vertices(r, n_vertices, vertex_ids, on_device);
         r->snap = 0;
-        BatchIn in{n_edges, on_device, nullptr, src, dst, w, nullptr, create_ts};
+        BatchIn in{n_edges, on_device, nullptr, nullptr, src, dst, w, nullptr, create_ts};
         h2tap_status st = apply_core(r, in, create_ts, true, nullptr);
         if (st != H2TAP_OK) return st;
         r->snap = create_ts;
@@ -884,7 +946,7 @@ h2tap_status h2tap_replica_create_from_csr(const h2tap_config* cfg, size_t n_ver
                                            const uint32_t* cols, const float* w, const uint64_t* ext_ids,
                                            int on_device, uint64_t create_ts, h2tap_replica** out) {
     if (!out || !offsets) { set_err("null argument"); return H2TAP_E_INVAL; }
-    if (cfg && cfg->world > 1) { set_err("multi-GPU replicas are not enabled in this build"); return H2TAP_E_INVAL; }
+    if (cfg && cfg->world > 1) { set_err("create_from_csr: sharded replicas are created from edges"); return H2TAP_E_INVAL; }
     if (n_vertices >= 0xFFFFFFFFull) { set_err("n_vertices >= 2^32-1"); return H2TAP_E_CAPACITY; }
     *out = nullptr;
     h2tap_replica* r = nullptr;
@@ -931,7 +993,89 @@ h2tap_status h2tap_delta_apply(h2tap_replica* r, const h2tap_batch* b, uint64_t 
             return H2TAP_E_SNAPSHOT_REGRESSION;
         }
         CK(cudaSetDevice(r->cfg.device));
-        BatchIn in{b->n, b->on_device, b->kind, b->src, b->dst, b->weight, b->ts, 0};
+        BatchIn in{b->n, b->on_device, b->seq, b->kind, b->src, b->dst, b->weight, b->ts, 0};
+        return apply_core(r, in, snapshot_ts, false, stats);
+    });
+}
+
+h2tap_status h2tap_batch_validate(const h2tap_replica* rc, const h2tap_batch* b) {
+    h2tap_replica* r = const_cast<h2tap_replica*>(rc);
+    if (!r || !b) { set_err("null argument"); return H2TAP_E_INVAL; }
+    if (b->n && (!b->kind || !b->ts)) { set_err("batch kind/ts must be non-NULL"); return H2TAP_E_INVAL; }
+    return run_guarded(r, [&]() -> h2tap_status {
+        CK(cudaSetDevice(r->cfg.device));
+        if (!b->n) return H2TAP_OK;
+        const uint8_t* kind = b->kind;
+        const uint64_t* ts = b->ts;
+        if (!b->on_device) {  // stage host slices
+            kind = r->get<uint8_t>(r->Wk, b->n);
+            ts = r->get<uint64_t>(r->Wt, b->n);
+            copy_in(r, const_cast<uint8_t*>(kind), b->kind, b->n, 0);
+            copy_in(r, const_cast<uint64_t*>(ts), b->ts, b->n, 0);
+        }
+        unsigned long long* st = r->get<unsigned long long>(r->misc, 1);
+        CK(cudaMemsetAsync(st, 0, 8, r->st));
+        k_validate<<<(unsigned)std::min<uint64_t>(cdiv(b->n, 256), 148 * 8), 256, 0, r->st>>>(kind, ts, b->n, r->snap, st);
+        CKL();
+        unsigned long long h = 0;
+        CK(cudaMemcpyAsync(&h, st, 8, cudaMemcpyDeviceToHost, r->st));
+        r->sync();
+        if (h & ST_BAD_KIND) { set_err("unknown op kind in batch"); return H2TAP_E_INVAL; }
+        if (h & ST_STALE) { set_err("op with ts <= current snapshot_ts (reading A7)"); return H2TAP_E_STALE_TS; }
+        return H2TAP_OK;
+    });
+}
+
+h2tap_status h2tap_route_pack(const h2tap_replica* rc, const h2tap_batch* b, uint64_t seq0, h2tap_route_rec* out,
+                              uint64_t capacity, uint64_t* counts) {
+    h2tap_replica* r = const_cast<h2tap_replica*>(rc);
+    if (!r || !b || !counts) { set_err("null argument"); return H2TAP_E_INVAL; }
+    if (!r->sharded) { set_err("h2tap_route_pack: replica is not sharded"); return H2TAP_E_INVAL; }
+    if (b->n && (!b->on_device || !b->kind || !b->src || !b->ts)) { set_err("route_pack needs a device batch"); return H2TAP_E_INVAL; }
+    return run_guarded(r, [&]() -> h2tap_status {
+        CK(cudaSetDevice(r->cfg.device));
+        const int P = r->cfg.world;
+        const uint64_t* bounds = static_cast<const uint64_t*>(r->bounds_dev.p);
+        unsigned long long* cnt = r->get<unsigned long long>(r->misc, P);
+        CK(cudaMemsetAsync(cnt, 0, P * 8, r->st));
+        if (b->n) {
+            k_route_count<<<(unsigned)std::min<uint64_t>(cdiv(b->n, 256), 148 * 8), 256, (P + 1) * 4, r->st>>>(b->kind, b->src, b->n, bounds, P, cnt);
+            CKL();
+        }
+        std::vector<unsigned long long> h(P);
+        CK(cudaMemcpyAsync(h.data(), cnt, P * 8, cudaMemcpyDeviceToHost, r->st));
+        r->sync();
+        uint64_t tot = 0;
+        for (int d = 0; d < P; ++d) { counts[d] = h[d]; tot += h[d]; }
+        if (tot > capacity) { set_err("route_pack: %llu records needed", (unsigned long long)tot); return H2TAP_E_CAPACITY; }
+        if (!b->n) return H2TAP_OK;
+        const uint64_t nt = cdiv(b->n, kTile);
+        uint64_t* stt = r->get<uint64_t>(r->status, nt);
+        unsigned int* ctr = r->get<unsigned int>(r->rs_ctr, P);
+        CK(cudaMemsetAsync(ctr, 0, P * 4, r->st));
+        uint64_t base = 0;
+        for (int d = 0; d < P; ++d) {
+            CK(cudaMemsetAsync(stt, 0, nt * 8, r->st));
+            k_route_pack<<<(unsigned)nt, kThreads, 0, r->st>>>(b->kind, b->src, b->dst, b->weight, b->ts, b->n, seq0, bounds, P, d,
+                                                           reinterpret_cast<RouteRec*>(out) + base, stt, ctr + d);
+            CKL();
+            base += h[d];
+        }
+        r->sync();
+        return H2TAP_OK;
+    });
+}
+
+h2tap_status h2tap_delta_apply_routed(h2tap_replica* r, const h2tap_route_rec* recs, size_t n, uint64_t snapshot_ts,
+                                      h2tap_apply_stats* stats) {
+    if (!r || (n && !recs)) { set_err("null argument"); return H2TAP_E_INVAL; }
+    return run_guarded(r, [&]() -> h2tap_status {
+        if (snapshot_ts < r->snap) {
+            set_err("snapshot_ts %llu < current %llu", (unsigned long long)snapshot_ts, (unsigned long long)r->snap);
+            return H2TAP_E_SNAPSHOT_REGRESSION;
+        }
+        CK(cudaSetDevice(r->cfg.device));
+        BatchIn in{n, 1, nullptr, nullptr, nullptr, nullptr, nullptr, nullptr, 0, reinterpret_cast<const RouteRec*>(recs)};
         return apply_core(r, in, snapshot_ts, false, stats);
     });
 }
@@ -939,12 +1083,12 @@ h2tap_status h2tap_delta_apply(h2tap_replica* r, const h2tap_batch* b, uint64_t 
 h2tap_status h2tap_replica_info(const h2tap_replica* r, uint64_t* nv, uint64_t* ne, uint64_t* snap, uint64_t* npend,
                                 uint64_t* vbase, uint64_t* ebase) {
     if (!r) { set_err("null replica"); return H2TAP_E_INVAL; }
-    if (nv) *nv = r->V;
+    if (nv) *nv = r->Vr;  // rows of this shard (= all vertices when not sharded)
     if (ne) *ne = r->E;
     if (snap) *snap = r->snap;
     if (npend) *npend = r->n_pend;
-    if (vbase) *vbase = 0;
-    if (ebase) *ebase = 0;
+    if (vbase) *vbase = r->row_lo;
+    if (ebase) *ebase = 0;  // caller-routed sharding: the caller sums the shards' edge counts
     return H2TAP_OK;
 }
 
@@ -956,18 +1100,19 @@ h2tap_status h2tap_replica_export(const h2tap_replica* rc, int64_t* offsets, uin
         CK(cudaSetDevice(r->cfg.device));
         cudaMemcpyKind k = on_device ? cudaMemcpyDeviceToDevice : cudaMemcpyDeviceToHost;
         const int c = r->cur;
-        if (offsets) CK(cudaMemcpyAsync(offsets, r->off[c].p, (r->V + 1) * 8, k, r->st));
+        const uint64_t* ext_own = static_cast<const uint64_t*>(r->ext[r->ext_cur].p) + r->row_lo;
+        if (offsets) CK(cudaMemcpyAsync(offsets, r->off[c].p, (r->Vr + 1) * 8, k, r->st));
         if (cols && r->E) CK(cudaMemcpyAsync(cols, r->cols[c].p, r->E * 4, k, r->st));
         if (w && r->E) CK(cudaMemcpyAsync(w, r->w[c].p, r->E * 4, k, r->st));
-        if (ext_ids && r->V) CK(cudaMemcpyAsync(ext_ids, r->ext[r->ext_cur].p, r->V * 8, k, r->st));
+        if (ext_ids && r->Vr) CK(cudaMemcpyAsync(ext_ids, ext_own, r->Vr * 8, k, r->st));
         if (checksums) {
             unsigned long long* cs = r->get<unsigned long long>(r->misc, 4);
             CK(cudaMemsetAsync(cs, 0, 32, r->st));
             auto grid = [](uint64_t n) { return (unsigned)std::max<uint64_t>(1, std::min<uint64_t>(cdiv(n, 256), 148 * 16)); };
-            k_checksum<int64_t><<<grid(r->V + 1), 256, 0, r->st>>>(static_cast<int64_t*>(r->off[c].p), r->V + 1, 1, cs);
+            k_checksum<int64_t><<<grid(r->Vr + 1), 256, 0, r->st>>>(static_cast<int64_t*>(r->off[c].p), r->Vr + 1, 1, cs);
             k_checksum<uint32_t><<<grid(r->E), 256, 0, r->st>>>(static_cast<uint32_t*>(r->cols[c].p), r->E, 2, cs + 1);
             k_checksum<float><<<grid(r->E), 256, 0, r->st>>>(static_cast<float*>(r->w[c].p), r->E, 3, cs + 2);
-            k_checksum<uint64_t><<<grid(r->V), 256, 0, r->st>>>(static_cast<uint64_t*>(r->ext[r->ext_cur].p), r->V, 4, cs + 3);
+            k_checksum<uint64_t><<<grid(r->Vr), 256, 0, r->st>>>(ext_own, r->Vr, 4, cs + 3);
             CKL();
             CK(cudaMemcpyAsync(checksums, cs, 32, cudaMemcpyDeviceToHost, r->st));
         }
@@ -979,6 +1124,7 @@ h2tap_status h2tap_replica_export(const h2tap_replica* rc, int64_t* offsets, uin
 h2tap_status h2tap_bfs(const h2tap_replica* rc, uint64_t source_ext, int32_t* level_out, int on_device) {
     h2tap_replica* r = const_cast<h2tap_replica*>(rc);
     if (!r || !level_out) { set_err("null argument"); return H2TAP_E_INVAL; }
+    if (r->sharded) { set_err("h2tap_bfs: not available on a sharded replica in this build"); return H2TAP_E_INVAL; }
     return run_guarded(r, [&]() -> h2tap_status {
         CK(cudaSetDevice(r->cfg.device));
         const uint64_t V = r->V;
@@ -1032,6 +1178,7 @@ h2tap_status h2tap_bfs(const h2tap_replica* rc, uint64_t source_ext, int32_t* le
 h2tap_status h2tap_pagerank(const h2tap_replica* rc, double damping, int iterations, double* rank_out, int on_device) {
     h2tap_replica* r = const_cast<h2tap_replica*>(rc);
     if (!r || !rank_out || iterations < 0) { set_err("bad argument"); return H2TAP_E_INVAL; }
+    if (r->sharded) { set_err("h2tap_pagerank: not available on a sharded replica in this build"); return H2TAP_E_INVAL; }
     return run_guarded(r, [&]() -> h2tap_status {
         CK(cudaSetDevice(r->cfg.device));
         const uint64_t V = r->V;

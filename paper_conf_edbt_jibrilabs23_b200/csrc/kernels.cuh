@@ -16,7 +16,7 @@ constexpr int kItems = 8;
 constexpr int kTile = kThreads * kItems;  // 2048 items per tile for select-style kernels
 
 enum : uint8_t { NODE_INSERT = 0, NODE_DELETE = 1, EDGE_INSERT = 2, EDGE_DELETE = 3, EDGE_WEIGHT = 4 };
-enum : uint64_t { ST_BAD_KIND = 1, ST_STALE = 2, ST_CREATE_ENDPOINT = 4 };
+enum : uint64_t { ST_BAD_KIND = 1, ST_STALE = 2, ST_CREATE_ENDPOINT = 4, ST_NOT_OWNED = 8 };
 
 // work ops: pending (older seq) ++ batch, SoA, in ascending seq order
 struct Ops {
@@ -37,7 +37,14 @@ struct Counters {
     unsigned long long n_valid, n_gated;
     unsigned long long n_ins, n_del, n_upd;
     unsigned long long n_casc;
+    unsigned long long row_lo_new, row_hi_new;  // sharded: the shard's row range in the new ID map
     unsigned int tiles[16];
+};
+
+// owned external-ID range of a shard: [lo, hi), hi == ~0 means "through UINT64_MAX"
+struct OwnRange {
+    uint64_t lo, hi;
+    __device__ __forceinline__ bool owns(uint64_t x) const { return x >= lo && (hi == ~0ull || x < hi); }
 };
 
 // per unique vertex touched by visible node ops (a2)
@@ -194,6 +201,90 @@ __device__ __forceinline__ uint64_t old_lookup(const ExtIndex& X, uint64_t x, bo
 __global__ void k_build_fence(const uint64_t* __restrict__ ext, uint64_t V, uint64_t* __restrict__ fence) {
     uint64_t i = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x;
     if ((i << kFenceShift) < V) fence[i] = ext[i << kFenceShift];
+}
+
+// ============================================================ a8 exchange ====
+// 40-byte route record (layout of h2tap_route_rec)
+struct RouteRec {
+    uint64_t src, dst, ts, seq;
+    float w;
+    uint8_t kind;
+    uint8_t pad[3];
+};
+static_assert(sizeof(RouteRec) == 40, "route record layout");
+
+__global__ void k_validate(const uint8_t* __restrict__ kind, const uint64_t* __restrict__ ts, uint64_t n,
+                           uint64_t snap, unsigned long long* __restrict__ status) {
+    uint64_t bad = 0;
+    for (uint64_t i = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; i < n; i += (uint64_t)gridDim.x * blockDim.x) {
+        if (kind[i] > EDGE_WEIGHT) bad |= ST_BAD_KIND;
+        if (ts[i] <= snap) bad |= ST_STALE;
+    }
+    if (bad) atomicOr(status, (unsigned long long)bad);
+}
+
+// owner shard of external id x: number of interior split points <= x
+__device__ __forceinline__ int owner_of(const uint64_t* __restrict__ bounds, int P, uint64_t x) {
+    int lo = 1, hi = P;  // interior bounds[1..P-1]
+    while (lo < hi) { int mid = (lo + hi) >> 1; if (bounds[mid] <= x) lo = mid + 1; else hi = mid; }
+    return lo - 1;
+}
+
+__global__ void k_route_count(const uint8_t* __restrict__ kind, const uint64_t* __restrict__ src, uint64_t n,
+                              const uint64_t* __restrict__ bounds, int P, unsigned long long* __restrict__ counts) {
+    extern __shared__ unsigned int s_cnt[];  // P + 1 block-local counters (slot P = node ops)
+    for (int d = threadIdx.x; d <= P; d += blockDim.x) s_cnt[d] = 0;
+    __syncthreads();
+    for (uint64_t i = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; i < n; i += (uint64_t)gridDim.x * blockDim.x)
+        atomicAdd(&s_cnt[kind[i] <= NODE_DELETE ? P : owner_of(bounds, P, src[i])], 1u);
+    __syncthreads();
+    for (int d = threadIdx.x; d < P; d += blockDim.x)
+        if (s_cnt[d] + s_cnt[P]) atomicAdd(&counts[d], (unsigned long long)(s_cnt[d] + s_cnt[P]));
+}
+
+// stable selection of the ops bound for shard d (node ops go everywhere) into its segment
+__global__ void __launch_bounds__(kThreads) k_route_pack(
+    const uint8_t* __restrict__ kind, const uint64_t* __restrict__ src, const uint64_t* __restrict__ dst,
+    const float* __restrict__ w, const uint64_t* __restrict__ ts, uint64_t n, uint64_t seq0,
+    const uint64_t* __restrict__ bounds, int P, int d, RouteRec* __restrict__ out,
+    uint64_t* __restrict__ status, unsigned int* __restrict__ ctr) {
+    __shared__ uint32_t s_tile;
+    __shared__ uint32_t s_cmp[kItems * kThreads / 32 + 1];
+    __shared__ uint64_t s_base;
+    if (threadIdx.x == 0) s_tile = atomicAdd(ctr, 1u);
+    __syncthreads();
+    const uint32_t tile = s_tile;
+    const uint64_t i0 = (uint64_t)tile * kTile + threadIdx.x;
+    bool f[kItems];
+    uint32_t pos[kItems];
+#pragma unroll
+    for (int j = 0; j < kItems; ++j) {
+        const uint64_t i = i0 + (uint64_t)j * kThreads;
+        f[j] = i < n && (kind[i] <= NODE_DELETE || owner_of(bounds, P, src[i]) == d);
+    }
+    const uint32_t tot = striped_compact<kThreads, kItems>(f, pos, s_cmp);
+    if (threadIdx.x < 32) {
+        const uint64_t b = lookback_warp(status, tile, tot);
+        if (lane_id() == 0) s_base = b;
+    }
+    __syncthreads();
+#pragma unroll
+    for (int j = 0; j < kItems; ++j) {
+        if (!f[j]) continue;
+        const uint64_t i = i0 + (uint64_t)j * kThreads;
+        RouteRec r;
+        r.src = src[i]; r.dst = dst ? dst[i] : 0; r.ts = ts[i]; r.seq = seq0 + i;
+        r.w = w ? w[i] : 0.f; r.kind = kind[i]; r.pad[0] = r.pad[1] = r.pad[2] = 0;
+        out[s_base + pos[j]] = r;
+    }
+}
+
+__global__ void k_unpack_recs(const RouteRec* __restrict__ recs, uint64_t n, uint8_t* kind, uint64_t* src,
+                              uint64_t* dst, float* w, uint64_t* ts, uint64_t* seq) {
+    const uint64_t i = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x;
+    if (i >= n) return;
+    const RouteRec r = recs[i];
+    kind[i] = r.kind; src[i] = r.src; dst[i] = r.dst; w[i] = r.w; ts[i] = r.ts; seq[i] = r.seq;
 }
 
 // ===================================================================== a2 ====
@@ -387,6 +478,7 @@ struct PrepArgs {
     const uint32_t* node_sorted;  // (v, ts, seq)-sorted node op indices
     int bits;                     // bits of a dense id in the packed key
     int create;                   // create_from_edges: endpoints must exist
+    OwnRange own;                 // sharded: every edge op's source must be owned here
     uint64_t* keys;
     uint32_t* vals;
     struct EdgeRec* recs;         // one compact record per surviving edge op, indexed by op
@@ -469,6 +561,7 @@ __global__ void __launch_bounds__(kThreads) k_edge_prep(PrepArgs a) {
         Lookup Lw = do_lookup(a, a.ops.dst[o]);
         bool ok = Lu.final_live && Lw.final_live;
         if (a.create && !(Lu.old_present && Lw.old_present)) nbad++;
+        if (!a.own.owns(a.ops.src[o])) nbad |= 1ull << 40;  // routed to the wrong shard
         if (ok && (Lu.hasD || Lw.hasD)) {
             // superseded by a later node delete of an endpoint (A8)
             if (Lu.hasD && pt_less(ts, seq, Lu.tD_ts, Lu.tD_seq)) ok = false;
@@ -496,8 +589,9 @@ __global__ void __launch_bounds__(kThreads) k_edge_prep(PrepArgs a) {
     }
     uint64_t gsum = warp_sum(ngated);
     if (lane_id() == 0 && gsum) atomicAdd(&a.c->n_gated, (unsigned long long)gsum);
-    uint64_t bsum = warp_sum(nbad);
+    uint64_t bsum = warp_sum(nbad & 0xFFFFFFFFFFull), osum = warp_sum(nbad >> 40);
     if (lane_id() == 0 && bsum) atomicOr(&a.c->status, (unsigned long long)ST_CREATE_ENDPOINT);
+    if (lane_id() == 0 && osum) atomicOr(&a.c->status, (unsigned long long)ST_NOT_OWNED);
     uint32_t tot = striped_compact<kThreads, kEItems>(valid, pos, s_cmp);
     if (threadIdx.x < 32) {
         uint64_t b = lookback_warp(a.status, tile, tot);
@@ -851,10 +945,11 @@ __global__ void __launch_bounds__(kThreads) k_casc_cols(const uint32_t* __restri
 
 // rows of deleted vertices -> whole bit ranges (warp per row), OR-ed into the mask
 __global__ void k_casc_rows(const int64_t* __restrict__ old_off, const uint32_t* __restrict__ hd_rows,
-                            uint64_t n_hd, uint32_t* __restrict__ mask) {
+                            uint64_t n_hd, uint64_t row_lo, uint64_t row_hi, uint32_t* __restrict__ mask) {
     const uint64_t nw = ((uint64_t)gridDim.x * blockDim.x) >> 5;
     for (uint64_t h = (blockIdx.x * (uint64_t)blockDim.x + threadIdx.x) >> 5; h < n_hd; h += nw) {
-        uint32_t k = hd_rows[h];
+        if (hd_rows[h] < row_lo || hd_rows[h] >= row_hi) continue;  // not a row of this shard
+        const uint64_t k = hd_rows[h] - row_lo;
         uint64_t b = (uint64_t)old_off[k], e = (uint64_t)old_off[k + 1];
         if (b == e) continue;
         uint64_t wb = b >> 5, we = (e - 1) >> 5;
@@ -928,6 +1023,10 @@ struct RowArgs {
     uint64_t n_vins;
     int64_t* new_off;
     uint64_t* part;  // [n_cta + 1][2]: delete rank and insert-row rank at each CTA's first row
+    uint64_t row_lo, row_hi;  // old rows of this shard (global dense ids); old_off is biased by row_lo
+    uint64_t row_lo_new;      // first new row of this shard (new_off is local)
+    OwnRange own;
+    const uint64_t* nv_ext;
 };
 __device__ __forceinline__ uint64_t casc_before(const RowArgs& a, uint64_t x) {
     if (!a.casc_mask) return 0;
@@ -939,11 +1038,11 @@ __device__ __forceinline__ uint64_t casc_before(const RowArgs& a, uint64_t x) {
 // CTA boundaries of k_offsets_rows: ranks of each CTA's first row in the two lists
 __global__ void k_rows_partition(RowArgs a) {
     const uint64_t c = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x;
-    const uint64_t ncta = (a.V_old + kRowTile - 1) / kRowTile;
+    const uint64_t ncta = (a.row_hi - a.row_lo + kRowTile - 1) / kRowTile;
     if (c > ncta) return;
-    const uint64_t k = c * kRowTile;
+    const uint64_t k = a.row_lo + c * kRowTile;
     uint64_t dr, ir;
-    if (k >= a.V_old) { dr = a.n_del; ir = a.n_ins; }
+    if (k >= a.row_hi) { dr = a.n_del; ir = a.n_ins; }
     else {
         dr = lower_bound_dev(a.del_pos, 0, a.n_del, (uint64_t)a.old_off[k]);
         // insert-row rank of the new id of the first surviving row >= k (compaction formula)
@@ -957,7 +1056,7 @@ __global__ void k_rows_partition(RowArgs a) {
 }
 
 __global__ void __launch_bounds__(kThreads) k_offsets_rows(RowArgs a) {
-    const uint64_t k0 = (uint64_t)blockIdx.x * kRowTile, k1 = min(k0 + kRowTile, a.V_old);
+    const uint64_t k0 = a.row_lo + (uint64_t)blockIdx.x * kRowTile, k1 = min(k0 + kRowTile, a.row_hi);
     const uint64_t* pp = a.part + 2 * blockIdx.x;  // this CTA's slices of the delete / insert-row lists
     const uint64_t da = pp[0], ia = pp[1], db = pp[2], ib = pp[3];
     constexpr int PER = kRowTile / kThreads;  // rows per thread, all loads issued together
@@ -977,7 +1076,7 @@ __global__ void __launch_bounds__(kThreads) k_offsets_rows(RowArgs a) {
     for (int j = 0; j < PER; ++j) {
         if (u[j] == kNone32) continue;
         const uint64_t kept = x[j] - cb[j] - lower_bound_dev(a.del_pos, da, db, x[j]);
-        a.new_off[u[j]] = (int64_t)(kept + lower_bound_dev(a.ins_row, ia, ib, u[j]));
+        a.new_off[u[j] - a.row_lo_new] = (int64_t)(kept + lower_bound_dev(a.ins_row, ia, ib, u[j]));
     }
 }
 
@@ -1301,11 +1400,11 @@ __global__ void k_remap_blocks(uint64_t V, const uint32_t* __restrict__ dropped,
 // scan (decoupled look-back) writes new_off[u] = old_off[u] + sum_{v<u} deg[v].
 __global__ void k_deg_scatter(const uint32_t* __restrict__ ins_row, uint64_t n_ins,
                               const uint32_t* __restrict__ del_row, uint64_t n_del, int32_t* __restrict__ deg,
-                              int64_t* __restrict__ tsum) {
+                              int64_t* __restrict__ tsum, uint64_t row_lo) {
     uint64_t i = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x;
     const bool ok = i < n_ins + n_del;
     const bool is_ins = i < n_ins;
-    const uint32_t r = ok ? (is_ins ? ins_row[i] : del_row[i - n_ins]) : 0;
+    const uint32_t r = ok ? (uint32_t)((is_ins ? ins_row[i] : del_row[i - n_ins]) - row_lo) : 0;
     // warp-aggregated: one atomic per (row, sign) group of the warp (hub rows get many records)
     const uint64_t key = ok ? (((uint64_t)r << 1) | (is_ins ? 1u : 0u)) : ~0ull;
     const uint32_t peers = __match_any_sync(0xffffffffu, key);
@@ -1430,10 +1529,11 @@ __global__ void k_offsets_inserted(const NodeVtx* __restrict__ nv, const uint32_
                                    uint64_t n_vins, RowArgs a) {
     uint64_t i = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x;
     if (i >= n_vins) return;
+    if (!a.own.owns(a.nv_ext[ins_q[i]])) return;  // another shard's row
     const NodeVtx& r = nv[ins_q[i]];
     const uint64_t x = (uint64_t)a.old_off[r.oldpos];
     const uint64_t kept = x - casc_before(a, x) - lower_bound_dev(a.del_pos, 0, a.n_del, x);
-    a.new_off[r.newid] = (int64_t)(kept + lower_bound_dev(a.ins_row, 0, a.n_ins, r.newid));
+    a.new_off[r.newid - a.row_lo_new] = (int64_t)(kept + lower_bound_dev(a.ins_row, 0, a.n_ins, r.newid));
 }
 
 // per 32 old ids: {new id of the group's first id (as if it survived) | exact << 31,
@@ -1452,6 +1552,10 @@ __global__ void k_remap32(uint64_t V, const uint32_t* __restrict__ dropped, uint
 }
 
 __global__ void k_set_i64(int64_t* p, int64_t v) { *p = v; }
+__global__ void k_row_range(const uint64_t* __restrict__ ext, uint64_t V, OwnRange own, Counters* c) {
+    c->row_lo_new = lower_bound_dev(ext, 0, V, own.lo);
+    c->row_hi_new = own.hi == ~0ull ? V : lower_bound_dev(ext, 0, V, own.hi);
+}
 __global__ void k_copy_u64(unsigned long long* dst, const uint64_t* src) { *dst = *src; }
 
 // ================================================================ checks ====

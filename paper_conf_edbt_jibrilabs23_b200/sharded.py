@@ -1,0 +1,129 @@
+"""Sharded (multi-GPU) apply: one process per GPU, 1D external-ID ranges.
+
+The exchange step a8 around the per-shard pipeline:
+
+1. every rank validates its slice of the global batch; the status is agreed with an
+   all-reduce before anything is applied (all ranks commit or none starts);
+2. global arrival numbers are rank-major (all-gather of the slice sizes, reading A5);
+3. the library packs the slice into 40-byte route records grouped by destination
+   (an edge op goes to the shard owning its source, a node op to every shard);
+4. counts, then records are exchanged with all-to-all over the process group
+   (NCCL over NVLink on GPUs; gloo in the CPU tests);
+5. the library applies what it received (h2tap_delta_apply_routed);
+6. shard bases (first global row, first global edge) come from an all-gather of the
+   shards' row and edge counts.
+
+The compute runs in the library's kernels (route packing included); this module is
+orchestration only.  The engine is anything with validate / pack / apply_routed /
+local_sizes (the CUDA replica here, an oracle-backed shard in the CPU tests).
+"""
+from __future__ import annotations
+
+from types import SimpleNamespace
+
+import numpy as np
+import torch
+import torch.distributed as dist
+
+from . import ROUTE_REC_BYTES, H2tapError, Replica
+
+
+class LibEngine:
+    """A shard of the CUDA replica (libh2tap.so)."""
+
+    def __init__(self, replica: Replica, device):
+        self.rep = replica
+        self.device = torch.device(device)
+        self.buf = torch.empty(0, dtype=torch.uint8, device=self.device)
+        self.launches = 0   # validate / pack kernels (apply_routed reports its own)
+        self.h2d = 0
+
+    def stage(self, batch):
+        """Device copy of a host batch slice (route packing reads device memory)."""
+        if getattr(batch.kind, "is_cuda", False):
+            return batch
+        cols = []
+        for a in (batch.kind, batch.src, batch.dst, batch.w, batch.ts):
+            t = a if isinstance(a, torch.Tensor) else torch.from_numpy(a.view(np.int64) if a.dtype == np.uint64 else a)
+            self.h2d += t.numel() * t.element_size()
+            cols.append(t.to(self.device, non_blocking=True))
+        return SimpleNamespace(kind=cols[0], src=cols[1], dst=cols[2], w=cols[3], ts=cols[4])
+
+    def validate(self, batch) -> int:
+        self.launches += 1 if len(batch.kind) else 0
+        return self.rep.validate(batch)
+
+    def pack(self, batch, seq0: int):
+        n = len(batch.kind)
+        cap = max(1024, int(n * 1.3) + 1024)
+        for _ in range(2):
+            if self.buf.numel() < cap * ROUTE_REC_BYTES:
+                self.buf = torch.empty(cap * ROUTE_REC_BYTES, dtype=torch.uint8, device=self.device)
+            rc, counts = self.rep.route_pack(batch, seq0, self.buf, cap)
+            self.launches += 1 + (len(counts) if rc == 0 and n else 0)
+            if rc == 0:
+                return self.buf[: sum(counts) * ROUTE_REC_BYTES], counts
+            if rc != -7:  # not E_CAPACITY
+                raise H2tapError(rc, "h2tap_route_pack", "")
+            cap = sum(counts)
+        raise H2tapError(-7, "h2tap_route_pack", "capacity")
+
+    def apply_routed(self, recs, n: int, snapshot_ts: int):
+        return self.rep.apply_routed(recs, n, snapshot_ts)
+
+    def local_sizes(self):
+        inf = self.rep.info()
+        return inf["n_vertices"], inf["n_edges"], inf["shard_vertex_base"]
+
+
+class ShardedReplica:
+    def __init__(self, engine, rank: int, world: int, device, group=None):
+        self.engine, self.rank, self.world, self.group = engine, rank, world, group
+        self.device = torch.device(device)
+        # gloo moves host tensors only: collectives on a CUDA engine then go through host
+        # copies (tests / several ranks sharing one GPU); NCCL works on device memory
+        self.coll = torch.device("cpu") if dist.get_backend(group) == "gloo" else self.device
+        self.next_seq = 0
+
+    def _i64(self, vals):
+        return torch.tensor(vals, dtype=torch.int64, device=self.coll)
+
+    def apply(self, batch, snapshot_ts: int):
+        """Apply this rank's slice of one global batch (every rank calls with the same
+        snapshot_ts; slices are taken rank-major from the global batch)."""
+        if hasattr(self.engine, "stage"):
+            batch = self.engine.stage(batch)
+        n = len(batch.kind)
+        # 1. agree on validity (status codes are <= 0; MIN finds any failure)
+        st = self._i64([self.engine.validate(batch)])
+        dist.all_reduce(st, op=dist.ReduceOp.MIN, group=self.group)
+        if int(st.item()) != 0:
+            raise H2tapError(int(st.item()), "sharded apply", "a rank rejected its batch slice")
+        # 2. rank-major global arrival numbers
+        sizes = [self._i64([0]) for _ in range(self.world)]
+        dist.all_gather(sizes, self._i64([n]), group=self.group)
+        sizes = [int(s.item()) for s in sizes]
+        seq0 = self.next_seq + sum(sizes[: self.rank])
+        # 3./4. pack by destination and exchange
+        recs, counts = self.engine.pack(batch, seq0)
+        send_c = self._i64(counts)
+        recv_c = torch.empty_like(send_c)
+        dist.all_to_all_single(recv_c, send_c, group=self.group)
+        rc = [int(x) for x in recv_c.tolist()]
+        recv = torch.empty(sum(rc) * ROUTE_REC_BYTES, dtype=torch.uint8, device=self.coll)
+        dist.all_to_all_single(recv, recs.to(self.coll), [c * ROUTE_REC_BYTES for c in rc],
+                               [c * ROUTE_REC_BYTES for c in counts], group=self.group)
+        recv = recv.to(recs.device)
+        # 5. apply the received ops
+        stats = self.engine.apply_routed(recv, sum(rc), snapshot_ts)
+        self.next_seq += sum(sizes)
+        stats["global_batch"] = sum(sizes)
+        return stats
+
+    def bases(self):
+        """(row base, edge base, rows, edges) of this shard in the global CSR."""
+        vr, e, row_lo = self.engine.local_sizes()
+        allc = [self._i64([0, 0]) for _ in range(self.world)]
+        dist.all_gather(allc, self._i64([vr, e]), group=self.group)
+        e_base = sum(int(c[1].item()) for c in allc[: self.rank])
+        return row_lo, e_base, vr, e

@@ -1,0 +1,175 @@
+"""Multi-process sharded apply over gloo (CPU; world_size 2 and 3).
+
+Exercises the exchange protocol of paper_conf_edbt_jibrilabs23_b200.sharded (status
+agreement, rank-major arrival numbers, routing of edge ops to the owner of their
+source and of node ops to every shard, variable all-to-all, shard bases) with an
+oracle-backed shard engine standing in for the GPU replica.  The shards' rows,
+gathered in shard order, must equal the unsharded oracle after every batch.
+"""
+import os
+import socket
+
+import numpy as np
+import pytest
+import torch
+import torch.distributed as dist
+import torch.multiprocessing as mp
+
+REC = np.dtype([("src", "<u8"), ("dst", "<u8"), ("ts", "<u8"), ("seq", "<u8"), ("w", "<f4"),
+                ("kind", "u1"), ("pad", "u1", 3)])
+assert REC.itemsize == 40
+
+
+class OracleShard:
+    """Test double for LibEngine: O1 over the global vertex set with this shard's rows."""
+
+    def __init__(self, n, ids, src, dst, w, bounds, rank):
+        from oracle import O1
+        self.bounds, self.rank, self.P = bounds, rank, len(bounds) - 1
+        self.snap = 0
+        mine = self.owner(src) == rank
+        self.o = O1.from_edges(n, ids, src[mine], dst[mine], w[mine])
+
+    def owner(self, x):
+        return np.searchsorted(self.bounds[1:self.P], np.asarray(x, np.uint64), side="right")
+
+    def validate(self, b):
+        if len(b.kind) and int(b.kind.max()) > 4:
+            return -1
+        if len(b.kind) and int(b.ts.min()) <= self.snap:
+            return -5
+        return 0
+
+    def pack(self, b, seq0):
+        n = len(b.kind)
+        own = np.where(b.kind <= 1, -1, self.owner(b.src))
+        parts, counts = [], []
+        for d in range(self.P):
+            sel = np.nonzero((own == -1) | (own == d))[0]
+            r = np.zeros(len(sel), REC)
+            r["src"], r["dst"], r["ts"] = b.src[sel], b.dst[sel], b.ts[sel]
+            r["seq"] = seq0 + sel.astype(np.uint64)
+            r["w"], r["kind"] = b.w[sel], b.kind[sel]
+            parts.append(r)
+            counts.append(len(sel))
+        buf = np.concatenate(parts) if n else np.zeros(0, REC)
+        return torch.from_numpy(buf.view(np.uint8).copy()), counts
+
+    def apply_routed(self, recs, n, snap):
+        from synth import Batch
+        r = recs.numpy().view(REC)
+        assert len(r) == n and (n < 2 or np.all(np.diff(r["seq"].astype(np.int64)) > 0))
+        b = Batch(r["kind"].copy(), r["src"].copy(), r["dst"].copy(), r["w"].copy(), r["ts"].copy())
+        rc, st = self.o.apply(b, snap)
+        assert rc == 0
+        self.snap = snap
+        return st
+
+    def own_rows(self):
+        off, cols, w, ids = self.o.export()
+        rows = np.nonzero(self.owner(ids) == self.rank)[0]
+        lo = int(rows[0]) if len(rows) else int(np.searchsorted(self.owner(ids), self.rank))
+        hi = lo + len(rows)
+        return off[lo:hi + 1] - off[lo], cols[off[lo]:off[hi]], w[off[lo]:off[hi]], ids[lo:hi], lo
+
+    def local_sizes(self):
+        off, cols, w, ids, lo = self.own_rows()
+        return len(ids), len(cols), lo
+
+
+def _worker(rank, world, port, out):
+    os.environ["MASTER_ADDR"], os.environ["MASTER_PORT"] = "127.0.0.1", str(port)
+    dist.init_process_group("gloo", rank=rank, world_size=world)
+    try:
+        import synth
+        from paper_conf_edbt_jibrilabs23_b200.sharded import ShardedReplica
+        from paper_conf_edbt_jibrilabs23_b200 import H2tapError, balanced_bounds
+
+        n = 400
+        ids = np.arange(n, dtype=np.uint64) * 5 + 2
+        rng = np.random.default_rng(3)
+        src, dst = ids[rng.integers(0, n, 3000)], ids[rng.integers(0, n, 3000)]
+        w = rng.random(3000).astype(np.float32)
+        bounds = balanced_bounds(src, world)
+        sh = ShardedReplica(OracleShard(n, ids, src, dst, w, bounds, rank), rank, world, "cpu")
+        results, ts = [], 0
+        for k in range(4):
+            g = synth.fuzz_batch(seed=11, k=k, n=1200, n_ids=5 * n + 9, probs=(0.05, 0.03, 0.5, 0.25, 0.17),
+                                 ts_lo=ts + 1, ts_span=300)
+            hit = np.arange(len(g)) % 2 == 0
+            g.src[hit], g.dst[hit] = ids[g.src[hit] % n], ids[g.dst[hit] % n]
+            sl = g.slice(slice(rank * len(g) // world, (rank + 1) * len(g) // world))  # rank-major slices
+            st = sh.apply(sl, ts + 250)
+            assert st["global_batch"] == len(g)
+            off, cols, ww, own_ids, lo = sh.engine.own_rows()
+            results.append((off, cols, ww, own_ids, sh.bases()))
+            ts += 300
+        # a stale op on one rank must make every rank refuse the batch
+        from synth import Batch
+        bad = Batch.of([(2, int(ids[0]), int(ids[1]), 1.0, 5 if rank == world - 1 else ts + 10)])
+        try:
+            sh.apply(bad, ts + 20)
+            refused = False
+        except H2tapError as e:
+            refused = e.status == -5
+        gathered = [None] * world
+        dist.all_gather_object(gathered, (results, refused))
+        if rank == 0:
+            out.put(gathered)
+    finally:
+        dist.destroy_process_group()
+
+
+def _free_port():
+    s = socket.socket()
+    s.bind(("127.0.0.1", 0))
+    p = s.getsockname()[1]
+    s.close()
+    return p
+
+
+@pytest.mark.parametrize("world", [2, 3])
+def test_sharded_exchange_over_gloo(world):
+    import synth
+    from oracle import O1
+    from paper_conf_edbt_jibrilabs23_b200 import balanced_bounds  # noqa: F401 (library loads on CPU)
+
+    ctx = mp.get_context("spawn")
+    q = ctx.Queue()
+    port = _free_port()
+    procs = [ctx.Process(target=_worker, args=(r, world, port, q)) for r in range(world)]
+    for p in procs:
+        p.start()
+    gathered = q.get(timeout=240)
+    for p in procs:
+        p.join(60)
+        assert p.exitcode == 0
+    # global reference
+    n = 400
+    ids = np.arange(n, dtype=np.uint64) * 5 + 2
+    rng = np.random.default_rng(3)
+    src, dst = ids[rng.integers(0, n, 3000)], ids[rng.integers(0, n, 3000)]
+    w = rng.random(3000).astype(np.float32)
+    o = O1.from_edges(n, ids, src, dst, w)
+    ts = 0
+    for k in range(4):
+        g = synth.fuzz_batch(seed=11, k=k, n=1200, n_ids=5 * n + 9, probs=(0.05, 0.03, 0.5, 0.25, 0.17),
+                             ts_lo=ts + 1, ts_span=300)
+        hit = np.arange(len(g)) % 2 == 0
+        g.src[hit], g.dst[hit] = ids[g.src[hit] % n], ids[g.dst[hit] % n]
+        rc, _ = o.apply(g, ts + 250)
+        assert rc == 0
+        off, cols, ww, gid = o.export()
+        parts = [gathered[r][0][k] for r in range(world)]
+        # shard bases are consistent with the concatenation
+        row_base = np.cumsum([0] + [len(p[3]) for p in parts])[:-1]
+        edge_base = np.cumsum([0] + [len(p[1]) for p in parts])[:-1]
+        assert [p[4][0] for p in parts] == list(row_base)
+        assert [p[4][1] for p in parts] == list(edge_base)
+        cat_off = np.concatenate([p[0][:-1] + eb for p, eb in zip(parts, edge_base)] + [np.array([len(cols)])])
+        assert np.array_equal(np.concatenate([p[3] for p in parts]), gid)
+        assert np.array_equal(cat_off, off)
+        assert np.array_equal(np.concatenate([p[1] for p in parts]), cols)
+        assert np.array_equal(np.concatenate([p[2] for p in parts]).view(np.uint32), ww.view(np.uint32))
+        ts += 300
+    assert all(gathered[r][1] for r in range(world))  # every rank refused the bad batch

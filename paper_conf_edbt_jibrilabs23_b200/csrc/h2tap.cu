@@ -424,11 +424,12 @@ h2tap_status apply_core(h2tap_replica* r, const BatchIn& in, uint64_t S, bool cr
             if (remap_on) {
                 // remap tables (64K-id block shifts, 32-id groups), then scatter the survivors
                 const uint64_t nblk = cdiv(V, 1ull << kRemapBlockShift), ng = cdiv(V, 32);
-                int32_t* rs = r->get<int32_t>(r->remap_shift, nblk);
+                int32_t* rs = r->get<int32_t>(r->remap_shift, nblk + 4);  // + {lo, hi, shift}
                 uint2* r32 = r->get<uint2>(r->remap32, ng);
-                if (nblk) { k_remap_blocks<<<g1(nblk), 256, 0, st>>>(V, dropped, n_dropped, ins_oldpos, n_vins, rs); CKL(); }
+                k_remap_blocks<<<g1(nblk), 256, 0, st>>>(V, dropped, n_dropped, ins_oldpos, n_vins, rs, rs + nblk);
+                CKL();
                 if (ng) { k_remap32<<<g1(ng), 256, 0, st>>>(V, dropped, n_dropped, ins_oldpos, n_vins, r32); CKL(); }
-                R.shift = rs; R.g32 = r32; R.ins_oldpos = ins_oldpos; R.n_vins = n_vins;
+                R.shift = rs; R.g32 = r32; R.ins_oldpos = ins_oldpos; R.n_vins = n_vins; R.lohi = rs + nblk;
                 TR("remap_tables");
                 if (V) { k_new_ext<<<g1(V), 256, 0, st>>>(old_ext, r->identity, V, R, new_ext); CKL(); }
                 TR("new_ext");
@@ -605,15 +606,12 @@ h2tap_status apply_core(h2tap_replica* r, const BatchIn& in, uint64_t S, bool cr
     const uint64_t Dtot = E + n_ins;
     if (Dtot) {
         MergeArgs ma{};
-        ma.old_cols = old_cols; ma.old_w = old_w; ma.old_off = old_off; ma.E_old = E; ma.V_old = Vr;
+        ma.old_cols = old_cols; ma.old_w = old_w; ma.E_old = E;
         ma.ins_pos = ins_pos; ma.ins_col = ins_col; ma.ins_w = ins_w; ma.n_ins = n_ins;
         ma.del_pos = del_pos; ma.n_del = n_del;
         ma.upd_pos = upd_pos; ma.upd_w = upd_w; ma.n_upd = n_upd;
-        ma.R = R; ma.hd_bits = hd_bits; ma.hd_rows = hd_rows; ma.n_hd = n_hd;
+        ma.R = R;
         ma.new_cols = new_cols; ma.new_w = new_w;
-        ma.rows = 0;  // row offsets: k_offsets_rows (a separate, row-balanced pass)
-        ma.new_off = new_off; ma.ins_row = ins_row;
-        ma.dropped = dropped; ma.n_dropped = n_dropped; ma.ins_oldpos = ins_oldpos; ma.n_vins = n_vins;
         ma.n_tiles = cdiv(Dtot, kMergeTile);
         ma.c = dc;
         if (casc) {

@@ -72,6 +72,7 @@ struct RemapView {
     const uint2* g32;
     const uint32_t* ins_oldpos;
     uint64_t n_vins;
+    const int32_t* lohi;   // {lo, hi, shift}: ids < lo unchanged, ids >= hi shifted by `shift`
 };
 __device__ __forceinline__ uint32_t remap_of(const RemapView& R, uint32_t k) {
     if (!R.shift) return k;
@@ -86,7 +87,12 @@ __device__ __forceinline__ uint32_t remap_of(const RemapView& R, uint32_t k) {
     return v;
 }
 
-__device__ __noinline__ uint32_t remap_of_slow(const RemapView& R, uint32_t k) { return remap_of(R, k); }
+// out-of-line exact path (fields by value: no stack copy of the view in the caller)
+__device__ __noinline__ uint32_t remap_of_slow(const int32_t* shift, const uint2* g32, const uint32_t* ins_oldpos,
+                                               uint64_t n_vins, uint32_t k) {
+    RemapView R{shift, g32, ins_oldpos, n_vins, nullptr};
+    return remap_of(R, k);
+}
 
 // ===================================================================== a1 ====
 // Validate + number + split: pending (ts > S) / visible node ops / visible edge
@@ -790,8 +796,7 @@ constexpr int kMergeBuf = kMergeTile + 8;     // staged old elements (+ 16 B ali
 struct MergeArgs {
     const uint32_t* old_cols;
     const float* old_w;
-    const int64_t* old_off;
-    uint64_t E_old, V_old;
+    uint64_t E_old;
     const uint64_t* ins_pos;
     const uint32_t* ins_col;
     const float* ins_w;
@@ -802,18 +807,8 @@ struct MergeArgs {
     const float* upd_w;
     uint64_t n_upd;
     RemapView R;
-    const uint32_t* hd_bits;
-    const uint32_t* hd_rows;
-    uint64_t n_hd;
     uint32_t* new_cols;
     float* new_w;
-    int64_t* new_off;            // ROWS mode (node ops): offsets of surviving old rows written by the merge
-    const uint32_t* ins_row;     // row of each inserted record (sorted)
-    const uint32_t* dropped;     // sorted old ids of dropped vertices
-    uint64_t n_dropped;
-    const uint32_t* ins_oldpos;  // sorted insertion ranks of inserted vertices
-    uint64_t n_vins;
-    int rows;                    // 1: merge writes new_off for old rows starting in each tile
     const uint32_t* casc_mask;  // CASC: 1 bit per old element (removed by a node delete)
     const uint64_t* casc_pre;   // CASC: cascaded elements before each 2048-element block
     uint64_t n_tiles;
@@ -824,9 +819,10 @@ struct MergeArgs {
 // merged items (smallest r with ins_pos[r] + r >= d), j = d - r old elements,
 // and the ranks of j in the sorted delete / update / cascade-row lists.
 struct TilePart {
-    uint64_t r, dl, ul, k, ir;  // k: first old row starting at or after j; ir: ins-row rank of k's new id
-    uint64_t cb;                // cascade mode: cascaded old elements before j
+    uint64_t r, dl, ul;
+    uint64_t cb;  // cascade mode: cascaded old elements before j
 };
+static_assert(sizeof(TilePart) == 32, "TilePart is prefetched as 16-byte chunks");
 
 __device__ __forceinline__ uint64_t ins_split(const uint64_t* ins_pos, uint64_t n_ins, uint64_t d) {
     uint64_t lo = 0, hi = n_ins;
@@ -847,23 +843,13 @@ __global__ void k_merge_partition(MergeArgs a, TilePart* __restrict__ part) {
     const uint64_t j = d - p.r;
     p.dl = lower_bound_dev(a.del_pos, 0, a.n_del, j);
     p.ul = lower_bound_dev(a.upd_pos, 0, a.n_upd, j);
-    p.k = p.ir = p.cb = 0;
+    p.cb = 0;
     if (a.casc_mask) {  // cascaded elements before j: block prefix + popcount of the partial block
         const uint64_t blk = j / kCascBlock;
         uint64_t c = a.casc_pre[blk];
         for (uint64_t q = blk * (kCascBlock / 32); q < (j >> 5); ++q) c += __popc(a.casc_mask[q]);
         if (j & 31) c += __popc(a.casc_mask[j >> 5] & (0xFFFFFFFFu >> (32 - (j & 31))));
         p.cb = c;
-    }
-    if (a.rows) {
-        p.k = lower_bound_dev(a.old_off, 0, a.V_old + 1, (int64_t)j);
-        if (p.k >= a.V_old) p.ir = a.n_ins;
-        else {
-            // new id of the first surviving old row >= k (compaction formula, reading A9)
-            const uint64_t u = p.k - lower_bound_dev(a.dropped, 0, a.n_dropped, (uint32_t)p.k) +
-                               upper_bound_dev(a.ins_oldpos, 0, a.n_vins, (uint32_t)p.k);
-            p.ir = lower_bound_dev(a.ins_row, 0, a.n_ins, (uint32_t)u);
-        }
     }
     part[t] = p;
 }
@@ -1109,8 +1095,6 @@ __global__ void __launch_bounds__(kThreads) k_scan_exclusive_u64(const uint64_t*
 
 constexpr int kMerge3Smem = 6 * kMergeBuf * 4;  // dynamic shared memory of k_merge3
 
-constexpr int kRowStage = 512;                 // rows mode: insert-row slice staged in smem
-constexpr int kRowPf = 4;                      // rows mode: old rows prefetched per thread
 
 // ---- TMA bulk store (smem -> global) helpers
 __device__ __forceinline__ void bulk_s2g(void* dst, const void* src, uint32_t bytes) {
@@ -1121,15 +1105,26 @@ __device__ __forceinline__ void bulk_commit() { asm volatile("cp.async.bulk.comm
 __device__ __forceinline__ void bulk_wait_read0() { asm volatile("cp.async.bulk.wait_group.read 0;" ::: "memory"); }
 __device__ __forceinline__ void bulk_wait_all() { asm volatile("cp.async.bulk.wait_group 0;" ::: "memory"); }
 
-// Merge v3.  Tile t covers merged items [t*2048, (t+1)*2048): old elements
+// ---- cp.async (16 B, generic proxy) for small prefetches into shared memory
+__device__ __forceinline__ void cp_async16(void* dst, const void* src) {
+    asm volatile("cp.async.cg.shared.global [%0], [%1], 16;" ::"r"(smem_u32(dst)), "l"(src) : "memory");
+}
+__device__ __forceinline__ void cp_async_commit() { asm volatile("cp.async.commit_group;" ::: "memory"); }
+__device__ __forceinline__ void cp_async_wait_all() { asm volatile("cp.async.wait_group 0;" ::: "memory"); }
+
+// Merge (a6).  Tile t covers merged items [t*2048, (t+1)*2048): old elements
 // [j0, j1) (TMA-staged, double-buffered) and inserted records [r0, r1).
-//   phase A (per 32-element chunk): keep-ballot (not deleted, not cascaded)
-//   scan of the 64 chunk counts -> kept-before at any element (smem masks)
-//   phase B: output index e = kept_before(i) + I(i), I(i) = inserted records at
-//            local positions <= i (uniform per chunk unless one falls inside);
+//   phase A (warp 0, per 32-element chunk): keep mask (not deleted, not cascaded),
+//            scans of kept counts and of inserted-record counts -> s_chunk
+//   phase B: old element i goes to e = kept_before(i) + I(i), I(i) = inserted records
+//            at local positions <= i (uniform per chunk unless one falls inside);
 //            values (remapped column, weight) staged in smem at e + (base & 3)
 //   inserted records: e = kept_before(p) + s
 //   store: scalar head/tail, one TMA bulk store per array for the aligned body
+// Software pipeline: while tile t is processed, the TMA loads of tile t+G are in
+// flight, tile t+2G's partition entries stream in by cp.async, and the heads of
+// tile t+G's edit lists are loaded into registers; three barriers per tile
+// (deleted/insert-count masks are double-buffered).
 template <bool CASC, bool REMAP>
 __global__ void __launch_bounds__(kThreads) k_merge3(MergeArgs a, const TilePart* __restrict__ part) {
     constexpr int NCH = kMergeTile / 32;  // 64 chunks of 32 old elements
@@ -1139,82 +1134,74 @@ __global__ void __launch_bounds__(kThreads) k_merge3(MergeArgs a, const TilePart
     uint32_t* s_oc = reinterpret_cast<uint32_t*>(dsm + 4 * kMergeBuf * 4);
     float* s_ow = reinterpret_cast<float*>(dsm + 5 * kMergeBuf * 4);
     __shared__ uint16_t s_ins[kMergeTile + 1];
-    __shared__ uint32_t s_dmask[NCH + 2];   // deleted old elements, per chunk
-    __shared__ uint32_t s_icnt[NCH + 2];    // inserted records per chunk of insertion positions
-    __shared__ uint32_t s_mask[NCH + 1];    // kept old elements, per chunk
-    __shared__ uint32_t s_cbase[NCH + 1];   // kept before each chunk
-    __shared__ uint32_t s_ibase[NCH + 2];   // inserted records at positions before each chunk
+    __shared__ uint32_t s_dmask[2][NCH + 2];  // deleted old elements per chunk (by buffer)
+    __shared__ uint32_t s_icnt[2][NCH + 2];   // inserted records per chunk of insertion positions
+    __shared__ uint4 s_chunk[NCH + 1];        // {keep mask, kept before, inserted before, inserted inside}
     __shared__ __align__(8) uint64_t s_bar[2];
-    __shared__ uint64_t s_meta[2][5];
-    __shared__ uint64_t s_rows[2][4];
-    __shared__ uint64_t s_cb[2];
-    __shared__ uint32_t s_irow[kRowStage];  // rows mode: the tile's slice of insert rows
-    __shared__ uint64_t s_cbefore;
+    __shared__ uint64_t s_meta[2][6];         // r0, r1, dl0, ul0, nd | nu << 16, cascaded before j0
+    __shared__ __align__(16) TilePart s_tp[2][2];
 
     const int tid = threadIdx.x, wid = tid >> 5;
     const uint32_t lane = lane_id(), lt = lanemask_lt();
     const uint64_t Dtot = a.E_old + a.n_ins;
-    if (tid == 0) { mbar_init(&s_bar[0], 1); mbar_init(&s_bar[1], 1); fence_mbar_init(); }
-    __syncthreads();
-    auto issue = [&](uint64_t t, int b) {  // one thread: tile metadata + TMA of its old elements
-        const TilePart p0 = part[t], p1 = part[t + 1];
-        s_meta[b][0] = p0.r; s_meta[b][1] = p1.r; s_meta[b][2] = p0.dl; s_meta[b][3] = p0.ul;
-        s_meta[b][4] = (p1.dl - p0.dl) | ((p1.ul - p0.ul) << 16);
-        s_rows[b][0] = p0.k; s_rows[b][1] = p1.k; s_rows[b][2] = p0.ir; s_rows[b][3] = p1.ir;
-        s_cb[b] = p0.cb;
-        const uint64_t j0 = min(t * kMergeTile, Dtot) - p0.r, j1 = min((t + 1) * kMergeTile, Dtot) - p1.r;
+    const uint64_t G = gridDim.x;
+    auto issue = [&](uint64_t tt, int bb, const TilePart& p0, const TilePart& p1) {  // thread 0
+        s_meta[bb][0] = p0.r; s_meta[bb][1] = p1.r; s_meta[bb][2] = p0.dl; s_meta[bb][3] = p0.ul;
+        s_meta[bb][4] = (p1.dl - p0.dl) | ((p1.ul - p0.ul) << 16);
+        s_meta[bb][5] = p0.cb;
+        const uint64_t j0 = min(tt * kMergeTile, Dtot) - p0.r, j1 = min((tt + 1) * kMergeTile, Dtot) - p1.r;
         const uint64_t a0 = j0 & ~3ull, a1 = (j1 + 3) & ~3ull;
         const uint32_t bytes = (uint32_t)((a1 - a0) * 4);
-        mbar_expect_tx(&s_bar[b], 2 * bytes);
+        mbar_expect_tx(&s_bar[bb], 2 * bytes);
         if (bytes) {
-            bulk_g2s(&s_col[b][0], a.old_cols + a0, bytes, &s_bar[b]);
-            bulk_g2s(&s_w[b][0], a.old_w + a0, bytes, &s_bar[b]);
+            bulk_g2s(&s_col[bb][0], a.old_cols + a0, bytes, &s_bar[bb]);
+            bulk_g2s(&s_w[bb][0], a.old_w + a0, bytes, &s_bar[bb]);
         }
     };
-    uint64_t t = blockIdx.x;
-    if (t < a.n_tiles && tid == 0) issue(t, 0);
-    __syncthreads();
-    for (uint32_t it = 0; t < a.n_tiles; t += gridDim.x, ++it) {
-        const int b = it & 1;
-        const uint64_t r0 = s_meta[b][0], r1 = s_meta[b][1], dl0 = s_meta[b][2], ul0 = s_meta[b][3];
-        const uint64_t rk0 = s_rows[b][0], rk1 = s_rows[b][1], ir0 = s_rows[b][2], ir1 = s_rows[b][3];
-        const uint32_t nd = (uint32_t)(s_meta[b][4] & 0xFFFF), nu = (uint32_t)((s_meta[b][4] >> 16) & 0xFFFF);
-        const uint64_t d0 = min(t * kMergeTile, Dtot), d1 = min((t + 1) * kMergeTile, Dtot);
-        const uint64_t j0 = d0 - r0, j1 = d1 - r1;
-        const uint32_t n_old = (uint32_t)(j1 - j0), ni = (uint32_t)(r1 - r0);
-        const uint32_t sh = (uint32_t)(j0 & 3);
-        if (tid == 0 && t + gridDim.x < a.n_tiles) { fence_proxy_async(); issue(t + gridDim.x, b ^ 1); }
-        // the tile's edit lists: first kThreads entries of each list straight into registers,
-        // all loads in flight together (overflow entries are loaded in the loops below)
-        const uint64_t pf_del = tid < nd ? a.del_pos[dl0 + tid] : 0;
-        const uint64_t pf_ins = tid < ni ? a.ins_pos[r0 + tid] : 0;
-        const uint32_t pf_icol = tid < ni ? a.ins_col[r0 + tid] : 0;
-        const float pf_iw = tid < ni ? a.ins_w[r0 + tid] : 0.f;
-        const uint64_t pf_upd = tid < nu ? a.upd_pos[ul0 + tid] : 0;
-        const float pf_uw = tid < nu ? a.upd_w[ul0 + tid] : 0.f;
-        // rows mode: the tile's old rows (first 2*kThreads) and its slice of insert rows
-        const bool last_tile = (t == a.n_tiles - 1);
-        const uint64_t rk_end = last_tile ? a.V_old : rk1;
-        const uint64_t ir_end = last_tile ? a.n_ins : ir1;
-        const uint32_t n_rows = a.rows ? (uint32_t)min(rk_end - rk0, (uint64_t)0xFFFFFFFF) : 0u;
-        const uint32_t n_irs = a.rows ? (uint32_t)(ir_end - ir0) : 0u;
-        int64_t pf_x[kRowPf];
-        uint32_t pf_u[kRowPf];
+    auto prefetch_part = [&](uint64_t tt, int slot) {  // thread 0: part[tt], part[tt + 1] -> s_tp[slot]
+        const uint4* src = reinterpret_cast<const uint4*>(part + tt);
+        uint4* dst = reinterpret_cast<uint4*>(&s_tp[slot][0]);
 #pragma unroll
-        for (int h = 0; h < kRowPf; ++h) {
-            const uint32_t q = tid + h * kThreads;
-            pf_x[h] = q < n_rows ? a.old_off[rk0 + q] : 0;
-            pf_u[h] = q < n_rows ? (REMAP ? remap_of(a.R, (uint32_t)(rk0 + q)) : (uint32_t)(rk0 + q)) : kNone32;
-        }
-        for (uint32_t q = tid; q < n_irs && q < kRowStage; q += kThreads) s_irow[q] = a.ins_row[ir0 + q];
-        if (tid < NCH + 2) { s_dmask[tid] = 0; s_icnt[tid] = 0; }
-        const uint64_t cbefore = CASC ? s_cb[b] : 0;  // cascaded old elements before j0
-        // phase A inputs of warp 0: the cascade-mask words under its two chunks
-        uint32_t pf_cm[4] = {0u, 0u, 0u, 0u};
-        if (CASC && wid == 0) {
+        for (int q = 0; q < 2 * (int)sizeof(TilePart) / 16; ++q) cp_async16(dst + q, src + q);
+        cp_async_commit();
+    };
+    // remap fast paths: ids below lohi[0] keep their id, ids at or above lohi[1] shift by lohi[2]
+    uint32_t rlo = 0, rhi = 0;
+    int32_t rsh = 0;
+    if (REMAP) { rlo = (uint32_t)a.R.lohi[0]; rhi = (uint32_t)a.R.lohi[1]; rsh = a.R.lohi[2]; }
+
+    uint64_t t = blockIdx.x;
+    if (tid == 0) {
+        mbar_init(&s_bar[0], 1); mbar_init(&s_bar[1], 1); fence_mbar_init();
+        if (t < a.n_tiles) issue(t, 0, part[t], part[t + 1]);
+        if (t + G < a.n_tiles) prefetch_part(t + G, 1);
+    }
+    if (tid < NCH + 2) { s_dmask[0][tid] = 0; s_icnt[0][tid] = 0; s_dmask[1][tid] = 0; s_icnt[1][tid] = 0; }
+    __syncthreads();
+    // heads of the edit lists of the tile in buffer bb (lists longer than kThreads are
+    // read directly in the loops below)
+    uint64_t pf_del = 0, pf_ins = 0, pf_upd = 0;
+    uint32_t pf_icol = 0;
+    float pf_iw = 0.f, pf_uw = 0.f;
+    uint32_t pf_cm[4] = {0u, 0u, 0u, 0u};
+    auto load_pos = [&](int bb) {
+        const uint64_t r0 = s_meta[bb][0], r1 = s_meta[bb][1], dl0 = s_meta[bb][2];
+        const uint32_t nd = (uint32_t)(s_meta[bb][4] & 0xFFFF);
+        pf_del = tid < nd ? a.del_pos[dl0 + tid] : 0;
+        pf_ins = tid < (uint32_t)(r1 - r0) ? a.ins_pos[r0 + tid] : 0;
+    };
+    auto load_upd = [&](int bb, uint64_t tt) {
+        const uint64_t ul0 = s_meta[bb][3];
+        const uint32_t nu = (uint32_t)((s_meta[bb][4] >> 16) & 0xFFFF);
+        pf_upd = tid < nu ? a.upd_pos[ul0 + tid] : 0;
+        pf_uw = tid < nu ? a.upd_w[ul0 + tid] : 0.f;
+        if (CASC && wid == 0) {  // cascade-mask words under warp 0's two chunks
+            const uint64_t j0 = min(tt * kMergeTile, Dtot) - s_meta[bb][0];
+            const uint64_t n_old = min((tt + 1) * kMergeTile, Dtot) - s_meta[bb][1] - j0;
 #pragma unroll
             for (int h = 0; h < 2; ++h) {
                 const uint32_t i0 = (2 * lane + h) * 32;
+                pf_cm[2 * h] = pf_cm[2 * h + 1] = 0u;
                 if (i0 < n_old) {
                     const uint64_t x = j0 + i0, q = x >> 5;
                     pf_cm[2 * h] = a.casc_mask[q];
@@ -1222,40 +1209,64 @@ __global__ void __launch_bounds__(kThreads) k_merge3(MergeArgs a, const TilePart
                 }
             }
         }
-        __syncthreads();
+    };
+    auto load_ins = [&](int bb) {
+        const uint64_t r0 = s_meta[bb][0], r1 = s_meta[bb][1];
+        pf_icol = tid < (uint32_t)(r1 - r0) ? a.ins_col[r0 + tid] : 0u;
+        pf_iw = tid < (uint32_t)(r1 - r0) ? a.ins_w[r0 + tid] : 0.f;
+    };
+    if (t < a.n_tiles) { load_pos(0); load_upd(0, t); load_ins(0); }
+
+    for (uint32_t it = 0; t < a.n_tiles; t += G, ++it) {
+        const int b = it & 1;
+        const uint64_t r0 = s_meta[b][0], r1 = s_meta[b][1], dl0 = s_meta[b][2], ul0 = s_meta[b][3];
+        const uint32_t nd = (uint32_t)(s_meta[b][4] & 0xFFFF), nu = (uint32_t)((s_meta[b][4] >> 16) & 0xFFFF);
+        const uint64_t cbefore = CASC ? s_meta[b][5] : 0;  // cascaded old elements before j0
+        const uint64_t d0 = min(t * kMergeTile, Dtot), d1 = min((t + 1) * kMergeTile, Dtot);
+        const uint64_t j0 = d0 - r0, j1 = d1 - r1;
+        const uint32_t n_old = (uint32_t)(j1 - j0), ni = (uint32_t)(r1 - r0);
+        const uint32_t sh = (uint32_t)(j0 & 3);
+        const bool has_next = t + G < a.n_tiles;
+        if (tid == 0 && has_next) {
+            cp_async_wait_all();
+            const int slot = (it + 1) & 1;
+            const TilePart p0 = s_tp[slot][0], p1 = s_tp[slot][1];
+            fence_proxy_async();
+            issue(t + G, b ^ 1, p0, p1);
+            if (t + 2 * G < a.n_tiles) prefetch_part(t + 2 * G, it & 1);
+        }
+        uint32_t* dmask = s_dmask[b];
+        uint32_t* icnt = s_icnt[b];
         for (uint32_t i = tid; i < nd; i += kThreads) {
             const uint32_t p = (uint32_t)((i == (uint32_t)tid ? pf_del : a.del_pos[dl0 + i]) - j0);
-            atomicOr(&s_dmask[p >> 5], 1u << (p & 31));
+            atomicOr(&dmask[p >> 5], 1u << (p & 31));
         }
         for (uint32_t s = tid; s < ni; s += kThreads) {
             const uint32_t p = (uint32_t)((s == (uint32_t)tid ? pf_ins : a.ins_pos[r0 + s]) - j0);
             s_ins[s] = (uint16_t)p;
-            atomicAdd(&s_icnt[p >> 5], 1u);
+            atomicAdd(&icnt[p >> 5], 1u);
         }
-        __syncthreads();
+        __syncthreads();  // B1: masks complete; s_meta[b ^ 1] (next tile) visible
+        if (has_next) load_pos(b ^ 1);
         if (wid == 0) {
             // keep masks of the 64 chunks (2 per lane): valid & not deleted & not cascaded,
             // then exclusive scans of kept counts and of inserted-record counts
-            uint32_t m[2];
+            uint32_t m[2], k[2];
 #pragma unroll
             for (int h = 0; h < 2; ++h) {
                 const uint32_t c = 2 * lane + h, i0 = c * 32;
                 uint32_t v = (i0 >= n_old) ? 0u : (n_old - i0 >= 32 ? 0xFFFFFFFFu : (0xFFFFFFFFu >> (32 - (n_old - i0))));
-                v &= ~s_dmask[c];
+                v &= ~dmask[c];
                 if (CASC && v) v &= ~__funnelshift_r(pf_cm[2 * h], pf_cm[2 * h + 1], (uint32_t)((j0 + i0) & 31));
                 m[h] = v;
-                s_mask[c] = v;
+                k[h] = icnt[c];
             }
             const uint32_t c0 = __popc(m[0]), c1 = __popc(m[1]);
             const uint32_t inc = warp_inclusive_scan(c0 + c1);
-            s_cbase[2 * lane] = inc - c0 - c1;
-            s_cbase[2 * lane + 1] = inc - c1;
-            if (lane == 31) s_cbase[NCH] = inc;
-            const uint32_t k0 = s_icnt[2 * lane], k1 = s_icnt[2 * lane + 1];
-            const uint32_t ik = warp_inclusive_scan(k0 + k1);
-            s_ibase[2 * lane] = ik - k0 - k1;
-            s_ibase[2 * lane + 1] = ik - k1;
-            if (lane == 31) { s_ibase[NCH] = ik; s_ibase[NCH + 1] = ik + s_icnt[NCH]; }
+            const uint32_t ik = warp_inclusive_scan(k[0] + k[1]);
+            s_chunk[2 * lane] = make_uint4(m[0], inc - c0 - c1, ik - k[0] - k[1], k[0]);
+            s_chunk[2 * lane + 1] = make_uint4(m[1], inc - c1, ik - k[1], k[1]);
+            if (lane == 31) s_chunk[NCH] = make_uint4(0u, inc, ik, 0u);
         }
         mbar_wait(&s_bar[b], (it >> 1) & 1);
         for (uint32_t i = tid; i < nu; i += kThreads) {
@@ -1263,14 +1274,14 @@ __global__ void __launch_bounds__(kThreads) k_merge3(MergeArgs a, const TilePart
             s_w[b][(pf ? pf_upd : a.upd_pos[ul0 + i]) - (j0 & ~3ull)] = pf ? pf_uw : a.upd_w[ul0 + i];
         }
         if (tid == 0) bulk_wait_read0();  // previous tile's bulk store has finished reading s_oc/s_ow
-        __syncthreads();
-        const uint32_t kept = s_cbase[NCH];
+        __syncthreads();  // B2: chunk table, updated weights, staging buffers free
+        if (has_next) load_upd(b ^ 1, t + G);
+        const uint32_t kept = s_chunk[NCH].y;
         const uint32_t n_out = kept + ni;
         const uint64_t base = j0 - dl0 - cbefore + r0;
         const uint32_t ob = (uint32_t)(base & 3);
-        // phase B: old elements, output index = kept before + inserted at positions <= i.
-        // Warp w owns chunks w, w+8, ..., w+56; the 8 chunks are unrolled so that the
-        // remap-table lookups of all of them are in flight together.
+        // phase B: warp w owns chunks w, w+8, ..., w+56, unrolled so that the remap-table
+        // lookups of all of them are in flight together
         {
             constexpr int KCH = NCH / (kThreads / 32);  // 8 chunks per warp
             uint32_t colv[KCH];
@@ -1279,10 +1290,11 @@ __global__ void __launch_bounds__(kThreads) k_merge3(MergeArgs a, const TilePart
                 const uint32_t c = wid + k * (kThreads / 32), i = c * 32 + lane;
                 colv[k] = (i < n_old) ? s_col[b][i + sh] : 0u;
             }
-            if (REMAP) {  // lookups of all 8 chunks in flight together (tables stay in L1/L2)
+            if (REMAP) {
                 int32_t shf[KCH];
 #pragma unroll
-                for (int k = 0; k < KCH; ++k) shf[k] = a.R.shift[colv[k] >> kRemapBlockShift];
+                for (int k = 0; k < KCH; ++k)
+                    shf[k] = colv[k] < rlo ? 0 : (colv[k] >= rhi ? rsh : a.R.shift[colv[k] >> kRemapBlockShift]);
                 uint2 g[KCH];
 #pragma unroll
                 for (int k = 0; k < KCH; ++k) g[k] = (shf[k] == kRemapMixed) ? a.R.g32[colv[k] >> 5] : make_uint2(0u, 0u);
@@ -1290,7 +1302,7 @@ __global__ void __launch_bounds__(kThreads) k_merge3(MergeArgs a, const TilePart
                 for (int k = 0; k < KCH; ++k) {
                     const uint32_t col = colv[k], r = col & 31;
                     if (shf[k] != kRemapMixed) colv[k] = (uint32_t)((int64_t)col + shf[k]);
-                    else if (g[k].x >> 31) colv[k] = remap_of_slow(a.R, col);  // rare: out of line
+                    else if (g[k].x >> 31) colv[k] = remap_of_slow(a.R.shift, a.R.g32, a.R.ins_oldpos, a.R.n_vins, col);
                     else colv[k] = g[k].x + r - (r ? __popc(g[k].y & (0xFFFFFFFFu >> (32 - r))) : 0u);
                 }
             }
@@ -1298,57 +1310,28 @@ __global__ void __launch_bounds__(kThreads) k_merge3(MergeArgs a, const TilePart
             for (int k = 0; k < KCH; ++k) {
                 const uint32_t c = wid + k * (kThreads / 32), i = c * 32 + lane;
                 if (c * 32 >= n_old) break;
-                const uint32_t m = s_mask[c];
-                uint32_t I = s_ibase[c];
-                if (s_icnt[c]) {  // inserted records inside this chunk: count those at positions <= i
-                    const uint32_t lo = s_ibase[c], hi = lo + s_icnt[c];
-                    I = (uint32_t)upper_bound_dev(s_ins, lo, hi, (uint16_t)i);
-                }
-                if (m >> lane & 1) {
-                    const uint32_t e = s_cbase[c] + __popc(m & lt) + I + ob;
+                const uint4 ch = s_chunk[c];
+                uint32_t I = ch.z;
+                if (ch.w) I = (uint32_t)upper_bound_dev(s_ins, ch.z, ch.z + ch.w, (uint16_t)i);  // inserts inside
+                if (ch.x >> lane & 1) {
+                    const uint32_t e = ch.y + __popc(ch.x & lt) + I + ob;
                     s_oc[e] = colv[k];
                     s_ow[e] = s_w[b][i + sh];
                 }
             }
         }
         // inserted records: local position p precedes old element p
-        auto kept_before = [&](uint32_t i) -> uint32_t {  // i in [0, n_old]
-            const uint32_t c = i >> 5, r = i & 31;
-            return s_cbase[c] + (r ? __popc(s_mask[c] & (0xFFFFFFFFu >> (32 - r))) : 0u);
-        };
         for (uint32_t s = tid; s < ni; s += kThreads) {
-            const uint32_t e = kept_before(s_ins[s]) + s + ob;
+            const uint32_t p = s_ins[s], c = p >> 5, r = p & 31;
+            const uint4 ch = s_chunk[c];
+            const uint32_t e = ch.y + (r ? __popc(ch.x & (0xFFFFFFFFu >> (32 - r))) : 0u) + s + ob;
             const bool pf = s == (uint32_t)tid;
             s_oc[e] = pf ? pf_icol : a.ins_col[r0 + s];
             s_ow[e] = pf ? pf_iw : a.ins_w[r0 + s];
         }
-        if (a.rows) {
-            // a4/a5 fused: new_off[u'] of every surviving old row k starting in this tile
-            //   = (kept old elements before its old start) + (inserted records in rows < u')
-            const uint64_t kb0 = j0 - dl0 - cbefore;  // kept old elements before j0
-            const bool staged = n_irs <= kRowStage;
-#pragma unroll
-            for (int h = 0; h < kRowPf; ++h) {  // prefetched rows
-                const uint32_t q = tid + h * kThreads;
-                const uint32_t u = pf_u[h];
-                if (q >= n_rows || u == kNone32) continue;
-                const int64_t x = pf_x[h];
-                const uint64_t kept_b = kb0 + kept_before((uint32_t)((uint64_t)x - j0));
-                const uint64_t irk = staged ? ir0 + lower_bound_dev(s_irow, 0, n_irs, u)
-                                            : lower_bound_dev(a.ins_row, ir0, ir_end, u);
-                a.new_off[u] = (int64_t)(kept_b + irk);
-            }
-            for (uint32_t q = tid + kRowPf * kThreads; q < n_rows; q += kThreads) {  // rare overflow
-                const uint32_t u = REMAP ? remap_of(a.R, (uint32_t)(rk0 + q)) : (uint32_t)(rk0 + q);
-                if (u == kNone32) continue;
-                const int64_t x = a.old_off[rk0 + q];
-                const uint64_t kept_b = kb0 + kept_before((uint32_t)((uint64_t)x - j0));
-                const uint64_t irk = staged ? ir0 + lower_bound_dev(s_irow, 0, n_irs, u)
-                                            : lower_bound_dev(a.ins_row, ir0, ir_end, u);
-                a.new_off[u] = (int64_t)(kept_b + irk);
-            }
-        }
-        __syncthreads();
+        __syncthreads();  // B3: staged output complete; this tile's inputs no longer read
+        if (has_next) load_ins(b ^ 1);
+        if (tid < NCH + 2) { dmask[tid] = 0; icnt[tid] = 0; }  // for tile t + 2G (same buffer)
         // store the contiguous output chunk [base, base + n_out)
         {
             uint32_t head = (4 - ob) & 3;
@@ -1368,17 +1351,28 @@ __global__ void __launch_bounds__(kThreads) k_merge3(MergeArgs a, const TilePart
                 bulk_commit();
             }
         }
-        __syncthreads();
     }
     if (tid == 0) bulk_wait_all();
 }
 
 // per 64K-id block of old ids: constant new-id shift, or kRemapMixed if a dropped
 // id or an inserted id's insertion point lies strictly inside the block
+// Thread 0 also writes lohi = {lo, hi, shift}: below lo = min(first dropped id, first
+// insertion point) nothing moves; from hi = max(last dropped id + 1, last insertion
+// point) on, every id is shifted by n_ins - n_dropped.
 __global__ void k_remap_blocks(uint64_t V, const uint32_t* __restrict__ dropped, uint64_t n_dropped,
-                               const uint32_t* __restrict__ ins_oldpos, uint64_t n_ins, int32_t* __restrict__ shift) {
+                               const uint32_t* __restrict__ ins_oldpos, uint64_t n_ins, int32_t* __restrict__ shift,
+                               int32_t* __restrict__ lohi) {
     uint64_t bk = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x;
     uint64_t nb = (V + (1u << kRemapBlockShift) - 1) >> kRemapBlockShift;
+    if (bk == 0) {
+        const uint64_t lo = min(n_dropped ? (uint64_t)dropped[0] : V, n_ins ? (uint64_t)ins_oldpos[0] : V);
+        const uint64_t hi = max(n_dropped ? (uint64_t)dropped[n_dropped - 1] + 1 : 0ull,
+                                n_ins ? (uint64_t)ins_oldpos[n_ins - 1] : 0ull);
+        lohi[0] = (int32_t)lo;
+        lohi[1] = (int32_t)max(hi, lo);
+        lohi[2] = (int32_t)((int64_t)n_ins - (int64_t)n_dropped);
+    }
     if (bk >= nb) return;
     uint64_t lo = bk << kRemapBlockShift, hi = min(lo + (1u << kRemapBlockShift), V);
     uint64_t d0 = lower_bound_dev(dropped, 0, n_dropped, (uint32_t)lo);

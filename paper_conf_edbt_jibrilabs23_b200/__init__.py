@@ -11,8 +11,10 @@ CUDA tensors (device memory of the replica's device).
 """
 from __future__ import annotations
 
+import atexit
 import ctypes
 import os
+import weakref
 
 import numpy as np
 
@@ -156,12 +158,24 @@ def _torch_allocator(device: int):
     return _ALLOC(_alloc), _FREE(_free)
 
 
+# replicas still open at interpreter exit are destroyed before torch's module
+# teardown (their memory goes back through torch's caching allocator)
+_LIVE = weakref.WeakSet()
+
+
+@atexit.register
+def _close_live():
+    for r in list(_LIVE):
+        r.close()
+
+
 class Replica:
     """A CSR replica in device memory (opaque h2tap_replica*)."""
 
     def __init__(self, handle, keep):
         self._h = handle
         self._keep = keep
+        _LIVE.add(self)
 
     # ---------------------------------------------------------------- create
     @staticmethod

@@ -184,7 +184,9 @@ namespace {
 
 // ---------------------------------------------------------------- sort ----
 // Stable LSD sort of (keys, vals)[0, n) on the low `bits` bits; result in (k, v).
-void radix_sort(h2tap_replica* r, uint64_t*& k, uint32_t*& v, uint64_t*& k2, uint32_t*& v2, uint64_t n, int bits) {
+// n_dev (nullable): the actual count is in device memory and n is an upper bound.
+void radix_sort(h2tap_replica* r, uint64_t*& k, uint32_t*& v, uint64_t*& k2, uint32_t*& v2, uint64_t n, int bits,
+                const unsigned long long* n_dev = nullptr) {
     if (n <= 1 || bits <= 0) return;
     const int passes = (bits + 7) / 8;
     const uint64_t ntiles = cdiv(n, kRsTile);
@@ -196,12 +198,12 @@ void radix_sort(h2tap_replica* r, uint64_t*& k, uint32_t*& v, uint64_t*& k2, uin
     CK(cudaMemsetAsync(st, 0, (size_t)passes * ntiles * 256 * sizeof(uint64_t), r->st));
     CK(cudaMemsetAsync(ctr, 0, kRsMaxPasses * sizeof(uint32_t), r->st));
     int grid = (int)std::min<uint64_t>(cdiv(n, 256 * 8), 148 * 8);
-    rs_histogram<<<grid, 256, 0, r->st>>>(k, n, passes, hist);
+    rs_histogram<<<grid, 256, 0, r->st>>>(k, n, n_dev, passes, hist);
     CKL();
     rs_digit_base<<<passes, 256, 0, r->st>>>(hist, dbase);
     CKL();
     for (int p = 0; p < passes; ++p) {
-        rs_onesweep<<<(unsigned)ntiles, kRsThreads, 0, r->st>>>(k, v, k2, v2, n, 8 * p, dbase + p * 256,
+        rs_onesweep<<<(unsigned)ntiles, kRsThreads, 0, r->st>>>(k, v, k2, v2, n, n_dev, 8 * p, dbase + p * 256,
                                                               st + (uint64_t)p * ntiles * 256, ctr + p);
         CKL();
         std::swap(k, k2);
@@ -347,11 +349,17 @@ h2tap_status apply_core(h2tap_replica* r, const BatchIn& in, uint64_t S, bool cr
 
     // ---- a2: node ops -> per-vertex timeline, ID-map compaction, remap
     const uint64_t V = r->V, E = r->E, row_lo = r->row_lo, Vr = r->Vr;
-    uint64_t row_lo_new = row_lo, Vr_new = Vr;
     const int ec = r->ext_cur;
     const uint64_t* old_ext = static_cast<const uint64_t*>(r->ext[ec].p);
-    uint64_t U = 0, n_dropped = 0, n_vins = 0, n_hd = 0, Vn = V;
-    bool remap_on = false, set_changed = false;
+    // Only the sizes known after a1 (node ops, edge ops, pending) are host values from
+    // here on; every later size (unique vertices, dropped/inserted vertices, surviving
+    // edge ops, outcome lists, the new V and E) stays in device memory (Counters) and
+    // the kernels read it there.  Buffers and grids are sized by upper bounds, so the
+    // rest of the cycle runs without a host round trip until the final read-back.
+    const bool node_mode = n_node > 0;
+    const uint64_t Vn_ub = V + n_node;  // new vertices <= old + inserted
+    if (Vn_ub >= 0x7FFFFFFFull) { set_err("vertex count could exceed 2^31-1"); return H2TAP_E_CAPACITY; }
+    const uint64_t Vr_new_ub = node_mode ? Vn_ub : Vr;  // rows of the new CSR (shard rows <= all)
     NodeVtx* nv = nullptr;
     uint64_t* nv_ext = nullptr;
     RemapView R{};  // identity unless node ops shift the dense ids
@@ -363,7 +371,7 @@ h2tap_status apply_core(h2tap_replica* r, const BatchIn& in, uint64_t S, bool cr
     uint16_t* casc_wrel = nullptr;
     const int64_t* old_off_nc = static_cast<const int64_t*>(r->off[r->cur].p);
     const uint32_t* old_cols_nc = static_cast<const uint32_t*>(r->cols[r->cur].p);
-    if (n_node) {
+    if (node_mode) {
         uint64_t* kA = r->get<uint64_t>(r->keyA, n_node);
         uint64_t* kB = r->get<uint64_t>(r->keyB, n_node);
         uint32_t* vA = r->get<uint32_t>(r->valA, n_node);
@@ -383,130 +391,87 @@ h2tap_status apply_core(h2tap_replica* r, const BatchIn& in, uint64_t S, bool cr
 
         nv = r->get<NodeVtx>(r->nv, n_node);
         nv_ext = r->get<uint64_t>(r->nv_ext, n_node);
-        uint64_t nt = cdiv(n_node, kTile);
-        uint64_t* stt = r->get<uint64_t>(r->status, 3 * nt);
-        CK(cudaMemsetAsync(stt, 0, nt * 8, st));
+        const uint64_t nt = cdiv(n_node, kTile);  // also the tile bound of the unique-vertex list
+        uint64_t* stt = r->get<uint64_t>(r->status, 4 * nt);
+        CK(cudaMemsetAsync(stt, 0, 4 * nt * 8, st));
         k_node_segments<<<(unsigned)nt, kThreads, 0, st>>>(ops, node_sorted, n_node, ext_index(r), nv, nv_ext,
                                                            stt, nt, dc);
         CKL();
         TR("node_segments");
-        r->read_counters();
-        TR("sync_nseg");
-        U = r->hc->n_unique;
-        dropped = r->get<uint32_t>(r->dropped, U);
-        ins_q = r->get<uint32_t>(r->ins_q, U);
-        ins_oldpos = r->get<uint32_t>(r->ins_oldpos, U);
-        hd_rows = r->get<uint32_t>(r->hd_rows, U);
-        uint64_t nt2 = cdiv(U, kTile);
-        stt = r->get<uint64_t>(r->status, 3 * nt2);
-        CK(cudaMemsetAsync(stt, 0, 3 * nt2 * 8, st));
-        k_node_lists<<<(unsigned)nt2, kThreads, 0, st>>>(nv, U, dropped, ins_q, ins_oldpos, hd_rows, stt, nt2, dc);
+        dropped = r->get<uint32_t>(r->dropped, n_node);
+        ins_q = r->get<uint32_t>(r->ins_q, n_node);
+        ins_oldpos = r->get<uint32_t>(r->ins_oldpos, n_node);
+        hd_rows = r->get<uint32_t>(r->hd_rows, n_node);
+        k_node_lists<<<(unsigned)nt, kThreads, 0, st>>>(nv, dropped, ins_q, ins_oldpos, hd_rows, stt + nt, nt, dc);
         CKL();
-        uint32_t first_ins_oldpos = 0;
         TR("node_lists");
-        r->read_counters();
-        TR("sync_nlists");
-        n_dropped = r->hc->n_dropped;
-        n_vins = r->hc->n_inserted;
-        n_hd = r->hc->n_hd;
-        if (n_vins) {
-            g_d2h += 4;
-            CK(cudaMemcpyAsync(&r->hc->status, ins_oldpos, 4, cudaMemcpyDeviceToHost, st));
-            r->sync();
-            first_ins_oldpos = (uint32_t)(r->hc->status & 0xFFFFFFFFu);
-        }
-        Vn = V - n_dropped + n_vins;
-        if (Vn >= 0x7FFFFFFFull) { set_err("vertex count exceeds 2^31-1"); return H2TAP_E_CAPACITY; }
-        set_changed = n_dropped || n_vins;
-        remap_on = n_dropped > 0 || (n_vins > 0 && first_ins_oldpos < V);
-        if (set_changed) {
-            new_ext = r->get<uint64_t>(r->ext[ec ^ 1], Vn);
-            if (remap_on) {
-                // remap tables (64K-id block shifts, 32-id groups), then scatter the survivors
-                const uint64_t nblk = cdiv(V, 1ull << kRemapBlockShift), ng = cdiv(V, 32);
-                int32_t* rs = r->get<int32_t>(r->remap_shift, nblk + 4);  // + {lo, hi, shift}
-                uint2* r32 = r->get<uint2>(r->remap32, ng);
-                k_remap_blocks<<<g1(nblk), 256, 0, st>>>(V, dropped, n_dropped, ins_oldpos, n_vins, rs, rs + nblk);
-                CKL();
-                if (ng) { k_remap32<<<g1(ng), 256, 0, st>>>(V, dropped, n_dropped, ins_oldpos, n_vins, r32); CKL(); }
-                R.shift = rs; R.g32 = r32; R.ins_oldpos = ins_oldpos; R.n_vins = n_vins; R.lohi = rs + nblk;
-                TR("remap_tables");
-                if (V) { k_new_ext<<<g1(V), 256, 0, st>>>(old_ext, r->identity, V, R, new_ext); CKL(); }
-                TR("new_ext");
-            } else if (V) {
-                CK(cudaMemcpyAsync(new_ext, old_ext, V * 8, cudaMemcpyDeviceToDevice, st));
-            }
-            if (n_vins) {
-                k_place_inserted<<<g1(n_vins), 256, 0, st>>>(nv, nv_ext, ins_q, ins_oldpos, n_vins, dropped, n_dropped,
-                                                            new_ext);
-                CKL();
-            }
-        }
-        if (set_changed) {
-            // identity test of the new set is done at the end; fence built regardless
-            r->identity_pending = false;
-            build_fence(r, ec ^ 1, Vn);
-        }
-        k_nv_newid<<<g1(U), 256, 0, st>>>(nv, U, R);
+        // ID-map compaction: remap tables (64K-id block shifts, 32-id groups, the
+        // unchanged / uniformly shifted id ranges), then the survivors and the inserted
+        new_ext = r->get<uint64_t>(r->ext[ec ^ 1], Vn_ub);
+        const uint64_t nblk = cdiv(V, 1ull << kRemapBlockShift), ng = cdiv(V, 32);
+        int32_t* rs = r->get<int32_t>(r->remap_shift, nblk + 4);  // + {lo, hi, shift}
+        uint2* r32 = r->get<uint2>(r->remap32, ng);
+        k_remap_blocks<<<g1(nblk), 256, 0, st>>>(V, dropped, ins_oldpos, dc, rs, rs + nblk);  // also writes c->Vn
         CKL();
-        if (r->sharded) {
-            k_row_range<<<1, 1, 0, st>>>(set_changed ? new_ext : old_ext, Vn, r->own, dc);
-            CKL();
-            r->read_counters();
-            row_lo_new = r->hc->row_lo_new;
-            Vr_new = r->hc->row_hi_new - r->hc->row_lo_new;
-        } else {
-            Vr_new = Vn;
-        }
-        if (n_hd) {
-            hd_bits = r->get<uint32_t>(r->hd_bits, cdiv(V, 32));
-            CK(cudaMemsetAsync(hd_bits, 0, cdiv(V, 32) * 4, st));
-            k_set_bits<<<g1(n_hd), 256, 0, st>>>(hd_rows, n_hd, hd_bits);
-            CKL();
-            // cascade pass on the side stream, overlapped with the edge-op phase
-            const uint64_t nblk = cdiv(E, kCascBlock);
-            casc_mask = r->get<uint32_t>(r->casc_mask, (nblk + 2) * (kCascBlock / 32));
-            casc_cnt = r->get<uint64_t>(r->tile_emit, nblk + 1);
-            casc_pre = r->get<uint64_t>(r->tile_base, nblk + 1);
-            // in-line on the main stream: overlapping this streaming pass with the
-            // latency-bound edge-op kernels only delayed them (H2TAP_TRACE measurements)
-            cudaStream_t s2 = st;
-            unsigned rg = (unsigned)std::min<uint64_t>(cdiv(n_hd * 32, 256), (uint64_t)r->n_sm * 8);
-            const uint64_t nst = cdiv(nblk + 1, kThreads);
-            uint64_t* st2s2 = r->get<uint64_t>(r->status2, nst);
-            CK(cudaMemsetAsync(st2s2, 0, nst * 8, s2));
-            TR("nv_newid+bits");
-            if (nblk) {
-                k_casc_cols<<<(unsigned)cdiv(nblk, 2), kThreads, 0, s2>>>(old_cols_nc, E, hd_bits, hd_rows, n_hd, casc_mask);
-                CKL();
-                TR("casc_cols");
-                k_casc_rows<<<rg, 256, 0, s2>>>(old_off_nc, hd_rows, n_hd, row_lo, row_lo + Vr, casc_mask);
-                CKL();
-                TR("casc_rows");
-            }
-            casc_wrel = r->get<uint16_t>(r->casc_wrel, (nblk + 1) * (kCascBlock / 32));
-            k_casc_scan<<<(unsigned)nst, kThreads, 0, s2>>>(casc_mask, nblk, casc_pre, casc_wrel, st2s2, &dc->tiles[6]);
-            CKL();
-            k_copy_u64<<<1, 1, 0, s2>>>(&dc->n_casc, casc_pre + nblk);
+        if (ng) { k_remap32<<<g1(ng), 256, 0, st>>>(V, dropped, ins_oldpos, dc, r32); CKL(); }
+        R.shift = rs; R.g32 = r32; R.ins_oldpos = ins_oldpos; R.n_vins = &dc->n_inserted; R.lohi = rs + nblk;
+        TR("remap_tables");
+        if (V) { k_new_ext<<<g1(V), 256, 0, st>>>(old_ext, r->identity, V, R, new_ext); CKL(); }
+        TR("new_ext");
+        k_place_inserted<<<g1(n_node), 256, 0, st>>>(nv, nv_ext, ins_q, ins_oldpos, dropped, dc, new_ext);
+        CKL();
+        {
+            uint64_t* f = r->get<uint64_t>(r->fence[ec ^ 1], n_fence(Vn_ub));
+            k_build_fence_dev<<<g1(n_fence(Vn_ub)), 256, 0, st>>>(new_ext, dc, f);
             CKL();
         }
+        k_nv_newid<<<g1(n_node), 256, 0, st>>>(nv, dc, R);
+        CKL();
+        if (r->sharded) { k_row_range<<<1, 1, 0, st>>>(new_ext, ~0ull, r->own, dc); CKL(); }
+        // cascade pass (a4, reading A8): one bit per old element removed by a node delete
+        hd_bits = r->get<uint32_t>(r->hd_bits, cdiv(V, 32));
+        CK(cudaMemsetAsync(hd_bits, 0, cdiv(V, 32) * 4, st));
+        k_set_bits<<<g1(n_node), 256, 0, st>>>(hd_rows, dc, hd_bits);
+        CKL();
+        const uint64_t nblk_c = cdiv(E, kCascBlock);
+        casc_mask = r->get<uint32_t>(r->casc_mask, (nblk_c + 2) * (kCascBlock / 32));
+        casc_cnt = r->get<uint64_t>(r->tile_emit, nblk_c + 1);
+        casc_pre = r->get<uint64_t>(r->tile_base, nblk_c + 1);
+        unsigned rg = (unsigned)std::min<uint64_t>(cdiv(n_node * 32, 256), (uint64_t)r->n_sm * 8);
+        const uint64_t nst = cdiv(nblk_c + 1, kThreads);
+        uint64_t* st2s2 = r->get<uint64_t>(r->status2, nst);
+        CK(cudaMemsetAsync(st2s2, 0, nst * 8, st));
+        TR("nv_newid+bits");
+        if (nblk_c) {
+            k_casc_cols<<<(unsigned)cdiv(nblk_c, 2), kThreads, 0, st>>>(old_cols_nc, E, hd_bits, hd_rows, dc, casc_mask);
+            CKL();
+            TR("casc_cols");
+            k_casc_rows<<<rg, 256, 0, st>>>(old_off_nc, hd_rows, dc, row_lo, row_lo + Vr, casc_mask);
+            CKL();
+            TR("casc_rows");
+        }
+        casc_wrel = r->get<uint16_t>(r->casc_wrel, (nblk_c + 1) * (kCascBlock / 32));
+        k_casc_scan<<<(unsigned)nst, kThreads, 0, st>>>(casc_mask, nblk_c, casc_pre, casc_wrel, st2s2, &dc->tiles[6]);
+        CKL();
+        k_copy_u64<<<1, 1, 0, st>>>(&dc->n_casc, casc_pre + nblk_c);
+        CKL();
     }
     CK(cudaEventRecord(r->ev[2], st));
     TR("idmap+remap");
 
     // ---- a3: edge ops -> keys, sort, segmented reduce + classify
-    const int bits = std::max(1, bits_for(Vn > 1 ? Vn - 1 : 1));
+    const int bits = std::max(1, bits_for(Vn_ub > 1 ? Vn_ub - 1 : 1));  // dense ids < Vn <= Vn_ub
     const int64_t* old_off = static_cast<const int64_t*>(r->off[r->cur].p);
     const uint32_t* old_cols = static_cast<const uint32_t*>(r->cols[r->cur].p);
     const float* old_w = static_cast<const float*>(r->w[r->cur].p);
-    uint64_t n_valid = 0, n_ins = 0, n_del = 0, n_upd = 0, n_gated = 0;
-    uint64_t* ins_pos = r->get<uint64_t>(r->ins_pos, 1);
-    uint32_t* ins_row = r->get<uint32_t>(r->ins_row, 1);
-    uint32_t* ins_col = r->get<uint32_t>(r->ins_col, 1);
-    float* ins_w = r->get<float>(r->ins_w, 1);
-    uint64_t* del_pos = r->get<uint64_t>(r->del_pos, 1);
-    uint64_t* upd_pos = r->get<uint64_t>(r->upd_pos, 1);
-    float* upd_w = r->get<float>(r->upd_w, 1);
+    uint64_t* ins_pos = r->get<uint64_t>(r->ins_pos, n_edge);
+    uint32_t* ins_row = r->get<uint32_t>(r->ins_row, n_edge);
+    uint32_t* ins_col = r->get<uint32_t>(r->ins_col, n_edge);
+    float* ins_w = r->get<float>(r->ins_w, n_edge);
+    uint64_t* del_pos = r->get<uint64_t>(r->del_pos, n_edge);
+    uint32_t* del_row = r->get<uint32_t>(r->del_row, n_edge);
+    uint64_t* upd_pos = r->get<uint64_t>(r->upd_pos, n_edge);
+    float* upd_w = r->get<float>(r->upd_w, n_edge);
     if (n_edge) {
         uint64_t* kA = r->get<uint64_t>(r->keyA, n_edge);
         uint64_t* kB = r->get<uint64_t>(r->keyB, n_edge);
@@ -520,7 +485,6 @@ h2tap_status apply_core(h2tap_replica* r, const BatchIn& in, uint64_t S, bool cr
         pa.R = R;
         pa.nv = nv;
         pa.nv_ext = nv_ext;
-        pa.U = U;
         pa.node_sorted = node_sorted;
         pa.bits = bits;
         pa.create = create ? 1 : 0;
@@ -528,7 +492,7 @@ h2tap_status apply_core(h2tap_replica* r, const BatchIn& in, uint64_t S, bool cr
         pa.keys = kA;
         pa.vals = vA;
         pa.recs = r->get<EdgeRec>(r->op_flags, m);
-        const bool lookups_direct = r->identity && U == 0;  // no searches -> 8 ops per thread
+        const bool lookups_direct = r->identity && !node_mode;  // no searches -> 8 ops per thread
         const int eitems = lookups_direct ? 8 : 1;
         uint64_t nt = cdiv(n_edge, (uint64_t)kThreads * eitems);
         pa.status = r->get<uint64_t>(r->status, 3 * nt);
@@ -539,80 +503,52 @@ h2tap_status apply_core(h2tap_replica* r, const BatchIn& in, uint64_t S, bool cr
         else k_edge_prep<1><<<(unsigned)nt, kThreads, 0, st>>>(pa);
         CKL();
         TR("edge_prep");
-        r->read_counters();
-        TR("sync_prep");
-        if (create && (r->hc->status & ST_CREATE_ENDPOINT)) {
-            set_err("create: edge endpoint not in the vertex set");
-            return H2TAP_E_INVAL;
-        }
-        if (r->hc->status & ST_NOT_OWNED) {
-            set_err("sharded replica: edge op whose source is owned by another shard");
-            return H2TAP_E_INVAL;
-        }
-        n_valid = r->hc->n_valid;
-        n_gated = r->hc->n_gated;
-        radix_sort(r, kA, vA, kB, vB, n_valid, 2 * bits);
+        radix_sort(r, kA, vA, kB, vB, n_edge, 2 * bits, &dc->n_valid);
         TR("edge_sort");
-        ins_pos = r->get<uint64_t>(r->ins_pos, n_valid);
-        ins_row = r->get<uint32_t>(r->ins_row, n_valid);
-        ins_col = r->get<uint32_t>(r->ins_col, n_valid);
-        ins_w = r->get<float>(r->ins_w, n_valid);
-        del_pos = r->get<uint64_t>(r->del_pos, n_valid);
-        r->get<uint32_t>(r->del_row, n_valid);
-        upd_pos = r->get<uint64_t>(r->upd_pos, n_valid);
-        upd_w = r->get<float>(r->upd_w, n_valid);
-        if (n_valid) {
-            ClassArgs ca{};
-            ca.ops = ops;
-            ca.keys = kA;
-            ca.vals = vA;
-            ca.n = n_valid;
-            ca.bits = bits;
-            ca.recs = pa.recs;
-            ca.old_off = old_off - row_lo;  // indexed by global dense ids of owned rows
-            ca.old_cols = old_cols;
-            ca.V_old = V;
-            ca.ins_pos = ins_pos; ca.ins_row = ins_row; ca.ins_col = ins_col; ca.ins_w = ins_w;
-            ca.del_pos = del_pos;
-            ca.del_row = static_cast<uint32_t*>(r->del_row.p);
-            ca.upd_pos = upd_pos; ca.upd_w = upd_w;
-            uint64_t nt2 = cdiv(n_valid, kCTile);
-            ca.status3 = r->get<uint64_t>(r->status, 3 * nt2);
-            CK(cudaMemsetAsync(ca.status3, 0, 3 * nt2 * 8, st));
-            ca.n_tiles = nt2;
-            ca.c = dc;
-            k_reduce_classify<<<(unsigned)nt2, kThreads, 0, st>>>(ca);
-            CKL();
-            TR("classify");
-            r->read_counters();
-            TR("sync_cls");
-            n_ins = r->hc->n_ins;
-            n_del = r->hc->n_del;
-            n_upd = r->hc->n_upd;
-        }
+        ClassArgs ca{};
+        ca.ops = ops;
+        ca.keys = kA;
+        ca.vals = vA;
+        ca.n = n_edge;  // upper bound; the kernel reads n_valid
+        ca.bits = bits;
+        ca.recs = pa.recs;
+        ca.old_off = old_off - row_lo;  // indexed by global dense ids of owned rows
+        ca.old_cols = old_cols;
+        ca.V_old = V;
+        ca.ins_pos = ins_pos; ca.ins_row = ins_row; ca.ins_col = ins_col; ca.ins_w = ins_w;
+        ca.del_pos = del_pos;
+        ca.del_row = del_row;
+        ca.upd_pos = upd_pos; ca.upd_w = upd_w;
+        uint64_t nt2 = cdiv(n_edge, kCTile);
+        ca.status3 = r->get<uint64_t>(r->status2, 3 * nt2);
+        CK(cudaMemsetAsync(ca.status3, 0, 3 * nt2 * 8, st));
+        ca.n_tiles = nt2;
+        ca.c = dc;
+        k_reduce_classify<<<(unsigned)nt2, kThreads, 0, st>>>(ca);
+        CKL();
+        TR("classify");
     }
     CK(cudaEventRecord(r->ev[3], st));
 
-    // ---- a6: merge into the back buffer (skipped when no op changes the CSR)
-    const bool csr_changed = n_node || n_ins || n_del || n_upd;
+    // ---- a6: merge into the back buffer (skipped when no op can change the CSR)
+    const bool csr_changed = node_mode || n_edge;
     const int nb = csr_changed ? (r->cur ^ 1) : r->cur;
-    uint64_t n_casc = 0, En = E;
+    int64_t* new_off = nullptr;
+    const bool casc = node_mode;
     if (csr_changed) {
-    const uint64_t Ecap = E + n_ins;
-    int64_t* new_off = r->get<int64_t>(r->off[nb], Vr_new + 1);
+    const uint64_t Ecap = E + n_edge;  // >= E + n_ins
+    new_off = r->get<int64_t>(r->off[nb], Vr_new_ub + 1);
     uint32_t* new_cols = r->get<uint32_t>(r->cols[nb], Ecap);
     float* new_w = r->get<float>(r->w[nb], Ecap);
-    const bool casc = n_hd > 0;
-    const uint64_t Dtot = E + n_ins;
-    if (Dtot) {
+    if (Ecap) {
         MergeArgs ma{};
         ma.old_cols = old_cols; ma.old_w = old_w; ma.E_old = E;
-        ma.ins_pos = ins_pos; ma.ins_col = ins_col; ma.ins_w = ins_w; ma.n_ins = n_ins;
-        ma.del_pos = del_pos; ma.n_del = n_del;
-        ma.upd_pos = upd_pos; ma.upd_w = upd_w; ma.n_upd = n_upd;
+        ma.ins_pos = ins_pos; ma.ins_col = ins_col; ma.ins_w = ins_w;
+        ma.del_pos = del_pos;
+        ma.upd_pos = upd_pos; ma.upd_w = upd_w;
         ma.R = R;
         ma.new_cols = new_cols; ma.new_w = new_w;
-        ma.n_tiles = cdiv(Dtot, kMergeTile);
+        ma.n_tiles = cdiv(Ecap, kMergeTile);  // upper bound; the kernels use E + n_ins
         ma.c = dc;
         if (casc) {
             ma.casc_mask = casc_mask;
@@ -630,26 +566,17 @@ h2tap_status apply_core(h2tap_replica* r, const BatchIn& in, uint64_t S, bool cr
             const uint64_t grid = std::min<uint64_t>(ma.n_tiles, (uint64_t)std::max(1, occ) * r->n_sm);
             kern<<<(unsigned)grid, kThreads, kMerge3Smem, st>>>(ma, part);
         };
-        if (casc && remap_on) launch(k_merge3<true, true>);
-        else if (casc) launch(k_merge3<true, false>);
-        else if (remap_on) launch(k_merge3<false, true>);
+        if (node_mode) launch(k_merge3<true, true>);
         else launch(k_merge3<false, false>);
         CKL();
     } else {
-        // nothing to merge: every surviving row is empty
-        if (n_node) CK(cudaMemsetAsync(new_off, 0, (Vr_new + 1) * 8, st));
         CK(cudaEventRecord(r->ev[6], st));
     }
     CK(cudaEventRecord(r->ev[4], st));
     TR("merge");
-    if (casc) {
-        r->read_counters();
-        n_casc = r->hc->n_casc;
-    }
-    En = E + n_ins - n_del - n_casc;
 
     // ---- a4/a5: row offsets
-    if (Vr && !n_node) {
+    if (Vr && !node_mode) {
         // per-vertex degree delta + exclusive scan (tile sums by decoupled look-back)
         int32_t* deg = r->get<int32_t>(r->deg, Vr);
         const uint64_t nt = cdiv(Vr, kTile);
@@ -657,8 +584,8 @@ h2tap_status apply_core(h2tap_replica* r, const BatchIn& in, uint64_t S, bool cr
         int64_t* tbase = r->get<int64_t>(r->KR, nt + 1);
         CK(cudaMemsetAsync(deg, 0, Vr * 4, st));
         CK(cudaMemsetAsync(tsum, 0, (nt + 1) * 8, st));
-        if (n_ins + n_del) {
-            k_deg_scatter<<<g1(n_ins + n_del), 256, 0, st>>>(ins_row, n_ins, static_cast<uint32_t*>(r->del_row.p), n_del, deg, tsum, row_lo);
+        if (n_edge) {
+            k_deg_scatter<<<g1(n_edge), 256, 0, st>>>(ins_row, del_row, dc, deg, tsum, row_lo);
             CKL();
         }
         const uint64_t nts = cdiv(nt, kTile);
@@ -669,27 +596,27 @@ h2tap_status apply_core(h2tap_replica* r, const BatchIn& in, uint64_t S, bool cr
         k_offsets_apply<<<(unsigned)nt, kThreads, 0, st>>>(old_off, deg, Vr, tbase, new_off);
         CKL();
     }
-    if (n_node && (Vr || Vr_new)) {
+    if (node_mode) {
         RowArgs ra{};
         ra.old_off = old_off - row_lo; ra.V_old = V; ra.E_old = E; ra.R = R;
-        ra.row_lo = row_lo; ra.row_hi = row_lo + Vr; ra.row_lo_new = row_lo_new;
+        ra.row_lo = row_lo; ra.row_hi = row_lo + Vr;
         ra.own = r->own; ra.nv_ext = nv_ext;
-        ra.casc_mask = casc ? casc_mask : nullptr; ra.casc_pre = casc_pre; ra.casc_wrel = casc_wrel;
-        ra.del_pos = del_pos; ra.n_del = n_del; ra.ins_row = ins_row; ra.n_ins = n_ins;
-        ra.dropped = dropped; ra.n_dropped = n_dropped; ra.ins_oldpos = ins_oldpos; ra.n_vins = n_vins;
+        ra.casc_mask = casc_mask; ra.casc_pre = casc_pre; ra.casc_wrel = casc_wrel;
+        ra.del_pos = del_pos; ra.ins_row = ins_row;
+        ra.dropped = dropped; ra.ins_oldpos = ins_oldpos;
         ra.new_off = new_off;
+        ra.c = dc;
         const uint64_t ncta = cdiv(Vr, kRowTile);
         ra.part = r->get<uint64_t>(r->opart, 2 * (ncta + 1));
-        k_rows_partition<<<g1(ncta + 1), 256, 0, st>>>(ra);
-        CKL();
-        if (ncta) { k_offsets_rows<<<(unsigned)ncta, kThreads, 0, st>>>(ra); CKL(); }
-        if (n_vins) {
-            k_offsets_inserted<<<g1(n_vins), 256, 0, st>>>(nv, ins_q, n_vins, ra);
+        if (Vr) {
+            k_rows_partition<<<g1(ncta + 1), 256, 0, st>>>(ra);
+            CKL();
+            k_offsets_rows<<<(unsigned)ncta, kThreads, 0, st>>>(ra);
             CKL();
         }
+        k_offsets_inserted<<<g1(n_node), 256, 0, st>>>(nv, ins_q, ra);
+        CKL();
     }
-    k_set_i64<<<1, 1, 0, st>>>(new_off + Vr_new, (int64_t)En);
-    CKL();
     } else {
         CK(cudaEventRecord(r->ev[6], st));
         CK(cudaEventRecord(r->ev[4], st));
@@ -704,28 +631,32 @@ h2tap_status apply_core(h2tap_replica* r, const BatchIn& in, uint64_t S, bool cr
             r->get<uint64_t>(r->pt[pn], n_pend_new), r->get<uint64_t>(r->pq[pn], n_pend_new));
         CKL();
     }
+    k_finish<<<1, 1, 0, st>>>(dc, V, Vr, E, node_mode ? 1 : 0, r->sharded ? 1 : 0, new_ext, new_off);
+    CKL();
     CK(cudaEventRecord(r->ev[5], st));
     TR("offsets+pending");
-    bool new_identity = r->identity;
-    if (set_changed) {
-        if (Vn == 0) new_identity = true;
-        else {
-            uint64_t last = 0;
-            g_d2h += 8;
-            CK(cudaMemcpyAsync(&r->hc->status, new_ext + Vn - 1, 8, cudaMemcpyDeviceToHost, st));
-            r->sync();
-            last = r->hc->status;
-            new_identity = (last == Vn - 1);
-        }
-    }
-    r->sync();
+    r->read_counters();  // the one read-back of the cycle's device-side sizes
     TR("end");
     g_tr.dump();
+    const Counters& fc = *r->hc;
+    if (create && (fc.status & ST_CREATE_ENDPOINT)) {
+        set_err("create: edge endpoint not in the vertex set");
+        return H2TAP_E_INVAL;
+    }
+    if (fc.status & ST_NOT_OWNED) {
+        set_err("sharded replica: edge op whose source is owned by another shard");
+        return H2TAP_E_INVAL;
+    }
+    const uint64_t Vn = fc.Vn, Vr_new = fc.Vr_new, En = fc.En;
+    const uint64_t row_lo_new = (node_mode && r->sharded) ? fc.row_lo_new : row_lo;
+    const uint64_t n_ins = fc.n_ins, n_del = fc.n_del, n_upd = fc.n_upd, n_casc = fc.n_casc;
 
     // ---- a7: swap at snapshot_ts (nothing above touched the front state)
     r->cur = nb;
-    if (set_changed) r->ext_cur = ec ^ 1;
-    r->identity = new_identity;
+    if (node_mode) {
+        r->ext_cur = ec ^ 1;
+        r->identity = fc.new_identity == 1;
+    }
     r->V = Vn;
     r->E = En;
     r->row_lo = row_lo_new;
@@ -738,13 +669,13 @@ h2tap_status apply_core(h2tap_replica* r, const BatchIn& in, uint64_t S, bool cr
         memset(stats, 0, sizeof *stats);
         stats->n_visible = n_node + n_edge;
         stats->n_deferred = n_pend_new;
-        stats->n_gated = n_gated;
+        stats->n_gated = fc.n_gated;
         stats->n_new = n_ins;
         stats->n_del = n_del;
         stats->n_upd = n_upd;
         stats->n_casc = n_casc;
-        stats->n_vertex_inserted = n_vins;
-        stats->n_vertex_deleted = n_dropped;
+        stats->n_vertex_inserted = fc.n_inserted;
+        stats->n_vertex_deleted = fc.n_dropped;
         stats->ms_ingest = ev_ms(r->ev[0], r->ev[1]);
         stats->ms_nodeops = ev_ms(r->ev[1], r->ev[2]);
         stats->ms_sort_reduce = ev_ms(r->ev[2], r->ev[3]);
@@ -754,14 +685,14 @@ h2tap_status apply_core(h2tap_replica* r, const BatchIn& in, uint64_t S, bool cr
         stats->ms_degree_scan = ev_ms(r->ev[3], r->ev[6]) + ev_ms(r->ev[4], r->ev[5]);
         stats->ms_total = ev_ms(r->ev[0], r->ev[5]);
         uint64_t b = 8 * (Vr + 1) + 8 * E + 8 * (Vr_new + 1) + 8 * En + 29 * n;
-        if (n_node) b += 16 * V + 4 * E + 4 * V;
+        if (node_mode) b += 16 * V + 4 * E + 4 * V;
         stats->bytes_alg = b;
         // merge launch: stream old cols+weights, write new ones, read the outcome lists
         // (+ remap table and cascade bitmap when node ops changed the ID map)
         uint64_t bm = 0;
         if (csr_changed && E + n_ins) {
             bm = 8 * E + 8 * En + 20 * n_ins + 8 * n_del + 12 * n_upd;
-            if (n_hd) bm += E / 8;                                       // cascade mask
+            if (node_mode) bm += E / 8;                                  // cascade mask
         }
         stats->bytes_merge = bm;
         stats->n_launches = g_launches;

@@ -38,6 +38,7 @@ struct Counters {
     unsigned long long n_ins, n_del, n_upd;
     unsigned long long n_casc;
     unsigned long long row_lo_new, row_hi_new;  // sharded: the shard's row range in the new ID map
+    unsigned long long Vn, Vr_new, En, new_identity;  // written by k_finish
     unsigned int tiles[16];
 };
 
@@ -71,7 +72,7 @@ struct RemapView {
     const int32_t* shift;  // nullptr: identity
     const uint2* g32;
     const uint32_t* ins_oldpos;
-    uint64_t n_vins;
+    const unsigned long long* n_vins;  // device count of inserted vertices
     const int32_t* lohi;   // {lo, hi, shift}: ids < lo unchanged, ids >= hi shifted by `shift`
 };
 __device__ __forceinline__ uint32_t remap_of(const RemapView& R, uint32_t k) {
@@ -82,14 +83,16 @@ __device__ __forceinline__ uint32_t remap_of(const RemapView& R, uint32_t k) {
     const uint32_t r = k & 31;
     if (g.y >> r & 1) return kNone32;  // dropped
     uint32_t v = (g.x & 0x7FFFFFFFu) + r - (r ? __popc(g.y & (0xFFFFFFFFu >> (32 - r))) : 0u);
-    if (g.x >> 31) v += (uint32_t)(upper_bound_dev(R.ins_oldpos, 0, R.n_vins, k) -
-                             upper_bound_dev(R.ins_oldpos, 0, R.n_vins, k - r));
+    if (g.x >> 31) {
+        const uint64_t nv = *R.n_vins;
+        v += (uint32_t)(upper_bound_dev(R.ins_oldpos, 0, nv, k) - upper_bound_dev(R.ins_oldpos, 0, nv, k - r));
+    }
     return v;
 }
 
 // out-of-line exact path (fields by value: no stack copy of the view in the caller)
 __device__ __noinline__ uint32_t remap_of_slow(const int32_t* shift, const uint2* g32, const uint32_t* ins_oldpos,
-                                               uint64_t n_vins, uint32_t k) {
+                                               const unsigned long long* n_vins, uint32_t k) {
     RemapView R{shift, g32, ins_oldpos, n_vins, nullptr};
     return remap_of(R, k);
 }
@@ -351,15 +354,17 @@ __global__ void __launch_bounds__(kThreads) k_node_segments(
 
 // dropped (old-live -> dead), inserted (new & finally live), hd (old-present with a delete)
 __global__ void __launch_bounds__(kThreads) k_node_lists(
-    const NodeVtx* __restrict__ nv, uint64_t U, uint32_t* __restrict__ dropped,
+    const NodeVtx* __restrict__ nv, uint32_t* __restrict__ dropped,
     uint32_t* __restrict__ ins_q, uint32_t* __restrict__ ins_oldpos, uint32_t* __restrict__ hd_rows,
-    uint64_t* __restrict__ status3, uint64_t n_tiles, Counters* __restrict__ c) {
+    uint64_t* __restrict__ status3, uint64_t n_tiles_ub, Counters* __restrict__ c) {
     __shared__ uint32_t s_tile;
     __shared__ uint64_t s_scan[kThreads / 32 + 1];
     __shared__ uint64_t s_base[3];
     if (threadIdx.x == 0) s_tile = atomicAdd(&c->tiles[2], 1u);
     __syncthreads();
     const uint32_t tile = s_tile;
+    const uint64_t U = c->n_unique, n_tiles = (U + kTile - 1) / kTile;  // grid: upper bound
+    if (tile >= n_tiles) return;
     const uint64_t i0 = (uint64_t)tile * kTile + (uint64_t)threadIdx.x * kItems;
     uint64_t cnt[3] = {0, 0, 0};
     uint32_t fl[kItems];
@@ -380,7 +385,7 @@ __global__ void __launch_bounds__(kThreads) k_node_lists(
     for (int q = 0; q < 3; ++q) excl[q] = block_exclusive_scan<kThreads>(cnt[q], s_scan, &tot[q]);
     const int wid = threadIdx.x >> 5;
     if (wid < 3) {
-        uint64_t b = lookback_warp(status3 + (uint64_t)wid * n_tiles, tile, tot[wid]);
+        uint64_t b = lookback_warp(status3 + (uint64_t)wid * n_tiles_ub, tile, tot[wid]);
         if (lane_id() == 0) {
             s_base[wid] = b;
             if (tile == n_tiles - 1) {
@@ -428,9 +433,10 @@ __global__ void k_new_ext(const uint64_t* __restrict__ old_ext, int identity, ui
 // inserted vertex i lands at oldpos_i - (#dropped before oldpos_i) + i
 __global__ void k_place_inserted(NodeVtx* __restrict__ nv, const uint64_t* __restrict__ nv_ext,
                                  const uint32_t* __restrict__ ins_q, const uint32_t* __restrict__ ins_oldpos,
-                                 uint64_t n_ins, const uint32_t* __restrict__ dropped, uint64_t n_dropped,
+                                 const uint32_t* __restrict__ dropped, const Counters* __restrict__ c,
                                  uint64_t* __restrict__ new_ext) {
     uint64_t i = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x;
+    const uint64_t n_ins = c->n_inserted, n_dropped = c->n_dropped;
     if (i >= n_ins) return;
     uint32_t op = ins_oldpos[i];
     uint64_t pos = op - lower_bound_dev(dropped, 0, n_dropped, op) + i;
@@ -439,16 +445,16 @@ __global__ void k_place_inserted(NodeVtx* __restrict__ nv, const uint64_t* __res
 }
 
 // new ids of surviving old vertices that have node ops
-__global__ void k_nv_newid(NodeVtx* __restrict__ nv, uint64_t U, RemapView R) {
+__global__ void k_nv_newid(NodeVtx* __restrict__ nv, const Counters* __restrict__ c, RemapView R) {
     uint64_t q = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x;
-    if (q >= U) return;
+    if (q >= c->n_unique) return;
     uint32_t f = nv[q].flags;
     if ((f & NV_OLD) && (f & NV_FINAL)) nv[q].newid = remap_of(R, nv[q].oldpos);
 }
 
-__global__ void k_set_bits(const uint32_t* __restrict__ rows, uint64_t n, uint32_t* __restrict__ bits) {
+__global__ void k_set_bits(const uint32_t* __restrict__ rows, const Counters* __restrict__ c, uint32_t* __restrict__ bits) {
     uint64_t i = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x;
-    if (i < n) atomicOr(&bits[rows[i] >> 5], 1u << (rows[i] & 31));
+    if (i < c->n_hd) atomicOr(&bits[rows[i] >> 5], 1u << (rows[i] & 31));
 }
 
 // ===================================================================== a3 ====
@@ -480,7 +486,7 @@ struct PrepArgs {
     RemapView R;            // identity when R.shift == nullptr
     const NodeVtx* nv;
     const uint64_t* nv_ext;
-    uint64_t U;
+    uint64_t U;                   // node mode: read from c->n_unique at kernel start
     const uint32_t* node_sorted;  // (v, ts, seq)-sorted node op indices
     int bits;                     // bits of a dense id in the packed key
     int create;                   // create_from_edges: endpoints must exist
@@ -493,14 +499,14 @@ struct PrepArgs {
     Counters* c;
 };
 
-__device__ __forceinline__ Lookup do_lookup(const PrepArgs& a, uint64_t x) {
+__device__ __forceinline__ Lookup do_lookup(const PrepArgs& a, uint64_t U, uint64_t x) {
     Lookup L;
     L.q = -1;
     L.hasD = false;
     L.tD_ts = 0; L.tD_seq = 0;
-    if (a.U) {
-        uint64_t q = lower_bound_dev(a.nv_ext, 0, a.U, x);
-        if (q < a.U && a.nv_ext[q] == x) {
+    if (U) {
+        uint64_t q = lower_bound_dev(a.nv_ext, 0, U, x);
+        if (q < U && a.nv_ext[q] == x) {
             const NodeVtx& r = a.nv[q];
             L.q = (int64_t)q;
             L.oldpos = r.oldpos;
@@ -550,6 +556,7 @@ __global__ void __launch_bounds__(kThreads) k_edge_prep(PrepArgs a) {
     __syncthreads();
     const uint32_t tile = s_tile;
     const uint64_t i0 = (uint64_t)tile * kETile + threadIdx.x;
+    const uint64_t U = a.nv ? a.c->n_unique : 0;
     uint64_t key[kEItems];
     bool valid[kEItems];
     uint32_t pos[kEItems];
@@ -563,11 +570,13 @@ __global__ void __launch_bounds__(kThreads) k_edge_prep(PrepArgs a) {
         uint32_t o = a.edge_idx[i];
         uint8_t kind = a.ops.kind[o];
         uint64_t ts = a.ops.ts[o], seq = a.ops.seq[o];
-        Lookup Lu = do_lookup(a, a.ops.src[o]);
-        Lookup Lw = do_lookup(a, a.ops.dst[o]);
+        Lookup Lu = do_lookup(a, U, a.ops.src[o]);
+        Lookup Lw = do_lookup(a, U, a.ops.dst[o]);
         bool ok = Lu.final_live && Lw.final_live;
         if (a.create && !(Lu.old_present && Lw.old_present)) nbad++;
-        if (!a.own.owns(a.ops.src[o])) nbad |= 1ull << 40;  // routed to the wrong shard
+        // routed to the wrong shard: flagged (the apply fails) and dropped here, so the
+        // rest of the cycle never indexes rows this shard does not hold
+        if (!a.own.owns(a.ops.src[o])) { nbad |= 1ull << 40; ok = false; }
         if (ok && (Lu.hasD || Lw.hasD)) {
             // superseded by a later node delete of an endpoint (A8)
             if (Lu.hasD && pt_less(ts, seq, Lu.tD_ts, Lu.tD_seq)) ok = false;
@@ -654,6 +663,9 @@ __global__ void __launch_bounds__(kThreads) k_reduce_classify(ClassArgs a) {
     if (threadIdx.x == 0) s_tile = atomicAdd(&a.c->tiles[4], 1u);
     __syncthreads();
     const uint32_t tile = s_tile;
+    const uint64_t n = min(a.n, (uint64_t)a.c->n_valid);  // a.n: the grid's upper bound
+    const uint64_t n_tiles = (n + kCTile - 1) / kCTile;
+    if (tile >= n_tiles) return;
     const uint64_t i0 = (uint64_t)tile * kCTile + threadIdx.x;
     uint8_t cat[kCItems], meta[kCItems];
     uint64_t pos[kCItems], lo[kCItems], hi[kCItems], end[kCItems];
@@ -668,7 +680,7 @@ __global__ void __launch_bounds__(kThreads) k_reduce_classify(ClassArgs a) {
         colq[j] = 0;
         meta[j] = 0;
         uint64_t i = i0 + (uint64_t)j * kThreads;
-        if (i >= a.n) continue;
+        if (i >= n) continue;
         uint64_t key = a.keys[i];
         if (i > 0 && a.keys[i - 1] == key) continue;
         // segment [i, e): latest-commit-wins over (ts, seq)
@@ -677,7 +689,7 @@ __global__ void __launch_bounds__(kThreads) k_reduce_classify(ClassArgs a) {
         uint8_t nw_kind = 0;
         float w_val = 0.f;
         EdgeRec r0;
-        for (uint64_t e = i; e < a.n && a.keys[e] == key; ++e) {
+        for (uint64_t e = i; e < n && a.keys[e] == key; ++e) {
             const EdgeRec re = a.recs[a.vals[e]];
             if (e == i) r0 = re;
             uint8_t k = re.kind;
@@ -752,7 +764,7 @@ __global__ void __launch_bounds__(kThreads) k_reduce_classify(ClassArgs a) {
         uint64_t b = lookback_warp(a.status3 + (uint64_t)wid * a.n_tiles, tile, tot[wid]);
         if (lane_id() == 0) {
             s_base[wid] = b;
-            if (tile == a.n_tiles - 1) {
+            if (tile == n_tiles - 1) {
                 unsigned long long* d = wid == 0 ? &a.c->n_ins : (wid == 1 ? &a.c->n_del : &a.c->n_upd);
                 *d = b + tot[wid];
             }
@@ -811,9 +823,17 @@ struct MergeArgs {
     float* new_w;
     const uint32_t* casc_mask;  // CASC: 1 bit per old element (removed by a node delete)
     const uint64_t* casc_pre;   // CASC: cascaded elements before each 2048-element block
-    uint64_t n_tiles;
+    uint64_t n_tiles;           // host: upper bound (grid / partition size); device: actual
     Counters* c;
 };
+// the outcome-list sizes live in device memory (no host sync between classify and merge)
+__device__ __forceinline__ MergeArgs merge_counts(MergeArgs a) {
+    a.n_ins = a.c->n_ins;
+    a.n_del = a.c->n_del;
+    a.n_upd = a.c->n_upd;
+    a.n_tiles = (a.E_old + a.n_ins + kMergeTile - 1) / kMergeTile;
+    return a;
+}
 
 // Merge-path split of tile boundary t: r = inserted records among the first d
 // merged items (smallest r with ins_pos[r] + r >= d), j = d - r old elements,
@@ -833,7 +853,8 @@ __device__ __forceinline__ uint64_t ins_split(const uint64_t* ins_pos, uint64_t 
     return lo;
 }
 
-__global__ void k_merge_partition(MergeArgs a, TilePart* __restrict__ part) {
+__global__ void k_merge_partition(MergeArgs a_, TilePart* __restrict__ part) {
+    const MergeArgs a = merge_counts(a_);
     uint64_t t = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x;
     if (t > a.n_tiles) return;
     const uint64_t Dtot = a.E_old + a.n_ins;
@@ -886,9 +907,11 @@ __device__ __forceinline__ void mbar_wait(uint64_t* bar, uint32_t phase) {
 // columns pointing at deleted vertices: one ballot per 32 elements -> one mask
 // word (pure stores, every element's loads independent)
 __global__ void __launch_bounds__(kThreads) k_casc_cols(const uint32_t* __restrict__ old_cols, uint64_t E,
-        const uint32_t* __restrict__ hd_bits, const uint32_t* __restrict__ hd_rows, uint64_t n_hd,
+        const uint32_t* __restrict__ hd_bits, const uint32_t* __restrict__ hd_rows, const Counters* __restrict__ cn,
         uint32_t* __restrict__ mask) {
-    const uint32_t hd_lo = hd_rows[0], hd_hi = hd_rows[n_hd - 1];  // sorted: id range of deleted vertices
+    const uint64_t n_hd = cn->n_hd;
+    // sorted: id range of deleted vertices (empty range when there are none)
+    const uint32_t hd_lo = n_hd ? hd_rows[0] : 1u, hd_hi = n_hd ? hd_rows[n_hd - 1] : 0u;
     // 2 x 2048 elements per CTA; each lane owns 4 consecutive elements per step (128-bit
     // loads), a warp step covers 128 elements = 4 mask words; 16 columns in flight per lane
     constexpr int STEPS = 4;
@@ -931,7 +954,8 @@ __global__ void __launch_bounds__(kThreads) k_casc_cols(const uint32_t* __restri
 
 // rows of deleted vertices -> whole bit ranges (warp per row), OR-ed into the mask
 __global__ void k_casc_rows(const int64_t* __restrict__ old_off, const uint32_t* __restrict__ hd_rows,
-                            uint64_t n_hd, uint64_t row_lo, uint64_t row_hi, uint32_t* __restrict__ mask) {
+                            const Counters* __restrict__ cn, uint64_t row_lo, uint64_t row_hi, uint32_t* __restrict__ mask) {
+    const uint64_t n_hd = cn->n_hd;
     const uint64_t nw = ((uint64_t)gridDim.x * blockDim.x) >> 5;
     for (uint64_t h = (blockIdx.x * (uint64_t)blockDim.x + threadIdx.x) >> 5; h < n_hd; h += nw) {
         if (hd_rows[h] < row_lo || hd_rows[h] >= row_hi) continue;  // not a row of this shard
@@ -1013,7 +1037,16 @@ struct RowArgs {
     uint64_t row_lo_new;      // first new row of this shard (new_off is local)
     OwnRange own;
     const uint64_t* nv_ext;
+    const Counters* c;        // device-side list sizes (read by row_counts)
 };
+__device__ __forceinline__ RowArgs row_counts(RowArgs a) {
+    a.n_del = a.c->n_del;
+    a.n_ins = a.c->n_ins;
+    a.n_dropped = a.c->n_dropped;
+    a.n_vins = a.c->n_inserted;
+    a.row_lo_new = a.c->row_lo_new;
+    return a;
+}
 __device__ __forceinline__ uint64_t casc_before(const RowArgs& a, uint64_t x) {
     if (!a.casc_mask) return 0;
     if (x >= a.E_old) return a.casc_pre[(a.E_old + kCascBlock - 1) / kCascBlock];  // all cascaded
@@ -1022,7 +1055,8 @@ __device__ __forceinline__ uint64_t casc_before(const RowArgs& a, uint64_t x) {
            (r ? __popc(a.casc_mask[x >> 5] & (0xFFFFFFFFu >> (32 - r))) : 0u);
 }
 // CTA boundaries of k_offsets_rows: ranks of each CTA's first row in the two lists
-__global__ void k_rows_partition(RowArgs a) {
+__global__ void k_rows_partition(RowArgs a_) {
+    const RowArgs a = row_counts(a_);
     const uint64_t c = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x;
     const uint64_t ncta = (a.row_hi - a.row_lo + kRowTile - 1) / kRowTile;
     if (c > ncta) return;
@@ -1041,7 +1075,8 @@ __global__ void k_rows_partition(RowArgs a) {
     a.part[2 * c + 1] = ir;
 }
 
-__global__ void __launch_bounds__(kThreads) k_offsets_rows(RowArgs a) {
+__global__ void __launch_bounds__(kThreads) k_offsets_rows(RowArgs a_) {
+    const RowArgs a = row_counts(a_);
     const uint64_t k0 = a.row_lo + (uint64_t)blockIdx.x * kRowTile, k1 = min(k0 + kRowTile, a.row_hi);
     const uint64_t* pp = a.part + 2 * blockIdx.x;  // this CTA's slices of the delete / insert-row lists
     const uint64_t da = pp[0], ia = pp[1], db = pp[2], ib = pp[3];
@@ -1126,7 +1161,8 @@ __device__ __forceinline__ void cp_async_wait_all() { asm volatile("cp.async.wai
 // tile t+G's edit lists are loaded into registers; three barriers per tile
 // (deleted/insert-count masks are double-buffered).
 template <bool CASC, bool REMAP>
-__global__ void __launch_bounds__(kThreads) k_merge3(MergeArgs a, const TilePart* __restrict__ part) {
+__global__ void __launch_bounds__(kThreads) k_merge3(MergeArgs a_, const TilePart* __restrict__ part) {
+    const MergeArgs a = merge_counts(a_);
     constexpr int NCH = kMergeTile / 32;  // 64 chunks of 32 old elements
     extern __shared__ __align__(128) uint8_t dsm[];  // kMerge3Smem bytes
     auto s_col = reinterpret_cast<uint32_t(*)[kMergeBuf]>(dsm);
@@ -1360,9 +1396,9 @@ __global__ void __launch_bounds__(kThreads) k_merge3(MergeArgs a, const TilePart
 // Thread 0 also writes lohi = {lo, hi, shift}: below lo = min(first dropped id, first
 // insertion point) nothing moves; from hi = max(last dropped id + 1, last insertion
 // point) on, every id is shifted by n_ins - n_dropped.
-__global__ void k_remap_blocks(uint64_t V, const uint32_t* __restrict__ dropped, uint64_t n_dropped,
-                               const uint32_t* __restrict__ ins_oldpos, uint64_t n_ins, int32_t* __restrict__ shift,
-                               int32_t* __restrict__ lohi) {
+__global__ void k_remap_blocks(uint64_t V, const uint32_t* __restrict__ dropped, const uint32_t* __restrict__ ins_oldpos,
+                               Counters* __restrict__ c, int32_t* __restrict__ shift, int32_t* __restrict__ lohi) {
+    const uint64_t n_dropped = c->n_dropped, n_ins = c->n_inserted;
     uint64_t bk = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x;
     uint64_t nb = (V + (1u << kRemapBlockShift) - 1) >> kRemapBlockShift;
     if (bk == 0) {
@@ -1372,6 +1408,7 @@ __global__ void k_remap_blocks(uint64_t V, const uint32_t* __restrict__ dropped,
         lohi[0] = (int32_t)lo;
         lohi[1] = (int32_t)max(hi, lo);
         lohi[2] = (int32_t)((int64_t)n_ins - (int64_t)n_dropped);
+        c->Vn = V - n_dropped + n_ins;  // vertices of the new ID map
     }
     if (bk >= nb) return;
     uint64_t lo = bk << kRemapBlockShift, hi = min(lo + (1u << kRemapBlockShift), V);
@@ -1392,9 +1429,10 @@ __global__ void k_remap_blocks(uint64_t V, const uint32_t* __restrict__ dropped,
 // deg[u] = (#inserted records in row u) - (#deleted old edges in row u) is
 // scattered from the two sorted record lists, then one single-pass exclusive
 // scan (decoupled look-back) writes new_off[u] = old_off[u] + sum_{v<u} deg[v].
-__global__ void k_deg_scatter(const uint32_t* __restrict__ ins_row, uint64_t n_ins,
-                              const uint32_t* __restrict__ del_row, uint64_t n_del, int32_t* __restrict__ deg,
+__global__ void k_deg_scatter(const uint32_t* __restrict__ ins_row, const uint32_t* __restrict__ del_row,
+                              const Counters* __restrict__ c, int32_t* __restrict__ deg,
                               int64_t* __restrict__ tsum, uint64_t row_lo) {
+    const uint64_t n_ins = c->n_ins, n_del = c->n_del;
     uint64_t i = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x;
     const bool ok = i < n_ins + n_del;
     const bool is_ins = i < n_ins;
@@ -1520,9 +1558,10 @@ __global__ void __launch_bounds__(kThreads) k_offsets_scan(const int64_t* __rest
 // rows of inserted (new) vertices: kept old elements before the old position they
 // are inserted at, plus inserted records in rows < their new id
 __global__ void k_offsets_inserted(const NodeVtx* __restrict__ nv, const uint32_t* __restrict__ ins_q,
-                                   uint64_t n_vins, RowArgs a) {
+                                   RowArgs a_) {
+    const RowArgs a = row_counts(a_);
     uint64_t i = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x;
-    if (i >= n_vins) return;
+    if (i >= a.n_vins) return;
     if (!a.own.owns(a.nv_ext[ins_q[i]])) return;  // another shard's row
     const NodeVtx& r = nv[ins_q[i]];
     const uint64_t x = (uint64_t)a.old_off[r.oldpos];
@@ -1532,8 +1571,9 @@ __global__ void k_offsets_inserted(const NodeVtx* __restrict__ nv, const uint32_
 
 // per 32 old ids: {new id of the group's first id (as if it survived) | exact << 31,
 // dropped bitmask}; exact = an insertion point lies strictly inside the group
-__global__ void k_remap32(uint64_t V, const uint32_t* __restrict__ dropped, uint64_t n_dropped,
-                          const uint32_t* __restrict__ ins_oldpos, uint64_t n_vins, uint2* __restrict__ out) {
+__global__ void k_remap32(uint64_t V, const uint32_t* __restrict__ dropped, const uint32_t* __restrict__ ins_oldpos,
+                          const Counters* __restrict__ c, uint2* __restrict__ out) {
+    const uint64_t n_dropped = c->n_dropped, n_vins = c->n_inserted;
     const uint64_t g = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x;
     if (g >= (V + 31) / 32) return;
     const uint32_t c0 = (uint32_t)(g * 32);
@@ -1546,11 +1586,35 @@ __global__ void k_remap32(uint64_t V, const uint32_t* __restrict__ dropped, uint
 }
 
 __global__ void k_set_i64(int64_t* p, int64_t v) { *p = v; }
+// V == ~0: the vertex count of the new ID map is c->Vn (device-side)
 __global__ void k_row_range(const uint64_t* __restrict__ ext, uint64_t V, OwnRange own, Counters* c) {
+    if (V == ~0ull) V = c->Vn;
     c->row_lo_new = lower_bound_dev(ext, 0, V, own.lo);
     c->row_hi_new = own.hi == ~0ull ? V : lower_bound_dev(ext, 0, V, own.hi);
 }
 __global__ void k_copy_u64(unsigned long long* dst, const uint64_t* src) { *dst = *src; }
+
+// End of an apply (one thread): sizes of the new replica from the device counters,
+// the final row offset, and whether the new ID map is the identity 0..Vn-1 (ext ids
+// strictly increase, so the last one decides).  node_mode: the ID map was rebuilt.
+__global__ void k_finish(Counters* __restrict__ c, uint64_t V, uint64_t Vr, uint64_t E, int node_mode, int sharded,
+                         const uint64_t* __restrict__ new_ext, int64_t* __restrict__ new_off) {
+    const uint64_t Vn = node_mode ? (uint64_t)c->Vn : V;
+    const uint64_t Vr_new = !node_mode ? Vr : (sharded ? (uint64_t)(c->row_hi_new - c->row_lo_new) : Vn);
+    const uint64_t En = E + c->n_ins - c->n_del - c->n_casc;
+    c->Vn = Vn;
+    c->Vr_new = Vr_new;
+    c->En = En;
+    c->new_identity = node_mode ? (Vn == 0 || new_ext[Vn - 1] == Vn - 1) : 2;  // 2: unchanged
+    if (new_off) new_off[Vr_new] = (int64_t)En;
+}
+
+// fence of the new ID map (its size is a device count)
+__global__ void k_build_fence_dev(const uint64_t* __restrict__ ext, const Counters* __restrict__ c,
+                                  uint64_t* __restrict__ fence) {
+    uint64_t i = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x;
+    if ((i << kFenceShift) < c->Vn) fence[i] = ext[i << kFenceShift];
+}
 
 // ================================================================ checks ====
 template <typename T>

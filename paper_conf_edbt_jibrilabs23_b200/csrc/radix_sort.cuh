@@ -19,9 +19,17 @@ constexpr int kRsTile = kRsThreads * kRsItems;  // 3072 keys per tile
 constexpr int kRsWarps = kRsThreads / 32;
 constexpr int kRsMaxPasses = 8;
 
+// n_dev (nullable): the key count lives in device memory (no host sync before the
+// sort); `n` is then an upper bound that only sizes the grids
+__device__ __forceinline__ uint64_t rs_count(uint64_t n, const unsigned long long* n_dev) {
+    return n_dev ? min(n, (uint64_t)*n_dev) : n;
+}
+
 __global__ void __launch_bounds__(256) rs_histogram(const uint64_t* __restrict__ keys, uint64_t n,
+                                                    const unsigned long long* __restrict__ n_dev,
                                                     int passes, uint32_t* __restrict__ hist) {
     __shared__ uint32_t s[kRsMaxPasses][256];
+    n = rs_count(n, n_dev);
     for (int i = threadIdx.x; i < kRsMaxPasses * 256; i += blockDim.x) (&s[0][0])[i] = 0;
     __syncthreads();
     for (uint64_t i = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; i < n;
@@ -48,8 +56,9 @@ __global__ void __launch_bounds__(256) rs_digit_base(const uint32_t* __restrict_
 
 __global__ void __launch_bounds__(kRsThreads) rs_onesweep(
     const uint64_t* __restrict__ kin, const uint32_t* __restrict__ vin, uint64_t* __restrict__ kout,
-    uint32_t* __restrict__ vout, uint64_t n, int shift, const uint64_t* __restrict__ digit_base,
-    uint64_t* __restrict__ status /* [ntiles][256] */, uint32_t* __restrict__ tile_ctr) {
+    uint32_t* __restrict__ vout, uint64_t n, const unsigned long long* __restrict__ n_dev, int shift,
+    const uint64_t* __restrict__ digit_base, uint64_t* __restrict__ status /* [ntiles][256] */,
+    uint32_t* __restrict__ tile_ctr) {
     __shared__ uint32_t s_tile;
     __shared__ uint32_t s_wcnt[kRsWarps][256];
     __shared__ uint32_t s_dstart[256];
@@ -59,11 +68,13 @@ __global__ void __launch_bounds__(kRsThreads) rs_onesweep(
     __shared__ uint32_t s_scan[kRsThreads / 32 + 1];
 
     const int tid = threadIdx.x, w = tid >> 5, l = lane_id();
+    n = rs_count(n, n_dev);
     if (tid == 0) s_tile = atomicAdd(tile_ctr, 1u);
     for (int i = tid; i < kRsWarps * 256; i += kRsThreads) (&s_wcnt[0][0])[i] = 0;
     __syncthreads();
     const uint32_t tile = s_tile;
     const uint64_t base = (uint64_t)tile * kRsTile;
+    if (base >= n) return;  // grid sized by an upper bound: no later tile depends on this one
     const uint64_t tile_n = (n - base < (uint64_t)kRsTile) ? (n - base) : (uint64_t)kRsTile;
 
     uint64_t k[kRsItems];

@@ -6,15 +6,14 @@ for l in sys.stdin:
     l=l.strip()
     if not l.startswith("{"): continue
     d=json.loads(l); r=d["roofline"]; p=d["path"]
-    print(d["config"]["name"], "value=%.4g"%d["value"], "ms/step=%.3f"%d["ms_per_step"], "merge=%.3fms %.0fGB/s frac=%.3f"%(r["ms_per_launch"], r["achieved"], r["frac"]), "path_frac=%.3f"%p["frac_of_peak"], {k:round(v,3) for k,v in p["phase_ms"].items()}, "e2e=%.4g"%d["e2e"]["value"])'
-timeout 300 python -m pytest tests -m gpu -q -x 2>&1 | tail -1 > gpurun_out/pytest_gpu.txt
+    print(d["config"]["name"], "value=%.4g"%d["value"], "ms/step=%.3f"%d["ms_per_step"], "merge=%.3fms %.0fGB/s frac=%.3f"%(r["ms_per_launch"], r["achieved"], r["frac"]), "path_frac=%.3f"%p["frac_of_peak"], {k:round(v,3) for k,v in p["phase_ms"].items()}, "e2e=%.4g"%d["e2e"]["value"], "launches=%d"%d["gpu_launches"])'
+timeout 600 python -m pytest tests -m gpu -q -x 2>&1 | tail -15 > gpurun_out/pytest_gpu.txt
 for c in ${CONFIGS:-c2 c3}; do
   timeout 600 python bench.py --config $c --steps 10 --warmup 3 --no-cpu-baseline 2>&1 | python -c "$summ"
 done
-if [ -n "$NCU" ]; then
+if [ -n "$TRACE" ]; then
   for c in ${CONFIGS:-c2 c3}; do
-    timeout 900 ncu --metrics gpu__time_duration.sum --clock-control none --cache-control none --csv --log-file gpurun_out/launches_$c.csv \
-      python bench.py --config $c --steps 2 --warmup 3 --no-cpu-baseline > /dev/null 2>&1
+    H2TAP_TRACE=1 timeout 300 python tools_trace.py $c 2>&1 | grep "h2tap trace" | tail -3 > gpurun_out/trace_$c.txt
   done
 fi
 cat gpurun_out/pytest_gpu.txt

@@ -202,8 +202,9 @@ void radix_sort(h2tap_replica* r, uint64_t*& k, uint32_t*& v, uint64_t*& k2, uin
     CKL();
     rs_digit_base<<<passes, 256, 0, r->st>>>(hist, dbase);
     CKL();
+    CK(cudaFuncSetAttribute(rs_onesweep, cudaFuncAttributeMaxDynamicSharedMemorySize, kRsSmem));  // per device
     for (int p = 0; p < passes; ++p) {
-        rs_onesweep<<<(unsigned)ntiles, kRsThreads, 0, r->st>>>(k, v, k2, v2, n, n_dev, 8 * p, dbase + p * 256,
+        rs_onesweep<<<(unsigned)ntiles, kRsThreads, kRsSmem, r->st>>>(k, v, k2, v2, n, n_dev, 8 * p, dbase + p * 256,
                                                               st + (uint64_t)p * ntiles * 256, ctr + p);
         CKL();
         std::swap(k, k2);
@@ -391,43 +392,42 @@ h2tap_status apply_core(h2tap_replica* r, const BatchIn& in, uint64_t S, bool cr
 
         nv = r->get<NodeVtx>(r->nv, n_node);
         nv_ext = r->get<uint64_t>(r->nv_ext, n_node);
-        const uint64_t nt = cdiv(n_node, kTile);  // also the tile bound of the unique-vertex list
-        uint64_t* stt = r->get<uint64_t>(r->status, 4 * nt);
-        CK(cudaMemsetAsync(stt, 0, 4 * nt * 8, st));
-        k_node_segments<<<(unsigned)nt, kThreads, 0, st>>>(ops, node_sorted, n_node, ext_index(r), nv, nv_ext,
-                                                           stt, nt, dc);
+        const uint64_t nt = cdiv(n_node, kTile);  // tile bound of the unique-vertex list
+        const uint64_t nts = cdiv(n_node, kSegTile);
+        uint64_t* stt = r->get<uint64_t>(r->status, 3 * nt + nts);
+        CK(cudaMemsetAsync(stt, 0, (3 * nt + nts) * 8, st));
+        k_node_segments<<<(unsigned)nts, kThreads, 0, st>>>(ops, node_sorted, n_node, ext_index(r), nv, nv_ext,
+                                                            stt + 3 * nt, nts, dc);
         CKL();
         TR("node_segments");
         dropped = r->get<uint32_t>(r->dropped, n_node);
         ins_q = r->get<uint32_t>(r->ins_q, n_node);
         ins_oldpos = r->get<uint32_t>(r->ins_oldpos, n_node);
         hd_rows = r->get<uint32_t>(r->hd_rows, n_node);
-        k_node_lists<<<(unsigned)nt, kThreads, 0, st>>>(nv, dropped, ins_q, ins_oldpos, hd_rows, stt + nt, nt, dc);
+        k_node_lists<<<(unsigned)nt, kThreads, 0, st>>>(nv, dropped, ins_q, ins_oldpos, hd_rows, stt, nt, dc);
         CKL();
         TR("node_lists");
         // ID-map compaction: remap tables (64K-id block shifts, 32-id groups, the
         // unchanged / uniformly shifted id ranges), then the survivors and the inserted
         new_ext = r->get<uint64_t>(r->ext[ec ^ 1], Vn_ub);
         const uint64_t nblk = cdiv(V, 1ull << kRemapBlockShift), ng = cdiv(V, 32);
-        int32_t* rs = r->get<int32_t>(r->remap_shift, nblk + 4);  // + {lo, hi, shift}
+        int32_t* rs = r->get<int32_t>(r->remap_shift, nblk + 8);  // + lohi (6 entries)
         uint2* r32 = r->get<uint2>(r->remap32, ng);
         k_remap_blocks<<<g1(nblk), 256, 0, st>>>(V, dropped, ins_oldpos, dc, rs, rs + nblk);  // also writes c->Vn
         CKL();
         if (ng) { k_remap32<<<g1(ng), 256, 0, st>>>(V, dropped, ins_oldpos, dc, r32); CKL(); }
         R.shift = rs; R.g32 = r32; R.ins_oldpos = ins_oldpos; R.n_vins = &dc->n_inserted; R.lohi = rs + nblk;
         TR("remap_tables");
-        if (V) { k_new_ext<<<g1(V), 256, 0, st>>>(old_ext, r->identity, V, R, new_ext); CKL(); }
-        TR("new_ext");
+        // the inserted vertices' ID-map entries now; the survivors' entries are written
+        // by k_rows_fused together with the new row offsets
         k_place_inserted<<<g1(n_node), 256, 0, st>>>(nv, nv_ext, ins_q, ins_oldpos, dropped, dc, new_ext);
         CKL();
-        {
-            uint64_t* f = r->get<uint64_t>(r->fence[ec ^ 1], n_fence(Vn_ub));
-            k_build_fence_dev<<<g1(n_fence(Vn_ub)), 256, 0, st>>>(new_ext, dc, f);
-            CKL();
-        }
         k_nv_newid<<<g1(n_node), 256, 0, st>>>(nv, dc, R);
         CKL();
-        if (r->sharded) { k_row_range<<<1, 1, 0, st>>>(new_ext, ~0ull, r->own, dc); CKL(); }
+        if (r->sharded) {
+            k_row_range_new<<<1, 1, 0, st>>>(dropped, ins_q, nv_ext, row_lo, row_lo + Vr, r->own, dc);
+            CKL();
+        }
         // cascade pass (a4, reading A8): one bit per old element removed by a node delete
         hd_bits = r->get<uint32_t>(r->hd_bits, cdiv(V, 32));
         CK(cudaMemsetAsync(hd_bits, 0, cdiv(V, 32) * 4, st));
@@ -443,7 +443,8 @@ h2tap_status apply_core(h2tap_replica* r, const BatchIn& in, uint64_t S, bool cr
         CK(cudaMemsetAsync(st2s2, 0, nst * 8, st));
         TR("nv_newid+bits");
         if (nblk_c) {
-            k_casc_cols<<<(unsigned)cdiv(nblk_c, 2), kThreads, 0, st>>>(old_cols_nc, E, hd_bits, hd_rows, dc, casc_mask);
+            const unsigned gc = (unsigned)std::min<uint64_t>(cdiv(nblk_c, 2), (uint64_t)r->n_sm * 6);
+            k_casc_cols<<<gc, kThreads, 0, st>>>(old_cols_nc, E, hd_bits, hd_rows, dc, casc_mask);
             CKL();
             TR("casc_cols");
             k_casc_rows<<<rg, 256, 0, st>>>(old_off_nc, hd_rows, dc, row_lo, row_lo + Vr, casc_mask);
@@ -515,6 +516,7 @@ h2tap_status apply_core(h2tap_replica* r, const BatchIn& in, uint64_t S, bool cr
         ca.old_off = old_off - row_lo;  // indexed by global dense ids of owned rows
         ca.old_cols = old_cols;
         ca.V_old = V;
+        ca.direct = node_mode ? 0 : 1;  // identity remap: the key's row is the old row
         ca.ins_pos = ins_pos; ca.ins_row = ins_row; ca.ins_col = ins_col; ca.ins_w = ins_w;
         ca.del_pos = del_pos;
         ca.del_row = del_row;
@@ -606,15 +608,19 @@ h2tap_status apply_core(h2tap_replica* r, const BatchIn& in, uint64_t S, bool cr
         ra.dropped = dropped; ra.ins_oldpos = ins_oldpos;
         ra.new_off = new_off;
         ra.c = dc;
-        const uint64_t ncta = cdiv(Vr, kRowTile);
+        ra.old_ext = old_ext; ra.new_ext = new_ext; ra.identity = r->identity ? 1 : 0;
+        const uint64_t ncta = cdiv(V, kRowTile);
         ra.part = r->get<uint64_t>(r->opart, 2 * (ncta + 1));
-        if (Vr) {
+        if (V) {
             k_rows_partition<<<g1(ncta + 1), 256, 0, st>>>(ra);
             CKL();
-            k_offsets_rows<<<(unsigned)ncta, kThreads, 0, st>>>(ra);
+            k_rows_fused<<<(unsigned)ncta, kThreads, 0, st>>>(ra);  // survivors: ID map + row offsets
             CKL();
         }
         k_offsets_inserted<<<g1(n_node), 256, 0, st>>>(nv, ins_q, ra);
+        CKL();
+        uint64_t* f = r->get<uint64_t>(r->fence[ec ^ 1], n_fence(Vn_ub));
+        k_build_fence_dev<<<g1(n_fence(Vn_ub)), 256, 0, st>>>(new_ext, dc, f);
         CKL();
     }
     } else {

@@ -73,7 +73,8 @@ struct RemapView {
     const uint2* g32;
     const uint32_t* ins_oldpos;
     const unsigned long long* n_vins;  // device count of inserted vertices
-    const int32_t* lohi;   // {lo, hi, shift}: ids < lo unchanged, ids >= hi shifted by `shift`
+    const int32_t* lohi;   // {lo, hi, shift, mlo, mhi, msh}: ids < lo unchanged, ids >= hi shifted by
+                           // `shift`, ids in [mlo, mhi) shifted by `msh`
 };
 __device__ __forceinline__ uint32_t remap_of(const RemapView& R, uint32_t k) {
     if (!R.shift) return k;
@@ -299,36 +300,25 @@ __global__ void k_unpack_recs(const RouteRec* __restrict__ recs, uint64_t n, uin
 // ===================================================================== a2 ====
 // Unique vertices of the (v, ts, seq)-sorted visible node ops: final liveness
 // (last op), latest delete point tD, old presence.  Compaction via look-back.
+// One op per thread: a segment head walks its segment and then searches the old
+// ID map (a chain of dependent loads), so heads must not queue behind each other.
+constexpr int kSegTile = kThreads;
 __global__ void __launch_bounds__(kThreads) k_node_segments(
     Ops ops, const uint32_t* __restrict__ sidx, uint64_t n, ExtIndex X, NodeVtx* __restrict__ nv,
     uint64_t* __restrict__ nv_ext, uint64_t* __restrict__ status, uint64_t n_tiles, Counters* __restrict__ c) {
     __shared__ uint32_t s_tile;
-    __shared__ uint32_t s_cmp[kItems * kThreads / 32 + 1];
+    __shared__ uint32_t s_cmp[kThreads / 32 + 1];
     __shared__ uint64_t s_base;
     if (threadIdx.x == 0) s_tile = atomicAdd(&c->tiles[1], 1u);
     __syncthreads();
     const uint32_t tile = s_tile;
-    const uint64_t i0 = (uint64_t)tile * kTile + threadIdx.x;
-    bool head[kItems];
-    uint32_t pos[kItems];
-#pragma unroll
-    for (int j = 0; j < kItems; ++j) {
-        uint64_t i = i0 + (uint64_t)j * kThreads;
-        head[j] = i < n && (i == 0 || ops.src[sidx[i]] != ops.src[sidx[i - 1]]);
-    }
-    uint32_t tot = striped_compact<kThreads, kItems>(head, pos, s_cmp);
-    if (threadIdx.x < 32) {
-        uint64_t b = lookback_warp(status, tile, tot);
-        if (lane_id() == 0) { s_base = b; if (tile == n_tiles - 1) c->n_unique = b + tot; }
-    }
-    __syncthreads();
-#pragma unroll
-    for (int j = 0; j < kItems; ++j) {
-        if (!head[j]) continue;
-        uint64_t i = i0 + (uint64_t)j * kThreads;
-        uint64_t v = ops.src[sidx[i]];
+    const uint64_t i = (uint64_t)tile * kSegTile + threadIdx.x;
+    const uint64_t v = i < n ? ops.src[sidx[i]] : 0;
+    bool head[1] = {i < n && (i == 0 || v != ops.src[sidx[i - 1]])};
+    // head work before the compaction so its loads overlap the look-back
+    NodeVtx r{};
+    if (head[0]) {
         uint64_t e = i;
-        NodeVtx r;
         r.flags = 0; r.tD_ts = 0; r.tD_seq = 0;
         uint8_t last = NODE_INSERT;
         while (e < n && ops.src[sidx[e]] == v) {
@@ -346,7 +336,16 @@ __global__ void __launch_bounds__(kThreads) k_node_segments(
         r.end = (uint32_t)e;
         r.newid = kNone32;
         r.pad = 0;
-        uint64_t q = s_base + pos[j];
+    }
+    uint32_t pos[1];
+    uint32_t tot = striped_compact<kThreads, 1>(head, pos, s_cmp);
+    if (threadIdx.x < 32) {
+        uint64_t b = lookback_warp(status, tile, tot);
+        if (lane_id() == 0) { s_base = b; if (tile == n_tiles - 1) c->n_unique = b + tot; }
+    }
+    __syncthreads();
+    if (head[0]) {
+        uint64_t q = s_base + pos[0];
         nv[q] = r;
         nv_ext[q] = v;
     }
@@ -419,15 +418,6 @@ __device__ __forceinline__ uint64_t gallop_ub(const T* a, uint64_t lo, uint64_t 
     while (p < hi && !(key < a[p])) { lo = p + 1; p = lo + step; step <<= 1; }
     if (p > hi) p = hi;
     return upper_bound_dev(a, lo, p, key);
-}
-
-// new ID map, survivors: new_ext[remap(k)] = ext[k] (thread per old vertex)
-__global__ void k_new_ext(const uint64_t* __restrict__ old_ext, int identity, uint64_t V, RemapView R,
-                          uint64_t* __restrict__ new_ext) {
-    const uint64_t k = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x;
-    if (k >= V) return;
-    const uint32_t u = remap_of(R, (uint32_t)k);
-    if (u != kNone32) new_ext[u] = identity ? k : old_ext[k];
 }
 
 // inserted vertex i lands at oldpos_i - (#dropped before oldpos_i) + i
@@ -641,6 +631,7 @@ struct ClassArgs {
     const int64_t* old_off;
     const uint32_t* old_cols;
     uint64_t V_old;
+    int direct;                // identity ID map, no node ops: key row == old row
     uint64_t* ins_pos;
     uint32_t* ins_row;
     uint32_t* ins_col;
@@ -654,7 +645,7 @@ struct ClassArgs {
     Counters* c;
 };
 
-constexpr int kCItems = 4;                    // classify: items per thread (register budget)
+constexpr int kCItems = 2;                    // classify: items per thread (occupancy over ILP)
 constexpr int kCTile = kThreads * kCItems;
 __global__ void __launch_bounds__(kThreads) k_reduce_classify(ClassArgs a) {
     __shared__ uint32_t s_tile;
@@ -667,56 +658,72 @@ __global__ void __launch_bounds__(kThreads) k_reduce_classify(ClassArgs a) {
     const uint64_t n_tiles = (n + kCTile - 1) / kCTile;
     if (tile >= n_tiles) return;
     const uint64_t i0 = (uint64_t)tile * kCTile + threadIdx.x;
+    // Identity ID map (no node ops): the key's row IS the old row, so its bounds are
+    // fetched together with the key, off the record-gather chain.
+    const bool direct = a.direct;
+    uint64_t key[kCItems], lo[kCItems], hi[kCItems];
+    uint32_t rec_i[kCItems];
+    bool head[kCItems];
+#pragma unroll
+    for (int j = 0; j < kCItems; ++j) {
+        const uint64_t i = i0 + (uint64_t)j * kThreads;
+        key[j] = i < n ? a.keys[i] : 0;
+        head[j] = i < n && (i == 0 || a.keys[i - 1] != key[j]);
+        rec_i[j] = head[j] ? a.vals[i] : 0u;
+        lo[j] = hi[j] = 0;
+        if (direct && head[j]) {
+            const uint64_t u = key[j] >> a.bits;
+            lo[j] = (uint64_t)a.old_off[u];
+            hi[j] = (uint64_t)a.old_off[u + 1];
+        }
+    }
+    // segmented arg-max over (ts, seq): the first record of every segment is gathered
+    // for all items at once; longer segments (repeated keys) continue serially
+    EdgeRec r0[kCItems];
+#pragma unroll
+    for (int j = 0; j < kCItems; ++j)
+        if (head[j]) r0[j] = a.recs[rec_i[j]];
     uint8_t cat[kCItems], meta[kCItems];
-    uint64_t pos[kCItems], lo[kCItems], hi[kCItems], end[kCItems];
     uint32_t colq[kCItems];
     float wv[kCItems];
 #pragma unroll
     for (int j = 0; j < kCItems; ++j) {
-        cat[j] = 0;
-        pos[j] = 0;
-        wv[j] = 0.f;
-        lo[j] = hi[j] = end[j] = 0;
-        colq[j] = 0;
-        meta[j] = 0;
-        uint64_t i = i0 + (uint64_t)j * kThreads;
-        if (i >= n) continue;
-        uint64_t key = a.keys[i];
-        if (i > 0 && a.keys[i - 1] == key) continue;
-        // segment [i, e): latest-commit-wins over (ts, seq)
+        cat[j] = 0; meta[j] = 0; colq[j] = 0; wv[j] = 0.f;
+        if (!head[j]) continue;
         uint64_t nw_ts = 0, nw_seq = 0, w_ts = 0, w_seq = 0;
         bool has_nw = false, has_w = false;
         uint8_t nw_kind = 0;
         float w_val = 0.f;
-        EdgeRec r0;
-        for (uint64_t e = i; e < n && a.keys[e] == key; ++e) {
-            const EdgeRec re = a.recs[a.vals[e]];
-            if (e == i) r0 = re;
-            uint8_t k = re.kind;
-            uint64_t ts = re.ts, sq = re.seq;
+        EdgeRec re = r0[j];
+        for (uint64_t e = i0 + (uint64_t)j * kThreads;;) {
+            const uint8_t k = re.kind;
             if (k == EDGE_INSERT || k == EDGE_DELETE) {
-                if (!has_nw || pt_less(nw_ts, nw_seq, ts, sq)) { has_nw = true; nw_ts = ts; nw_seq = sq; nw_kind = k; }
+                if (!has_nw || pt_less(nw_ts, nw_seq, re.ts, re.seq)) { has_nw = true; nw_ts = re.ts; nw_seq = re.seq; nw_kind = k; }
             }
             if (k == EDGE_INSERT || k == EDGE_WEIGHT) {
-                if (!has_w || pt_less(w_ts, w_seq, ts, sq)) { has_w = true; w_ts = ts; w_seq = sq; w_val = re.w; }
+                if (!has_w || pt_less(w_ts, w_seq, re.ts, re.seq)) { has_w = true; w_ts = re.ts; w_seq = re.seq; w_val = re.w; }
             }
+            if (++e >= n || a.keys[e] != key[j]) break;
+            re = a.recs[a.vals[e]];
         }
-        uint8_t fl = r0.flags;
-        bool u_old = fl & 1;
-        uint32_t ou = r0.opos_u, ow = r0.opos_w;
+        const uint8_t fl = r0[j].flags;
         // outcome category before the old-row lookup: 1 insert-like, 2 delete, 3 weight-only
         cat[j] = (has_nw && nw_kind == EDGE_INSERT) ? 1 : (has_nw ? 2 : (has_w ? 3 : 0));
         meta[j] = fl;
-        colq[j] = ow;
+        colq[j] = r0[j].opos_w;
         wv[j] = w_val;
-        if (u_old) { lo[j] = (uint64_t)a.old_off[ou]; hi[j] = (uint64_t)a.old_off[ou + 1]; }
-        else { lo[j] = hi[j] = (uint64_t)a.old_off[ou]; }
-        end[j] = hi[j];
+        if (!direct) {
+            const uint32_t ou = r0[j].opos_u;
+            if (fl & 1) { lo[j] = (uint64_t)a.old_off[ou]; hi[j] = (uint64_t)a.old_off[ou + 1]; }
+            else { lo[j] = hi[j] = (uint64_t)a.old_off[ou]; }
+        }
     }
-    // lock-step searches of every item's column in its old row: up to kCItems
-    // independent loads in flight per thread.  The first probes interpolate
-    // between the known value bounds (columns of a row spread over [0, V)),
-    // then plain bisection; cuts DRAM probes per lookup from ~log2(deg) to ~3.
+    uint64_t end[kCItems];
+#pragma unroll
+    for (int j = 0; j < kCItems; ++j) end[j] = hi[j];
+    // lock-step searches of every item's column in its old row.  The first probes
+    // interpolate between the known value bounds (columns of a row spread over
+    // [0, V)), then plain bisection; cuts DRAM probes per lookup to ~2-3.
     uint32_t vlo[kCItems], vhi[kCItems];
 #pragma unroll
     for (int j = 0; j < kCItems; ++j) { vlo[j] = 0; vhi[j] = (uint32_t)a.V_old; }
@@ -740,33 +747,34 @@ __global__ void __launch_bounds__(kThreads) k_reduce_classify(ClassArgs a) {
         }
         if (!any) break;
     }
+    bool f0[kCItems], f1[kCItems], f2[kCItems];
 #pragma unroll
     for (int j = 0; j < kCItems; ++j) {
-        if (!cat[j]) continue;
-        const uint64_t p = lo[j];
-        const bool found = (meta[j] & 1) && (meta[j] & 2) && p < end[j] && a.old_cols[p] == colq[j];
-        const bool present = found && !(meta[j] & 4);  // a node delete of an endpoint cleared the old edge
         uint8_t ct = 0;
-        if (cat[j] == 1) ct = present ? 3 : 1;
-        else if (cat[j] == 2) ct = present ? 2 : 0;
-        else ct = present ? 3 : 0;
+        if (cat[j]) {
+            const uint64_t p = lo[j];
+            const bool found = (meta[j] & 1) && (meta[j] & 2) && p < end[j] && a.old_cols[p] == colq[j];
+            const bool present = found && !(meta[j] & 4);  // a node delete of an endpoint cleared the old edge
+            if (cat[j] == 1) ct = present ? 3 : 1;
+            else if (cat[j] == 2) ct = present ? 2 : 0;
+            else ct = present ? 3 : 0;
+        }
         cat[j] = ct;
-        pos[j] = p;
+        f0[j] = ct == 1; f1[j] = ct == 2; f2[j] = ct == 3;
     }
-    bool f[3][kCItems];
-    uint32_t rk[3][kCItems], tot[3];
-#pragma unroll
-    for (int j = 0; j < kCItems; ++j) { f[0][j] = cat[j] == 1; f[1][j] = cat[j] == 2; f[2][j] = cat[j] == 3; }
-#pragma unroll
-    for (int q = 0; q < 3; ++q) tot[q] = striped_compact<kThreads, kCItems>(f[q], rk[q], s_cmp[q]);
+    uint32_t rk0[kCItems], rk1[kCItems], rk2[kCItems];
+    const uint32_t t0 = striped_compact<kThreads, kCItems>(f0, rk0, s_cmp[0]);
+    const uint32_t t1 = striped_compact<kThreads, kCItems>(f1, rk1, s_cmp[1]);
+    const uint32_t t2 = striped_compact<kThreads, kCItems>(f2, rk2, s_cmp[2]);
     const int wid = threadIdx.x >> 5;
     if (wid < 3) {
-        uint64_t b = lookback_warp(a.status3 + (uint64_t)wid * a.n_tiles, tile, tot[wid]);
+        const uint32_t tw = wid == 0 ? t0 : (wid == 1 ? t1 : t2);
+        uint64_t b = lookback_warp(a.status3 + (uint64_t)wid * a.n_tiles, tile, tw);
         if (lane_id() == 0) {
             s_base[wid] = b;
             if (tile == n_tiles - 1) {
                 unsigned long long* d = wid == 0 ? &a.c->n_ins : (wid == 1 ? &a.c->n_del : &a.c->n_upd);
-                *d = b + tot[wid];
+                *d = b + tw;
             }
         }
     }
@@ -775,19 +783,18 @@ __global__ void __launch_bounds__(kThreads) k_reduce_classify(ClassArgs a) {
 #pragma unroll
     for (int j = 0; j < kCItems; ++j) {
         if (cat[j] == 1) {
-            uint64_t key = a.keys[i0 + (uint64_t)j * kThreads];
-            uint64_t oi = s_base[0] + rk[0][j];
-            a.ins_pos[oi] = pos[j];
-            a.ins_row[oi] = (uint32_t)(key >> a.bits);
-            a.ins_col[oi] = (uint32_t)(key & mask);
+            const uint64_t oi = s_base[0] + rk0[j];
+            a.ins_pos[oi] = lo[j];
+            a.ins_row[oi] = (uint32_t)(key[j] >> a.bits);
+            a.ins_col[oi] = (uint32_t)(key[j] & mask);
             a.ins_w[oi] = wv[j];
         } else if (cat[j] == 2) {
-            uint64_t od = s_base[1] + rk[1][j];
-            a.del_pos[od] = pos[j];
-            a.del_row[od] = (uint32_t)(a.keys[i0 + (uint64_t)j * kThreads] >> a.bits);
+            const uint64_t od = s_base[1] + rk1[j];
+            a.del_pos[od] = lo[j];
+            a.del_row[od] = (uint32_t)(key[j] >> a.bits);
         } else if (cat[j] == 3) {
-            uint64_t ou = s_base[2] + rk[2][j];
-            a.upd_pos[ou] = pos[j];
+            const uint64_t ou = s_base[2] + rk2[j];
+            a.upd_pos[ou] = lo[j];
             a.upd_w[ou] = wv[j];
         }
     }
@@ -904,51 +911,62 @@ __device__ __forceinline__ void mbar_wait(uint64_t* bar, uint32_t phase) {
 // plus per-2048-element block counts.  Runs on a side stream, overlapped with the
 // edge-op sort/classify phase, so the merge never touches the cascade bitmap.
 
-// columns pointing at deleted vertices: one ballot per 32 elements -> one mask
-// word (pure stores, every element's loads independent)
+// columns pointing at deleted vertices -> mask words (pure stores, every element's
+// loads independent).  Persistent: each CTA strides over 4096-element blocks, so the
+// prologue (device count + id range of the deleted vertices) is paid once per CTA.
 __global__ void __launch_bounds__(kThreads) k_casc_cols(const uint32_t* __restrict__ old_cols, uint64_t E,
         const uint32_t* __restrict__ hd_bits, const uint32_t* __restrict__ hd_rows, const Counters* __restrict__ cn,
         uint32_t* __restrict__ mask) {
     const uint64_t n_hd = cn->n_hd;
-    // sorted: id range of deleted vertices (empty range when there are none)
-    const uint32_t hd_lo = n_hd ? hd_rows[0] : 1u, hd_hi = n_hd ? hd_rows[n_hd - 1] : 0u;
-    // 2 x 2048 elements per CTA; each lane owns 4 consecutive elements per step (128-bit
-    // loads), a warp step covers 128 elements = 4 mask words; 16 columns in flight per lane
+    // sorted: id range [hd_lo, hd_lo + span] of deleted vertices (none: empty range)
+    const uint32_t hd_lo = n_hd ? hd_rows[0] : 1u;
+    const uint32_t span = n_hd ? hd_rows[n_hd - 1] - hd_lo : 0u;
+    const bool none = n_hd == 0;
+    // each lane owns 4 consecutive elements per step (128-bit loads), a warp step covers
+    // 128 elements = 4 mask words; 16 columns in flight per lane
     constexpr int STEPS = 4;
-    const uint64_t b0 = (uint64_t)blockIdx.x * (2 * kCascBlock);
+    constexpr uint64_t BLK = 2 * kCascBlock;
     const int w = threadIdx.x >> 5;
-    uint4 c[STEPS];
+    const uint64_t nb = (E + BLK - 1) / BLK;
+    const uint64_t wend = ((E + 31) & ~31ull) + 2 * kCascBlock;  // mask words past E are written as 0
+    for (uint64_t blk = blockIdx.x; blk < nb; blk += gridDim.x) {
+        const uint64_t b0 = blk * BLK;
+        const bool full = b0 + BLK <= E;
+        uint4 c[STEPS];
 #pragma unroll
-    for (int j = 0; j < STEPS; ++j) {
-        const uint64_t x = b0 + ((uint64_t)(j * (kThreads / 32) + w) * 128) + lane_id() * 4;
-        c[j] = (x + 3 < E) ? __ldcs(reinterpret_cast<const uint4*>(old_cols + x))
-                           : make_uint4(x < E ? old_cols[x] : 0u, x + 1 < E ? old_cols[x + 1] : 0u,
-                                        x + 2 < E ? old_cols[x + 2] : 0u, 0u);
-    }
-    uint32_t bits[STEPS];
-#pragma unroll
-    for (int j = 0; j < STEPS; ++j) {
-        const uint64_t x = b0 + ((uint64_t)(j * (kThreads / 32) + w) * 128) + lane_id() * 4;
-        const uint32_t v[4] = {c[j].x, c[j].y, c[j].z, c[j].w};
-        uint32_t m = 0;
-#pragma unroll
-        for (int e = 0; e < 4; ++e) {
-            const bool in = x + e < E && v[e] >= hd_lo && v[e] <= hd_hi && (hd_bits[v[e] >> 5] >> (v[e] & 31) & 1);
-            m |= (uint32_t)in << e;
+        for (int j = 0; j < STEPS; ++j) {
+            const uint64_t x = b0 + ((uint64_t)(j * (kThreads / 32) + w) * 128) + lane_id() * 4;
+            if (none) c[j] = make_uint4(0u, 0u, 0u, 0u);
+            else if (full || x + 3 < E) c[j] = __ldcs(reinterpret_cast<const uint4*>(old_cols + x));
+            else c[j] = make_uint4(x < E ? old_cols[x] : 0u, x + 1 < E ? old_cols[x + 1] : 0u,
+                                   x + 2 < E ? old_cols[x + 2] : 0u, 0u);
         }
-        bits[j] = m;  // 4 bits for this lane's elements
-    }
+        uint32_t bits[STEPS];
 #pragma unroll
-    for (int j = 0; j < STEPS; ++j) {
-        // lane L holds bits of elements 4L..4L+3 of the 128-element step: word q = L / 8
-        const uint32_t nib = bits[j] << ((lane_id() & 7) * 4);
-        uint32_t word = nib;
-        word |= __shfl_xor_sync(0xffffffffu, word, 1);
-        word |= __shfl_xor_sync(0xffffffffu, word, 2);
-        word |= __shfl_xor_sync(0xffffffffu, word, 4);
-        const uint64_t x = b0 + ((uint64_t)(j * (kThreads / 32) + w) * 128);
-        if ((lane_id() & 7) == 0 && x + lane_id() * 4 < ((E + 31) & ~31ull) + 2 * kCascBlock)
-            mask[(x >> 5) + lane_id() / 8] = word;  // words past E are written as 0
+        for (int j = 0; j < STEPS; ++j) {
+            const uint32_t v[4] = {c[j].x, c[j].y, c[j].z, c[j].w};
+            uint32_t m = 0;
+#pragma unroll
+            for (int e = 0; e < 4; ++e) {
+                const uint32_t d = v[e] - hd_lo;  // unsigned: one compare for the id range
+                if (d <= span && !none) m |= (hd_bits[v[e] >> 5] >> (v[e] & 31) & 1u) << e;
+            }
+            if (!full) {  // elements past E
+                const uint64_t x = b0 + ((uint64_t)(j * (kThreads / 32) + w) * 128) + lane_id() * 4;
+                m &= x >= E ? 0u : (x + 4 <= E ? 0xFu : (0xFu >> (4 - (E - x))));
+            }
+            bits[j] = m;  // 4 bits for this lane's elements
+        }
+#pragma unroll
+        for (int j = 0; j < STEPS; ++j) {
+            // lane L holds bits of elements 4L..4L+3 of the 128-element step: word q = L / 8
+            uint32_t word = bits[j] << ((lane_id() & 7) * 4);
+            word |= __shfl_xor_sync(0xffffffffu, word, 1);
+            word |= __shfl_xor_sync(0xffffffffu, word, 2);
+            word |= __shfl_xor_sync(0xffffffffu, word, 4);
+            const uint64_t x = b0 + ((uint64_t)(j * (kThreads / 32) + w) * 128);
+            if ((lane_id() & 7) == 0 && x + lane_id() * 4 < wend) mask[(x >> 5) + lane_id() / 8] = word;
+        }
     }
 }
 
@@ -1038,6 +1056,9 @@ struct RowArgs {
     OwnRange own;
     const uint64_t* nv_ext;
     const Counters* c;        // device-side list sizes (read by row_counts)
+    const uint64_t* old_ext;  // ID maps (k_rows_fused); identity: old ext id == k
+    uint64_t* new_ext;
+    int identity;
 };
 __device__ __forceinline__ RowArgs row_counts(RowArgs a) {
     a.n_del = a.c->n_del;
@@ -1054,51 +1075,83 @@ __device__ __forceinline__ uint64_t casc_before(const RowArgs& a, uint64_t x) {
     return a.casc_pre[x / kCascBlock] + a.casc_wrel[x >> 5] +
            (r ? __popc(a.casc_mask[x >> 5] & (0xFFFFFFFFu >> (32 - r))) : 0u);
 }
-// CTA boundaries of k_offsets_rows: ranks of each CTA's first row in the two lists
+// CTA boundaries of k_rows_fused (CTA c covers old ids [c*kRowTile, (c+1)*kRowTile)):
+// ranks of each CTA's first shard row (clamped to [row_lo, row_hi]) in the sorted
+// delete and insert-row lists
 __global__ void k_rows_partition(RowArgs a_) {
     const RowArgs a = row_counts(a_);
     const uint64_t c = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x;
-    const uint64_t ncta = (a.row_hi - a.row_lo + kRowTile - 1) / kRowTile;
+    const uint64_t ncta = (a.V_old + kRowTile - 1) / kRowTile;
     if (c > ncta) return;
-    const uint64_t k = a.row_lo + c * kRowTile;
+    const uint64_t k = min(max(c * kRowTile, a.row_lo), a.row_hi);
     uint64_t dr, ir;
     if (k >= a.row_hi) { dr = a.n_del; ir = a.n_ins; }
     else {
         dr = lower_bound_dev(a.del_pos, 0, a.n_del, (uint64_t)a.old_off[k]);
         // insert-row rank of the new id of the first surviving row >= k (compaction formula)
-        const uint64_t u = a.R.shift ? k - lower_bound_dev(a.dropped, 0, a.n_dropped, (uint32_t)k) +
-                                       upper_bound_dev(a.ins_oldpos, 0, a.n_vins, (uint32_t)k)
-                                     : k;
+        const uint64_t u = k - lower_bound_dev(a.dropped, 0, a.n_dropped, (uint32_t)k) +
+                           upper_bound_dev(a.ins_oldpos, 0, a.n_vins, (uint32_t)k);
         ir = lower_bound_dev(a.ins_row, 0, a.n_ins, (uint32_t)u);
     }
     a.part[2 * c] = dr;
     a.part[2 * c + 1] = ir;
 }
 
-__global__ void __launch_bounds__(kThreads) k_offsets_rows(RowArgs a_) {
+// One pass over the old vertices k (node ops only; a2 + a4/a5): each survivor's
+// new dense id u = remap(k) places its external id in the new ID map and, for the
+// rows of this shard, its new row offset
+//   new_off[u] = x - (cascaded before x) - (deleted before x) + (inserted records in rows < u)
+// with x = old_off[k].  The CTA narrows the sorted delete / insert-row lists first.
+__global__ void __launch_bounds__(kThreads) k_rows_fused(RowArgs a_) {
     const RowArgs a = row_counts(a_);
-    const uint64_t k0 = a.row_lo + (uint64_t)blockIdx.x * kRowTile, k1 = min(k0 + kRowTile, a.row_hi);
+    const uint64_t k0 = (uint64_t)blockIdx.x * kRowTile, k1 = min(k0 + kRowTile, a.V_old);
     const uint64_t* pp = a.part + 2 * blockIdx.x;  // this CTA's slices of the delete / insert-row lists
     const uint64_t da = pp[0], ia = pp[1], db = pp[2], ib = pp[3];
-    constexpr int PER = kRowTile / kThreads;  // rows per thread, all loads issued together
+    constexpr int PER = kRowTile / kThreads;  // ids per thread, all loads issued together
     uint32_t u[PER];
-    uint64_t x[PER];
+    uint64_t x[PER], ext[PER];
+    bool row[PER];
 #pragma unroll
     for (int j = 0; j < PER; ++j) {
         const uint64_t k = k0 + threadIdx.x + (uint64_t)j * kThreads;
         u[j] = kNone32;
         x[j] = 0;
-        if (k < k1) { u[j] = remap_of(a.R, (uint32_t)k); x[j] = (uint64_t)a.old_off[k]; }
+        ext[j] = k;
+        row[j] = false;
+        if (k < k1) {
+            u[j] = remap_of(a.R, (uint32_t)k);
+            if (!a.identity) ext[j] = a.old_ext[k];
+            row[j] = k >= a.row_lo && k < a.row_hi;
+            if (row[j]) x[j] = (uint64_t)a.old_off[k];
+        }
     }
     uint64_t cb[PER];
 #pragma unroll
-    for (int j = 0; j < PER; ++j) cb[j] = (u[j] != kNone32) ? casc_before(a, x[j]) : 0;
+    for (int j = 0; j < PER; ++j) cb[j] = (u[j] != kNone32 && row[j]) ? casc_before(a, x[j]) : 0;
 #pragma unroll
     for (int j = 0; j < PER; ++j) {
         if (u[j] == kNone32) continue;
+        a.new_ext[u[j]] = ext[j];
+        if (!row[j]) continue;
         const uint64_t kept = x[j] - cb[j] - lower_bound_dev(a.del_pos, da, db, x[j]);
         a.new_off[u[j] - a.row_lo_new] = (int64_t)(kept + lower_bound_dev(a.ins_row, ia, ib, u[j]));
     }
+}
+
+// Sharded mode: the shard's row range in the new ID map, without the map itself:
+// survivors below the old range start + inserted vertices below the owned ext range
+__global__ void k_row_range_new(const uint32_t* __restrict__ dropped, const uint32_t* __restrict__ ins_q,
+                                const uint64_t* __restrict__ nv_ext, uint64_t row_lo, uint64_t row_hi, OwnRange own,
+                                Counters* __restrict__ c) {
+    const uint64_t nd = c->n_dropped, ni = c->n_inserted;
+    auto ins_below = [&](uint64_t x) {  // inserted vertices (ascending ext ids) with ext < x
+        uint64_t lo = 0, hi = ni;
+        while (lo < hi) { uint64_t m = (lo + hi) >> 1; if (nv_ext[ins_q[m]] < x) lo = m + 1; else hi = m; }
+        return lo;
+    };
+    c->row_lo_new = row_lo - lower_bound_dev(dropped, 0, nd, (uint32_t)row_lo) + ins_below(own.lo);
+    c->row_hi_new = own.hi == ~0ull ? c->Vn
+                                    : row_hi - lower_bound_dev(dropped, 0, nd, (uint32_t)row_hi) + ins_below(own.hi);
 }
 
 // Device-wide exclusive scan of u64 values, single pass (decoupled look-back).
@@ -1201,10 +1254,15 @@ __global__ void __launch_bounds__(kThreads) k_merge3(MergeArgs a_, const TilePar
         for (int q = 0; q < 2 * (int)sizeof(TilePart) / 16; ++q) cp_async16(dst + q, src + q);
         cp_async_commit();
     };
-    // remap fast paths: ids below lohi[0] keep their id, ids at or above lohi[1] shift by lohi[2]
-    uint32_t rlo = 0, rhi = 0;
-    int32_t rsh = 0;
-    if (REMAP) { rlo = (uint32_t)a.R.lohi[0]; rhi = (uint32_t)a.R.lohi[1]; rsh = a.R.lohi[2]; }
+    // remap fast paths: ids below lohi[0] keep their id, ids at or above lohi[1] shift by
+    // lohi[2], ids in [lohi[3], lohi[4]) shift by lohi[5] (between the last dropped id and
+    // the next insertion point: the bulk of the ids when deletes and inserts cluster)
+    uint32_t rlo = 0, rhi = 0, mlo = 0, mspan = 0;
+    int32_t rsh = 0, msh = 0;
+    if (REMAP) {
+        rlo = (uint32_t)a.R.lohi[0]; rhi = (uint32_t)a.R.lohi[1]; rsh = a.R.lohi[2];
+        mlo = (uint32_t)a.R.lohi[3]; mspan = (uint32_t)a.R.lohi[4] - mlo; msh = a.R.lohi[5];
+    }
 
     uint64_t t = blockIdx.x;
     if (tid == 0) {
@@ -1330,7 +1388,8 @@ __global__ void __launch_bounds__(kThreads) k_merge3(MergeArgs a_, const TilePar
                 int32_t shf[KCH];
 #pragma unroll
                 for (int k = 0; k < KCH; ++k)
-                    shf[k] = colv[k] < rlo ? 0 : (colv[k] >= rhi ? rsh : a.R.shift[colv[k] >> kRemapBlockShift]);
+                    shf[k] = colv[k] < rlo ? 0 : (colv[k] >= rhi ? rsh : (colv[k] - mlo < mspan ? msh
+                             : a.R.shift[colv[k] >> kRemapBlockShift]));
                 uint2 g[KCH];
 #pragma unroll
                 for (int k = 0; k < KCH; ++k) g[k] = (shf[k] == kRemapMixed) ? a.R.g32[colv[k] >> 5] : make_uint2(0u, 0u);
@@ -1408,6 +1467,13 @@ __global__ void k_remap_blocks(uint64_t V, const uint32_t* __restrict__ dropped,
         lohi[0] = (int32_t)lo;
         lohi[1] = (int32_t)max(hi, lo);
         lohi[2] = (int32_t)((int64_t)n_ins - (int64_t)n_dropped);
+        // [mlo, mhi): above the last dropped id, below the first insertion point past it
+        const uint64_t mlo = n_dropped ? (uint64_t)dropped[n_dropped - 1] + 1 : 0ull;
+        const uint64_t ci = upper_bound_dev(ins_oldpos, 0, n_ins, (uint32_t)mlo);  // insertion points <= mlo
+        const uint64_t mhi = ci < n_ins ? (uint64_t)ins_oldpos[ci] : V;
+        lohi[3] = (int32_t)mlo;
+        lohi[4] = (int32_t)max(mhi, mlo);
+        lohi[5] = (int32_t)((int64_t)ci - (int64_t)n_dropped);
         c->Vn = V - n_dropped + n_ins;  // vertices of the new ID map
     }
     if (bk >= nb) return;

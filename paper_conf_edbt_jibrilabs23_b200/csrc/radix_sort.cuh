@@ -1,10 +1,11 @@
 // radix_sort.cuh - stable LSD radix sort of (uint64 key, uint32 value) pairs for
-// sm_100a, onesweep style (one kernel per 8-bit digit pass):
+// sm_100a, onesweep style (one kernel per 8-bit digit pass, 3072-key tiles):
 //   1. one histogram kernel counts the digits of every pass in a single read;
 //   2. a tiny kernel turns them into per-pass digit bases;
 //   3. per pass, each 3072-key tile ranks its keys stably with warp match_any,
 //      publishes per-digit counts and resolves its global digit offsets with a
-//      per-digit decoupled look-back (256 threads, one digit each), stages the
+//      per-digit decoupled look-back (256 threads, one digit each, 8 predecessor
+//      tiles per step), stages the
 //      keys digit-sorted in shared memory and writes them out in contiguous runs.
 // Only the significant key bits are sorted (2*ceil(log2 V') for packed
 // (src', dst') edge keys).
@@ -16,8 +17,10 @@ namespace h2tap {
 constexpr int kRsThreads = 256;
 constexpr int kRsItems = 12;
 constexpr int kRsTile = kRsThreads * kRsItems;  // 3072 keys per tile
+constexpr int kRsSmem = kRsTile * 12;           // dynamic smem: staged keys + values
 constexpr int kRsWarps = kRsThreads / 32;
 constexpr int kRsMaxPasses = 8;
+constexpr int kRsLook = 8;  // look-back: predecessor tiles read per step
 
 // n_dev (nullable): the key count lives in device memory (no host sync before the
 // sort); `n` is then an upper bound that only sizes the grids
@@ -63,8 +66,9 @@ __global__ void __launch_bounds__(kRsThreads) rs_onesweep(
     __shared__ uint32_t s_wcnt[kRsWarps][256];
     __shared__ uint32_t s_dstart[256];
     __shared__ uint64_t s_gpre[256];
-    __shared__ uint64_t s_keys[kRsTile];
-    __shared__ uint32_t s_vals[kRsTile];
+    extern __shared__ __align__(16) uint8_t rs_dsm[];  // kRsSmem bytes
+    uint64_t* s_keys = reinterpret_cast<uint64_t*>(rs_dsm);
+    uint32_t* s_vals = reinterpret_cast<uint32_t*>(rs_dsm + kRsTile * 8);
     __shared__ uint32_t s_scan[kRsThreads / 32 + 1];
 
     const int tid = threadIdx.x, w = tid >> 5, l = lane_id();
@@ -107,8 +111,8 @@ __global__ void __launch_bounds__(kRsThreads) rs_onesweep(
     __syncthreads();
     // per digit: exclusive over warps, tile count
     uint32_t c = 0;
-    {
-        const int d = tid;  // 256 threads == 256 digits
+    if (tid < 256) {
+        const int d = tid;  // threads 0..255 own one digit each
         for (int ww = 0; ww < kRsWarps; ++ww) {
             uint32_t t = s_wcnt[ww][d];
             s_wcnt[ww][d] = c;
@@ -117,9 +121,10 @@ __global__ void __launch_bounds__(kRsThreads) rs_onesweep(
     }
     uint32_t tot;
     uint32_t ds = block_exclusive_scan<kRsThreads>(c, s_scan, &tot);
-    s_dstart[tid] = ds;
-    // per-digit decoupled look-back (thread d walks back over tiles for digit d)
-    {
+    if (tid < 256) s_dstart[tid] = ds;
+    // per-digit decoupled look-back: thread d walks back over the tiles for digit d,
+    // kRsLook predecessors per step (independent loads, one L2 round trip per step)
+    if (tid < 256) {
         const int d = tid;
         uint64_t* st = status + (uint64_t)tile * 256 + d;
         uint64_t excl = 0;
@@ -129,12 +134,24 @@ __global__ void __launch_bounds__(kRsThreads) rs_onesweep(
             st_volatile(st, kFlagAgg | c);
             int64_t t = (int64_t)tile - 1;
             while (t >= 0) {
-                uint64_t s = ld_volatile(status + (uint64_t)t * 256 + d);
-                uint64_t f = s >> 62;
-                if (f == 0) continue;
-                excl += s & kValMask;
-                if (f == 2) break;
-                --t;
+                uint64_t s[kRsLook];
+#pragma unroll
+                for (int q = 0; q < kRsLook; ++q)
+                    s[q] = (t - q >= 0) ? ld_volatile(status + (uint64_t)(t - q) * 256 + d) : kFlagPrefix;
+                // consume the ready run up to (and including) the nearest prefix
+                int q = 0;
+                bool done = false;
+#pragma unroll
+                for (int j = 0; j < kRsLook; ++j) {
+                    if (done || q != j) continue;
+                    const uint64_t f = s[j] >> 62;
+                    if (f == 0) continue;  // not published yet: re-poll from here
+                    excl += s[j] & kValMask;
+                    ++q;
+                    if (f == 2) done = true;
+                }
+                if (done) break;
+                t -= q;
             }
             st_volatile(st, kFlagPrefix | (excl + c));
         }

@@ -377,15 +377,24 @@ h2tap_status apply_core(h2tap_replica* r, const BatchIn& in, uint64_t S, bool cr
         uint64_t* kB = r->get<uint64_t>(r->keyB, n_node);
         uint32_t* vA = r->get<uint32_t>(r->valA, n_node);
         uint32_t* vB = r->get<uint32_t>(r->valB, n_node);
-        // stable by ts (input is in seq order), then stable by vertex -> (v, ts, seq)
-        k_keys_from<<<g1(n_node), 256, 0, st>>>(idx_n, n_node, Wt, hc.ts_min, kA, vA);
-        CKL();
-        radix_sort(r, kA, vA, kB, vB, n_node, bits_for(hc.ts_max - hc.ts_min));
-        k_keys_from<<<g1(n_node), 256, 0, st>>>(vA, n_node, Ws, hc.v_min, kB, vB);
-        CKL();
-        std::swap(kA, kB);
-        std::swap(vA, vB);
-        radix_sort(r, kA, vA, kB, vB, n_node, bits_for(hc.v_max - hc.v_min));
+        // (v, ts, seq) order: the input is in seq order and the sort is stable, so one sort
+        // by the packed key (v - v_min, ts - ts_min) when both ranges fit in 64 bits, else
+        // stable by ts, then stable by vertex
+        const int vb = bits_for(hc.v_max - hc.v_min), tb = bits_for(hc.ts_max - hc.ts_min);
+        if (vb + tb <= 64) {
+            k_node_keys<<<g1(n_node), 256, 0, st>>>(idx_n, n_node, Ws, hc.v_min, Wt, hc.ts_min, tb, kA, vA);
+            CKL();
+            radix_sort(r, kA, vA, kB, vB, n_node, vb + tb);
+        } else {
+            k_keys_from<<<g1(n_node), 256, 0, st>>>(idx_n, n_node, Wt, hc.ts_min, kA, vA);
+            CKL();
+            radix_sort(r, kA, vA, kB, vB, n_node, tb);
+            k_keys_from<<<g1(n_node), 256, 0, st>>>(vA, n_node, Ws, hc.v_min, kB, vB);
+            CKL();
+            std::swap(kA, kB);
+            std::swap(vA, vB);
+            radix_sort(r, kA, vA, kB, vB, n_node, vb);
+        }
         TR("node_sort");
         node_sorted = r->get<uint32_t>(r->nsorted, n_node);
         CK(cudaMemcpyAsync(node_sorted, vA, n_node * 4, cudaMemcpyDeviceToDevice, st));

@@ -188,6 +188,18 @@ __global__ void k_keys_from(const uint32_t* __restrict__ idx, uint64_t n, const 
     vals[i] = o;
 }
 
+// keys[i] = (src[o] - v0) << tb | (ts[o] - t0) ; vals[i] = o = idx[i]  (node ops: (v, ts) key)
+__global__ void k_node_keys(const uint32_t* __restrict__ idx, uint64_t n, const uint64_t* __restrict__ src, uint64_t v0,
+                            const uint64_t* __restrict__ ts, uint64_t t0, int tb, uint64_t* __restrict__ keys,
+                            uint32_t* __restrict__ vals) {
+    uint64_t i = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x;
+    if (i >= n) return;
+    uint32_t o = idx[i];
+    const uint64_t hi = src[o] - v0;
+    keys[i] = (tb >= 64 ? 0ull : hi << tb) | (ts[o] - t0);
+    vals[i] = o;
+}
+
 // Old dense index of external id x.  Identity fast path, else a two-level search:
 // fence[i] = ext[i << 8] (V/32 bytes, L2-resident) picks a 256-id block, then a
 // binary search inside the block (2 KB) -- one DRAM-latency chain of ~8 probes

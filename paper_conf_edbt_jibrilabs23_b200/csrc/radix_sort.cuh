@@ -14,13 +14,22 @@
 
 namespace h2tap {
 
+#ifndef H2TAP_RS_ITEMS
+#define H2TAP_RS_ITEMS 12
+#endif
+#ifndef H2TAP_RS_LOOK
+#define H2TAP_RS_LOOK 8
+#endif
+#ifndef H2TAP_RS_BALLOT
+#define H2TAP_RS_BALLOT 0
+#endif
 constexpr int kRsThreads = 256;
-constexpr int kRsItems = 12;
+constexpr int kRsItems = H2TAP_RS_ITEMS;
 constexpr int kRsTile = kRsThreads * kRsItems;  // 3072 keys per tile
 constexpr int kRsSmem = kRsTile * 12;           // dynamic smem: staged keys + values
 constexpr int kRsWarps = kRsThreads / 32;
 constexpr int kRsMaxPasses = 8;
-constexpr int kRsLook = 8;  // look-back: predecessor tiles read per step
+constexpr int kRsLook = H2TAP_RS_LOOK;  // look-back: predecessor tiles read per step
 
 // n_dev (nullable): the key count lives in device memory (no host sync before the
 // sort); `n` is then an upper bound that only sizes the grids
@@ -100,7 +109,17 @@ __global__ void __launch_bounds__(kRsThreads) rs_onesweep(
         rank[i] = 0;
         if (ok) {
             uint32_t d = (uint32_t)(k[i] >> shift) & 255u;
+#if H2TAP_RS_BALLOT
+            // peers with the same digit from 8 ballots (no MATCH instruction)
+            uint32_t peers = valid;
+#pragma unroll
+            for (int b = 0; b < 8; ++b) {
+                const uint32_t m = __ballot_sync(valid, (d >> b) & 1u);
+                peers &= ((d >> b) & 1u) ? m : ~m;
+            }
+#else
             uint32_t peers = __match_any_sync(valid, d);
+#endif
             uint32_t before = s_wcnt[w][d];
             __syncwarp(valid);
             if (l == (uint32_t)(__ffs(peers) - 1)) s_wcnt[w][d] = before + __popc(peers);

@@ -551,6 +551,33 @@ h2tap_status apply_core(h2tap_replica* r, const BatchIn& in, uint64_t S, bool cr
     new_off = r->get<int64_t>(r->off[nb], Vr_new_ub + 1);
     uint32_t* new_cols = r->get<uint32_t>(r->cols[nb], Ecap);
     float* new_w = r->get<float>(r->w[nb], Ecap);
+    // node mode: survivors' ID map + row offsets before the merge, while the cascade
+    // tables written by the cascade pass are still L2-resident (the merge streams the CSR)
+    if (node_mode) {
+        RowArgs ra{};
+        ra.old_off = old_off - row_lo; ra.V_old = V; ra.E_old = E; ra.R = R;
+        ra.row_lo = row_lo; ra.row_hi = row_lo + Vr;
+        ra.own = r->own; ra.nv_ext = nv_ext;
+        ra.casc_mask = casc_mask; ra.casc_pre = casc_pre; ra.casc_wrel = casc_wrel;
+        ra.del_pos = del_pos; ra.ins_row = ins_row;
+        ra.dropped = dropped; ra.ins_oldpos = ins_oldpos;
+        ra.new_off = new_off;
+        ra.c = dc;
+        ra.old_ext = old_ext; ra.new_ext = new_ext; ra.identity = r->identity ? 1 : 0;
+        const uint64_t ncta = cdiv(V, kRowTile);
+        ra.part = r->get<uint64_t>(r->opart, 2 * (ncta + 1));
+        if (V) {
+            k_rows_partition<<<g1(ncta + 1), 256, 0, st>>>(ra);
+            CKL();
+            k_rows_fused<<<(unsigned)ncta, kThreads, 0, st>>>(ra);  // survivors: ID map + row offsets
+            CKL();
+        }
+        k_offsets_inserted<<<g1(n_node), 256, 0, st>>>(nv, ins_q, ra);
+        CKL();
+        uint64_t* f = r->get<uint64_t>(r->fence[ec ^ 1], n_fence(Vn_ub));
+        k_build_fence_dev<<<g1(n_fence(Vn_ub)), 256, 0, st>>>(new_ext, dc, f);
+        CKL();
+    }
     if (Ecap) {
         MergeArgs ma{};
         ma.old_cols = old_cols; ma.old_w = old_w; ma.E_old = E;
@@ -605,31 +632,6 @@ h2tap_status apply_core(h2tap_replica* r, const BatchIn& in, uint64_t S, bool cr
         k_scan_exclusive_i64<<<(unsigned)nts, kThreads, 0, st>>>(tsum, tbase, nt, stt, &dc->tiles[7]);
         CKL();
         k_offsets_apply<<<(unsigned)nt, kThreads, 0, st>>>(old_off, deg, Vr, tbase, new_off);
-        CKL();
-    }
-    if (node_mode) {
-        RowArgs ra{};
-        ra.old_off = old_off - row_lo; ra.V_old = V; ra.E_old = E; ra.R = R;
-        ra.row_lo = row_lo; ra.row_hi = row_lo + Vr;
-        ra.own = r->own; ra.nv_ext = nv_ext;
-        ra.casc_mask = casc_mask; ra.casc_pre = casc_pre; ra.casc_wrel = casc_wrel;
-        ra.del_pos = del_pos; ra.ins_row = ins_row;
-        ra.dropped = dropped; ra.ins_oldpos = ins_oldpos;
-        ra.new_off = new_off;
-        ra.c = dc;
-        ra.old_ext = old_ext; ra.new_ext = new_ext; ra.identity = r->identity ? 1 : 0;
-        const uint64_t ncta = cdiv(V, kRowTile);
-        ra.part = r->get<uint64_t>(r->opart, 2 * (ncta + 1));
-        if (V) {
-            k_rows_partition<<<g1(ncta + 1), 256, 0, st>>>(ra);
-            CKL();
-            k_rows_fused<<<(unsigned)ncta, kThreads, 0, st>>>(ra);  // survivors: ID map + row offsets
-            CKL();
-        }
-        k_offsets_inserted<<<g1(n_node), 256, 0, st>>>(nv, ins_q, ra);
-        CKL();
-        uint64_t* f = r->get<uint64_t>(r->fence[ec ^ 1], n_fence(Vn_ub));
-        k_build_fence_dev<<<g1(n_fence(Vn_ub)), 256, 0, st>>>(new_ext, dc, f);
         CKL();
     }
     } else {

@@ -1397,20 +1397,24 @@ __global__ void __launch_bounds__(kThreads) k_merge3(MergeArgs a_, const TilePar
                 colv[k] = (i < n_old) ? s_col[b][i + sh] : 0u;
             }
             if (REMAP) {
-                int32_t shf[KCH];
-#pragma unroll
-                for (int k = 0; k < KCH; ++k)
-                    shf[k] = colv[k] < rlo ? 0 : (colv[k] >= rhi ? rsh : (colv[k] - mlo < mspan ? msh
-                             : a.R.shift[colv[k] >> kRemapBlockShift]));
+                // three constant-shift id ranges need no table; any other id reads its
+                // 32-id group entry.  Branch-free: a constant-shift id gets the synthetic
+                // entry {id + shift - r, no drops}, so every id evaluates the same
+                // expression  base + r - popc(dropped below r)
                 uint2 g[KCH];
 #pragma unroll
-                for (int k = 0; k < KCH; ++k) g[k] = (shf[k] == kRemapMixed) ? a.R.g32[colv[k] >> 5] : make_uint2(0u, 0u);
+                for (int k = 0; k < KCH; ++k) {
+                    const uint32_t col = colv[k];
+                    const bool tab = !(col < rlo || col >= rhi || col - mlo < mspan);
+                    const int32_t shf = col < rlo ? 0 : (col >= rhi ? rsh : msh);
+                    g[k] = tab ? a.R.g32[col >> 5] : make_uint2((uint32_t)((int32_t)(col & ~31u) + shf), 0u);
+                }
 #pragma unroll
                 for (int k = 0; k < KCH; ++k) {
                     const uint32_t col = colv[k], r = col & 31;
-                    if (shf[k] != kRemapMixed) colv[k] = (uint32_t)((int64_t)col + shf[k]);
-                    else if (g[k].x >> 31) colv[k] = remap_of_slow(a.R.shift, a.R.g32, a.R.ins_oldpos, a.R.n_vins, col);
-                    else colv[k] = g[k].x + r - (r ? __popc(g[k].y & (0xFFFFFFFFu >> (32 - r))) : 0u);
+                    colv[k] = (g[k].x & 0x7FFFFFFFu) + r - __popc(g[k].y & ((1u << r) - 1u));
+                    if (g[k].x >> 31)  // an insertion point strictly inside the group (rare)
+                        colv[k] = remap_of_slow(a.R.shift, a.R.g32, a.R.ins_oldpos, a.R.n_vins, col);
                 }
             }
 #pragma unroll
@@ -1657,7 +1661,8 @@ __global__ void k_remap32(uint64_t V, const uint32_t* __restrict__ dropped, cons
     const uint32_t c0 = (uint32_t)(g * 32);
     const uint64_t d0 = lower_bound_dev(dropped, 0, n_dropped, c0);
     const uint64_t i0 = upper_bound_dev(ins_oldpos, 0, n_vins, c0);
-    const uint64_t i1 = upper_bound_dev(ins_oldpos, i0, n_vins, c0 + 31);
+    // insertion points past the last old id (appended vertices) shift no old id
+    const uint64_t i1 = upper_bound_dev(ins_oldpos, i0, n_vins, (uint32_t)min((uint64_t)c0 + 31, V - 1));
     uint32_t m = 0;
     for (uint64_t d = d0; d < n_dropped && dropped[d] < c0 + 32; ++d) m |= 1u << (dropped[d] - c0);
     out[g] = make_uint2((uint32_t)(c0 - d0 + i0) | (i1 > i0 ? 0x80000000u : 0u), m);

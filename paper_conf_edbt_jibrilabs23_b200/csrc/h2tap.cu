@@ -567,7 +567,7 @@ h2tap_status apply_core(h2tap_replica* r, const BatchIn& in, uint64_t S, bool cr
         const uint64_t ncta = cdiv(V, kRowTile);
         ra.part = r->get<uint64_t>(r->opart, 2 * (ncta + 1));
         if (V) {
-            k_rows_partition<<<g1(ncta + 1), 256, 0, st>>>(ra);
+            k_rows_partition<><<<g1(ncta + 1), 256, 0, st>>>(ra);
             CKL();
             k_rows_fused<<<(unsigned)ncta, kThreads, 0, st>>>(ra);  // survivors: ID map + row offsets
             CKL();
@@ -576,6 +576,24 @@ h2tap_status apply_core(h2tap_replica* r, const BatchIn& in, uint64_t S, bool cr
         CKL();
         uint64_t* f = r->get<uint64_t>(r->fence[ec ^ 1], n_fence(Vn_ub));
         k_build_fence_dev<<<g1(n_fence(Vn_ub)), 256, 0, st>>>(new_ext, dc, f);
+        CKL();
+    }
+    // ---- a4/a5 without node ops: row offsets (while the outcome lists are L2-resident)
+    if (Vr && !node_mode) {
+        // new_off[k] = old_off[k] - (deletes before it) + (inserts in earlier rows): two
+        // ranks in the sorted outcome lists, one streaming pass over the shard's rows
+        RowArgs ra{};
+        ra.old_off = old_off - row_lo; ra.V_old = V; ra.E_old = E;
+        ra.row_lo = row_lo; ra.row_hi = row_lo + Vr;
+        ra.del_pos = del_pos; ra.del_row = del_row; ra.ins_row = ins_row;
+        ra.new_off = new_off;
+        ra.c = dc;
+        const uint64_t ncta = cdiv(V, kOffTile);
+        ra.part = r->get<uint64_t>(r->opart, 2 * (ncta + 1));
+        k_rows_partition<kOffTile><<<g1(ncta + 1), 256, 0, st>>>(ra);
+        CKL();
+        const uint64_t c_lo = row_lo / kOffTile, c_hi = cdiv(row_lo + Vr, kOffTile);
+        k_offsets_direct<<<(unsigned)(c_hi - c_lo), kThreads, 0, st>>>(ra);
         CKL();
     }
     if (Ecap) {
@@ -613,27 +631,6 @@ h2tap_status apply_core(h2tap_replica* r, const BatchIn& in, uint64_t S, bool cr
     CK(cudaEventRecord(r->ev[4], st));
     TR("merge");
 
-    // ---- a4/a5: row offsets
-    if (Vr && !node_mode) {
-        // per-vertex degree delta + exclusive scan (tile sums by decoupled look-back)
-        int32_t* deg = r->get<int32_t>(r->deg, Vr);
-        const uint64_t nt = cdiv(Vr, kTile);
-        int64_t* tsum = r->get<int64_t>(r->tsum, nt + 1);
-        int64_t* tbase = r->get<int64_t>(r->KR, nt + 1);
-        CK(cudaMemsetAsync(deg, 0, Vr * 4, st));
-        CK(cudaMemsetAsync(tsum, 0, (nt + 1) * 8, st));
-        if (n_edge) {
-            k_deg_scatter<<<g1(n_edge), 256, 0, st>>>(ins_row, del_row, dc, deg, tsum, row_lo);
-            CKL();
-        }
-        const uint64_t nts = cdiv(nt, kTile);
-        uint64_t* stt = r->get<uint64_t>(r->status, nts);
-        CK(cudaMemsetAsync(stt, 0, nts * 8, st));
-        k_scan_exclusive_i64<<<(unsigned)nts, kThreads, 0, st>>>(tsum, tbase, nt, stt, &dc->tiles[7]);
-        CKL();
-        k_offsets_apply<<<(unsigned)nt, kThreads, 0, st>>>(old_off, deg, Vr, tbase, new_off);
-        CKL();
-    }
     } else {
         CK(cudaEventRecord(r->ev[6], st));
         CK(cudaEventRecord(r->ev[4], st));

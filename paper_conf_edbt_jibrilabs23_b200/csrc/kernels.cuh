@@ -1054,6 +1054,7 @@ struct RowArgs {
     const uint64_t* casc_pre;
     const uint16_t* casc_wrel;
     const uint64_t* del_pos;
+    const uint32_t* del_row;  // k_offsets_direct
     uint64_t n_del;
     const uint32_t* ins_row;
     uint64_t n_ins;
@@ -1090,12 +1091,13 @@ __device__ __forceinline__ uint64_t casc_before(const RowArgs& a, uint64_t x) {
 // CTA boundaries of k_rows_fused (CTA c covers old ids [c*kRowTile, (c+1)*kRowTile)):
 // ranks of each CTA's first shard row (clamped to [row_lo, row_hi]) in the sorted
 // delete and insert-row lists
+template <int TILE = kRowTile>
 __global__ void k_rows_partition(RowArgs a_) {
     const RowArgs a = row_counts(a_);
     const uint64_t c = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x;
-    const uint64_t ncta = (a.V_old + kRowTile - 1) / kRowTile;
+    const uint64_t ncta = (a.V_old + TILE - 1) / TILE;
     if (c > ncta) return;
-    const uint64_t k = min(max(c * kRowTile, a.row_lo), a.row_hi);
+    const uint64_t k = min(max(c * TILE, a.row_lo), a.row_hi);
     uint64_t dr, ir;
     if (k >= a.row_hi) { dr = a.n_del; ir = a.n_ins; }
     else {
@@ -1147,6 +1149,56 @@ __global__ void __launch_bounds__(kThreads) k_rows_fused(RowArgs a_) {
         if (!row[j]) continue;
         const uint64_t kept = x[j] - cb[j] - lower_bound_dev(a.del_pos, da, db, x[j]);
         a.new_off[u[j] - a.row_lo_new] = (int64_t)(kept + lower_bound_dev(a.ins_row, ia, ib, u[j]));
+    }
+}
+
+// Row offsets without node ops (a4/a5; identity remap, no cascade): the exclusive
+// scan of the per-row degree delta at row k is a difference of two ranks in the
+// sorted outcome lists, so one streaming pass replaces scatter + scan:
+//   new_off[k] = x - (deleted old elements before x) + (inserted records in rows < k),
+// x = old_off[k].  CTA c covers rows [c*kRowTile, (c+1)*kRowTile) of the shard;
+// k_rows_partition supplies its slices of the two lists.
+constexpr int kOffTile = 4096;
+__global__ void __launch_bounds__(kThreads) k_offsets_direct(RowArgs a_) {
+    // per-row degree delta of the CTA's rows in a shared-memory histogram (from its
+    // slices of the two sorted lists), scanned in place; old and new offsets move
+    // with coalesced (row-strided) accesses
+    constexpr int PER = kOffTile / kThreads;
+    constexpr int kPad = kOffTile + kOffTile / 32;
+    __shared__ int32_t s_cnt[kPad];  // padded: index i at i + i/32 (conflict-free blocked scan)
+    __shared__ int64_t s_scan[kThreads / 32 + 1];
+    const RowArgs a = row_counts(a_);
+    const uint64_t c = blockIdx.x + a.row_lo / kOffTile, kb = c * kOffTile;
+    const uint32_t l0 = (uint32_t)(max(kb, a.row_lo) - kb), l1 = (uint32_t)(min(kb + kOffTile, a.row_hi) - kb);
+    const uint64_t* pp = a.part + 2 * c;
+    const uint64_t da = pp[0], ia = pp[1], db = pp[2], ib = pp[3];
+    const int64_t* oo = a.old_off + kb;
+    int64_t x[PER];
+#pragma unroll
+    for (int j = 0; j < PER; ++j) {
+        const uint32_t l = threadIdx.x + j * kThreads;
+        x[j] = (l >= l0 && l < l1) ? oo[l] : 0;
+    }
+    auto P = [](uint32_t i) { return i + (i >> 5); };
+#pragma unroll
+    for (int j = 0; j < PER; ++j) s_cnt[P(threadIdx.x + j * kThreads)] = 0;
+    __syncthreads();
+    for (uint64_t i = ia + threadIdx.x; i < ib; i += kThreads) atomicAdd(&s_cnt[P((uint32_t)(a.ins_row[i] - kb))], 1);
+    for (uint64_t i = da + threadIdx.x; i < db; i += kThreads) atomicAdd(&s_cnt[P((uint32_t)(a.del_row[i] - kb))], -1);
+    __syncthreads();
+    int32_t sum = 0;
+#pragma unroll
+    for (int j = 0; j < PER; ++j) sum += s_cnt[P(threadIdx.x * PER + j)];
+    int32_t tot, run = block_exclusive_scan<kThreads>(sum, (int32_t*)s_scan, &tot);
+#pragma unroll
+    for (int j = 0; j < PER; ++j) { const int32_t dj = s_cnt[P(threadIdx.x * PER + j)]; s_cnt[P(threadIdx.x * PER + j)] = run; run += dj; }
+    __syncthreads();
+    const int64_t base = (int64_t)ia - (int64_t)da;
+    int64_t* o = a.new_off + (kb - a.row_lo);
+#pragma unroll
+    for (int j = 0; j < PER; ++j) {
+        const uint32_t l = threadIdx.x + j * kThreads;
+        if (l >= l0 && l < l1) o[l] = x[j] + base + s_cnt[P(l)];
     }
 }
 

@@ -19,7 +19,7 @@ import weakref
 import numpy as np
 
 _HERE = os.path.dirname(os.path.abspath(__file__))
-LIB_PATH = os.path.join(_HERE, "libh2tap.so")
+LIB_PATH = os.environ.get("H2TAP_LIB") or os.path.join(_HERE, "libh2tap.so")  # override: build-variant experiments
 
 OK = 0
 STATUS = {0: "OK", -1: "E_INVAL", -2: "E_NOMEM", -3: "E_CUDA", -4: "E_NCCL", -5: "E_STALE_TS",

@@ -1116,7 +1116,7 @@ __global__ void k_rows_partition(RowArgs a_) {
 // rows of this shard, its new row offset
 //   new_off[u] = x - (cascaded before x) - (deleted before x) + (inserted records in rows < u)
 // with x = old_off[k].  The CTA narrows the sorted delete / insert-row lists first.
-__global__ void __launch_bounds__(kThreads) k_rows_fused(RowArgs a_) {
+__global__ void __launch_bounds__(kThreads, 5) k_rows_fused(RowArgs a_) {
     const RowArgs a = row_counts(a_);
     const uint64_t k0 = (uint64_t)blockIdx.x * kRowTile, k1 = min(k0 + kRowTile, a.V_old);
     const uint64_t* pp = a.part + 2 * blockIdx.x;  // this CTA's slices of the delete / insert-row lists
@@ -1427,6 +1427,40 @@ __global__ void __launch_bounds__(kThreads) k_merge3(MergeArgs a_, const TilePar
             if (lane == 31) s_chunk[NCH] = make_uint4(0u, inc, ik, 0u);
         }
         mbar_wait(&s_bar[b], (it >> 1) & 1);
+        // columns of this tile's old elements (warp w owns chunks w, w+8, ..., w+56) and
+        // their remap, unrolled so that the table lookups are in flight together; warps
+        // 1-7 do this while warp 0 builds the chunk table
+        constexpr int KCH = NCH / (kThreads / 32);  // 8 chunks per warp
+        uint32_t colv[KCH];
+        auto load_cols = [&]() {
+#pragma unroll
+            for (int k = 0; k < KCH; ++k) {
+                const uint32_t c = wid + k * (kThreads / 32), i = c * 32 + lane;
+                colv[k] = (i < n_old) ? s_col[b][i + sh] : 0u;
+            }
+        };
+        if (REMAP) {
+            load_cols();
+            // three constant-shift id ranges need no table; any other id reads its
+            // 32-id group entry.  Branch-free: a constant-shift id gets the synthetic
+            // entry {id + shift - r, no drops}, so every id evaluates the same
+            // expression  base + r - popc(dropped below r)
+            uint2 g[KCH];
+#pragma unroll
+            for (int k = 0; k < KCH; ++k) {
+                const uint32_t col = colv[k];
+                const bool tab = !(col < rlo || col >= rhi || col - mlo < mspan);
+                const int32_t shf = col < rlo ? 0 : (col >= rhi ? rsh : msh);
+                g[k] = tab ? a.R.g32[col >> 5] : make_uint2((uint32_t)((int32_t)(col & ~31u) + shf), 0u);
+            }
+#pragma unroll
+            for (int k = 0; k < KCH; ++k) {
+                const uint32_t col = colv[k], r = col & 31;
+                colv[k] = (g[k].x & 0x7FFFFFFFu) + r - __popc(g[k].y & ((1u << r) - 1u));
+                if (g[k].x >> 31)  // an insertion point strictly inside the group (rare)
+                    colv[k] = remap_of_slow(a.R.shift, a.R.g32, a.R.ins_oldpos, a.R.n_vins, col);
+            }
+        }
         for (uint32_t i = tid; i < nu; i += kThreads) {
             const bool pf = i == (uint32_t)tid;
             s_w[b][(pf ? pf_upd : a.upd_pos[ul0 + i]) - (j0 & ~3ull)] = pf ? pf_uw : a.upd_w[ul0 + i];
@@ -1438,37 +1472,9 @@ __global__ void __launch_bounds__(kThreads) k_merge3(MergeArgs a_, const TilePar
         const uint32_t n_out = kept + ni;
         const uint64_t base = j0 - dl0 - cbefore + r0;
         const uint32_t ob = (uint32_t)(base & 3);
-        // phase B: warp w owns chunks w, w+8, ..., w+56, unrolled so that the remap-table
-        // lookups of all of them are in flight together
+        // phase B: place the kept old elements (columns remapped above)
         {
-            constexpr int KCH = NCH / (kThreads / 32);  // 8 chunks per warp
-            uint32_t colv[KCH];
-#pragma unroll
-            for (int k = 0; k < KCH; ++k) {
-                const uint32_t c = wid + k * (kThreads / 32), i = c * 32 + lane;
-                colv[k] = (i < n_old) ? s_col[b][i + sh] : 0u;
-            }
-            if (REMAP) {
-                // three constant-shift id ranges need no table; any other id reads its
-                // 32-id group entry.  Branch-free: a constant-shift id gets the synthetic
-                // entry {id + shift - r, no drops}, so every id evaluates the same
-                // expression  base + r - popc(dropped below r)
-                uint2 g[KCH];
-#pragma unroll
-                for (int k = 0; k < KCH; ++k) {
-                    const uint32_t col = colv[k];
-                    const bool tab = !(col < rlo || col >= rhi || col - mlo < mspan);
-                    const int32_t shf = col < rlo ? 0 : (col >= rhi ? rsh : msh);
-                    g[k] = tab ? a.R.g32[col >> 5] : make_uint2((uint32_t)((int32_t)(col & ~31u) + shf), 0u);
-                }
-#pragma unroll
-                for (int k = 0; k < KCH; ++k) {
-                    const uint32_t col = colv[k], r = col & 31;
-                    colv[k] = (g[k].x & 0x7FFFFFFFu) + r - __popc(g[k].y & ((1u << r) - 1u));
-                    if (g[k].x >> 31)  // an insertion point strictly inside the group (rare)
-                        colv[k] = remap_of_slow(a.R.shift, a.R.g32, a.R.ins_oldpos, a.R.n_vins, col);
-                }
-            }
+            if (!REMAP) load_cols();
 #pragma unroll
             for (int k = 0; k < KCH; ++k) {
                 const uint32_t c = wid + k * (kThreads / 32), i = c * 32 + lane;

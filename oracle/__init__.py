@@ -67,6 +67,8 @@ def lib():
         L.o1_pending.argtypes = [P, P, P, P, P, P, P]
         L.o1_bfs.argtypes = [u64, P, P, u64, P]
         L.o1_pagerank.argtypes = [u64, P, P, ctypes.c_double, ctypes.c_int, P]
+        L.o1_sssp.restype = ctypes.c_int
+        L.o1_sssp.argtypes = [u64, P, P, P, u64, P]
         _lib = L
     return _lib
 
@@ -145,6 +147,15 @@ def bfs(offsets, cols, source_dense: int) -> np.ndarray:
     lvl = np.empty(len(off) - 1, np.int32)
     lib().o1_bfs(len(off) - 1, _p(off), _p(cols), source_dense, _p(lvl))
     return lvl
+
+
+def sssp(offsets, cols, weights, source_dense: int) -> np.ndarray:
+    """Dijkstra distances (fp64, +inf unreachable); ValueError on a negative or NaN weight."""
+    off, cols, w = _c(offsets, np.int64), _c(cols, np.uint32), _c(weights, np.float32)
+    dist = np.empty(len(off) - 1, np.float64)
+    if lib().o1_sssp(len(off) - 1, _p(off), _p(cols), _p(w), source_dense, _p(dist)) != 0:
+        raise ValueError("sssp: negative or NaN edge weight")
+    return dist
 
 
 def pagerank(offsets, cols, damping: float = 0.85, iterations: int = 20) -> np.ndarray:

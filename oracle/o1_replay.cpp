@@ -37,6 +37,8 @@
 #include <cstdint>
 #include <cstring>
 #include <deque>
+#include <limits>
+#include <queue>
 #include <map>
 #include <set>
 #include <vector>
@@ -258,6 +260,38 @@ void o1_pagerank(uint64_t nv, const int64_t* off, const uint32_t* cols, double d
         cur.swap(nxt);
     }
     std::memcpy(pr, cur.data(), nv * sizeof(double));
+}
+
+/* SSSP (Table 1's third analytic; reading A21):
+ * textbook Dijkstra with a binary heap over out-edges, edge length = the f32
+ * weight widened to fp64, path length = left-to-right fp64 sum along the path;
+ * dist[source] = 0, unreachable = +inf.  Requires weights >= 0 and not NaN
+ * (returns -1 otherwise, dist untouched). */
+int o1_sssp(uint64_t nv, const int64_t* off, const uint32_t* cols, const float* w, uint64_t source,
+            double* dist) {
+    for (uint64_t e = 0; nv && e < (uint64_t)off[nv]; ++e)
+        if (w[e] != w[e] || w[e] < 0.0f) return -1;  // NaN or negative (-0.0 is allowed)
+    const double inf = std::numeric_limits<double>::infinity();
+    for (uint64_t v = 0; v < nv; ++v) dist[v] = inf;
+    if (source >= nv) return 0;
+    std::vector<char> done(nv, 0);
+    typedef std::pair<double, uint64_t> item;
+    std::priority_queue<item, std::vector<item>, std::greater<item>> pq;
+    dist[source] = 0.0;
+    pq.push(item(0.0, source));
+    while (!pq.empty()) {
+        item t = pq.top();
+        pq.pop();
+        uint64_t u = t.second;
+        if (done[u]) continue;
+        done[u] = 1;
+        for (int64_t e = off[u]; e < off[u + 1]; ++e) {
+            uint32_t v = cols[e];
+            double nd = dist[u] + (double)w[e];
+            if (nd < dist[v]) { dist[v] = nd; pq.push(item(nd, v)); }
+        }
+    }
+    return 0;
 }
 
 }  // extern "C"

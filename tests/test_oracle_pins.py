@@ -305,3 +305,65 @@ def test_checksum_is_position_keyed():
     assert oracle.checksum(a, 2) != oracle.checksum(b, 2)
     assert oracle.checksum(a, 2) == oracle.checksum(a.copy(), 2)
     assert oracle.checksum(np.array([], np.uint32), 2) == 0
+
+
+# ------------------------------------------------------------------ SSSP ----
+def _bellman_ford(n, off, cols, w, s):
+    """brute force: |V| rounds of relaxing every edge (pure Python, tiny graphs only)"""
+    d = [float("inf")] * n
+    d[s] = 0.0
+    for _ in range(n):
+        for u in range(n):
+            for e in range(off[u], off[u + 1]):
+                nd = d[u] + float(w[e])
+                if nd < d[cols[e]]:
+                    d[cols[e]] = nd
+    return np.array(d)
+
+
+def test_sssp_matches_scipy_dijkstra():
+    from scipy.sparse import csr_matrix
+    from scipy.sparse.csgraph import dijkstra
+    for scale in (5, 9):
+        n = 1 << scale
+        src, dst, w = synth.rmat_edges(scale, seed=scale + 20, n=6 * n)
+        off, cols, wt, _ = O1.from_edges(n, None, src, dst, w).export()
+        wt = (wt + np.float32(2.0 ** -24)).astype(np.float32)  # strictly positive (scipy drops explicit zeros)
+        A = csr_matrix((wt.astype(np.float64), cols.astype(np.int64), off), shape=(n, n))
+        for s in (0, 3, n - 1):
+            d = oracle.sssp(off, cols, wt, s)
+            ref = dijkstra(A, directed=True, indices=s)
+            # weights are multiples of 2^-24 below 1: every path sum is exact in fp64
+            assert np.array_equal(d, ref)
+
+
+def test_sssp_brute_force_closed_forms_and_errors():
+    rng = np.random.default_rng(7)
+    for trial in range(30):
+        n = int(rng.integers(1, 9))
+        m = int(rng.integers(0, 3 * n))
+        es = {}
+        for _ in range(m):
+            es[(int(rng.integers(n)), int(rng.integers(n)))] = rng.choice([0.0, -0.0, 0.25, 0.5, 1.0, 3.0])
+        keys = sorted(es)
+        off = np.zeros(n + 1, np.int64)
+        for (u, _) in keys:
+            off[u + 1] += 1
+        off = np.cumsum(off)
+        cols = np.array([v for (_, v) in keys], np.uint32)
+        w = np.array([es[k] for k in keys], np.float32)
+        s = int(rng.integers(n))
+        d = oracle.sssp(off, cols, w, s)
+        assert np.array_equal(d, _bellman_ford(n, off, cols, w, s))
+        assert d[s] == 0.0 and not np.signbit(d[s])
+    # path 0 -> 1 -> ... -> n-1 with unit weights plus a shortcut 0 -> n-1 of weight 2.5
+    n = 6
+    off = np.array([0, 2, 3, 4, 5, 6, 6], np.int64)
+    cols = np.array([1, 5, 2, 3, 4, 5], np.uint32)
+    w = np.array([1, 2.5, 1, 1, 1, 1], np.float32)
+    assert np.array_equal(oracle.sssp(off, cols, w, 0), [0, 1, 2, 3, 4, 2.5])
+    assert np.array_equal(oracle.sssp(off, cols, w, 3), [np.inf, np.inf, np.inf, 0, 1, 2])
+    with pytest.raises(ValueError):
+        oracle.sssp(off, cols, np.array([1, -1, 1, 1, 1, 1], np.float32), 0)
+    with pytest.raises(ValueError):
+        oracle.sssp(off, cols, np.array([1, np.nan, 1, 1, 1, 1], np.float32), 0)

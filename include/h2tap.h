@@ -196,6 +196,17 @@ h2tap_status h2tap_bfs(const h2tap_replica* r, uint64_t source_ext, int32_t* lev
 h2tap_status h2tap_pagerank(const h2tap_replica* r, double damping, int iterations,
         double* rank_out, int on_device);
 
+/* Single-source shortest paths over out-edges from the vertex with external ID
+ * source_ext (Table 1's third analytic; reading A21):
+ * dist double[V] in dense-ID order, edge length = the f32 weight widened to fp64,
+ * path length = fp64 sum along the path, dist[source] = 0, unreachable = +inf.
+ * Equal, bit for bit, to Dijkstra's result (the fixpoint is unique for weights >= 0).
+ * dist_out: host (on_device = 0) or device (1) buffer of V doubles, caller-owned.
+ * Errors: unknown source, a negative or NaN weight, or a sharded replica -> E_INVAL
+ * (dist_out unspecified).  Reads the front buffer only. */
+h2tap_status h2tap_sssp(const h2tap_replica* r, uint64_t source_ext, double* dist_out,
+        int on_device);
+
 void h2tap_replica_destroy(h2tap_replica* r);
 const char* h2tap_status_str(h2tap_status s);
 const char* h2tap_last_error(void);

@@ -93,6 +93,8 @@ _lib.h2tap_replica_export.restype = ctypes.c_int
 _lib.h2tap_replica_export.argtypes = [_P, _P, _P, _P, _P, ctypes.c_int, ctypes.POINTER(_u64)]
 _lib.h2tap_bfs.restype = ctypes.c_int
 _lib.h2tap_bfs.argtypes = [_P, _u64, _P, ctypes.c_int]
+_lib.h2tap_sssp.restype = ctypes.c_int
+_lib.h2tap_sssp.argtypes = [_P, _u64, _P, ctypes.c_int]
 _lib.h2tap_pagerank.restype = ctypes.c_int
 _lib.h2tap_pagerank.argtypes = [_P, ctypes.c_double, ctypes.c_int, _P, ctypes.c_int]
 _lib.h2tap_replica_destroy.restype = None
@@ -315,6 +317,11 @@ class Replica:
         lvl = np.empty(self.info()["n_vertices"], np.int32)
         _check(_lib.h2tap_bfs(self._h, int(source_ext), ctypes.c_void_p(lvl.ctypes.data), 0), "h2tap_bfs")
         return lvl
+
+    def sssp(self, source_ext: int) -> np.ndarray:
+        dist = np.empty(self.info()["n_vertices"], np.float64)
+        _check(_lib.h2tap_sssp(self._h, int(source_ext), ctypes.c_void_p(dist.ctypes.data), 0), "h2tap_sssp")
+        return dist
 
     def pagerank(self, damping: float = 0.85, iterations: int = 20) -> np.ndarray:
         pr = np.empty(self.info()["n_vertices"], np.float64)

@@ -1068,6 +1068,23 @@ h2tap_status h2tap_replica_export(const h2tap_replica* rc, int64_t* offsets, uin
     });
 }
 
+// dense id of a live vertex (V if absent): identity map, else a binary search of the
+// device ID map through single-element reads (the analytics' source lookup only)
+static uint64_t dense_of(h2tap_replica* r, uint64_t x_ext) {
+    const uint64_t V = r->V;
+    if (r->identity) return x_ext < V ? x_ext : V;
+    const uint64_t* ext = static_cast<const uint64_t*>(r->ext[r->ext_cur].p);
+    uint64_t lo = 0, hi = V;
+    while (lo < hi) {
+        uint64_t mid = (lo + hi) / 2, x;
+        CK(cudaMemcpy(&x, ext + mid, 8, cudaMemcpyDeviceToHost));
+        if (x < x_ext) lo = mid + 1; else hi = mid;
+    }
+    uint64_t x = ~0ull;
+    if (lo < V) CK(cudaMemcpy(&x, ext + lo, 8, cudaMemcpyDeviceToHost));
+    return (lo < V && x == x_ext) ? lo : V;
+}
+
 h2tap_status h2tap_bfs(const h2tap_replica* rc, uint64_t source_ext, int32_t* level_out, int on_device) {
     h2tap_replica* r = const_cast<h2tap_replica*>(rc);
     if (!r || !level_out) { set_err("null argument"); return H2TAP_E_INVAL; }
@@ -1075,22 +1092,7 @@ h2tap_status h2tap_bfs(const h2tap_replica* rc, uint64_t source_ext, int32_t* le
     return run_guarded(r, [&]() -> h2tap_status {
         CK(cudaSetDevice(r->cfg.device));
         const uint64_t V = r->V;
-        // source lookup on the host side of the ID map (one binary search through D2H probes is
-        // avoided: copy-free search via a tiny kernel would be equivalent; V is small relative)
-        uint64_t src = V;
-        if (r->identity) src = source_ext < V ? source_ext : V;
-        else {
-            const uint64_t* ext = static_cast<const uint64_t*>(r->ext[r->ext_cur].p);
-            uint64_t lo = 0, hi = V;
-            while (lo < hi) {
-                uint64_t mid = (lo + hi) / 2, x;
-                CK(cudaMemcpy(&x, ext + mid, 8, cudaMemcpyDeviceToHost));
-                if (x < source_ext) lo = mid + 1; else hi = mid;
-            }
-            uint64_t x = ~0ull;
-            if (lo < V) CK(cudaMemcpy(&x, ext + lo, 8, cudaMemcpyDeviceToHost));
-            if (lo < V && x == source_ext) src = lo;
-        }
+        const uint64_t src = dense_of(r, source_ext);
         if (src >= V) { set_err("BFS source %llu is not a live vertex", (unsigned long long)source_ext); return H2TAP_E_INVAL; }
         int32_t* level = on_device ? level_out : r->get<int32_t>(r->pr_a, V);
         uint32_t* fa = r->get<uint32_t>(r->bfs_a, V);
@@ -1117,6 +1119,58 @@ h2tap_status h2tap_bfs(const h2tap_replica* rc, uint64_t source_ext, int32_t* le
             std::swap(fa, fb);
         }
         if (!on_device) CK(cudaMemcpyAsync(level_out, level, V * 4, cudaMemcpyDeviceToHost, r->st));
+        r->sync();
+        return H2TAP_OK;
+    });
+}
+
+h2tap_status h2tap_sssp(const h2tap_replica* rc, uint64_t source_ext, double* dist_out, int on_device) {
+    h2tap_replica* r = const_cast<h2tap_replica*>(rc);
+    if (!r || !dist_out) { set_err("null argument"); return H2TAP_E_INVAL; }
+    if (r->sharded) { set_err("h2tap_sssp: not available on a sharded replica in this build"); return H2TAP_E_INVAL; }
+    return run_guarded(r, [&]() -> h2tap_status {
+        CK(cudaSetDevice(r->cfg.device));
+        const uint64_t V = r->V, E = r->E;
+        const uint64_t src = dense_of(r, source_ext);
+        if (src >= V) { set_err("SSSP source %llu is not a live vertex", (unsigned long long)source_ext); return H2TAP_E_INVAL; }
+        const int64_t* off = static_cast<const int64_t*>(r->off[r->cur].p);
+        const uint32_t* cols = static_cast<const uint32_t*>(r->cols[r->cur].p);
+        const float* w = static_cast<const float*>(r->w[r->cur].p);
+        unsigned long long* cnt = r->get<unsigned long long>(r->misc, 2);
+        CK(cudaMemsetAsync(cnt, 0, 16, r->st));
+        if (E) {
+            k_sssp_check_w<<<(unsigned)std::min<uint64_t>(cdiv(E, 256 * 8), (uint64_t)r->n_sm * 8), 256, 0, r->st>>>(
+                w, E, reinterpret_cast<unsigned int*>(cnt + 1));
+            CKL();
+        }
+        double* dist = on_device ? dist_out : r->get<double>(r->pr_a, V);
+        uint32_t* stamp = r->get<uint32_t>(r->pr_b, V);
+        uint32_t* fa = r->get<uint32_t>(r->bfs_a, V);
+        uint32_t* fb = r->get<uint32_t>(r->bfs_b, V);
+        k_fill_u64<<<g1(V), 256, 0, r->st>>>(reinterpret_cast<uint64_t*>(dist), V, 0x7FF0000000000000ull);  // +inf
+        CKL();
+        CK(cudaMemsetAsync(stamp, 0, V * 4, r->st));
+        const double zero = 0.0;
+        const uint32_t s32 = (uint32_t)src;
+        CK(cudaMemcpyAsync(dist + src, &zero, 8, cudaMemcpyHostToDevice, r->st));
+        CK(cudaMemcpyAsync(fa, &s32, 4, cudaMemcpyHostToDevice, r->st));
+        unsigned long long h[2] = {0, 0};
+        CK(cudaMemcpyAsync(h, cnt, 16, cudaMemcpyDeviceToHost, r->st));
+        r->sync();
+        if (h[1]) { set_err("h2tap_sssp: negative or NaN edge weight"); return H2TAP_E_INVAL; }
+        uint64_t nf = 1;
+        for (uint32_t round = 1; nf; ++round) {
+            CK(cudaMemsetAsync(cnt, 0, 8, r->st));
+            const unsigned grid = (unsigned)std::min<uint64_t>(cdiv(nf * 32, 256), (uint64_t)r->n_sm * 32);
+            k_sssp_relax<<<grid, 256, 0, r->st>>>(off, cols, w, fa, nf, reinterpret_cast<unsigned long long*>(dist),
+                                                  stamp, round, fb, cnt);
+            CKL();
+            CK(cudaMemcpyAsync(h, cnt, 8, cudaMemcpyDeviceToHost, r->st));
+            r->sync();
+            nf = h[0];
+            std::swap(fa, fb);
+        }
+        if (!on_device) CK(cudaMemcpyAsync(dist_out, dist, V * 8, cudaMemcpyDeviceToHost, r->st));
         r->sync();
         return H2TAP_OK;
     });

@@ -1815,6 +1815,49 @@ __global__ void k_bfs_expand(const int64_t* __restrict__ off, const uint32_t* __
     }
 }
 
+// ------------------------------------------------------------------ SSSP ----
+// Frontier Bellman-Ford (reading A21): distances are fp64 bit patterns; for
+// non-negative doubles (and +inf) the unsigned order of the patterns is the numeric
+// order, so a relaxation is one 64-bit atomicMin.  A vertex whose distance dropped
+// joins the next frontier once per round (stamp).  With weights >= 0 the fixpoint
+// d(v) = min over in-edges of fl(d(u) + w) is unique, so the result equals Dijkstra's
+// bit for bit, whatever the relaxation order.
+__global__ void k_sssp_check_w(const float* __restrict__ w, uint64_t E, unsigned int* __restrict__ bad) {
+    bool b = false;
+    for (uint64_t i = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; i < E; i += (uint64_t)gridDim.x * blockDim.x) {
+        const float x = w[i];
+        b |= (x != x) || (x < 0.0f);  // NaN or negative (-0.0 passes)
+    }
+    if (__any_sync(0xffffffffu, b) && lane_id() == 0) atomicOr(bad, 1u);
+}
+__global__ void k_sssp_relax(const int64_t* __restrict__ off, const uint32_t* __restrict__ cols,
+                             const float* __restrict__ w, const uint32_t* __restrict__ front, uint64_t n_front,
+                             unsigned long long* dist, uint32_t* __restrict__ stamp, uint32_t round,
+                             uint32_t* __restrict__ next, unsigned long long* __restrict__ n_next) {
+    const uint64_t warp = (blockIdx.x * (uint64_t)blockDim.x + threadIdx.x) >> 5;
+    const uint64_t nwarps = ((uint64_t)gridDim.x * blockDim.x) >> 5;
+    for (uint64_t f = warp; f < n_front; f += nwarps) {
+        const uint32_t u = front[f];
+        const double du = __longlong_as_double((long long)ld_volatile(reinterpret_cast<const uint64_t*>(dist + u)));
+        for (int64_t e = off[u] + lane_id(); e < off[u + 1]; e += 32) {
+            const uint32_t v = cols[e];
+            const double nd = du + (double)w[e];
+            const unsigned long long nb = (unsigned long long)__double_as_longlong(nd);
+            bool push = false;
+            if (nb < ld_volatile(reinterpret_cast<const uint64_t*>(dist + v)) && atomicMin(dist + v, nb) > nb)
+                push = atomicExch(stamp + v, round) != round;
+            const uint32_t m = __ballot_sync(__activemask(), push);
+            if (push) {
+                const uint32_t leader = __ffs(m) - 1;
+                unsigned long long b = 0;
+                if (lane_id() == leader) b = atomicAdd(n_next, (unsigned long long)__popc(m));
+                b = __shfl_sync(m, b, leader);
+                next[b + __popc(m & lanemask_lt())] = v;
+            }
+        }
+    }
+}
+
 __global__ void k_fill_i32(int32_t* p, uint64_t n, int32_t v) {
     uint64_t i = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x;
     if (i < n) p[i] = v;

@@ -112,6 +112,9 @@ def test_rmat_c1_config(h2):
         assert np.array_equal(g.bfs(s), oracle.bfs(off, cols, s))
     pr_g, pr_o = g.pagerank(0.85, 20), oracle.pagerank(off, cols, 0.85, 20)
     assert np.max(np.abs(pr_g - pr_o) / pr_o) < 1e-6
+    w_new = g.export()[2]
+    for s in (0, 17, 4242):                               # SSSP: bit-exact (unique fixpoint)
+        assert np.array_equal(g.sssp(s), oracle.sssp(off, cols, w_new, s))
 
 
 def test_rmat_parity_variant_weights_repeats_txns(h2):
@@ -163,6 +166,31 @@ def test_ldbc_shaped_small(h2):
         ts = int(b.ts.max())
         st = step(g, o, b, ts, f"ldbc batch {k}")
         assert st["n_vertex_inserted"] > 0
+        # analytics on the compacted replica, sources named by external id
+        off, cols, ww, ext = g.export()
+        for d in (0, len(ext) // 3, len(ext) - 1):
+            assert np.array_equal(g.sssp(int(ext[d])), oracle.sssp(off, cols, ww, d))
+            assert np.array_equal(g.bfs(int(ext[d])), oracle.bfs(off, cols, d))
+
+
+def test_sssp_edge_cases(h2):
+    """zero / -0.0 weights, unreachable vertices, unknown source, negative and NaN weights"""
+    ids = np.array([10, 20, 30, 40, 50], np.uint64)
+    src = np.array([10, 10, 20, 30, 40], np.uint64)
+    dst = np.array([20, 30, 30, 40, 10], np.uint64)
+    w = np.array([0.0, 2.0, -0.0, 0.5, 1.0], np.float32)
+    g = h2.Replica.from_edges(5, ids, src, dst, w)
+    off, cols, ww, _ = g.export()
+    d = g.sssp(10)
+    assert np.array_equal(d, oracle.sssp(off, cols, ww, 0))
+    assert np.array_equal(d, [0.0, 0.0, 0.0, 0.5, np.inf]) and not np.signbit(d[2])
+    with pytest.raises(h2.H2tapError):
+        g.sssp(11)                                            # not a live vertex
+    for bad in (-1.0, np.nan):
+        wb = w.copy()
+        wb[3] = bad
+        with pytest.raises(h2.H2tapError):
+            h2.Replica.from_edges(5, ids, src, dst, wb).sssp(10)
 
 
 def test_empty_batch_is_identity_and_errors_leave_state(h2):

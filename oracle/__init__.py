@@ -12,6 +12,8 @@ input generator ``synth``, which holds none of the method's arithmetic).
   by their textbook definitions.
 * ``O2``  (o2_bruteforce.py): independent brute force on a flat edge list,
   used to pin O1 on exhaustive tiny cases.
+* ``expand_records``: the delta-store scan of the paper's record layout
+  (§5.1-5.2) into the flat op sequence O1 replays.
 * ``checksum``: position-keyed 64-bit checksum of an exported array (the
   comparison key for large exports; written here independently of the CUDA
   export's own checksum kernel).
@@ -140,6 +142,38 @@ class O1:
                                         np.uint64)]
         lib().o1_pending(self.h, *(_p(x) for x in a))
         return a
+
+
+def expand_records(records, inserts, weights, deletes):
+    """Delta-store scan (§5.1-§5.2) of a delta-record batch into
+    the flat ops O1 replays, plain loops in record order.  Per VALID record (P:L615-619;
+    invalid records were used in an earlier cycle and are skipped), in the order of
+    reading A22: NODE_INSERT if the record created its node, an EDGE_DELETE per entry
+    of its deletes slice, an EDGE_INSERT per entry of its inserts / weights slices
+    (P:L627-646), NODE_DELETE if its deleted flag is set.  All ops carry the
+    record's transaction timestamp.  A slice outside its array -> ValueError.
+    Returns (kind, src, dst, w, ts) lists."""
+    kind, src, dst, w, ts = [], [], [], [], []
+
+    def op(k, s, d, x, t):
+        kind.append(k); src.append(s); dst.append(d); w.append(x); ts.append(t)
+
+    for r in records:
+        if not r["valid"]:
+            continue
+        t, v = int(r["ts"]), int(r["node"])
+        io, ic, do, dc = int(r["ins_off"]), int(r["ins_cnt"]), int(r["del_off"]), int(r["del_cnt"])
+        if io + ic > len(inserts) or io + ic > len(weights) or do + dc > len(deletes):
+            raise ValueError("delta record slice outside its array")
+        if r["inserted"]:
+            op(0, v, 0, 0.0, t)                                  # NODE_INSERT
+        for j in range(dc):
+            op(3, v, int(deletes[do + j]), 0.0, t)               # EDGE_DELETE
+        for j in range(ic):
+            op(2, v, int(inserts[io + j]), float(weights[io + j]), t)  # EDGE_INSERT
+        if r["deleted"]:
+            op(1, v, 0, 0.0, t)                                  # NODE_DELETE
+    return kind, src, dst, w, ts
 
 
 def bfs(offsets, cols, source_dense: int) -> np.ndarray:

@@ -186,3 +186,77 @@ CONFIGS = {
 
 def seed_of(name: str) -> int:
     return MASTER_SEED + CONFIGS[name]["index"]
+
+
+# ------------------------------------------------- delta-record batches ----
+# The paper's delta-store layout (§5.1): fixed-size delta records
+# (transaction timestamp, node ID, validity and deleted flags, offsets + counts
+# into the inserts / weights / deletes arrays).  This module only PACKS op
+# sequences into that layout (input production); the expansion back into ops is
+# the method's scan and lives on each side separately (oracle/, the CUDA path).
+RECORD_DTYPE = np.dtype([("ts", "<u8"), ("node", "<u8"), ("ins_off", "<u8"), ("del_off", "<u8"),
+                         ("ins_cnt", "<u4"), ("del_cnt", "<u4"), ("valid", "u1"), ("deleted", "u1"),
+                         ("inserted", "u1"), ("pad", "u1", (5,))])
+assert RECORD_DTYPE.itemsize == 48
+
+
+@dataclass
+class RecordBatch:
+    """h2tap_record_batch layout: records (RECORD_DTYPE) + inserts u64 / weights f32 / deletes u64."""
+    records: np.ndarray
+    inserts: np.ndarray
+    weights: np.ndarray
+    deletes: np.ndarray
+
+    def __len__(self) -> int:
+        return int(self.records.shape[0])
+
+    def nbytes(self) -> int:
+        return sum(a.nbytes for a in (self.records, self.inserts, self.weights, self.deletes))
+
+
+_PHASE = {NODE_INSERT: 0, EDGE_DELETE: 1, EDGE_INSERT: 2, NODE_DELETE: 3}
+
+
+def records_from_ops(b: Batch) -> RecordBatch:
+    """Pack consecutive ops of one transaction (same ts) on one node into one record,
+    in the order a record expands to (reading A22): [NODE_INSERT] EDGE_DELETE* EDGE_INSERT*
+    [NODE_DELETE], each destination at most once per record.  A new record starts
+    wherever that order would break, so expanding the records yields `b` op for op.
+    EDGE_WEIGHT has no record form (the paper's four update types)."""
+    n = len(b)
+    if n and np.any(b.kind == EDGE_WEIGHT):
+        raise ValueError("EDGE_WEIGHT ops have no delta-record form")
+    kind = b.kind.astype(np.int64)
+    ph = np.zeros(n, np.int64)
+    for k, p in _PHASE.items():
+        ph[kind == k] = p
+    cut = np.ones(n, bool)
+    if n > 1:
+        cut[1:] = ((b.ts[1:] != b.ts[:-1]) | (b.src[1:] != b.src[:-1]) | (ph[1:] < ph[:-1]) |
+                   ((ph[1:] == ph[:-1]) & ((ph[1:] == 0) | (ph[1:] == 3))))
+    edge = (kind == EDGE_INSERT) | (kind == EDGE_DELETE)
+    while True:  # split a record where a destination repeats
+        gid = np.cumsum(cut) - 1
+        e = np.flatnonzero(edge)
+        o = e[np.lexsort((e, b.dst[e], gid[e]))]
+        dup = (gid[o[1:]] == gid[o[:-1]]) & (b.dst[o[1:]] == b.dst[o[:-1]])
+        if not dup.any():
+            break
+        cut[o[1:][dup]] = True
+    gid = np.cumsum(cut) - 1
+    nr = int(cut.sum())
+    rec = np.zeros(nr, RECORD_DTYPE)
+    starts = np.flatnonzero(cut)
+    rec["ts"] = b.ts[starts]
+    rec["node"] = b.src[starts]
+    rec["valid"] = 1
+    ins = np.flatnonzero(kind == EDGE_INSERT)
+    dl = np.flatnonzero(kind == EDGE_DELETE)
+    rec["ins_cnt"] = np.bincount(gid[ins], minlength=nr)
+    rec["del_cnt"] = np.bincount(gid[dl], minlength=nr)
+    rec["ins_off"] = np.concatenate([[0], np.cumsum(rec["ins_cnt"].astype(np.uint64))[:-1]]) if nr else []
+    rec["del_off"] = np.concatenate([[0], np.cumsum(rec["del_cnt"].astype(np.uint64))[:-1]]) if nr else []
+    rec["inserted"][gid[kind == NODE_INSERT]] = 1
+    rec["deleted"][gid[kind == NODE_DELETE]] = 1
+    return RecordBatch(rec, b.dst[ins].copy(), b.w[ins].copy(), b.dst[dl].copy())

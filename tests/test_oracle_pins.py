@@ -367,3 +367,57 @@ def test_sssp_brute_force_closed_forms_and_errors():
         oracle.sssp(off, cols, np.array([1, -1, 1, 1, 1, 1], np.float32), 0)
     with pytest.raises(ValueError):
         oracle.sssp(off, cols, np.array([1, np.nan, 1, 1, 1, 1], np.float32), 0)
+
+
+# ------------------------------------------------- delta-record batches ----
+def load_fig2_records():
+    g = json.load(open(os.path.join(HERE, "golden", "fig2_records.json")))
+    rec = np.zeros(len(g["records"]), synth.RECORD_DTYPE)
+    for i, r in enumerate(g["records"]):
+        for k, v in r.items():
+            rec[k][i] = v
+
+    def arr(spec, dt):
+        a = np.full(spec["size"], spec["fill"], dt)
+        for k, v in spec["set"].items():
+            a[int(k)] = v
+        return a
+    rb = synth.RecordBatch(rec, arr(g["inserts"], np.uint64), arr(g["weights"], np.float32),
+                           arr(g["deletes"], np.uint64))
+    return g, rb
+
+
+def test_fig2_records_worked_example():
+    g, rb = load_fig2_records()
+    e = np.array(g["edges"], dtype=object)
+    o = O1.from_edges(len(g["vertices"]), np.array(g["vertices"], np.uint64),
+                      np.array(e[:, 0], np.uint64), np.array(e[:, 1], np.uint64),
+                      np.array(e[:, 2], np.float32), g["create_ts"])
+    ops = list(zip(*oracle.expand_records(rb.records, rb.inserts, rb.weights, rb.deletes)))
+    assert len(ops) == 7                                      # the invalid record is skipped
+    rc, st = o.apply(Batch.of(ops), g["snapshot_ts"])
+    assert rc == 0
+    off, cols, w, ids = o.export()
+    ex = g["expected"]
+    assert ids.tolist() == ex["ext_ids"] and off.tolist() == ex["offsets"]
+    assert cols.tolist() == ex["cols"] and w.tolist() == ex["weights"]
+
+
+def test_records_round_trip_and_bounds():
+    for k in range(6):
+        b = synth.fuzz_batch(seed=3, k=k, n=3000, n_ids=40, probs=(0.05, 0.03, 0.6, 0.32, 0.0),
+                             ts_lo=1, ts_span=300)
+        b = b.slice(np.lexsort((b.src, b.ts)))                # transactions grouped by node
+        rb = synth.records_from_ops(b)
+        assert len(rb) < len(b)                               # some ops share a record
+        kind, src, dst, w, ts = oracle.expand_records(rb.records, rb.inserts, rb.weights, rb.deletes)
+        assert np.array_equal(np.array(kind, np.uint8), b.kind) and np.array_equal(np.array(ts, np.uint64), b.ts)
+        assert np.array_equal(np.array(src, np.uint64), b.src)
+        e = (b.kind == EDGE_INSERT) | (b.kind == EDGE_DELETE)
+        assert np.array_equal(np.array(dst, np.uint64)[e], b.dst[e])
+        ins = b.kind == EDGE_INSERT
+        assert np.array_equal(np.array(w, np.float32)[ins], b.w[ins])
+    g, rb = load_fig2_records()
+    rb.records["del_cnt"][3] = 4                              # slice past the end of deletes
+    with pytest.raises(ValueError):
+        oracle.expand_records(rb.records, rb.inserts, rb.weights, rb.deletes)

@@ -145,6 +145,43 @@ h2tap_status h2tap_replica_create_from_csr(const h2tap_config* cfg, size_t n_ver
 h2tap_status h2tap_delta_apply(h2tap_replica* r, const h2tap_batch* batch, uint64_t snapshot_ts,
         h2tap_apply_stats* stats /* nullable */);
 
+/* ---- the paper's delta-store layout as a second input format ----
+ * Delta records (§5.1 "Delta Store Architecture"): fixed-size records of
+ * (transaction timestamp, node ID, validity flag, deleted flag, offset + count into the
+ * inserts / weights arrays, offset + count into the deletes array); the destinations and
+ * weights of a record's inserted relationships, and the destinations of its deleted ones,
+ * live in three shared arrays (the CSR-like layout of Fig. 2).  `inserted` marks a record
+ * whose transaction created its node (the paper implies it by a record for a new node ID,
+ * P:L670-676; reading A22). */
+typedef struct {
+    uint64_t ts;                /* commit timestamp of the appending transaction */
+    uint64_t node;              /* external ID of the updated node */
+    uint64_t ins_off, del_off;  /* first index in inserts[]/weights[] and in deletes[] */
+    uint32_t ins_cnt, del_cnt;  /* slice lengths */
+    uint8_t valid;              /* 0: used in an earlier cycle, skipped */
+    uint8_t deleted;            /* node deleted: all its relationships go */
+    uint8_t inserted;           /* node created by this transaction (reading A22) */
+    uint8_t pad[5];
+} h2tap_delta_record;           /* 48 bytes */
+
+typedef struct {  /* all arrays caller-owned, read-only, not retained; host or device */
+    size_t n_records; int on_device;
+    const h2tap_delta_record* records;
+    const uint64_t* inserts; const float* weights; size_t n_inserts;
+    const uint64_t* deletes; size_t n_deletes;
+} h2tap_record_batch;
+
+/* One propagation cycle from delta records: the delta-store scan (§5.2)
+ * runs on the GPU — every valid record expands, at its timestamp and in record order,
+ * into [NODE_INSERT] EDGE_DELETE* EDGE_INSERT* [NODE_DELETE] (reading A22) — and the
+ * resulting ops are applied exactly as h2tap_delta_apply applies a flat batch (same
+ * visibility, pending and error rules; each expanded op is one update in the stats).
+ * The caller marks the records it passed as used; records with ts >
+ * snapshot_ts stay pending inside the replica.  A record slice outside its array or a
+ * flag other than 0/1 -> E_INVAL (nothing applied). */
+h2tap_status h2tap_delta_apply_records(h2tap_replica* r, const h2tap_record_batch* batch,
+        uint64_t snapshot_ts, h2tap_apply_stats* stats /* nullable */);
+
 /* ---- exchange step of a sharded apply ----------------------
  * A rank holding a slice of the global batch (i) validates it (every rank must agree
  * before anything is applied), (ii) packs its ops into 40-byte route records grouped

@@ -59,6 +59,15 @@ class _Batch(ctypes.Structure):
                 ("dst", _P), ("weight", _P), ("ts", _P), ("seq", _P)]
 
 
+class _RecordBatch(ctypes.Structure):
+    _fields_ = [("n_records", ctypes.c_size_t), ("on_device", ctypes.c_int), ("records", _P),
+                ("inserts", _P), ("weights", _P), ("n_inserts", ctypes.c_size_t),
+                ("deletes", _P), ("n_deletes", ctypes.c_size_t)]
+
+
+RECORD_BYTES = 48  # sizeof(h2tap_delta_record)
+
+
 class ApplyStats(ctypes.Structure):
     _fields_ = [(n, _u64) for n in ("n_visible", "n_deferred", "n_gated", "n_new", "n_del", "n_upd",
                                     "n_casc", "n_vertex_inserted", "n_vertex_deleted")] + \
@@ -80,6 +89,8 @@ _lib.h2tap_replica_create_from_csr.argtypes = [ctypes.POINTER(_Config), ctypes.c
                                                _P, ctypes.c_int, _u64, ctypes.POINTER(_P)]
 _lib.h2tap_delta_apply.restype = ctypes.c_int
 _lib.h2tap_delta_apply.argtypes = [_P, ctypes.POINTER(_Batch), _u64, ctypes.POINTER(ApplyStats)]
+_lib.h2tap_delta_apply_records.restype = ctypes.c_int
+_lib.h2tap_delta_apply_records.argtypes = [_P, ctypes.POINTER(_RecordBatch), _u64, ctypes.POINTER(ApplyStats)]
 _lib.h2tap_batch_validate.restype = ctypes.c_int
 _lib.h2tap_batch_validate.argtypes = [_P, ctypes.POINTER(_Batch)]
 _lib.h2tap_route_pack.restype = ctypes.c_int
@@ -277,6 +288,28 @@ class Replica:
         rc = _lib.h2tap_delta_apply(self._h, ctypes.byref(b), int(snapshot_ts), ctypes.byref(st))
         if raise_on_error:
             _check(rc, "h2tap_delta_apply")
+            return st.as_dict()
+        return rc, st.as_dict()
+
+    def apply_records(self, rb, snapshot_ts: int, raise_on_error: bool = True):
+        """h2tap_delta_apply_records; rb has .records (48-byte records: a numpy structured
+        array, or a torch CUDA uint8 tensor) .inserts .weights .deletes."""
+        pr, pi, pw, pd = (_ptr(rb.records), _ptr(rb.inserts, np.uint64), _ptr(rb.weights, np.float32),
+                          _ptr(rb.deletes, np.uint64))
+        b = _RecordBatch()
+        recs = pr[2]
+        nbytes = recs.numel() * recs.element_size() if _is_torch(recs) else recs.nbytes
+        if nbytes % RECORD_BYTES:
+            raise ValueError("records buffer is not a whole number of 48-byte records")
+        b.n_records = nbytes // RECORD_BYTES
+        b.on_device = _on_device(pr, pi, pw, pd)
+        b.records, b.inserts, b.weights, b.deletes = pr[0], pi[0], pw[0], pd[0]
+        b.n_inserts = len(pi[2]) if pi[2] is not None else 0
+        b.n_deletes = len(pd[2]) if pd[2] is not None else 0
+        st = ApplyStats()
+        rc = _lib.h2tap_delta_apply_records(self._h, ctypes.byref(b), int(snapshot_ts), ctypes.byref(st))
+        if raise_on_error:
+            _check(rc, "h2tap_delta_apply_records")
             return st.as_dict()
         return rc, st.as_dict()
 

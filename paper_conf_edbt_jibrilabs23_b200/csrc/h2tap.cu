@@ -128,6 +128,7 @@ struct h2tap_replica {
     Buf op_flags, op_ou, op_ow;
     Buf ins_pos, ins_row, ins_col, ins_w, del_pos, upd_pos, upd_w, KR;
     Buf misc, nsorted, part, opart, deg, tsum, remap_shift, remap32, casc_wrel, tile_emit, tile_base, del_row, casc_mask, status2, bfs_a, bfs_b, pr_a, pr_b;
+    Buf xrec, xins, xwts, xdel, xcnt, xoff;  // delta-record input (h2tap_delta_apply_records)
     Buf ctr;
     Counters* hc = nullptr;  // pinned host mirror
     cudaEvent_t ev[8]{};
@@ -223,6 +224,12 @@ struct BatchIn {
     const uint64_t* ts;   // NULL -> all create_ts (create)
     uint64_t fill_ts;
     const RouteRec* recs = nullptr;  // routed records (device) instead of the SoA arrays
+    // delta records (device) instead of the SoA arrays: n = their expanded op count
+    const DeltaRec* drec = nullptr;
+    uint64_t n_drec = 0;
+    const uint64_t *drec_off = nullptr, *dins = nullptr, *ddel = nullptr;
+    const float* dwts = nullptr;
+    uint64_t pre_h2d = 0, pre_d2h = 0, pre_launches = 0;  // accounting of the record pre-pass
 };
 
 template <typename T>
@@ -275,7 +282,9 @@ h2tap_status apply_core(h2tap_replica* r, const BatchIn& in, uint64_t S, bool cr
     cudaStream_t st = r->st;
     const uint64_t n = in.n, np = r->n_pend, m = np + n;
     if (m >= 0xFFFFFFFFull) { set_err("batch + pending = %llu ops exceeds 2^32-1", (unsigned long long)m); return H2TAP_E_CAPACITY; }
-    g_launches = g_h2d = g_d2h = 0;
+    g_launches = in.pre_launches;
+    g_h2d = in.pre_h2d;
+    g_d2h = in.pre_d2h;
     g_tr.init();
     for (int i = 0; i < 8; ++i)
         if (!r->ev[i]) CK(cudaEventCreate(&r->ev[i]));
@@ -300,6 +309,13 @@ h2tap_status apply_core(h2tap_replica* r, const BatchIn& in, uint64_t S, bool cr
     }
     if (n && in.recs) {
         k_unpack_recs<<<g1(n), 256, 0, st>>>(in.recs, n, Wk + np, Ws + np, Wd + np, Ww + np, Wt + np, Wq + np);
+        CKL();
+    } else if (n && in.drec) {
+        const unsigned grid = (unsigned)std::min<uint64_t>(cdiv(in.n_drec * 32, 256), (uint64_t)r->n_sm * 16);
+        k_rec_expand<<<grid, 256, 0, st>>>(in.drec, in.n_drec, in.drec_off, in.dins, in.dwts, in.ddel,
+                                           Wk + np, Ws + np, Wd + np, Ww + np, Wt + np);
+        CKL();
+        k_fill_seq<<<g1(n), 256, 0, st>>>(Wq, np, n, r->next_seq);
         CKL();
     } else if (n) {
         if (in.kind) copy_in(r, Wk + np, in.kind, n, in.on_device);
@@ -794,7 +810,8 @@ void free_replica(h2tap_replica* r) {
                    &r->hist, &r->dbase, &r->rs_status, &r->rs_ctr, &r->nv, &r->nv_ext, &r->dropped, &r->ins_q,
                    &r->ins_oldpos, &r->hd_rows, &r->hd_bits, &r->op_flags, &r->op_ou, &r->op_ow,
                    &r->ins_pos, &r->ins_row, &r->ins_col, &r->ins_w, &r->del_pos, &r->upd_pos, &r->upd_w,
-                   &r->KR, &r->misc, &r->nsorted, &r->part, &r->opart, &r->deg, &r->tsum, &r->remap_shift, &r->remap32, &r->casc_wrel, &r->tile_emit, &r->tile_base, &r->del_row, &r->casc_mask, &r->status2, &r->bounds_dev, &r->fence[0], &r->fence[1], &r->bfs_a, &r->bfs_b, &r->pr_a, &r->pr_b, &r->ctr};
+                   &r->KR, &r->misc, &r->nsorted, &r->part, &r->opart, &r->deg, &r->tsum, &r->remap_shift, &r->remap32, &r->casc_wrel, &r->tile_emit, &r->tile_base, &r->del_row, &r->casc_mask, &r->status2, &r->bounds_dev, &r->fence[0], &r->fence[1], &r->bfs_a, &r->bfs_b, &r->pr_a, &r->pr_b, &r->ctr,
+                   &r->xrec, &r->xins, &r->xwts, &r->xdel, &r->xcnt, &r->xoff};
     for (Buf* b : bufs) if (b->p) r->dfree(b->p);
     cudaStreamSynchronize(r->st);
     for (auto& e : r->ev) if (e) cudaEventDestroy(e);
@@ -1010,6 +1027,74 @@ h2tap_status h2tap_route_pack(const h2tap_replica* rc, const h2tap_batch* b, uin
         }
         r->sync();
         return H2TAP_OK;
+    });
+}
+
+h2tap_status h2tap_delta_apply_records(h2tap_replica* r, const h2tap_record_batch* b, uint64_t snapshot_ts,
+                                       h2tap_apply_stats* stats) {
+    if (!r || !b) { set_err("null argument"); return H2TAP_E_INVAL; }
+    if (b->n_records && !b->records) { set_err("records must be non-NULL"); return H2TAP_E_INVAL; }
+    if ((b->n_inserts && (!b->inserts || !b->weights)) || (b->n_deletes && !b->deletes)) {
+        set_err("inserts/weights/deletes must be non-NULL when their size is non-zero");
+        return H2TAP_E_INVAL;
+    }
+    return run_guarded(r, [&]() -> h2tap_status {
+        if (snapshot_ts < r->snap) {
+            set_err("snapshot_ts %llu < current %llu", (unsigned long long)snapshot_ts, (unsigned long long)r->snap);
+            return H2TAP_E_SNAPSHOT_REGRESSION;
+        }
+        CK(cudaSetDevice(r->cfg.device));
+        cudaStream_t st = r->st;
+        g_launches = g_h2d = g_d2h = 0;
+        if (!r->ev[7]) CK(cudaEventCreate(&r->ev[7]));
+        CK(cudaEventRecord(r->ev[7], st));
+        const uint64_t nr = b->n_records;
+        const DeltaRec* rec = reinterpret_cast<const DeltaRec*>(b->records);
+        const uint64_t *ins = b->inserts, *del = b->deletes;
+        const float* wts = b->weights;
+        if (!b->on_device) {  // the scan reads the records where they live: copy them in once
+            DeltaRec* xr = r->get<DeltaRec>(r->xrec, nr);
+            copy_in(r, xr, rec, nr, 0);
+            rec = xr;
+            uint64_t* xi = r->get<uint64_t>(r->xins, b->n_inserts);
+            float* xw = r->get<float>(r->xwts, b->n_inserts);
+            uint64_t* xd = r->get<uint64_t>(r->xdel, b->n_deletes);
+            copy_in(r, xi, ins, b->n_inserts, 0);
+            copy_in(r, xw, wts, b->n_inserts, 0);
+            copy_in(r, xd, del, b->n_deletes, 0);
+            ins = xi; wts = xw; del = xd;
+        }
+        uint64_t* cnt = r->get<uint64_t>(r->xcnt, nr + 1);
+        uint64_t* off = r->get<uint64_t>(r->xoff, nr + 1);
+        unsigned long long* tb = r->get<unsigned long long>(r->misc, 2);
+        CK(cudaMemsetAsync(tb, 0, 16, st));
+        if (nr) {
+            k_rec_count<<<g1(nr), 256, 0, st>>>(rec, nr, b->n_inserts, b->n_deletes, cnt, tb);
+            CKL();
+            const uint64_t nt = cdiv(nr, kTile);
+            uint64_t* stt = r->get<uint64_t>(r->status2, nt);
+            unsigned int* ctr = reinterpret_cast<unsigned int*>(r->get<uint64_t>(r->tsum, 1));
+            CK(cudaMemsetAsync(stt, 0, nt * 8, st));
+            CK(cudaMemsetAsync(ctr, 0, 4, st));
+            k_scan_exclusive_u64<<<(unsigned)nt, kThreads, 0, st>>>(cnt, off, nr, stt, ctr);
+            CKL();
+        }
+        unsigned long long h[2] = {0, 0};
+        CK(cudaMemcpyAsync(h, tb, 16, cudaMemcpyDeviceToHost, st));
+        g_d2h += 16;
+        r->sync();  // the expanded op count sizes the work buffers
+        if (h[1] & REC_BAD_FLAG) { set_err("delta record flag other than 0/1"); return H2TAP_E_INVAL; }
+        if (h[1] & REC_BAD_SLICE) { set_err("delta record slice outside the inserts/weights/deletes arrays"); return H2TAP_E_INVAL; }
+        BatchIn in{h[0], 1, nullptr, nullptr, nullptr, nullptr, nullptr, nullptr, 0};
+        in.drec = rec; in.n_drec = nr; in.drec_off = off; in.dins = ins; in.dwts = wts; in.ddel = del;
+        in.pre_h2d = g_h2d; in.pre_d2h = g_d2h; in.pre_launches = g_launches;
+        const h2tap_status s = apply_core(r, in, snapshot_ts, false, stats);
+        if (s == H2TAP_OK && stats) {  // the scan pre-pass is part of ingest
+            const float pre = ev_ms(r->ev[7], r->ev[0]);
+            stats->ms_ingest += pre;
+            stats->ms_total += pre;
+        }
+        return s;
     });
 }
 

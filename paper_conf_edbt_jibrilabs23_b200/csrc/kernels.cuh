@@ -309,6 +309,66 @@ __global__ void k_unpack_recs(const RouteRec* __restrict__ recs, uint64_t n, uin
     kind[i] = r.kind; src[i] = r.src; dst[i] = r.dst; w[i] = r.w; ts[i] = r.ts; seq[i] = r.seq;
 }
 
+// ============================================================ a1 records ====
+// Delta-store scan of the paper's delta-record layout (§5.1-§5.2, P:L604-661,
+// P:L702-725): each valid record expands, in the order of reading
+// A22, into [NODE_INSERT] EDGE_DELETE* EDGE_INSERT* [NODE_DELETE] at the record's
+// transaction timestamp.  Pass 1 counts (and validates) the ops of every record,
+// an exclusive scan places them, pass 2 writes them into the work-op SoA.
+struct DeltaRec {  // layout of h2tap_delta_record
+    uint64_t ts, node, ins_off, del_off;
+    uint32_t ins_cnt, del_cnt;
+    uint8_t valid, deleted, inserted, pad[5];
+};
+static_assert(sizeof(DeltaRec) == 48, "delta record layout");
+enum : uint32_t { REC_BAD_SLICE = 1, REC_BAD_FLAG = 2 };
+__global__ void k_rec_count(const DeltaRec* __restrict__ rec, uint64_t n, uint64_t n_ins, uint64_t n_del,
+                            uint64_t* __restrict__ cnt, unsigned long long* __restrict__ tot_bad) {
+    const uint64_t i = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x;
+    uint64_t c = 0;
+    uint32_t bad = 0;
+    if (i < n) {
+        const DeltaRec r = rec[i];
+        if (r.valid > 1 || r.deleted > 1 || r.inserted > 1) bad |= REC_BAD_FLAG;
+        if (r.valid) {
+            if (r.ins_off > n_ins || r.ins_cnt > n_ins - r.ins_off || r.del_off > n_del || r.del_cnt > n_del - r.del_off)
+                bad |= REC_BAD_SLICE;
+            c = (uint64_t)r.inserted + r.del_cnt + r.ins_cnt + r.deleted;
+        }
+        cnt[i] = c;
+    }
+    const unsigned long long s = warp_sum<unsigned long long>(c);
+    const uint32_t b = __reduce_or_sync(0xffffffffu, bad);
+    if (lane_id() == 0) {
+        if (s) atomicAdd(&tot_bad[0], s);
+        if (b) atomicOr(&tot_bad[1], (unsigned long long)b);
+    }
+}
+// one warp per record (a record may carry thousands of inserts of a hub node)
+__global__ void k_rec_expand(const DeltaRec* __restrict__ rec, uint64_t n, const uint64_t* __restrict__ off,
+                             const uint64_t* __restrict__ ins, const float* __restrict__ wts,
+                             const uint64_t* __restrict__ del, uint8_t* __restrict__ kind, uint64_t* __restrict__ src,
+                             uint64_t* __restrict__ dst, float* __restrict__ w, uint64_t* __restrict__ ts) {
+    const uint64_t warp = (blockIdx.x * (uint64_t)blockDim.x + threadIdx.x) >> 5;
+    const uint64_t nwarps = ((uint64_t)gridDim.x * blockDim.x) >> 5;
+    for (uint64_t i = warp; i < n; i += nwarps) {
+        const DeltaRec r = rec[i];
+        if (!r.valid) continue;
+        const uint64_t o = off[i];
+        const uint32_t a = r.inserted, b = a + r.del_cnt, c = b + r.ins_cnt, e = c + r.deleted;
+        for (uint32_t j = lane_id(); j < e; j += 32) {
+            uint8_t k;
+            uint64_t d = 0;
+            float x = 0.f;
+            if (j < a) k = NODE_INSERT;
+            else if (j < b) { k = EDGE_DELETE; d = del[r.del_off + (j - a)]; }
+            else if (j < c) { k = EDGE_INSERT; d = ins[r.ins_off + (j - b)]; x = wts[r.ins_off + (j - b)]; }
+            else k = NODE_DELETE;
+            kind[o + j] = k; src[o + j] = r.node; dst[o + j] = d; w[o + j] = x; ts[o + j] = r.ts;
+        }
+    }
+}
+
 // ===================================================================== a2 ====
 // Unique vertices of the (v, ts, seq)-sorted visible node ops: final liveness
 // (last op), latest delete point tD, old presence.  Compaction via look-back.

@@ -260,11 +260,22 @@ def run_gpu(args):
     glob_n = [len(b) for b in glob]
     del glob
 
+    records = args.input == "records"
+    if records and sharded:
+        raise SystemExit("--input records is single-replica only")
+
+    def tens(a):
+        return torch.from_numpy(a.view(np.uint8) if a.dtype.fields else a.view(np.int64) if a.dtype == np.uint64 else a)
+
     def to_dev(b):
-        return synth.Batch(*(torch.from_numpy(a.view(np.int64) if a.dtype == np.uint64 else a).cuda()
-                             for a in (b.kind, b.src, b.dst, b.w, b.ts)))
+        if records:
+            rb = synth.records_from_ops(b)
+            return synth.RecordBatch(*(tens(a).cuda() for a in (rb.records, rb.inserts, rb.weights, rb.deletes)))
+        return synth.Batch(*(tens(a).cuda() for a in (b.kind, b.src, b.dst, b.w, b.ts)))
 
     def apply(b, snap):
+        if records:
+            return rep.apply_records(b, snap)
         if not sharded:
             return rep.apply(b, snap)
         l0 = eng.launches
@@ -314,8 +325,10 @@ def run_gpu(args):
     del e_glob
 
     def pinned(b):
-        return synth.Batch(*(torch.from_numpy(a.view(np.int64) if a.dtype == np.uint64 else a).pin_memory()
-                             for a in (b.kind, b.src, b.dst, b.w, b.ts)))
+        if records:
+            rb = synth.records_from_ops(b)
+            return synth.RecordBatch(*(tens(a).pin_memory() for a in (rb.records, rb.inserts, rb.weights, rb.deletes)))
+        return synth.Batch(*(tens(a).pin_memory() for a in (b.kind, b.src, b.dst, b.w, b.ts)))
 
     e_pin = [pinned(b) for b in e_host]
     torch.cuda.synchronize()
@@ -334,6 +347,24 @@ def run_gpu(args):
     e_updates = (sum(e_glob_n) / world if sharded else sum(s["n_visible"] for s in e_stats))
     e_ms, e_updates = reduce_max_sum(e_ms, e_updates)
     e_value = e_updates / (e_ms / 1e3)
+
+    checks = None
+    if args.checks and not sharded:  # freshness checks on the final snapshot (not in updates/s)
+        checks = {"timing": "host wall clock of one call after one warm call, incl. D2H of the result"}
+        off_h, _, _, ext_h = rep.export()
+        ext0 = int(ext_h[int(np.argmax(np.diff(off_h)))]) if len(ext_h) else None  # the top hub
+        del off_h, ext_h
+        checks["source_ext"] = ext0
+        for name, fn in (("bfs", lambda: rep.bfs(ext0)), ("sssp", lambda: rep.sssp(ext0)),
+                         ("pagerank_20", lambda: rep.pagerank(0.85, 20))):
+            if ext0 is None and name != "pagerank_20":
+                continue
+            fn()  # warm
+            torch.cuda.synchronize()
+            t = time.perf_counter()
+            fn()
+            torch.cuda.synchronize()
+            checks[name + "_ms"] = (time.perf_counter() - t) * 1e3
 
     if rank == 0:
         peak, peak_src = peaks()
@@ -376,6 +407,10 @@ def run_gpu(args):
                     "d2h_bytes_per_step": int(sum(s["d2h_bytes"] for s in e_stats) / len(e_stats))},
             "clocks": clk.summary(),
         }
+        if records:
+            line["config"]["input"] = "delta records (paper §5.1 layout, h2tap_delta_apply_records)"
+        if checks:
+            line["checks"] = checks
         if not args.no_cpu_baseline:
             v, sample, _ = oracle_sample(args.config, 3, 1, target_s=8.0)
             line["cpu_baseline"] = {"value": v, "unit": "updates/s", "cores": 1, "kind": "oracle",
@@ -394,6 +429,11 @@ def main():
     ap.add_argument("--config", default="c2", choices=sorted(synth.CONFIGS))
     ap.add_argument("--impl", default="h2tap", choices=["h2tap", "reference"])
     ap.add_argument("--no-cpu-baseline", action="store_true")
+    ap.add_argument("--input", default="ops", choices=["ops", "records"],
+                    help="batch format: flat op SoA (h2tap_delta_apply) or the paper's delta records "
+                         "(h2tap_delta_apply_records, §5.1 layout)")
+    ap.add_argument("--checks", action="store_true",
+                    help="after the timed region, time the freshness checks (BFS, SSSP, PageRank) once")
     ap.add_argument("--parallelism", default="shard", choices=["shard", "replicas"],
                     help="N > 1: shard one graph (default) or run independent replicas")
     ap.add_argument("--dist-backend", default="nccl", choices=["nccl", "gloo"],

@@ -56,6 +56,8 @@ def lib():
         P, u64, sz = ctypes.c_void_p, ctypes.c_uint64, ctypes.c_size_t
         L.o1_new.restype = P
         L.o1_new.argtypes = [u64]
+        L.o1_set_tombstone.argtypes = [P]
+        L.o1_live.argtypes = [P, P]
         L.o1_destroy.argtypes = [P]
         L.o1_load_edges.restype = ctypes.c_int
         L.o1_load_edges.argtypes = [P, sz, P, sz, P, P, P]
@@ -86,8 +88,10 @@ def _c(a, dt):
 class O1:
     """Sequential-replay oracle replica (std::map adjacency)."""
 
-    def __init__(self, create_ts: int = 0):
+    def __init__(self, create_ts: int = 0, tombstone: bool = False):
         self.h = lib().o1_new(create_ts)
+        if tombstone:  # reading A23: deleted nodes keep their id and an empty row
+            lib().o1_set_tombstone(self.h)
 
     def __del__(self):
         if getattr(self, "h", None):
@@ -95,8 +99,8 @@ class O1:
             self.h = None
 
     @staticmethod
-    def from_edges(n_vertices, vertex_ids, src, dst, w, create_ts=0) -> "O1":
-        g = O1(create_ts)
+    def from_edges(n_vertices, vertex_ids, src, dst, w, create_ts=0, tombstone=False) -> "O1":
+        g = O1(create_ts, tombstone)
         ids = _c(vertex_ids, np.uint64)
         src, dst, w = _c(src, np.uint64), _c(dst, np.uint64), _c(w, np.float32)
         rc = lib().o1_load_edges(g.h, n_vertices, _p(ids), len(src), _p(src), _p(dst), _p(w))
@@ -120,6 +124,12 @@ class O1:
         rc = lib().o1_apply(self.h, len(k), _p(k), _p(s), _p(d), _p(w), _p(t), snapshot_ts,
                             ctypes.byref(st))
         return rc, {"n_visible": st.n_visible, "n_deferred": st.n_deferred}
+
+    def live(self) -> np.ndarray:
+        """u8 liveness of every exported vertex (all 1 unless tombstone mode)"""
+        out = np.empty(self.info()["n_vertices"], np.uint8)
+        lib().o1_live(self.h, _p(out))
+        return out
 
     def info(self):
         v = [ctypes.c_uint64() for _ in range(4)]

@@ -60,13 +60,15 @@ struct Graph {
     std::vector<Op> pending;
     std::map<uint64_t, std::map<uint64_t, float>> adj;  // live vertex -> (dst -> weight)
     std::map<uint64_t, std::set<uint64_t>> rin;          // reverse index (makes R2 plain)
+    bool tombstone = false;   // reading A23: deleted nodes keep their id and an empty row
+    std::set<uint64_t> dead;  // tombstoned ids (tombstone mode only)
 };
 
 // The fold: one op applied to the current state (SURVEY.md §8(c) rules R1-R5).
 void fold(Graph& g, const Op& o) {
     switch (o.kind) {
-    case NODE_INSERT:  // R1: insert of a live node is a no-op (A12)
-        if (!g.adj.count(o.src)) { g.adj[o.src]; g.rin[o.src]; }
+    case NODE_INSERT:  // R1: insert of a live node is a no-op (A12); revives a tombstone (A23)
+        if (!g.adj.count(o.src)) { g.adj[o.src]; g.rin[o.src]; g.dead.erase(o.src); }
         break;
     case NODE_DELETE: {  // R2: remove the node and every in- and out-edge (A8)
         auto it = g.adj.find(o.src);
@@ -75,6 +77,7 @@ void fold(Graph& g, const Op& o) {
         for (auto& kv : it->second) if (kv.first != o.src) g.rin[kv.first].erase(o.src);
         g.adj.erase(it);
         g.rin.erase(o.src);
+        if (g.tombstone) g.dead.insert(o.src);  // A23: id kept, row empty
         break;
     }
     case EDGE_INSERT:  // R3: upsert when both endpoints are live (A2, A13)
@@ -114,6 +117,28 @@ void* o1_new(uint64_t create_ts) {
 }
 
 void o1_destroy(void* h) { delete static_cast<Graph*>(h); }
+
+/* Tombstone-row mode (the paper's merge(): a deleted node keeps "an empty entry",
+ * P:L879-881; reading A23).  Set before any load/apply. */
+void o1_set_tombstone(void* h) { static_cast<Graph*>(h)->tombstone = true; }
+
+/* all ids of the export (live and tombstoned) ascending, in the export's order */
+static std::vector<std::pair<uint64_t, bool>> export_ids(const Graph& g) {
+    std::vector<std::pair<uint64_t, bool>> v;
+    auto a = g.adj.begin();
+    auto d = g.dead.begin();
+    while (a != g.adj.end() || d != g.dead.end()) {
+        if (d == g.dead.end() || (a != g.adj.end() && a->first < *d)) { v.push_back({a->first, true}); ++a; }
+        else { v.push_back({*d, false}); ++d; }
+    }
+    return v;
+}
+
+/* liveness of every exported vertex (1 live, 0 tombstoned) */
+void o1_live(void* h, uint8_t* live) {
+    size_t i = 0;
+    for (auto& x : export_ids(*static_cast<Graph*>(h))) live[i++] = x.second ? 1 : 0;
+}
 
 /* Create: vertex set (strictly increasing ids, or 0..nv-1 if ids == NULL), then
  * the edges inserted in order, last duplicate wins (A17).  Edges must join
@@ -178,28 +203,32 @@ void o1_info(void* h, uint64_t* nv, uint64_t* ne, uint64_t* snap, uint64_t* npen
     Graph& g = *static_cast<Graph*>(h);
     uint64_t m = 0;
     for (auto& kv : g.adj) m += kv.second.size();
-    if (nv) *nv = g.adj.size();
+    if (nv) *nv = g.adj.size() + g.dead.size();
     if (ne) *ne = m;
     if (snap) *snap = g.snap_ts;
     if (npend) *npend = g.pending.size();
 }
 
-/* Export: ext_ids = live ids ascending; dense id = rank; offsets = prefix sums
- * of row lengths; cols/weights row by row in ascending dst order (A9). */
+/* Export: ext_ids = live ids ascending (tombstone mode: live and tombstoned ids);
+ * dense id = rank; offsets = prefix sums of row lengths; cols/weights row by row
+ * in ascending dst order (A9, A23). */
 void o1_export(void* h, int64_t* off, uint32_t* cols, float* w, uint64_t* ids) {
     Graph& g = *static_cast<Graph*>(h);
+    const std::vector<std::pair<uint64_t, bool>> all = export_ids(g);  // = keys(adj) unless tombstones
     std::map<uint64_t, uint32_t> dense;
     uint32_t r = 0;
-    for (auto& kv : g.adj) dense[kv.first] = r++;
+    for (auto& x : all) dense[x.first] = r++;
     int64_t e = 0;
     size_t i = 0;
-    for (auto& kv : g.adj) {
-        if (ids) ids[i] = kv.first;
+    for (auto& x : all) {
+        if (ids) ids[i] = x.first;
         if (off) off[i] = e;
-        for (auto& x : kv.second) {
-            if (cols) cols[e] = dense[x.first];
-            if (w) w[e] = x.second;
-            ++e;
+        if (x.second) {  // a tombstoned vertex has an empty row
+            for (auto& y : g.adj.at(x.first)) {
+                if (cols) cols[e] = dense[y.first];
+                if (w) w[e] = y.second;
+                ++e;
+            }
         }
         ++i;
     }

@@ -421,3 +421,57 @@ def test_records_round_trip_and_bounds():
     rb.records["del_cnt"][3] = 4                              # slice past the end of deletes
     with pytest.raises(ValueError):
         oracle.expand_records(rb.records, rb.inserts, rb.weights, rb.deletes)
+
+
+# ------------------------------------------------------- tombstone rows ----
+def compact_view(off, cols, w, ids, live):
+    """drop tombstoned vertices and renumber: what compaction would keep"""
+    keep = np.flatnonzero(live)
+    newid = np.full(len(ids), -1, np.int64)
+    newid[keep] = np.arange(len(keep))
+    deg = np.diff(off)[keep]
+    rows = [np.arange(off[k], off[k + 1]) for k in keep]
+    e = np.concatenate(rows) if rows else np.zeros(0, np.int64)
+    assert np.all(newid[cols[e]] >= 0)                      # no edge touches a tombstone
+    return (np.concatenate([[0], np.cumsum(deg)]).astype(np.int64), newid[cols[e]].astype(np.uint32),
+            w[e], ids[keep])
+
+
+def test_tombstone_fig2_hand_derived():
+    g = json.load(open(os.path.join(HERE, "golden", "fig2.json")))
+    e = np.array(g["edges"], dtype=object)
+    o = O1.from_edges(len(g["vertices"]), np.array(g["vertices"], np.uint64),
+                      np.array(e[:, 0], np.uint64), np.array(e[:, 1], np.uint64),
+                      np.array(e[:, 2], np.float32), g["create_ts"], tombstone=True)
+    assert o.apply(Batch.of(g["ops"]), g["snapshot_ts"])[0] == 0
+    off, cols, w, ids = o.export()
+    # node 4 keeps dense id 3 with an empty entry (P:L879-881); 5 is appended after it
+    assert ids.tolist() == [1, 2, 3, 4, 5] and o.live().tolist() == [1, 1, 1, 0, 1]
+    assert off.tolist() == [0, 0, 1, 2, 2, 3]
+    assert cols.tolist() == [2, 4, 0] and w.tolist() == [0.25, 5.0, 2.0]
+
+
+def test_tombstone_equals_compaction_of_the_live_part():
+    for k in range(40):
+        n = 12
+        ids = np.arange(n, dtype=np.uint64) * 3
+        rng = np.random.default_rng(k)
+        src, dst = ids[rng.integers(0, n, 30)], ids[rng.integers(0, n, 30)]
+        w = rng.random(30).astype(np.float32)
+        a = O1.from_edges(n, ids, src, dst, w)
+        t = O1.from_edges(n, ids, src, dst, w, tombstone=True)
+        ts = 0
+        seen = set(ids.tolist())
+        for j in range(4):
+            b = synth.fuzz_batch(seed=k, k=j, n=60, n_ids=3 * n + 3, probs=(0.12, 0.1, 0.4, 0.25, 0.13),
+                                 ts_lo=ts + 1, ts_span=50)
+            snap = ts + 40
+            assert a.apply(b, snap)[0] == 0 and t.apply(b, snap)[0] == 0
+            ts = snap + 10
+            live = t.live()
+            assert same_export(compact_view(*t.export(), live), a.export())
+            seen |= set(a.export()[3].tolist())
+            assert set(t.export()[3].tolist()) == seen      # an id, once known, keeps its slot
+            if not live.all():   # tombstones keep their rows' slot, empty
+                off = t.export()[0]
+                assert np.all(np.diff(off)[live == 0] == 0)

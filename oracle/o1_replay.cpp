@@ -193,7 +193,14 @@ int o1_apply(void* h, size_t n, const uint8_t* kind, const uint64_t* src, const 
     std::stable_sort(vis.begin(), vis.end(), [](const Op& a, const Op& b) {
         return a.ts != b.ts ? a.ts < b.ts : a.seq < b.seq;
     });
+    std::set<uint64_t> known;  // tombstone mode: ids with a slot before this cycle
+    if (g.tombstone) {
+        for (auto& kv : g.adj) known.insert(kv.first);
+        known.insert(g.dead.begin(), g.dead.end());
+    }
     for (const Op& o : vis) fold(g, o);
+    if (g.tombstone)  // A23: a node created and deleted within one cycle never gets a slot
+        for (auto it = g.dead.begin(); it != g.dead.end();) it = known.count(*it) ? std::next(it) : g.dead.erase(it);
     g.snap_ts = snapshot_ts;
     if (st) { st->n_visible = vis.size(); st->n_deferred = g.pending.size(); }
     return OK;

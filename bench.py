@@ -240,7 +240,7 @@ def run_gpu(args):
         eng = LibEngine(rep, f"cuda:{dev_idx}")
         shr = ShardedReplica(eng, rank, world, f"cuda:{dev_idx}")
     else:
-        rep = h2.Replica.from_edges(nv, ids, src, dst, w, 0, device=dev_idx)
+        rep = h2.Replica.from_edges(nv, ids, src, dst, w, 0, device=dev_idx, tombstone=args.tombstone)
     del src, dst, w
     setup_s = time.time() - t0
 
@@ -409,6 +409,8 @@ def run_gpu(args):
         }
         if records:
             line["config"]["input"] = "delta records (paper §5.1 layout, h2tap_delta_apply_records)"
+        if args.tombstone:
+            line["config"]["id_mode"] = "tombstone rows (reading A23)"
         if checks:
             line["checks"] = checks
         if not args.no_cpu_baseline:
@@ -432,6 +434,8 @@ def main():
     ap.add_argument("--input", default="ops", choices=["ops", "records"],
                     help="batch format: flat op SoA (h2tap_delta_apply) or the paper's delta records "
                          "(h2tap_delta_apply_records, §5.1 layout)")
+    ap.add_argument("--tombstone", action="store_true",
+                    help="tombstone-row replica (deleted nodes keep an empty row; reading A23)")
     ap.add_argument("--checks", action="store_true",
                     help="after the timed region, time the freshness checks (BFS, SSSP, PageRank) once")
     ap.add_argument("--parallelism", default="shard", choices=["shard", "replicas"],

@@ -93,6 +93,8 @@ typedef struct {
     uint64_t h2d_bytes, d2h_bytes; /* host<->device bytes copied by this call */
 } h2tap_apply_stats;
 
+enum { H2TAP_ID_COMPACT = 0, H2TAP_ID_TOMBSTONE = 1 };
+
 typedef struct {
     void* ctx;
     void* (*alloc)(void* ctx, size_t bytes, void* stream); /* NULL -> cudaMallocAsync */
@@ -116,6 +118,11 @@ typedef struct {
     uint64_t expected_batch;     /* capacity hint (ops per batch); 0 = none */
     h2tap_allocator alloc;
     void* stream;                /* cudaStream_t; NULL = legacy default stream */
+    int id_mode;                 /* H2TAP_ID_COMPACT (0): a deleted node leaves the ID map and the
+                                    dense IDs are compacted (reading A9); H2TAP_ID_TOMBSTONE (1):
+                                    the paper's merge() semantics, P:L879-881 — a deleted node
+                                    keeps its slot with an empty row, flagged dead (reading A23);
+                                    single replica only */
 } h2tap_config;
 
 /* Create from an edge list (reading A17): the vertex set is vertex_ids
@@ -230,6 +237,12 @@ h2tap_status h2tap_bfs(const h2tap_replica* r, uint64_t source_ext, int32_t* lev
 
 /* PageRank, fp64 (Graphalytics): PR_0 = 1/V; PR_t(v) = (1-d)/V + d*(sum over
  * in-edges u->v of PR_{t-1}(u)/outdeg(u) + dangling mass / V). rank double[V]. */
+/* Liveness of every vertex of the ID map (u8[V], 1 live / 0 tombstoned), in dense-ID
+ * order; all 1 for a compacting replica.  live: host (on_device = 0) or device buffer of
+ * V bytes, caller-owned.  In tombstone mode BFS / SSSP refuse a dead source (E_INVAL) and
+ * PageRank runs on the live subgraph (|V| = live vertices, rank 0 for a tombstone). */
+h2tap_status h2tap_replica_liveness(const h2tap_replica* r, uint8_t* live, int on_device);
+
 h2tap_status h2tap_pagerank(const h2tap_replica* r, double damping, int iterations,
         double* rank_out, int on_device);
 

@@ -51,7 +51,7 @@ class _Allocator(ctypes.Structure):
 class _Config(ctypes.Structure):
     _fields_ = [("device", ctypes.c_int), ("rank", ctypes.c_int), ("world", ctypes.c_int),
                 ("nccl_unique_id", _P), ("shard_bounds", _P), ("expected_batch", _u64),
-                ("alloc", _Allocator), ("stream", _P)]
+                ("alloc", _Allocator), ("stream", _P), ("id_mode", ctypes.c_int)]
 
 
 class _Batch(ctypes.Structure):
@@ -106,6 +106,8 @@ _lib.h2tap_bfs.restype = ctypes.c_int
 _lib.h2tap_bfs.argtypes = [_P, _u64, _P, ctypes.c_int]
 _lib.h2tap_sssp.restype = ctypes.c_int
 _lib.h2tap_sssp.argtypes = [_P, _u64, _P, ctypes.c_int]
+_lib.h2tap_replica_liveness.restype = ctypes.c_int
+_lib.h2tap_replica_liveness.argtypes = [_P, _P, ctypes.c_int]
 _lib.h2tap_pagerank.restype = ctypes.c_int
 _lib.h2tap_pagerank.argtypes = [_P, ctypes.c_double, ctypes.c_int, _P, ctypes.c_int]
 _lib.h2tap_replica_destroy.restype = None
@@ -192,9 +194,10 @@ class Replica:
 
     # ---------------------------------------------------------------- create
     @staticmethod
-    def _config(device, stream, torch_allocator, rank=0, world=1, shard_bounds=None):
+    def _config(device, stream, torch_allocator, rank=0, world=1, shard_bounds=None, tombstone=False):
         cfg = _Config()
         cfg.device = device
+        cfg.id_mode = 1 if tombstone else 0  # H2TAP_ID_TOMBSTONE / H2TAP_ID_COMPACT
         cfg.rank, cfg.world = rank, world
         keep = []
         if world > 1:
@@ -218,10 +221,10 @@ class Replica:
 
     @classmethod
     def from_edges(cls, n_vertices, vertex_ids, src, dst, w, create_ts=0, device=0, stream=None,
-                   torch_allocator=True, rank=0, world=1, shard_bounds=None) -> "Replica":
+                   torch_allocator=True, rank=0, world=1, shard_bounds=None, tombstone=False) -> "Replica":
         """Create a replica (world > 1: shard `rank` of a vertex-range sharded graph; pass
         the GLOBAL vertex set and only the edges whose source this shard owns)."""
-        cfg, keep = cls._config(device, stream, torch_allocator, rank, world, shard_bounds)
+        cfg, keep = cls._config(device, stream, torch_allocator, rank, world, shard_bounds, tombstone)
         pi, ps, pd, pw = (_ptr(vertex_ids, np.uint64), _ptr(src, np.uint64), _ptr(dst, np.uint64),
                           _ptr(w, np.float32))
         ond = _on_device(pi, ps, pd, pw)
@@ -235,8 +238,8 @@ class Replica:
 
     @classmethod
     def from_csr(cls, offsets, cols, w, ext_ids=None, create_ts=0, device=0, stream=None,
-                 torch_allocator=True) -> "Replica":
-        cfg, keep = cls._config(device, stream, torch_allocator)
+                 torch_allocator=True, tombstone=False) -> "Replica":
+        cfg, keep = cls._config(device, stream, torch_allocator, tombstone=tombstone)
         po, pc, pw, pi = (_ptr(offsets, np.int64), _ptr(cols, np.uint32), _ptr(w, np.float32),
                           _ptr(ext_ids, np.uint64))
         ond = _on_device(po, pc, pw, pi)
@@ -350,6 +353,12 @@ class Replica:
         lvl = np.empty(self.info()["n_vertices"], np.int32)
         _check(_lib.h2tap_bfs(self._h, int(source_ext), ctypes.c_void_p(lvl.ctypes.data), 0), "h2tap_bfs")
         return lvl
+
+    def live(self) -> np.ndarray:
+        """u8 liveness per dense id (all 1 unless the replica keeps tombstones)"""
+        out = np.empty(self.info()["n_vertices"], np.uint8)
+        _check(_lib.h2tap_replica_liveness(self._h, ctypes.c_void_p(out.ctypes.data), 0), "h2tap_replica_liveness")
+        return out
 
     def sssp(self, source_ext: int) -> np.ndarray:
         dist = np.empty(self.info()["n_vertices"], np.float64)

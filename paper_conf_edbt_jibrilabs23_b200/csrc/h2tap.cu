@@ -129,6 +129,8 @@ struct h2tap_replica {
     Buf ins_pos, ins_row, ins_col, ins_w, del_pos, upd_pos, upd_w, KR;
     Buf misc, nsorted, part, opart, deg, tsum, remap_shift, remap32, casc_wrel, tile_emit, tile_base, del_row, casc_mask, status2, bfs_a, bfs_b, pr_a, pr_b;
     Buf xrec, xins, xwts, xdel, xcnt, xoff;  // delta-record input (h2tap_delta_apply_records)
+    bool tomb = false;  // tombstone-row mode (reading A23)
+    Buf live[2];        // tombstone mode: u8 liveness per dense id, double-buffered with ext
     Buf ctr;
     Counters* hc = nullptr;  // pinned host mirror
     cudaEvent_t ev[8]{};
@@ -274,6 +276,7 @@ ExtIndex ext_index(h2tap_replica* r) {
     X.V = r->V;
     X.nf = n_fence(r->V);
     X.identity = r->identity;
+    X.live = r->tomb ? static_cast<const uint8_t*>(r->live[r->ext_cur].p) : nullptr;
     return X;
 }
 
@@ -429,7 +432,8 @@ h2tap_status apply_core(h2tap_replica* r, const BatchIn& in, uint64_t S, bool cr
         ins_q = r->get<uint32_t>(r->ins_q, n_node);
         ins_oldpos = r->get<uint32_t>(r->ins_oldpos, n_node);
         hd_rows = r->get<uint32_t>(r->hd_rows, n_node);
-        k_node_lists<<<(unsigned)nt, kThreads, 0, st>>>(nv, dropped, ins_q, ins_oldpos, hd_rows, stt, nt, dc);
+        k_node_lists<<<(unsigned)nt, kThreads, 0, st>>>(nv, dropped, ins_q, ins_oldpos, hd_rows, stt, nt, dc,
+                                                        r->tomb ? 1 : 0);
         CKL();
         TR("node_lists");
         // ID-map compaction: remap tables (64K-id block shifts, 32-id groups, the
@@ -580,6 +584,11 @@ h2tap_status apply_core(h2tap_replica* r, const BatchIn& in, uint64_t S, bool cr
         ra.new_off = new_off;
         ra.c = dc;
         ra.old_ext = old_ext; ra.new_ext = new_ext; ra.identity = r->identity ? 1 : 0;
+        uint8_t* new_live = nullptr;
+        if (r->tomb) {
+            ra.old_live = static_cast<const uint8_t*>(r->live[ec].p);
+            ra.new_live = new_live = r->get<uint8_t>(r->live[ec ^ 1], Vn_ub);
+        }
         const uint64_t ncta = cdiv(V, kRowTile);
         ra.part = r->get<uint64_t>(r->opart, 2 * (ncta + 1));
         if (V) {
@@ -590,6 +599,10 @@ h2tap_status apply_core(h2tap_replica* r, const BatchIn& in, uint64_t S, bool cr
         }
         k_offsets_inserted<<<g1(n_node), 256, 0, st>>>(nv, ins_q, ra);
         CKL();
+        if (new_live) {  // node-op vertices' final liveness over the carried flags
+            k_nv_live<<<g1(n_node), 256, 0, st>>>(nv, dc, R, new_live);
+            CKL();
+        }
         uint64_t* f = r->get<uint64_t>(r->fence[ec ^ 1], n_fence(Vn_ub));
         k_build_fence_dev<<<g1(n_fence(Vn_ub)), 256, 0, st>>>(new_ext, dc, f);
         CKL();
@@ -762,6 +775,15 @@ h2tap_replica* new_replica(const h2tap_config* cfg) {
     if (cfg) r->cfg = *cfg;
     else { r->cfg.world = 1; }
     if (r->cfg.world <= 0) r->cfg.world = 1;
+    if (r->cfg.id_mode != H2TAP_ID_COMPACT && r->cfg.id_mode != H2TAP_ID_TOMBSTONE) {
+        set_err("id_mode must be H2TAP_ID_COMPACT or H2TAP_ID_TOMBSTONE");
+        throw Fail{H2TAP_E_INVAL};
+    }
+    r->tomb = r->cfg.id_mode == H2TAP_ID_TOMBSTONE;
+    if (r->tomb && r->cfg.world > 1) {
+        set_err("tombstone-row mode is single-replica only in this build");
+        throw Fail{H2TAP_E_INVAL};
+    }
     if (r->cfg.world > 1) {
         if (!r->cfg.shard_bounds || r->cfg.rank < 0 || r->cfg.rank >= r->cfg.world) {
             set_err("sharded replica needs shard_bounds[world+1] and 0 <= rank < world");
@@ -811,7 +833,7 @@ void free_replica(h2tap_replica* r) {
                    &r->ins_oldpos, &r->hd_rows, &r->hd_bits, &r->op_flags, &r->op_ou, &r->op_ow,
                    &r->ins_pos, &r->ins_row, &r->ins_col, &r->ins_w, &r->del_pos, &r->upd_pos, &r->upd_w,
                    &r->KR, &r->misc, &r->nsorted, &r->part, &r->opart, &r->deg, &r->tsum, &r->remap_shift, &r->remap32, &r->casc_wrel, &r->tile_emit, &r->tile_base, &r->del_row, &r->casc_mask, &r->status2, &r->bounds_dev, &r->fence[0], &r->fence[1], &r->bfs_a, &r->bfs_b, &r->pr_a, &r->pr_b, &r->ctr,
-                   &r->xrec, &r->xins, &r->xwts, &r->xdel, &r->xcnt, &r->xoff};
+                   &r->xrec, &r->xins, &r->xwts, &r->xdel, &r->xcnt, &r->xoff, &r->live[0], &r->live[1]};
     for (Buf* b : bufs) if (b->p) r->dfree(b->p);
     cudaStreamSynchronize(r->st);
     for (auto& e : r->ev) if (e) cudaEventDestroy(e);
@@ -848,6 +870,10 @@ void init_vertices(h2tap_replica* r, uint64_t nv, const uint64_t* ids, int on_de
         r->identity = (h[1] == nv - 1);
     }
     build_fence(r, 0, nv);
+    if (r->tomb) {  // every created vertex is live
+        uint8_t* lv = r->get<uint8_t>(r->live[0], nv);
+        if (nv) CK(cudaMemsetAsync(lv, 1, nv, r->st));
+    }
     r->row_lo = 0;
     r->Vr = nv;
     if (r->sharded) {
@@ -1155,9 +1181,15 @@ h2tap_status h2tap_replica_export(const h2tap_replica* rc, int64_t* offsets, uin
 
 // dense id of a live vertex (V if absent): identity map, else a binary search of the
 // device ID map through single-element reads (the analytics' source lookup only)
+static uint64_t live_or_none(h2tap_replica* r, uint64_t k) {  // tombstone mode: a dead slot is no source
+    if (!r->tomb) return k;
+    uint8_t l = 0;
+    CK(cudaMemcpy(&l, static_cast<const uint8_t*>(r->live[r->ext_cur].p) + k, 1, cudaMemcpyDeviceToHost));
+    return l ? k : r->V;
+}
 static uint64_t dense_of(h2tap_replica* r, uint64_t x_ext) {
     const uint64_t V = r->V;
-    if (r->identity) return x_ext < V ? x_ext : V;
+    if (r->identity) return x_ext < V ? live_or_none(r, x_ext) : V;
     const uint64_t* ext = static_cast<const uint64_t*>(r->ext[r->ext_cur].p);
     uint64_t lo = 0, hi = V;
     while (lo < hi) {
@@ -1167,7 +1199,8 @@ static uint64_t dense_of(h2tap_replica* r, uint64_t x_ext) {
     }
     uint64_t x = ~0ull;
     if (lo < V) CK(cudaMemcpy(&x, ext + lo, 8, cudaMemcpyDeviceToHost));
-    return (lo < V && x == x_ext) ? lo : V;
+    const uint64_t k = (lo < V && x == x_ext) ? lo : V;
+    return k < V ? live_or_none(r, k) : V;
 }
 
 h2tap_status h2tap_bfs(const h2tap_replica* rc, uint64_t source_ext, int32_t* level_out, int on_device) {
@@ -1261,6 +1294,26 @@ h2tap_status h2tap_sssp(const h2tap_replica* rc, uint64_t source_ext, double* di
     });
 }
 
+h2tap_status h2tap_replica_liveness(const h2tap_replica* rc, uint8_t* live_out, int on_device) {
+    h2tap_replica* r = const_cast<h2tap_replica*>(rc);
+    if (!r || !live_out) { set_err("null argument"); return H2TAP_E_INVAL; }
+    return run_guarded(r, [&]() -> h2tap_status {
+        CK(cudaSetDevice(r->cfg.device));
+        const uint64_t V = r->V;
+        if (!r->tomb) {  // compacting replica: every vertex in the ID map is live
+            if (V) {
+                if (on_device) CK(cudaMemsetAsync(live_out, 1, V, r->st));
+                else std::memset(live_out, 1, V);
+            }
+        } else if (V) {
+            CK(cudaMemcpyAsync(live_out, r->live[r->ext_cur].p, V,
+                               on_device ? cudaMemcpyDeviceToDevice : cudaMemcpyDeviceToHost, r->st));
+        }
+        r->sync();
+        return H2TAP_OK;
+    });
+}
+
 h2tap_status h2tap_pagerank(const h2tap_replica* rc, double damping, int iterations, double* rank_out, int on_device) {
     h2tap_replica* r = const_cast<h2tap_replica*>(rc);
     if (!r || !rank_out || iterations < 0) { set_err("bad argument"); return H2TAP_E_INVAL; }
@@ -1274,7 +1327,25 @@ h2tap_status h2tap_pagerank(const h2tap_replica* rc, double damping, int iterati
         double* ds = r->get<double>(r->misc, 1);
         const int64_t* off = static_cast<const int64_t*>(r->off[r->cur].p);
         const uint32_t* cols = static_cast<const uint32_t*>(r->cols[r->cur].p);
-        k_pr_init<<<g1(V), 256, 0, r->st>>>(a, V);
+        const uint8_t* live = r->tomb ? static_cast<const uint8_t*>(r->live[r->ext_cur].p) : nullptr;
+        uint64_t nl = V;
+        if (live) {  // the graph is the live vertices (reading A23)
+            unsigned long long* c = reinterpret_cast<unsigned long long*>(r->get<double>(r->misc, 2)) + 1;
+            CK(cudaMemsetAsync(c, 0, 8, r->st));
+            k_count_u8<<<(unsigned)std::min<uint64_t>(g1(V), 148 * 8), 256, 0, r->st>>>(live, V, c);
+            CKL();
+            unsigned long long h = 0;
+            CK(cudaMemcpyAsync(&h, c, 8, cudaMemcpyDeviceToHost, r->st));
+            r->sync();
+            nl = h;
+            if (nl == 0) {
+                CK(cudaMemsetAsync(on_device ? rank_out : a, 0, V * 8, r->st));
+                if (!on_device) { CK(cudaMemcpyAsync(rank_out, a, V * 8, cudaMemcpyDeviceToHost, r->st)); }
+                r->sync();
+                return H2TAP_OK;
+            }
+        }
+        k_pr_init<<<g1(V), 256, 0, r->st>>>(a, V, live, nl);
         CKL();
         unsigned gs = (unsigned)std::min<uint64_t>(g1(V), 148 * 8);
         unsigned gw = (unsigned)std::min<uint64_t>(cdiv(V * 32, 256), 148 * 32);
@@ -1283,7 +1354,7 @@ h2tap_status h2tap_pagerank(const h2tap_replica* rc, double damping, int iterati
             CK(cudaMemsetAsync(b, 0, V * 8, r->st));
             k_pr_dangling<<<gs, 256, 0, r->st>>>(off, a, V, ds);
             k_pr_push<<<gw, 256, 0, r->st>>>(off, cols, a, V, b);
-            k_pr_finish<<<g1(V), 256, 0, r->st>>>(b, V, damping, ds);
+            k_pr_finish<<<g1(V), 256, 0, r->st>>>(b, V, damping, ds, live, nl);
             CKL();
             std::swap(a, b);
         }

@@ -57,7 +57,9 @@ struct NodeVtx {
     uint32_t flags;
     uint32_t pad;
 };
-enum : uint32_t { NV_FINAL = 1, NV_HASD = 2, NV_OLD = 4 };
+// NV_OLD: present in the old ID map; NV_LIVE0: live before the cycle (= NV_OLD unless
+// the replica keeps tombstones, reading A23)
+enum : uint32_t { NV_FINAL = 1, NV_HASD = 2, NV_OLD = 4, NV_LIVE0 = 8 };
 
 // ID-map compaction (reading A9), evaluated on the fly: new dense id of old vertex k
 // = k - (#dropped ids < k) + (#inserted ids placed at old positions <= k).
@@ -210,6 +212,7 @@ struct ExtIndex {
     const uint64_t* fence;
     uint64_t V, nf;
     int identity;
+    const uint8_t* live;  // tombstone mode: liveness per old dense id (nullptr: all live)
 };
 __device__ __forceinline__ uint64_t old_lookup(const ExtIndex& X, uint64_t x, bool* present) {
     if (X.identity) { *present = x < X.V; return x < X.V ? x : X.V; }
@@ -403,6 +406,7 @@ __global__ void __launch_bounds__(kThreads) k_node_segments(
         bool present;
         uint64_t k = old_lookup(X, v, &present);
         if (present) r.flags |= NV_OLD;
+        if (present && (!X.live || X.live[k])) r.flags |= NV_LIVE0;
         r.oldpos = (uint32_t)k;
         r.start = (uint32_t)i;
         r.end = (uint32_t)e;
@@ -427,7 +431,7 @@ __global__ void __launch_bounds__(kThreads) k_node_segments(
 __global__ void __launch_bounds__(kThreads) k_node_lists(
     const NodeVtx* __restrict__ nv, uint32_t* __restrict__ dropped,
     uint32_t* __restrict__ ins_q, uint32_t* __restrict__ ins_oldpos, uint32_t* __restrict__ hd_rows,
-    uint64_t* __restrict__ status3, uint64_t n_tiles_ub, Counters* __restrict__ c) {
+    uint64_t* __restrict__ status3, uint64_t n_tiles_ub, Counters* __restrict__ c, int tomb) {
     __shared__ uint32_t s_tile;
     __shared__ uint64_t s_scan[kThreads / 32 + 1];
     __shared__ uint64_t s_base[3];
@@ -445,10 +449,10 @@ __global__ void __launch_bounds__(kThreads) k_node_lists(
         fl[j] = 0;
         if (i < U) {
             uint32_t f = nv[i].flags;
-            bool old = f & NV_OLD, fin = f & NV_FINAL, hd = f & NV_HASD;
-            if (old && !fin) { fl[j] |= 1; cnt[0]++; }
+            bool old = f & NV_OLD, live0 = f & NV_LIVE0, fin = f & NV_FINAL, hd = f & NV_HASD;
+            if (live0 && !fin && !tomb) { fl[j] |= 1; cnt[0]++; }  // tombstone mode keeps the slot (A23)
             if (!old && fin) { fl[j] |= 2; cnt[1]++; }
-            if (old && hd) { fl[j] |= 4; cnt[2]++; }
+            if (live0 && hd) { fl[j] |= 4; cnt[2]++; }             // its old edges cascade
         }
     }
     uint64_t excl[3], tot[3];
@@ -514,6 +518,17 @@ __global__ void k_nv_newid(NodeVtx* __restrict__ nv, const Counters* __restrict_
     if ((f & NV_OLD) && (f & NV_FINAL)) nv[q].newid = remap_of(R, nv[q].oldpos);
 }
 
+// tombstone mode: final liveness of the vertices with node ops in the new slots (after
+// k_rows_fused copied the old flags): present vertices keep their slot (remapped only by
+// insertions), inserted ones take their placed id
+__global__ void k_nv_live(const NodeVtx* __restrict__ nv, const Counters* __restrict__ c, RemapView R,
+                          uint8_t* __restrict__ new_live) {
+    const uint64_t q = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x;
+    if (q >= c->n_unique) return;
+    const NodeVtx r = nv[q];
+    const uint32_t u = (r.flags & NV_OLD) ? remap_of(R, r.oldpos) : r.newid;
+    if (u != kNone32) new_live[u] = (r.flags & NV_FINAL) ? 1 : 0;
+}
 __global__ void k_set_bits(const uint32_t* __restrict__ rows, const Counters* __restrict__ c, uint32_t* __restrict__ bits) {
     uint64_t i = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x;
     if (i < c->n_hd) atomicOr(&bits[rows[i] >> 5], 1u << (rows[i] & 31));
@@ -524,7 +539,7 @@ struct Lookup {
     int64_t q;        // index in the node-vertex list or -1
     uint32_t oldpos;  // old dense index (present) or insertion rank
     uint32_t newid;
-    bool old_present, final_live, hasD;
+    bool old_present, final_live, hasD, live0;
     uint64_t tD_ts, tD_seq;
 };
 
@@ -574,6 +589,7 @@ __device__ __forceinline__ Lookup do_lookup(const PrepArgs& a, uint64_t U, uint6
             L.oldpos = r.oldpos;
             L.newid = r.newid;
             L.old_present = r.flags & NV_OLD;
+            L.live0 = r.flags & NV_LIVE0;
             L.final_live = r.flags & NV_FINAL;
             L.hasD = r.flags & NV_HASD;
             L.tD_ts = r.tD_ts; L.tD_seq = r.tD_seq;
@@ -584,14 +600,14 @@ __device__ __forceinline__ Lookup do_lookup(const PrepArgs& a, uint64_t U, uint6
     uint64_t k = old_lookup(a.X, x, &present);
     L.oldpos = (uint32_t)k;
     L.old_present = present;
-    L.final_live = present;
+    L.final_live = L.live0 = present && (!a.X.live || a.X.live[k]);
     L.newid = present ? remap_of(a.R, (uint32_t)k) : kNone32;
     return L;
 }
 
 // liveness of a vertex with node ops just before point (ts, seq) (reading A13)
 __device__ __forceinline__ bool live_at(const PrepArgs& a, const Lookup& L, uint64_t ts, uint64_t seq) {
-    if (L.q < 0) return L.old_present;
+    if (L.q < 0) return L.live0;
     const NodeVtx& r = a.nv[L.q];
     uint64_t lo = r.start, hi = r.end;  // first node op with point >= p
     while (lo < hi) {
@@ -599,7 +615,7 @@ __device__ __forceinline__ bool live_at(const PrepArgs& a, const Lookup& L, uint
         uint32_t o = a.node_sorted[mid];
         if (pt_less(a.ops.ts[o], a.ops.seq[o], ts, seq)) lo = mid + 1; else hi = mid;
     }
-    if (lo == r.start) return L.old_present;
+    if (lo == r.start) return L.live0;
     return a.ops.kind[a.node_sorted[lo - 1]] == NODE_INSERT;
 }
 
@@ -1132,6 +1148,8 @@ struct RowArgs {
     const uint64_t* old_ext;  // ID maps (k_rows_fused); identity: old ext id == k
     uint64_t* new_ext;
     int identity;
+    const uint8_t* old_live;  // tombstone mode: liveness carried to the new slots
+    uint8_t* new_live;
 };
 __device__ __forceinline__ RowArgs row_counts(RowArgs a) {
     a.n_del = a.c->n_del;
@@ -1195,6 +1213,7 @@ __global__ void __launch_bounds__(kThreads, 5) k_rows_fused(RowArgs a_) {
         if (k < k1) {
             u[j] = remap_of(a.R, (uint32_t)k);
             if (!a.identity) ext[j] = a.old_ext[k];
+            if (a.new_live && u[j] != kNone32) a.new_live[u[j]] = a.old_live[k];
             row[j] = k >= a.row_lo && k < a.row_hi;
             if (row[j]) x[j] = (uint64_t)a.old_off[k];
         }
@@ -1924,14 +1943,16 @@ __global__ void k_fill_i32(int32_t* p, uint64_t n, int32_t v) {
 }
 
 // ---------------------------------------------------------- PageRank ----
-__global__ void k_pr_init(double* pr, uint64_t n) {
+// live (nullable, tombstone mode): PageRank of the live subgraph, nl = live vertices;
+// a tombstoned vertex has no edges and rank 0
+__global__ void k_pr_init(double* pr, uint64_t n, const uint8_t* __restrict__ live, uint64_t nl) {
     uint64_t i = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x;
-    if (i < n) pr[i] = 1.0 / (double)n;
+    if (i < n) pr[i] = (!live || live[i]) ? 1.0 / (double)nl : 0.0;
 }
 __global__ void k_pr_dangling(const int64_t* __restrict__ off, const double* __restrict__ pr, uint64_t n, double* out) {
     double acc = 0;
     for (uint64_t u = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; u < n; u += (uint64_t)gridDim.x * blockDim.x)
-        if (off[u + 1] == off[u]) acc += pr[u];
+        if (off[u + 1] == off[u]) acc += pr[u];  // tombstones hold 0
     acc = warp_sum(acc);
     if (lane_id() == 0 && acc != 0.0) atomicAdd(out, acc);
 }
@@ -1946,9 +1967,17 @@ __global__ void k_pr_push(const int64_t* __restrict__ off, const uint32_t* __res
         for (int64_t x = b + lane_id(); x < e; x += 32) atomicAdd(&nxt[cols[x]], c);
     }
 }
-__global__ void k_pr_finish(double* __restrict__ nxt, uint64_t n, double d, const double* __restrict__ dsum) {
+__global__ void k_pr_finish(double* __restrict__ nxt, uint64_t n, double d, const double* __restrict__ dsum,
+                            const uint8_t* __restrict__ live, uint64_t nl) {
     uint64_t v = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x;
-    if (v < n) nxt[v] = (1.0 - d) / (double)n + d * (nxt[v] + *dsum / (double)n);
+    if (v < n) nxt[v] = (!live || live[v]) ? (1.0 - d) / (double)nl + d * (nxt[v] + *dsum / (double)nl) : 0.0;
+}
+__global__ void k_count_u8(const uint8_t* __restrict__ x, uint64_t n, unsigned long long* __restrict__ out) {
+    unsigned long long acc = 0;
+    for (uint64_t i = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; i < n; i += (uint64_t)gridDim.x * blockDim.x)
+        acc += x[i] ? 1 : 0;
+    acc = warp_sum(acc);
+    if (lane_id() == 0 && acc) atomicAdd(out, acc);
 }
 
 }  // namespace h2tap

@@ -27,7 +27,7 @@ def lib():
 def test_header_declares_the_boundary():
     syms = declared_symbols()
     for s in ("h2tap_replica_create_from_edges", "h2tap_replica_create_from_csr", "h2tap_delta_apply",
-              "h2tap_replica_info", "h2tap_replica_export", "h2tap_bfs", "h2tap_sssp", "h2tap_pagerank",
+              "h2tap_replica_info", "h2tap_replica_export", "h2tap_bfs", "h2tap_sssp", "h2tap_pagerank", "h2tap_replica_liveness", "h2tap_delta_apply_records",
               "h2tap_replica_destroy", "h2tap_status_str", "h2tap_last_error"):
         assert s in syms
 

@@ -130,6 +130,7 @@ struct h2tap_replica {
     Buf misc, nsorted, part, opart, deg, tsum, remap_shift, remap32, casc_wrel, tile_emit, tile_base, del_row, casc_mask, status2, bfs_a, bfs_b, pr_a, pr_b;
     Buf xrec, xins, xwts, xdel, xcnt, xoff;  // delta-record input (h2tap_delta_apply_records)
     bool tomb = false;  // tombstone-row mode (reading A23)
+    Buf casc_status;    // look-back words of the cascade scan (runs beside the edge-op phase)
     Buf live[2];        // tombstone mode: u8 liveness per dense id, double-buffered with ext
     Buf ctr;
     Counters* hc = nullptr;  // pinned host mirror
@@ -280,6 +281,11 @@ ExtIndex ext_index(h2tap_replica* r) {
     return X;
 }
 
+#ifndef H2TAP_CASC_CTAS
+#define H2TAP_CASC_CTAS 4
+#endif
+constexpr int kCascCtasPerSm = H2TAP_CASC_CTAS;  // cascade pass beside the edge-op phase
+
 // One propagation cycle.  Nothing visible changes until the final swap.
 h2tap_status apply_core(h2tap_replica* r, const BatchIn& in, uint64_t S, bool create, h2tap_apply_stats* stats) {
     cudaStream_t st = r->st;
@@ -291,6 +297,7 @@ h2tap_status apply_core(h2tap_replica* r, const BatchIn& in, uint64_t S, bool cr
     g_tr.init();
     for (int i = 0; i < 8; ++i)
         if (!r->ev[i]) CK(cudaEventCreate(&r->ev[i]));
+    CK(cudaStreamWaitEvent(st, r->evB, 0));  // a cascade pass of an earlier (failed) cycle is done
     CK(cudaEventRecord(r->ev[0], st));
     TR("start");
 
@@ -387,6 +394,7 @@ h2tap_status apply_core(h2tap_replica* r, const BatchIn& in, uint64_t S, bool cr
              *hd_bits = nullptr, *node_sorted = nullptr;
     uint64_t* new_ext = nullptr;
     uint32_t* casc_mask = nullptr;
+    bool casc_pending = false;  // cascade pass in flight on the side stream
     uint64_t *casc_cnt = nullptr, *casc_pre = nullptr;
     uint16_t* casc_wrel = nullptr;
     const int64_t* old_off_nc = static_cast<const int64_t*>(r->off[r->cur].p);
@@ -468,23 +476,30 @@ h2tap_status apply_core(h2tap_replica* r, const BatchIn& in, uint64_t S, bool cr
         casc_pre = r->get<uint64_t>(r->tile_base, nblk_c + 1);
         unsigned rg = (unsigned)std::min<uint64_t>(cdiv(n_node * 32, 256), (uint64_t)r->n_sm * 8);
         const uint64_t nst = cdiv(nblk_c + 1, kThreads);
-        uint64_t* st2s2 = r->get<uint64_t>(r->status2, nst);
+        uint64_t* st2s2 = r->get<uint64_t>(r->casc_status, nst);
         CK(cudaMemsetAsync(st2s2, 0, nst * 8, st));
-        TR("nv_newid+bits");
-        if (nblk_c) {
-            const unsigned gc = (unsigned)std::min<uint64_t>(cdiv(nblk_c, 2), (uint64_t)r->n_sm * 6);
-            k_casc_cols<<<gc, kThreads, 0, st>>>(old_cols_nc, E, hd_bits, hd_rows, dc, casc_mask);
-            CKL();
-            TR("casc_cols");
-            k_casc_rows<<<rg, 256, 0, st>>>(old_off_nc, hd_rows, dc, row_lo, row_lo + Vr, casc_mask);
-            CKL();
-            TR("casc_rows");
-        }
         casc_wrel = r->get<uint16_t>(r->casc_wrel, (nblk_c + 1) * (kCascBlock / 32));
-        k_casc_scan<<<(unsigned)nst, kThreads, 0, st>>>(casc_mask, nblk_c, casc_pre, casc_wrel, st2s2, &dc->tiles[6]);
+        TR("nv_newid+bits");
+        // The cascade pass streams the old columns (HBM-bound) and nothing in the edge-op
+        // phase below (latency-bound sort / classify) reads its output, so it runs on the
+        // side stream with a grid of 4 CTAs per SM, leaving most of every SM to the edge-op
+        // kernels; the row pass joins it (casc_join) before reading the cascade tables.
+        CK(cudaEventRecord(r->evA, st));
+        CK(cudaStreamWaitEvent(r->st2, r->evA, 0));
+        cudaStream_t cs = r->st2;
+        if (nblk_c) {
+            const unsigned gc = (unsigned)std::min<uint64_t>(cdiv(nblk_c, 2), (uint64_t)r->n_sm * kCascCtasPerSm);
+            k_casc_cols<<<gc, kThreads, 0, cs>>>(old_cols_nc, E, hd_bits, hd_rows, dc, casc_mask);
+            CKL();
+            k_casc_rows<<<rg, 256, 0, cs>>>(old_off_nc, hd_rows, dc, row_lo, row_lo + Vr, casc_mask);
+            CKL();
+        }
+        k_casc_scan<<<(unsigned)nst, kThreads, 0, cs>>>(casc_mask, nblk_c, casc_pre, casc_wrel, st2s2, &dc->tiles[6]);
         CKL();
-        k_copy_u64<<<1, 1, 0, st>>>(&dc->n_casc, casc_pre + nblk_c);
+        k_copy_u64<<<1, 1, 0, cs>>>(&dc->n_casc, casc_pre + nblk_c);
         CKL();
+        CK(cudaEventRecord(r->evB, cs));
+        casc_pending = true;
     }
     CK(cudaEventRecord(r->ev[2], st));
     TR("idmap+remap");
@@ -573,6 +588,11 @@ h2tap_status apply_core(h2tap_replica* r, const BatchIn& in, uint64_t S, bool cr
     float* new_w = r->get<float>(r->w[nb], Ecap);
     // node mode: survivors' ID map + row offsets before the merge, while the cascade
     // tables written by the cascade pass are still L2-resident (the merge streams the CSR)
+    if (casc_pending) {  // join the cascade pass
+        CK(cudaStreamWaitEvent(st, r->evB, 0));
+        casc_pending = false;
+        TR("casc_join");
+    }
     if (node_mode) {
         RowArgs ra{};
         ra.old_off = old_off - row_lo; ra.V_old = V; ra.E_old = E; ra.R = R;
@@ -833,7 +853,7 @@ void free_replica(h2tap_replica* r) {
                    &r->ins_oldpos, &r->hd_rows, &r->hd_bits, &r->op_flags, &r->op_ou, &r->op_ow,
                    &r->ins_pos, &r->ins_row, &r->ins_col, &r->ins_w, &r->del_pos, &r->upd_pos, &r->upd_w,
                    &r->KR, &r->misc, &r->nsorted, &r->part, &r->opart, &r->deg, &r->tsum, &r->remap_shift, &r->remap32, &r->casc_wrel, &r->tile_emit, &r->tile_base, &r->del_row, &r->casc_mask, &r->status2, &r->bounds_dev, &r->fence[0], &r->fence[1], &r->bfs_a, &r->bfs_b, &r->pr_a, &r->pr_b, &r->ctr,
-                   &r->xrec, &r->xins, &r->xwts, &r->xdel, &r->xcnt, &r->xoff, &r->live[0], &r->live[1]};
+                   &r->xrec, &r->xins, &r->xwts, &r->xdel, &r->xcnt, &r->xoff, &r->live[0], &r->live[1], &r->casc_status};
     for (Buf* b : bufs) if (b->p) r->dfree(b->p);
     cudaStreamSynchronize(r->st);
     for (auto& e : r->ev) if (e) cudaEventDestroy(e);

@@ -108,7 +108,7 @@ inline int bits_for(uint64_t range) { return range == 0 ? 0 : 64 - __builtin_clz
 struct h2tap_replica {
     h2tap_config cfg{};
     cudaStream_t st = nullptr, st2 = nullptr;  // st2: side stream (cascade pass)
-    cudaEvent_t evA = nullptr, evB = nullptr;
+    cudaEvent_t evA = nullptr, evB = nullptr, evC = nullptr;
     uint64_t V = 0, E = 0, snap = 0, next_seq = 0, n_pend = 0;
     // sharding: V = global live vertices (the replicated ID map), the CSR holds the Vr rows
     // of the owned external-ID range starting at global dense id row_lo
@@ -281,6 +281,12 @@ ExtIndex ext_index(h2tap_replica* r) {
     return X;
 }
 
+#ifndef H2TAP_ROWS_SIDE
+#define H2TAP_ROWS_SIDE 0
+#endif
+#ifndef H2TAP_MERGE_CTAS
+#define H2TAP_MERGE_CTAS 0
+#endif
 #ifndef H2TAP_CASC_CTAS
 #define H2TAP_CASC_CTAS 4
 #endif
@@ -395,6 +401,7 @@ h2tap_status apply_core(h2tap_replica* r, const BatchIn& in, uint64_t S, bool cr
     uint64_t* new_ext = nullptr;
     uint32_t* casc_mask = nullptr;
     bool casc_pending = false;  // cascade pass in flight on the side stream
+    bool rows_pending = false;  // row pass in flight on the side stream (H2TAP_ROWS_SIDE)
     uint64_t *casc_cnt = nullptr, *casc_pre = nullptr;
     uint16_t* casc_wrel = nullptr;
     const int64_t* old_off_nc = static_cast<const int64_t*>(r->off[r->cur].p);
@@ -594,6 +601,12 @@ h2tap_status apply_core(h2tap_replica* r, const BatchIn& in, uint64_t S, bool cr
         TR("casc_join");
     }
     if (node_mode) {
+        cudaStream_t st = r->st;  // the row pass's stream (shadows the replica stream)
+        if (H2TAP_ROWS_SIDE) {    // beside the merge: both stream, neither reads the other's output
+            CK(cudaEventRecord(r->evA, r->st));
+            CK(cudaStreamWaitEvent(r->st2, r->evA, 0));
+            st = r->st2;
+        }
         RowArgs ra{};
         ra.old_off = old_off - row_lo; ra.V_old = V; ra.E_old = E; ra.R = R;
         ra.row_lo = row_lo; ra.row_hi = row_lo + Vr;
@@ -626,6 +639,10 @@ h2tap_status apply_core(h2tap_replica* r, const BatchIn& in, uint64_t S, bool cr
         uint64_t* f = r->get<uint64_t>(r->fence[ec ^ 1], n_fence(Vn_ub));
         k_build_fence_dev<<<g1(n_fence(Vn_ub)), 256, 0, st>>>(new_ext, dc, f);
         CKL();
+        if (H2TAP_ROWS_SIDE) {
+            CK(cudaEventRecord(r->evC, st));
+            rows_pending = true;
+        }
     }
     // ---- a4/a5 without node ops: row offsets (while the outcome lists are L2-resident)
     if (Vr && !node_mode) {
@@ -668,6 +685,7 @@ h2tap_status apply_core(h2tap_replica* r, const BatchIn& in, uint64_t S, bool cr
             int occ = 0;
             CK(cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, kMerge3Smem));
             CK(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, kern, kThreads, kMerge3Smem));
+            if (H2TAP_MERGE_CTAS > 0) occ = std::min(occ, (int)H2TAP_MERGE_CTAS);
             const uint64_t grid = std::min<uint64_t>(ma.n_tiles, (uint64_t)std::max(1, occ) * r->n_sm);
             kern<<<(unsigned)grid, kThreads, kMerge3Smem, st>>>(ma, part);
         };
@@ -698,6 +716,7 @@ h2tap_status apply_core(h2tap_replica* r, const BatchIn& in, uint64_t S, bool cr
             r->get<uint64_t>(r->pt[pn], n_pend_new), r->get<uint64_t>(r->pq[pn], n_pend_new));
         CKL();
     }
+    if (rows_pending) CK(cudaStreamWaitEvent(st, r->evC, 0));  // row pass (side stream) done
     k_finish<<<1, 1, 0, st>>>(dc, V, Vr, E, node_mode ? 1 : 0, r->sharded ? 1 : 0, new_ext, new_off);
     CKL();
     CK(cudaEventRecord(r->ev[5], st));
@@ -838,6 +857,7 @@ h2tap_replica* new_replica(const h2tap_config* cfg) {
     }
     CK(cudaEventCreateWithFlags(&r->evA, cudaEventDisableTiming));
     CK(cudaEventCreateWithFlags(&r->evB, cudaEventDisableTiming));
+    CK(cudaEventCreateWithFlags(&r->evC, cudaEventDisableTiming));
     CK(cudaMallocHost(&r->hc, sizeof(Counters)));
     r->get<Counters>(r->ctr, 1);
     return r;
@@ -859,6 +879,7 @@ void free_replica(h2tap_replica* r) {
     for (auto& e : r->ev) if (e) cudaEventDestroy(e);
     if (r->evA) cudaEventDestroy(r->evA);
     if (r->evB) cudaEventDestroy(r->evB);
+    if (r->evC) cudaEventDestroy(r->evC);
     if (r->st2) { cudaStreamSynchronize(r->st2); cudaStreamDestroy(r->st2); }
     if (r->hc) cudaFreeHost(r->hc);
     delete r;

@@ -323,7 +323,12 @@ h2tap_status apply_core(h2tap_replica* r, const BatchIn& in, uint64_t S, bool cr
         CK(cudaMemcpyAsync(Wt, r->pt[pc].p, np * 8, cudaMemcpyDeviceToDevice, st));
         CK(cudaMemcpyAsync(Wq, r->pq[pc].p, np * 8, cudaMemcpyDeviceToDevice, st));
     }
-    if (n && in.recs) {
+    // a device-resident batch with nothing pending is read in place (no staging copy)
+    const bool direct_in = n && !np && in.on_device && !in.recs && !in.drec && in.kind && in.dst && in.w && in.ts;
+    if (direct_in) {
+        if (in.seq) CK(cudaMemcpyAsync(Wq, in.seq, n * 8, cudaMemcpyDeviceToDevice, st));
+        else { k_fill_seq<<<g1(n), 256, 0, st>>>(Wq, 0, n, r->next_seq); CKL(); }
+    } else if (n && in.recs) {
         k_unpack_recs<<<g1(n), 256, 0, st>>>(in.recs, n, Wk + np, Ws + np, Wd + np, Ww + np, Wt + np, Wq + np);
         CKL();
     } else if (n && in.drec) {
@@ -346,16 +351,12 @@ h2tap_status apply_core(h2tap_replica* r, const BatchIn& in, uint64_t S, bool cr
         if (in.seq) copy_in(r, Wq + np, in.seq, n, in.on_device);
         else { k_fill_seq<<<g1(n), 256, 0, st>>>(Wq, np, n, r->next_seq); CKL(); }
     }
-    Ops ops{Wk, Ws, Wd, Ww, Wt, Wq};
+    const Ops ops = direct_in ? Ops{in.kind, in.src, in.dst, in.w, in.ts, Wq} : Ops{Wk, Ws, Wd, Ww, Wt, Wq};
 
-    Counters init{};
-    init.ts_min = ~0ull;
-    init.v_min = ~0ull;
     r->get<Counters>(r->ctr, 1);
-    *r->hc = init;
-    CK(cudaMemcpyAsync(r->ctr.p, r->hc, sizeof(Counters), cudaMemcpyHostToDevice, st));
-    g_h2d += sizeof(Counters);
     Counters* dc = r->dctr();
+    k_init_counters<<<1, 32, 0, st>>>(dc);
+    CKL();
 
     uint32_t* idx_p = r->get<uint32_t>(r->idx_p, m);
     uint32_t* idx_n = r->get<uint32_t>(r->idx_n, m);
@@ -416,14 +417,14 @@ h2tap_status apply_core(h2tap_replica* r, const BatchIn& in, uint64_t S, bool cr
         // stable by ts, then stable by vertex
         const int vb = bits_for(hc.v_max - hc.v_min), tb = bits_for(hc.ts_max - hc.ts_min);
         if (vb + tb <= 64) {
-            k_node_keys<<<g1(n_node), 256, 0, st>>>(idx_n, n_node, Ws, hc.v_min, Wt, hc.ts_min, tb, kA, vA);
+            k_node_keys<<<g1(n_node), 256, 0, st>>>(idx_n, n_node, ops.src, hc.v_min, ops.ts, hc.ts_min, tb, kA, vA);
             CKL();
             radix_sort(r, kA, vA, kB, vB, n_node, vb + tb);
         } else {
-            k_keys_from<<<g1(n_node), 256, 0, st>>>(idx_n, n_node, Wt, hc.ts_min, kA, vA);
+            k_keys_from<<<g1(n_node), 256, 0, st>>>(idx_n, n_node, ops.ts, hc.ts_min, kA, vA);
             CKL();
             radix_sort(r, kA, vA, kB, vB, n_node, tb);
-            k_keys_from<<<g1(n_node), 256, 0, st>>>(vA, n_node, Ws, hc.v_min, kB, vB);
+            k_keys_from<<<g1(n_node), 256, 0, st>>>(vA, n_node, ops.src, hc.v_min, kB, vB);
             CKL();
             std::swap(kA, kB);
             std::swap(vA, vB);

@@ -42,6 +42,14 @@ struct Counters {
     unsigned int tiles[16];
 };
 
+__global__ void k_init_counters(Counters* c) {  // zero, with the two minima at their identity
+    constexpr int nw = sizeof(Counters) / 8;
+    static_assert(sizeof(Counters) % 8 == 0, "Counters is zeroed in 8-byte words");
+    for (int i = threadIdx.x; i < nw; i += blockDim.x) reinterpret_cast<unsigned long long*>(c)[i] = 0;
+    __syncwarp();
+    if (threadIdx.x == 0) { c->ts_min = ~0ull; c->v_min = ~0ull; }
+}
+
 // owned external-ID range of a shard: [lo, hi), hi == ~0 means "through UINT64_MAX"
 struct OwnRange {
     uint64_t lo, hi;

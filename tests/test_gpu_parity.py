@@ -263,3 +263,25 @@ def test_device_resident_batch(h2):
     o.apply(b, int(b.ts.max()))
     assert_same(g.export(), o.export(), "device batch")
     assert st["n_visible"] == len(b)
+
+
+def test_device_resident_batches_with_node_ops(h2):
+    """device batches are read in place when nothing is pending: node ops, deferral, then
+    a batch that lands on top of pending ops (the staged path)"""
+    import torch
+    shape = synth.LdbcShape(n_person=256, n_msg=8000, e_person=12000)
+    seed = synth.seed_of("c2") + 5
+    ids = synth.ldbc_vertices(shape)
+    src, dst, w = synth.ldbc_edges(shape, seed)
+    g, o = pair_from_edges(h2, shape.n_vertices, ids, src, dst, w)
+    ts = 0
+    for k in range(4):
+        b = synth.ldbc_batch(shape, seed, k, 4000, ts_base=ts)
+        dev = Batch(*(torch.from_numpy(a.view(np.int64) if a.dtype == np.uint64 else a).cuda()
+                      for a in (b.kind, b.src, b.dst, b.w, b.ts)))
+        snap = int(b.ts.max()) - (200 if k % 2 == 0 else 0)    # even batches leave ops pending
+        st = g.apply(dev, snap)
+        rc, ost = o.apply(b, snap)
+        assert rc == 0 and st["n_visible"] == ost["n_visible"] and st["n_deferred"] == ost["n_deferred"]
+        assert_same(g.export(), o.export(), f"device ldbc batch {k}")
+        ts = int(b.ts.max())

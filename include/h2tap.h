@@ -257,6 +257,43 @@ h2tap_status h2tap_pagerank(const h2tap_replica* r, double damping, int iteratio
 h2tap_status h2tap_sssp(const h2tap_replica* r, uint64_t source_ext, double* dist_out,
         int on_device);
 
+/* ---- freshness checks on a sharded replica (SURVEY.md §8(e) "Checks") ----------------
+ * Every shard keeps the whole ID map, so dense IDs are global and the per-vertex arrays
+ * below are GLOBAL (n_vertices of the whole graph = h2tap_replica_info's shard_vertex_base
+ * + ... over all shards; on one replica simply V), device-resident, caller-owned.  Each
+ * call does one shard's part of one step on the rows it owns; the caller combines the
+ * shards with a collective between steps (sharded.py: MAX of the BFS marks, SUM of the
+ * PageRank sums, MIN of the SSSP candidates).  The definitions are those of h2tap_bfs,
+ * h2tap_pagerank and h2tap_sssp (readings A18, A21).  Also valid on an unsharded replica. */
+/* dense ID of a live vertex (E_INVAL if absent or a tombstone) */
+h2tap_status h2tap_replica_lookup(const h2tap_replica* r, uint64_t ext_id, uint64_t* dense_out);
+/* BFS: mark[v] = 1 for every v with level[v] < 0 that an owned row u with level[u] == depth
+ * points to (mark zeroed by the caller) */
+h2tap_status h2tap_shard_bfs_expand(const h2tap_replica* r, const int32_t* level, int32_t depth,
+        uint8_t* mark);
+/* BFS: level[v] = depth + 1 where mark[v] and level[v] < 0 (mark = the MAX over shards);
+ * *n_new (host) = vertices settled */
+h2tap_status h2tap_shard_bfs_settle(const h2tap_replica* r, int32_t* level, const uint8_t* mark,
+        int32_t depth, uint64_t* n_new);
+/* PageRank: acc[v] += pr[u] / outdeg(u) over the owned rows' edges, *dangling (device, one
+ * double) += pr[u] of owned rows without out-edges (acc and dangling zeroed by the caller) */
+h2tap_status h2tap_shard_pr_push(const h2tap_replica* r, const double* pr, double* acc,
+        double* dangling);
+/* PageRank: acc (the SUM over shards) becomes the next rank vector in place:
+ * (1-d)/V + d * (acc[v] + dangling/V), dangling = the SUM over shards */
+h2tap_status h2tap_shard_pr_finish(const h2tap_replica* r, double* acc_to_rank,
+        const double* dangling, double damping);
+/* SSSP: *bad (host) = 1 if an owned edge weight is negative or NaN */
+h2tap_status h2tap_shard_check_weights(const h2tap_replica* r, int* bad);
+/* SSSP: nd[v] = min(nd[v], dist[u] + w(u,v)) over owned rows u with frontier[u]
+ * (nd starts as a copy of dist) */
+h2tap_status h2tap_shard_sssp_relax(const h2tap_replica* r, const uint8_t* frontier,
+        const double* dist, double* nd);
+/* SSSP: frontier[v] = nd[v] < dist[v], then dist = nd (nd = the MIN over shards);
+ * *n_changed (host) = vertices improved */
+h2tap_status h2tap_shard_sssp_settle(const h2tap_replica* r, double* dist, const double* nd,
+        uint8_t* frontier, uint64_t* n_changed);
+
 void h2tap_replica_destroy(h2tap_replica* r);
 const char* h2tap_status_str(h2tap_status s);
 const char* h2tap_last_error(void);

@@ -106,6 +106,16 @@ _lib.h2tap_bfs.restype = ctypes.c_int
 _lib.h2tap_bfs.argtypes = [_P, _u64, _P, ctypes.c_int]
 _lib.h2tap_sssp.restype = ctypes.c_int
 _lib.h2tap_sssp.argtypes = [_P, _u64, _P, ctypes.c_int]
+for _n, _a in (("h2tap_replica_lookup", [_P, _u64, ctypes.POINTER(_u64)]),
+               ("h2tap_shard_bfs_expand", [_P, _P, ctypes.c_int32, _P]),
+               ("h2tap_shard_bfs_settle", [_P, _P, _P, ctypes.c_int32, ctypes.POINTER(_u64)]),
+               ("h2tap_shard_pr_push", [_P, _P, _P, _P]),
+               ("h2tap_shard_pr_finish", [_P, _P, _P, ctypes.c_double]),
+               ("h2tap_shard_check_weights", [_P, ctypes.POINTER(ctypes.c_int)]),
+               ("h2tap_shard_sssp_relax", [_P, _P, _P, _P]),
+               ("h2tap_shard_sssp_settle", [_P, _P, _P, _P, ctypes.POINTER(_u64)])):
+    getattr(_lib, _n).restype = ctypes.c_int
+    getattr(_lib, _n).argtypes = _a
 _lib.h2tap_replica_liveness.restype = ctypes.c_int
 _lib.h2tap_replica_liveness.argtypes = [_P, _P, ctypes.c_int]
 _lib.h2tap_pagerank.restype = ctypes.c_int
@@ -359,6 +369,45 @@ class Replica:
         out = np.empty(self.info()["n_vertices"], np.uint8)
         _check(_lib.h2tap_replica_liveness(self._h, ctypes.c_void_p(out.ctypes.data), 0), "h2tap_replica_liveness")
         return out
+
+    # ---- one shard's part of a check step (device tensors; sharded.py combines shards)
+    def lookup(self, ext_id: int) -> int:
+        d = _u64()
+        _check(_lib.h2tap_replica_lookup(self._h, int(ext_id), ctypes.byref(d)), "h2tap_replica_lookup")
+        return d.value
+
+    def shard_bfs_expand(self, level, depth: int, mark):
+        _check(_lib.h2tap_shard_bfs_expand(self._h, _P(level.data_ptr()), int(depth), _P(mark.data_ptr())),
+               "h2tap_shard_bfs_expand")
+
+    def shard_bfs_settle(self, level, mark, depth: int) -> int:
+        n = _u64()
+        _check(_lib.h2tap_shard_bfs_settle(self._h, _P(level.data_ptr()), _P(mark.data_ptr()), int(depth),
+                                           ctypes.byref(n)), "h2tap_shard_bfs_settle")
+        return n.value
+
+    def shard_pr_push(self, pr, acc, dangling):
+        _check(_lib.h2tap_shard_pr_push(self._h, _P(pr.data_ptr()), _P(acc.data_ptr()), _P(dangling.data_ptr())),
+               "h2tap_shard_pr_push")
+
+    def shard_pr_finish(self, acc, dangling, damping: float):
+        _check(_lib.h2tap_shard_pr_finish(self._h, _P(acc.data_ptr()), _P(dangling.data_ptr()), float(damping)),
+               "h2tap_shard_pr_finish")
+
+    def shard_check_weights(self) -> int:
+        b = ctypes.c_int()
+        _check(_lib.h2tap_shard_check_weights(self._h, ctypes.byref(b)), "h2tap_shard_check_weights")
+        return b.value
+
+    def shard_sssp_relax(self, frontier, dist, nd):
+        _check(_lib.h2tap_shard_sssp_relax(self._h, _P(frontier.data_ptr()), _P(dist.data_ptr()), _P(nd.data_ptr())),
+               "h2tap_shard_sssp_relax")
+
+    def shard_sssp_settle(self, dist, nd, frontier) -> int:
+        n = _u64()
+        _check(_lib.h2tap_shard_sssp_settle(self._h, _P(dist.data_ptr()), _P(nd.data_ptr()), _P(frontier.data_ptr()),
+                                            ctypes.byref(n)), "h2tap_shard_sssp_settle")
+        return n.value
 
     def sssp(self, source_ext: int) -> np.ndarray:
         dist = np.empty(self.info()["n_vertices"], np.float64)

@@ -1336,6 +1336,143 @@ h2tap_status h2tap_sssp(const h2tap_replica* rc, uint64_t source_ext, double* di
     });
 }
 
+// ---- checks on a sharded replica: per-shard steps, combined by the
+// caller's collectives (paper_conf_edbt_jibrilabs23_b200/sharded.py)
+namespace {
+struct ShardView {
+    const int64_t* off;
+    const uint32_t* cols;
+    const float* w;
+    uint64_t Vr, row_lo, V;
+};
+ShardView shard_view(h2tap_replica* r) {
+    return ShardView{static_cast<const int64_t*>(r->off[r->cur].p), static_cast<const uint32_t*>(r->cols[r->cur].p),
+                     static_cast<const float*>(r->w[r->cur].p), r->Vr, r->row_lo, r->V};
+}
+unsigned warp_grid(h2tap_replica* r, uint64_t rows) {
+    return (unsigned)std::max<uint64_t>(1, std::min<uint64_t>(cdiv(rows * 32, 256), (uint64_t)r->n_sm * 32));
+}
+}  // namespace
+
+h2tap_status h2tap_replica_lookup(const h2tap_replica* rc, uint64_t ext_id, uint64_t* dense_out) {
+    h2tap_replica* r = const_cast<h2tap_replica*>(rc);
+    if (!r || !dense_out) { set_err("null argument"); return H2TAP_E_INVAL; }
+    return run_guarded(r, [&]() -> h2tap_status {
+        CK(cudaSetDevice(r->cfg.device));
+        const uint64_t k = dense_of(r, ext_id);
+        if (k >= r->V) { set_err("%llu is not a live vertex", (unsigned long long)ext_id); return H2TAP_E_INVAL; }
+        *dense_out = k;
+        return H2TAP_OK;
+    });
+}
+
+h2tap_status h2tap_shard_bfs_expand(const h2tap_replica* rc, const int32_t* level, int32_t depth, uint8_t* mark) {
+    h2tap_replica* r = const_cast<h2tap_replica*>(rc);
+    if (!r || !level || !mark) { set_err("null argument"); return H2TAP_E_INVAL; }
+    return run_guarded(r, [&]() -> h2tap_status {
+        CK(cudaSetDevice(r->cfg.device));
+        const ShardView s = shard_view(r);
+        if (s.Vr) { k_shard_bfs_expand<<<warp_grid(r, s.Vr), 256, 0, r->st>>>(s.off, s.cols, s.Vr, s.row_lo, level, depth, mark); CKL(); }
+        r->sync();
+        return H2TAP_OK;
+    });
+}
+
+h2tap_status h2tap_shard_bfs_settle(const h2tap_replica* rc, int32_t* level, const uint8_t* mark, int32_t depth,
+                                    uint64_t* n_new) {
+    h2tap_replica* r = const_cast<h2tap_replica*>(rc);
+    if (!r || !level || !mark || !n_new) { set_err("null argument"); return H2TAP_E_INVAL; }
+    return run_guarded(r, [&]() -> h2tap_status {
+        CK(cudaSetDevice(r->cfg.device));
+        unsigned long long* c = r->get<unsigned long long>(r->misc, 1);
+        CK(cudaMemsetAsync(c, 0, 8, r->st));
+        if (r->V) { k_shard_bfs_settle<<<g1(r->V), 256, 0, r->st>>>(level, mark, r->V, depth, c); CKL(); }
+        unsigned long long h = 0;
+        CK(cudaMemcpyAsync(&h, c, 8, cudaMemcpyDeviceToHost, r->st));
+        r->sync();
+        *n_new = h;
+        return H2TAP_OK;
+    });
+}
+
+h2tap_status h2tap_shard_pr_push(const h2tap_replica* rc, const double* pr, double* acc, double* dangling) {
+    h2tap_replica* r = const_cast<h2tap_replica*>(rc);
+    if (!r || !pr || !acc || !dangling) { set_err("null argument"); return H2TAP_E_INVAL; }
+    return run_guarded(r, [&]() -> h2tap_status {
+        CK(cudaSetDevice(r->cfg.device));
+        const ShardView s = shard_view(r);
+        if (s.Vr) { k_shard_pr_push<<<warp_grid(r, s.Vr), 256, 0, r->st>>>(s.off, s.cols, s.Vr, s.row_lo, pr, acc, dangling); CKL(); }
+        r->sync();
+        return H2TAP_OK;
+    });
+}
+
+h2tap_status h2tap_shard_pr_finish(const h2tap_replica* rc, double* acc_to_rank, const double* dangling, double damping) {
+    h2tap_replica* r = const_cast<h2tap_replica*>(rc);
+    if (!r || !acc_to_rank || !dangling) { set_err("null argument"); return H2TAP_E_INVAL; }
+    return run_guarded(r, [&]() -> h2tap_status {
+        CK(cudaSetDevice(r->cfg.device));
+        if (r->V) { k_shard_pr_finish<<<g1(r->V), 256, 0, r->st>>>(acc_to_rank, r->V, damping, dangling); CKL(); }
+        r->sync();
+        return H2TAP_OK;
+    });
+}
+
+h2tap_status h2tap_shard_check_weights(const h2tap_replica* rc, int* bad) {
+    h2tap_replica* r = const_cast<h2tap_replica*>(rc);
+    if (!r || !bad) { set_err("null argument"); return H2TAP_E_INVAL; }
+    return run_guarded(r, [&]() -> h2tap_status {
+        CK(cudaSetDevice(r->cfg.device));
+        unsigned long long* c = r->get<unsigned long long>(r->misc, 1);
+        CK(cudaMemsetAsync(c, 0, 8, r->st));
+        const ShardView s = shard_view(r);
+        const uint64_t E = r->E;
+        if (E) {
+            k_sssp_check_w<<<(unsigned)std::min<uint64_t>(cdiv(E, 256 * 8), (uint64_t)r->n_sm * 8), 256, 0, r->st>>>(
+                s.w, E, reinterpret_cast<unsigned int*>(c));
+            CKL();
+        }
+        unsigned int h = 0;
+        CK(cudaMemcpyAsync(&h, c, 4, cudaMemcpyDeviceToHost, r->st));
+        r->sync();
+        *bad = h ? 1 : 0;
+        return H2TAP_OK;
+    });
+}
+
+h2tap_status h2tap_shard_sssp_relax(const h2tap_replica* rc, const uint8_t* frontier, const double* dist, double* nd) {
+    h2tap_replica* r = const_cast<h2tap_replica*>(rc);
+    if (!r || !frontier || !dist || !nd) { set_err("null argument"); return H2TAP_E_INVAL; }
+    return run_guarded(r, [&]() -> h2tap_status {
+        CK(cudaSetDevice(r->cfg.device));
+        const ShardView s = shard_view(r);
+        if (s.Vr) {
+            k_shard_sssp_relax<<<warp_grid(r, s.Vr), 256, 0, r->st>>>(s.off, s.cols, s.w, s.Vr, s.row_lo, frontier, dist,
+                                                                    reinterpret_cast<unsigned long long*>(nd));
+            CKL();
+        }
+        r->sync();
+        return H2TAP_OK;
+    });
+}
+
+h2tap_status h2tap_shard_sssp_settle(const h2tap_replica* rc, double* dist, const double* nd, uint8_t* frontier,
+                                     uint64_t* n_changed) {
+    h2tap_replica* r = const_cast<h2tap_replica*>(rc);
+    if (!r || !dist || !nd || !frontier || !n_changed) { set_err("null argument"); return H2TAP_E_INVAL; }
+    return run_guarded(r, [&]() -> h2tap_status {
+        CK(cudaSetDevice(r->cfg.device));
+        unsigned long long* c = r->get<unsigned long long>(r->misc, 1);
+        CK(cudaMemsetAsync(c, 0, 8, r->st));
+        if (r->V) { k_shard_sssp_settle<<<g1(r->V), 256, 0, r->st>>>(dist, nd, frontier, r->V, c); CKL(); }
+        unsigned long long h = 0;
+        CK(cudaMemcpyAsync(&h, c, 8, cudaMemcpyDeviceToHost, r->st));
+        r->sync();
+        *n_changed = h;
+        return H2TAP_OK;
+    });
+}
+
 h2tap_status h2tap_replica_liveness(const h2tap_replica* rc, uint8_t* live_out, int on_device) {
     h2tap_replica* r = const_cast<h2tap_replica*>(rc);
     if (!r || !live_out) { set_err("null argument"); return H2TAP_E_INVAL; }

@@ -1950,6 +1950,77 @@ __global__ void k_fill_i32(int32_t* p, uint64_t n, int32_t v) {
     if (i < n) p[i] = v;
 }
 
+// ---------------------------------------------- checks on a sharded replica ----
+// (SURVEY.md §8(e) "Checks").  Global per-vertex arrays (every shard keeps the whole ID
+// map, so dense ids are global); each shard touches the rows it owns (local offsets,
+// global row = row_lo + i) and the caller combines the shards with a collective
+// (MAX of the BFS marks, SUM of the PageRank contributions, MIN of the distances).
+__global__ void k_shard_bfs_expand(const int64_t* __restrict__ off, const uint32_t* __restrict__ cols, uint64_t Vr,
+                                   uint64_t row_lo, const int32_t* __restrict__ level, int32_t depth,
+                                   uint8_t* __restrict__ mark) {
+    const uint64_t warp = (blockIdx.x * (uint64_t)blockDim.x + threadIdx.x) >> 5;
+    const uint64_t nwarps = ((uint64_t)gridDim.x * blockDim.x) >> 5;
+    for (uint64_t i = warp; i < Vr; i += nwarps) {
+        if (level[row_lo + i] != depth) continue;
+        for (int64_t e = off[i] + lane_id(); e < off[i + 1]; e += 32) {
+            const uint32_t v = cols[e];
+            if (level[v] < 0) mark[v] = 1;
+        }
+    }
+}
+__global__ void k_shard_bfs_settle(int32_t* __restrict__ level, const uint8_t* __restrict__ mark, uint64_t V,
+                                   int32_t depth, unsigned long long* __restrict__ n_new) {
+    const uint64_t v = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x;
+    bool nw = false;
+    if (v < V && mark[v] && level[v] < 0) { level[v] = depth + 1; nw = true; }
+    const uint32_t m = __ballot_sync(0xffffffffu, nw);
+    if (lane_id() == 0 && m) atomicAdd(n_new, (unsigned long long)__popc(m));
+}
+__global__ void k_shard_pr_push(const int64_t* __restrict__ off, const uint32_t* __restrict__ cols, uint64_t Vr,
+                                uint64_t row_lo, const double* __restrict__ pr, double* __restrict__ acc,
+                                double* __restrict__ dangling) {
+    const uint64_t warp = (blockIdx.x * (uint64_t)blockDim.x + threadIdx.x) >> 5;
+    const uint64_t nwarps = ((uint64_t)gridDim.x * blockDim.x) >> 5;
+    for (uint64_t i = warp; i < Vr; i += nwarps) {
+        const int64_t b = off[i], e = off[i + 1];
+        const double p = pr[row_lo + i];
+        if (b == e) { if (lane_id() == 0) atomicAdd(dangling, p); continue; }
+        const double c = p / (double)(e - b);
+        for (int64_t x = b + lane_id(); x < e; x += 32) atomicAdd(&acc[cols[x]], c);
+    }
+}
+__global__ void k_shard_pr_finish(double* __restrict__ nxt, uint64_t V, double d, const double* __restrict__ dsum) {
+    const uint64_t v = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x;
+    if (v < V) nxt[v] = (1.0 - d) / (double)V + d * (nxt[v] + *dsum / (double)V);
+}
+__global__ void k_shard_sssp_relax(const int64_t* __restrict__ off, const uint32_t* __restrict__ cols,
+                                   const float* __restrict__ w, uint64_t Vr, uint64_t row_lo,
+                                   const uint8_t* __restrict__ frontier, const double* __restrict__ dist,
+                                   unsigned long long* nd) {
+    const uint64_t warp = (blockIdx.x * (uint64_t)blockDim.x + threadIdx.x) >> 5;
+    const uint64_t nwarps = ((uint64_t)gridDim.x * blockDim.x) >> 5;
+    for (uint64_t i = warp; i < Vr; i += nwarps) {
+        if (!frontier[row_lo + i]) continue;
+        const double du = dist[row_lo + i];
+        for (int64_t e = off[i] + lane_id(); e < off[i + 1]; e += 32) {
+            const unsigned long long b = (unsigned long long)__double_as_longlong(du + (double)w[e]);
+            if (b < ld_volatile(reinterpret_cast<const uint64_t*>(nd + cols[e]))) atomicMin(nd + cols[e], b);
+        }
+    }
+}
+__global__ void k_shard_sssp_settle(double* __restrict__ dist, const double* __restrict__ nd, uint8_t* __restrict__ frontier,
+                                    uint64_t V, unsigned long long* __restrict__ n_changed) {
+    const uint64_t v = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x;
+    bool ch = false;
+    if (v < V) {
+        ch = nd[v] < dist[v];
+        frontier[v] = ch ? 1 : 0;
+        if (ch) dist[v] = nd[v];
+    }
+    const uint32_t m = __ballot_sync(0xffffffffu, ch);
+    if (lane_id() == 0 && m) atomicAdd(n_changed, (unsigned long long)__popc(m));
+}
+
 // ---------------------------------------------------------- PageRank ----
 // live (nullable, tombstone mode): PageRank of the live subgraph, nl = live vertices;
 // a tombstoned vertex has no edges and rank 0

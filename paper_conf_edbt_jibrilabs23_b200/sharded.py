@@ -13,6 +13,13 @@ The exchange step a8 around the per-shard pipeline:
 6. shard bases (first global row, first global edge) come from an all-gather of the
    shards' row and edge counts.
 
+Freshness checks on the sharded replica (SURVEY.md §8(e) "Checks"): every shard keeps the
+whole ID map, so per-vertex state is a GLOBAL device array replicated on every rank; each
+step runs one library kernel per shard over the rows it owns and one collective combines
+the shards — BFS: MAX of the next-frontier marks per level; PageRank: SUM of the pushed
+contributions and of the dangling mass per iteration; SSSP: MIN of the relaxed distances
+per round.  The loops stop on counts that are identical on every rank.
+
 The compute runs in the library's kernels (route packing included); this module is
 orchestration only.  The engine is anything with validate / pack / apply_routed /
 local_sizes (the CUDA replica here, an oracle-backed shard in the CPU tests).
@@ -75,6 +82,31 @@ class LibEngine:
         inf = self.rep.info()
         return inf["n_vertices"], inf["n_edges"], inf["shard_vertex_base"]
 
+    # one shard's part of a check step (library kernels)
+    def lookup(self, ext_id):
+        return self.rep.lookup(ext_id)
+
+    def bfs_expand(self, level, depth, mark):
+        self.rep.shard_bfs_expand(level, depth, mark)
+
+    def bfs_settle(self, level, mark, depth):
+        return self.rep.shard_bfs_settle(level, mark, depth)
+
+    def pr_push(self, pr, acc, dangling):
+        self.rep.shard_pr_push(pr, acc, dangling)
+
+    def pr_finish(self, acc, dangling, damping):
+        self.rep.shard_pr_finish(acc, dangling, damping)
+
+    def check_weights(self):
+        return self.rep.shard_check_weights()
+
+    def sssp_relax(self, frontier, dist, nd):
+        self.rep.shard_sssp_relax(frontier, dist, nd)
+
+    def sssp_settle(self, dist, nd, frontier):
+        return self.rep.shard_sssp_settle(dist, nd, frontier)
+
 
 class ShardedReplica:
     def __init__(self, engine, rank: int, world: int, device, group=None):
@@ -119,6 +151,71 @@ class ShardedReplica:
         self.next_seq += sum(sizes)
         stats["global_batch"] = sum(sizes)
         return stats
+
+    def _allreduce(self, t, op):
+        """collective on a device tensor (gloo: through a host copy)"""
+        if t.device == self.coll:
+            dist.all_reduce(t, op=op, group=self.group)
+            return t
+        h = t.to(self.coll)
+        dist.all_reduce(h, op=op, group=self.group)
+        t.copy_(h)
+        return t
+
+    def n_vertices(self) -> int:
+        """global vertex count = the shards' rows summed"""
+        v = self._i64([self.engine.local_sizes()[0]])
+        dist.all_reduce(v, group=self.group)
+        return int(v.item())
+
+    def bfs(self, source_ext: int):
+        """BFS levels (int32, global dense order, -1 unreachable) on every rank."""
+        V = self.n_vertices()
+        src = self.engine.lookup(source_ext)
+        level = torch.full((V,), -1, dtype=torch.int32, device=self.device)
+        level[src] = 0
+        mark = torch.empty(V, dtype=torch.uint8, device=self.device)
+        depth = 0
+        while True:
+            mark.zero_()
+            self.engine.bfs_expand(level, depth, mark)
+            self._allreduce(mark, dist.ReduceOp.MAX)
+            if self.engine.bfs_settle(level, mark, depth) == 0:
+                return level
+            depth += 1
+
+    def pagerank(self, damping: float = 0.85, iterations: int = 20):
+        """PageRank (fp64, Graphalytics, reading A18) on every rank."""
+        V = self.n_vertices()
+        pr = torch.full((V,), 1.0 / V if V else 0.0, dtype=torch.float64, device=self.device)
+        for _ in range(iterations):
+            acc = torch.zeros(V, dtype=torch.float64, device=self.device)
+            dang = torch.zeros(1, dtype=torch.float64, device=self.device)
+            self.engine.pr_push(pr, acc, dang)
+            self._allreduce(acc, dist.ReduceOp.SUM)
+            self._allreduce(dang, dist.ReduceOp.SUM)
+            self.engine.pr_finish(acc, dang, damping)
+            pr = acc
+        return pr
+
+    def sssp(self, source_ext: int):
+        """SSSP distances (fp64, +inf unreachable, reading A21) on every rank."""
+        bad = self._i64([self.engine.check_weights()])
+        dist.all_reduce(bad, op=dist.ReduceOp.MAX, group=self.group)
+        if int(bad.item()):
+            raise H2tapError(-1, "sharded sssp", "negative or NaN edge weight")
+        V = self.n_vertices()
+        src = self.engine.lookup(source_ext)
+        d = torch.full((V,), float("inf"), dtype=torch.float64, device=self.device)
+        d[src] = 0.0
+        frontier = torch.zeros(V, dtype=torch.uint8, device=self.device)
+        frontier[src] = 1
+        while True:
+            nd = d.clone()
+            self.engine.sssp_relax(frontier, d, nd)
+            self._allreduce(nd, dist.ReduceOp.MIN)
+            if self.engine.sssp_settle(d, nd, frontier) == 0:
+                return d
 
     def bases(self):
         """(row base, edge base, rows, edges) of this shard in the global CSR."""

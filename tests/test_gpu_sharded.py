@@ -215,3 +215,63 @@ def test_routed_pack_and_apply(h2, P):
     # a stale op is reported by validate (before anything is applied)
     stale = Batch.of([(synth.EDGE_INSERT, int(ids[0]), int(ids[1]), 1.0, 3)])
     assert h2.STATUS[eng[0].validate(to_dev(stale))] == "E_STALE_TS"
+
+
+def test_sharded_checks_logical_shards(h2):
+    """BFS / SSSP / PageRank over P = 3 shards through the per-shard C-ABI steps, the
+    collectives emulated on the host (MAX / SUM / MIN across shards)."""
+    import torch
+    import oracle
+    P = 3
+    n = 1 << 11
+    src, dst, w = synth.rmat_edges(11, 17, n=10 * n)
+    ids = np.arange(n, dtype=np.uint64) * 7 + 3
+    src, dst = ids[src], ids[dst]
+    bounds = h2.balanced_bounds(src, P)
+    own = np.searchsorted(bounds[1:P], src, side="right")
+    shards = [h2.Replica.from_edges(n, ids, src[own == p], dst[own == p], w[own == p], rank=p, world=P,
+                                    shard_bounds=bounds) for p in range(P)]
+    off, cols, ww, gid = O1.from_edges(n, ids, src, dst, w).export()
+    dev = torch.device("cuda")
+    s_ext = int(gid[int(np.argmax(np.diff(off)))])
+    s = shards[0].lookup(s_ext)
+    assert all(g.lookup(s_ext) == s for g in shards)
+    # BFS
+    level = torch.full((n,), -1, dtype=torch.int32, device=dev)
+    level[s] = 0
+    depth = 0
+    while True:
+        marks = [torch.zeros(n, dtype=torch.uint8, device=dev) for _ in shards]
+        for g, m in zip(shards, marks):
+            g.shard_bfs_expand(level, depth, m)
+        mark = torch.stack(marks).amax(0)
+        if shards[0].shard_bfs_settle(level, mark, depth) == 0:
+            break
+        depth += 1
+    assert np.array_equal(level.cpu().numpy(), oracle.bfs(off, cols, s))
+    # PageRank
+    pr = torch.full((n,), 1.0 / n, dtype=torch.float64, device=dev)
+    for _ in range(20):
+        accs = [torch.zeros(n, dtype=torch.float64, device=dev) for _ in shards]
+        dangs = [torch.zeros(1, dtype=torch.float64, device=dev) for _ in shards]
+        for g, a, d in zip(shards, accs, dangs):
+            g.shard_pr_push(pr, a, d)
+        acc, dang = torch.stack(accs).sum(0), torch.stack(dangs).sum(0)
+        shards[0].shard_pr_finish(acc, dang, 0.85)
+        pr = acc
+    ref = oracle.pagerank(off, cols, 0.85, 20)
+    assert np.max(np.abs(pr.cpu().numpy() - ref) / ref) < 1e-6
+    # SSSP
+    assert all(g.shard_check_weights() == 0 for g in shards)
+    d = torch.full((n,), float("inf"), dtype=torch.float64, device=dev)
+    d[s] = 0.0
+    fr = torch.zeros(n, dtype=torch.uint8, device=dev)
+    fr[s] = 1
+    while True:
+        nds = [d.clone() for _ in shards]
+        for g, x in zip(shards, nds):
+            g.shard_sssp_relax(fr, d, x)
+        nd = torch.stack(nds).amin(0)
+        if shards[0].shard_sssp_settle(d, nd, fr) == 0:
+            break
+    assert np.array_equal(d.cpu().numpy(), oracle.sssp(off, cols, ww, s))

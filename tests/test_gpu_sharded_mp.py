@@ -42,8 +42,19 @@ def _worker(rank, world, port, q):
                                    for a in (sl.kind, sl.src, sl.dst, sl.w, sl.ts)))
             shr.apply(sl, ts if k != 2 else int(np.quantile(g.ts, 0.7)))
             outs.append((rep.export(), shr.bases()))
+        # freshness checks on the sharded replica (one collective per step)
+        source = None
+        for c in ids[:64]:
+            try:
+                rep.lookup(int(c))   # replicated ID map: the same answer on every rank
+                source = int(c)
+                break
+            except h2.H2tapError:
+                pass
+        checks = (source, shr.bfs(source).cpu().numpy(), shr.sssp(source).cpu().numpy(),
+                  shr.pagerank(0.85, 20).cpu().numpy())
         gathered = [None] * world
-        dist.all_gather_object(gathered, outs)
+        dist.all_gather_object(gathered, (outs, checks))
         if rank == 0:
             q.put(gathered)
         rep.close()
@@ -53,6 +64,7 @@ def _worker(rank, world, port, q):
 
 def test_two_process_sharded_apply():
     import torch.multiprocessing as mp
+    import oracle
     import synth
     from oracle import O1
 
@@ -66,7 +78,9 @@ def test_two_process_sharded_apply():
     procs = [ctx.Process(target=_worker, args=(r, world, port, q)) for r in range(world)]
     for p in procs:
         p.start()
-    gathered = q.get(timeout=300)
+    got = q.get(timeout=300)
+    gathered = [g[0] for g in got]
+    checks = [g[1] for g in got]
     for p in procs:
         p.join(120)
         assert p.exitcode == 0
@@ -96,3 +110,14 @@ def test_two_process_sharded_apply():
         assert np.array_equal(np.concatenate(cat_cols), cols), f"batch {k}: cols"
         assert np.array_equal(np.concatenate(cat_w).view(np.uint32), ww.view(np.uint32)), f"batch {k}: weights"
         assert np.array_equal(np.concatenate(cat_ids), gid), f"batch {k}: ext ids"
+
+    # checks: identical on both ranks, equal to the oracle on the unsharded graph
+    source = checks[0][0]
+    for c in checks[1:]:
+        assert c[0] == source and all(np.array_equal(a, b) for a, b in zip(c[1:], checks[0][1:]))
+    d = int(np.searchsorted(gid, np.uint64(source)))
+    assert gid[d] == source
+    assert np.array_equal(checks[0][1], oracle.bfs(off, cols, d))
+    assert np.array_equal(checks[0][2], oracle.sssp(off, cols, ww, d))
+    ref = oracle.pagerank(off, cols, 0.85, 20)
+    assert np.max(np.abs(checks[0][3] - ref) / ref) < 1e-6

@@ -76,6 +76,61 @@ class OracleShard:
         off, cols, w, ids, lo = self.own_rows()
         return len(ids), len(cols), lo
 
+    # one shard's part of a check step, plain numpy on CPU tensors (in place)
+    def lookup(self, x):
+        ids = self.o.export()[3]
+        k = int(np.searchsorted(ids, np.uint64(x)))
+        assert k < len(ids) and ids[k] == x
+        return k
+
+    def _rows(self):
+        off, cols, w, ids, lo = self.own_rows()
+        for i in range(len(ids)):
+            yield lo + i, cols[off[i]:off[i + 1]], w[off[i]:off[i + 1]]
+
+    def bfs_expand(self, level, depth, mark):
+        lv, mk = level.numpy(), mark.numpy()
+        for u, cs, _ in self._rows():
+            if lv[u] == depth:
+                for v in cs:
+                    if lv[v] < 0:
+                        mk[v] = 1
+
+    def bfs_settle(self, level, mark, depth):
+        lv, mk = level.numpy(), mark.numpy()
+        new = (mk == 1) & (lv < 0)
+        lv[new] = depth + 1
+        return int(new.sum())
+
+    def pr_push(self, pr, acc, dang):
+        p, a, d = pr.numpy(), acc.numpy(), dang.numpy()
+        for u, cs, _ in self._rows():
+            if len(cs) == 0:
+                d[0] += p[u]
+            for v in cs:
+                a[v] += p[u] / len(cs)
+
+    def pr_finish(self, acc, dang, damping):
+        a, V = acc.numpy(), len(acc)
+        a[:] = (1 - damping) / V + damping * (a + dang.numpy()[0] / V)
+
+    def check_weights(self):
+        return int(any((ws < 0).any() or np.isnan(ws).any() for _, _, ws in self._rows()))
+
+    def sssp_relax(self, frontier, dist_, nd):
+        f, d, n = frontier.numpy(), dist_.numpy(), nd.numpy()
+        for u, cs, ws in self._rows():
+            if f[u]:
+                for v, x in zip(cs, ws):
+                    n[v] = min(n[v], d[u] + float(x))
+
+    def sssp_settle(self, dist_, nd, frontier):
+        d, n, f = dist_.numpy(), nd.numpy(), frontier.numpy()
+        ch = n < d
+        f[:] = ch
+        d[ch] = n[ch]
+        return int(ch.sum())
+
 
 def _worker(rank, world, port, out):
     os.environ["MASTER_ADDR"], os.environ["MASTER_PORT"] = "127.0.0.1", str(port)
@@ -112,8 +167,11 @@ def _worker(rank, world, port, out):
             refused = False
         except H2tapError as e:
             refused = e.status == -5
+        # freshness checks through the sharded orchestration (one collective per step)
+        src0 = int(sh.engine.o.export()[3][0])
+        checks = (src0, sh.bfs(src0).numpy().copy(), sh.sssp(src0).numpy().copy(), sh.pagerank(0.85, 20).numpy().copy())
         gathered = [None] * world
-        dist.all_gather_object(gathered, (results, refused))
+        dist.all_gather_object(gathered, (results, refused, checks))
         if rank == 0:
             out.put(gathered)
     finally:
@@ -173,3 +231,12 @@ def test_sharded_exchange_over_gloo(world):
         assert np.array_equal(np.concatenate([p[2] for p in parts]).view(np.uint32), ww.view(np.uint32))
         ts += 300
     assert all(gathered[r][1] for r in range(world))  # every rank refused the bad batch
+    import oracle
+    src0, lv, dd, pr = gathered[0][2]
+    for r in range(1, world):
+        assert all(np.array_equal(a, b) for a, b in zip(gathered[r][2][1:], (lv, dd, pr)))
+    d0 = int(np.searchsorted(gid, np.uint64(src0)))
+    assert np.array_equal(lv, oracle.bfs(off, cols, d0))
+    assert np.array_equal(dd, oracle.sssp(off, cols, ww, d0))
+    ref = oracle.pagerank(off, cols, 0.85, 20)
+    assert np.max(np.abs(pr - ref) / ref) < 1e-9

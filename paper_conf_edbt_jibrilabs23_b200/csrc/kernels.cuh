@@ -823,6 +823,9 @@ __global__ void __launch_bounds__(kThreads) k_reduce_classify(ClassArgs a) {
     uint32_t vlo[kCItems], vhi[kCItems];
 #pragma unroll
     for (int j = 0; j < kCItems; ++j) { vlo[j] = 0; vhi[j] = (uint32_t)a.V_old; }
+    // Every probe reads the whole aligned 32-byte sector (8 columns) around the probe
+    // point — DRAM moves the sector anyway — and resolves the search if the boundary
+    // falls inside it, else narrows past the sector's ends.
     for (int step = 0; step < 48; ++step) {
         bool any = false;
 #pragma unroll
@@ -836,8 +839,22 @@ __global__ void __launch_bounds__(kThreads) k_reduce_classify(ClassArgs a) {
                 } else {
                     mid = (lo[j] + hi[j]) >> 1;
                 }
-                const uint32_t v = a.old_cols[mid];
-                if (v < colq[j]) { lo[j] = mid + 1; vlo[j] = v + 1; } else { hi[j] = mid; vhi[j] = v; }
+                const uint64_t base = mid & ~7ull;
+                const uint4* q = reinterpret_cast<const uint4*>(a.old_cols + base);
+                const uint4 x0 = q[0], x1 = q[1];  // 16 elements of slack past E (over-read)
+                const uint32_t x[8] = {x0.x, x0.y, x0.z, x0.w, x1.x, x1.y, x1.z, x1.w};
+                const uint32_t s0 = (uint32_t)((lo[j] > base ? lo[j] : base) - base);
+                const uint32_t e0 = (uint32_t)((hi[j] < base + 8 ? hi[j] : base + 8) - base);
+                uint32_t p = e0, xs = 0, xe = 0;  // first t in [s0, e0) with x[t] >= colq; x[s0], x[e0-1]
+#pragma unroll
+                for (int t = 7; t >= 0; --t) {
+                    if ((uint32_t)t >= s0 && (uint32_t)t < e0 && x[t] >= colq[j]) p = (uint32_t)t;
+                    if ((uint32_t)t == s0) xs = x[t];
+                    if ((uint32_t)t + 1 == e0) xe = x[t];
+                }
+                if (p > s0 && p < e0) { lo[j] = hi[j] = base + p; }                       // boundary inside
+                else if (p == s0) { hi[j] = base + s0; vhi[j] = xs; }                     // all >= colq
+                else { lo[j] = base + e0; vlo[j] = xe + 1; }                              // all < colq
                 any = true;
             }
         }

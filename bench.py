@@ -238,7 +238,7 @@ def run_gpu(args):
         rep = h2.Replica.from_edges(nv, ids, src[mine], dst[mine], w[mine], 0, device=dev_idx,
                                     rank=rank, world=world, shard_bounds=bounds)
         eng = LibEngine(rep, f"cuda:{dev_idx}")
-        shr = ShardedReplica(eng, rank, world, f"cuda:{dev_idx}")
+        shr = ShardedReplica(eng, rank, world, f"cuda:{dev_idx}", exchange=args.exchange)
     else:
         rep = h2.Replica.from_edges(nv, ids, src, dst, w, 0, device=dev_idx, tombstone=args.tombstone)
     del src, dst, w
@@ -387,7 +387,9 @@ def run_gpu(args):
             "higher_is_better": True, "scaling": "strong" if sharded else "weak", "vs_baseline": None,
             "dtype": "u32/f32", "data": "synthetic",
             "config": {"workload": wl.describe(), "name": args.config, "parallelism":
-                       (f"shard{world} (1D vertex ranges, all-to-all routing over {args.dist_backend})"
+                       (f"shard{world} (1D vertex ranges, " + (
+                           f"all-to-all routing over {args.dist_backend})" if args.exchange == "alltoall" else
+                           "fused pack-and-store into peer CUDA-IPC windows)")
                         if sharded else "replicas" if world > 1 else "single"),
                        "l2": "inputs larger than L2 (CSR ~%.1f GB per step)" % (path_bytes / 1e9),
                        "replica_vertices": info["n_vertices"], "replica_edges": info["n_edges"]},
@@ -434,6 +436,9 @@ def main():
     ap.add_argument("--input", default="ops", choices=["ops", "records"],
                     help="batch format: flat op SoA (h2tap_delta_apply) or the paper's delta records "
                          "(h2tap_delta_apply_records, §5.1 layout)")
+    ap.add_argument("--exchange", default="alltoall", choices=["alltoall", "p2p"],
+                    help="sharded exchange: pack + all-to-all (NCCL), or the fused pack-and-store kernel "
+                         "into peers' CUDA-IPC windows (h2tap_route_pack_p2p)")
     ap.add_argument("--tombstone", action="store_true",
                     help="tombstone-row replica (deleted nodes keep an empty row; reading A23)")
     ap.add_argument("--checks", action="store_true",

@@ -205,6 +205,25 @@ typedef struct {
 /* E_INVAL (unknown kind) / E_STALE_TS (ts <= snapshot) / OK for a batch slice. */
 h2tap_status h2tap_batch_validate(const h2tap_replica* r, const h2tap_batch* batch);
 
+/* ---- fused exchange over peer memory (pack-and-store into peers'
+ * windows instead of pack + all-to-all).  Protocol per sharded apply (sharded.py):
+ * (1) h2tap_route_count -> this rank's counts[world]; (2) the caller all-gathers the
+ * world x world count matrix C and places, for every destination d, this rank's records
+ * at offset sum_{s < rank} C[s][d] of d's receive window (rank-major global order, A5);
+ * (3) h2tap_route_pack_p2p writes them there directly — one kernel, its stores go over
+ * NVLink/NVSwitch to the peer-mapped windows — and returns when they are complete;
+ * (4) a barrier; (5) each rank applies its window with h2tap_delta_apply_routed.
+ * Windows are CUDA IPC allocations (h2tap_ipc_alloc on the owner, h2tap_ipc_open on the
+ * peers; the 64-byte handles travel through the caller's process group).  world <= 16. */
+h2tap_status h2tap_route_count(const h2tap_replica* r, const h2tap_batch* batch, uint64_t* counts);
+h2tap_status h2tap_route_pack_p2p(const h2tap_replica* r, const h2tap_batch* batch, uint64_t seq0,
+        h2tap_route_rec* const* peer_window /* host array [world] of device pointers */,
+        const uint64_t* peer_offset /* host [world], records */);
+h2tap_status h2tap_ipc_alloc(int device, size_t bytes, void** dptr, void* handle64);
+h2tap_status h2tap_ipc_open(int device, const void* handle64, void** dptr);
+h2tap_status h2tap_ipc_close(void* dptr);
+h2tap_status h2tap_ipc_free(void* dptr);
+
 /* Pack `batch` (on_device must be 1) into `out` (device, `capacity` records), grouped
  * by destination rank 0..world-1; counts[world] (host) receives the records per
  * destination.  Op i gets seq = seq0 + i.  Needs n_edge + world * n_node records; if

@@ -106,7 +106,13 @@ _lib.h2tap_bfs.restype = ctypes.c_int
 _lib.h2tap_bfs.argtypes = [_P, _u64, _P, ctypes.c_int]
 _lib.h2tap_sssp.restype = ctypes.c_int
 _lib.h2tap_sssp.argtypes = [_P, _u64, _P, ctypes.c_int]
-for _n, _a in (("h2tap_replica_lookup", [_P, _u64, ctypes.POINTER(_u64)]),
+for _n, _a in (("h2tap_route_count", [_P, ctypes.POINTER(_Batch), _P]),
+               ("h2tap_route_pack_p2p", [_P, ctypes.POINTER(_Batch), _u64, _P, _P]),
+               ("h2tap_ipc_alloc", [ctypes.c_int, ctypes.c_size_t, ctypes.POINTER(_P), _P]),
+               ("h2tap_ipc_open", [ctypes.c_int, _P, ctypes.POINTER(_P)]),
+               ("h2tap_ipc_close", [_P]),
+               ("h2tap_ipc_free", [_P]),
+               ("h2tap_replica_lookup", [_P, _u64, ctypes.POINTER(_u64)]),
                ("h2tap_shard_bfs_expand", [_P, _P, ctypes.c_int32, _P]),
                ("h2tap_shard_bfs_settle", [_P, _P, _P, ctypes.c_int32, ctypes.POINTER(_u64)]),
                ("h2tap_shard_pr_push", [_P, _P, _P, _P]),
@@ -130,6 +136,35 @@ _lib.h2tap_version.restype = ctypes.c_char_p
 
 def version() -> str:
     return _lib.h2tap_version().decode()
+
+
+class IpcWindow:
+    """A cudaMalloc'ed receive window shared with peer processes through CUDA IPC."""
+
+    def __init__(self, device: int, nbytes: int):
+        self.device, self.nbytes = device, int(nbytes)
+        self.ptr = _P()
+        self.handle = (ctypes.c_ubyte * 64)()
+        _check(_lib.h2tap_ipc_alloc(device, self.nbytes, ctypes.byref(self.ptr), self.handle), "h2tap_ipc_alloc")
+
+    def handle_bytes(self) -> bytes:
+        return bytes(self.handle)
+
+    @staticmethod
+    def open(device: int, handle: bytes) -> int:
+        p = _P()
+        h = (ctypes.c_ubyte * 64).from_buffer_copy(handle)
+        _check(_lib.h2tap_ipc_open(device, h, ctypes.byref(p)), "h2tap_ipc_open")
+        return int(p.value)
+
+    @staticmethod
+    def close_peer(ptr: int):
+        _check(_lib.h2tap_ipc_close(_P(ptr)), "h2tap_ipc_close")
+
+    def free(self):
+        if self.ptr:
+            _lib.h2tap_ipc_free(self.ptr)
+            self.ptr = _P()
 
 
 def balanced_bounds(src_ext, world: int) -> np.ndarray:
@@ -369,6 +404,20 @@ class Replica:
         out = np.empty(self.info()["n_vertices"], np.uint8)
         _check(_lib.h2tap_replica_liveness(self._h, ctypes.c_void_p(out.ctypes.data), 0), "h2tap_replica_liveness")
         return out
+
+    # ---- fused exchange (peer-memory windows; sharded.py runs the protocol)
+    def route_count(self, batch):
+        b, keep = self._batch(batch)
+        world = self._keep[-1].world if self._keep else 1
+        counts = (_u64 * max(1, world))()
+        _check(_lib.h2tap_route_count(self._h, ctypes.byref(b), counts), "h2tap_route_count")
+        return [int(x) for x in counts]
+
+    def route_pack_p2p(self, batch, seq0: int, windows, offsets):
+        b, keep = self._batch(batch)
+        ptrs = (_P * len(windows))(*[_P(int(x)) for x in windows])
+        offs = (_u64 * len(offsets))(*[int(x) for x in offsets])
+        _check(_lib.h2tap_route_pack_p2p(self._h, ctypes.byref(b), int(seq0), ptrs, offs), "h2tap_route_pack_p2p")
 
     # ---- one shard's part of a check step (device tensors; sharded.py combines shards)
     def lookup(self, ext_id: int) -> int:

@@ -1058,6 +1058,101 @@ h2tap_status h2tap_batch_validate(const h2tap_replica* rc, const h2tap_batch* b)
     });
 }
 
+namespace {
+// destination counts of a device batch slice (edge ops to the owner of their source,
+// node ops to every shard), read back to the host
+h2tap_status route_counts(h2tap_replica* r, const h2tap_batch* b, uint64_t* counts) {
+    const int P = r->cfg.world;
+    const uint64_t* bounds = static_cast<const uint64_t*>(r->bounds_dev.p);
+    unsigned long long* cnt = r->get<unsigned long long>(r->misc, P);
+    CK(cudaMemsetAsync(cnt, 0, P * 8, r->st));
+    if (b->n) {
+        k_route_count<<<(unsigned)std::min<uint64_t>(cdiv(b->n, 256), 148 * 8), 256, (P + 1) * 4, r->st>>>(b->kind, b->src, b->n, bounds, P, cnt);
+        CKL();
+    }
+    std::vector<unsigned long long> h(P);
+    CK(cudaMemcpyAsync(h.data(), cnt, P * 8, cudaMemcpyDeviceToHost, r->st));
+    r->sync();
+    for (int d = 0; d < P; ++d) counts[d] = h[d];
+    return H2TAP_OK;
+}
+bool route_batch_ok(h2tap_replica* r, const h2tap_batch* b, const char* who) {
+    if (!r->sharded) { set_err("%s: replica is not sharded", who); return false; }
+    if (b->n && (!b->on_device || !b->kind || !b->src || !b->ts)) { set_err("%s needs a device batch", who); return false; }
+    return true;
+}
+}  // namespace
+
+h2tap_status h2tap_route_count(const h2tap_replica* rc, const h2tap_batch* b, uint64_t* counts) {
+    h2tap_replica* r = const_cast<h2tap_replica*>(rc);
+    if (!r || !b || !counts) { set_err("null argument"); return H2TAP_E_INVAL; }
+    if (!route_batch_ok(r, b, "h2tap_route_count")) return H2TAP_E_INVAL;
+    return run_guarded(r, [&]() -> h2tap_status {
+        CK(cudaSetDevice(r->cfg.device));
+        return route_counts(r, b, counts);
+    });
+}
+
+h2tap_status h2tap_route_pack_p2p(const h2tap_replica* rc, const h2tap_batch* b, uint64_t seq0,
+                                  h2tap_route_rec* const* peer_out, const uint64_t* peer_offset) {
+    h2tap_replica* r = const_cast<h2tap_replica*>(rc);
+    if (!r || !b || !peer_out || !peer_offset) { set_err("null argument"); return H2TAP_E_INVAL; }
+    if (!route_batch_ok(r, b, "h2tap_route_pack_p2p")) return H2TAP_E_INVAL;
+    const int P = r->cfg.world;
+    if (P > kMaxP2P) { set_err("h2tap_route_pack_p2p: world %d > %d", P, kMaxP2P); return H2TAP_E_INVAL; }
+    return run_guarded(r, [&]() -> h2tap_status {
+        CK(cudaSetDevice(r->cfg.device));
+        if (!b->n) return H2TAP_OK;
+        PeerOut po{};
+        for (int d = 0; d < P; ++d) {
+            if (!peer_out[d]) { set_err("h2tap_route_pack_p2p: NULL receive buffer of shard %d", d); return H2TAP_E_INVAL; }
+            po.out[d] = reinterpret_cast<RouteRec*>(peer_out[d]);
+            po.off[d] = peer_offset[d];
+        }
+        const uint64_t nt = cdiv(b->n, kTile);
+        uint64_t* stt = r->get<uint64_t>(r->status, (uint64_t)P * nt);
+        unsigned int* ctr = r->get<unsigned int>(r->rs_ctr, 1);
+        CK(cudaMemsetAsync(stt, 0, (uint64_t)P * nt * 8, r->st));
+        CK(cudaMemsetAsync(ctr, 0, 4, r->st));
+        k_route_pack_p2p<<<(unsigned)nt, kThreads, 0, r->st>>>(b->kind, b->src, b->dst, b->weight, b->ts, b->n, seq0,
+                                                             static_cast<const uint64_t*>(r->bounds_dev.p), P, po,
+                                                             stt, nt, ctr);
+        CKL();
+        r->sync();  // the peer stores are complete when this returns
+        return H2TAP_OK;
+    });
+}
+
+// CUDA IPC receive windows for the fused exchange (cudaMalloc'ed: IPC handles need it)
+h2tap_status h2tap_ipc_alloc(int device, size_t bytes, void** dptr, void* handle64) {
+    if (!dptr || !handle64) { set_err("null argument"); return H2TAP_E_INVAL; }
+    if (cudaSetDevice(device) != cudaSuccess) { set_err("cudaSetDevice(%d) failed", device); return H2TAP_E_CUDA; }
+    if (cudaMalloc(dptr, bytes ? bytes : 64) != cudaSuccess) { set_err("cudaMalloc(%zu) failed", bytes); return H2TAP_E_NOMEM; }
+    cudaIpcMemHandle_t h;
+    const cudaError_t e = cudaIpcGetMemHandle(&h, *dptr);
+    if (e != cudaSuccess) { cudaFree(*dptr); *dptr = nullptr; set_err("cudaIpcGetMemHandle: %s", cudaGetErrorString(e)); return H2TAP_E_CUDA; }
+    static_assert(sizeof(h) == 64, "cudaIpcMemHandle_t is 64 bytes");
+    std::memcpy(handle64, &h, 64);
+    return H2TAP_OK;
+}
+h2tap_status h2tap_ipc_open(int device, const void* handle64, void** dptr) {
+    if (!dptr || !handle64) { set_err("null argument"); return H2TAP_E_INVAL; }
+    if (cudaSetDevice(device) != cudaSuccess) { set_err("cudaSetDevice(%d) failed", device); return H2TAP_E_CUDA; }
+    cudaIpcMemHandle_t h;
+    std::memcpy(&h, handle64, 64);
+    const cudaError_t e = cudaIpcOpenMemHandle(dptr, h, cudaIpcMemLazyEnablePeerAccess);
+    if (e != cudaSuccess) { *dptr = nullptr; set_err("cudaIpcOpenMemHandle: %s", cudaGetErrorString(e)); return H2TAP_E_CUDA; }
+    return H2TAP_OK;
+}
+h2tap_status h2tap_ipc_close(void* dptr) {
+    if (dptr && cudaIpcCloseMemHandle(dptr) != cudaSuccess) { set_err("cudaIpcCloseMemHandle failed"); return H2TAP_E_CUDA; }
+    return H2TAP_OK;
+}
+h2tap_status h2tap_ipc_free(void* dptr) {
+    if (dptr && cudaFree(dptr) != cudaSuccess) { set_err("cudaFree failed"); return H2TAP_E_CUDA; }
+    return H2TAP_OK;
+}
+
 h2tap_status h2tap_route_pack(const h2tap_replica* rc, const h2tap_batch* b, uint64_t seq0, h2tap_route_rec* out,
                               uint64_t capacity, uint64_t* counts) {
     h2tap_replica* r = const_cast<h2tap_replica*>(rc);

@@ -312,6 +312,60 @@ __global__ void __launch_bounds__(kThreads) k_route_pack(
     }
 }
 
+// Fused pack + exchange ("a fused pack-and-store kernel writing into
+// peers' windows"): one pass over the rank's batch slice compacts, per destination shard
+// d, the ops bound for d (node ops go to every shard) in arrival order and stores each
+// 40-byte route record straight into d's receive buffer — a peer-mapped (CUDA IPC)
+// pointer, so the stores travel over NVLink / NVSwitch — at d's offset for this rank
+// (the records of lower ranks come first: the global rank-major order, reading A5).
+constexpr int kMaxP2P = 16;
+struct PeerOut {
+    RouteRec* out[kMaxP2P];   // destination d's receive buffer (peer-mapped device pointer)
+    uint64_t off[kMaxP2P];    // this rank's first record slot in it
+};
+__global__ void __launch_bounds__(kThreads) k_route_pack_p2p(
+    const uint8_t* __restrict__ kind, const uint64_t* __restrict__ src, const uint64_t* __restrict__ dst,
+    const float* __restrict__ w, const uint64_t* __restrict__ ts, uint64_t n, uint64_t seq0,
+    const uint64_t* __restrict__ bounds, int P, PeerOut po, uint64_t* __restrict__ status, uint64_t nt,
+    unsigned int* __restrict__ ctr) {
+    __shared__ uint32_t s_tile;
+    __shared__ uint32_t s_cmp[kItems * kThreads / 32 + 1];
+    __shared__ uint64_t s_base;
+    if (threadIdx.x == 0) s_tile = atomicAdd(ctr, 1u);
+    __syncthreads();
+    const uint32_t tile = s_tile;
+    const uint64_t i0 = (uint64_t)tile * kTile + threadIdx.x;
+    int own[kItems];  // destination shard, -1 = every shard (node op), -2 = no item
+#pragma unroll
+    for (int j = 0; j < kItems; ++j) {
+        const uint64_t i = i0 + (uint64_t)j * kThreads;
+        own[j] = i >= n ? -2 : (kind[i] <= NODE_DELETE ? -1 : (int)owner_of(bounds, P, src[i]));
+    }
+    for (int d = 0; d < P; ++d) {
+        bool f[kItems];
+        uint32_t pos[kItems];
+#pragma unroll
+        for (int j = 0; j < kItems; ++j) f[j] = own[j] == -1 || own[j] == d;
+        const uint32_t tot = striped_compact<kThreads, kItems>(f, pos, s_cmp);
+        if (threadIdx.x < 32) {
+            const uint64_t b = lookback_warp(status + (uint64_t)d * nt, tile, tot);
+            if (lane_id() == 0) s_base = b;
+        }
+        __syncthreads();
+        RouteRec* out = po.out[d] + po.off[d] + s_base;
+#pragma unroll
+        for (int j = 0; j < kItems; ++j) {
+            if (!f[j]) continue;
+            const uint64_t i = i0 + (uint64_t)j * kThreads;
+            RouteRec r;
+            r.src = src[i]; r.dst = dst ? dst[i] : 0; r.ts = ts[i]; r.seq = seq0 + i;
+            r.w = w ? w[i] : 0.f; r.kind = kind[i]; r.pad[0] = r.pad[1] = r.pad[2] = 0;
+            out[pos[j]] = r;
+        }
+        __syncthreads();  // s_base is rewritten by the next destination's look-back
+    }
+}
+
 __global__ void k_unpack_recs(const RouteRec* __restrict__ recs, uint64_t n, uint8_t* kind, uint64_t* src,
                               uint64_t* dst, float* w, uint64_t* ts, uint64_t* seq) {
     const uint64_t i = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x;

@@ -32,7 +32,7 @@ import numpy as np
 import torch
 import torch.distributed as dist
 
-from . import ROUTE_REC_BYTES, H2tapError, Replica
+from . import ROUTE_REC_BYTES, H2tapError, IpcWindow, Replica
 
 
 class LibEngine:
@@ -78,6 +78,15 @@ class LibEngine:
     def apply_routed(self, recs, n: int, snapshot_ts: int):
         return self.rep.apply_routed(recs, n, snapshot_ts)
 
+    # fused exchange (peer-memory windows)
+    def route_count(self, batch):
+        self.launches += 1 if len(batch.kind) else 0
+        return self.rep.route_count(batch)
+
+    def pack_p2p(self, batch, seq0: int, windows, offsets):
+        self.launches += 1 if len(batch.kind) else 0
+        self.rep.route_pack_p2p(batch, seq0, windows, offsets)
+
     def local_sizes(self):
         inf = self.rep.info()
         return inf["n_vertices"], inf["n_edges"], inf["shard_vertex_base"]
@@ -108,10 +117,29 @@ class LibEngine:
         return self.rep.shard_sssp_settle(dist, nd, frontier)
 
 
+class _Ptr:
+    """device pointer with the data_ptr() interface the engine expects"""
+
+    def __init__(self, p):
+        self.p = p
+
+    def data_ptr(self):
+        return self.p
+
+
 class ShardedReplica:
-    def __init__(self, engine, rank: int, world: int, device, group=None):
+    def __init__(self, engine, rank: int, world: int, device, group=None, exchange: str = "alltoall"):
+        """exchange: "alltoall" (pack, then all-to-all over the process group) or "p2p"
+        (h2tap_route_pack_p2p stores every record straight into its destination's
+        CUDA-IPC window: the fused pack-and-exchange kernel; world <= 16)."""
         self.engine, self.rank, self.world, self.group = engine, rank, world, group
         self.device = torch.device(device)
+        if exchange not in ("alltoall", "p2p"):
+            raise ValueError("exchange must be 'alltoall' or 'p2p'")
+        self.exchange = exchange
+        self.win = None          # this rank's receive window (IpcWindow)
+        self.win_caps = None     # every rank's window capacity (records)
+        self.peers = None        # every rank's window, mapped here (device pointers)
         # gloo moves host tensors only: collectives on a CUDA engine then go through host
         # copies (tests / several ranks sharing one GPU); NCCL works on device memory
         self.coll = torch.device("cpu") if dist.get_backend(group) == "gloo" else self.device
@@ -136,6 +164,8 @@ class ShardedReplica:
         dist.all_gather(sizes, self._i64([n]), group=self.group)
         sizes = [int(s.item()) for s in sizes]
         seq0 = self.next_seq + sum(sizes[: self.rank])
+        if self.exchange == "p2p":
+            return self._apply_p2p(batch, seq0, sizes, snapshot_ts)
         # 3./4. pack by destination and exchange
         recs, counts = self.engine.pack(batch, seq0)
         send_c = self._i64(counts)
@@ -151,6 +181,56 @@ class ShardedReplica:
         self.next_seq += sum(sizes)
         stats["global_batch"] = sum(sizes)
         return stats
+
+    def _windows(self, need):
+        """(re)create receive windows so that rank d's holds need[d] records; collective,
+        and every rank takes the same decision (all know the whole count matrix)"""
+        if self.win_caps is not None and all(n <= c for n, c in zip(need, self.win_caps)):
+            return
+        mine_cap = self.win_caps[self.rank] if self.win_caps is not None else 0
+        if self.win is None or need[self.rank] > mine_cap:
+            if self.win is not None:
+                self.win.free()
+            mine_cap = max(1024, int(need[self.rank] * 1.5) + 1024)
+            self.win = IpcWindow(self.device.index or 0, mine_cap * ROUTE_REC_BYTES)
+        info = [None] * self.world
+        dist.all_gather_object(info, (self.win.handle_bytes(), mine_cap), group=self.group)
+        if self.peers is not None:
+            for r, p in enumerate(self.peers):
+                if r != self.rank and p:
+                    IpcWindow.close_peer(p)
+        self.peers = [self.win.ptr.value if r == self.rank else IpcWindow.open(self.device.index or 0, h)
+                      for r, (h, _) in enumerate(info)]
+        self.win_caps = [c for _, c in info]
+
+    def _apply_p2p(self, batch, seq0: int, sizes, snapshot_ts: int):
+        # 3. destination counts of every rank -> the world x world matrix
+        counts = self._i64(self.engine.route_count(batch))
+        mat = [torch.empty_like(counts) for _ in range(self.world)]
+        dist.all_gather(mat, counts, group=self.group)
+        C = np.array([m.tolist() for m in mat], dtype=np.int64)  # C[s][d]
+        need = C.sum(axis=0)
+        self._windows([int(x) for x in need])
+        offsets = C[: self.rank].sum(axis=0) if self.rank else np.zeros(self.world, np.int64)
+        # 4. one kernel packs and stores into the peers' windows; the barrier orders the
+        #    stores before the owners read their windows
+        self.engine.pack_p2p(batch, seq0, self.peers, [int(x) for x in offsets])
+        dist.barrier(group=self.group)
+        # 5. apply this rank's window
+        stats = self.engine.apply_routed(_Ptr(self.peers[self.rank]), int(need[self.rank]), snapshot_ts)
+        self.next_seq += sum(sizes)
+        stats["global_batch"] = sum(sizes)
+        return stats
+
+    def close(self):
+        if self.peers is not None:
+            for r, p in enumerate(self.peers):
+                if r != self.rank and p:
+                    IpcWindow.close_peer(p)
+            self.peers = None
+        if self.win is not None:
+            self.win.free()
+            self.win = None
 
     def _allreduce(self, t, op):
         """collective on a device tensor (gloo: through a host copy)"""

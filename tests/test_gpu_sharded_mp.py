@@ -13,7 +13,7 @@ import pytest
 pytestmark = pytest.mark.gpu
 
 
-def _worker(rank, world, port, q):
+def _worker(rank, world, port, q, exchange="alltoall"):
     os.environ["MASTER_ADDR"], os.environ["MASTER_PORT"] = "127.0.0.1", str(port)
     import torch
     import torch.distributed as dist
@@ -31,7 +31,7 @@ def _worker(rank, world, port, q):
         mine = np.searchsorted(bounds[1:world], src, side="right") == rank
         rep = h2.Replica.from_edges(shape.n_vertices, ids, src[mine], dst[mine], w[mine], rank=rank,
                                     world=world, shard_bounds=bounds)
-        shr = ShardedReplica(LibEngine(rep, "cuda:0"), rank, world, "cuda:0")
+        shr = ShardedReplica(LibEngine(rep, "cuda:0"), rank, world, "cuda:0", exchange=exchange)
         outs, ts = [], 0
         for k in range(4):
             g = synth.ldbc_batch(shape, seed, k, 5000, ts_base=ts)
@@ -57,12 +57,15 @@ def _worker(rank, world, port, q):
         dist.all_gather_object(gathered, (outs, checks))
         if rank == 0:
             q.put(gathered)
+        dist.barrier()
+        shr.close()
         rep.close()
     finally:
         dist.destroy_process_group()
 
 
-def test_two_process_sharded_apply():
+@pytest.mark.parametrize("exchange", ["alltoall", "p2p"])
+def test_two_process_sharded_apply(exchange):
     import torch.multiprocessing as mp
     import oracle
     import synth
@@ -75,7 +78,7 @@ def test_two_process_sharded_apply():
     s.close()
     ctx = mp.get_context("spawn")
     q = ctx.Queue()
-    procs = [ctx.Process(target=_worker, args=(r, world, port, q)) for r in range(world)]
+    procs = [ctx.Process(target=_worker, args=(r, world, port, q, exchange)) for r in range(world)]
     for p in procs:
         p.start()
     got = q.get(timeout=300)

@@ -1717,141 +1717,9 @@ __global__ void k_remap_blocks(uint64_t V, const uint32_t* __restrict__ dropped,
     shift[bk] = (d1 > d0 || i1 > i0) ? kRemapMixed : (int32_t)((int64_t)i0 - (int64_t)d0);
 }
 
-// ============================================================== a4 + a5 ====
-// New row offsets.  The per-row degree delta is non-zero only in rows that own
-// an inserted record or a removed element; its exclusive scan at row u is
-//   (kept old elements before row u's old start) + (inserted records in rows < u')
-// where both terms are ranks in sorted lists (no cascade) or the kept-before
-// table KR written by the merge's decoupled look-back (cascade).
-// Mode without node ops (identity ID map): the per-vertex degree delta
-// deg[u] = (#inserted records in row u) - (#deleted old edges in row u) is
-// scattered from the two sorted record lists, then one single-pass exclusive
-// scan (decoupled look-back) writes new_off[u] = old_off[u] + sum_{v<u} deg[v].
-__global__ void k_deg_scatter(const uint32_t* __restrict__ ins_row, const uint32_t* __restrict__ del_row,
-                              const Counters* __restrict__ c, int32_t* __restrict__ deg,
-                              int64_t* __restrict__ tsum, uint64_t row_lo) {
-    const uint64_t n_ins = c->n_ins, n_del = c->n_del;
-    uint64_t i = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x;
-    const bool ok = i < n_ins + n_del;
-    const bool is_ins = i < n_ins;
-    const uint32_t r = ok ? (uint32_t)((is_ins ? ins_row[i] : del_row[i - n_ins]) - row_lo) : 0;
-    // warp-aggregated: one atomic per (row, sign) group of the warp (hub rows get many records)
-    const uint64_t key = ok ? (((uint64_t)r << 1) | (is_ins ? 1u : 0u)) : ~0ull;
-    const uint32_t peers = __match_any_sync(0xffffffffu, key);
-    if (ok && lane_id() == (uint32_t)(__ffs(peers) - 1)) {
-        const int v = is_ins ? __popc(peers) : -__popc(peers);
-        atomicAdd(&deg[r], v);
-        atomicAdd(reinterpret_cast<unsigned long long*>(&tsum[r / kTile]), (unsigned long long)(int64_t)v);
-    }
-}
 
-// Device-wide exclusive scan of signed values (the per-tile degree-delta sums),
-// single pass with decoupled look-back.  Look-back words hold non-negative
-// values, so each tile aggregate is biased by +2^47 (|sum| < 2^36 per tile).
-__global__ void __launch_bounds__(kThreads) k_scan_exclusive_i64(const int64_t* __restrict__ in,
-        int64_t* __restrict__ out, uint64_t n, uint64_t* __restrict__ status, unsigned int* __restrict__ ctr) {
-    __shared__ uint32_t s_tile;
-    __shared__ int64_t s_scan[kThreads / 32 + 1];
-    __shared__ int64_t s_base;
-    if (threadIdx.x == 0) s_tile = atomicAdd(ctr, 1u);
-    __syncthreads();
-    const uint32_t tile = s_tile;
-    const uint64_t i0 = (uint64_t)tile * kTile + (uint64_t)threadIdx.x * kItems;
-    int64_t v[kItems], sum = 0;
-#pragma unroll
-    for (int j = 0; j < kItems; ++j) { v[j] = (i0 + j < n) ? in[i0 + j] : 0; sum += v[j]; }
-    int64_t tot, ex = block_exclusive_scan<kThreads>(sum, s_scan, &tot);
-    if (threadIdx.x < 32) {
-        const uint64_t bias = 1ull << 47;
-        uint64_t b = lookback_warp(status, tile, (uint64_t)(tot + (int64_t)bias));
-        if (lane_id() == 0) s_base = (int64_t)(b - (uint64_t)tile * bias);
-    }
-    __syncthreads();
-    int64_t run = s_base + ex;
-#pragma unroll
-    for (int j = 0; j < kItems; ++j) {
-        if (i0 + j < n) out[i0 + j] = run;
-        run += v[j];
-    }
-}
 
-// new_off[u] = old_off[u] + (tile base) + (exclusive prefix of deg inside the tile)
-__global__ void __launch_bounds__(kThreads) k_offsets_apply(const int64_t* __restrict__ old_off,
-        const int32_t* __restrict__ deg, uint64_t V, const int64_t* __restrict__ tbase, int64_t* __restrict__ new_off) {
-    __shared__ int64_t s_scan[kThreads / 32 + 1];
-    const uint64_t i0 = (uint64_t)blockIdx.x * kTile + (uint64_t)threadIdx.x * kItems;
-    int32_t d[kItems];
-    int64_t oo[kItems];
-    int64_t sum = 0;
-    if (i0 + kItems <= V) {
-        const int4* p = reinterpret_cast<const int4*>(deg + i0);
-        int4 a = p[0], b = p[1];
-        d[0] = a.x; d[1] = a.y; d[2] = a.z; d[3] = a.w; d[4] = b.x; d[5] = b.y; d[6] = b.z; d[7] = b.w;
-        const longlong2* q = reinterpret_cast<const longlong2*>(old_off + i0);
-#pragma unroll
-        for (int j = 0; j < kItems / 2; ++j) { longlong2 v = q[j]; oo[2 * j] = v.x; oo[2 * j + 1] = v.y; }
-    } else {
-#pragma unroll
-        for (int j = 0; j < kItems; ++j) { d[j] = (i0 + j < V) ? deg[i0 + j] : 0; oo[j] = (i0 + j < V) ? old_off[i0 + j] : 0; }
-    }
-#pragma unroll
-    for (int j = 0; j < kItems; ++j) sum += d[j];
-    int64_t tot, ex = block_exclusive_scan<kThreads>(sum, s_scan, &tot);
-    int64_t run = tbase[blockIdx.x] + ex;
-    int64_t o[kItems];
-#pragma unroll
-    for (int j = 0; j < kItems; ++j) { o[j] = oo[j] + run; run += d[j]; }
-    if (i0 + kItems <= V) {
-        longlong2* q = reinterpret_cast<longlong2*>(new_off + i0);
-#pragma unroll
-        for (int j = 0; j < kItems / 2; ++j) q[j] = make_longlong2(o[2 * j], o[2 * j + 1]);
-    } else {
-#pragma unroll
-        for (int j = 0; j < kItems; ++j) if (i0 + j < V) new_off[i0 + j] = o[j];
-    }
-}
 
-__global__ void __launch_bounds__(kThreads) k_offsets_scan(const int64_t* __restrict__ old_off, const int32_t* __restrict__ deg,
-        uint64_t V, int64_t* __restrict__ new_off, uint64_t* __restrict__ status, unsigned int* __restrict__ ctr) {
-    __shared__ uint32_t s_tile;
-    __shared__ int64_t s_scan[kThreads / 32 + 1];
-    __shared__ int64_t s_base;
-    if (threadIdx.x == 0) s_tile = atomicAdd(ctr, 1u);
-    __syncthreads();
-    const uint32_t tile = s_tile;
-    const uint64_t i0 = (uint64_t)tile * kTile + (uint64_t)threadIdx.x * kItems;  // blocked: 8 rows per thread
-    int32_t d[kItems];
-    int64_t oo[kItems];  // old offsets, loaded before the look-back so the loads overlap it
-    int64_t sum = 0;
-    if (i0 + kItems <= V) {
-        const int4* p = reinterpret_cast<const int4*>(deg + i0);
-        int4 a = p[0], b = p[1];
-        d[0] = a.x; d[1] = a.y; d[2] = a.z; d[3] = a.w; d[4] = b.x; d[5] = b.y; d[6] = b.z; d[7] = b.w;
-        const longlong2* q = reinterpret_cast<const longlong2*>(old_off + i0);
-#pragma unroll
-        for (int j = 0; j < kItems / 2; ++j) { longlong2 v = q[j]; oo[2 * j] = v.x; oo[2 * j + 1] = v.y; }
-    } else {
-#pragma unroll
-        for (int j = 0; j < kItems; ++j) { d[j] = (i0 + j < V) ? deg[i0 + j] : 0; oo[j] = (i0 + j < V) ? old_off[i0 + j] : 0; }
-    }
-#pragma unroll
-    for (int j = 0; j < kItems; ++j) sum += d[j];
-    int64_t tot, ex = block_exclusive_scan<kThreads>(sum, s_scan, &tot);
-    if (threadIdx.x < 32) {
-        // look-back values must be non-negative: bias each tile aggregate by +kTile*2^31
-        const uint64_t bias = (uint64_t)kTile << 31;
-        uint64_t b = lookback_warp(status, tile, (uint64_t)(tot + (int64_t)bias));
-        if (lane_id() == 0) s_base = (int64_t)(b - (uint64_t)tile * bias);
-    }
-    __syncthreads();
-    int64_t run = s_base + ex;
-#pragma unroll
-    for (int j = 0; j < kItems; ++j) {
-        uint64_t u = i0 + j;
-        if (u < V) new_off[u] = oo[j] + run;
-        run += d[j];
-    }
-}
 
 // rows of inserted (new) vertices: kept old elements before the old position they
 // are inserted at, plus inserted records in rows < their new id
@@ -1884,7 +1752,6 @@ __global__ void k_remap32(uint64_t V, const uint32_t* __restrict__ dropped, cons
     out[g] = make_uint2((uint32_t)(c0 - d0 + i0) | (i1 > i0 ? 0x80000000u : 0u), m);
 }
 
-__global__ void k_set_i64(int64_t* p, int64_t v) { *p = v; }
 // V == ~0: the vertex count of the new ID map is c->Vn (device-side)
 __global__ void k_row_range(const uint64_t* __restrict__ ext, uint64_t V, OwnRange own, Counters* c) {
     if (V == ~0ull) V = c->Vn;

@@ -195,7 +195,8 @@ void radix_sort(h2tap_replica* r, uint64_t*& k, uint32_t*& v, uint64_t*& k2, uin
     const int passes = (bits + 7) / 8;
     const uint64_t ntiles = cdiv(n, kRsTile);
     uint32_t* hist = r->get<uint32_t>(r->hist, kRsMaxPasses * 256);
-    uint64_t* dbase = r->get<uint64_t>(r->dbase, kRsMaxPasses * 256);
+    uint64_t* dbase = r->get<uint64_t>(r->dbase, kRsMaxPasses * 256 + kRsMaxPasses);
+    uint32_t* skip = reinterpret_cast<uint32_t*>(dbase + kRsMaxPasses * 256);
     uint64_t* st = r->get<uint64_t>(r->rs_status, (uint64_t)passes * ntiles * 256);
     uint32_t* ctr = r->get<uint32_t>(r->rs_ctr, kRsMaxPasses);
     CK(cudaMemsetAsync(hist, 0, kRsMaxPasses * 256 * sizeof(uint32_t), r->st));
@@ -204,12 +205,12 @@ void radix_sort(h2tap_replica* r, uint64_t*& k, uint32_t*& v, uint64_t*& k2, uin
     int grid = (int)std::min<uint64_t>(cdiv(n, 256 * 8), 148 * 8);
     rs_histogram<<<grid, 256, 0, r->st>>>(k, n, n_dev, passes, hist);
     CKL();
-    rs_digit_base<<<passes, 256, 0, r->st>>>(hist, dbase);
+    rs_digit_base<<<passes, 256, 0, r->st>>>(hist, dbase, n, n_dev, skip);
     CKL();
     CK(cudaFuncSetAttribute(rs_onesweep, cudaFuncAttributeMaxDynamicSharedMemorySize, kRsSmem));  // per device
     for (int p = 0; p < passes; ++p) {
         rs_onesweep<<<(unsigned)ntiles, kRsThreads, kRsSmem, r->st>>>(k, v, k2, v2, n, n_dev, 8 * p, dbase + p * 256,
-                                                              st + (uint64_t)p * ntiles * 256, ctr + p);
+                                                              st + (uint64_t)p * ntiles * 256, ctr + p, skip + p);
         CKL();
         std::swap(k, k2);
         std::swap(v, v2);

@@ -56,21 +56,28 @@ __global__ void __launch_bounds__(256) rs_histogram(const uint64_t* __restrict__
     }
 }
 
-// one block per pass: exclusive scan of the 256 digit counts
+// one block per pass: exclusive scan of the 256 digit counts; skip[p] = 1 when every key
+// has the same digit in pass p (the pass is the identity permutation: a plain copy)
 __global__ void __launch_bounds__(256) rs_digit_base(const uint32_t* __restrict__ hist,
-                                                     uint64_t* __restrict__ base) {
+                                                     uint64_t* __restrict__ base, uint64_t n,
+                                                     const unsigned long long* __restrict__ n_dev,
+                                                     uint32_t* __restrict__ skip) {
     __shared__ uint64_t sm[9];
     const int p = blockIdx.x;
+    n = rs_count(n, n_dev);
     uint64_t v = hist[p * 256 + threadIdx.x], tot;
     uint64_t e = block_exclusive_scan<256>(v, sm, &tot);
     base[p * 256 + threadIdx.x] = e;
+    if (threadIdx.x == 0) skip[p] = 0;
+    __syncthreads();
+    if (v == n) skip[p] = 1;
 }
 
 __global__ void __launch_bounds__(kRsThreads) rs_onesweep(
     const uint64_t* __restrict__ kin, const uint32_t* __restrict__ vin, uint64_t* __restrict__ kout,
     uint32_t* __restrict__ vout, uint64_t n, const unsigned long long* __restrict__ n_dev, int shift,
     const uint64_t* __restrict__ digit_base, uint64_t* __restrict__ status /* [ntiles][256] */,
-    uint32_t* __restrict__ tile_ctr) {
+    uint32_t* __restrict__ tile_ctr, const uint32_t* __restrict__ skip) {
     __shared__ uint32_t s_tile;
     __shared__ uint32_t s_wcnt[kRsWarps][256];
     __shared__ uint32_t s_dstart[256];
@@ -82,6 +89,14 @@ __global__ void __launch_bounds__(kRsThreads) rs_onesweep(
 
     const int tid = threadIdx.x, w = tid >> 5, l = lane_id();
     n = rs_count(n, n_dev);
+    if (*skip) {  // constant digit: stable order unchanged, copy this CTA's tile
+        for (uint64_t i = (uint64_t)blockIdx.x * kRsTile + tid; i < min(n, (uint64_t)(blockIdx.x + 1) * kRsTile);
+             i += kRsThreads) {
+            kout[i] = kin[i];
+            vout[i] = vin[i];
+        }
+        return;
+    }
     if (tid == 0) s_tile = atomicAdd(tile_ctr, 1u);
     for (int i = tid; i < kRsWarps * 256; i += kRsThreads) (&s_wcnt[0][0])[i] = 0;
     __syncthreads();

@@ -318,7 +318,9 @@ def run_gpu(args):
     value = updates_all / (ms_max / 1e3)
 
     # ---- e2e: pinned host batches through the public API, H2D inside the timed region
-    e_glob = [wl.batch(k0 + n_total + k) for k in range(args.steps)]
+    pipelined = not sharded and not records
+    n_ewarm = 2 if pipelined else 0  # staging slots allocated and warm before the timed region
+    e_glob = [wl.batch(k0 + n_total + k) for k in range(args.steps + n_ewarm)]
     e_host = [my_part(b) for b in e_glob]
     e_snaps = [int(b.ts.max()) for b in e_glob]
     e_glob_n = [len(b) for b in e_glob]
@@ -331,14 +333,26 @@ def run_gpu(args):
         return synth.Batch(*(tens(a).pin_memory() for a in (b.kind, b.src, b.dst, b.w, b.ts)))
 
     e_pin = [pinned(b) for b in e_host]
+    for k in range(n_ewarm):
+        apply(rep.stage(e_pin[k]), e_snaps[k])
+    e_pin, e_snaps, e_glob_n = e_pin[n_ewarm:], e_snaps[n_ewarm:], e_glob_n[n_ewarm:]
     torch.cuda.synchronize()
     if world > 1:
         dist.barrier()
     e_stats = []
     h2d0 = eng.h2d if sharded else 0
     ev0.record(stream)
-    for k in range(args.steps):
-        e_stats.append(apply(e_pin[k], e_snaps[k]))
+    if pipelined:
+        # h2tap_batch_stage: the H2D copy of batch k+1 runs on the copy engine while batch k
+        # is applied (the copies stay inside the timed region)
+        staged = rep.stage(e_pin[0])
+        for k in range(args.steps):
+            nxt = rep.stage(e_pin[k + 1]) if k + 1 < args.steps else None
+            e_stats.append(apply(staged, e_snaps[k]))
+            staged = nxt
+    else:
+        for k in range(args.steps):
+            e_stats.append(apply(e_pin[k], e_snaps[k]))
     ev1.record(stream)
     torch.cuda.synchronize()
     e_ms = ev0.elapsed_time(ev1)
@@ -405,6 +419,8 @@ def run_gpu(args):
                      "setup_s": setup_s},
             "gpu_launches": int(sum(s["n_launches"] for s in stats)),
             "e2e": {"value": e_value, "unit": "updates/s",
+                    "how": ("pinned host batches; h2tap_batch_stage copies batch k+1 while batch k is applied"
+                            if pipelined else "pinned host batches copied inside each apply"),
                     "h2d_bytes_per_step": int(sum(s["h2d_bytes"] for s in e_stats) / len(e_stats)),
                     "d2h_bytes_per_step": int(sum(s["d2h_bytes"] for s in e_stats) / len(e_stats))},
             "clocks": clk.summary(),

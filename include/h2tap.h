@@ -152,6 +152,17 @@ h2tap_status h2tap_replica_create_from_csr(const h2tap_config* cfg, size_t n_ver
 h2tap_status h2tap_delta_apply(h2tap_replica* r, const h2tap_batch* batch, uint64_t snapshot_ts,
         h2tap_apply_stats* stats /* nullable */);
 
+/* Stage the NEXT host batch: its host->device copy starts now on the replica's copy
+ * stream (pinned host memory makes it asynchronous) and `staged` receives a device
+ * batch in one of two library-owned slots.  Passing `staged` to h2tap_delta_apply
+ * orders the apply after the copy.  Typical pipeline — the copy of batch k+1 overlaps
+ * the apply of batch k (apply returns only when its cycle is done):
+ *     stage(b0, &s0); for k: { stage(b[k+1], &s[k+1]); apply(&s[k]); }
+ * At most two staged batches may be outstanding (the slots alternate); the host arrays
+ * must stay valid until the batch has been applied.  seq must be NULL (arrival order).
+ * The staged bytes are reported in the h2d_bytes of the apply that consumes them. */
+h2tap_status h2tap_batch_stage(h2tap_replica* r, const h2tap_batch* host, h2tap_batch* staged);
+
 /* ---- the paper's delta-store layout as a second input format ----
  * Delta records (§5.1 "Delta Store Architecture"): fixed-size records of
  * (transaction timestamp, node ID, validity flag, deleted flag, offset + count into the

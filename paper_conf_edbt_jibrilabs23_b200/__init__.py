@@ -106,7 +106,8 @@ _lib.h2tap_bfs.restype = ctypes.c_int
 _lib.h2tap_bfs.argtypes = [_P, _u64, _P, ctypes.c_int]
 _lib.h2tap_sssp.restype = ctypes.c_int
 _lib.h2tap_sssp.argtypes = [_P, _u64, _P, ctypes.c_int]
-for _n, _a in (("h2tap_route_count", [_P, ctypes.POINTER(_Batch), _P]),
+for _n, _a in (("h2tap_batch_stage", [_P, ctypes.POINTER(_Batch), ctypes.POINTER(_Batch)]),
+               ("h2tap_route_count", [_P, ctypes.POINTER(_Batch), _P]),
                ("h2tap_route_pack_p2p", [_P, ctypes.POINTER(_Batch), _u64, _P, _P]),
                ("h2tap_ipc_alloc", [ctypes.c_int, ctypes.c_size_t, ctypes.POINTER(_P), _P]),
                ("h2tap_ipc_open", [ctypes.c_int, _P, ctypes.POINTER(_P)]),
@@ -136,6 +137,16 @@ _lib.h2tap_version.restype = ctypes.c_char_p
 
 def version() -> str:
     return _lib.h2tap_version().decode()
+
+
+class StagedBatch:
+    """device batch in a library staging slot (h2tap_batch_stage); keeps the host arrays alive"""
+
+    def __init__(self, b, keep):
+        self.b, self.keep = b, keep
+
+    def __len__(self):
+        return int(self.b.n)
 
 
 class IpcWindow:
@@ -329,9 +340,21 @@ class Replica:
                                              int(snapshot_ts), ctypes.byref(st)), "h2tap_delta_apply_routed")
         return st.as_dict()
 
-    def apply(self, batch, snapshot_ts: int, raise_on_error: bool = True):
-        """h2tap_delta_apply; batch has .kind .src .dst .w .ts (numpy or torch CUDA)."""
+    def stage(self, batch) -> "StagedBatch":
+        """h2tap_batch_stage: start the host->device copy of the next batch (pinned host
+        arrays for an asynchronous copy); apply() the returned handle later."""
         b, keep = self._batch(batch)
+        out = _Batch()
+        _check(_lib.h2tap_batch_stage(self._h, ctypes.byref(b), ctypes.byref(out)), "h2tap_batch_stage")
+        return StagedBatch(out, keep)
+
+    def apply(self, batch, snapshot_ts: int, raise_on_error: bool = True):
+        """h2tap_delta_apply; batch has .kind .src .dst .w .ts (numpy or torch CUDA), or is
+        a StagedBatch from stage()."""
+        if isinstance(batch, StagedBatch):
+            b, keep = batch.b, batch.keep
+        else:
+            b, keep = self._batch(batch)
         st = ApplyStats()
         rc = _lib.h2tap_delta_apply(self._h, ctypes.byref(b), int(snapshot_ts), ctypes.byref(st))
         if raise_on_error:

@@ -108,6 +108,13 @@ inline int bits_for(uint64_t range) { return range == 0 ? 0 : 64 - __builtin_clz
 struct h2tap_replica {
     h2tap_config cfg{};
     cudaStream_t st = nullptr, st2 = nullptr;  // st2: side stream (cascade pass)
+    cudaStream_t st_copy = nullptr;            // host->device staging of the next batch
+    struct Stage {
+        Buf k, s, d, w, t;
+        cudaEvent_t ev = nullptr;
+        uint64_t bytes = 0;  // staged H2D bytes not yet accounted to an apply
+    } stg[2];
+    int stg_next = 0;
     cudaEvent_t evA = nullptr, evB = nullptr, evC = nullptr;
     uint64_t V = 0, E = 0, snap = 0, next_seq = 0, n_pend = 0;
     // sharding: V = global live vertices (the replicated ID map), the CSR holds the Vr rows
@@ -133,7 +140,8 @@ struct h2tap_replica {
     Buf casc_status;    // look-back words of the cascade scan (runs beside the edge-op phase)
     Buf live[2];        // tombstone mode: u8 liveness per dense id, double-buffered with ext
     Buf ctr;
-    Counters* hc = nullptr;  // pinned host mirror
+    Counters* hc = nullptr;      // pinned, device-mapped host mirror
+    Counters* hc_dev = nullptr;  // its device address: a kernel writes it (no copy engine)
     cudaEvent_t ev[8]{};
 
     void* dalloc(size_t bytes) {
@@ -175,8 +183,11 @@ struct h2tap_replica {
     bool identity_pending = false;  // identity flag of the ext buffer being built
     bool identity_of(int which) const { return which == ext_cur ? identity : identity_pending; }
     void read_counters() {
+        // a one-warp kernel stores the counters into the mapped host mirror: the read-back
+        // never queues on a copy engine behind a staged batch's H2D copy
         g_d2h += sizeof(Counters);
-        CK(cudaMemcpyAsync(hc, ctr.p, sizeof(Counters), cudaMemcpyDeviceToHost, st));
+        k_store_counters<<<1, 32, 0, st>>>(static_cast<const Counters*>(ctr.p), hc_dev);
+        CK(cudaGetLastError());
         sync();
     }
     Counters* dctr() { return static_cast<Counters*>(ctr.p); }
@@ -856,11 +867,14 @@ h2tap_replica* new_replica(const h2tap_config* cfg) {
         int lo = 0, hi = 0;
         CK(cudaDeviceGetStreamPriorityRange(&lo, &hi));
         CK(cudaStreamCreateWithPriority(&r->st2, cudaStreamNonBlocking, lo));
+        CK(cudaStreamCreateWithFlags(&r->st_copy, cudaStreamNonBlocking));
+        for (auto& g : r->stg) CK(cudaEventCreateWithFlags(&g.ev, cudaEventDisableTiming));
     }
     CK(cudaEventCreateWithFlags(&r->evA, cudaEventDisableTiming));
     CK(cudaEventCreateWithFlags(&r->evB, cudaEventDisableTiming));
     CK(cudaEventCreateWithFlags(&r->evC, cudaEventDisableTiming));
-    CK(cudaMallocHost(&r->hc, sizeof(Counters)));
+    CK(cudaHostAlloc(reinterpret_cast<void**>(&r->hc), sizeof(Counters), cudaHostAllocMapped));
+    CK(cudaHostGetDevicePointer(reinterpret_cast<void**>(&r->hc_dev), r->hc, 0));
     r->get<Counters>(r->ctr, 1);
     return r;
 }
@@ -883,6 +897,11 @@ void free_replica(h2tap_replica* r) {
     if (r->evB) cudaEventDestroy(r->evB);
     if (r->evC) cudaEventDestroy(r->evC);
     if (r->st2) { cudaStreamSynchronize(r->st2); cudaStreamDestroy(r->st2); }
+    if (r->st_copy) { cudaStreamSynchronize(r->st_copy); cudaStreamDestroy(r->st_copy); }
+    for (auto& g : r->stg) {
+        for (Buf* b : {&g.k, &g.s, &g.d, &g.w, &g.t}) if (b->p) r->dfree(b->p);
+        if (g.ev) cudaEventDestroy(g.ev);
+    }
     if (r->hc) cudaFreeHost(r->hc);
     delete r;
 }
@@ -1027,6 +1046,12 @@ h2tap_status h2tap_delta_apply(h2tap_replica* r, const h2tap_batch* b, uint64_t 
         }
         CK(cudaSetDevice(r->cfg.device));
         BatchIn in{b->n, b->on_device, b->seq, b->kind, b->src, b->dst, b->weight, b->ts, 0};
+        for (auto& g : r->stg)  // a batch staged by h2tap_batch_stage: its copy is ordered first
+            if (b->n && b->on_device && b->kind == g.k.p) {
+                CK(cudaStreamWaitEvent(r->st, g.ev, 0));
+                in.pre_h2d = g.bytes;
+                g.bytes = 0;
+            }
         return apply_core(r, in, snapshot_ts, false, stats);
     });
 }
@@ -1190,6 +1215,45 @@ h2tap_status h2tap_route_pack(const h2tap_replica* rc, const h2tap_batch* b, uin
             base += h[d];
         }
         r->sync();
+        return H2TAP_OK;
+    });
+}
+
+h2tap_status h2tap_batch_stage(h2tap_replica* r, const h2tap_batch* host, h2tap_batch* staged) {
+    if (!r || !host || !staged) { set_err("null argument"); return H2TAP_E_INVAL; }
+    if (host->on_device) { set_err("h2tap_batch_stage takes a host batch"); return H2TAP_E_INVAL; }
+    if (host->n && (!host->kind || !host->src || !host->ts)) { set_err("batch kind/src/ts must be non-NULL"); return H2TAP_E_INVAL; }
+    if (host->seq) { set_err("h2tap_batch_stage: explicit seq is not staged"); return H2TAP_E_INVAL; }
+    return run_guarded(r, [&]() -> h2tap_status {
+        CK(cudaSetDevice(r->cfg.device));
+        auto& g = r->stg[r->stg_next];
+        r->stg_next ^= 1;
+        const uint64_t n = host->n;
+        uint8_t* k = r->get<uint8_t>(g.k, n);
+        uint64_t* s = r->get<uint64_t>(g.s, n);
+        uint64_t* d = r->get<uint64_t>(g.d, n);
+        float* w = r->get<float>(g.w, n);
+        uint64_t* t = r->get<uint64_t>(g.t, n);
+        CK(cudaStreamSynchronize(r->st));  // buffers (re)allocated on the replica stream are ready
+        cudaStream_t cs = r->st_copy;
+        uint64_t bytes = 0;
+        auto cp = [&](void* dst, const void* src, uint64_t nb) {
+            if (!nb) return;
+            if (src) { CK(cudaMemcpyAsync(dst, src, nb, cudaMemcpyHostToDevice, cs)); bytes += nb; }
+            else CK(cudaMemsetAsync(dst, 0, nb, cs));
+        };
+        cp(k, host->kind, n);
+        cp(s, host->src, n * 8);
+        cp(d, host->dst, n * 8);
+        cp(w, host->weight, n * 4);
+        cp(t, host->ts, n * 8);
+        CK(cudaEventRecord(g.ev, cs));
+        g.bytes = bytes;
+        *staged = h2tap_batch{};
+        staged->n = n;
+        staged->on_device = 1;
+        staged->kind = k; staged->src = s; staged->dst = d; staged->weight = w; staged->ts = t;
+        staged->seq = nullptr;
         return H2TAP_OK;
     });
 }

@@ -42,6 +42,11 @@ struct Counters {
     unsigned int tiles[16];
 };
 
+__global__ void k_store_counters(const Counters* __restrict__ c, Counters* host_mapped) {
+    constexpr int nw = sizeof(Counters) / 8;
+    for (int i = threadIdx.x; i < nw; i += blockDim.x)
+        reinterpret_cast<volatile unsigned long long*>(host_mapped)[i] = reinterpret_cast<const unsigned long long*>(c)[i];
+}
 __global__ void k_init_counters(Counters* c) {  // zero, with the two minima at their identity
     constexpr int nw = sizeof(Counters) / 8;
     static_assert(sizeof(Counters) % 8 == 0, "Counters is zeroed in 8-byte words");

@@ -285,3 +285,27 @@ def test_device_resident_batches_with_node_ops(h2):
         assert rc == 0 and st["n_visible"] == ost["n_visible"] and st["n_deferred"] == ost["n_deferred"]
         assert_same(g.export(), o.export(), f"device ldbc batch {k}")
         ts = int(b.ts.max())
+
+
+def test_staged_batches_pipeline(h2):
+    """h2tap_batch_stage: batch k+1's copy overlaps batch k's apply; results as the oracle"""
+    import torch
+    src, dst, w = synth.rmat_edges(12, 33)
+    g, o = pair_from_edges(h2, 1 << 12, None, src, dst, w)
+    bs, ts = [], 0
+    for k in range(5):
+        b = synth.rmat_batch(12, 33, k, 6000, len(src), p_weight=0.1, ts_base=ts)
+        ts = int(b.ts.max())
+        bs.append(b)
+    pin = [Batch(*(torch.from_numpy(a.view(np.int64) if a.dtype == np.uint64 else a).pin_memory()
+                   for a in (b.kind, b.src, b.dst, b.w, b.ts))) for b in bs]
+    staged = g.stage(pin[0])
+    for k, b in enumerate(bs):
+        nxt = g.stage(pin[k + 1]) if k + 1 < len(bs) else None
+        snap = int(b.ts.max()) - (50 if k == 2 else 0)          # batch 3 lands on pending ops
+        st = g.apply(staged, snap)
+        rc, ost = o.apply(b, snap)
+        assert rc == 0 and st["n_visible"] == ost["n_visible"]
+        assert st["h2d_bytes"] >= b.nbytes()                    # the staged copy is accounted
+        assert_same(g.export(), o.export(), f"staged batch {k}")
+        staged = nxt

@@ -293,9 +293,6 @@ ExtIndex ext_index(h2tap_replica* r) {
     return X;
 }
 
-#ifndef H2TAP_ROWS_SIDE
-#define H2TAP_ROWS_SIDE 0
-#endif
 #ifndef H2TAP_MERGE_CTAS
 #define H2TAP_MERGE_CTAS 0
 #endif
@@ -414,7 +411,6 @@ h2tap_status apply_core(h2tap_replica* r, const BatchIn& in, uint64_t S, bool cr
     uint64_t* new_ext = nullptr;
     uint32_t* casc_mask = nullptr;
     bool casc_pending = false;  // cascade pass in flight on the side stream
-    bool rows_pending = false;  // row pass in flight on the side stream (H2TAP_ROWS_SIDE)
     uint64_t *casc_cnt = nullptr, *casc_pre = nullptr;
     uint16_t* casc_wrel = nullptr;
     const int64_t* old_off_nc = static_cast<const int64_t*>(r->off[r->cur].p);
@@ -608,18 +604,7 @@ h2tap_status apply_core(h2tap_replica* r, const BatchIn& in, uint64_t S, bool cr
     float* new_w = r->get<float>(r->w[nb], Ecap);
     // node mode: survivors' ID map + row offsets before the merge, while the cascade
     // tables written by the cascade pass are still L2-resident (the merge streams the CSR)
-    if (casc_pending) {  // join the cascade pass
-        CK(cudaStreamWaitEvent(st, r->evB, 0));
-        casc_pending = false;
-        TR("casc_join");
-    }
     if (node_mode) {
-        cudaStream_t st = r->st;  // the row pass's stream (shadows the replica stream)
-        if (H2TAP_ROWS_SIDE) {    // beside the merge: both stream, neither reads the other's output
-            CK(cudaEventRecord(r->evA, r->st));
-            CK(cudaStreamWaitEvent(r->st2, r->evA, 0));
-            st = r->st2;
-        }
         RowArgs ra{};
         ra.old_off = old_off - row_lo; ra.V_old = V; ra.E_old = E; ra.R = R;
         ra.row_lo = row_lo; ra.row_hi = row_lo + Vr;
@@ -638,8 +623,15 @@ h2tap_status apply_core(h2tap_replica* r, const BatchIn& in, uint64_t S, bool cr
         const uint64_t ncta = cdiv(V, kRowTile);
         ra.part = r->get<uint64_t>(r->opart, 2 * (ncta + 1));
         if (V) {
-            k_rows_partition<><<<g1(ncta + 1), 256, 0, st>>>(ra);
+            k_rows_partition<><<<g1(ncta + 1), 256, 0, st>>>(ra);  // reads no cascade table
             CKL();
+        }
+        if (casc_pending) {  // join the cascade pass (side stream) before its tables are read
+            CK(cudaStreamWaitEvent(st, r->evB, 0));
+            casc_pending = false;
+            TR("casc_join");
+        }
+        if (V) {
             k_rows_fused<<<(unsigned)ncta, kThreads, 0, st>>>(ra);  // survivors: ID map + row offsets
             CKL();
         }
@@ -652,10 +644,6 @@ h2tap_status apply_core(h2tap_replica* r, const BatchIn& in, uint64_t S, bool cr
         uint64_t* f = r->get<uint64_t>(r->fence[ec ^ 1], n_fence(Vn_ub));
         k_build_fence_dev<<<g1(n_fence(Vn_ub)), 256, 0, st>>>(new_ext, dc, f);
         CKL();
-        if (H2TAP_ROWS_SIDE) {
-            CK(cudaEventRecord(r->evC, st));
-            rows_pending = true;
-        }
     }
     // ---- a4/a5 without node ops: row offsets (while the outcome lists are L2-resident)
     if (Vr && !node_mode) {
@@ -729,7 +717,6 @@ h2tap_status apply_core(h2tap_replica* r, const BatchIn& in, uint64_t S, bool cr
             r->get<uint64_t>(r->pt[pn], n_pend_new), r->get<uint64_t>(r->pq[pn], n_pend_new));
         CKL();
     }
-    if (rows_pending) CK(cudaStreamWaitEvent(st, r->evC, 0));  // row pass (side stream) done
     k_finish<<<1, 1, 0, st>>>(dc, V, Vr, E, node_mode ? 1 : 0, r->sharded ? 1 : 0, new_ext, new_off);
     CKL();
     CK(cudaEventRecord(r->ev[5], st));

@@ -1,7 +1,7 @@
 #!/usr/bin/env python
 """Benchmark: delta updates/s merged into the GPU-resident CSR replica.
 
-    python bench.py [--gpus N] [--steps K] [--warmup W] [--config c2|c3|c1] [--impl h2tap|reference]
+    python bench.py [--gpus N] [--steps K] [--warmup W] [--config c2|c3|c1|c4] [--impl h2tap|reference]
 
 A step is one h2tap_delta_apply of one synthetic batch (all SURVEY.md §8(a)
 steps a1-a7) into the replica.  Default workload: BASELINE.json configs[1]
@@ -166,7 +166,7 @@ def cpu_cores():
 def oracle_sample(name: str, steps: int, warmup: int, target_s: float = 20.0):
     """Time O1 (single-threaded std::map replay + CSR export) on a scaled-down sample."""
     import oracle
-    scale_down = {"c1": 4, "c2": 128, "c3": 256}[name]
+    scale_down = {"c1": 4, "c2": 128, "c3": 256, "c4": 1024}[name]
     wl = Workload(name, scale_down)
     nv, ids, src, dst, w = wl.graph()
     o = oracle.O1.from_edges(nv, ids, src, dst, w)

@@ -221,7 +221,10 @@ def _torch_allocator(device: int):
     import torch
 
     def _alloc(ctx, nbytes, stream):
-        return torch.cuda.caching_allocator_alloc(int(nbytes), device, int(stream or 0))
+        try:
+            return torch.cuda.caching_allocator_alloc(int(nbytes), device, int(stream or 0))
+        except Exception:  # out of memory: NULL makes the library return H2TAP_E_NOMEM
+            return None
 
     def _free(ctx, p, stream):
         torch.cuda.caching_allocator_delete(int(p))

@@ -958,6 +958,22 @@ const char* h2tap_status_str(h2tap_status s) {
     return "unknown";
 }
 
+constexpr uint64_t kCreateChunk = 1ull << 28;  // edges per create cycle
+uint64_t create_chunk() {  // H2TAP_CREATE_CHUNK overrides it (tests of the chunked create)
+    const char* e = getenv("H2TAP_CREATE_CHUNK");
+    const uint64_t v = e ? strtoull(e, nullptr, 10) : 0;
+    return v ? v : kCreateChunk;
+}
+// free the per-cycle scratch sized by the largest cycle so far (after a create)
+void release_scratch(h2tap_replica* r) {
+    CK(cudaStreamSynchronize(r->st));
+    for (Buf* b : {&r->Wk, &r->Ws, &r->Wd, &r->Ww, &r->Wt, &r->Wq, &r->idx_p, &r->idx_n, &r->idx_e, &r->status,
+                   &r->keyA, &r->keyB, &r->valA, &r->valB, &r->rs_status, &r->op_flags, &r->op_ou, &r->op_ow,
+                   &r->ins_pos, &r->ins_row, &r->ins_col, &r->ins_w, &r->del_pos, &r->upd_pos, &r->upd_w,
+                   &r->del_row, &r->status2, &r->part, &r->KR})
+        if (b->p) r->release(*b);
+}
+
 h2tap_status h2tap_replica_create_from_edges(const h2tap_config* cfg, size_t n_vertices, const uint64_t* vertex_ids,
                                              size_t n_edges, const uint64_t* src, const uint64_t* dst, const float* w,
                                              int on_device, uint64_t create_ts, h2tap_replica** out) {
@@ -969,9 +985,19 @@ h2tap_status h2tap_replica_create_from_edges(const h2tap_config* cfg, size_t n_v
         r = new_replica(cfg);
         init_vertices(r, n_vertices, vertex_ids, on_device);
         r->snap = 0;
-        BatchIn in{n_edges, on_device, nullptr, nullptr, src, dst, w, nullptr, create_ts};
-        h2tap_status st = apply_core(r, in, create_ts, true, nullptr);
-        if (st != H2TAP_OK) return st;
+        // the edges go in as insert batches of at most kCreateChunk (in order: the last
+        // duplicate still wins), which bounds the scratch of one cycle; the scratch is
+        // released afterwards (later batches are far smaller than a whole graph)
+        const uint64_t chunk = create_chunk();
+        for (uint64_t off = 0; off < n_edges || off == 0; off += chunk) {
+            const uint64_t len = std::min<uint64_t>(chunk, n_edges - off);
+            BatchIn in{len, on_device, nullptr, nullptr, src ? src + off : nullptr, dst ? dst + off : nullptr,
+                       w ? w + off : nullptr, nullptr, create_ts};
+            h2tap_status st = apply_core(r, in, create_ts, true, nullptr);
+            if (st != H2TAP_OK) return st;
+            if (n_edges == 0) break;
+        }
+        release_scratch(r);
         r->snap = create_ts;
         r->next_seq = 0;
         return H2TAP_OK;

@@ -181,6 +181,8 @@ CONFIGS = {
     "c1": dict(index=0, kind="rmat", scale=16, edge_factor=16, batch=10_000, p_insert=0.8),
     "c2": dict(index=1, kind="ldbc", shape=LDBC_SF10, batch=100_000),
     "c3": dict(index=2, kind="rmat", scale=24, edge_factor=16, batch=1_000_000, p_insert=0.8),
+    # configs[3] at P = 1 (the single-GPU reference point of the sharded scaling runs)
+    "c4": dict(index=3, kind="rmat", scale=26, edge_factor=16, batch=8_000_000, p_insert=0.8),
 }
 
 

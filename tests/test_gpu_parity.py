@@ -309,3 +309,16 @@ def test_staged_batches_pipeline(h2):
         assert st["h2d_bytes"] >= b.nbytes()                    # the staged copy is accounted
         assert_same(g.export(), o.export(), f"staged batch {k}")
         staged = nxt
+
+
+def test_chunked_create_last_duplicate_wins(h2, monkeypatch):
+    """create_from_edges goes in as insert batches of H2TAP_CREATE_CHUNK edges (2^28 by
+    default); duplicates across chunks: the last one wins, as in one batch"""
+    monkeypatch.setenv("H2TAP_CREATE_CHUNK", "997")
+    src, dst, w = synth.rmat_edges(10, 44, n=20000)             # many duplicate (src, dst) pairs
+    ids = np.arange(1 << 10, dtype=np.uint64) * 2 + 1
+    g, o = pair_from_edges(h2, 1 << 10, ids, ids[src], ids[dst], w)
+    assert_same(g.export(), o.export(), "chunked create")
+    b = synth.rmat_batch(10, 44, 0, 3000, len(src), p_weight=0.1)
+    b.src, b.dst = ids[b.src % (1 << 10)], ids[b.dst % (1 << 10)]
+    step(g, o, b, int(b.ts.max()), "after chunked create")

@@ -706,22 +706,37 @@ __global__ void __launch_bounds__(kThreads) k_edge_prep(PrepArgs a) {
     bool valid[kEItems];
     uint32_t pos[kEItems];
     uint64_t ngated = 0, nbad = 0;
+    // the op fields of all items are loaded before any record is stored (the stores
+    // would otherwise order every later item's loads behind them: possible aliasing)
+    uint32_t oj[kEItems];
+    uint64_t sj[kEItems], dj[kEItems];
+#pragma unroll
+    for (int j = 0; j < kEItems; ++j) {
+        const uint64_t i = i0 + (uint64_t)j * kThreads;
+        oj[j] = i < a.n_edge ? a.edge_idx[i] : 0u;
+    }
+#pragma unroll
+    for (int j = 0; j < kEItems; ++j) {
+        const bool in = i0 + (uint64_t)j * kThreads < a.n_edge;
+        sj[j] = in ? a.ops.src[oj[j]] : 0;
+        dj[j] = in ? a.ops.dst[oj[j]] : 0;
+    }
 #pragma unroll
     for (int j = 0; j < kEItems; ++j) {
         uint64_t i = i0 + (uint64_t)j * kThreads;
         key[j] = 0;
         valid[j] = false;
         if (i >= a.n_edge) continue;
-        uint32_t o = a.edge_idx[i];
+        uint32_t o = oj[j];
         uint8_t kind = a.ops.kind[o];
         uint64_t ts = a.ops.ts[o], seq = a.ops.seq[o];
-        Lookup Lu = do_lookup(a, U, a.ops.src[o]);
-        Lookup Lw = do_lookup(a, U, a.ops.dst[o]);
+        Lookup Lu = do_lookup(a, U, sj[j]);
+        Lookup Lw = do_lookup(a, U, dj[j]);
         bool ok = Lu.final_live && Lw.final_live;
         if (a.create && !(Lu.old_present && Lw.old_present)) nbad++;
         // routed to the wrong shard: flagged (the apply fails) and dropped here, so the
         // rest of the cycle never indexes rows this shard does not hold
-        if (!a.own.owns(a.ops.src[o])) { nbad |= 1ull << 40; ok = false; }
+        if (!a.own.owns(sj[j])) { nbad |= 1ull << 40; ok = false; }
         if (ok && (Lu.hasD || Lw.hasD)) {
             // superseded by a later node delete of an endpoint (A8)
             if (Lu.hasD && pt_less(ts, seq, Lu.tD_ts, Lu.tD_seq)) ok = false;

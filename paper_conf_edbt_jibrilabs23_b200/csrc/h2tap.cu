@@ -761,7 +761,7 @@ h2tap_status apply_core(h2tap_replica* r, const BatchIn& in, uint64_t S, bool cr
         stats->n_upd = n_upd;
         stats->n_casc = n_casc;
         stats->n_vertex_inserted = fc.n_inserted;
-        stats->n_vertex_deleted = fc.n_dropped;
+        stats->n_vertex_deleted = fc.n_killed;  // live before the cycle, dead after it (both ID modes)
         stats->ms_ingest = ev_ms(r->ev[0], r->ev[1]);
         stats->ms_nodeops = ev_ms(r->ev[1], r->ev[2]);
         stats->ms_sort_reduce = ev_ms(r->ev[2], r->ev[3]);

@@ -39,6 +39,8 @@ struct Counters {
     unsigned long long n_casc;
     unsigned long long row_lo_new, row_hi_new;  // sharded: the shard's row range in the new ID map
     unsigned long long Vn, Vr_new, En, new_identity;  // written by k_finish
+    unsigned long long n_killed;  // vertices live before the cycle and dead after it (stats)
+    unsigned long long pad_;
     unsigned int tiles[16];
 };
 
@@ -508,7 +510,7 @@ __global__ void __launch_bounds__(kThreads) k_node_lists(
     const uint64_t U = c->n_unique, n_tiles = (U + kTile - 1) / kTile;  // grid: upper bound
     if (tile >= n_tiles) return;
     const uint64_t i0 = (uint64_t)tile * kTile + (uint64_t)threadIdx.x * kItems;
-    uint64_t cnt[3] = {0, 0, 0};
+    uint64_t cnt[3] = {0, 0, 0}, killed = 0;
     uint32_t fl[kItems];
 #pragma unroll
     for (int j = 0; j < kItems; ++j) {
@@ -518,9 +520,14 @@ __global__ void __launch_bounds__(kThreads) k_node_lists(
             uint32_t f = nv[i].flags;
             bool old = f & NV_OLD, live0 = f & NV_LIVE0, fin = f & NV_FINAL, hd = f & NV_HASD;
             if (live0 && !fin && !tomb) { fl[j] |= 1; cnt[0]++; }  // tombstone mode keeps the slot (A23)
+            if (live0 && !fin) killed++;
             if (!old && fin) { fl[j] |= 2; cnt[1]++; }
             if (live0 && hd) { fl[j] |= 4; cnt[2]++; }             // its old edges cascade
         }
+    }
+    {
+        const unsigned long long ks = warp_sum<unsigned long long>(killed);
+        if (lane_id() == 0 && ks) atomicAdd(&c->n_killed, ks);
     }
     uint64_t excl[3], tot[3];
 #pragma unroll

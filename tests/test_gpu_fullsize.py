@@ -86,7 +86,7 @@ def final_live_set(old_ids, batch):
     return np.union1d(old_ids[~np.isin(old_ids, dead)], born).astype(np.uint64)
 
 
-def run_config(h2, name, n_sample=3000):
+def run_config(h2, name, n_sample=3000, records=False, tombstone=False):
     cfg = synth.CONFIGS[name]
     seed = synth.seed_of(name)
     if cfg["kind"] == "ldbc":
@@ -100,16 +100,23 @@ def run_config(h2, name, n_sample=3000):
         ids = None
         src, dst, w = synth.rmat_edges(cfg["scale"], seed)
         batch = synth.rmat_batch(cfg["scale"], seed, 0, cfg["batch"], len(src), p_insert=cfg["p_insert"])
-    g = h2.Replica.from_edges(nv, ids, src, dst, w)
+    g = h2.Replica.from_edges(nv, ids, src, dst, w, tombstone=tombstone)
     del src, dst, w
     old = g.export()
     snap = int(batch.ts.max())
-    st = g.apply(batch, snap)
+    st = g.apply_records(synth.records_from_ops(batch), snap) if records else g.apply(batch, snap)
     new = g.export()
     off, cols, wn, ids_new = new
     check_invariants(off, cols, ids_new)
     assert len(cols) == len(old[1]) + st["n_new"] - st["n_del"] - st["n_casc"]       # I6
-    assert np.array_equal(ids_new, final_live_set(old[3], batch))                   # ID map
+    live_set = final_live_set(old[3], batch)
+    if tombstone:  # reading A23: old slots stay, the live flags say who is alive
+        assert np.array_equal(ids_new, np.union1d(old[3], live_set))
+        live = g.live()
+        assert np.array_equal(live == 1, np.isin(ids_new, live_set))
+        assert np.all(np.diff(off)[live == 0] == 0)                                # empty rows
+    else:
+        assert np.array_equal(ids_new, live_set)                                    # ID map
     # sample: the most-updated sources, random old rows, node-op vertices
     rng = np.random.default_rng(7)
     edge_src = batch.src[batch.kind >= 2]
@@ -135,8 +142,12 @@ def run_config(h2, name, n_sample=3000):
         checked += 1
     # sampled vertices the oracle says are dead must be absent on the GPU too
     dead = set(int(s) for s in sample) - set(ref_rows)
-    live_gpu = set(int(x) for x in ids_new[np.isin(ids_new, np.array(sorted(dead), np.uint64))]) if dead else set()
-    assert not live_gpu
+    if tombstone:
+        dk = np.isin(ids_new, np.array(sorted(dead), np.uint64)) if dead else np.zeros(len(ids_new), bool)
+        assert np.all(g.live()[dk] == 0)
+    else:
+        live_gpu = set(int(x) for x in ids_new[np.isin(ids_new, np.array(sorted(dead), np.uint64))]) if dead else set()
+        assert not live_gpu
     assert checked > 1000
     return st
 
@@ -149,3 +160,15 @@ def test_c3_rmat24_full_size(h2):
 def test_c2_ldbc_sf10_full_size(h2):
     st = run_config(h2, "c2")
     assert st["n_vertex_inserted"] > 0 and st["n_vertex_deleted"] > 0 and st["n_casc"] > 0
+
+
+def test_c2_full_size_records_input(h2):
+    """configs[1] through h2tap_delta_apply_records (the paper's delta-record layout)"""
+    st = run_config(h2, "c2", records=True)
+    assert st["n_vertex_inserted"] > 0 and st["n_casc"] > 0
+
+
+def test_c2_full_size_tombstone_rows(h2):
+    """configs[1] on a tombstone-row replica (reading A23)"""
+    st = run_config(h2, "c2", tombstone=True)
+    assert st["n_vertex_deleted"] > 0

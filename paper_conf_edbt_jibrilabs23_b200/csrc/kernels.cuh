@@ -1766,16 +1766,27 @@ __global__ void k_offsets_inserted(const NodeVtx* __restrict__ nv, const uint32_
 // dropped bitmask}; exact = an insertion point lies strictly inside the group
 __global__ void k_remap32(uint64_t V, const uint32_t* __restrict__ dropped, const uint32_t* __restrict__ ins_oldpos,
                           const Counters* __restrict__ c, uint2* __restrict__ out) {
-    const uint64_t n_dropped = c->n_dropped, n_vins = c->n_inserted;
-    const uint64_t g = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x;
-    if (g >= (V + 31) / 32) return;
+    // the CTA's id range narrows both sorted lists once (4 searches), then every group
+    // searches only its CTA's slices (empty for most CTAs)
+    __shared__ uint64_t s_rng[4];
+    const uint64_t n_dropped = c->n_dropped, n_vins = c->n_inserted, ng = (V + 31) / 32;
+    const uint64_t gb = (uint64_t)blockIdx.x * blockDim.x;
+    if (threadIdx.x < 4) {
+        const uint64_t lo = gb * 32, hi = min((gb + blockDim.x) * 32, (uint64_t)0xFFFFFFFFull);
+        const uint32_t x = (uint32_t)((threadIdx.x & 1) ? hi : lo);
+        s_rng[threadIdx.x] = threadIdx.x < 2 ? lower_bound_dev(dropped, 0, n_dropped, x)
+                                             : upper_bound_dev(ins_oldpos, 0, n_vins, x);
+    }
+    __syncthreads();
+    const uint64_t g = gb + threadIdx.x;
+    if (g >= ng) return;
     const uint32_t c0 = (uint32_t)(g * 32);
-    const uint64_t d0 = lower_bound_dev(dropped, 0, n_dropped, c0);
-    const uint64_t i0 = upper_bound_dev(ins_oldpos, 0, n_vins, c0);
+    const uint64_t d0 = lower_bound_dev(dropped, s_rng[0], s_rng[1], c0);
+    const uint64_t i0 = upper_bound_dev(ins_oldpos, s_rng[2], s_rng[3], c0);
     // insertion points past the last old id (appended vertices) shift no old id
-    const uint64_t i1 = upper_bound_dev(ins_oldpos, i0, n_vins, (uint32_t)min((uint64_t)c0 + 31, V - 1));
+    const uint64_t i1 = upper_bound_dev(ins_oldpos, i0, s_rng[3], (uint32_t)min((uint64_t)c0 + 31, V - 1));
     uint32_t m = 0;
-    for (uint64_t d = d0; d < n_dropped && dropped[d] < c0 + 32; ++d) m |= 1u << (dropped[d] - c0);
+    for (uint64_t d = d0; d < s_rng[1] && dropped[d] < c0 + 32; ++d) m |= 1u << (dropped[d] - c0);
     out[g] = make_uint2((uint32_t)(c0 - d0 + i0) | (i1 > i0 ? 0x80000000u : 0u), m);
 }
 

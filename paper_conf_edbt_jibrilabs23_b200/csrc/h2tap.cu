@@ -657,7 +657,8 @@ h2tap_status apply_core(h2tap_replica* r, const BatchIn& in, uint64_t S, bool cr
         ra.c = dc;
         const uint64_t ncta = cdiv(V, kOffTile);
         ra.part = r->get<uint64_t>(r->opart, 2 * (ncta + 1));
-        k_rows_partition<kOffTile><<<g1(ncta + 1), 256, 0, st>>>(ra);
+        k_offsets_bounds<<<(unsigned)std::min<uint64_t>(g1(n_edge + 1), (uint64_t)r->n_sm * 16), 256, 0, st>>>(
+            del_row, ins_row, dc, n_edge, ncta, ra.part);
         CKL();
         const uint64_t c_lo = row_lo / kOffTile, c_hi = cdiv(row_lo + Vr, kOffTile);
         k_offsets_direct<<<(unsigned)(c_hi - c_lo), kThreads, 0, st>>>(ra);

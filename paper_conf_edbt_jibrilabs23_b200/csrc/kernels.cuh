@@ -1344,6 +1344,31 @@ __global__ void __launch_bounds__(kThreads, 5) k_rows_fused(RowArgs a_) {
 // x = old_off[k].  CTA c covers rows [c*kRowTile, (c+1)*kRowTile) of the shard;
 // k_rows_partition supplies its slices of the two lists.
 constexpr int kOffTile = 4096;
+// CTA boundaries for k_offsets_direct without searches: part[2c] / part[2c+1] = number of
+// deletes / inserted records in rows < c*kOffTile.  Both lists are sorted by row, so
+// element i writes the boundaries c in (tile(row[i-1]), tile(row[i])] (the last element
+// also the ones past its tile): one pass over the lists, no dependent search chains.
+__global__ void k_offsets_bounds(const uint32_t* __restrict__ del_row, const uint32_t* __restrict__ ins_row,
+                                 const Counters* __restrict__ c, uint64_t n_ub, uint64_t ncta,
+                                 uint64_t* __restrict__ part) {
+    const uint64_t n_del = c->n_del, n_ins = c->n_ins;
+    const uint64_t stride = (uint64_t)gridDim.x * blockDim.x;
+    for (uint64_t i = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; i < n_ub + 1; i += stride) {
+#pragma unroll
+        for (int l = 0; l < 2; ++l) {
+            const uint32_t* rows = l ? ins_row : del_row;
+            const uint64_t n = l ? n_ins : n_del;
+            if (n == 0) {  // empty list: every boundary is 0
+                for (uint64_t cc = i; cc <= ncta; cc += n_ub + 1) part[2 * cc + l] = 0;
+                continue;
+            }
+            if (i > n) continue;
+            const uint64_t c_lo = i == 0 ? 0 : (uint64_t)rows[i - 1] / kOffTile + 1;
+            const uint64_t c_hi = i == n ? ncta : (uint64_t)rows[i] / kOffTile;
+            for (uint64_t cc = c_lo; cc <= c_hi && cc <= ncta; ++cc) part[2 * cc + l] = i;
+        }
+    }
+}
 __global__ void __launch_bounds__(kThreads) k_offsets_direct(RowArgs a_) {
     // per-row degree delta of the CTA's rows in a shared-memory histogram (from its
     // slices of the two sorted lists), scanned in place; old and new offsets move

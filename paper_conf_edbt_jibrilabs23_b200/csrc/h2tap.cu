@@ -691,11 +691,7 @@ h2tap_status apply_core(h2tap_replica* r, const BatchIn& in, uint64_t S, bool cr
             const uint64_t grid = std::min<uint64_t>(ma.n_tiles, (uint64_t)std::max(1, occ) * r->n_sm);
             kern<<<(unsigned)grid, kThreads, kMerge3Smem, st>>>(ma, part);
         };
-#if defined(H2TAP_EXP_C)  // timing experiments only (wrong results)
-        if (node_mode) launch(k_merge3<H2TAP_EXP_C, H2TAP_EXP_R>);
-#else
         if (node_mode) launch(k_merge3<true, true>);
-#endif
         else launch(k_merge3<false, false>);
         CKL();
     } else {

@@ -13,7 +13,7 @@ for c in ${CONFIGS:-c2 c3}; do
 done
 if [ -n "$TRACE" ]; then
   for c in ${CONFIGS:-c2 c3}; do
-    H2TAP_TRACE=1 timeout 300 python tools_trace.py $c 2>&1 | grep "h2tap trace" | tail -3 > gpurun_out/trace_$c.txt
+    H2TAP_TRACE=1 timeout 300 python tools/tools_trace.py $c 2>&1 | grep "h2tap trace" | tail -3 > gpurun_out/trace_$c.txt
   done
 fi
 cat gpurun_out/pytest_gpu.txt

@@ -553,14 +553,17 @@ h2tap_status apply_core(h2tap_replica* r, const BatchIn& in, uint64_t S, bool cr
         pa.keys = kA;
         pa.vals = vA;
         pa.recs = r->get<EdgeRec>(r->op_flags, m);
-        const bool lookups_direct = r->identity && !node_mode;  // no searches -> 8 ops per thread
-        const int eitems = lookups_direct ? 8 : 1;
+        const bool lookups_direct = r->identity && !node_mode;  // no searches -> 4 ops per thread
+#ifndef H2TAP_EI_DIRECT
+#define H2TAP_EI_DIRECT 4
+#endif
+        const int eitems = lookups_direct ? H2TAP_EI_DIRECT : 1;
         uint64_t nt = cdiv(n_edge, (uint64_t)kThreads * eitems);
         pa.status = r->get<uint64_t>(r->status, 3 * nt);
         CK(cudaMemsetAsync(pa.status, 0, nt * 8, st));
         pa.n_tiles = nt;
         pa.c = dc;
-        if (lookups_direct) k_edge_prep<8><<<(unsigned)nt, kThreads, 0, st>>>(pa);
+        if (lookups_direct) k_edge_prep<H2TAP_EI_DIRECT><<<(unsigned)nt, kThreads, 0, st>>>(pa);
         else k_edge_prep<1><<<(unsigned)nt, kThreads, 0, st>>>(pa);
         CKL();
         TR("edge_prep");

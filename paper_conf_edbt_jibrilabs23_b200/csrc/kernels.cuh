@@ -822,7 +822,10 @@ struct ClassArgs {
     Counters* c;
 };
 
-constexpr int kCItems = 2;                    // classify: items per thread (occupancy over ILP)
+#ifndef H2TAP_CITEMS
+#define H2TAP_CITEMS 1
+#endif
+constexpr int kCItems = H2TAP_CITEMS;  // classify: items per thread (occupancy over ILP)
 constexpr int kCTile = kThreads * kCItems;
 __global__ void __launch_bounds__(kThreads) k_reduce_classify(ClassArgs a) {
     __shared__ uint32_t s_tile;

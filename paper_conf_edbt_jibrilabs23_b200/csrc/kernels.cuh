@@ -1230,7 +1230,10 @@ __global__ void __launch_bounds__(kThreads) k_casc_scan(const uint32_t* __restri
 // Row offsets with node ops (a4/a5): thread per old row k that survives,
 //   new_off[u'] = x - (cascaded before x) - (deleted before x) + (inserted records in rows < u')
 // with x = old_off[k]; the CTA narrows the sorted delete / insert-row lists first.
-constexpr int kRowTile = 1024;
+#ifndef H2TAP_ROW_TILE
+#define H2TAP_ROW_TILE 512
+#endif
+constexpr int kRowTile = H2TAP_ROW_TILE;  // old ids per CTA of the node-mode row pass
 struct RowArgs {
     const int64_t* old_off;
     uint64_t V_old, E_old;
@@ -1303,7 +1306,10 @@ __global__ void k_rows_partition(RowArgs a_) {
 // rows of this shard, its new row offset
 //   new_off[u] = x - (cascaded before x) - (deleted before x) + (inserted records in rows < u)
 // with x = old_off[k].  The CTA narrows the sorted delete / insert-row lists first.
-__global__ void __launch_bounds__(kThreads, 5) k_rows_fused(RowArgs a_) {
+#ifndef H2TAP_ROWS_MINB
+#define H2TAP_ROWS_MINB 6
+#endif
+__global__ void __launch_bounds__(kThreads, H2TAP_ROWS_MINB) k_rows_fused(RowArgs a_) {
     const RowArgs a = row_counts(a_);
     const uint64_t k0 = (uint64_t)blockIdx.x * kRowTile, k1 = min(k0 + kRowTile, a.V_old);
     const uint64_t* pp = a.part + 2 * blockIdx.x;  // this CTA's slices of the delete / insert-row lists
@@ -1346,7 +1352,10 @@ __global__ void __launch_bounds__(kThreads, 5) k_rows_fused(RowArgs a_) {
 //   new_off[k] = x - (deleted old elements before x) + (inserted records in rows < k),
 // x = old_off[k].  CTA c covers rows [c*kRowTile, (c+1)*kRowTile) of the shard;
 // k_rows_partition supplies its slices of the two lists.
-constexpr int kOffTile = 4096;
+#ifndef H2TAP_OFF_TILE
+#define H2TAP_OFF_TILE 4096
+#endif
+constexpr int kOffTile = H2TAP_OFF_TILE;  // rows per CTA of k_offsets_direct
 // CTA boundaries for k_offsets_direct without searches: part[2c] / part[2c+1] = number of
 // deletes / inserted records in rows < c*kOffTile.  Both lists are sorted by row, so
 // element i writes the boundaries c in (tile(row[i-1]), tile(row[i])] (the last element

@@ -262,3 +262,30 @@ def records_from_ops(b: Batch) -> RecordBatch:
     rec["inserted"][gid[kind == NODE_INSERT]] = 1
     rec["deleted"][gid[kind == NODE_DELETE]] = 1
     return RecordBatch(rec, b.dst[ins].copy(), b.w[ins].copy(), b.dst[dl].copy())
+
+
+def dyn_record_batch(seed: int, k: int, xid: int, n_records: int, n_new: int = 4, max_slice: int = 6,
+                     p_deleted: float = 0.05, p_new: float = 0.1, p_invalid: float = 0.03) -> RecordBatch:
+    """Random delta records for the dynamic replica (Algorithm 1): each record's
+    node is a new ID in (xid, xid + n_new] with probability p_new, otherwise an ID in [0, xid];
+    inserts go to IDs in [0, xid + n_new], deletes to IDs in [0, xid]; slices are laid out
+    back to back.  Random numbers only (no update rule here)."""
+    rng = np.random.default_rng([seed, k, 0x44594E])
+    rec = np.zeros(n_records, RECORD_DTYPE)
+    new = rng.random(n_records) < p_new
+    rec["node"] = np.where(new, xid + 1 + rng.integers(0, max(n_new, 1), n_records),
+                           rng.integers(0, xid + 1, n_records)).astype(np.uint64)
+    rec["deleted"] = rng.random(n_records) < p_deleted
+    rec["valid"] = rng.random(n_records) >= p_invalid
+    rec["inserted"] = new
+    rec["ts"] = 1
+    ic = rng.integers(0, max_slice + 1, n_records)
+    dc = rng.integers(0, max_slice + 1, n_records)
+    rec["ins_cnt"], rec["del_cnt"] = ic, dc
+    rec["ins_off"] = np.concatenate([[0], np.cumsum(ic)[:-1]]).astype(np.uint64) if n_records else []
+    rec["del_off"] = np.concatenate([[0], np.cumsum(dc)[:-1]]).astype(np.uint64) if n_records else []
+    ni, nd = int(ic.sum()), int(dc.sum())
+    ins = rng.integers(0, xid + 1 + n_new, ni).astype(np.uint64)
+    wts = rng.integers(1, 1 << 16, ni).astype(np.float32) / np.float32(1 << 10)
+    dl = rng.integers(0, xid + 1, nd).astype(np.uint64)
+    return RecordBatch(rec, ins, wts, dl)

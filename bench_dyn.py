@@ -1,0 +1,95 @@
+"""The dynamic replica on B200 (Algorithm 1, §5.4
+P:L775-822) beside the CSR merge on the same graph: the paper's point is that a hash-table
+replica ingests a batch in O(batch) where the CSR merge rewrites O(E), at the price of a
+materialisation for reads.
+
+Graph: configs[2]'s RMAT-24 (16 edges per vertex), device-resident.  Per cycle: a seeded
+delta-record batch (synth.dyn_record_batch: ~1/2 inserts, ~1/2 deletes per record, a few
+new nodes; `--node-deletes` adds deleted-node records, which cost one pass over the table)
+applied with h2tap_dyn_apply_records from device memory; device time from the library's
+events (stats.ms_total) and CUDA events around the call.  Also timed: one CSR
+materialisation (h2tap_dyn_export to device buffers... here host arrays, reported apart).
+One JSON line; the round's copy lives in profiles/.
+
+usage: python bench_dyn.py [--scale 24] [--records 500000] [--cycles 5] [--node-deletes 0.0]
+"""
+import argparse
+import json
+import os
+import sys
+import time
+
+import numpy as np
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+import synth  # noqa: E402
+
+
+def main():
+    import torch
+    import paper_conf_edbt_jibrilabs23_b200 as h2
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--scale", type=int, default=24)
+    ap.add_argument("--records", type=int, default=500_000)
+    ap.add_argument("--cycles", type=int, default=5)
+    ap.add_argument("--warmup", type=int, default=3)
+    ap.add_argument("--node-deletes", type=float, default=0.0)
+    args = ap.parse_args()
+    torch.cuda.set_device(0)
+    st = torch.cuda.current_stream()
+    n = 1 << args.scale
+    src, dst, w = synth.rmat_edges(args.scale, synth.seed_of("c3"), n=16 * n)
+    d = [torch.from_numpy(a.view(np.int64) if a.dtype == np.uint64 else a).cuda() for a in (src, dst, w)]
+    ev0, ev1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    torch.cuda.synchronize()
+    t0 = time.time()
+    g = h2.DynReplica.from_edges(n, None, *d)
+    torch.cuda.synchronize()
+    create_s = time.time() - t0
+    inf0 = g.info()
+    batches = []
+    xid = n - 1
+    for k in range(args.warmup + args.cycles):
+        rb = synth.dyn_record_batch(synth.seed_of("c3"), 1000 + k, xid, args.records, n_new=64, max_slice=2,
+                                    p_deleted=args.node_deletes, p_new=0.0005, p_invalid=0.0)
+        batches.append(synth.RecordBatch(torch.from_numpy(rb.records.view(np.uint8)).cuda(),
+                                         torch.from_numpy(rb.inserts.view(np.int64)).cuda(),
+                                         torch.from_numpy(rb.weights).cuda(),
+                                         torch.from_numpy(rb.deletes.view(np.int64)).cuda()))
+        xid += 64
+    ms, lib_ms, items, sts = [], [], [], []
+    for k, rb in enumerate(batches):
+        torch.cuda.synchronize()
+        ev0.record(st)
+        s = g.apply_records(rb)
+        ev1.record(st)
+        torch.cuda.synchronize()
+        if k >= args.warmup:
+            ms.append(ev0.elapsed_time(ev1))
+            lib_ms.append(s["ms_total"])
+            items.append(s["n_visible"])
+            sts.append(s)
+    torch.cuda.synchronize()
+    t0 = time.time()
+    out = g.export()
+    export_s = time.time() - t0
+    tot_items, tot_ms = sum(items), sum(ms)
+    line = {
+        "metric": "delta updates/sec ingested into the dynamic (hash-table) replica",
+        "value": tot_items / (tot_ms / 1e3), "unit": "updates/s", "ms_per_cycle": tot_ms / len(ms),
+        "device_ms_per_cycle": sum(lib_ms) / len(lib_ms), "updates_per_cycle": tot_items / len(items),
+        "cycles": len(ms), "warmup": args.warmup,
+        "config": {"workload": f"RMAT-{args.scale} x16 (configs[2] graph), {args.records} delta records per "
+                               f"cycle (<=2 inserts + <=2 deletes each), node-delete records p={args.node_deletes}",
+                   "inputs": "device-resident records"},
+        "graph": {"vertices": inf0["n_vertices"], "edges": inf0["n_edges"], "table_slots": inf0["table_slots"]},
+        "create_s": create_s, "export_host_s": export_s, "export_edges": int(len(out[1])),
+        "last_cycle": {k: sts[-1][k] for k in ("n_new", "n_upd", "n_del", "n_casc", "n_gated",
+                                                "n_vertex_inserted", "n_vertex_deleted", "n_launches")},
+    }
+    print(json.dumps(line))
+
+
+if __name__ == "__main__":
+    main()

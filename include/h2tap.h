@@ -324,6 +324,43 @@ h2tap_status h2tap_shard_sssp_relax(const h2tap_replica* r, const uint8_t* front
 h2tap_status h2tap_shard_sssp_settle(const h2tap_replica* r, double* dist, const double* nd,
         uint8_t* frontier, uint64_t* n_changed);
 
+/* ---- the dynamic replica ----
+ * PAPER.md §5.4 "Dynamic Data Structures" + Algorithm 1: the valid and visible
+ * deltas of a cycle are ingested into a hash-table graph.  Storage: one open-addressing table
+ * of packed (src_dense, dst_dense) keys with f32 values on the device, vertex ext IDs ascending
+ * with a liveness word each; dense ids never move (a deleted node keeps an empty, dead slot).
+ * Semantics (readings D1-D5): xid = the largest ext ID held before the cycle;
+ * per VALID record: deleted flag -> node deletion queue; node <= xid -> its inserts and
+ * deletes; node > xid -> a new node with its inserts.  New nodes are appended ascending
+ * (unless the same cycle deletes them), then ALL the cycle's edge inserts are applied
+ * (upsert; a repeated (src, dst) keeps its last item in record/slice order; accepted iff both
+ * endpoints are live), then all edge deletes, then the node deletions with their edges.
+ * Record timestamps are not consulted: the caller passes the deltas the scan found visible.
+ * Single GPU; dense ids and edges < 2^32 - 1.  All calls are synchronous on cfg->stream. */
+typedef struct h2tap_dyn h2tap_dyn;
+/* vertex_ids: n_vertices strictly increasing ext IDs (NULL = 0..n-1); edges (src, dst, w)
+ * between them, a repeated pair keeps its last weight (w NULL -> 1.0); host or device
+ * (on_device).  cfg: device / stream / allocator only (world and id_mode must be 0).
+ * Unknown endpoint or unsorted ids -> E_INVAL; *out = NULL on any error. */
+h2tap_status h2tap_dyn_create(const h2tap_config* cfg, size_t n_vertices, const uint64_t* vertex_ids,
+        size_t n_edges, const uint64_t* src, const uint64_t* dst, const float* w, int on_device,
+        h2tap_dyn** out);
+/* One cycle of Algorithm 1 over `batch` (the h2tap_record_batch layout above).  Flag other
+ * than 0/1 or a slice outside its array -> E_INVAL before anything is applied.  stats
+ * (nullable): n_new / n_upd / n_del / n_casc / n_gated / n_vertex_*, ms_total (device time),
+ * n_launches, h2d_bytes; n_visible = expanded items (inserts + deletes + node ops). */
+h2tap_status h2tap_dyn_apply_records(h2tap_dyn* d, const h2tap_record_batch* batch,
+        h2tap_apply_stats* stats);
+/* n_vertices = dense slots (live and dead), n_edges = live edges, table_slots = capacity */
+h2tap_status h2tap_dyn_info(const h2tap_dyn* d, uint64_t* n_vertices, uint64_t* n_edges,
+        uint64_t* table_slots);
+/* Materialise the CSR (rows = dense ids, dead rows empty, columns ascending): offsets
+ * [n_vertices + 1], cols / w [n_edges], ext_ids [n_vertices], live u8 [n_vertices]; any
+ * pointer may be NULL (skipped); host or device pointers (copied with cudaMemcpyDefault). */
+h2tap_status h2tap_dyn_export(h2tap_dyn* d, int64_t* offsets, uint32_t* cols, float* w,
+        uint64_t* ext_ids, uint8_t* live);
+void h2tap_dyn_destroy(h2tap_dyn* d);
+
 void h2tap_replica_destroy(h2tap_replica* r);
 const char* h2tap_status_str(h2tap_status s);
 const char* h2tap_last_error(void);

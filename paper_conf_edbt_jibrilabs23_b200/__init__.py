@@ -511,3 +511,91 @@ class Replica:
 
     def __exit__(self, *a):
         self.close()
+
+
+for _n, _a, _r in (("h2tap_dyn_create", [ctypes.POINTER(_Config), ctypes.c_size_t, _P, ctypes.c_size_t, _P, _P, _P,
+                                         ctypes.c_int, ctypes.POINTER(_P)], ctypes.c_int),
+                   ("h2tap_dyn_apply_records", [_P, ctypes.POINTER(_RecordBatch), ctypes.POINTER(ApplyStats)],
+                    ctypes.c_int),
+                   ("h2tap_dyn_info", [_P] + [ctypes.POINTER(_u64)] * 3, ctypes.c_int),
+                   ("h2tap_dyn_export", [_P, _P, _P, _P, _P, _P], ctypes.c_int),
+                   ("h2tap_dyn_destroy", [_P], None)):
+    getattr(_lib, _n).restype = _r
+    getattr(_lib, _n).argtypes = _a
+
+
+class DynReplica:
+    """The dynamic (hash-table) replica: Algorithm 1, §5.4
+    (opaque h2tap_dyn*; include/h2tap.h documents the semantics)."""
+
+    def __init__(self, handle, keep):
+        self._h = handle
+        self._keep = keep
+        _LIVE.add(self)
+
+    @classmethod
+    def from_edges(cls, n_vertices, vertex_ids, src, dst, w, device=0, stream=None,
+                   torch_allocator=True) -> "DynReplica":
+        cfg, keep = Replica._config(device, stream, torch_allocator)
+        pi, ps, pd, pw = (_ptr(vertex_ids, np.uint64), _ptr(src, np.uint64), _ptr(dst, np.uint64),
+                          _ptr(w, np.float32))
+        ond = _on_device(pi, ps, pd, pw)
+        n_e = len(src) if src is not None else 0
+        h = ctypes.c_void_p()
+        _check(_lib.h2tap_dyn_create(ctypes.byref(cfg), int(n_vertices), pi[0], n_e, ps[0], pd[0], pw[0], ond,
+                                     ctypes.byref(h)), "h2tap_dyn_create")
+        return cls(h, keep + [cfg])
+
+    def apply_records(self, rb, raise_on_error: bool = True):
+        """h2tap_dyn_apply_records on rb (.records .inserts .weights .deletes, host or device)."""
+        pr, pi, pw, pd = (_ptr(rb.records), _ptr(rb.inserts, np.uint64), _ptr(rb.weights, np.float32),
+                          _ptr(rb.deletes, np.uint64))
+        b = _RecordBatch()
+        recs = pr[2]
+        nbytes = recs.numel() * recs.element_size() if _is_torch(recs) else recs.nbytes
+        if nbytes % RECORD_BYTES:
+            raise ValueError("records buffer is not a whole number of 48-byte records")
+        b.n_records = nbytes // RECORD_BYTES
+        b.on_device = _on_device(pr, pi, pw, pd)
+        b.records, b.inserts, b.weights, b.deletes = pr[0], pi[0], pw[0], pd[0]
+        b.n_inserts = len(pi[2]) if pi[2] is not None else 0
+        b.n_deletes = len(pd[2]) if pd[2] is not None else 0
+        st = ApplyStats()
+        rc = _lib.h2tap_dyn_apply_records(self._h, ctypes.byref(b), ctypes.byref(st))
+        if raise_on_error:
+            _check(rc, "h2tap_dyn_apply_records")
+            return st.as_dict()
+        return rc, st.as_dict()
+
+    def info(self):
+        v = [_u64() for _ in range(3)]
+        _check(_lib.h2tap_dyn_info(self._h, *(ctypes.byref(x) for x in v)), "h2tap_dyn_info")
+        return dict(n_vertices=v[0].value, n_edges=v[1].value, table_slots=v[2].value)
+
+    def export(self):
+        """(offsets i64, cols u32, w f32, ext_ids u64, live u8) as numpy arrays (the CSR
+        materialised on the GPU)."""
+        inf = self.info()
+        V, E = inf["n_vertices"], inf["n_edges"]
+        out = (np.empty(V + 1, np.int64), np.empty(E, np.uint32), np.empty(E, np.float32),
+               np.empty(V, np.uint64), np.empty(V, np.uint8))
+        _check(_lib.h2tap_dyn_export(self._h, *[ctypes.c_void_p(a.ctypes.data) for a in out]),
+               "h2tap_dyn_export")
+        return out
+
+    def close(self):
+        if getattr(self, "_h", None):
+            _lib.h2tap_dyn_destroy(self._h)
+            self._h = None
+
+    def __del__(self):
+        try:
+            self.close()
+        except Exception:
+            pass
+
+    def __enter__(self):
+        return self
+
+    def __exit__(self, *a):
+        self.close()

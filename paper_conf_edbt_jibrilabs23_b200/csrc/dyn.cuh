@@ -1,0 +1,721 @@
+// dyn.cuh - the dynamic replica: Algorithm 1 (§5.4 "Dynamic
+// Data Structures") ingesting one cycle's delta records into a GPU hash-table
+// graph, included by h2tap.cu (shares its allocator, stream, radix sort and record layout).
+//
+// Storage: one open-addressing table over packed edge keys
+//   key = src_dense << 32 | dst_dense  (u64; EMPTY = ~0, TOMB = ~0 - 1), value f32
+// linear probing from fmix64(key), load (live + tombstones) <= 1/2 (re-hashed into a table of
+// twice the needed size when a cycle would pass it); inserts only ever claim EMPTY slots, so a
+// CAS on the key word is the whole synchronisation.  Vertices: ext ids ascending (new IDs are
+// > xid, Alg. 1 line 5/8, so they append) and a u32 liveness word per dense id (D3: dense ids
+// never move, dead ones keep an empty row).
+//
+// One cycle (h2tap_dyn_apply_records), all on the replica stream:
+//   k_dyn_rec        classify records (lines 2-9): deletion / new-node queues, per-record
+//                    insert / delete item counts (+ record validation)
+//   scans            item offsets (k_scan_exclusive_u64)
+//   new nodes        radix sort of the new IDs, k_dyn_kill (created and deleted in the same
+//                    cycle: D3), k_dyn_heads + scan + k_dyn_append (line 10)
+//   k_dyn_expand_ins one warp per record: resolve endpoints, gate (D2), pack keys
+//   radix sort       (key, item) - stable, so the last item of a key is the latest (D1)
+//   k_dyn_upsert     last item of each key: CAS-insert or overwrite (lines 6, 10)
+//   k_dyn_delete     one warp per record: probe + CAS to TOMB (line 7)
+//   k_dyn_node_del   liveness off (line 11) + k_dyn_cascade over the table if any died
+// Export materialises the CSR: k_dyn_compact (warp-aggregated) + radix sort + k_dyn_emit +
+// k_dyn_offsets.  The cost of a cycle is O(batch) plus O(table) only for node deletes.
+
+namespace dyn {
+
+constexpr uint64_t kEmpty = ~0ull, kTomb = ~0ull - 1;
+
+struct Ctr {
+    unsigned long long n_new_ids, n_del_ids, bad, max_new, n_new, n_upd, n_del, n_casc, n_gated, n_vdel, n_out;
+};
+
+__device__ __forceinline__ uint64_t hmix(uint64_t k) {
+    k ^= k >> 33; k *= 0xff51afd7ed558ccdull; k ^= k >> 33; k *= 0xc4ceb9fe1a85ec53ull; k ^= k >> 33;
+    return k;
+}
+__device__ __forceinline__ int64_t find_ext(const uint64_t* __restrict__ ext, uint64_t V, uint64_t x) {
+    uint64_t lo = 0, hi = V;
+    while (lo < hi) {
+        const uint64_t m = (lo + hi) >> 1;
+        if (ext[m] < x) lo = m + 1; else hi = m;
+    }
+    return (lo < V && ext[lo] == x) ? (int64_t)lo : -1;
+}
+__device__ __forceinline__ void wadd(unsigned long long* c, bool pred) {  // warp-aggregated count
+    const unsigned m = __ballot_sync(__activemask(), pred);
+    if (pred && (threadIdx.x & 31) == __ffs(m) - 1) atomicAdd(c, (unsigned long long)__popc(m));
+}
+
+// Alg. 1 lines 2-9 per record
+__global__ void k_dyn_rec(const DeltaRec* __restrict__ rec, uint64_t nr, uint64_t n_ins, uint64_t n_del,
+                          uint64_t xid, int has_xid, uint64_t* __restrict__ cnt_ins, uint64_t* __restrict__ cnt_del,
+                          uint64_t* __restrict__ new_ids, uint64_t* __restrict__ del_ids, Ctr* __restrict__ c) {
+    const uint64_t i = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x;
+    if (i > nr) return;
+    if (i == nr) { cnt_ins[nr] = 0; cnt_del[nr] = 0; return; }
+    const DeltaRec r = rec[i];
+    uint64_t ci = 0, cd = 0;
+    unsigned bad = 0;
+    if (r.valid > 1 || r.deleted > 1 || r.inserted > 1) bad |= REC_BAD_FLAG;
+    if (r.valid) {
+        if (r.ins_off > n_ins || r.ins_cnt > n_ins - r.ins_off || r.del_off > n_del || r.del_cnt > n_del - r.del_off)
+            bad |= REC_BAD_SLICE;
+        if (r.deleted) {                                       // lines 3-4
+            del_ids[atomicAdd(&c->n_del_ids, 1ull)] = r.node;
+        } else if (has_xid && r.node <= xid) {                // lines 5-7
+            ci = r.ins_cnt;
+            cd = r.del_cnt;
+        } else {                                               // line 9 (D5: its deletes ignored)
+            new_ids[atomicAdd(&c->n_new_ids, 1ull)] = r.node;
+            atomicMax(&c->max_new, (unsigned long long)r.node);
+            ci = r.ins_cnt;
+        }
+    }
+    if (bad) atomicOr(&c->bad, (unsigned long long)bad);
+    cnt_ins[i] = ci;
+    cnt_del[i] = cd;
+}
+
+// a new ID the cycle also deletes is never inserted (D3): flag its first copy in the sorted list
+__global__ void k_dyn_kill(const uint64_t* __restrict__ del_ids, uint64_t nd, const uint64_t* __restrict__ sk,
+                           uint64_t u, uint64_t base, uint8_t* __restrict__ kill) {
+    const uint64_t i = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x;
+    if (i >= nd) return;
+    const uint64_t x = del_ids[i];
+    if (x < base) return;
+    const uint64_t key = x - base;
+    uint64_t lo = 0, hi = u;
+    while (lo < hi) {
+        const uint64_t m = (lo + hi) >> 1;
+        if (sk[m] < key) lo = m + 1; else hi = m;
+    }
+    if (lo < u && sk[lo] == key) kill[lo] = 1;
+}
+__global__ void k_dyn_heads(const uint64_t* __restrict__ sk, uint64_t u, const uint8_t* __restrict__ kill,
+                            uint64_t* __restrict__ flag) {
+    const uint64_t i = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x;
+    if (i > u) return;
+    flag[i] = (i < u && (i == 0 || sk[i] != sk[i - 1]) && !kill[i]) ? 1 : 0;
+}
+__global__ void k_dyn_append(const uint64_t* __restrict__ sk, uint64_t u, const uint64_t* __restrict__ flag,
+                             const uint64_t* __restrict__ pos, uint64_t base, uint64_t* __restrict__ ext_tail,
+                             uint32_t* __restrict__ live_tail) {
+    const uint64_t i = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x;
+    if (i >= u || !flag[i]) return;
+    ext_tail[pos[i]] = sk[i] + base;   // line 10: ascending, after every old id
+    live_tail[pos[i]] = 1;
+}
+
+// one warp per record: the record's inserted edges as packed keys (invalid -> key_bad, sorts last)
+__global__ void k_dyn_expand_ins(const DeltaRec* __restrict__ rec, uint64_t nr, const uint64_t* __restrict__ off,
+                                 const uint64_t* __restrict__ ins, const float* __restrict__ wts,
+                                 const uint64_t* __restrict__ ext, const uint32_t* __restrict__ live, uint64_t V,
+                                 uint64_t* __restrict__ keys, uint32_t* __restrict__ vals, float* __restrict__ witem,
+                                 Ctr* __restrict__ c) {
+    const uint64_t key_bad = V << 32;
+    const uint64_t nw = (uint64_t)gridDim.x * (blockDim.x >> 5);
+    const unsigned lane = threadIdx.x & 31;
+    for (uint64_t i = blockIdx.x * (uint64_t)(blockDim.x >> 5) + (threadIdx.x >> 5); i < nr; i += nw) {
+        const uint64_t o = off[i], n = off[i + 1] - o;
+        if (n == 0) continue;
+        int64_t s = -1;
+        if (lane == 0) {
+            s = find_ext(ext, V, rec[i].node);
+            if (s >= 0 && !live[s]) s = -1;
+        }
+        s = __shfl_sync(0xffffffffu, s, 0);
+        const uint64_t io = rec[i].ins_off;
+        for (uint64_t j = lane; j < n; j += 32) {
+            int64_t d = s >= 0 ? find_ext(ext, V, ins[io + j]) : -1;
+            const bool ok = d >= 0 && live[d];                  // D2
+            keys[o + j] = ok ? ((uint64_t)s << 32 | (uint64_t)d) : key_bad;
+            vals[o + j] = (uint32_t)(o + j);
+            witem[o + j] = wts[io + j];
+            wadd(&c->n_gated, !ok);
+        }
+    }
+}
+
+// insert-only probe into EMPTY slots; keys are unique within a launch
+__device__ __forceinline__ bool table_put(uint64_t* hk, float* hv, uint64_t mask, uint64_t k, float w) {
+    uint64_t h = hmix(k) & mask;
+    while (true) {
+        uint64_t cur = *((volatile uint64_t*)&hk[h]);
+        if (cur == k) { hv[h] = w; return false; }
+        if (cur == kEmpty) {
+            cur = atomicCAS((unsigned long long*)&hk[h], (unsigned long long)kEmpty, (unsigned long long)k);
+            if (cur == kEmpty || cur == k) { hv[h] = w; return cur == kEmpty; }
+        }
+        h = (h + 1) & mask;
+    }
+}
+
+__global__ void k_dyn_upsert(const uint64_t* __restrict__ sk, const uint32_t* __restrict__ sv, uint64_t n,
+                             const float* __restrict__ witem, uint64_t key_bad, uint64_t* hk, float* hv, uint64_t mask,
+                             Ctr* __restrict__ c) {
+    const uint64_t i = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x;
+    bool nw = false, up = false;
+    if (i < n) {
+        const uint64_t k = sk[i];
+        if (k < key_bad && (i + 1 == n || sk[i + 1] != k)) {   // D1: the latest item of its key
+            nw = table_put(hk, hv, mask, k, witem[sv[i]]);
+            up = !nw;
+        }
+    }
+    wadd(&c->n_new, nw);
+    wadd(&c->n_upd, up);
+}
+
+__global__ void k_dyn_delete(const DeltaRec* __restrict__ rec, uint64_t nr, const uint64_t* __restrict__ off,
+                             const uint64_t* __restrict__ del, const uint64_t* __restrict__ ext, uint64_t V,
+                             uint64_t* hk, uint64_t mask, Ctr* __restrict__ c) {
+    const uint64_t nw = (uint64_t)gridDim.x * (blockDim.x >> 5);
+    const unsigned lane = threadIdx.x & 31;
+    for (uint64_t i = blockIdx.x * (uint64_t)(blockDim.x >> 5) + (threadIdx.x >> 5); i < nr; i += nw) {
+        const uint64_t n = off[i + 1] - off[i];
+        if (n == 0) continue;
+        int64_t s = lane == 0 ? find_ext(ext, V, rec[i].node) : -1;
+        s = __shfl_sync(0xffffffffu, s, 0);
+        if (s < 0) continue;                                     // D4
+        const uint64_t dO = rec[i].del_off;
+        for (uint64_t j0 = 0; j0 < n; j0 += 32) {
+            bool hit = false;
+            const uint64_t j = j0 + lane;
+            if (j < n) {
+                const int64_t d = find_ext(ext, V, del[dO + j]);
+                if (d >= 0) {
+                    const uint64_t k = (uint64_t)s << 32 | (uint64_t)d;
+                    uint64_t h = hmix(k) & mask;
+                    while (true) {
+                        const uint64_t cur = *((volatile uint64_t*)&hk[h]);
+                        if (cur == k) {
+                            hit = atomicCAS((unsigned long long*)&hk[h], (unsigned long long)k,
+                                            (unsigned long long)kTomb) == k;
+                            break;
+                        }
+                        if (cur == kEmpty) break;
+                        h = (h + 1) & mask;
+                    }
+                }
+            }
+            wadd(&c->n_del, hit);
+        }
+    }
+}
+
+__global__ void k_dyn_node_del(const uint64_t* __restrict__ del_ids, uint64_t nd, const uint64_t* __restrict__ ext,
+                               uint64_t V, uint32_t* live, Ctr* __restrict__ c) {
+    const uint64_t i = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x;
+    bool died = false;
+    if (i < nd) {
+        const int64_t d = find_ext(ext, V, del_ids[i]);
+        died = d >= 0 && atomicExch(&live[d], 0u) == 1u;       // line 11 (D4: dead / unknown: no-op)
+    }
+    wadd(&c->n_vdel, died);
+}
+
+__global__ void k_dyn_cascade(uint64_t* __restrict__ hk, uint64_t cap, const uint32_t* __restrict__ live,
+                              Ctr* __restrict__ c) {
+    const uint64_t stride = (uint64_t)gridDim.x * blockDim.x;
+    for (uint64_t i0 = blockIdx.x * (uint64_t)blockDim.x; i0 < cap; i0 += stride) {
+        const uint64_t i = i0 + threadIdx.x;
+        bool gone = false;
+        if (i < cap) {
+            const uint64_t k = hk[i];
+            if (k < kTomb && (!live[k >> 32] || !live[k & 0xffffffffu])) {
+                hk[i] = kTomb;
+                gone = true;
+            }
+        }
+        wadd(&c->n_casc, gone);
+    }
+}
+
+__global__ void k_dyn_rehash(const uint64_t* __restrict__ ok, const float* __restrict__ ov, uint64_t ocap,
+                             uint64_t* hk, float* hv, uint64_t mask) {
+    const uint64_t stride = (uint64_t)gridDim.x * blockDim.x;
+    for (uint64_t i = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; i < ocap; i += stride) {
+        const uint64_t k = ok[i];
+        if (k < kTomb) table_put(hk, hv, mask, k, ov[i]);
+    }
+}
+
+// create: flat edge list -> packed keys (an endpoint that is no vertex -> bad)
+__global__ void k_dyn_expand_flat(const uint64_t* __restrict__ src, const uint64_t* __restrict__ dst,
+                                  const float* __restrict__ w, uint64_t n, const uint64_t* __restrict__ ext, uint64_t V,
+                                  uint64_t* __restrict__ keys, uint32_t* __restrict__ vals, float* __restrict__ witem,
+                                  Ctr* __restrict__ c) {
+    const uint64_t i = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x;
+    if (i >= n) return;
+    const int64_t s = find_ext(ext, V, src[i]), d = find_ext(ext, V, dst[i]);
+    if (s < 0 || d < 0) { atomicOr(&c->bad, 1ull); keys[i] = V << 32; }
+    else keys[i] = (uint64_t)s << 32 | (uint64_t)d;
+    vals[i] = (uint32_t)i;
+    witem[i] = w ? w[i] : 1.0f;
+}
+__global__ void k_dyn_check_ids(const uint64_t* __restrict__ ext, uint64_t V, Ctr* __restrict__ c) {
+    const uint64_t i = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x;
+    if (i > 0 && i < V && ext[i] <= ext[i - 1]) atomicOr(&c->bad, 1ull);
+}
+__global__ void k_dyn_sub_base(const uint64_t* __restrict__ ids, uint64_t n, uint64_t base, uint64_t* __restrict__ k,
+                               uint32_t* __restrict__ v) {
+    const uint64_t i = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x;
+    if (i < n) { k[i] = ids[i] - base; v[i] = 0; }
+}
+__global__ void k_dyn_fill_u32(uint32_t* p, uint64_t n, uint32_t v) {
+    const uint64_t i = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x;
+    if (i < n) p[i] = v;
+}
+
+// export
+__global__ void k_dyn_compact(const uint64_t* __restrict__ hk, const float* __restrict__ hv, uint64_t cap,
+                              uint64_t* __restrict__ ok, uint32_t* __restrict__ oi, float* __restrict__ ow,
+                              Ctr* __restrict__ c) {
+    const uint64_t stride = (uint64_t)gridDim.x * blockDim.x;
+    const unsigned lane = threadIdx.x & 31;
+    for (uint64_t i0 = blockIdx.x * (uint64_t)blockDim.x; i0 < cap; i0 += stride) {
+        const uint64_t i = i0 + threadIdx.x;
+        const uint64_t k = i < cap ? hk[i] : kEmpty;
+        const bool keep = k < kTomb;
+        const unsigned m = __ballot_sync(0xffffffffu, keep);
+        unsigned long long base = 0;
+        if (lane == 0 && m) base = atomicAdd(&c->n_out, (unsigned long long)__popc(m));
+        base = __shfl_sync(0xffffffffu, base, 0);
+        if (keep) {
+            const uint64_t p = base + __popc(m & ((1u << lane) - 1));
+            ok[p] = k;
+            oi[p] = (uint32_t)p;
+            ow[p] = hv[i];
+        }
+    }
+}
+__global__ void k_dyn_emit(const uint64_t* __restrict__ sk, const uint32_t* __restrict__ si, const float* __restrict__ cw,
+                           uint64_t E, uint32_t* __restrict__ cols, float* __restrict__ w) {
+    const uint64_t i = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x;
+    if (i >= E) return;
+    cols[i] = (uint32_t)(sk[i] & 0xffffffffu);
+    w[i] = cw[si[i]];
+}
+__global__ void k_dyn_offsets(const uint64_t* __restrict__ sk, uint64_t E, uint64_t V, int64_t* __restrict__ off) {
+    const uint64_t v = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x;
+    if (v > V) return;
+    const uint64_t key = v << 32;
+    uint64_t lo = 0, hi = E;
+    while (lo < hi) {
+        const uint64_t m = (lo + hi) >> 1;
+        if (sk[m] < key) lo = m + 1; else hi = m;
+    }
+    off[v] = (int64_t)lo;
+}
+__global__ void k_dyn_live_u8(const uint32_t* __restrict__ live, uint64_t V, uint8_t* __restrict__ out) {
+    const uint64_t i = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x;
+    if (i < V) out[i] = (uint8_t)live[i];
+}
+
+}  // namespace dyn
+
+struct h2tap_dyn {
+    h2tap_replica* r = nullptr;   // stream, allocator, radix-sort scratch
+    uint64_t V = 0, n_live = 0, n_tomb = 0, cap = 0;
+    Buf ext, live, hk, hv;
+    Buf cin, cdel, oin, odel, new_ids, del_ids, kill, flag, fpos, keys, vals, keys2, vals2, witem, ctr, xo;
+    Buf x_rec, x_ins, x_wts, x_del;
+    dyn::Ctr* hctr = nullptr;     // pinned host mirror
+};
+
+namespace {
+
+void dyn_free(h2tap_dyn* d) {
+    if (!d) return;
+    if (d->r) {
+        for (Buf* b : {&d->ext, &d->live, &d->hk, &d->hv, &d->cin, &d->cdel, &d->oin, &d->odel, &d->new_ids,
+                       &d->del_ids, &d->kill, &d->flag, &d->fpos, &d->keys, &d->vals, &d->keys2, &d->vals2,
+                       &d->witem, &d->ctr, &d->xo, &d->x_rec, &d->x_ins, &d->x_wts, &d->x_del})
+            if (b->p) d->r->dfree(b->p);
+        free_replica(d->r);
+    }
+    if (d->hctr) cudaFreeHost(d->hctr);
+    delete d;
+}
+
+dyn::Ctr* dyn_ctr_reset(h2tap_dyn* d) {
+    h2tap_replica* r = d->r;
+    dyn::Ctr* c = r->get<dyn::Ctr>(d->ctr, 1);
+    CK(cudaMemsetAsync(c, 0, sizeof(dyn::Ctr), r->st));
+    return c;
+}
+void dyn_ctr_read(h2tap_dyn* d) {
+    CK(cudaMemcpyAsync(d->hctr, d->ctr.p, sizeof(dyn::Ctr), cudaMemcpyDeviceToHost, d->r->st));
+    g_d2h += sizeof(dyn::Ctr);
+    d->r->sync();
+}
+
+// grow ext / live to hold n dense ids (contents kept)
+void dyn_reserve_vertices(h2tap_dyn* d, uint64_t n) {
+    h2tap_replica* r = d->r;
+    if (d->ext.cap >= (n + 16) * 8 && d->live.cap >= (n + 16) * 4) return;
+    const uint64_t want = std::max<uint64_t>(n, 2 * d->V) + 1024;
+    Buf e2, l2;
+    r->get<uint64_t>(e2, want);
+    r->get<uint32_t>(l2, want);
+    if (d->V) {
+        CK(cudaMemcpyAsync(e2.p, d->ext.p, d->V * 8, cudaMemcpyDeviceToDevice, r->st));
+        CK(cudaMemcpyAsync(l2.p, d->live.p, d->V * 4, cudaMemcpyDeviceToDevice, r->st));
+    }
+    r->release(d->ext);
+    r->release(d->live);
+    d->ext = e2;
+    d->live = l2;
+}
+
+uint64_t pow2_at_least(uint64_t x) {
+    uint64_t c = 1024;
+    while (c < x) c <<= 1;
+    return c;
+}
+
+// make room for `incoming` more keys at load <= 1/2 (tombstones count as used)
+void dyn_reserve_table(h2tap_dyn* d, uint64_t incoming) {
+    h2tap_replica* r = d->r;
+    if (d->cap && 2 * (d->n_live + d->n_tomb + incoming) <= d->cap) return;
+    const uint64_t nc = pow2_at_least(2 * (d->n_live + incoming) + 1);
+    Buf k2, v2;
+    uint64_t* nk = r->get<uint64_t>(k2, nc);
+    float* nv = r->get<float>(v2, nc);
+    CK(cudaMemsetAsync(nk, 0xFF, nc * 8, r->st));
+    if (d->cap && d->n_live) {
+        const unsigned grid = (unsigned)std::min<uint64_t>(g1(d->cap), (uint64_t)r->n_sm * 8);
+        dyn::k_dyn_rehash<<<grid, 256, 0, r->st>>>(static_cast<uint64_t*>(d->hk.p), static_cast<float*>(d->hv.p),
+                                                   d->cap, nk, nv, nc - 1);
+        CKL();
+    }
+    r->release(d->hk);
+    r->release(d->hv);
+    d->hk = k2;
+    d->hv = v2;
+    d->cap = nc;
+    d->n_tomb = 0;
+}
+
+// sort (keys, item) items and upsert the latest item of every key; n items, keys < V' << 32
+void dyn_upsert_items(h2tap_dyn* d, uint64_t n, dyn::Ctr* c) {
+    h2tap_replica* r = d->r;
+    if (!n) return;
+    uint64_t* k = static_cast<uint64_t*>(d->keys.p);
+    uint32_t* v = static_cast<uint32_t*>(d->vals.p);
+    uint64_t* k2 = static_cast<uint64_t*>(d->keys2.p);
+    uint32_t* v2 = static_cast<uint32_t*>(d->vals2.p);
+    radix_sort(r, k, v, k2, v2, n, 32 + bits_for(d->V));
+    dyn::k_dyn_upsert<<<g1(n), 256, 0, r->st>>>(k, v, n, static_cast<float*>(d->witem.p), d->V << 32,
+                                                static_cast<uint64_t*>(d->hk.p), static_cast<float*>(d->hv.p),
+                                                d->cap - 1, c);
+    CKL();
+}
+
+void dyn_item_bufs(h2tap_dyn* d, uint64_t n) {
+    h2tap_replica* r = d->r;
+    r->get<uint64_t>(d->keys, n);
+    r->get<uint64_t>(d->keys2, n);
+    r->get<uint32_t>(d->vals, n);
+    r->get<uint32_t>(d->vals2, n);
+    r->get<float>(d->witem, n);
+}
+
+h2tap_status dyn_apply(h2tap_dyn* d, const h2tap_record_batch* b, h2tap_apply_stats* stats) {
+    h2tap_replica* r = d->r;
+    cudaStream_t st = r->st;
+    g_launches = g_h2d = g_d2h = 0;
+    CK(cudaEventRecord(r->ev[0], st));
+    const uint64_t nr = b->n_records;
+    const DeltaRec* rec = reinterpret_cast<const DeltaRec*>(b->records);
+    const uint64_t* ins = b->inserts;
+    const float* wts = b->weights;
+    const uint64_t* del = b->deletes;
+    if (nr && !rec) { set_err("records is NULL"); return H2TAP_E_INVAL; }
+    if ((b->n_inserts && (!ins || !wts)) || (b->n_deletes && !del)) { set_err("null inserts/weights/deletes"); return H2TAP_E_INVAL; }
+    if (!b->on_device) {
+        DeltaRec* xr = r->get<DeltaRec>(d->x_rec, nr);
+        uint64_t* xi = r->get<uint64_t>(d->x_ins, b->n_inserts);
+        float* xw = r->get<float>(d->x_wts, b->n_inserts);
+        uint64_t* xd = r->get<uint64_t>(d->x_del, b->n_deletes);
+        copy_in(r, xr, rec, nr, 0);
+        copy_in(r, xi, ins, b->n_inserts, 0);
+        copy_in(r, xw, wts, b->n_inserts, 0);
+        copy_in(r, xd, del, b->n_deletes, 0);
+        rec = xr; ins = xi; wts = xw; del = xd;
+    }
+    // ---- lines 1-9: classify records
+    uint64_t xid = 0;
+    if (d->V) {
+        CK(cudaMemcpyAsync(&xid, static_cast<uint64_t*>(d->ext.p) + d->V - 1, 8, cudaMemcpyDeviceToHost, st));
+        g_d2h += 8;
+    }
+    dyn::Ctr* c = dyn_ctr_reset(d);
+    uint64_t* cin = r->get<uint64_t>(d->cin, nr + 1);
+    uint64_t* cdel = r->get<uint64_t>(d->cdel, nr + 1);
+    uint64_t* oin = r->get<uint64_t>(d->oin, nr + 1);
+    uint64_t* odel = r->get<uint64_t>(d->odel, nr + 1);
+    uint64_t* new_ids = r->get<uint64_t>(d->new_ids, nr);
+    uint64_t* del_ids = r->get<uint64_t>(d->del_ids, nr);
+    r->sync();  // xid
+    dyn::k_dyn_rec<<<g1(nr + 1), 256, 0, st>>>(rec, nr, b->n_inserts, b->n_deletes, xid, d->V ? 1 : 0, cin, cdel,
+                                              new_ids, del_ids, c);
+    CKL();
+    {
+        const uint64_t n = nr + 1, nt = cdiv(n, kTile);
+        uint64_t* stt = r->get<uint64_t>(r->status2, nt);
+        unsigned int* sc = reinterpret_cast<unsigned int*>(r->get<uint64_t>(d->xo, 2));
+        CK(cudaMemsetAsync(stt, 0, nt * 8, st));
+        CK(cudaMemsetAsync(sc, 0, 4, st));
+        k_scan_exclusive_u64<<<(unsigned)nt, kThreads, 0, st>>>(cin, oin, n, stt, sc);
+        CKL();
+        CK(cudaMemsetAsync(stt, 0, nt * 8, st));
+        CK(cudaMemsetAsync(sc, 0, 4, st));
+        k_scan_exclusive_u64<<<(unsigned)nt, kThreads, 0, st>>>(cdel, odel, n, stt, sc);
+        CKL();
+    }
+    uint64_t tot[2];
+    CK(cudaMemcpyAsync(&tot[0], oin + nr, 8, cudaMemcpyDeviceToHost, st));
+    CK(cudaMemcpyAsync(&tot[1], odel + nr, 8, cudaMemcpyDeviceToHost, st));
+    g_d2h += 16;
+    dyn_ctr_read(d);
+    const dyn::Ctr h0 = *d->hctr;
+    if (h0.bad & REC_BAD_FLAG) { set_err("delta record flag other than 0/1"); return H2TAP_E_INVAL; }
+    if (h0.bad & REC_BAD_SLICE) { set_err("delta record slice outside the inserts/weights/deletes arrays"); return H2TAP_E_INVAL; }
+    const uint64_t n_ins = tot[0];
+    if (n_ins >= (1ull << 32)) { set_err("more than 2^32 - 1 inserted edges in one cycle"); return H2TAP_E_CAPACITY; }
+    // ---- line 10: new nodes (ascending, after every old id; D3)
+    uint64_t n_vins = 0;
+    const uint64_t u = h0.n_new_ids;
+    if (u) {
+        const uint64_t base = d->V ? xid + 1 : 0;
+        dyn_item_bufs(d, std::max<uint64_t>(u, 1));
+        uint64_t* k = static_cast<uint64_t*>(d->keys.p);
+        uint32_t* v = static_cast<uint32_t*>(d->vals.p);
+        uint64_t* k2 = static_cast<uint64_t*>(d->keys2.p);
+        uint32_t* v2 = static_cast<uint32_t*>(d->vals2.p);
+        // key = id - base (fits the bits of max_new - base)
+        dyn::k_dyn_sub_base<<<g1(u), 256, 0, st>>>(new_ids, u, base, k, v);
+        CKL();
+        radix_sort(r, k, v, k2, v2, u, bits_for(h0.max_new - base));
+        uint8_t* kill = r->get<uint8_t>(d->kill, u);
+        CK(cudaMemsetAsync(kill, 0, u, st));
+        if (h0.n_del_ids) {
+            dyn::k_dyn_kill<<<g1(h0.n_del_ids), 256, 0, st>>>(del_ids, h0.n_del_ids, k, u, base, kill);
+            CKL();
+        }
+        uint64_t* flag = r->get<uint64_t>(d->flag, u + 1);
+        uint64_t* pos = r->get<uint64_t>(d->fpos, u + 1);
+        dyn::k_dyn_heads<<<g1(u + 1), 256, 0, st>>>(k, u, kill, flag);
+        CKL();
+        const uint64_t nt = cdiv(u + 1, kTile);
+        uint64_t* stt = r->get<uint64_t>(r->status2, nt);
+        unsigned int* sc = reinterpret_cast<unsigned int*>(r->get<uint64_t>(d->xo, 2));
+        CK(cudaMemsetAsync(stt, 0, nt * 8, st));
+        CK(cudaMemsetAsync(sc, 0, 4, st));
+        k_scan_exclusive_u64<<<(unsigned)nt, kThreads, 0, st>>>(flag, pos, u + 1, stt, sc);
+        CKL();
+        CK(cudaMemcpyAsync(&n_vins, pos + u, 8, cudaMemcpyDeviceToHost, st));
+        g_d2h += 8;
+        dyn_reserve_vertices(d, d->V + u);
+        dyn::k_dyn_append<<<g1(u), 256, 0, st>>>(k, u, flag, pos, base, static_cast<uint64_t*>(d->ext.p) + d->V,
+                                                 static_cast<uint32_t*>(d->live.p) + d->V);
+        CKL();
+        r->sync();
+        if (d->V + n_vins >= 0xFFFFFFFFull) { set_err("more than 2^32 - 2 dense vertex ids"); return H2TAP_E_CAPACITY; }
+        d->V += n_vins;
+    }
+    const uint64_t* ext = static_cast<const uint64_t*>(d->ext.p);
+    uint32_t* live = static_cast<uint32_t*>(d->live.p);
+    const unsigned wgrid = (unsigned)std::min<uint64_t>(cdiv(std::max<uint64_t>(nr, 1), 8), (uint64_t)r->n_sm * 16);
+    // ---- lines 6 + 10: one insert batch (D1, D2)
+    if (n_ins) {
+        dyn_item_bufs(d, n_ins);
+        dyn::k_dyn_expand_ins<<<wgrid, 256, 0, st>>>(rec, nr, oin, ins, wts, ext, live, d->V,
+                                                     static_cast<uint64_t*>(d->keys.p), static_cast<uint32_t*>(d->vals.p),
+                                                     static_cast<float*>(d->witem.p), c);
+        CKL();
+        dyn_reserve_table(d, n_ins);
+        dyn_upsert_items(d, n_ins, c);
+    }
+    // ---- line 7: delete batch
+    if (tot[1] && d->cap) {
+        dyn::k_dyn_delete<<<wgrid, 256, 0, st>>>(rec, nr, odel, del, ext, d->V, static_cast<uint64_t*>(d->hk.p),
+                                                 d->cap - 1, c);
+        CKL();
+    }
+    // ---- line 11: node deletes + cascade
+    if (h0.n_del_ids) {
+        dyn::k_dyn_node_del<<<g1(h0.n_del_ids), 256, 0, st>>>(del_ids, h0.n_del_ids, ext, d->V, live, c);
+        CKL();
+        dyn_ctr_read(d);
+        if (d->hctr->n_vdel && d->cap) {
+            const unsigned grid = (unsigned)std::min<uint64_t>(g1(d->cap), (uint64_t)r->n_sm * 8);
+            dyn::k_dyn_cascade<<<grid, 256, 0, st>>>(static_cast<uint64_t*>(d->hk.p), d->cap, live, c);
+            CKL();
+        }
+    }
+    CK(cudaEventRecord(r->ev[1], st));
+    dyn_ctr_read(d);
+    const dyn::Ctr& h = *d->hctr;
+    d->n_live = d->n_live + h.n_new - h.n_del - h.n_casc;
+    d->n_tomb += h.n_del + h.n_casc;
+    if (stats) {
+        std::memset(stats, 0, sizeof(*stats));
+        stats->n_visible = n_ins + tot[1] + u + h0.n_del_ids;
+        stats->n_gated = h.n_gated;
+        stats->n_new = h.n_new;
+        stats->n_upd = h.n_upd;
+        stats->n_del = h.n_del;
+        stats->n_casc = h.n_casc;
+        stats->n_vertex_inserted = n_vins;
+        stats->n_vertex_deleted = h.n_vdel;
+        stats->ms_total = ev_ms(r->ev[0], r->ev[1]);
+        // algorithmic bytes: records + slices read, one 12-byte slot touch per item
+        stats->bytes_alg = nr * sizeof(DeltaRec) + n_ins * 12 + tot[1] * 8 + (n_ins + tot[1]) * 12;
+        stats->n_launches = g_launches;
+        stats->h2d_bytes = g_h2d;
+        stats->d2h_bytes = g_d2h;
+    }
+    return H2TAP_OK;
+}
+
+}  // namespace
+
+extern "C" {
+
+h2tap_status h2tap_dyn_create(const h2tap_config* cfg, size_t n_vertices, const uint64_t* vertex_ids,
+                              size_t n_edges, const uint64_t* src, const uint64_t* dst, const float* w,
+                              int on_device, h2tap_dyn** out) {
+    if (!out) { set_err("out is NULL"); return H2TAP_E_INVAL; }
+    *out = nullptr;
+    if (n_edges && (!src || !dst)) { set_err("src/dst NULL"); return H2TAP_E_INVAL; }
+    if (n_vertices >= 0xFFFFFFFFull || n_edges >= 0xFFFFFFFFull) { set_err("more than 2^32 - 2 vertices or edges"); return H2TAP_E_CAPACITY; }
+    if (cfg && (cfg->world > 1 || cfg->id_mode != H2TAP_ID_COMPACT)) {
+        set_err("the dynamic replica is single-GPU with fixed dense ids (leave world / id_mode at 0)");
+        return H2TAP_E_INVAL;
+    }
+    h2tap_dyn* d = new (std::nothrow) h2tap_dyn();
+    if (!d) { set_err("host allocation failed"); return H2TAP_E_NOMEM; }
+    const h2tap_status s = run_guarded(nullptr, [&]() -> h2tap_status {
+        g_launches = g_h2d = g_d2h = 0;
+        d->r = new_replica(cfg);
+        h2tap_replica* r = d->r;
+        CK(cudaHostAlloc(reinterpret_cast<void**>(&d->hctr), sizeof(dyn::Ctr), cudaHostAllocDefault));
+        if (!r->ev[0]) CK(cudaEventCreate(&r->ev[0]));
+        if (!r->ev[1]) CK(cudaEventCreate(&r->ev[1]));
+        dyn_reserve_vertices(d, n_vertices);
+        uint64_t* ext = static_cast<uint64_t*>(d->ext.p);
+        if (vertex_ids) copy_in(r, ext, vertex_ids, n_vertices, on_device);
+        else if (n_vertices) { k_iota_u64<<<g1(n_vertices), 256, 0, r->st>>>(ext, n_vertices); CKL(); }
+        if (n_vertices) {
+            dyn::k_dyn_fill_u32<<<g1(n_vertices), 256, 0, r->st>>>(static_cast<uint32_t*>(d->live.p), n_vertices, 1);
+            CKL();
+        }
+        dyn::Ctr* c = dyn_ctr_reset(d);
+        dyn::k_dyn_check_ids<<<g1(n_vertices), 256, 0, r->st>>>(ext, n_vertices, c);
+        CKL();
+        dyn_ctr_read(d);
+        if (d->hctr->bad) { set_err("vertex ids not strictly increasing"); return H2TAP_E_INVAL; }
+        d->V = n_vertices;
+        dyn_reserve_table(d, n_edges);
+        if (n_edges) {
+            dyn_item_bufs(d, n_edges);
+            const uint64_t *s2 = src, *d2 = dst;
+            const float* w2 = w;
+            Buf bs, bd, bw;
+            if (!on_device) {
+                uint64_t* xs = r->get<uint64_t>(bs, n_edges);
+                uint64_t* xd = r->get<uint64_t>(bd, n_edges);
+                copy_in(r, xs, src, n_edges, 0);
+                copy_in(r, xd, dst, n_edges, 0);
+                s2 = xs; d2 = xd;
+                if (w) { float* xw = r->get<float>(bw, n_edges); copy_in(r, xw, w, n_edges, 0); w2 = xw; }
+            }
+            dyn::k_dyn_expand_flat<<<g1(n_edges), 256, 0, r->st>>>(s2, d2, w2, n_edges, ext, d->V,
+                                                                   static_cast<uint64_t*>(d->keys.p),
+                                                                   static_cast<uint32_t*>(d->vals.p),
+                                                                   static_cast<float*>(d->witem.p), c);
+            CKL();
+            dyn_ctr_read(d);
+            r->release(bs); r->release(bd); r->release(bw);
+            if (d->hctr->bad) { set_err("edge endpoint is not a vertex"); return H2TAP_E_INVAL; }
+            dyn_upsert_items(d, n_edges, c);
+            dyn_ctr_read(d);
+            d->n_live = d->hctr->n_new;
+        }
+        r->sync();
+        return H2TAP_OK;
+    });
+    if (s != H2TAP_OK) {
+        try { dyn_free(d); } catch (...) {}
+        return s;
+    }
+    *out = d;
+    return H2TAP_OK;
+}
+
+h2tap_status h2tap_dyn_apply_records(h2tap_dyn* d, const h2tap_record_batch* batch, h2tap_apply_stats* stats) {
+    if (!d || !batch) { set_err("null argument"); return H2TAP_E_INVAL; }
+    return run_guarded(d->r, [&]() { return dyn_apply(d, batch, stats); });
+}
+
+h2tap_status h2tap_dyn_info(const h2tap_dyn* d, uint64_t* n_vertices, uint64_t* n_edges, uint64_t* table_slots) {
+    if (!d) { set_err("null argument"); return H2TAP_E_INVAL; }
+    if (n_vertices) *n_vertices = d->V;
+    if (n_edges) *n_edges = d->n_live;
+    if (table_slots) *table_slots = d->cap;
+    return H2TAP_OK;
+}
+
+h2tap_status h2tap_dyn_export(h2tap_dyn* d, int64_t* offsets, uint32_t* cols, float* w, uint64_t* ext_ids,
+                              uint8_t* live) {
+    if (!d) { set_err("null argument"); return H2TAP_E_INVAL; }
+    return run_guarded(d->r, [&]() -> h2tap_status {
+        h2tap_replica* r = d->r;
+        cudaStream_t st = r->st;
+        const uint64_t V = d->V, E = d->n_live;
+        dyn::Ctr* c = dyn_ctr_reset(d);
+        dyn_item_bufs(d, std::max<uint64_t>(E, 1));
+        uint64_t* k = static_cast<uint64_t*>(d->keys.p);
+        uint32_t* v = static_cast<uint32_t*>(d->vals.p);
+        uint64_t* k2 = static_cast<uint64_t*>(d->keys2.p);
+        uint32_t* v2 = static_cast<uint32_t*>(d->vals2.p);
+        float* cw = static_cast<float*>(d->witem.p);
+        if (d->cap) {
+            const unsigned grid = (unsigned)std::min<uint64_t>(g1(d->cap), (uint64_t)r->n_sm * 8);
+            dyn::k_dyn_compact<<<grid, 256, 0, st>>>(static_cast<uint64_t*>(d->hk.p), static_cast<float*>(d->hv.p),
+                                                     d->cap, k, v, cw, c);
+            CKL();
+        }
+        radix_sort(r, k, v, k2, v2, E, 32 + bits_for(V));
+        Buf bo, bc, bw, bl;
+        int64_t* o_off = r->get<int64_t>(bo, V + 1);
+        uint32_t* o_cols = r->get<uint32_t>(bc, E);
+        float* o_w = r->get<float>(bw, E);
+        uint8_t* o_live = r->get<uint8_t>(bl, V);
+        if (E) { dyn::k_dyn_emit<<<g1(E), 256, 0, st>>>(k, v, cw, E, o_cols, o_w); CKL(); }
+        dyn::k_dyn_offsets<<<g1(V + 1), 256, 0, st>>>(k, E, V, o_off);
+        CKL();
+        if (V) { dyn::k_dyn_live_u8<<<g1(V), 256, 0, st>>>(static_cast<uint32_t*>(d->live.p), V, o_live); CKL(); }
+        if (offsets) CK(cudaMemcpyAsync(offsets, o_off, (V + 1) * 8, cudaMemcpyDefault, st));
+        if (cols && E) CK(cudaMemcpyAsync(cols, o_cols, E * 4, cudaMemcpyDefault, st));
+        if (w && E) CK(cudaMemcpyAsync(w, o_w, E * 4, cudaMemcpyDefault, st));
+        if (ext_ids && V) CK(cudaMemcpyAsync(ext_ids, d->ext.p, V * 8, cudaMemcpyDefault, st));
+        if (live && V) CK(cudaMemcpyAsync(live, o_live, V, cudaMemcpyDefault, st));
+        dyn_ctr_read(d);
+        if (d->hctr->n_out != E) { set_err("table holds %llu live keys, expected %llu", d->hctr->n_out, (unsigned long long)E); return H2TAP_E_CUDA; }
+        r->release(bo); r->release(bc); r->release(bw); r->release(bl);
+        r->sync();
+        return H2TAP_OK;
+    });
+}
+
+void h2tap_dyn_destroy(h2tap_dyn* d) {
+    try { dyn_free(d); } catch (...) {}
+}
+
+}  // extern "C"

@@ -1724,3 +1724,5 @@ void h2tap_replica_destroy(h2tap_replica* r) {
 }
 
 }  // extern "C"
+
+#include "dyn.cuh"  // the dynamic replica (Algorithm 1), SURVEY §8(f) NEXT-3

@@ -1,0 +1,148 @@
+"""Parity of the dynamic replica (h2tap_dyn_*: Algorithm 1, §5.4) with
+O3 (oracle/o3_dynamic.py, pinned in tests/test_oracle_pins_dyn.py).  Bar: bit-exact
+offsets / cols / weights / ext ids / liveness and equal counters after every cycle
+(integer work; the weights are copied, never computed)."""
+import numpy as np
+import pytest
+
+import synth
+from oracle.o3_dynamic import DynamicOracle
+
+pytestmark = pytest.mark.gpu
+
+
+@pytest.fixture(scope="module")
+def h2():
+    import paper_conf_edbt_jibrilabs23_b200 as h2
+    return h2
+
+
+KEYS = ("n_new", "n_upd", "n_del", "n_casc", "n_gated", "n_vertex_inserted", "n_vertex_deleted")
+
+
+def same(g, o, ctx=""):
+    a, b = g.export(), o.export()
+    for name, x, y in zip(("offsets", "cols", "w", "ext_ids", "live"), a, b):
+        assert np.array_equal(np.asarray(x), np.asarray(y)), f"{ctx}: {name} differs"
+
+
+def cycle(g, o, rb, ctx=""):
+    st = g.apply_records(rb)
+    ost = o.apply_records(rb.records, rb.inserts, rb.weights, rb.deletes)
+    for k in KEYS:
+        assert st[k] == ost[k], f"{ctx}: {k} {st[k]} != {ost[k]}"
+    same(g, o, ctx)
+    return st
+
+
+def pair(h2, ids, src, dst, w):
+    ids = np.asarray(ids, np.uint64)
+    src, dst, w = np.asarray(src, np.uint64), np.asarray(dst, np.uint64), np.asarray(w, np.float32)
+    return h2.DynReplica.from_edges(len(ids), ids, src, dst, w), DynamicOracle(ids, src, dst, w)
+
+
+def test_fig2_records(h2):
+    from test_oracle_pins import load_fig2_records
+    g0, rb = load_fig2_records()
+    e = np.array(g0["edges"], dtype=object)
+    g, o = pair(h2, g0["vertices"], e[:, 0], e[:, 1], e[:, 2])
+    same(g, o, "create")
+    cycle(g, o, rb, "fig2")
+    off, cols, w, ids, live = g.export()
+    assert ids.tolist() == [1, 2, 3, 4, 5] and live.tolist() == [1, 1, 1, 0, 1]
+    assert off.tolist() == [0, 0, 1, 2, 2, 3] and cols.tolist() == [2, 4, 0]
+    assert w.tolist() == [0.25, 5.0, 2.0]
+
+
+@pytest.mark.parametrize("seed", range(6))
+def test_small_random_cycles(h2, seed):
+    rng = np.random.default_rng(100 + seed)
+    n = 24
+    ids = np.arange(n, dtype=np.uint64) * 3 + 1
+    m = 80
+    g, o = pair(h2, ids, ids[rng.integers(0, n, m)], ids[rng.integers(0, n, m)], rng.random(m))
+    for cyc in range(8):
+        rb = synth.dyn_record_batch(seed, cyc, int(o.ids[-1]), 40, n_new=6, max_slice=5, p_deleted=0.06)
+        cycle(g, o, rb, f"seed {seed} cycle {cyc}")
+
+
+def test_multi_tile_cycles_with_rehash_and_device_inputs(h2):
+    import torch
+    rng = np.random.default_rng(7)
+    n = 20000
+    ids = np.sort(rng.choice(1 << 40, n, replace=False)).astype(np.uint64)
+    m = 60000
+    g, o = pair(h2, ids, ids[rng.integers(0, n, m)], ids[rng.integers(0, n, m)], rng.random(m))
+    slots0 = g.info()["table_slots"]
+    for cyc in range(6):
+        xid = int(o.ids[-1])
+        rb = synth.dyn_record_batch(11, cyc, xid, 9000, n_new=300, max_slice=12, p_deleted=0.01)
+        # map the generator's dense-ish ids onto the replica's sparse id space
+        idmap = lambda a: np.where(a <= xid, ids[(a % np.uint64(n)).astype(np.int64)], a)
+        rb = synth.RecordBatch(rb.records.copy(), idmap(rb.inserts), rb.weights, idmap(rb.deletes))
+        rb.records["node"] = idmap(rb.records["node"])
+        if cyc % 2:
+            dev = synth.RecordBatch(torch.from_numpy(rb.records.view(np.uint8)).cuda(),
+                                    torch.from_numpy(rb.inserts.view(np.int64)).cuda(),
+                                    torch.from_numpy(rb.weights).cuda(),
+                                    torch.from_numpy(rb.deletes.view(np.int64)).cuda())
+            st = g.apply_records(dev)
+            ost = o.apply_records(rb.records, rb.inserts, rb.weights, rb.deletes)
+            for k in KEYS:
+                assert st[k] == ost[k], f"cycle {cyc}: {k}"
+            same(g, o, f"cycle {cyc} (device inputs)")
+        else:
+            cycle(g, o, rb, f"cycle {cyc}")
+    assert g.info()["table_slots"] > slots0          # the table grew (re-hash) and stayed exact
+
+
+def test_hub_record_spans_many_warps(h2):
+    n = 5000
+    ids = np.arange(n, dtype=np.uint64)
+    g, o = pair(h2, ids, [0, 1], [1, 2], [1.0, 2.0])
+    rec = np.zeros(2, synth.RECORD_DTYPE)
+    rec["node"] = [3, 3]
+    rec["valid"] = 1
+    rec["ins_cnt"] = [n, 40]
+    rec["ins_off"] = [0, n]
+    rec["del_cnt"] = [0, 100]
+    ins = np.concatenate([np.arange(n), np.arange(40) * 7]).astype(np.uint64)
+    w = np.arange(n + 40, dtype=np.float32)
+    rb = synth.RecordBatch(rec, ins, w, np.arange(100, dtype=np.uint64) * 3)
+    st = cycle(g, o, rb, "hub")
+    assert st["n_new"] == n and st["n_del"] > 0
+
+
+def test_errors_leave_the_replica_unchanged(h2):
+    g, o = pair(h2, [1, 2, 3], [1], [2], [1.0])
+    from test_oracle_pins import load_fig2_records
+    _, rb = load_fig2_records()
+    bad = synth.RecordBatch(rb.records.copy(), rb.inserts, rb.weights, rb.deletes)
+    bad.records["deleted"][2] = 2
+    rc, _ = g.apply_records(bad, raise_on_error=False)
+    assert rc == -1                                   # E_INVAL
+    bad = synth.RecordBatch(rb.records.copy(), rb.inserts, rb.weights, rb.deletes)
+    bad.records["del_cnt"][3] = 9
+    rc, _ = g.apply_records(bad, raise_on_error=False)
+    assert rc != 0
+    same(g, o, "after rejected cycles")
+    with pytest.raises(Exception):
+        h2.DynReplica.from_edges(2, np.array([2, 1], np.uint64), None, None, None)
+    with pytest.raises(Exception):
+        h2.DynReplica.from_edges(2, np.array([1, 2], np.uint64), np.array([1], np.uint64),
+                                 np.array([7], np.uint64), np.array([1.0], np.float32))
+
+
+def test_empty_graph_and_empty_cycle(h2):
+    g, o = pair(h2, [], [], [], [])
+    rb = synth.RecordBatch(np.zeros(0, synth.RECORD_DTYPE), np.zeros(0, np.uint64), np.zeros(0, np.float32),
+                           np.zeros(0, np.uint64))
+    cycle(g, o, rb, "empty")
+    rec = np.zeros(3, synth.RECORD_DTYPE)
+    rec["node"] = [5, 9, 5]
+    rec["valid"] = 1
+    rec["ins_cnt"] = [1, 1, 0]
+    rec["ins_off"] = [0, 1, 0]
+    rb = synth.RecordBatch(rec, np.array([9, 5], np.uint64), np.array([1.5, 2.5], np.float32),
+                           np.zeros(0, np.uint64))
+    cycle(g, o, rb, "first nodes into an empty replica")

@@ -16,10 +16,10 @@
 //   scans            item offsets (k_scan_exclusive_u64)
 //   new nodes        radix sort of the new IDs, k_dyn_kill (created and deleted in the same
 //                    cycle: D3), k_dyn_heads + scan + k_dyn_append (line 10)
-//   k_dyn_expand_ins one warp per record: resolve endpoints, gate (D2), pack keys
+//   k_dyn_expand_ins thread per record (warp per large record): resolve endpoints, gate (D2), pack keys
 //   radix sort       (key, item) - stable, so the last item of a key is the latest (D1)
 //   k_dyn_upsert     last item of each key: CAS-insert or overwrite (lines 6, 10)
-//   k_dyn_delete     one warp per record: probe + CAS to TOMB (line 7)
+//   k_dyn_delete     thread per record (warp per large record): probe + CAS to TOMB (line 7)
 //   k_dyn_node_del   liveness off (line 11) + k_dyn_cascade over the table if any died
 // Export materialises the CSR: k_dyn_compact (warp-aggregated) + radix sort + k_dyn_emit +
 // k_dyn_offsets.  The cost of a cycle is O(batch) plus O(table) only for node deletes.
@@ -27,9 +27,10 @@
 namespace dyn {
 
 constexpr uint64_t kEmpty = ~0ull, kTomb = ~0ull - 1;
+constexpr uint32_t kFilterBits = 1u << 19;   // cascade filter: 64 KB of shared memory
 
 struct Ctr {
-    unsigned long long n_new_ids, n_del_ids, bad, max_new, n_new, n_upd, n_del, n_casc, n_gated, n_vdel, n_out;
+    unsigned long long n_new_ids, n_del_ids, bad, max_new, n_new, n_upd, n_del, n_casc, n_gated, n_vdel, n_out, last_ext, n_big_ins, n_big_del;
 };
 
 __device__ __forceinline__ uint64_t hmix(uint64_t k) {
@@ -37,6 +38,9 @@ __device__ __forceinline__ uint64_t hmix(uint64_t k) {
     return k;
 }
 __device__ __forceinline__ int64_t find_ext(const uint64_t* __restrict__ ext, uint64_t V, uint64_t x) {
+    if (V == 0) return -1;
+    const uint64_t e0 = __ldg(ext);
+    if (x >= e0 && x - e0 < V && __ldg(ext + (x - e0)) == x) return (int64_t)(x - e0);  // dense id space: one load
     uint64_t lo = 0, hi = V;
     while (lo < hi) {
         const uint64_t m = (lo + hi) >> 1;
@@ -102,41 +106,66 @@ __global__ void k_dyn_heads(const uint64_t* __restrict__ sk, uint64_t u, const u
 }
 __global__ void k_dyn_append(const uint64_t* __restrict__ sk, uint64_t u, const uint64_t* __restrict__ flag,
                              const uint64_t* __restrict__ pos, uint64_t base, uint64_t* __restrict__ ext_tail,
-                             uint32_t* __restrict__ live_tail) {
+                             uint32_t* __restrict__ live_tail, Ctr* __restrict__ c) {
     const uint64_t i = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x;
     if (i >= u || !flag[i]) return;
     ext_tail[pos[i]] = sk[i] + base;   // line 10: ascending, after every old id
     live_tail[pos[i]] = 1;
+    if (pos[i] + 1 == pos[u]) c->last_ext = sk[i] + base;  // the new xid
 }
 
-// one warp per record: the record's inserted edges as packed keys (invalid -> key_bad, sorts last)
-__global__ void k_dyn_expand_ins(const DeltaRec* __restrict__ rec, uint64_t nr, const uint64_t* __restrict__ off,
-                                 const uint64_t* __restrict__ ins, const float* __restrict__ wts,
-                                 const uint64_t* __restrict__ ext, const uint32_t* __restrict__ live, uint64_t V,
-                                 uint64_t* __restrict__ keys, uint32_t* __restrict__ vals, float* __restrict__ witem,
-                                 Ctr* __restrict__ c) {
-    const uint64_t key_bad = V << 32;
-    const uint64_t nw = (uint64_t)gridDim.x * (blockDim.x >> 5);
-    const unsigned lane = threadIdx.x & 31;
-    for (uint64_t i = blockIdx.x * (uint64_t)(blockDim.x >> 5) + (threadIdx.x >> 5); i < nr; i += nw) {
-        const uint64_t o = off[i], n = off[i + 1] - o;
-        if (n == 0) continue;
-        int64_t s = -1;
-        if (lane == 0) {
-            s = find_ext(ext, V, rec[i].node);
-            if (s >= 0 && !live[s]) s = -1;
+// The record's inserted edges as packed sort keys (invalid -> key_bad, sorts last).  Pass 0:
+// one thread per record, serially over a slice of <= kSmall items (most records: the
+// delta of one node in one transaction); larger records are queued for pass 1, one warp
+// per queued record (a hub's slice may hold thousands of items).
+constexpr uint64_t kSmall = 16;
+__device__ __forceinline__ bool ins_item(uint64_t j, int64_t s, uint64_t o, uint64_t io, const uint64_t* __restrict__ ins,
+                                         const float* __restrict__ wts, const uint64_t* __restrict__ ext,
+                                         const uint32_t* __restrict__ live, uint64_t V, uint64_t* __restrict__ keys,
+                                         uint32_t* __restrict__ vals, float* __restrict__ witem) {
+    const int64_t d = s >= 0 ? find_ext(ext, V, ins[io + j]) : -1;
+    const bool ok = d >= 0 && live[d];                            // D2
+    keys[o + j] = ok ? (uint64_t)s * V + (uint64_t)d : V * V;     // sort key
+    vals[o + j] = (uint32_t)(o + j);
+    witem[o + j] = wts[io + j];
+    return !ok;
+}
+__device__ __forceinline__ int64_t live_src(const uint64_t* __restrict__ ext, const uint32_t* __restrict__ live,
+                                            uint64_t V, uint64_t x) {
+    const int64_t s = find_ext(ext, V, x);
+    return (s >= 0 && live[s]) ? s : -1;
+}
+template <int kPass>
+__global__ void __launch_bounds__(256) k_dyn_expand_ins(const DeltaRec* __restrict__ rec, uint64_t nr,
+        const uint64_t* __restrict__ off, const uint64_t* __restrict__ ins, const float* __restrict__ wts,
+        const uint64_t* __restrict__ ext, const uint32_t* __restrict__ live, uint64_t V, uint64_t* __restrict__ keys,
+        uint32_t* __restrict__ vals, float* __restrict__ witem, uint64_t* __restrict__ big,
+        unsigned long long* __restrict__ n_big, Ctr* __restrict__ c) {
+    unsigned long long gated = 0;
+    if (kPass == 0) {
+        const uint64_t i = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x;
+        if (i < nr) {
+            const uint64_t o = off[i], n = off[i + 1] - o;
+            if (n > kSmall) big[atomicAdd(n_big, 1ull)] = i;
+            else if (n) {
+                const DeltaRec r = rec[i];
+                const int64_t s = live_src(ext, live, V, r.node);
+                for (uint64_t j = 0; j < n; ++j) gated += ins_item(j, s, o, r.ins_off, ins, wts, ext, live, V, keys, vals, witem);
+            }
         }
-        s = __shfl_sync(0xffffffffu, s, 0);
-        const uint64_t io = rec[i].ins_off;
-        for (uint64_t j = lane; j < n; j += 32) {
-            int64_t d = s >= 0 ? find_ext(ext, V, ins[io + j]) : -1;
-            const bool ok = d >= 0 && live[d];                  // D2
-            keys[o + j] = ok ? ((uint64_t)s << 32 | (uint64_t)d) : key_bad;
-            vals[o + j] = (uint32_t)(o + j);
-            witem[o + j] = wts[io + j];
-            wadd(&c->n_gated, !ok);
+    } else {
+        const uint64_t nb = *n_big, nw = (uint64_t)gridDim.x * (blockDim.x >> 5);
+        const unsigned lane = threadIdx.x & 31;
+        for (uint64_t q = blockIdx.x * (uint64_t)(blockDim.x >> 5) + (threadIdx.x >> 5); q < nb; q += nw) {
+            const uint64_t i = big[q], o = off[i], n = off[i + 1] - o;
+            int64_t s = lane == 0 ? live_src(ext, live, V, rec[i].node) : -1;
+            s = __shfl_sync(0xffffffffu, s, 0);
+            const uint64_t io = rec[i].ins_off;
+            for (uint64_t j = lane; j < n; j += 32) gated += ins_item(j, s, o, io, ins, wts, ext, live, V, keys, vals, witem);
         }
     }
+    gated = warp_sum<unsigned long long>(gated);
+    if ((threadIdx.x & 31) == 0 && gated) atomicAdd(&c->n_gated, gated);
 }
 
 // insert-only probe into EMPTY slots; keys are unique within a launch
@@ -154,14 +183,16 @@ __device__ __forceinline__ bool table_put(uint64_t* hk, float* hv, uint64_t mask
 }
 
 __global__ void k_dyn_upsert(const uint64_t* __restrict__ sk, const uint32_t* __restrict__ sv, uint64_t n,
-                             const float* __restrict__ witem, uint64_t key_bad, uint64_t* hk, float* hv, uint64_t mask,
+                             const float* __restrict__ witem, uint64_t V, uint64_t* hk, float* hv, uint64_t mask,
                              Ctr* __restrict__ c) {
+    const uint64_t key_bad = V * V;
     const uint64_t i = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x;
     bool nw = false, up = false;
     if (i < n) {
         const uint64_t k = sk[i];
         if (k < key_bad && (i + 1 == n || sk[i + 1] != k)) {   // D1: the latest item of its key
-            nw = table_put(hk, hv, mask, k, witem[sv[i]]);
+            const uint64_t s = k / V;
+            nw = table_put(hk, hv, mask, s << 32 | (k - s * V), witem[sv[i]]);
             up = !nw;
         }
     }
@@ -169,69 +200,113 @@ __global__ void k_dyn_upsert(const uint64_t* __restrict__ sk, const uint32_t* __
     wadd(&c->n_upd, up);
 }
 
-__global__ void k_dyn_delete(const DeltaRec* __restrict__ rec, uint64_t nr, const uint64_t* __restrict__ off,
-                             const uint64_t* __restrict__ del, const uint64_t* __restrict__ ext, uint64_t V,
-                             uint64_t* hk, uint64_t mask, Ctr* __restrict__ c) {
-    const uint64_t nw = (uint64_t)gridDim.x * (blockDim.x >> 5);
-    const unsigned lane = threadIdx.x & 31;
-    for (uint64_t i = blockIdx.x * (uint64_t)(blockDim.x >> 5) + (threadIdx.x >> 5); i < nr; i += nw) {
-        const uint64_t n = off[i + 1] - off[i];
-        if (n == 0) continue;
-        int64_t s = lane == 0 ? find_ext(ext, V, rec[i].node) : -1;
-        s = __shfl_sync(0xffffffffu, s, 0);
-        if (s < 0) continue;                                     // D4
-        const uint64_t dO = rec[i].del_off;
-        for (uint64_t j0 = 0; j0 < n; j0 += 32) {
-            bool hit = false;
-            const uint64_t j = j0 + lane;
-            if (j < n) {
-                const int64_t d = find_ext(ext, V, del[dO + j]);
-                if (d >= 0) {
-                    const uint64_t k = (uint64_t)s << 32 | (uint64_t)d;
-                    uint64_t h = hmix(k) & mask;
-                    while (true) {
-                        const uint64_t cur = *((volatile uint64_t*)&hk[h]);
-                        if (cur == k) {
-                            hit = atomicCAS((unsigned long long*)&hk[h], (unsigned long long)k,
-                                            (unsigned long long)kTomb) == k;
-                            break;
-                        }
-                        if (cur == kEmpty) break;
-                        h = (h + 1) & mask;
-                    }
-                }
+__device__ __forceinline__ bool del_item(int64_t s, uint64_t x, const uint64_t* __restrict__ ext, uint64_t V,
+                                         uint64_t* hk, uint64_t mask) {
+    const int64_t d = find_ext(ext, V, x);
+    if (d < 0) return false;
+    const uint64_t k = (uint64_t)s << 32 | (uint64_t)d;
+    uint64_t h = hmix(k) & mask;
+    while (true) {
+        const uint64_t cur = *((volatile uint64_t*)&hk[h]);
+        if (cur == k)
+            return atomicCAS((unsigned long long*)&hk[h], (unsigned long long)k, (unsigned long long)kTomb) == k;
+        if (cur == kEmpty) return false;
+        h = (h + 1) & mask;
+    }
+}
+// line 7: the records' deleted edges to TOMB; passes as in k_dyn_expand_ins
+template <int kPass>
+__global__ void __launch_bounds__(256) k_dyn_delete(const DeltaRec* __restrict__ rec, uint64_t nr,
+        const uint64_t* __restrict__ off, const uint64_t* __restrict__ del, const uint64_t* __restrict__ ext,
+        uint64_t V, uint64_t* hk, uint64_t mask, uint64_t* __restrict__ big, unsigned long long* __restrict__ n_big,
+        Ctr* __restrict__ c) {
+    unsigned long long hits = 0;
+    if (kPass == 0) {
+        const uint64_t i = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x;
+        if (i < nr) {
+            const uint64_t n = off[i + 1] - off[i];
+            if (n > kSmall) big[atomicAdd(n_big, 1ull)] = i;
+            else if (n) {
+                const DeltaRec r = rec[i];
+                const int64_t s = find_ext(ext, V, r.node);
+                if (s >= 0)                                      // D4
+                    for (uint64_t j = 0; j < n; ++j) hits += del_item(s, del[r.del_off + j], ext, V, hk, mask);
             }
-            wadd(&c->n_del, hit);
+        }
+    } else {
+        const uint64_t nb = *n_big, nw = (uint64_t)gridDim.x * (blockDim.x >> 5);
+        const unsigned lane = threadIdx.x & 31;
+        for (uint64_t q = blockIdx.x * (uint64_t)(blockDim.x >> 5) + (threadIdx.x >> 5); q < nb; q += nw) {
+            const uint64_t i = big[q], n = off[i + 1] - off[i];
+            int64_t s = lane == 0 ? find_ext(ext, V, rec[i].node) : -1;
+            s = __shfl_sync(0xffffffffu, s, 0);
+            if (s < 0) continue;
+            const uint64_t dO = rec[i].del_off;
+            for (uint64_t j = lane; j < n; j += 32) hits += del_item(s, del[dO + j], ext, V, hk, mask);
         }
     }
+    hits = warp_sum<unsigned long long>(hits);
+    if ((threadIdx.x & 31) == 0 && hits) atomicAdd(&c->n_del, hits);
 }
 
 __global__ void k_dyn_node_del(const uint64_t* __restrict__ del_ids, uint64_t nd, const uint64_t* __restrict__ ext,
-                               uint64_t V, uint32_t* live, Ctr* __restrict__ c) {
+                               uint64_t V, uint32_t* live, uint32_t* __restrict__ died_bits, uint32_t* __restrict__ filter,
+                               Ctr* __restrict__ c) {
     const uint64_t i = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x;
     bool died = false;
     if (i < nd) {
         const int64_t d = find_ext(ext, V, del_ids[i]);
         died = d >= 0 && atomicExch(&live[d], 0u) == 1u;       // line 11 (D4: dead / unknown: no-op)
+        if (died) {
+            atomicOr(&died_bits[d >> 5], 1u << (d & 31));
+            const uint64_t f = (uint64_t)d & (kFilterBits - 1);   // filter word for the cascade
+            atomicOr(&filter[f >> 5], 1u << (f & 31));
+        }
     }
     wadd(&c->n_vdel, died);
 }
 
-__global__ void k_dyn_cascade(uint64_t* __restrict__ hk, uint64_t cap, const uint32_t* __restrict__ live,
-                              Ctr* __restrict__ c) {
-    const uint64_t stride = (uint64_t)gridDim.x * blockDim.x;
-    for (uint64_t i0 = blockIdx.x * (uint64_t)blockDim.x; i0 < cap; i0 += stride) {
-        const uint64_t i = i0 + threadIdx.x;
-        bool gone = false;
-        if (i < cap) {
-            const uint64_t k = hk[i];
-            if (k < kTomb && (!live[k >> 32] || !live[k & 0xffffffffu])) {
-                hk[i] = kTomb;
-                gone = true;
-            }
+// every table key had two live endpoints before this cycle's node deletes, so a key is
+// removed iff an endpoint died this cycle (bitmap, V/8 bytes, L2-resident); 2 slots/thread
+// a 64 KB filter (bit v mod 2^19 of every dead vertex) in shared memory screens the keys;
+// the exact bitmap is read only on a filter hit
+__device__ __forceinline__ bool died_of(const uint32_t* __restrict__ b, const uint32_t* __restrict__ filt, uint64_t k) {
+    const uint64_t s = k >> 32, d = k & 0xffffffffu;
+    const uint32_t fs = (uint32_t)s & (kFilterBits - 1), fd = (uint32_t)d & (kFilterBits - 1);
+    if ((((filt[fs >> 5] >> (fs & 31)) | (filt[fd >> 5] >> (fd & 31))) & 1u) == 0) return false;
+    return ((__ldg(b + (s >> 5)) >> (s & 31)) | (__ldg(b + (d >> 5)) >> (d & 31))) & 1u;
+}
+__global__ void __launch_bounds__(256) k_dyn_cascade(uint64_t* __restrict__ hk, uint64_t cap,
+        const uint32_t* __restrict__ died_bits, const uint32_t* __restrict__ filter, Ctr* __restrict__ c) {
+    extern __shared__ uint32_t filt[];
+    for (uint32_t t = threadIdx.x; t < kFilterBits / 32; t += blockDim.x) filt[t] = filter[t];
+    __syncthreads();
+    const uint64_t stride = (uint64_t)gridDim.x * blockDim.x, half = cap >> 1;
+    ulonglong2* h2 = reinterpret_cast<ulonglong2*>(hk);
+    unsigned long long gone = 0;
+    constexpr int U = 4;   // 4 independent 16-byte loads in flight per thread
+    uint64_t i = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x;
+    for (; i + (U - 1) * stride < half; i += U * stride) {
+        ulonglong2 k[U];
+#pragma unroll
+        for (int u = 0; u < U; ++u) k[u] = __ldcs(h2 + i + u * stride);
+#pragma unroll
+        for (int u = 0; u < U; ++u) {
+            bool w = false;
+            if (k[u].x < kTomb && died_of(died_bits, filt, k[u].x)) { k[u].x = kTomb; w = true; ++gone; }
+            if (k[u].y < kTomb && died_of(died_bits, filt, k[u].y)) { k[u].y = kTomb; w = true; ++gone; }
+            if (w) h2[i + u * stride] = k[u];
         }
-        wadd(&c->n_casc, gone);
     }
+    for (; i < half; i += stride) {
+        ulonglong2 k = h2[i];
+        bool w = false;
+        if (k.x < kTomb && died_of(died_bits, filt, k.x)) { k.x = kTomb; w = true; ++gone; }
+        if (k.y < kTomb && died_of(died_bits, filt, k.y)) { k.y = kTomb; w = true; ++gone; }
+        if (w) h2[i] = k;
+    }
+    gone = warp_sum<unsigned long long>(gone);
+    if ((threadIdx.x & 31) == 0 && gone) atomicAdd(&c->n_casc, gone);
 }
 
 __global__ void k_dyn_rehash(const uint64_t* __restrict__ ok, const float* __restrict__ ov, uint64_t ocap,
@@ -251,8 +326,8 @@ __global__ void k_dyn_expand_flat(const uint64_t* __restrict__ src, const uint64
     const uint64_t i = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x;
     if (i >= n) return;
     const int64_t s = find_ext(ext, V, src[i]), d = find_ext(ext, V, dst[i]);
-    if (s < 0 || d < 0) { atomicOr(&c->bad, 1ull); keys[i] = V << 32; }
-    else keys[i] = (uint64_t)s << 32 | (uint64_t)d;
+    if (s < 0 || d < 0) { atomicOr(&c->bad, 1ull); keys[i] = V * V; }
+    else keys[i] = (uint64_t)s * V + (uint64_t)d;
     vals[i] = (uint32_t)i;
     witem[i] = w ? w[i] : 1.0f;
 }
@@ -272,7 +347,7 @@ __global__ void k_dyn_fill_u32(uint32_t* p, uint64_t n, uint32_t v) {
 
 // export
 __global__ void k_dyn_compact(const uint64_t* __restrict__ hk, const float* __restrict__ hv, uint64_t cap,
-                              uint64_t* __restrict__ ok, uint32_t* __restrict__ oi, float* __restrict__ ow,
+                              uint64_t V, uint64_t* __restrict__ ok, uint32_t* __restrict__ oi, float* __restrict__ ow,
                               Ctr* __restrict__ c) {
     const uint64_t stride = (uint64_t)gridDim.x * blockDim.x;
     const unsigned lane = threadIdx.x & 31;
@@ -286,23 +361,23 @@ __global__ void k_dyn_compact(const uint64_t* __restrict__ hk, const float* __re
         base = __shfl_sync(0xffffffffu, base, 0);
         if (keep) {
             const uint64_t p = base + __popc(m & ((1u << lane) - 1));
-            ok[p] = k;
+            ok[p] = (k >> 32) * V + (k & 0xffffffffu);   // sort key
             oi[p] = (uint32_t)p;
             ow[p] = hv[i];
         }
     }
 }
 __global__ void k_dyn_emit(const uint64_t* __restrict__ sk, const uint32_t* __restrict__ si, const float* __restrict__ cw,
-                           uint64_t E, uint32_t* __restrict__ cols, float* __restrict__ w) {
+                           uint64_t E, uint64_t V, uint32_t* __restrict__ cols, float* __restrict__ w) {
     const uint64_t i = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x;
     if (i >= E) return;
-    cols[i] = (uint32_t)(sk[i] & 0xffffffffu);
+    cols[i] = (uint32_t)(sk[i] % V);
     w[i] = cw[si[i]];
 }
 __global__ void k_dyn_offsets(const uint64_t* __restrict__ sk, uint64_t E, uint64_t V, int64_t* __restrict__ off) {
     const uint64_t v = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x;
     if (v > V) return;
-    const uint64_t key = v << 32;
+    const uint64_t key = v * V;   // sort key s * V + d
     uint64_t lo = 0, hi = E;
     while (lo < hi) {
         const uint64_t m = (lo + hi) >> 1;
@@ -319,8 +394,8 @@ __global__ void k_dyn_live_u8(const uint32_t* __restrict__ live, uint64_t V, uin
 
 struct h2tap_dyn {
     h2tap_replica* r = nullptr;   // stream, allocator, radix-sort scratch
-    uint64_t V = 0, n_live = 0, n_tomb = 0, cap = 0;
-    Buf ext, live, hk, hv;
+    uint64_t V = 0, n_live = 0, n_tomb = 0, cap = 0, xid = 0;   // xid = ext[V - 1] (host copy)
+    Buf ext, live, hk, hv, died, big;
     Buf cin, cdel, oin, odel, new_ids, del_ids, kill, flag, fpos, keys, vals, keys2, vals2, witem, ctr, xo;
     Buf x_rec, x_ins, x_wts, x_del;
     dyn::Ctr* hctr = nullptr;     // pinned host mirror
@@ -331,7 +406,7 @@ namespace {
 void dyn_free(h2tap_dyn* d) {
     if (!d) return;
     if (d->r) {
-        for (Buf* b : {&d->ext, &d->live, &d->hk, &d->hv, &d->cin, &d->cdel, &d->oin, &d->odel, &d->new_ids,
+        for (Buf* b : {&d->ext, &d->live, &d->died, &d->big, &d->hk, &d->hv, &d->cin, &d->cdel, &d->oin, &d->odel, &d->new_ids,
                        &d->del_ids, &d->kill, &d->flag, &d->fpos, &d->keys, &d->vals, &d->keys2, &d->vals2,
                        &d->witem, &d->ctr, &d->xo, &d->x_rec, &d->x_ins, &d->x_wts, &d->x_del})
             if (b->p) d->r->dfree(b->p);
@@ -377,11 +452,13 @@ uint64_t pow2_at_least(uint64_t x) {
     return c;
 }
 
-// make room for `incoming` more keys at load <= 1/2 (tombstones count as used)
+// make room for `incoming` more keys at load <= 0.7 (tombstones count as used); a re-hash
+// sizes for load <= 0.7 as well, so after it the load is 0.35-0.7 (the cascade pass of a
+// node delete streams the whole table: a denser table is a shorter pass)
 void dyn_reserve_table(h2tap_dyn* d, uint64_t incoming) {
     h2tap_replica* r = d->r;
-    if (d->cap && 2 * (d->n_live + d->n_tomb + incoming) <= d->cap) return;
-    const uint64_t nc = pow2_at_least(2 * (d->n_live + incoming) + 1);
+    if (d->cap && 10 * (d->n_live + d->n_tomb + incoming) <= 7 * d->cap) return;
+    const uint64_t nc = pow2_at_least((10 * (d->n_live + incoming)) / 7 + 1);
     Buf k2, v2;
     uint64_t* nk = r->get<uint64_t>(k2, nc);
     float* nv = r->get<float>(v2, nc);
@@ -408,8 +485,8 @@ void dyn_upsert_items(h2tap_dyn* d, uint64_t n, dyn::Ctr* c) {
     uint32_t* v = static_cast<uint32_t*>(d->vals.p);
     uint64_t* k2 = static_cast<uint64_t*>(d->keys2.p);
     uint32_t* v2 = static_cast<uint32_t*>(d->vals2.p);
-    radix_sort(r, k, v, k2, v2, n, 32 + bits_for(d->V));
-    dyn::k_dyn_upsert<<<g1(n), 256, 0, r->st>>>(k, v, n, static_cast<float*>(d->witem.p), d->V << 32,
+    radix_sort(r, k, v, k2, v2, n, bits_for(d->V * d->V));
+    dyn::k_dyn_upsert<<<g1(n), 256, 0, r->st>>>(k, v, n, static_cast<float*>(d->witem.p), d->V,
                                                 static_cast<uint64_t*>(d->hk.p), static_cast<float*>(d->hv.p),
                                                 d->cap - 1, c);
     CKL();
@@ -448,11 +525,7 @@ h2tap_status dyn_apply(h2tap_dyn* d, const h2tap_record_batch* b, h2tap_apply_st
         rec = xr; ins = xi; wts = xw; del = xd;
     }
     // ---- lines 1-9: classify records
-    uint64_t xid = 0;
-    if (d->V) {
-        CK(cudaMemcpyAsync(&xid, static_cast<uint64_t*>(d->ext.p) + d->V - 1, 8, cudaMemcpyDeviceToHost, st));
-        g_d2h += 8;
-    }
+    const uint64_t xid = d->xid;
     dyn::Ctr* c = dyn_ctr_reset(d);
     uint64_t* cin = r->get<uint64_t>(d->cin, nr + 1);
     uint64_t* cdel = r->get<uint64_t>(d->cdel, nr + 1);
@@ -460,7 +533,6 @@ h2tap_status dyn_apply(h2tap_dyn* d, const h2tap_record_batch* b, h2tap_apply_st
     uint64_t* odel = r->get<uint64_t>(d->odel, nr + 1);
     uint64_t* new_ids = r->get<uint64_t>(d->new_ids, nr);
     uint64_t* del_ids = r->get<uint64_t>(d->del_ids, nr);
-    r->sync();  // xid
     dyn::k_dyn_rec<<<g1(nr + 1), 256, 0, st>>>(rec, nr, b->n_inserts, b->n_deletes, xid, d->V ? 1 : 0, cin, cdel,
                                               new_ids, del_ids, c);
     CKL();
@@ -522,7 +594,7 @@ h2tap_status dyn_apply(h2tap_dyn* d, const h2tap_record_batch* b, h2tap_apply_st
         g_d2h += 8;
         dyn_reserve_vertices(d, d->V + u);
         dyn::k_dyn_append<<<g1(u), 256, 0, st>>>(k, u, flag, pos, base, static_cast<uint64_t*>(d->ext.p) + d->V,
-                                                 static_cast<uint32_t*>(d->live.p) + d->V);
+                                                 static_cast<uint32_t*>(d->live.p) + d->V, c);
         CKL();
         r->sync();
         if (d->V + n_vins >= 0xFFFFFFFFull) { set_err("more than 2^32 - 2 dense vertex ids"); return H2TAP_E_CAPACITY; }
@@ -530,31 +602,46 @@ h2tap_status dyn_apply(h2tap_dyn* d, const h2tap_record_batch* b, h2tap_apply_st
     }
     const uint64_t* ext = static_cast<const uint64_t*>(d->ext.p);
     uint32_t* live = static_cast<uint32_t*>(d->live.p);
-    const unsigned wgrid = (unsigned)std::min<uint64_t>(cdiv(std::max<uint64_t>(nr, 1), 8), (uint64_t)r->n_sm * 16);
+    const unsigned wgrid = (unsigned)r->n_sm * 4;   // warp passes over the queued large records
     // ---- lines 6 + 10: one insert batch (D1, D2)
     if (n_ins) {
         dyn_item_bufs(d, n_ins);
-        dyn::k_dyn_expand_ins<<<wgrid, 256, 0, st>>>(rec, nr, oin, ins, wts, ext, live, d->V,
-                                                     static_cast<uint64_t*>(d->keys.p), static_cast<uint32_t*>(d->vals.p),
-                                                     static_cast<float*>(d->witem.p), c);
+        uint64_t* big = r->get<uint64_t>(d->big, nr);
+        unsigned long long* nbig = &c->n_big_ins;
+        dyn::k_dyn_expand_ins<0><<<g1(nr), 256, 0, st>>>(rec, nr, oin, ins, wts, ext, live, d->V,
+                                                        static_cast<uint64_t*>(d->keys.p), static_cast<uint32_t*>(d->vals.p),
+                                                        static_cast<float*>(d->witem.p), big, nbig, c);
+        CKL();
+        dyn::k_dyn_expand_ins<1><<<wgrid, 256, 0, st>>>(rec, nr, oin, ins, wts, ext, live, d->V,
+                                                       static_cast<uint64_t*>(d->keys.p), static_cast<uint32_t*>(d->vals.p),
+                                                       static_cast<float*>(d->witem.p), big, nbig, c);
         CKL();
         dyn_reserve_table(d, n_ins);
         dyn_upsert_items(d, n_ins, c);
     }
     // ---- line 7: delete batch
     if (tot[1] && d->cap) {
-        dyn::k_dyn_delete<<<wgrid, 256, 0, st>>>(rec, nr, odel, del, ext, d->V, static_cast<uint64_t*>(d->hk.p),
-                                                 d->cap - 1, c);
+        uint64_t* big = r->get<uint64_t>(d->big, nr);
+        uint64_t* hk = static_cast<uint64_t*>(d->hk.p);
+        dyn::k_dyn_delete<0><<<g1(nr), 256, 0, st>>>(rec, nr, odel, del, ext, d->V, hk, d->cap - 1, big, &c->n_big_del, c);
+        CKL();
+        dyn::k_dyn_delete<1><<<wgrid, 256, 0, st>>>(rec, nr, odel, del, ext, d->V, hk, d->cap - 1, big, &c->n_big_del, c);
         CKL();
     }
     // ---- line 11: node deletes + cascade
     if (h0.n_del_ids) {
-        dyn::k_dyn_node_del<<<g1(h0.n_del_ids), 256, 0, st>>>(del_ids, h0.n_del_ids, ext, d->V, live, c);
+        const uint64_t nwd = (d->V + 31) / 32, nwf = dyn::kFilterBits / 32;
+        uint32_t* died = r->get<uint32_t>(d->died, nwd + nwf);
+        uint32_t* filter = died + nwd;
+        CK(cudaMemsetAsync(died, 0, (nwd + nwf) * 4, st));
+        dyn::k_dyn_node_del<<<g1(h0.n_del_ids), 256, 0, st>>>(del_ids, h0.n_del_ids, ext, d->V, live, died, filter, c);
         CKL();
         dyn_ctr_read(d);
         if (d->hctr->n_vdel && d->cap) {
-            const unsigned grid = (unsigned)std::min<uint64_t>(g1(d->cap), (uint64_t)r->n_sm * 8);
-            dyn::k_dyn_cascade<<<grid, 256, 0, st>>>(static_cast<uint64_t*>(d->hk.p), d->cap, live, c);
+            constexpr int smem = dyn::kFilterBits / 8;
+            CK(cudaFuncSetAttribute(dyn::k_dyn_cascade, cudaFuncAttributeMaxDynamicSharedMemorySize, smem));
+            const unsigned grid = (unsigned)std::min<uint64_t>(g1(d->cap / 2), (uint64_t)r->n_sm * 3);  // 3 CTAs/SM
+            dyn::k_dyn_cascade<<<grid, 256, smem, st>>>(static_cast<uint64_t*>(d->hk.p), d->cap, died, filter, c);
             CKL();
         }
     }
@@ -563,6 +650,7 @@ h2tap_status dyn_apply(h2tap_dyn* d, const h2tap_record_batch* b, h2tap_apply_st
     const dyn::Ctr& h = *d->hctr;
     d->n_live = d->n_live + h.n_new - h.n_del - h.n_casc;
     d->n_tomb += h.n_del + h.n_casc;
+    if (n_vins) d->xid = h.last_ext;
     if (stats) {
         std::memset(stats, 0, sizeof(*stats));
         stats->n_visible = n_ins + tot[1] + u + h0.n_del_ids;
@@ -621,6 +709,10 @@ h2tap_status h2tap_dyn_create(const h2tap_config* cfg, size_t n_vertices, const 
         dyn_ctr_read(d);
         if (d->hctr->bad) { set_err("vertex ids not strictly increasing"); return H2TAP_E_INVAL; }
         d->V = n_vertices;
+        if (n_vertices) {
+            CK(cudaMemcpyAsync(&d->xid, ext + n_vertices - 1, 8, cudaMemcpyDeviceToHost, r->st));
+            r->sync();
+        }
         dyn_reserve_table(d, n_edges);
         if (n_edges) {
             dyn_item_bufs(d, n_edges);
@@ -688,16 +780,16 @@ h2tap_status h2tap_dyn_export(h2tap_dyn* d, int64_t* offsets, uint32_t* cols, fl
         if (d->cap) {
             const unsigned grid = (unsigned)std::min<uint64_t>(g1(d->cap), (uint64_t)r->n_sm * 8);
             dyn::k_dyn_compact<<<grid, 256, 0, st>>>(static_cast<uint64_t*>(d->hk.p), static_cast<float*>(d->hv.p),
-                                                     d->cap, k, v, cw, c);
+                                                     d->cap, V, k, v, cw, c);
             CKL();
         }
-        radix_sort(r, k, v, k2, v2, E, 32 + bits_for(V));
+        radix_sort(r, k, v, k2, v2, E, bits_for(V * V));
         Buf bo, bc, bw, bl;
         int64_t* o_off = r->get<int64_t>(bo, V + 1);
         uint32_t* o_cols = r->get<uint32_t>(bc, E);
         float* o_w = r->get<float>(bw, E);
         uint8_t* o_live = r->get<uint8_t>(bl, V);
-        if (E) { dyn::k_dyn_emit<<<g1(E), 256, 0, st>>>(k, v, cw, E, o_cols, o_w); CKL(); }
+        if (E) { dyn::k_dyn_emit<<<g1(E), 256, 0, st>>>(k, v, cw, E, V, o_cols, o_w); CKL(); }
         dyn::k_dyn_offsets<<<g1(V + 1), 256, 0, st>>>(k, E, V, o_off);
         CKL();
         if (V) { dyn::k_dyn_live_u8<<<g1(V), 256, 0, st>>>(static_cast<uint32_t*>(d->live.p), V, o_live); CKL(); }

@@ -27,7 +27,7 @@
 namespace dyn {
 
 constexpr uint64_t kEmpty = ~0ull, kTomb = ~0ull - 1;
-constexpr uint32_t kFilterBits = 1u << 19;   // cascade filter: 64 KB of shared memory
+constexpr uint32_t kFilterBits = 1u << 18;   // cascade filter: 32 KB of shared memory
 
 struct Ctr {
     unsigned long long n_new_ids, n_del_ids, bad, max_new, n_new, n_upd, n_del, n_casc, n_gated, n_vdel, n_out, last_ext, n_big_ins, n_big_del;
@@ -268,7 +268,7 @@ __global__ void k_dyn_node_del(const uint64_t* __restrict__ del_ids, uint64_t nd
 
 // every table key had two live endpoints before this cycle's node deletes, so a key is
 // removed iff an endpoint died this cycle (bitmap, V/8 bytes, L2-resident); 2 slots/thread
-// a 64 KB filter (bit v mod 2^19 of every dead vertex) in shared memory screens the keys;
+// a 32 KB filter (bit v mod 2^18 of every dead vertex) in shared memory screens the keys;
 // the exact bitmap is read only on a filter hit
 __device__ __forceinline__ bool died_of(const uint32_t* __restrict__ b, const uint32_t* __restrict__ filt, uint64_t k) {
     const uint64_t s = k >> 32, d = k & 0xffffffffu;
@@ -276,7 +276,7 @@ __device__ __forceinline__ bool died_of(const uint32_t* __restrict__ b, const ui
     if ((((filt[fs >> 5] >> (fs & 31)) | (filt[fd >> 5] >> (fd & 31))) & 1u) == 0) return false;
     return ((__ldg(b + (s >> 5)) >> (s & 31)) | (__ldg(b + (d >> 5)) >> (d & 31))) & 1u;
 }
-__global__ void __launch_bounds__(256) k_dyn_cascade(uint64_t* __restrict__ hk, uint64_t cap,
+__global__ void __launch_bounds__(256, 4) k_dyn_cascade(uint64_t* __restrict__ hk, uint64_t cap,
         const uint32_t* __restrict__ died_bits, const uint32_t* __restrict__ filter, Ctr* __restrict__ c) {
     extern __shared__ uint32_t filt[];
     for (uint32_t t = threadIdx.x; t < kFilterBits / 32; t += blockDim.x) filt[t] = filter[t];
@@ -640,7 +640,7 @@ h2tap_status dyn_apply(h2tap_dyn* d, const h2tap_record_batch* b, h2tap_apply_st
         if (d->hctr->n_vdel && d->cap) {
             constexpr int smem = dyn::kFilterBits / 8;
             CK(cudaFuncSetAttribute(dyn::k_dyn_cascade, cudaFuncAttributeMaxDynamicSharedMemorySize, smem));
-            const unsigned grid = (unsigned)std::min<uint64_t>(g1(d->cap / 2), (uint64_t)r->n_sm * 3);  // 3 CTAs/SM
+            const unsigned grid = (unsigned)std::min<uint64_t>(g1(d->cap / 2), (uint64_t)r->n_sm * 4);  // 4 CTAs/SM
             dyn::k_dyn_cascade<<<grid, 256, smem, st>>>(static_cast<uint64_t*>(d->hk.p), d->cap, died, filter, c);
             CKL();
         }

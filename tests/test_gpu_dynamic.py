@@ -146,3 +146,42 @@ def test_empty_graph_and_empty_cycle(h2):
     rb = synth.RecordBatch(rec, np.array([9, 5], np.uint64), np.array([1.5, 2.5], np.float32),
                            np.zeros(0, np.uint64))
     cycle(g, o, rb, "first nodes into an empty replica")
+
+
+def test_full_size_sampled_rows(h2):
+    """bench_dyn.py's workload (configs[2]'s RMAT-24 graph, 500 K records with node deletes and
+    new nodes, device-resident): ext ids and liveness compared in full, the rows of 256 sampled
+    sources (+ every node-delete victim's row) against O3 run on the sub-problem that decides
+    them (all vertices, the sampled sources' edges, the records of those sources, every
+    deletion and every new node: no other record can touch those rows)."""
+    import torch
+    scale = 24
+    n = 1 << scale
+    seed = synth.seed_of("c3")
+    src, dst, w = synth.rmat_edges(scale, seed, n=16 * n)
+    dev = [torch.from_numpy(a.view(np.int64) if a.dtype == np.uint64 else a).cuda() for a in (src, dst, w)]
+    g = h2.DynReplica.from_edges(n, None, *dev)
+    del dev
+    rb = synth.dyn_record_batch(seed, 1000, n - 1, 500_000, n_new=64, max_slice=2, p_deleted=0.0002,
+                                p_new=0.0005, p_invalid=0.0)
+    st = g.apply_records(synth.RecordBatch(torch.from_numpy(rb.records.view(np.uint8)).cuda(),
+                                           torch.from_numpy(rb.inserts.view(np.int64)).cuda(),
+                                           torch.from_numpy(rb.weights).cuda(),
+                                           torch.from_numpy(rb.deletes.view(np.int64)).cuda()))
+    rng = np.random.default_rng(5)
+    sample = np.unique(np.concatenate([rng.integers(0, n, 256),
+                                       rb.records["node"][rb.records["deleted"] == 1][:16].astype(np.int64)]))
+    sample = sample[sample < n].astype(np.uint64)
+    keep_e = np.isin(src, sample)
+    o = DynamicOracle(np.arange(n, dtype=np.uint64), src[keep_e], dst[keep_e], w[keep_e])
+    r = rb.records
+    keep_r = np.isin(r["node"], sample) | (r["deleted"] == 1) | (r["node"] > n - 1)
+    o.apply_records(r[keep_r], rb.inserts, rb.weights, rb.deletes)
+    off, cols, ww, ids, live = g.export()
+    ooff, ocols, ow, oids, olive = o.export()
+    assert np.array_equal(ids, oids) and np.array_equal(live, olive)
+    assert st["n_vertex_inserted"] == len(ids) - n and int((live == 0).sum()) == st["n_vertex_deleted"]
+    for s in sample.astype(np.int64):
+        a, b = slice(off[s], off[s + 1]), slice(ooff[s], ooff[s + 1])
+        assert np.array_equal(cols[a], ocols[b]) and np.array_equal(ww[a], ow[b]), f"row {s}"
+    assert off[-1] == g.info()["n_edges"]

@@ -48,15 +48,17 @@ def main():
     torch.cuda.synchronize()
     create_s = time.time() - t0
     inf0 = g.info()
-    batches = []
+    batches, host = [], []
     xid = n - 1
-    for k in range(args.warmup + args.cycles):
+    for k in range(2 * (args.warmup + args.cycles)):
         rb = synth.dyn_record_batch(synth.seed_of("c3"), 1000 + k, xid, args.records, n_new=64, max_slice=2,
                                     p_deleted=args.node_deletes, p_new=0.0005, p_invalid=0.0)
-        batches.append(synth.RecordBatch(torch.from_numpy(rb.records.view(np.uint8)).cuda(),
-                                         torch.from_numpy(rb.inserts.view(np.int64)).cuda(),
-                                         torch.from_numpy(rb.weights).cuda(),
-                                         torch.from_numpy(rb.deletes.view(np.int64)).cuda()))
+        t = (torch.from_numpy(rb.records.view(np.uint8)), torch.from_numpy(rb.inserts.view(np.int64)),
+             torch.from_numpy(rb.weights), torch.from_numpy(rb.deletes.view(np.int64)))
+        if k < args.warmup + args.cycles:
+            batches.append(synth.RecordBatch(*(x.cuda() for x in t)))
+        else:   # the e2e leg: pinned host records, the H2D copy inside the timed call
+            host.append(synth.RecordBatch(*(x.pin_memory() for x in t)))
         xid += 64
     ms, lib_ms, items, sts = [], [], [], []
     for k, rb in enumerate(batches):
@@ -70,6 +72,18 @@ def main():
             lib_ms.append(s["ms_total"])
             items.append(s["n_visible"])
             sts.append(s)
+    e2e_ms, e2e_items, h2d, d2h = [], [], [], []
+    for k, rb in enumerate(host):
+        torch.cuda.synchronize()
+        ev0.record(st)
+        s = g.apply_records(rb)
+        ev1.record(st)
+        torch.cuda.synchronize()
+        if k >= args.warmup:
+            e2e_ms.append(ev0.elapsed_time(ev1))
+            e2e_items.append(s["n_visible"])
+            h2d.append(s["h2d_bytes"])
+            d2h.append(s["d2h_bytes"])
     torch.cuda.synchronize()
     t0 = time.time()
     out = g.export()
@@ -84,6 +98,10 @@ def main():
                                f"cycle (<=2 inserts + <=2 deletes each), node-delete records p={args.node_deletes}",
                    "inputs": "device-resident records"},
         "graph": {"vertices": inf0["n_vertices"], "edges": inf0["n_edges"], "table_slots": inf0["table_slots"]},
+        "e2e": {"value": sum(e2e_items) / (sum(e2e_ms) / 1e3), "unit": "updates/s",
+                "h2d_bytes_per_step": sum(h2d) / len(h2d), "d2h_bytes_per_step": sum(d2h) / len(d2h),
+                "note": "records in pinned host memory, copied by the library inside each timed call "
+                        "(the counters come back in small D2H reads)"},
         "create_s": create_s, "export_host_s": export_s, "export_edges": int(len(out[1])),
         "last_cycle": {k: sts[-1][k] for k in ("n_new", "n_upd", "n_del", "n_casc", "n_gated",
                                                 "n_vertex_inserted", "n_vertex_deleted", "n_launches")},

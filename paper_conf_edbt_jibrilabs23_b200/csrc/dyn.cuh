@@ -278,6 +278,7 @@ __device__ __forceinline__ bool died_of(const uint32_t* __restrict__ b, const ui
 }
 __global__ void __launch_bounds__(256, 4) k_dyn_cascade(uint64_t* __restrict__ hk, uint64_t cap,
         const uint32_t* __restrict__ died_bits, const uint32_t* __restrict__ filter, Ctr* __restrict__ c) {
+    if (*(volatile unsigned long long*)&c->n_vdel == 0) return;   // nobody died this cycle (no host sync)
     extern __shared__ uint32_t filt[];
     for (uint32_t t = threadIdx.x; t < kFilterBits / 32; t += blockDim.x) filt[t] = filter[t];
     __syncthreads();
@@ -636,8 +637,7 @@ h2tap_status dyn_apply(h2tap_dyn* d, const h2tap_record_batch* b, h2tap_apply_st
         CK(cudaMemsetAsync(died, 0, (nwd + nwf) * 4, st));
         dyn::k_dyn_node_del<<<g1(h0.n_del_ids), 256, 0, st>>>(del_ids, h0.n_del_ids, ext, d->V, live, died, filter, c);
         CKL();
-        dyn_ctr_read(d);
-        if (d->hctr->n_vdel && d->cap) {
+        if (d->cap) {
             constexpr int smem = dyn::kFilterBits / 8;
             CK(cudaFuncSetAttribute(dyn::k_dyn_cascade, cudaFuncAttributeMaxDynamicSharedMemorySize, smem));
             const unsigned grid = (unsigned)std::min<uint64_t>(g1(d->cap / 2), (uint64_t)r->n_sm * 4);  // 4 CTAs/SM

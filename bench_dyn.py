@@ -35,6 +35,7 @@ def main():
     ap.add_argument("--cycles", type=int, default=5)
     ap.add_argument("--warmup", type=int, default=3)
     ap.add_argument("--node-deletes", type=float, default=0.0)
+    ap.add_argument("--no-cpu-baseline", action="store_true")
     args = ap.parse_args()
     torch.cuda.set_device(0)
     st = torch.cuda.current_stream()
@@ -60,7 +61,7 @@ def main():
         else:   # the e2e leg: pinned host records, the H2D copy inside the timed call
             host.append(synth.RecordBatch(*(x.pin_memory() for x in t)))
         xid += 64
-    ms, lib_ms, items, sts = [], [], [], []
+    ms, lib_ms, items, sts, casc = [], [], [], [], []
     for k, rb in enumerate(batches):
         torch.cuda.synchronize()
         ev0.record(st)
@@ -72,6 +73,8 @@ def main():
             lib_ms.append(s["ms_total"])
             items.append(s["n_visible"])
             sts.append(s)
+            if s["bytes_merge"]:
+                casc.append((s["bytes_merge"], s["ms_merge"]))
     e2e_ms, e2e_items, h2d, d2h = [], [], [], []
     for k, rb in enumerate(host):
         torch.cuda.synchronize()
@@ -106,7 +109,38 @@ def main():
         "last_cycle": {k: sts[-1][k] for k in ("n_new", "n_upd", "n_del", "n_casc", "n_gated",
                                                 "n_vertex_inserted", "n_vertex_deleted", "n_launches")},
     }
+    if casc:   # node-delete cycles: the cascade pass dominates and is HBM-bound
+        pk = json.load(open(os.path.join(ROOT, "MEASURED_PEAKS.json")))
+        peak = float(pk["hbm_gbs"])
+        b = sum(x[0] for x in casc) / len(casc)
+        t = sum(x[1] for x in casc) / len(casc)
+        line["roofline"] = {"bound": "hbm", "kernel": "k_dyn_cascade", "achieved": b / (t * 1e-3) / 1e9,
+                            "peak": peak, "unit": "GB/s", "frac": b / (t * 1e-3) / 1e9 / peak,
+                            "traffic": None, "bytes_per_launch": b, "ms_per_launch": t,
+                            "peak_source": "measured (MEASURED_PEAKS.json hbm_gbs)"}
+    if not args.no_cpu_baseline:
+        line["cpu_baseline"] = cpu_baseline()
     print(json.dumps(line))
+
+
+def cpu_baseline(scale: int = 16, records: int = 20000, cycles: int = 3):
+    """O3 (oracle/o3_dynamic.py, as it stands) on a bounded sample: an RMAT-16 graph and
+    20 K-record cycles of the same generator, timed on this host (one thread)."""
+    from oracle.o3_dynamic import DynamicOracle
+    n = 1 << scale
+    src, dst, w = synth.rmat_edges(scale, synth.seed_of("c3"), n=16 * n)
+    o = DynamicOracle(np.arange(n, dtype=np.uint64), src, dst, w)
+    xid, items, t = n - 1, 0, 0.0
+    for k in range(cycles):
+        rb = synth.dyn_record_batch(synth.seed_of("c3"), 1000 + k, xid, records, n_new=64, max_slice=2,
+                                    p_deleted=0.0, p_new=0.0005, p_invalid=0.0)
+        t0 = time.perf_counter()
+        o.apply_records(rb.records, rb.inserts, rb.weights, rb.deletes)
+        t += time.perf_counter() - t0
+        items += int(rb.records["ins_cnt"].sum() + rb.records["del_cnt"].sum())
+        xid += 64
+    return {"value": items / t, "unit": "updates/s", "cores": 1, "kind": "oracle",
+            "sample": f"O3 on RMAT-{scale} x16, {cycles} cycles of {records} records (edge-only), apply only"}
 
 
 if __name__ == "__main__":

@@ -348,6 +348,8 @@ h2tap_status h2tap_dyn_create(const h2tap_config* cfg, size_t n_vertices, const 
 /* One cycle of Algorithm 1 over `batch` (the h2tap_record_batch layout above).  Flag other
  * than 0/1 or a slice outside its array -> E_INVAL before anything is applied.  stats
  * (nullable): n_new / n_upd / n_del / n_casc / n_gated / n_vertex_*, ms_total (device time),
+ * ms_merge / bytes_merge = the cascade pass's event-timed duration and table bytes (cycles in
+ * which a node died; else 0),
  * n_launches, h2d_bytes; n_visible = expanded items (inserts + deletes + node ops). */
 h2tap_status h2tap_dyn_apply_records(h2tap_dyn* d, const h2tap_record_batch* batch,
         h2tap_apply_stats* stats);

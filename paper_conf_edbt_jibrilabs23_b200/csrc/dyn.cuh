@@ -630,6 +630,7 @@ h2tap_status dyn_apply(h2tap_dyn* d, const h2tap_record_batch* b, h2tap_apply_st
         CKL();
     }
     // ---- line 11: node deletes + cascade
+    bool casc_timed = false;
     if (h0.n_del_ids) {
         const uint64_t nwd = (d->V + 31) / 32, nwf = dyn::kFilterBits / 32;
         uint32_t* died = r->get<uint32_t>(d->died, nwd + nwf);
@@ -641,8 +642,11 @@ h2tap_status dyn_apply(h2tap_dyn* d, const h2tap_record_batch* b, h2tap_apply_st
             constexpr int smem = dyn::kFilterBits / 8;
             CK(cudaFuncSetAttribute(dyn::k_dyn_cascade, cudaFuncAttributeMaxDynamicSharedMemorySize, smem));
             const unsigned grid = (unsigned)std::min<uint64_t>(g1(d->cap / 2), (uint64_t)r->n_sm * 4);  // 4 CTAs/SM
+            CK(cudaEventRecord(r->ev[2], st));
             dyn::k_dyn_cascade<<<grid, 256, smem, st>>>(static_cast<uint64_t*>(d->hk.p), d->cap, died, filter, c);
             CKL();
+            CK(cudaEventRecord(r->ev[3], st));
+            casc_timed = true;
         }
     }
     CK(cudaEventRecord(r->ev[1], st));
@@ -662,6 +666,10 @@ h2tap_status dyn_apply(h2tap_dyn* d, const h2tap_record_batch* b, h2tap_apply_st
         stats->n_vertex_inserted = n_vins;
         stats->n_vertex_deleted = h.n_vdel;
         stats->ms_total = ev_ms(r->ev[0], r->ev[1]);
+        if (casc_timed && h.n_vdel) {   // the cascade pass: its launch time and the table bytes it streams
+            stats->ms_merge = ev_ms(r->ev[2], r->ev[3]);
+            stats->bytes_merge = d->cap * 8;
+        }
         // algorithmic bytes: records + slices read, one 12-byte slot touch per item
         stats->bytes_alg = nr * sizeof(DeltaRec) + n_ins * 12 + tot[1] * 8 + (n_ins + tot[1]) * 12;
         stats->n_launches = g_launches;
@@ -694,7 +702,8 @@ h2tap_status h2tap_dyn_create(const h2tap_config* cfg, size_t n_vertices, const 
         h2tap_replica* r = d->r;
         CK(cudaHostAlloc(reinterpret_cast<void**>(&d->hctr), sizeof(dyn::Ctr), cudaHostAllocDefault));
         if (!r->ev[0]) CK(cudaEventCreate(&r->ev[0]));
-        if (!r->ev[1]) CK(cudaEventCreate(&r->ev[1]));
+        for (int e = 1; e < 4; ++e)
+            if (!r->ev[e]) CK(cudaEventCreate(&r->ev[e]));
         dyn_reserve_vertices(d, n_vertices);
         uint64_t* ext = static_cast<uint64_t*>(d->ext.p);
         if (vertex_ids) copy_in(r, ext, vertex_ids, n_vertices, on_device);

@@ -75,18 +75,43 @@ def main():
             sts.append(s)
             if s["bytes_merge"]:
                 casc.append((s["bytes_merge"], s["ms_merge"]))
-    e2e_ms, e2e_items, h2d, d2h = [], [], [], []
-    for k, rb in enumerate(host):
-        torch.cuda.synchronize()
-        ev0.record(st)
-        s = g.apply_records(rb)
-        ev1.record(st)
-        torch.cuda.synchronize()
-        if k >= args.warmup:
-            e2e_ms.append(ev0.elapsed_time(ev1))
-            e2e_items.append(s["n_visible"])
-            h2d.append(s["h2d_bytes"])
-            d2h.append(s["d2h_bytes"])
+    # e2e leg, pipelined through the public API: batch k+1's records are copied from pinned host
+    # memory into one of two device slots on a copy stream while batch k is applied; every copy
+    # of the timed cycles is inside the timed region (one region over all of them)
+    cs = torch.cuda.Stream()
+    slots = [None, None]
+    evs = [torch.cuda.Event(), torch.cuda.Event()]
+
+    def stage(k):
+        with torch.cuda.stream(cs):
+            slots[k % 2] = synth.RecordBatch(*(x.to("cuda", non_blocking=True) for x in
+                                               (host[k].records, host[k].inserts, host[k].weights, host[k].deletes)))
+            evs[k % 2].record(cs)
+
+    def run(lo, hi):
+        items, h2d_b, d2h_b = 0, 0, 0
+        stage(lo)
+        for k in range(lo, hi):
+            st.wait_event(evs[k % 2])
+            cur = slots[k % 2]
+            if k + 1 < hi:
+                cs.wait_stream(st)          # slot (k+1)%2 was last read by apply k-1
+                stage(k + 1)
+            s = g.apply_records(cur)
+            items += s["n_visible"]
+            h2d_b += sum(int(x.numel() * x.element_size()) for x in
+                         (host[k].records, host[k].inserts, host[k].weights, host[k].deletes))
+            d2h_b += s["d2h_bytes"]
+        return items, h2d_b, d2h_b
+
+    run(0, args.warmup)
+    torch.cuda.synchronize()
+    ev0.record(st)
+    e2e_items, h2d_b, d2h_b = run(args.warmup, len(host))
+    ev1.record(st)
+    torch.cuda.synchronize()
+    e2e_ms = ev0.elapsed_time(ev1)
+    n_e2e = len(host) - args.warmup
     torch.cuda.synchronize()
     t0 = time.time()
     out = g.export()
@@ -101,10 +126,11 @@ def main():
                                f"cycle (<=2 inserts + <=2 deletes each), node-delete records p={args.node_deletes}",
                    "inputs": "device-resident records"},
         "graph": {"vertices": inf0["n_vertices"], "edges": inf0["n_edges"], "table_slots": inf0["table_slots"]},
-        "e2e": {"value": sum(e2e_items) / (sum(e2e_ms) / 1e3), "unit": "updates/s",
-                "h2d_bytes_per_step": sum(h2d) / len(h2d), "d2h_bytes_per_step": sum(d2h) / len(d2h),
-                "note": "records in pinned host memory, copied by the library inside each timed call "
-                        "(the counters come back in small D2H reads)"},
+        "e2e": {"value": e2e_items / (e2e_ms / 1e3), "unit": "updates/s",
+                "h2d_bytes_per_step": h2d_b / n_e2e, "d2h_bytes_per_step": d2h_b / n_e2e,
+                "note": "records in pinned host memory; the next cycle's records are copied on a copy "
+                        "stream into one of two device slots while the current cycle is applied; one timed "
+                        "region over all cycles (copies included)"},
         "create_s": create_s, "export_host_s": export_s, "export_edges": int(len(out[1])),
         "last_cycle": {k: sts[-1][k] for k in ("n_new", "n_upd", "n_del", "n_casc", "n_gated",
                                                 "n_vertex_inserted", "n_vertex_deleted", "n_launches")},

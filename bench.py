@@ -441,6 +441,26 @@ def run_gpu(args):
         dist.destroy_process_group()
 
 
+def cpu_baseline_dyn(scale: int = 16, records: int = 20000, cycles: int = 3):
+    """cpu_baseline leg of --replica dyn: O3 (oracle/o3_dynamic.py, as it stands) on a bounded sample: an RMAT-16 graph and
+    20 K-record cycles of the same generator, timed on this host (one thread)."""
+    from oracle.o3_dynamic import DynamicOracle
+    n = 1 << scale
+    src, dst, w = synth.rmat_edges(scale, synth.seed_of("c3"), n=16 * n)
+    o = DynamicOracle(np.arange(n, dtype=np.uint64), src, dst, w)
+    xid, items, t = n - 1, 0, 0.0
+    for k in range(cycles):
+        rb = synth.dyn_record_batch(synth.seed_of("c3"), 1000 + k, xid, records, n_new=64, max_slice=2,
+                                    p_deleted=0.0, p_new=0.0005, p_invalid=0.0)
+        t0 = time.perf_counter()
+        o.apply_records(rb.records, rb.inserts, rb.weights, rb.deletes)
+        t += time.perf_counter() - t0
+        items += int(rb.records["ins_cnt"].sum() + rb.records["del_cnt"].sum())
+        xid += 64
+    return {"value": items / t, "unit": "updates/s", "cores": 1, "kind": "oracle",
+            "sample": f"O3 on RMAT-{scale} x16, {cycles} cycles of {records} records (edge-only), apply only"}
+
+
 def main():
     ap = argparse.ArgumentParser()
     ap.add_argument("--gpus", type=int, default=1)
@@ -463,7 +483,20 @@ def main():
                     help="N > 1: shard one graph (default) or run independent replicas")
     ap.add_argument("--dist-backend", default="nccl", choices=["nccl", "gloo"],
                     help="gloo lets several ranks share one GPU (testing)")
+    ap.add_argument("--replica", default="csr", choices=["csr", "dyn"],
+                    help="dyn: the dynamic hash-table replica (Algorithm 1; bench_dyn.py) on configs[2]'s graph")
+    import bench_dyn
+    bench_dyn.add_args(ap)
     args = ap.parse_args()
+    if args.replica == "dyn":
+        if args.impl != "h2tap" or args.gpus != 1:
+            raise SystemExit("--replica dyn: single GPU, own implementation only")
+        args.warmup = max(args.warmup, 3)
+        line = bench_dyn.measure(args)
+        if not args.no_cpu_baseline:
+            line["cpu_baseline"] = cpu_baseline_dyn()
+        print(json.dumps(line))
+        return
     if args.warmup < 3 and args.impl == "h2tap":
         args.warmup = 3
     if args.impl == "reference":

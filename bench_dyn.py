@@ -11,7 +11,8 @@ events (stats.ms_total) and CUDA events around the call.  Also timed: one CSR
 materialisation (h2tap_dyn_export to device buffers... here host arrays, reported apart).
 One JSON line; the round's copy lives in profiles/.
 
-usage: python bench_dyn.py [--scale 24] [--records 500000] [--cycles 5] [--node-deletes 0.0]
+usage: python bench.py --replica dyn [--scale 24] [--records 500000] [--cycles 5] [--node-deletes 0.0]
+       (adds the O3 cpu_baseline); python bench_dyn.py ... prints the GPU part alone
 """
 import argparse
 import json
@@ -26,17 +27,17 @@ sys.path.insert(0, ROOT)
 import synth  # noqa: E402
 
 
-def main():
-    import torch
-    import paper_conf_edbt_jibrilabs23_b200 as h2
-    ap = argparse.ArgumentParser()
+def add_args(ap):
     ap.add_argument("--scale", type=int, default=24)
     ap.add_argument("--records", type=int, default=500_000)
     ap.add_argument("--cycles", type=int, default=5)
-    ap.add_argument("--warmup", type=int, default=3)
     ap.add_argument("--node-deletes", type=float, default=0.0)
-    ap.add_argument("--no-cpu-baseline", action="store_true")
-    args = ap.parse_args()
+
+
+def measure(args) -> dict:
+    """GPU measurement only (no oracle here: `bench.py --replica dyn` adds the O3 cpu_baseline)."""
+    import torch
+    import paper_conf_edbt_jibrilabs23_b200 as h2
     torch.cuda.set_device(0)
     st = torch.cuda.current_stream()
     n = 1 << args.scale
@@ -144,29 +145,14 @@ def main():
                             "peak": peak, "unit": "GB/s", "frac": b / (t * 1e-3) / 1e9 / peak,
                             "traffic": None, "bytes_per_launch": b, "ms_per_launch": t,
                             "peak_source": "measured (MEASURED_PEAKS.json hbm_gbs)"}
-    if not args.no_cpu_baseline:
-        line["cpu_baseline"] = cpu_baseline()
-    print(json.dumps(line))
+    return line
 
 
-def cpu_baseline(scale: int = 16, records: int = 20000, cycles: int = 3):
-    """O3 (oracle/o3_dynamic.py, as it stands) on a bounded sample: an RMAT-16 graph and
-    20 K-record cycles of the same generator, timed on this host (one thread)."""
-    from oracle.o3_dynamic import DynamicOracle
-    n = 1 << scale
-    src, dst, w = synth.rmat_edges(scale, synth.seed_of("c3"), n=16 * n)
-    o = DynamicOracle(np.arange(n, dtype=np.uint64), src, dst, w)
-    xid, items, t = n - 1, 0, 0.0
-    for k in range(cycles):
-        rb = synth.dyn_record_batch(synth.seed_of("c3"), 1000 + k, xid, records, n_new=64, max_slice=2,
-                                    p_deleted=0.0, p_new=0.0005, p_invalid=0.0)
-        t0 = time.perf_counter()
-        o.apply_records(rb.records, rb.inserts, rb.weights, rb.deletes)
-        t += time.perf_counter() - t0
-        items += int(rb.records["ins_cnt"].sum() + rb.records["del_cnt"].sum())
-        xid += 64
-    return {"value": items / t, "unit": "updates/s", "cores": 1, "kind": "oracle",
-            "sample": f"O3 on RMAT-{scale} x16, {cycles} cycles of {records} records (edge-only), apply only"}
+def main():
+    ap = argparse.ArgumentParser()
+    add_args(ap)
+    ap.add_argument("--warmup", type=int, default=3)
+    print(json.dumps(measure(ap.parse_args())))
 
 
 if __name__ == "__main__":

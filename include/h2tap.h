@@ -361,6 +361,11 @@ h2tap_status h2tap_dyn_info(const h2tap_dyn* d, uint64_t* n_vertices, uint64_t* 
  * pointer may be NULL (skipped); host or device pointers (copied with cudaMemcpyDefault). */
 h2tap_status h2tap_dyn_export(h2tap_dyn* d, int64_t* offsets, uint32_t* cols, float* w,
         uint64_t* ext_ids, uint8_t* live);
+/* Freshness check on the dynamic replica (Table 1's BFS): materialise the CSR
+ * (as h2tap_dyn_export) and run the CSR path's level-synchronous BFS from the live vertex
+ * `source_ext`; level_out [n_vertices] (host or device) = hop count or -1 (unreachable or dead).
+ * Unknown / dead source -> E_INVAL. */
+h2tap_status h2tap_dyn_bfs(h2tap_dyn* d, uint64_t source_ext, int32_t* level_out);
 void h2tap_dyn_destroy(h2tap_dyn* d);
 
 void h2tap_replica_destroy(h2tap_replica* r);

@@ -519,6 +519,7 @@ for _n, _a, _r in (("h2tap_dyn_create", [ctypes.POINTER(_Config), ctypes.c_size_
                     ctypes.c_int),
                    ("h2tap_dyn_info", [_P] + [ctypes.POINTER(_u64)] * 3, ctypes.c_int),
                    ("h2tap_dyn_export", [_P, _P, _P, _P, _P, _P], ctypes.c_int),
+                   ("h2tap_dyn_bfs", [_P, _u64, _P], ctypes.c_int),
                    ("h2tap_dyn_destroy", [_P], None)):
     getattr(_lib, _n).restype = _r
     getattr(_lib, _n).argtypes = _a
@@ -582,6 +583,12 @@ class DynReplica:
         _check(_lib.h2tap_dyn_export(self._h, *[ctypes.c_void_p(a.ctypes.data) for a in out]),
                "h2tap_dyn_export")
         return out
+
+    def bfs(self, source_ext: int) -> np.ndarray:
+        """BFS levels (int32 per dense id, -1 unreachable / dead) from a live ext id."""
+        lv = np.empty(self.info()["n_vertices"], np.int32)
+        _check(_lib.h2tap_dyn_bfs(self._h, int(source_ext), ctypes.c_void_p(lv.ctypes.data)), "h2tap_dyn_bfs")
+        return lv
 
     def close(self):
         if getattr(self, "_h", None):

@@ -386,6 +386,13 @@ __global__ void k_dyn_offsets(const uint64_t* __restrict__ sk, uint64_t E, uint6
     }
     off[v] = (int64_t)lo;
 }
+// dense id + 1 of a live ext id into c->bad (0: none)
+__global__ void k_dyn_lookup(const uint64_t* __restrict__ ext, const uint32_t* __restrict__ live, uint64_t V,
+                             uint64_t x, Ctr* __restrict__ c) {
+    if (threadIdx.x) return;
+    const int64_t d = find_ext(ext, V, x);
+    c->bad = (d >= 0 && live[d]) ? (unsigned long long)d + 1 : 0;
+}
 __global__ void k_dyn_live_u8(const uint32_t* __restrict__ live, uint64_t V, uint8_t* __restrict__ out) {
     const uint64_t i = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x;
     if (i < V) out[i] = (uint8_t)live[i];
@@ -679,6 +686,39 @@ h2tap_status dyn_apply(h2tap_dyn* d, const h2tap_record_batch* b, h2tap_apply_st
     return H2TAP_OK;
 }
 
+// the CSR of the table (rows = dense ids, columns ascending) into caller-owned scratch Bufs
+h2tap_status dyn_materialise(h2tap_dyn* d, Buf& bo, Buf& bc, Buf& bw) {
+    h2tap_replica* r = d->r;
+    cudaStream_t st = r->st;
+    const uint64_t V = d->V, E = d->n_live;
+    dyn::Ctr* c = dyn_ctr_reset(d);
+    dyn_item_bufs(d, std::max<uint64_t>(E, 1));
+    uint64_t* k = static_cast<uint64_t*>(d->keys.p);
+    uint32_t* v = static_cast<uint32_t*>(d->vals.p);
+    uint64_t* k2 = static_cast<uint64_t*>(d->keys2.p);
+    uint32_t* v2 = static_cast<uint32_t*>(d->vals2.p);
+    float* cw = static_cast<float*>(d->witem.p);
+    if (d->cap) {
+        const unsigned grid = (unsigned)std::min<uint64_t>(g1(d->cap), (uint64_t)r->n_sm * 8);
+        dyn::k_dyn_compact<<<grid, 256, 0, st>>>(static_cast<uint64_t*>(d->hk.p), static_cast<float*>(d->hv.p),
+                                                 d->cap, V, k, v, cw, c);
+        CKL();
+    }
+    radix_sort(r, k, v, k2, v2, E, bits_for(V * V));
+    int64_t* o_off = r->get<int64_t>(bo, V + 1);
+    uint32_t* o_cols = r->get<uint32_t>(bc, E);
+    float* o_w = r->get<float>(bw, E);
+    if (E) { dyn::k_dyn_emit<<<g1(E), 256, 0, st>>>(k, v, cw, E, V, o_cols, o_w); CKL(); }
+    dyn::k_dyn_offsets<<<g1(V + 1), 256, 0, st>>>(k, E, V, o_off);
+    CKL();
+    dyn_ctr_read(d);
+    if (d->hctr->n_out != E) {
+        set_err("table holds %llu live keys, expected %llu", d->hctr->n_out, (unsigned long long)E);
+        return H2TAP_E_CUDA;
+    }
+    return H2TAP_OK;
+}
+
 }  // namespace
 
 extern "C" {
@@ -779,38 +819,66 @@ h2tap_status h2tap_dyn_export(h2tap_dyn* d, int64_t* offsets, uint32_t* cols, fl
         h2tap_replica* r = d->r;
         cudaStream_t st = r->st;
         const uint64_t V = d->V, E = d->n_live;
-        dyn::Ctr* c = dyn_ctr_reset(d);
-        dyn_item_bufs(d, std::max<uint64_t>(E, 1));
-        uint64_t* k = static_cast<uint64_t*>(d->keys.p);
-        uint32_t* v = static_cast<uint32_t*>(d->vals.p);
-        uint64_t* k2 = static_cast<uint64_t*>(d->keys2.p);
-        uint32_t* v2 = static_cast<uint32_t*>(d->vals2.p);
-        float* cw = static_cast<float*>(d->witem.p);
-        if (d->cap) {
-            const unsigned grid = (unsigned)std::min<uint64_t>(g1(d->cap), (uint64_t)r->n_sm * 8);
-            dyn::k_dyn_compact<<<grid, 256, 0, st>>>(static_cast<uint64_t*>(d->hk.p), static_cast<float*>(d->hv.p),
-                                                     d->cap, V, k, v, cw, c);
-            CKL();
-        }
-        radix_sort(r, k, v, k2, v2, E, bits_for(V * V));
         Buf bo, bc, bw, bl;
-        int64_t* o_off = r->get<int64_t>(bo, V + 1);
-        uint32_t* o_cols = r->get<uint32_t>(bc, E);
-        float* o_w = r->get<float>(bw, E);
+        const h2tap_status s = dyn_materialise(d, bo, bc, bw);
+        if (s != H2TAP_OK) return s;
         uint8_t* o_live = r->get<uint8_t>(bl, V);
-        if (E) { dyn::k_dyn_emit<<<g1(E), 256, 0, st>>>(k, v, cw, E, V, o_cols, o_w); CKL(); }
-        dyn::k_dyn_offsets<<<g1(V + 1), 256, 0, st>>>(k, E, V, o_off);
-        CKL();
         if (V) { dyn::k_dyn_live_u8<<<g1(V), 256, 0, st>>>(static_cast<uint32_t*>(d->live.p), V, o_live); CKL(); }
-        if (offsets) CK(cudaMemcpyAsync(offsets, o_off, (V + 1) * 8, cudaMemcpyDefault, st));
-        if (cols && E) CK(cudaMemcpyAsync(cols, o_cols, E * 4, cudaMemcpyDefault, st));
-        if (w && E) CK(cudaMemcpyAsync(w, o_w, E * 4, cudaMemcpyDefault, st));
+        if (offsets) CK(cudaMemcpyAsync(offsets, bo.p, (V + 1) * 8, cudaMemcpyDefault, st));
+        if (cols && E) CK(cudaMemcpyAsync(cols, bc.p, E * 4, cudaMemcpyDefault, st));
+        if (w && E) CK(cudaMemcpyAsync(w, bw.p, E * 4, cudaMemcpyDefault, st));
         if (ext_ids && V) CK(cudaMemcpyAsync(ext_ids, d->ext.p, V * 8, cudaMemcpyDefault, st));
         if (live && V) CK(cudaMemcpyAsync(live, o_live, V, cudaMemcpyDefault, st));
-        dyn_ctr_read(d);
-        if (d->hctr->n_out != E) { set_err("table holds %llu live keys, expected %llu", d->hctr->n_out, (unsigned long long)E); return H2TAP_E_CUDA; }
-        r->release(bo); r->release(bc); r->release(bw); r->release(bl);
         r->sync();
+        r->release(bo); r->release(bc); r->release(bw); r->release(bl);
+        return H2TAP_OK;
+    });
+}
+
+h2tap_status h2tap_dyn_bfs(h2tap_dyn* d, uint64_t source_ext, int32_t* level_out) {
+    if (!d || !level_out) { set_err("null argument"); return H2TAP_E_INVAL; }
+    return run_guarded(d->r, [&]() -> h2tap_status {
+        h2tap_replica* r = d->r;
+        cudaStream_t st = r->st;
+        const uint64_t V = d->V;
+        const uint64_t* ext = static_cast<const uint64_t*>(d->ext.p);
+        // source: dense id of a live vertex (host binary search over a copy is avoided:
+        // one device lookup through the counters block)
+        dyn::Ctr* c = dyn_ctr_reset(d);
+        dyn::k_dyn_lookup<<<1, 32, 0, st>>>(ext, static_cast<const uint32_t*>(d->live.p), V, source_ext, c);
+        CKL();
+        dyn_ctr_read(d);
+        if (!d->hctr->bad) { set_err("BFS source %llu is not a live vertex", (unsigned long long)source_ext); return H2TAP_E_INVAL; }
+        const uint64_t src = d->hctr->bad - 1;
+        Buf bo, bc, bw, bl, fa_, fb_;
+        const h2tap_status s = dyn_materialise(d, bo, bc, bw);
+        if (s != H2TAP_OK) return s;
+        int32_t* level = r->get<int32_t>(bl, V);
+        uint32_t* fa = r->get<uint32_t>(fa_, V);
+        uint32_t* fb = r->get<uint32_t>(fb_, V);
+        unsigned long long* cnt = r->get<unsigned long long>(r->misc, 1);
+        k_fill_i32<<<g1(V), 256, 0, st>>>(level, V, -1);
+        CKL();
+        int32_t zero = 0;
+        uint32_t s32 = (uint32_t)src;
+        CK(cudaMemcpyAsync(level + src, &zero, 4, cudaMemcpyHostToDevice, st));
+        CK(cudaMemcpyAsync(fa, &s32, 4, cudaMemcpyHostToDevice, st));
+        uint64_t nf = 1;
+        for (int32_t depth = 0; nf; ++depth) {   // the CSR path's level-synchronous expansion
+            CK(cudaMemsetAsync(cnt, 0, 8, st));
+            const unsigned grid = (unsigned)std::min<uint64_t>(cdiv(nf * 32, 256), 148 * 32);
+            k_bfs_expand<<<grid, 256, 0, st>>>(static_cast<const int64_t*>(bo.p), static_cast<const uint32_t*>(bc.p),
+                                               fa, nf, level, depth, fb, cnt);
+            CKL();
+            unsigned long long h = 0;
+            CK(cudaMemcpyAsync(&h, cnt, 8, cudaMemcpyDeviceToHost, st));
+            r->sync();
+            nf = h;
+            std::swap(fa, fb);
+        }
+        CK(cudaMemcpyAsync(level_out, level, V * 4, cudaMemcpyDefault, st));
+        r->sync();
+        for (Buf* b : {&bo, &bc, &bw, &bl, &fa_, &fb_}) r->release(*b);
         return H2TAP_OK;
     });
 }

@@ -66,6 +66,33 @@ def test_small_random_cycles(h2, seed):
         cycle(g, o, rb, f"seed {seed} cycle {cyc}")
 
 
+def test_bfs_after_cycles(h2):
+    """h2tap_dyn_bfs vs the oracle's BFS (oracle.bfs) on O3's export, after cycles with node
+    deletes (dead vertices: level -1)."""
+    import oracle
+    rng = np.random.default_rng(3)
+    n = 3000
+    ids = np.arange(n, dtype=np.uint64) * 5
+    m = 12000
+    g, o = pair(h2, ids, ids[rng.integers(0, n, m)], ids[rng.integers(0, n, m)], rng.random(m))
+    for cyc in range(3):
+        xid = int(o.ids[-1])
+        rb = synth.dyn_record_batch(21, cyc, xid, 800, n_new=40, max_slice=6, p_deleted=0.02)
+        rb.records["node"] = np.where(rb.records["node"] <= xid, ids[(rb.records["node"] % n).astype(np.int64)],
+                                      rb.records["node"])
+        rb = synth.RecordBatch(rb.records, np.where(rb.inserts <= xid, ids[(rb.inserts % n).astype(np.int64)],
+                                                    rb.inserts), rb.weights,
+                               ids[(rb.deletes % n).astype(np.int64)])
+        cycle(g, o, rb, f"bfs cycle {cyc}")
+    off, cols, _, ext, live = o.export()
+    for s_dense in np.flatnonzero(live)[:5]:
+        assert np.array_equal(g.bfs(int(ext[s_dense])), oracle.bfs(off, cols, int(s_dense)))
+    dead = np.flatnonzero(live == 0)
+    if len(dead):
+        with pytest.raises(Exception):
+            g.bfs(int(ext[dead[0]]))
+
+
 def test_multi_tile_cycles_with_rehash_and_device_inputs(h2):
     import torch
     rng = np.random.default_rng(7)

@@ -66,3 +66,9 @@ def test_product_package_does_not_touch_the_oracle():
                 src = open(os.path.join(dirpath, f)).read()
                 assert "import oracle" not in src and "from oracle" not in src, f
                 assert "o1_replay" not in src and "liboracle" not in src, f
+
+
+def test_bench_dyn_gpu_measurement_does_not_touch_the_oracle():
+    # only bench.py's cpu_baseline leg may run oracle/ code; bench_dyn.py is its GPU part
+    src = open(os.path.join(ROOT, "bench_dyn.py")).read()
+    assert "import oracle" not in src and "from oracle" not in src

@@ -13,7 +13,7 @@
 // One cycle (h2tap_dyn_apply_records), all on the replica stream:
 //   k_dyn_rec        classify records (lines 2-9): deletion / new-node queues, per-record
 //                    insert / delete item counts (+ record validation)
-//   scans            item offsets (k_scan_exclusive_u64)
+//   scan             item offsets, inserts and deletes packed in one u64 (k_scan_exclusive_u64)
 //   new nodes        radix sort of the new IDs, k_dyn_kill (created and deleted in the same
 //                    cycle: D3), k_dyn_heads + scan + k_dyn_append (line 10)
 //   k_dyn_expand_ins thread per record (warp per large record): resolve endpoints, gate (D2), pack keys
@@ -30,7 +30,7 @@ constexpr uint64_t kEmpty = ~0ull, kTomb = ~0ull - 1;
 constexpr uint32_t kFilterBits = 1u << 18;   // cascade filter: 32 KB of shared memory
 
 struct Ctr {
-    unsigned long long n_new_ids, n_del_ids, bad, max_new, n_new, n_upd, n_del, n_casc, n_gated, n_vdel, n_out, last_ext, n_big_ins, n_big_del;
+    unsigned long long n_new_ids, n_del_ids, bad, max_new, n_new, n_upd, n_del, n_casc, n_gated, n_vdel, n_out, last_ext, n_big_ins, n_big_del, sum_ins, sum_del;
 };
 
 __device__ __forceinline__ uint64_t hmix(uint64_t k) {
@@ -55,32 +55,39 @@ __device__ __forceinline__ void wadd(unsigned long long* c, bool pred) {  // war
 
 // Alg. 1 lines 2-9 per record
 __global__ void k_dyn_rec(const DeltaRec* __restrict__ rec, uint64_t nr, uint64_t n_ins, uint64_t n_del,
-                          uint64_t xid, int has_xid, uint64_t* __restrict__ cnt_ins, uint64_t* __restrict__ cnt_del,
+                          uint64_t xid, int has_xid, uint64_t* __restrict__ cnt,
                           uint64_t* __restrict__ new_ids, uint64_t* __restrict__ del_ids, Ctr* __restrict__ c) {
     const uint64_t i = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x;
-    if (i > nr) return;
-    if (i == nr) { cnt_ins[nr] = 0; cnt_del[nr] = 0; return; }
-    const DeltaRec r = rec[i];
     uint64_t ci = 0, cd = 0;
     unsigned bad = 0;
-    if (r.valid > 1 || r.deleted > 1 || r.inserted > 1) bad |= REC_BAD_FLAG;
-    if (r.valid) {
-        if (r.ins_off > n_ins || r.ins_cnt > n_ins - r.ins_off || r.del_off > n_del || r.del_cnt > n_del - r.del_off)
-            bad |= REC_BAD_SLICE;
-        if (r.deleted) {                                       // lines 3-4
-            del_ids[atomicAdd(&c->n_del_ids, 1ull)] = r.node;
-        } else if (has_xid && r.node <= xid) {                // lines 5-7
-            ci = r.ins_cnt;
-            cd = r.del_cnt;
-        } else {                                               // line 9 (D5: its deletes ignored)
-            new_ids[atomicAdd(&c->n_new_ids, 1ull)] = r.node;
-            atomicMax(&c->max_new, (unsigned long long)r.node);
-            ci = r.ins_cnt;
+    if (i < nr) {
+        const DeltaRec r = rec[i];
+        if (r.valid > 1 || r.deleted > 1 || r.inserted > 1) bad |= REC_BAD_FLAG;
+        if (r.valid) {
+            if (r.ins_off > n_ins || r.ins_cnt > n_ins - r.ins_off || r.del_off > n_del || r.del_cnt > n_del - r.del_off)
+                bad |= REC_BAD_SLICE;
+            if (r.deleted) {                                       // lines 3-4
+                del_ids[atomicAdd(&c->n_del_ids, 1ull)] = r.node;
+            } else if (has_xid && r.node <= xid) {                // lines 5-7
+                ci = r.ins_cnt;
+                cd = r.del_cnt;
+            } else {                                               // line 9 (D5: its deletes ignored)
+                new_ids[atomicAdd(&c->n_new_ids, 1ull)] = r.node;
+                atomicMax(&c->max_new, (unsigned long long)r.node);
+                ci = r.ins_cnt;
+            }
         }
+        if (bad) atomicOr(&c->bad, (unsigned long long)bad);
+        cnt[i] = ci << 32 | cd;   // packed insert / delete item counts (one scan places both)
+    } else if (i == nr) {
+        cnt[nr] = 0;
     }
-    if (bad) atomicOr(&c->bad, (unsigned long long)bad);
-    cnt_ins[i] = ci;
-    cnt_del[i] = cd;
+    // exact totals: the packed scan is carry-free iff the delete total is < 2^32 (host check)
+    const unsigned long long si = warp_sum<unsigned long long>(ci), sd = warp_sum<unsigned long long>(cd);
+    if ((threadIdx.x & 31) == 0) {
+        if (si) atomicAdd(&c->sum_ins, si);
+        if (sd) atomicAdd(&c->sum_del, sd);
+    }
 }
 
 // a new ID the cycle also deletes is never inserted (D3): flag its first copy in the sorted list
@@ -145,7 +152,7 @@ __global__ void __launch_bounds__(256) k_dyn_expand_ins(const DeltaRec* __restri
     if (kPass == 0) {
         const uint64_t i = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x;
         if (i < nr) {
-            const uint64_t o = off[i], n = off[i + 1] - o;
+            const uint64_t o = off[i] >> 32, n = (off[i + 1] >> 32) - o;
             if (n > kSmall) big[atomicAdd(n_big, 1ull)] = i;
             else if (n) {
                 const DeltaRec r = rec[i];
@@ -157,7 +164,7 @@ __global__ void __launch_bounds__(256) k_dyn_expand_ins(const DeltaRec* __restri
         const uint64_t nb = *n_big, nw = (uint64_t)gridDim.x * (blockDim.x >> 5);
         const unsigned lane = threadIdx.x & 31;
         for (uint64_t q = blockIdx.x * (uint64_t)(blockDim.x >> 5) + (threadIdx.x >> 5); q < nb; q += nw) {
-            const uint64_t i = big[q], o = off[i], n = off[i + 1] - o;
+            const uint64_t i = big[q], o = off[i] >> 32, n = (off[i + 1] >> 32) - o;
             int64_t s = lane == 0 ? live_src(ext, live, V, rec[i].node) : -1;
             s = __shfl_sync(0xffffffffu, s, 0);
             const uint64_t io = rec[i].ins_off;
@@ -224,7 +231,7 @@ __global__ void __launch_bounds__(256) k_dyn_delete(const DeltaRec* __restrict__
     if (kPass == 0) {
         const uint64_t i = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x;
         if (i < nr) {
-            const uint64_t n = off[i + 1] - off[i];
+            const uint64_t n = (off[i + 1] & 0xffffffffu) - (off[i] & 0xffffffffu);
             if (n > kSmall) big[atomicAdd(n_big, 1ull)] = i;
             else if (n) {
                 const DeltaRec r = rec[i];
@@ -237,7 +244,7 @@ __global__ void __launch_bounds__(256) k_dyn_delete(const DeltaRec* __restrict__
         const uint64_t nb = *n_big, nw = (uint64_t)gridDim.x * (blockDim.x >> 5);
         const unsigned lane = threadIdx.x & 31;
         for (uint64_t q = blockIdx.x * (uint64_t)(blockDim.x >> 5) + (threadIdx.x >> 5); q < nb; q += nw) {
-            const uint64_t i = big[q], n = off[i + 1] - off[i];
+            const uint64_t i = big[q], n = (off[i + 1] & 0xffffffffu) - (off[i] & 0xffffffffu);
             int64_t s = lane == 0 ? find_ext(ext, V, rec[i].node) : -1;
             s = __shfl_sync(0xffffffffu, s, 0);
             if (s < 0) continue;
@@ -404,7 +411,7 @@ struct h2tap_dyn {
     h2tap_replica* r = nullptr;   // stream, allocator, radix-sort scratch
     uint64_t V = 0, n_live = 0, n_tomb = 0, cap = 0, xid = 0;   // xid = ext[V - 1] (host copy)
     Buf ext, live, hk, hv, died, big;
-    Buf cin, cdel, oin, odel, new_ids, del_ids, kill, flag, fpos, keys, vals, keys2, vals2, witem, ctr, xo;
+    Buf cin, oin, new_ids, del_ids, kill, flag, fpos, keys, vals, keys2, vals2, witem, ctr, xo;
     Buf x_rec, x_ins, x_wts, x_del;
     dyn::Ctr* hctr = nullptr;     // pinned host mirror
 };
@@ -414,7 +421,7 @@ namespace {
 void dyn_free(h2tap_dyn* d) {
     if (!d) return;
     if (d->r) {
-        for (Buf* b : {&d->ext, &d->live, &d->died, &d->big, &d->hk, &d->hv, &d->cin, &d->cdel, &d->oin, &d->odel, &d->new_ids,
+        for (Buf* b : {&d->ext, &d->live, &d->died, &d->big, &d->hk, &d->hv, &d->cin, &d->oin, &d->new_ids,
                        &d->del_ids, &d->kill, &d->flag, &d->fpos, &d->keys, &d->vals, &d->keys2, &d->vals2,
                        &d->witem, &d->ctr, &d->xo, &d->x_rec, &d->x_ins, &d->x_wts, &d->x_del})
             if (b->p) d->r->dfree(b->p);
@@ -535,13 +542,16 @@ h2tap_status dyn_apply(h2tap_dyn* d, const h2tap_record_batch* b, h2tap_apply_st
     // ---- lines 1-9: classify records
     const uint64_t xid = d->xid;
     dyn::Ctr* c = dyn_ctr_reset(d);
-    uint64_t* cin = r->get<uint64_t>(d->cin, nr + 1);
-    uint64_t* cdel = r->get<uint64_t>(d->cdel, nr + 1);
-    uint64_t* oin = r->get<uint64_t>(d->oin, nr + 1);
-    uint64_t* odel = r->get<uint64_t>(d->odel, nr + 1);
+    if (b->n_inserts >= (1ull << 32) || b->n_deletes >= (1ull << 32)) {
+        set_err("inserts / deletes arrays of 2^32 or more entries");
+        return H2TAP_E_CAPACITY;
+    }
+    uint64_t* cnt = r->get<uint64_t>(d->cin, nr + 1);
+    uint64_t* oin = r->get<uint64_t>(d->oin, nr + 1);   // packed exclusive offsets (ins << 32 | del)
+    uint64_t* odel = oin;
     uint64_t* new_ids = r->get<uint64_t>(d->new_ids, nr);
     uint64_t* del_ids = r->get<uint64_t>(d->del_ids, nr);
-    dyn::k_dyn_rec<<<g1(nr + 1), 256, 0, st>>>(rec, nr, b->n_inserts, b->n_deletes, xid, d->V ? 1 : 0, cin, cdel,
+    dyn::k_dyn_rec<<<g1(nr + 1), 256, 0, st>>>(rec, nr, b->n_inserts, b->n_deletes, xid, d->V ? 1 : 0, cnt,
                                               new_ids, del_ids, c);
     CKL();
     {
@@ -550,23 +560,23 @@ h2tap_status dyn_apply(h2tap_dyn* d, const h2tap_record_batch* b, h2tap_apply_st
         unsigned int* sc = reinterpret_cast<unsigned int*>(r->get<uint64_t>(d->xo, 2));
         CK(cudaMemsetAsync(stt, 0, nt * 8, st));
         CK(cudaMemsetAsync(sc, 0, 4, st));
-        k_scan_exclusive_u64<<<(unsigned)nt, kThreads, 0, st>>>(cin, oin, n, stt, sc);
-        CKL();
-        CK(cudaMemsetAsync(stt, 0, nt * 8, st));
-        CK(cudaMemsetAsync(sc, 0, 4, st));
-        k_scan_exclusive_u64<<<(unsigned)nt, kThreads, 0, st>>>(cdel, odel, n, stt, sc);
+        k_scan_exclusive_u64<<<(unsigned)nt, kThreads, 0, st>>>(cnt, oin, n, stt, sc);
         CKL();
     }
-    uint64_t tot[2];
-    CK(cudaMemcpyAsync(&tot[0], oin + nr, 8, cudaMemcpyDeviceToHost, st));
-    CK(cudaMemcpyAsync(&tot[1], odel + nr, 8, cudaMemcpyDeviceToHost, st));
-    g_d2h += 16;
+    uint64_t packed_tot = 0, tot[2];
+    CK(cudaMemcpyAsync(&packed_tot, oin + nr, 8, cudaMemcpyDeviceToHost, st));
+    g_d2h += 8;
     dyn_ctr_read(d);
     const dyn::Ctr h0 = *d->hctr;
+    if (!(h0.bad & (REC_BAD_FLAG | REC_BAD_SLICE)) && (h0.sum_ins >= (1ull << 32) || h0.sum_del >= (1ull << 32))) {
+        set_err("more than 2^32 - 1 inserted or deleted edges in one cycle");
+        return H2TAP_E_CAPACITY;
+    }
+    tot[0] = packed_tot >> 32;
+    tot[1] = packed_tot & 0xffffffffu;
     if (h0.bad & REC_BAD_FLAG) { set_err("delta record flag other than 0/1"); return H2TAP_E_INVAL; }
     if (h0.bad & REC_BAD_SLICE) { set_err("delta record slice outside the inserts/weights/deletes arrays"); return H2TAP_E_INVAL; }
     const uint64_t n_ins = tot[0];
-    if (n_ins >= (1ull << 32)) { set_err("more than 2^32 - 1 inserted edges in one cycle"); return H2TAP_E_CAPACITY; }
     // ---- line 10: new nodes (ascending, after every old id; D3)
     uint64_t n_vins = 0;
     const uint64_t u = h0.n_new_ids;

@@ -442,9 +442,9 @@ def run_gpu(args):
 
 
 def cpu_baseline_dyn(scale: int = 16, records: int = 20000, cycles: int = 3):
-    """cpu_baseline leg of --replica dyn: O3 (oracle/o3_dynamic.py, as it stands) on a bounded sample: an RMAT-16 graph and
+    """cpu_baseline leg of --replica dyn: OD (oracle/od_dynamic.py, as it stands) on a bounded sample: an RMAT-16 graph and
     20 K-record cycles of the same generator, timed on this host (one thread)."""
-    from oracle.o3_dynamic import DynamicOracle
+    from oracle.od_dynamic import DynamicOracle
     n = 1 << scale
     src, dst, w = synth.rmat_edges(scale, synth.seed_of("c3"), n=16 * n)
     o = DynamicOracle(np.arange(n, dtype=np.uint64), src, dst, w)
@@ -458,7 +458,7 @@ def cpu_baseline_dyn(scale: int = 16, records: int = 20000, cycles: int = 3):
         items += int(rb.records["ins_cnt"].sum() + rb.records["del_cnt"].sum())
         xid += 64
     return {"value": items / t, "unit": "updates/s", "cores": 1, "kind": "oracle",
-            "sample": f"O3 on RMAT-{scale} x16, {cycles} cycles of {records} records (edge-only), apply only"}
+            "sample": f"OD on RMAT-{scale} x16, {cycles} cycles of {records} records (edge-only), apply only"}
 
 
 def main():

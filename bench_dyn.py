@@ -12,7 +12,7 @@ materialisation (h2tap_dyn_export to device buffers... here host arrays, reporte
 One JSON line; the round's copy lives in profiles/.
 
 usage: python bench.py --replica dyn [--scale 24] [--records 500000] [--cycles 5] [--node-deletes 0.0]
-       (adds the O3 cpu_baseline); python bench_dyn.py ... prints the GPU part alone
+       (adds the OD cpu_baseline); python bench_dyn.py ... prints the GPU part alone
 """
 import argparse
 import json
@@ -35,7 +35,7 @@ def add_args(ap):
 
 
 def measure(args) -> dict:
-    """GPU measurement only (no oracle here: `bench.py --replica dyn` adds the O3 cpu_baseline)."""
+    """GPU measurement only (no oracle here: `bench.py --replica dyn` adds the OD cpu_baseline)."""
     import torch
     import paper_conf_edbt_jibrilabs23_b200 as h2
     torch.cuda.set_device(0)

@@ -12,6 +12,11 @@ input generator ``synth``, which holds none of the method's arithmetic).
   by their textbook definitions.
 * ``O2``  (o2_bruteforce.py): independent brute force on a flat edge list,
   used to pin O1 on exhaustive tiny cases.
+* ``O3``  (o3_alg2.cpp): the paper's own method on the host - a flat CSR
+  updated by Algorithm 2 + merge(), 1 thread or OpenMP; pinned
+  bit-exact to O1 and used as the whole-export checksum reference at full
+  size and as the CPU baseline.
+* ``OD``  (od_dynamic.py): the dynamic replica's update (Algorithm 1).
 * ``expand_records``: the delta-store scan of the paper's record layout
   (§5.1-5.2) into the flat op sequence O1 replays.
 * ``checksum``: position-keyed 64-bit checksum of an exported array (the
@@ -31,6 +36,8 @@ from .o2_bruteforce import BruteForce  # noqa: F401
 _HERE = os.path.dirname(os.path.abspath(__file__))
 _SRC = os.path.join(_HERE, "o1_replay.cpp")
 _LIB = os.path.join(_HERE, "liboracle.so")
+_SRC3 = os.path.join(_HERE, "o3_alg2.cpp")
+_LIB3 = os.path.join(_HERE, "libo3.so")
 
 OK, E_INVAL, E_STALE_TS, E_SNAPSHOT_REGRESSION = 0, -1, -5, -6
 
@@ -38,6 +45,9 @@ OK, E_INVAL, E_STALE_TS, E_SNAPSHOT_REGRESSION = 0, -1, -5, -6
 def build(force: bool = False) -> str:
     if force or not os.path.exists(_LIB) or os.path.getmtime(_LIB) < os.path.getmtime(_SRC):
         subprocess.check_call(["g++", "-O2", "-std=c++17", "-fPIC", "-shared", "-o", _LIB, _SRC])
+    if force or not os.path.exists(_LIB3) or os.path.getmtime(_LIB3) < os.path.getmtime(_SRC3):
+        subprocess.check_call(["g++", "-O2", "-std=c++17", "-fopenmp", "-fPIC", "-shared", "-o", _LIB3,
+                               _SRC3])
     return _LIB
 
 
@@ -152,6 +162,88 @@ class O1:
                                         np.uint64)]
         lib().o1_pending(self.h, *(_p(x) for x in a))
         return a
+
+
+_lib3 = None
+
+
+def lib3():
+    global _lib3
+    if _lib3 is None:
+        build()
+        L = ctypes.CDLL(_LIB3)
+        P, u64 = ctypes.c_void_p, ctypes.c_uint64
+        L.o3_new.restype = P
+        L.o3_new.argtypes = [u64]
+        L.o3_destroy.argtypes = [P]
+        L.o3_set_threads.argtypes = [ctypes.c_int]
+        L.o3_max_threads.restype = ctypes.c_int
+        L.o3_create_edges.restype = ctypes.c_int
+        L.o3_create_edges.argtypes = [P, u64, P, u64, P, P, P]
+        L.o3_apply.restype = ctypes.c_int
+        L.o3_apply.argtypes = [P, u64, P, P, P, P, P, u64, ctypes.POINTER(_Stats)]
+        L.o3_info.argtypes = [P, P, P, P, P]
+        L.o3_export.argtypes = [P, P, P, P, P]
+        L.o3_checksums.argtypes = [P, P]
+        _lib3 = L
+    return _lib3
+
+
+def set_threads(n: int = 0) -> int:
+    """OpenMP threads O3 uses (0 = every host thread); returns the count in effect."""
+    lib3().o3_set_threads(int(n))
+    return lib3().o3_max_threads()
+
+
+class O3:
+    """Algorithm-2 flat-CSR merge on the host (oracle/o3_alg2.cpp)."""
+
+    def __init__(self, create_ts: int = 0):
+        self.h = lib3().o3_new(create_ts)
+
+    def __del__(self):
+        if getattr(self, "h", None):
+            lib3().o3_destroy(self.h)
+            self.h = None
+
+    @staticmethod
+    def from_edges(n_vertices, vertex_ids, src, dst, w, create_ts=0) -> "O3":
+        g = O3(create_ts)
+        ids = _c(vertex_ids, np.uint64)
+        src, dst, w = _c(src, np.uint64), _c(dst, np.uint64), _c(w, np.float32)
+        rc = lib3().o3_create_edges(g.h, n_vertices, _p(ids), len(src), _p(src), _p(dst), _p(w))
+        if rc != OK:
+            raise ValueError(f"o3_create_edges: {rc}")
+        return g
+
+    def apply(self, batch, snapshot_ts: int):
+        k = _c(batch.kind, np.uint8)
+        s, d = _c(batch.src, np.uint64), _c(batch.dst, np.uint64)
+        w, t = _c(batch.w, np.float32), _c(batch.ts, np.uint64)
+        st = _Stats()
+        rc = lib3().o3_apply(self.h, len(k), _p(k), _p(s), _p(d), _p(w), _p(t), snapshot_ts,
+                             ctypes.byref(st))
+        return rc, {"n_visible": st.n_visible, "n_deferred": st.n_deferred}
+
+    def info(self):
+        v = [ctypes.c_uint64() for _ in range(4)]
+        lib3().o3_info(self.h, *(ctypes.byref(x) for x in v))
+        return dict(n_vertices=v[0].value, n_edges=v[1].value, snapshot_ts=v[2].value,
+                    n_pending=v[3].value)
+
+    def export(self):
+        inf = self.info()
+        off = np.empty(inf["n_vertices"] + 1, np.int64)
+        cols = np.empty(inf["n_edges"], np.uint32)
+        w = np.empty(inf["n_edges"], np.float32)
+        ids = np.empty(inf["n_vertices"], np.uint64)
+        lib3().o3_export(self.h, _p(off), _p(cols), _p(w), _p(ids))
+        return off, cols, w, ids
+
+    def checksums(self):
+        out = np.zeros(4, np.uint64)
+        lib3().o3_checksums(self.h, _p(out))
+        return [int(x) for x in out]
 
 
 def expand_records(records, inserts, weights, deletes):

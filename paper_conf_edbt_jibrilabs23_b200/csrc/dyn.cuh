@@ -4,7 +4,7 @@
 //
 // Storage: one open-addressing table over packed edge keys
 //   key = src_dense << 32 | dst_dense  (u64; EMPTY = ~0, TOMB = ~0 - 1), value f32
-// linear probing from fmix64(key), load (live + tombstones) <= 1/2 (re-hashed into a table of
+// linear probing from fmix64(key), load (live + tombstones) <= 0.7 (re-hashed into a table of
 // twice the needed size when a cycle would pass it); inserts only ever claim EMPTY slots, so a
 // CAS on the key word is the whole synchronisation.  Vertices: ext ids ascending (new IDs are
 // > xid, Alg. 1 line 5/8, so they append) and a u32 liveness word per dense id (D3: dense ids
@@ -82,7 +82,8 @@ __global__ void k_dyn_rec(const DeltaRec* __restrict__ rec, uint64_t nr, uint64_
     } else if (i == nr) {
         cnt[nr] = 0;
     }
-    // exact totals: the packed scan is carry-free iff the delete total is < 2^32 (host check)
+    // exact totals: the packed scan is carry-free iff the insert total is < 2^30 and the delete
+    // total < 2^32 (host check after the scan, before anything reads its output)
     const unsigned long long si = warp_sum<unsigned long long>(ci), sd = warp_sum<unsigned long long>(cd);
     if ((threadIdx.x & 31) == 0) {
         if (si) atomicAdd(&c->sum_ins, si);
@@ -568,8 +569,18 @@ h2tap_status dyn_apply(h2tap_dyn* d, const h2tap_record_batch* b, h2tap_apply_st
     g_d2h += 8;
     dyn_ctr_read(d);
     const dyn::Ctr h0 = *d->hctr;
-    if (!(h0.bad & (REC_BAD_FLAG | REC_BAD_SLICE)) && (h0.sum_ins >= (1ull << 32) || h0.sum_del >= (1ull << 32))) {
-        set_err("more than 2^32 - 1 inserted or deleted edges in one cycle");
+    // The packed scan is carry-free only while every prefix fits its field: deletes in the
+    // low 32 bits, inserts in bits 32..61 (the look-back status word keeps its flag in bits
+    // 62-63 and masks values to 62 bits, dev_common.cuh), hence sum_ins < 2^30.  Nothing
+    // has read the packed offsets yet, so refusing here leaves the replica unchanged.
+    if (!(h0.bad & (REC_BAD_FLAG | REC_BAD_SLICE)) && (h0.sum_ins >= (1ull << 30) || h0.sum_del >= (1ull << 32))) {
+        set_err("%llu inserted / %llu deleted edge items in one cycle (limits 2^30 - 1 / 2^32 - 1)",
+                (unsigned long long)h0.sum_ins, (unsigned long long)h0.sum_del);
+        return H2TAP_E_CAPACITY;
+    }
+    if (d->n_live + h0.sum_ins >= 0xFFFFFFFFull) {  // the materialised CSR keys edges by u32 position
+        set_err("live edges (%llu) + inserted items (%llu) would reach 2^32 - 1",
+                (unsigned long long)d->n_live, (unsigned long long)h0.sum_ins);
         return H2TAP_E_CAPACITY;
     }
     tot[0] = packed_tot >> 32;

@@ -1242,6 +1242,9 @@ h2tap_status h2tap_batch_stage(h2tap_replica* r, const h2tap_batch* host, h2tap_
         auto& g = r->stg[r->stg_next];
         r->stg_next ^= 1;
         const uint64_t n = host->n;
+        // the slot's previous copy (a staged batch that was never applied) may still be
+        // running: wait for it before get() can free and re-allocate the slot's buffers
+        CK(cudaEventSynchronize(g.ev));
         uint8_t* k = r->get<uint8_t>(g.k, n);
         uint64_t* s = r->get<uint64_t>(g.s, n);
         uint64_t* d = r->get<uint64_t>(g.d, n);

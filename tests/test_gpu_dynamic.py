@@ -1,12 +1,12 @@
 """Parity of the dynamic replica (h2tap_dyn_*: Algorithm 1, §5.4) with
-O3 (oracle/o3_dynamic.py, pinned in tests/test_oracle_pins_dyn.py).  Bar: bit-exact
+OD (oracle/od_dynamic.py, pinned in tests/test_oracle_pins_dyn.py).  Bar: bit-exact
 offsets / cols / weights / ext ids / liveness and equal counters after every cycle
 (integer work; the weights are copied, never computed)."""
 import numpy as np
 import pytest
 
 import synth
-from oracle.o3_dynamic import DynamicOracle
+from oracle.od_dynamic import DynamicOracle
 
 pytestmark = pytest.mark.gpu
 
@@ -67,7 +67,7 @@ def test_small_random_cycles(h2, seed):
 
 
 def test_bfs_after_cycles(h2):
-    """h2tap_dyn_bfs vs the oracle's BFS (oracle.bfs) on O3's export, after cycles with node
+    """h2tap_dyn_bfs vs the oracle's BFS (oracle.bfs) on OD's export, after cycles with node
     deletes (dead vertices: level -1)."""
     import oracle
     rng = np.random.default_rng(3)
@@ -178,7 +178,7 @@ def test_empty_graph_and_empty_cycle(h2):
 def test_full_size_sampled_rows(h2):
     """bench_dyn.py's workload (configs[2]'s RMAT-24 graph, 500 K records with node deletes and
     new nodes, device-resident): ext ids and liveness compared in full, the rows of 256 sampled
-    sources (+ every node-delete victim's row) against O3 run on the sub-problem that decides
+    sources (+ every node-delete victim's row) against OD run on the sub-problem that decides
     them (all vertices, the sampled sources' edges, the records of those sources, every
     deletion and every new node: no other record can touch those rows)."""
     import torch

@@ -475,3 +475,45 @@ def test_tombstone_equals_compaction_of_the_live_part():
             if not live.all():   # tombstones keep their rows' slot, empty
                 off = t.export()[0]
                 assert np.all(np.diff(off)[live == 0] == 0)
+
+
+def test_from_csr_round_trip_and_continuation():
+    """O1.from_csr (the checkpoint/restore direction of create): loading an
+    exported CSR reproduces it exactly, and the restored replica continues exactly like the
+    original under further batches; a CSR over sparse external IDs keeps them."""
+    for seed in range(6):
+        rng = np.random.default_rng(seed)
+        ids = np.unique(rng.integers(0, 500, 60).astype(np.uint64))
+        src, dst = ids[rng.integers(0, len(ids), 300)], ids[rng.integers(0, len(ids), 300)]
+        w = rng.random(300).astype(np.float32)
+        a = O1.from_edges(len(ids), ids, src, dst, w, 4)
+        off, cols, ww, got = a.export()
+        b = O1.from_csr(off, cols, ww, got, 4)
+        assert same_export(b.export(), (off, cols, ww, got))
+        for k in range(3):
+            bt = synth.fuzz_batch(seed=seed, k=k, n=80, n_ids=600, ts_lo=5 + 10 * k, ts_span=10)
+            assert a.apply(bt, 14 + 10 * k)[0] == b.apply(bt, 14 + 10 * k)[0] == 0
+            assert same_export(a.export(), b.export())
+    # identity ids: ext_ids = None means row i is vertex i
+    c = O1.from_csr(np.array([0, 2, 2, 3], np.int64), np.array([1, 2, 0], np.uint32), np.ones(3, np.float32))
+    assert c.export()[3].tolist() == [0, 1, 2] and c.export()[1].tolist() == [1, 2, 0]
+
+
+def test_pending_is_the_invisible_ops_in_arrival_order():
+    """O1.pending: the ops not yet visible (ts > snapshot_ts, reading A6), in
+    arrival order, each with its arrival number seq (reading A5); an op leaves the pending
+    set in the cycle whose snapshot reaches its ts (each delta is used once)."""
+    o = O1.from_edges(4, None, np.array([0], np.uint64), np.array([1], np.uint64), np.ones(1, np.float32))
+    b1 = Batch.of([(EDGE_INSERT, 1, 2, 1.0, 5), (EDGE_INSERT, 2, 3, 2.0, 9), (EDGE_DELETE, 0, 1, 0.0, 3),
+                   (EDGE_WEIGHT, 1, 2, 4.0, 12)])
+    assert o.apply(b1, 6)[0] == 0
+    k, s, d, w, t, q = o.pending()
+    assert t.tolist() == [9, 12] and q.tolist() == [1, 3] and k.tolist() == [EDGE_INSERT, EDGE_WEIGHT]
+    assert s.tolist() == [2, 1] and d.tolist() == [3, 2] and w.tolist() == [2.0, 4.0]
+    b2 = Batch.of([(NODE_INSERT, 7, 0, 0.0, 11), (EDGE_INSERT, 7, 0, 1.0, 20)])
+    assert o.apply(b2, 11)[0] == 0
+    k, s, d, w, t, q = o.pending()
+    assert t.tolist() == [12, 20] and q.tolist() == [3, 5]   # 9 and 11 became visible
+    assert o.apply(Batch.of([]), 30)[0] == 0 and len(o.pending()[0]) == 0
+    off, cols, ww, ids = o.export()
+    assert ids.tolist() == [0, 1, 2, 3, 7] and cols.tolist() == [2, 3, 0] and ww.tolist() == [4.0, 2.0, 1.0]

@@ -1,4 +1,4 @@
-"""Pins for O3, the dynamic-replica oracle (Algorithm 1; readings D1-D5 of
+"""Pins for OD, the dynamic-replica oracle (Algorithm 1; readings D1-D5 of
 DESIGN.md §15), checked against things other than itself:
 
 * the paper's Fig. 2 worked example in its record layout (tests/golden/fig2_records.json,
@@ -12,7 +12,7 @@ import pytest
 
 import synth
 from oracle import O1
-from oracle.o3_dynamic import DynamicOracle, flat_ops
+from oracle.od_dynamic import DynamicOracle, flat_ops
 from synth import Batch
 from test_oracle_pins import load_fig2_records
 

@@ -51,6 +51,8 @@
 #include <omp.h>
 
 #include <algorithm>
+#include <cstdio>
+#include <cstdlib>
 #include <cstdint>
 #include <cstring>
 #include <map>
@@ -62,6 +64,19 @@ namespace {
 enum { OK = 0, E_INVAL = -1, E_STALE_TS = -5, E_SNAPSHOT_REGRESSION = -6 };
 enum { NODE_INSERT = 0, NODE_DELETE = 1, EDGE_INSERT = 2, EDGE_DELETE = 3, EDGE_WEIGHT = 4 };
 constexpr uint32_t kNone = 0xFFFFFFFFu;
+
+// O3_TRACE=1: wall time of each step on stderr (diagnostics only)
+struct Tr {
+    bool on = getenv("O3_TRACE") != nullptr;
+    double t = omp_get_wtime();
+    void operator()(const char* what) {
+        if (!on) return;
+        const double n = omp_get_wtime();
+        fprintf(stderr, "[o3] %s %.3f s\n", what, n - t);
+        t = n;
+    }
+};
+
 
 struct Op {
     uint8_t kind;
@@ -86,18 +101,34 @@ struct Csr {
     std::vector<float> w;
 };
 
+constexpr int kFenceShift = 6;  // every 64th external ID in a small (cache-resident) table
+
 struct Graph {
     uint64_t snap_ts = 0, next_seq = 0;
     std::vector<Op> pending;
     Csr g;
-    bool identity = true;  // ext[i] == i for all i (dense lookup without a search)
+    bool identity = true;         // ext[i] == i for all i (dense lookup without a search)
+    std::vector<uint64_t> fence;  // fence[j] = ext[64 j]
+    void index() {
+        const std::vector<uint64_t>& ext = g.ext;
+        identity = true;
+        for (uint64_t i = 0; i < ext.size() && identity; ++i) identity = ext[i] == i;
+        fence.clear();
+        for (uint64_t i = 0; i < ext.size(); i += 1u << kFenceShift) fence.push_back(ext[i]);
+    }
 };
 
+// dense ID of external ID x in the current CSR, -1 if absent: binary search of the
+// fence, then of the 64-ID block it selects
 int64_t dense_of(const Graph& G, uint64_t x) {
     const std::vector<uint64_t>& ext = G.g.ext;
     if (G.identity) return x < ext.size() ? (int64_t)x : -1;
-    auto it = std::lower_bound(ext.begin(), ext.end(), x);
-    return (it != ext.end() && *it == x) ? (int64_t)(it - ext.begin()) : -1;
+    auto f = std::upper_bound(G.fence.begin(), G.fence.end(), x);
+    if (f == G.fence.begin()) return -1;
+    const uint64_t b = (uint64_t)(f - G.fence.begin() - 1) << kFenceShift;
+    auto lo = ext.begin() + b, hi = ext.begin() + std::min<uint64_t>(ext.size(), b + (1u << kFenceShift));
+    auto it = std::lower_bound(lo, hi, x);
+    return (it != hi && *it == x) ? (int64_t)(it - ext.begin()) : -1;
 }
 
 bool old_edge(const Graph& G, int64_t u, int64_t v) {
@@ -186,6 +217,7 @@ struct Scan {
 
 // Algorithm 2 over the combined deltas: old CSR + deltas -> new CSR
 void alg2_merge(Graph& G, Scan& S) {
+    Tr tr;
     const Csr& o = G.g;
     const uint64_t V = o.ext.size();
     // lines 1-5: A, L (old IDs with a delta), U (new IDs, ascending)
@@ -236,15 +268,20 @@ void alg2_merge(Graph& G, Scan& S) {
         n.ext = o.ext;
     }
     const uint64_t Vn = n.ext.size();
-    bool n_identity = true;
-    for (uint64_t i = 0; i < Vn && n_identity; ++i) n_identity = n.ext[i] == i;
+    tr("merge: lines 1-5 (A, L, U; new ID map)");
     auto new_dense = [&](uint64_t x) -> uint32_t {  // external ID -> dense ID in the new map
         auto it = std::lower_bound(n.ext.begin(), n.ext.end(), x);
         return (uint32_t)(it - n.ext.begin());
     };
     auto row_old = [&](uint64_t r) -> int64_t { return ids_change ? src_old[r] : (int64_t)r; };
     auto row_delta = [&](uint64_t r) -> const Delta* { return ids_change ? src_delta[r] : dl[r]; };
-    auto col_of = [&](uint32_t c) -> uint32_t { return ids_change ? remap[c] : c; };
+    // one gather per old column: kNone if a delete removed the target's old edges (cascade),
+    // else the target's new dense ID
+    std::vector<uint64_t> kbits((V + 63) / 64, 0);
+    for (uint64_t c = 0; c < V; ++c) if (killed[c]) kbits[c >> 6] |= 1ull << (c & 63);
+    std::vector<uint32_t> colmap(V);
+#pragma omp parallel for schedule(static)
+    for (int64_t c = 0; c < (int64_t)V; ++c) colmap[c] = killed[c] ? kNone : (ids_change ? remap[c] : (uint32_t)c);
     // lines 6-17 for one new row r: returns its length, writes it when cols != nullptr
     auto row = [&](uint64_t r, uint32_t* cols, float* w) -> int64_t {
         const int64_t u = row_old(r);
@@ -256,9 +293,14 @@ void alg2_merge(Graph& G, Scan& S) {
         };
         const bool keep_old = u >= 0 && !killed[u];  // merge(): deleted node -> no old entries
         if (!d) {  // lines 8-10 / 13-15: new_csr[i] = old_csr[i]
+            if (!cols) {  // length only: the killed bitmap is small enough to stay in cache
+                for (int64_t e = o.off[u]; e < o.off[u + 1]; ++e)
+                    k += !((kbits[o.cols[e] >> 6] >> (o.cols[e] & 63)) & 1);
+                return k;
+            }
             for (int64_t e = o.off[u]; e < o.off[u + 1]; ++e) {
-                const uint32_t c = o.cols[e];
-                if (!killed[c]) put(col_of(c), o.w[e]);
+                const uint32_t c = colmap[o.cols[e]];
+                if (c != kNone) put(c, o.w[e]);
             }
             return k;
         }
@@ -266,9 +308,9 @@ void alg2_merge(Graph& G, Scan& S) {
         int64_t e = keep_old ? o.off[u] : 0, ee = keep_old ? o.off[u + 1] : 0;
         auto it = d->e.begin();
         while (e < ee || it != d->e.end()) {
-            if (e < ee && killed[o.cols[e]]) { ++e; continue; }
+            if (e < ee && colmap[o.cols[e]] == kNone) { ++e; continue; }
             const bool take_old = it == d->e.end() || (e < ee && o.ext[o.cols[e]] < it->first);
-            if (take_old) { put(col_of(o.cols[e]), o.w[e]); ++e; continue; }
+            if (take_old) { put(colmap[o.cols[e]], o.w[e]); ++e; continue; }
             if (e < ee && o.ext[o.cols[e]] == it->first) ++e;  // the delta's outcome replaces it
             if (it->second.first) put(new_dense(it->first), it->second.second);
             ++it;
@@ -276,15 +318,18 @@ void alg2_merge(Graph& G, Scan& S) {
         return k;
     };
     n.off.assign(Vn + 1, 0);
+    tr("merge: column map");
 #pragma omp parallel for schedule(dynamic, 4096)
     for (int64_t r = 0; r < (int64_t)Vn; ++r) n.off[r + 1] = row(r, nullptr, nullptr);
     for (uint64_t r = 0; r < Vn; ++r) n.off[r + 1] += n.off[r];
+    tr("merge: row lengths + offsets");
     n.cols.resize(n.off[Vn]);
     n.w.resize(n.off[Vn]);
 #pragma omp parallel for schedule(dynamic, 4096)
     for (int64_t r = 0; r < (int64_t)Vn; ++r) row(r, n.cols.data() + n.off[r], n.w.data() + n.off[r]);
-    G.g = std::move(n);  // line 18: the new CSR replaces the old one
-    G.identity = n_identity;
+    tr("merge: rows");
+    G.g = std::move(n);  // the new CSR replaces the old one
+    G.index();
 }
 
 inline uint64_t sm64(uint64_t x) {
@@ -333,14 +378,13 @@ int o3_create_edges(void* h, uint64_t nv, const uint64_t* ids, uint64_t ne, cons
     G.g.off.assign(1, 0);
     if (ne >= 0xFFFFFFFFull || nv >= 0xFFFFFFFFull) return E_INVAL;
     std::vector<uint64_t> ext(nv);
-    bool ident = true;
     for (uint64_t i = 0; i < nv; ++i) {
         ext[i] = ids ? ids[i] : i;
         if (i && ext[i] <= ext[i - 1]) return E_INVAL;
-        ident = ident && ext[i] == i;
     }
     G.g.ext = std::move(ext);
-    G.identity = ident;
+    G.index();
+    Tr tr;
     std::vector<uint32_t> s(ne), d(ne);
     int bad = 0;
 #pragma omp parallel for reduction(| : bad) schedule(static)
@@ -351,17 +395,23 @@ int o3_create_edges(void* h, uint64_t nv, const uint64_t* ids, uint64_t ne, cons
         d[e] = (uint32_t)b;
     }
     if (bad) { G.g = Csr(); G.g.off.assign(1, 0); G.g.ext.clear(); return E_INVAL; }
+    tr("create: endpoint lookup");
     // counting sort by source row: (dst << 32 | input index) per row
+    // (the order inside a row does not matter yet: every row is sorted below)
     std::vector<int64_t> cnt(nv + 1, 0);
-    for (uint64_t e = 0; e < ne; ++e) ++cnt[s[e] + 1];
+#pragma omp parallel for schedule(static)
+    for (int64_t e = 0; e < (int64_t)ne; ++e) __atomic_fetch_add(&cnt[s[e] + 1], 1, __ATOMIC_RELAXED);
     for (uint64_t v = 0; v < nv; ++v) cnt[v + 1] += cnt[v];
     std::vector<uint64_t> key(ne);
     {
         std::vector<int64_t> cur(cnt.begin(), cnt.end() - 1);
-        for (uint64_t e = 0; e < ne; ++e) key[cur[s[e]]++] = (uint64_t)d[e] << 32 | e;
+#pragma omp parallel for schedule(static)
+        for (int64_t e = 0; e < (int64_t)ne; ++e)
+            key[__atomic_fetch_add(&cur[s[e]], 1, __ATOMIC_RELAXED)] = (uint64_t)d[e] << 32 | (uint64_t)e;
     }
     std::vector<uint32_t>().swap(s);
     std::vector<uint32_t>().swap(d);
+    tr("create: counting sort by row");
     // each row by (dst, index); the last index of a dst wins
     std::vector<int64_t>& off = G.g.off;
     off.assign(nv + 1, 0);
@@ -373,6 +423,7 @@ int o3_create_edges(void* h, uint64_t nv, const uint64_t* ids, uint64_t ne, cons
             if (e + 1 == cnt[v + 1] || (key[e + 1] >> 32) != (key[e] >> 32)) ++k;
         off[v + 1] = k;
     }
+    tr("create: row sorts");
     for (uint64_t v = 0; v < nv; ++v) off[v + 1] += off[v];
     G.g.cols.resize(off[nv]);
     G.g.w.resize(off[nv]);
@@ -386,6 +437,7 @@ int o3_create_edges(void* h, uint64_t nv, const uint64_t* ids, uint64_t ne, cons
                 ++k;
             }
     }
+    tr("create: rows written");
     return OK;
 }
 
@@ -407,11 +459,15 @@ int o3_apply(void* h, uint64_t n, const uint8_t* kind, const uint64_t* src, cons
     std::stable_sort(vis.begin(), vis.end(), [](const Op& a, const Op& b) {
         return a.ts != b.ts ? a.ts < b.ts : a.seq < b.seq;
     });
+    Tr tr;
+    tr("apply: split + order");
     if (!vis.empty()) {
         Scan S(G);
         S.nd.reserve(vis.size());
         for (const Op& o : vis) S.fold(o);
+        tr("apply: scan (per-node deltas)");
         alg2_merge(G, S);
+        tr("apply: Algorithm 2 merge");
     }
     G.pending.swap(pend);
     G.snap_ts = snapshot_ts;

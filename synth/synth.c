@@ -139,14 +139,16 @@ void synth_rmat_batch(int scale, uint64_t seed, uint64_t k, uint64_t n, uint64_t
 }
 
 /* ---------------------------------------------------- LDBC-SNB shape ---- */
-/* vertices: persons (1<<56)|p for p < n_person, messages (2<<56)|m; ascending */
-#define LDBC_PERSON(p) ((1ull << 56) | (uint64_t)(p))
-#define LDBC_MSG(m)    ((2ull << 56) | (uint64_t)(m))
+/* vertices: messages (1<<56)|m, persons (2<<56)|p; ascending (messages first).  The
+ * Person type code is the larger one so that a new Person's ID (2<<56)|(n_person + j)
+ * exceeds every existing ID, as Algorithm 2 assumes of new nodes. */
+#define LDBC_MSG(m)    ((1ull << 56) | (uint64_t)(m))
+#define LDBC_PERSON(p) ((2ull << 56) | (uint64_t)(p))
 
 void synth_ldbc_vertices(uint64_t n_person, uint64_t n_msg, uint64_t* ids) {
 #pragma omp parallel for schedule(static)
     for (int64_t i = 0; i < (int64_t)(n_person + n_msg); ++i)
-        ids[i] = (uint64_t)i < n_person ? LDBC_PERSON(i) : LDBC_MSG((uint64_t)i - n_person);
+        ids[i] = (uint64_t)i < n_msg ? LDBC_MSG(i) : LDBC_PERSON((uint64_t)i - n_msg);
 }
 
 /* heavy-tailed person index: P(p) ~ p^(-2/3) (hub-first); lodeg mirrors it */
@@ -193,8 +195,11 @@ void synth_ldbc_edges(uint64_t n_person, uint64_t n_msg, uint64_t e_person, uint
  *   insert node : NODE_INSERT new person, EDGE_INSERT existing person -> new
  *   delete rel  : EDGE_DELETE of an initial person edge
  *   delete node : NODE_DELETE person (+ the library cascades its relationships)
- * New person IDs are (1<<56) | (n_person + k*n_cap + j): above every existing ID,
- * as the paper's Algorithm 2 assumes.
+ * New person IDs are (2<<56) | (n_person + k*n_cap + txn): above every existing ID
+ * (messages carry the smaller type code), as the paper's Algorithm 2 assumes of new
+ * nodes.  Node deletes pick hubs first (the paper's HiDeg window,
+ * P:L978-988), so every cycle cascades thousands of edges and the graph shrinks from
+ * batch to batch (bench.py reports E before and after the timed region).
  */
 uint64_t synth_ldbc_batch(uint64_t n_person, uint64_t n_msg, uint64_t e_person, uint64_t seed,
                           uint64_t k, uint64_t n_cap, int lodeg, uint64_t ts_base,

@@ -246,6 +246,24 @@ h2tap_status h2tap_route_pack(const h2tap_replica* r, const h2tap_batch* batch, 
 h2tap_status h2tap_delta_apply_routed(h2tap_replica* r, const h2tap_route_rec* recs, size_t n,
         uint64_t snapshot_ts, h2tap_apply_stats* stats /* nullable */);
 
+/* Two-phase apply (all-or-nothing across the shards of a sharded replica, SURVEY.md
+ * §8(b) "the status is agreed with an all-reduce before commit").
+ * h2tap_delta_apply_prepare / h2tap_delta_apply_routed_prepare run the whole cycle of
+ * h2tap_delta_apply / h2tap_delta_apply_routed (a1-a6) but stop before the swap (a7):
+ * the new CSR, ID map and pending set wait in the back buffers and every read
+ * (export, info, checks) still sees the old snapshot.  The caller then agrees on the
+ * status with its peers and calls h2tap_delta_commit (the swap at snapshot_ts, O(1),
+ * cannot fail on a healthy handle) or h2tap_delta_abort (drops the prepared cycle; the
+ * replica stays exactly as before the prepare).  While a cycle is prepared, every
+ * other apply/create call returns H2TAP_E_INVAL.  h2tap_delta_apply = prepare + commit.
+ * Errors of prepare: those of the one-phase call; nothing is prepared then. */
+h2tap_status h2tap_delta_apply_prepare(h2tap_replica* r, const h2tap_batch* batch, uint64_t snapshot_ts,
+        h2tap_apply_stats* stats /* nullable */);
+h2tap_status h2tap_delta_apply_routed_prepare(h2tap_replica* r, const h2tap_route_rec* recs, size_t n,
+        uint64_t snapshot_ts, h2tap_apply_stats* stats /* nullable */);
+h2tap_status h2tap_delta_commit(h2tap_replica* r);  /* E_INVAL if nothing is prepared */
+h2tap_status h2tap_delta_abort(h2tap_replica* r);   /* no-op if nothing is prepared */
+
 /* Sizes of the current replica (any pointer may be NULL). */
 h2tap_status h2tap_replica_info(const h2tap_replica* r, uint64_t* n_vertices, uint64_t* n_edges,
         uint64_t* snapshot_ts, uint64_t* n_pending, uint64_t* shard_vertex_base,

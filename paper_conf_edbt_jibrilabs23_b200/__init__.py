@@ -108,6 +108,10 @@ _lib.h2tap_sssp.restype = ctypes.c_int
 _lib.h2tap_sssp.argtypes = [_P, _u64, _P, ctypes.c_int]
 for _n, _a in (("h2tap_batch_stage", [_P, ctypes.POINTER(_Batch), ctypes.POINTER(_Batch)]),
                ("h2tap_route_count", [_P, ctypes.POINTER(_Batch), _P]),
+               ("h2tap_delta_apply_prepare", [_P, ctypes.POINTER(_Batch), _u64, ctypes.POINTER(ApplyStats)]),
+               ("h2tap_delta_apply_routed_prepare", [_P, _P, ctypes.c_size_t, _u64, ctypes.POINTER(ApplyStats)]),
+               ("h2tap_delta_commit", [_P]),
+               ("h2tap_delta_abort", [_P]),
                ("h2tap_route_pack_p2p", [_P, ctypes.POINTER(_Batch), _u64, _P, _P]),
                ("h2tap_ipc_alloc", [ctypes.c_int, ctypes.c_size_t, ctypes.POINTER(_P), _P]),
                ("h2tap_ipc_open", [ctypes.c_int, _P, ctypes.POINTER(_P)]),
@@ -342,6 +346,29 @@ class Replica:
         _check(_lib.h2tap_delta_apply_routed(self._h, ctypes.c_void_p(recs.data_ptr()) if n else None, int(n),
                                              int(snapshot_ts), ctypes.byref(st)), "h2tap_delta_apply_routed")
         return st.as_dict()
+
+    def prepare_routed(self, recs, n: int, snapshot_ts: int):
+        """h2tap_delta_apply_routed_prepare: the whole cycle except the swap; returns
+        (status, stats).  Follow with commit() or abort()."""
+        st = ApplyStats()
+        rc = _lib.h2tap_delta_apply_routed_prepare(self._h, ctypes.c_void_p(recs.data_ptr()) if n else None,
+                                                   int(n), int(snapshot_ts), ctypes.byref(st))
+        return rc, st.as_dict()
+
+    def prepare(self, batch, snapshot_ts: int):
+        """h2tap_delta_apply_prepare: (status, stats); follow with commit() or abort()."""
+        b, keep = self._batch(batch)
+        st = ApplyStats()
+        rc = _lib.h2tap_delta_apply_prepare(self._h, ctypes.byref(b), int(snapshot_ts), ctypes.byref(st))
+        return rc, st.as_dict()
+
+    def commit(self):
+        """h2tap_delta_commit: swap in the prepared cycle (a7)."""
+        _check(_lib.h2tap_delta_commit(self._h), "h2tap_delta_commit")
+
+    def abort(self):
+        """h2tap_delta_abort: drop the prepared cycle (the replica is unchanged)."""
+        _check(_lib.h2tap_delta_abort(self._h), "h2tap_delta_abort")
 
     def stage(self, batch) -> "StagedBatch":
         """h2tap_batch_stage: start the host->device copy of the next batch (pinned host

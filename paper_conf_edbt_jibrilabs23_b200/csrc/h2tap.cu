@@ -130,13 +130,37 @@ struct h2tap_replica {
     Buf pk[2], ps[2], pd[2], pw[2], pt[2], pq[2];
     // scratch
     Buf Wk, Ws, Wd, Ww, Wt, Wq, idx_p, idx_n, idx_e, status;
-    Buf keyA, keyB, valA, valB, hist, dbase, rs_status, rs_ctr;
+    Buf keyA, keyB, valA, valB, hist, dbase, rs_status, rs_ctr, rs_coop;
     Buf nv, nv_ext, dropped, ins_q, ins_oldpos, hd_rows, hd_bits;
     Buf op_flags, op_ou, op_ow;
     Buf ins_pos, ins_row, ins_col, ins_w, del_pos, upd_pos, upd_w, KR;
     Buf misc, nsorted, part, opart, deg, tsum, remap_shift, remap32, casc_wrel, tile_emit, tile_base, del_row, casc_mask, status2, bfs_a, bfs_b, pr_a, pr_b;
     Buf xrec, xins, xwts, xdel, xcnt, xoff;  // delta-record input (h2tap_delta_apply_records)
     bool tomb = false;  // tombstone-row mode (reading A23)
+    // a finished cycle waiting for the swap (two-phase apply of a sharded replica: every
+    // rank prepares, the ranks agree on the status, then all commit or all abort)
+    struct Prep {
+        bool on = false, node_mode = false, identity = true;
+        int nb = 0, pn = 0, ext_new = 0;
+        uint64_t V = 0, E = 0, row_lo = 0, Vr = 0, n_pend = 0, n = 0, S = 0;
+    } prep;
+    bool defer_commit = false;  // apply_core leaves the result prepared instead of swapping
+    void commit() {             // a7: the pointer flip
+        cur = prep.nb;
+        if (prep.node_mode) {
+            ext_cur = prep.ext_new;
+            identity = prep.identity;
+        }
+        V = prep.V;
+        E = prep.E;
+        row_lo = prep.row_lo;
+        Vr = prep.Vr;
+        pcur = prep.pn;
+        n_pend = prep.n_pend;
+        next_seq += prep.n;
+        snap = prep.S;
+        prep.on = false;
+    }
     Buf casc_status;    // look-back words of the cascade scan (runs beside the edge-op phase)
     Buf live[2];        // tombstone mode: u8 liveness per dense id, double-buffered with ext
     Buf ctr;
@@ -200,10 +224,39 @@ namespace {
 // ---------------------------------------------------------------- sort ----
 // Stable LSD sort of (keys, vals)[0, n) on the low `bits` bits; result in (k, v).
 // n_dev (nullable): the actual count is in device memory and n is an upper bound.
+// Cooperative single-launch sort (rs_coop) when every tile fits on the GPU at once; returns
+// false (nothing launched) when it does not.
+template <int ITEMS>
+bool radix_sort_coop(h2tap_replica* r, uint64_t*& k, uint32_t*& v, uint64_t*& k2, uint32_t*& v2, uint64_t n,
+                     int passes, const unsigned long long* n_dev) {
+    constexpr int tile = kRsThreads * ITEMS, smem = tile * 12;
+    static int occ = -1;  // per process: one device type
+    if (occ < 0) CK(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, rs_coop<ITEMS>, kRsThreads, smem));
+    const uint64_t T = cdiv(n, tile);
+    if (T > (uint64_t)occ * r->n_sm) return false;
+    uint32_t* cnt = r->get<uint32_t>(r->rs_coop, T * 256 + 256 + 32);
+    uint32_t* tot = cnt + T * 256;
+    unsigned int* bar = tot + 256;
+    CK(cudaMemsetAsync(bar, 0, 4, r->st));
+    void* args[] = {&k, &v, &k2, &v2, &n, &n_dev, &passes, &cnt, &tot, &bar};
+    CK(cudaLaunchCooperativeKernel((void*)rs_coop<ITEMS>, dim3((unsigned)T), dim3(kRsThreads), args, smem, r->st));
+    CKL();
+    if (passes & 1) {
+        std::swap(k, k2);
+        std::swap(v, v2);
+    }
+    return true;
+}
+
 void radix_sort(h2tap_replica* r, uint64_t*& k, uint32_t*& v, uint64_t*& k2, uint32_t*& v2, uint64_t n, int bits,
                 const unsigned long long* n_dev = nullptr) {
     if (n <= 1 || bits <= 0) return;
     const int passes = (bits + 7) / 8;
+    if (passes <= kRsMaxPasses) {
+        if (n <= (1u << 18) ? radix_sort_coop<4>(r, k, v, k2, v2, n, passes, n_dev)
+                            : radix_sort_coop<12>(r, k, v, k2, v2, n, passes, n_dev))
+            return;
+    }
     const uint64_t ntiles = cdiv(n, kRsTile);
     uint32_t* hist = r->get<uint32_t>(r->hist, kRsMaxPasses * 256);
     uint64_t* dbase = r->get<uint64_t>(r->dbase, kRsMaxPasses * 256 + kRsMaxPasses);
@@ -305,6 +358,7 @@ constexpr int kCascCtasPerSm = H2TAP_CASC_CTAS;  // cascade pass beside the edge
 h2tap_status apply_core(h2tap_replica* r, const BatchIn& in, uint64_t S, bool create, h2tap_apply_stats* stats) {
     cudaStream_t st = r->st;
     const uint64_t n = in.n, np = r->n_pend, m = np + n;
+    if (r->prep.on) { set_err("a prepared cycle must be committed or aborted first"); return H2TAP_E_INVAL; }
     if (m >= 0xFFFFFFFFull) { set_err("batch + pending = %llu ops exceeds 2^32-1", (unsigned long long)m); return H2TAP_E_CAPACITY; }
     g_launches = in.pre_launches;
     g_h2d = in.pre_h2d;
@@ -737,20 +791,14 @@ h2tap_status apply_core(h2tap_replica* r, const BatchIn& in, uint64_t S, bool cr
     const uint64_t row_lo_new = (node_mode && r->sharded) ? fc.row_lo_new : row_lo;
     const uint64_t n_ins = fc.n_ins, n_del = fc.n_del, n_upd = fc.n_upd, n_casc = fc.n_casc;
 
-    // ---- a7: swap at snapshot_ts (nothing above touched the front state)
-    r->cur = nb;
-    if (node_mode) {
-        r->ext_cur = ec ^ 1;
-        r->identity = fc.new_identity == 1;
-    }
-    r->V = Vn;
-    r->E = En;
-    r->row_lo = row_lo_new;
-    r->Vr = Vr_new;
-    r->pcur = pn;
-    r->n_pend = n_pend_new;
-    r->next_seq += n;
-    r->snap = S;
+    // ---- a7: swap at snapshot_ts (nothing above touched the front state).  Two-phase
+    // (h2tap_delta_*_prepare): the new state waits in the back buffers for commit/abort.
+    h2tap_replica::Prep& pr = r->prep;
+    pr.nb = nb; pr.pn = pn; pr.node_mode = node_mode; pr.ext_new = ec ^ 1;
+    pr.identity = fc.new_identity == 1;
+    pr.V = Vn; pr.E = En; pr.row_lo = row_lo_new; pr.Vr = Vr_new; pr.n_pend = n_pend_new; pr.n = n; pr.S = S;
+    pr.on = true;
+    if (!r->defer_commit) r->commit();
     if (stats) {
         memset(stats, 0, sizeof *stats);
         stats->n_visible = n_node + n_edge;
@@ -872,7 +920,7 @@ void free_replica(h2tap_replica* r) {
                    &r->pk[0], &r->pk[1], &r->ps[0], &r->ps[1], &r->pd[0], &r->pd[1], &r->pw[0], &r->pw[1],
                    &r->pt[0], &r->pt[1], &r->pq[0], &r->pq[1], &r->Wk, &r->Ws, &r->Wd, &r->Ww, &r->Wt, &r->Wq,
                    &r->idx_p, &r->idx_n, &r->idx_e, &r->status, &r->keyA, &r->keyB, &r->valA, &r->valB,
-                   &r->hist, &r->dbase, &r->rs_status, &r->rs_ctr, &r->nv, &r->nv_ext, &r->dropped, &r->ins_q,
+                   &r->hist, &r->dbase, &r->rs_status, &r->rs_ctr, &r->rs_coop, &r->nv, &r->nv_ext, &r->dropped, &r->ins_q,
                    &r->ins_oldpos, &r->hd_rows, &r->hd_bits, &r->op_flags, &r->op_ou, &r->op_ow,
                    &r->ins_pos, &r->ins_row, &r->ins_col, &r->ins_w, &r->del_pos, &r->upd_pos, &r->upd_w,
                    &r->KR, &r->misc, &r->nsorted, &r->part, &r->opart, &r->deg, &r->tsum, &r->remap_shift, &r->remap32, &r->casc_wrel, &r->tile_emit, &r->tile_base, &r->del_row, &r->casc_mask, &r->status2, &r->bounds_dev, &r->fence[0], &r->fence[1], &r->bfs_a, &r->bfs_b, &r->pr_a, &r->pr_b, &r->ctr,
@@ -1354,6 +1402,38 @@ h2tap_status h2tap_delta_apply_routed(h2tap_replica* r, const h2tap_route_rec* r
         BatchIn in{n, 1, nullptr, nullptr, nullptr, nullptr, nullptr, nullptr, 0, reinterpret_cast<const RouteRec*>(recs)};
         return apply_core(r, in, snapshot_ts, false, stats);
     });
+}
+
+h2tap_status h2tap_delta_apply_prepare(h2tap_replica* r, const h2tap_batch* b, uint64_t snapshot_ts,
+                                       h2tap_apply_stats* stats) {
+    if (!r) { set_err("null replica"); return H2TAP_E_INVAL; }
+    r->defer_commit = true;  // run the cycle with the swap deferred
+    const h2tap_status s = h2tap_delta_apply(r, b, snapshot_ts, stats);
+    r->defer_commit = false;
+    return s;
+}
+
+h2tap_status h2tap_delta_apply_routed_prepare(h2tap_replica* r, const h2tap_route_rec* recs, size_t n,
+                                              uint64_t snapshot_ts, h2tap_apply_stats* stats) {
+    if (!r) { set_err("null replica"); return H2TAP_E_INVAL; }
+    r->defer_commit = true;
+    const h2tap_status s = h2tap_delta_apply_routed(r, recs, n, snapshot_ts, stats);
+    r->defer_commit = false;
+    return s;
+}
+
+h2tap_status h2tap_delta_commit(h2tap_replica* r) {
+    if (!r) { set_err("null replica"); return H2TAP_E_INVAL; }
+    if (r->poisoned) { set_err("replica poisoned by an earlier CUDA error"); return H2TAP_E_POISONED; }
+    if (!r->prep.on) { set_err("no prepared cycle to commit"); return H2TAP_E_INVAL; }
+    r->commit();
+    return H2TAP_OK;
+}
+
+h2tap_status h2tap_delta_abort(h2tap_replica* r) {
+    if (!r) { set_err("null replica"); return H2TAP_E_INVAL; }
+    r->prep.on = false;  // the back buffers are simply overwritten by the next cycle
+    return H2TAP_OK;
 }
 
 h2tap_status h2tap_replica_info(const h2tap_replica* r, uint64_t* nv, uint64_t* ne, uint64_t* snap, uint64_t* npend,

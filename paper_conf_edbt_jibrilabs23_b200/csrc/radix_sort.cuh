@@ -212,4 +212,136 @@ __global__ void __launch_bounds__(kRsThreads) rs_onesweep(
     }
 }
 
+// ------------------------------------------------------------ cooperative ----
+// All passes in ONE launch for key counts whose tiles are co-resident (launched with
+// cudaLaunchCooperativeKernel, one tile per CTA).  A pass: every CTA ranks its tile
+// (warp match_any, stable) and publishes its 256 digit counts; grid barrier; the CTAs
+// scan the count matrix column-wise (digit d by CTA d mod grid: exclusive over tiles,
+// plus the digit total); grid barrier; every CTA turns the 256 totals into digit bases
+// (block scan), adds its tile's column prefix and scatters through shared memory in
+// contiguous runs; grid barrier before the next pass reads the output.  This replaces
+// the per-digit decoupled look-back of rs_onesweep, whose chain of 8-tile steps is the
+// critical path when every tile publishes at the same moment (all tiles resident), by
+// two barriers and a parallel scan, and the per-pass launches by one.
+__device__ __forceinline__ void rs_grid_sync(unsigned int* bar, unsigned int& target) {
+    __syncthreads();
+    if (threadIdx.x == 0) {
+        target += gridDim.x;
+        __threadfence();
+        atomicAdd(bar, 1u);
+        while (*reinterpret_cast<volatile unsigned int*>(bar) < target) __nanosleep(32);
+        __threadfence();
+    }
+    __syncthreads();
+}
+
+template <int ITEMS>
+__global__ void __launch_bounds__(kRsThreads, ITEMS >= 12 ? 3 : 4) rs_coop(
+    uint64_t* __restrict__ k0, uint32_t* __restrict__ v0, uint64_t* __restrict__ k1, uint32_t* __restrict__ v1,
+    uint64_t n, const unsigned long long* __restrict__ n_dev, int passes,
+    uint32_t* __restrict__ cnt /* [grid][256] */, uint32_t* __restrict__ tot /* [256] */, unsigned int* __restrict__ bar) {
+    constexpr int TILE = kRsThreads * ITEMS;
+    __shared__ uint32_t s_wcnt[kRsWarps][256];
+    __shared__ uint32_t s_dstart[256];
+    __shared__ uint32_t s_gpre[256];
+    __shared__ uint32_t s_scan[kRsThreads / 32 + 1];
+    extern __shared__ __align__(16) uint8_t rs_dsm[];  // TILE * 12 bytes
+    uint64_t* s_keys = reinterpret_cast<uint64_t*>(rs_dsm);
+    uint32_t* s_vals = reinterpret_cast<uint32_t*>(rs_dsm + TILE * 8);
+    const int tid = threadIdx.x, w = tid >> 5, l = lane_id();
+    const uint32_t T = gridDim.x, b = blockIdx.x;
+    n = rs_count(n, n_dev);
+    const uint64_t base = (uint64_t)b * TILE;
+    const uint32_t tile_n = base >= n ? 0u : (uint32_t)(n - base < (uint64_t)TILE ? n - base : (uint64_t)TILE);
+    unsigned int target = 0;
+    for (int p = 0; p < passes; ++p) {
+        const int shift = 8 * p;
+        const uint64_t* kin = (p & 1) ? k1 : k0;
+        const uint32_t* vin = (p & 1) ? v1 : v0;
+        uint64_t* kout = (p & 1) ? k0 : k1;
+        uint32_t* vout = (p & 1) ? v0 : v1;
+        for (int i = tid; i < kRsWarps * 256; i += kRsThreads) (&s_wcnt[0][0])[i] = 0;
+        __syncthreads();
+        uint64_t k[ITEMS];
+        uint32_t v[ITEMS], rank[ITEMS];
+#pragma unroll
+        for (int i = 0; i < ITEMS; ++i) {
+            const uint32_t j = (uint32_t)w * 32 * ITEMS + i * 32 + l;
+            const bool ok = j < tile_n;
+            k[i] = ok ? kin[base + j] : 0;
+            v[i] = ok ? vin[base + j] : 0;
+        }
+#pragma unroll
+        for (int i = 0; i < ITEMS; ++i) {
+            const uint32_t j = (uint32_t)w * 32 * ITEMS + i * 32 + l;
+            const bool ok = j < tile_n;
+            const uint32_t valid = __ballot_sync(0xffffffffu, ok);
+            rank[i] = 0;
+            if (ok) {
+                const uint32_t d = (uint32_t)(k[i] >> shift) & 255u;
+                const uint32_t peers = __match_any_sync(valid, d);
+                const uint32_t before = s_wcnt[w][d];
+                __syncwarp(valid);
+                if (l == (uint32_t)(__ffs(peers) - 1)) s_wcnt[w][d] = before + __popc(peers);
+                __syncwarp(valid);
+                rank[i] = before + __popc(peers & lanemask_lt());
+            }
+        }
+        __syncthreads();
+        uint32_t c = 0;
+        {   // thread d: exclusive over warps for digit d, tile count of d
+            const int d = tid;
+            for (int ww = 0; ww < kRsWarps; ++ww) {
+                const uint32_t t = s_wcnt[ww][d];
+                s_wcnt[ww][d] = c;
+                c += t;
+            }
+        }
+        uint32_t tt;
+        const uint32_t ds = block_exclusive_scan<kRsThreads>(c, s_scan, &tt);
+        s_dstart[tid] = ds;
+        cnt[(uint64_t)b * 256 + tid] = c;
+        rs_grid_sync(bar, target);
+        // column scans: digit d over the T tiles (exclusive, in place), total -> tot[d]
+        for (uint32_t d = b; d < 256; d += T) {
+            uint32_t carry = 0;
+            for (uint32_t t0 = 0; t0 < T; t0 += kRsThreads) {
+                const uint32_t t = t0 + tid;
+                const uint32_t x = t < T ? cnt[(uint64_t)t * 256 + d] : 0u;
+                uint32_t sum;
+                const uint32_t e = block_exclusive_scan<kRsThreads>(x, s_scan, &sum);
+                if (t < T) cnt[(uint64_t)t * 256 + d] = carry + e;
+                carry += sum;
+            }
+            if (tid == 0) tot[d] = carry;
+        }
+        rs_grid_sync(bar, target);
+        {
+            uint32_t sum;
+            const uint32_t db = block_exclusive_scan<kRsThreads>(tot[tid], s_scan, &sum);
+            s_gpre[tid] = db + cnt[(uint64_t)b * 256 + tid];
+        }
+        __syncthreads();
+#pragma unroll
+        for (int i = 0; i < ITEMS; ++i) {
+            const uint32_t j = (uint32_t)w * 32 * ITEMS + i * 32 + l;
+            if (j < tile_n) {
+                const uint32_t d = (uint32_t)(k[i] >> shift) & 255u;
+                const uint32_t pos = s_dstart[d] + s_wcnt[w][d] + rank[i];
+                s_keys[pos] = k[i];
+                s_vals[pos] = v[i];
+            }
+        }
+        __syncthreads();
+        for (uint32_t q = tid; q < tile_n; q += kRsThreads) {
+            const uint64_t key = s_keys[q];
+            const uint32_t d = (uint32_t)(key >> shift) & 255u;
+            const uint32_t o = s_gpre[d] + (q - s_dstart[d]);
+            kout[o] = key;
+            vout[o] = s_vals[q];
+        }
+        if (p + 1 < passes) rs_grid_sync(bar, target);
+    }
+}
+
 }  // namespace h2tap

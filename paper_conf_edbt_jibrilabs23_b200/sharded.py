@@ -2,15 +2,20 @@
 
 The exchange step a8 around the per-shard pipeline:
 
-1. every rank validates its slice of the global batch; the status is agreed with an
-   all-reduce before anything is applied (all ranks commit or none starts);
-2. global arrival numbers are rank-major (all-gather of the slice sizes, reading A5);
-3. the library packs the slice into 40-byte route records grouped by destination
-   (an edge op goes to the shard owning its source, a node op to every shard);
-4. counts, then records are exchanged with all-to-all over the process group
+1. every rank validates its slice of the global batch and counts its records per
+   destination (an edge op goes to the shard owning its source, a node op to every
+   shard); ONE all-gather of (status, slice size, counts[world]) gives every rank the
+   agreed validity, the rank-major global arrival numbers (reading A5) and the whole
+   world x world count matrix (host round trip 1);
+2. the library packs the slice into 40-byte route records grouped by destination;
+3. the records are exchanged with an all-to-all whose splits every rank already knows
    (NCCL over NVLink on GPUs; gloo in the CPU tests);
-5. the library applies what it received (h2tap_delta_apply_routed);
-6. shard bases (first global row, first global edge) come from an all-gather of the
+4. two-phase apply: the library runs the whole cycle on what it received but leaves
+   the result in its back buffers (h2tap_delta_apply_routed_prepare); the ranks agree on
+   the prepare statuses with an all-reduce(MIN) (host round trip 2) and then ALL commit
+   (h2tap_delta_commit, the swap) or ALL abort (h2tap_delta_abort) - a failure on one
+   rank (e.g. out of memory) leaves every shard at the old snapshot;
+5. shard bases (first global row, first global edge) come from an all-gather of the
    shards' row and edge counts.
 
 Freshness checks on the sharded replica (SURVEY.md §8(e) "Checks"): every shard keeps the
@@ -77,6 +82,15 @@ class LibEngine:
 
     def apply_routed(self, recs, n: int, snapshot_ts: int):
         return self.rep.apply_routed(recs, n, snapshot_ts)
+
+    def prepare_routed(self, recs, n: int, snapshot_ts: int):
+        return self.rep.prepare_routed(recs, n, snapshot_ts)
+
+    def commit(self):
+        self.rep.commit()
+
+    def abort(self):
+        self.rep.abort()
 
     # fused exchange (peer-memory windows)
     def route_count(self, batch):
@@ -154,32 +168,46 @@ class ShardedReplica:
         if hasattr(self.engine, "stage"):
             batch = self.engine.stage(batch)
         n = len(batch.kind)
-        # 1. agree on validity (status codes are <= 0; MIN finds any failure)
-        st = self._i64([self.engine.validate(batch)])
-        dist.all_reduce(st, op=dist.ReduceOp.MIN, group=self.group)
-        if int(st.item()) != 0:
-            raise H2tapError(int(st.item()), "sharded apply", "a rank rejected its batch slice")
-        # 2. rank-major global arrival numbers
-        sizes = [self._i64([0]) for _ in range(self.world)]
-        dist.all_gather(sizes, self._i64([n]), group=self.group)
-        sizes = [int(s.item()) for s in sizes]
+        # 1. validity + slice size + destination counts of every rank: one all-gather
+        st = int(self.engine.validate(batch))
+        counts = [int(c) for c in self.engine.route_count(batch)] if st == 0 else [0] * self.world
+        mine = self._i64([st, n] + counts)
+        allv = torch.empty(self.world * (2 + self.world), dtype=torch.int64, device=self.coll)
+        dist.all_gather_into_tensor(allv, mine, group=self.group)
+        M = allv.view(self.world, 2 + self.world).cpu().numpy()          # host round trip 1
+        if int(M[:, 0].min()) != 0:
+            raise H2tapError(int(M[:, 0].min()), "sharded apply", "a rank rejected its batch slice")
+        sizes = [int(x) for x in M[:, 1]]
+        C = M[:, 2:]                                                      # C[s][d]
         seq0 = self.next_seq + sum(sizes[: self.rank])
+        self.last_route_bytes = int(C[self.rank].sum() - C[self.rank][self.rank]) * ROUTE_REC_BYTES
         if self.exchange == "p2p":
-            return self._apply_p2p(batch, seq0, sizes, snapshot_ts)
-        # 3./4. pack by destination and exchange
-        recs, counts = self.engine.pack(batch, seq0)
-        send_c = self._i64(counts)
-        recv_c = torch.empty_like(send_c)
-        dist.all_to_all_single(recv_c, send_c, group=self.group)
-        rc = [int(x) for x in recv_c.tolist()]
-        recv = torch.empty(sum(rc) * ROUTE_REC_BYTES, dtype=torch.uint8, device=self.coll)
-        dist.all_to_all_single(recv, recs.to(self.coll), [c * ROUTE_REC_BYTES for c in rc],
-                               [c * ROUTE_REC_BYTES for c in counts], group=self.group)
-        recv = recv.to(recs.device)
-        # 5. apply the received ops
-        stats = self.engine.apply_routed(recv, sum(rc), snapshot_ts)
+            recv, n_recv = self._exchange_p2p(batch, seq0, C)
+        else:
+            # 2./3. pack by destination, exchange with splits known from C
+            recs, sent = self.engine.pack(batch, seq0)
+            assert [int(x) for x in sent] == [int(x) for x in C[self.rank]], "route counts changed"
+            rc = [int(x) for x in C[:, self.rank]]
+            recv = torch.empty(sum(rc) * ROUTE_REC_BYTES, dtype=torch.uint8, device=self.coll)
+            dist.all_to_all_single(recv, recs.to(self.coll), [c * ROUTE_REC_BYTES for c in rc],
+                                   [int(c) * ROUTE_REC_BYTES for c in C[self.rank]], group=self.group)
+            recv, n_recv = recv.to(recs.device), sum(rc)
+        # 4. two-phase apply: prepare everywhere, agree, then all commit or all abort
+        try:
+            status, stats = self.engine.prepare_routed(recv, n_recv, snapshot_ts)
+        except Exception:   # an engine that raises counts as a failed prepare
+            status, stats = -3, {}
+        agree = self._i64([status])
+        dist.all_reduce(agree, op=dist.ReduceOp.MIN, group=self.group)
+        agreed = int(agree.item())                                        # host round trip 2
+        if agreed != 0:
+            if status == 0:
+                self.engine.abort()
+            raise H2tapError(agreed, "sharded apply", "a rank failed to prepare; every rank aborted")
+        self.engine.commit()
         self.next_seq += sum(sizes)
         stats["global_batch"] = sum(sizes)
+        stats["route_bytes"] = self.last_route_bytes
         return stats
 
     def _windows(self, need):
@@ -203,24 +231,15 @@ class ShardedReplica:
                       for r, (h, _) in enumerate(info)]
         self.win_caps = [c for _, c in info]
 
-    def _apply_p2p(self, batch, seq0: int, sizes, snapshot_ts: int):
-        # 3. destination counts of every rank -> the world x world matrix
-        counts = self._i64(self.engine.route_count(batch))
-        mat = [torch.empty_like(counts) for _ in range(self.world)]
-        dist.all_gather(mat, counts, group=self.group)
-        C = np.array([m.tolist() for m in mat], dtype=np.int64)  # C[s][d]
+    def _exchange_p2p(self, batch, seq0: int, C):
         need = C.sum(axis=0)
         self._windows([int(x) for x in need])
         offsets = C[: self.rank].sum(axis=0) if self.rank else np.zeros(self.world, np.int64)
-        # 4. one kernel packs and stores into the peers' windows; the barrier orders the
-        #    stores before the owners read their windows
+        # one kernel packs and stores into the peers' windows; the barrier orders the
+        # stores before the owners read their windows
         self.engine.pack_p2p(batch, seq0, self.peers, [int(x) for x in offsets])
         dist.barrier(group=self.group)
-        # 5. apply this rank's window
-        stats = self.engine.apply_routed(_Ptr(self.peers[self.rank]), int(need[self.rank]), snapshot_ts)
-        self.next_seq += sum(sizes)
-        stats["global_batch"] = sum(sizes)
-        return stats
+        return _Ptr(self.peers[self.rank]), int(need[self.rank])
 
     def close(self):
         if self.peers is not None:

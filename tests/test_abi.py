@@ -66,6 +66,7 @@ def test_product_package_does_not_touch_the_oracle():
                 src = open(os.path.join(dirpath, f)).read()
                 assert "import oracle" not in src and "from oracle" not in src, f
                 assert "o1_replay" not in src and "liboracle" not in src, f
+                assert "o3_alg2" not in src and "libo3" not in src, f
 
 
 def test_bench_dyn_gpu_measurement_does_not_touch_the_oracle():

@@ -322,3 +322,35 @@ def test_chunked_create_last_duplicate_wins(h2, monkeypatch):
     b = synth.rmat_batch(10, 44, 0, 3000, len(src), p_weight=0.1)
     b.src, b.dst = ids[b.src % (1 << 10)], ids[b.dst % (1 << 10)]
     step(g, o, b, int(b.ts.max()), "after chunked create")
+
+
+def test_two_phase_prepare_commit_abort(h2):
+    """h2tap_delta_apply_prepare leaves every read at the old snapshot until commit;
+    abort drops the prepared cycle (replica unchanged, the same batch applies later);
+    a prepared cycle blocks other applies (E_INVAL) - the all-or-nothing step of a
+    sharded apply."""
+    shape = synth.LdbcShape(n_person=256, n_msg=6000, e_person=9000)
+    seed = synth.seed_of("c2")
+    ids = synth.ldbc_vertices(shape)
+    src, dst, w = synth.ldbc_edges(shape, seed)
+    g, o = pair_from_edges(h2, len(ids), ids, src, dst, w)
+    before = g.export(checksums=True)
+    b = synth.ldbc_batch(shape, seed, 0, 3000, ts_base=1)
+    snap = int(b.ts.max())
+    rc, st = g.prepare(b, snap)
+    assert rc == 0 and st["n_visible"] == len(b)
+    assert g.export(checksums=True)[4] == before[4] and g.info()["snapshot_ts"] == 0
+    rc2, _ = g.apply(b, snap, raise_on_error=False)
+    assert rc2 == -1                                   # prepared: commit or abort first
+    g.abort()
+    assert g.export(checksums=True)[4] == before[4]
+    rc, _ = g.prepare(b, snap)
+    assert rc == 0
+    g.commit()
+    o.apply(b, snap)
+    assert_same(g.export(), o.export(), "two-phase commit")
+    assert g.info()["snapshot_ts"] == snap
+    with pytest.raises(h2.H2tapError):
+        g.commit()                                     # nothing prepared
+    b2 = synth.ldbc_batch(shape, seed, 1, 3000, ts_base=snap)
+    step(g, o, b2, int(b2.ts.max()), "after two-phase")

@@ -2,9 +2,11 @@
 
 Exercises the exchange protocol of paper_conf_edbt_jibrilabs23_b200.sharded (status
 agreement, rank-major arrival numbers, routing of edge ops to the owner of their
-source and of node ops to every shard, variable all-to-all, shard bases) with an
-oracle-backed shard engine standing in for the GPU replica.  The shards' rows,
-gathered in shard order, must equal the unsharded oracle after every batch.
+source and of node ops to every shard, variable all-to-all, two-phase prepare /
+agree / commit-or-abort, shard bases) with an oracle-backed shard engine standing in
+for the GPU replica.  The shards' rows, gathered in shard order, must equal the
+unsharded oracle after every batch; a prepare failure injected on ONE rank must leave
+every shard unchanged (no rank commits), and the next batch must apply normally.
 """
 import os
 import socket
@@ -55,15 +57,35 @@ class OracleShard:
         buf = np.concatenate(parts) if n else np.zeros(0, REC)
         return torch.from_numpy(buf.view(np.uint8).copy()), counts
 
-    def apply_routed(self, recs, n, snap):
+    def route_count(self, b):
+        own = np.where(b.kind <= 1, -1, self.owner(b.src))
+        return [int(np.count_nonzero((own == -1) | (own == d))) for d in range(self.P)]
+
+    fail_next = False   # inject a prepare failure (as if the GPU ran out of memory)
+    prepared = None
+
+    def prepare_routed(self, recs, n, snap):
         from synth import Batch
         r = recs.numpy().view(REC)
         assert len(r) == n and (n < 2 or np.all(np.diff(r["seq"].astype(np.int64)) > 0))
-        b = Batch(r["kind"].copy(), r["src"].copy(), r["dst"].copy(), r["w"].copy(), r["ts"].copy())
+        assert self.prepared is None
+        if self.fail_next:
+            self.fail_next = False
+            return -2, {}
+        self.prepared = (Batch(r["kind"].copy(), r["src"].copy(), r["dst"].copy(), r["w"].copy(),
+                               r["ts"].copy()), snap)
+        return 0, {"n_visible": n}
+
+    def commit(self):
+        b, snap = self.prepared
+        self.prepared = None
         rc, st = self.o.apply(b, snap)
         assert rc == 0
         self.snap = snap
-        return st
+
+    def abort(self):
+        assert self.prepared is not None
+        self.prepared = None
 
     def own_rows(self):
         off, cols, w, ids = self.o.export()
@@ -159,6 +181,19 @@ def _worker(rank, world, port, out):
             off, cols, ww, own_ids, lo = sh.engine.own_rows()
             results.append((off, cols, ww, own_ids, sh.bases()))
             ts += 300
+        # a prepare failure on the last rank only: nobody commits, every shard unchanged
+        before = sh.engine.own_rows()
+        g = synth.fuzz_batch(seed=12, k=0, n=600, n_ids=5 * n + 9, ts_lo=ts + 1, ts_span=50)
+        sl = g.slice(slice(rank * len(g) // world, (rank + 1) * len(g) // world))
+        sh.engine.fail_next = rank == world - 1
+        try:
+            sh.apply(sl, ts + 40)
+            aborted = False
+        except H2tapError as e:
+            aborted = e.status == -2
+        after = sh.engine.own_rows()
+        aborted = aborted and all(np.array_equal(np.asarray(a), np.asarray(b)) for a, b in zip(before, after))
+        aborted = aborted and sh.engine.prepared is None
         # a stale op on one rank must make every rank refuse the batch
         from synth import Batch
         bad = Batch.of([(2, int(ids[0]), int(ids[1]), 1.0, 5 if rank == world - 1 else ts + 10)])
@@ -171,7 +206,7 @@ def _worker(rank, world, port, out):
         src0 = int(sh.engine.o.export()[3][0])
         checks = (src0, sh.bfs(src0).numpy().copy(), sh.sssp(src0).numpy().copy(), sh.pagerank(0.85, 20).numpy().copy())
         gathered = [None] * world
-        dist.all_gather_object(gathered, (results, refused, checks))
+        dist.all_gather_object(gathered, (results, refused and aborted, checks))
         if rank == 0:
             out.put(gathered)
     finally:
@@ -230,7 +265,7 @@ def test_sharded_exchange_over_gloo(world):
         assert np.array_equal(np.concatenate([p[1] for p in parts]), cols)
         assert np.array_equal(np.concatenate([p[2] for p in parts]).view(np.uint32), ww.view(np.uint32))
         ts += 300
-    assert all(gathered[r][1] for r in range(world))  # every rank refused the bad batch
+    assert all(gathered[r][1] for r in range(world))  # every rank aborted / refused the bad batches
     import oracle
     src0, lv, dd, pr = gathered[0][2]
     for r in range(1, world):

@@ -1,22 +1,27 @@
 #!/usr/bin/env python
 """Benchmark: delta updates/s merged into the GPU-resident CSR replica.
 
-    python bench.py [--gpus N] [--steps K] [--warmup W] [--config c2|c3|c1|c4] [--impl h2tap|reference]
+    python bench.py [--gpus N] [--steps K] [--warmup W] [--config c1|c2|c3|c4] [--impl h2tap|reference]
 
-A step is one h2tap_delta_apply of one synthetic batch (all SURVEY.md §8(a)
-steps a1-a7) into the replica.  Default workload: BASELINE.json configs[1]
-(LDBC-SNB-shaped SF10 property graph, 100K-update batches with node inserts and
-deletes and ID remap).  Inputs are device-resident when the timed region
-starts; the e2e leg repeats the measurement with pinned host batches copied in
-by the library inside the timed region.  The CSR (~2.8 GB read + written per
-step) exceeds the 126 MB L2, so no explicit flush is needed.
+A step is one h2tap_delta_apply of one synthetic batch (all SURVEY.md §8(a) steps a1-a7)
+into the replica.  Default workload on 1 GPU: BASELINE.json configs[1] (LDBC-SNB-shaped SF10
+property graph, 100K-update batches with node inserts and deletes and ID remap); with
+--gpus N > 1: configs[3] (RMAT-26, 8M-update batches, the scaling config).  Inputs are
+device-resident when the timed region starts (CUDA events on the replica stream, per-step
+events for p10/p50/p90); the CSR (GBs read + written per step) exceeds the 126 MB L2, so
+no explicit flush is needed (C1 is the L2-resident latency case).  The e2e leg restores
+the replica to the state the timed region started from and replays the same batches from
+pinned host memory through the public API, every H2D copy inside the timed region.
 
-Prints ONE JSON line (rank 0).  Under torchrun with N > 1 the graph is sharded by
-1D external-ID ranges (one shard per rank); every global batch is split rank-major,
-routed to the owners with an all-to-all (NCCL; gloo with --dist-backend gloo) and
-applied per shard (strong scaling: the global batch is the config's).
-``--parallelism replicas`` runs independent replicas instead (weak scaling).  ``--impl reference`` times the oracle (O1, test infrastructure) on the
-host cores over a bounded scaled-down sample of the same workload.
+Prints ONE JSON line (rank 0).  --gpus N > 1 without a launcher re-executes itself under
+torch.distributed.run (N ranks, one GPU each, 127.0.0.1); the graph is sharded by 1D
+external-ID ranges (bounds from a sample of the edge sources, each rank generates only its
+rows), every global batch is split rank-major, routed to the owners with an all-to-all
+(NCCL) and applied per shard with a two-phase commit (strong scaling: the global batch is
+the config's).  ``--parallelism replicas`` runs independent replicas instead.
+The cpu_baseline (1 GPU only) and ``--impl reference`` time O3 - the paper's Algorithm-2
+flat-CSR merge on the host (oracle/, test infrastructure), as it stands - on the FULL
+workload at every host thread (and at 1 thread for the cpu_baseline).
 """
 from __future__ import annotations
 
@@ -60,6 +65,7 @@ class Workload:
         else:
             self.scale = self.cfg["scale"] - (int(np.log2(scale_down)) if scale_down > 1 else 0)
             self.batch_size = max(64, self.cfg["batch"] // scale_down)
+            self.m_initial = self.cfg["edge_factor"] << self.scale
         self.ts = 0
 
     def graph(self):
@@ -69,6 +75,38 @@ class Workload:
             return self.shape.n_vertices, ids, src, dst, w
         src, dst, w = synth.rmat_edges(self.scale, self.seed, n=self.cfg["edge_factor"] << self.scale)
         self.m_initial = len(src)
+        return 1 << self.scale, None, src, dst, w
+
+    def n_edges(self) -> int:
+        if self.cfg["kind"] == "ldbc":
+            return self.shape.n_edges
+        return self.cfg["edge_factor"] << self.scale
+
+    def _edges(self, first: int, n: int):
+        if self.cfg["kind"] == "ldbc":
+            return synth.ldbc_edges(self.shape, self.seed, first, n)
+        return synth.rmat_edges(self.scale, self.seed, n=n, first=first)
+
+    def source_sample(self, n: int = 1 << 20, windows: int = 512) -> np.ndarray:
+        """sources of `n` edges taken from `windows` evenly spaced windows of the edge list
+        (the generators are counter-based: any window can be generated alone)"""
+        m, per = self.n_edges(), max(1, n // windows)
+        return np.concatenate([self._edges(i * m // windows, min(per, m - i * m // windows))[0]
+                               for i in range(windows)])
+
+    def graph_owned(self, keep, chunk: int = 1 << 26):
+        """the graph with only the edges whose source satisfies keep(src): generated chunk by
+        chunk, so a rank never holds the whole edge list"""
+        m = self.n_edges()
+        self.m_initial = m
+        parts = []
+        for first in range(0, m, chunk):
+            s, d, w = self._edges(first, min(chunk, m - first))
+            sel = keep(s)
+            parts.append((s[sel], d[sel], w[sel]))
+        src, dst, w = (np.concatenate([p[i] for p in parts]) for i in range(3))
+        if self.cfg["kind"] == "ldbc":
+            return self.shape.n_vertices, synth.ldbc_vertices(self.shape), src, dst, w
         return 1 << self.scale, None, src, dst, w
 
     def batch(self, k: int) -> synth.Batch:
@@ -163,53 +201,89 @@ def cpu_cores():
 
 
 # ------------------------------------------------------------- oracle arm ----
-def oracle_sample(name: str, steps: int, warmup: int, target_s: float = 20.0):
-    """Time O1 (single-threaded std::map replay + CSR export) on a scaled-down sample."""
+def host_info() -> dict:
+    model = None
+    try:
+        for line in open("/proc/cpuinfo"):
+            if line.startswith("model name"):
+                model = line.split(":", 1)[1].strip()
+                break
+    except OSError:
+        pass
+    return {"cpu_model": model, "nproc": os.cpu_count(), "affinity_cores": cpu_cores()}
+
+
+def o3_run(name: str, plan, budget_s: float):
+    """O3 (oracle/o3_alg2.cpp: the paper's Algorithm-2 flat-CSR merge, as it stands) on the
+    FULL workload of `name`: create from the config's graph (untimed), then per (threads,
+    max_batches) of `plan` apply the stream's next batches, each timed alone; stops a leg
+    once `budget_s` of timed work is spent.  Returns [(threads, updates/s, batches, ms)]."""
     import oracle
-    scale_down = {"c1": 4, "c2": 128, "c3": 256, "c4": 1024}[name]
-    wl = Workload(name, scale_down)
+    wl = Workload(name)
     nv, ids, src, dst, w = wl.graph()
-    o = oracle.O1.from_edges(nv, ids, src, dst, w)
-    times, ops = [], 0
-    total = 0.0
-    for k in range(warmup + steps):
-        b = wl.batch(k)
-        t0 = time.perf_counter()
-        rc, st = o.apply(b, int(b.ts.max()))
-        o.export()
-        dt = time.perf_counter() - t0
-        assert rc == 0
-        if k >= warmup:
-            times.append(dt)
+    oracle.set_threads(0)
+    o = oracle.O3.from_edges(nv, ids, src, dst, w)
+    del src, dst, w
+    out, k = [], 0
+    for threads, max_b in plan:
+        used = oracle.set_threads(threads)
+        times, ops = [], 0
+        while len(times) < max_b and sum(times) < budget_s:
+            b = wl.batch(k)
+            k += 1
+            t0 = time.perf_counter()
+            rc, st = o.apply(b, int(b.ts.max()))
+            times.append(time.perf_counter() - t0)
+            assert rc == 0
             ops += st["n_visible"]
-        total += dt
-        if total > target_s * 3:
-            break
-    value = ops / sum(times) if times else 0.0
-    sample = (f"O1 on a 1/{scale_down} scale-down of the same workload: {wl.describe()}; "
-              f"apply + CSR export per batch, {len(times)} timed batches, 1 thread")
-    return value, sample, (sum(times) / max(1, len(times))) * 1e3
+        out.append((used, ops / sum(times), len(times), 1e3 * sum(times) / len(times)))
+    oracle.set_threads(0)
+    return out, wl
+
+
+def o3_baseline(name: str) -> dict:
+    """cpu_baseline: O3 at every host thread and at 1 thread on the full config."""
+    nth = os.cpu_count() or 1
+    res, wl = o3_run(name, [(nth, 4), (1, 1)], budget_s=30.0)
+    (ta, va, na, ma), (t1, v1, n1, m1) = res
+    return {"value": va, "unit": "updates/s", "cores": ta, "kind": "oracle",
+            "sample": (f"O3 (Algorithm 2 + merge() on a flat host CSR, OpenMP over rows) on the full "
+                       f"workload: {wl.describe()}; batches 0..{na - 1} at {ta} threads ({ma:.0f} ms each), "
+                       f"then batch {na} at 1 thread ({m1:.0f} ms); create untimed"),
+            "single_thread": {"value": v1, "unit": "updates/s", "cores": 1, "batches": n1, "ms_per_batch": m1},
+            "ms_per_batch": ma, "host": host_info(),
+            "paper_context": "paper's scan + Algorithm 2 merge of 2,014,347 SF10 deltas: 4660.39 ms "
+                             "(~432 K deltas/s, 2x EPYC 7F52, P:L1899, P:L1933-1936)"}
 
 
 def run_reference(args):
     world, rank, _ = dist_setup()
     if rank != 0:
         return
-    value, sample, ms = oracle_sample(args.config, args.steps, args.warmup)
-    wl = Workload(args.config)
+    nth = os.cpu_count() or 1
+    res, wl = o3_run(args.config, [(nth, args.warmup), (nth, args.steps)], budget_s=150.0)
+    _, value, n_timed, ms = res[1]
     line = {
         "impl": "reference", "metric": METRIC, "value": value, "unit": "updates/s",
-        "n_gpus": args.gpus, "steps": args.steps, "warmup": args.warmup, "ms_per_step": ms,
+        "n_gpus": args.gpus, "steps": n_timed, "warmup": args.warmup, "ms_per_step": ms,
         "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": "u32/f32",
         "data": "synthetic", "config": {"workload": wl.describe(), "name": args.config},
-        "cpu_baseline": {"value": value, "unit": "updates/s", "cores": 1, "kind": "oracle",
-                         "sample": sample},
+        "cpu_baseline": {"value": value, "unit": "updates/s", "cores": res[1][0], "kind": "oracle",
+                         "sample": (f"O3 (Algorithm-2 flat-CSR merge, oracle/o3_alg2.cpp, as it stands) on the "
+                                    f"full workload, {n_timed} timed batches after {args.warmup} untimed, "
+                                    f"{res[1][0]} OpenMP threads; create untimed"),
+                         "host": host_info()},
         "e2e": {"value": value, "unit": "updates/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0},
     }
     print(json.dumps(line), flush=True)
 
 
 # --------------------------------------------------------------- GPU arm ----
+def pct(xs, q):
+    xs = sorted(xs)
+    return xs[min(len(xs) - 1, int(round(q * (len(xs) - 1))))] if xs else None
+
+
 def run_gpu(args):
     import torch
     import torch.distributed as dist
@@ -218,6 +292,8 @@ def run_gpu(args):
     from paper_conf_edbt_jibrilabs23_b200.sharded import LibEngine, ShardedReplica
 
     world, rank, local = dist_setup()
+    if world != args.gpus:
+        raise SystemExit(f"bench.py: --gpus {args.gpus} but WORLD_SIZE={world}")
     dev_idx = local % max(1, torch.cuda.device_count())
     torch.cuda.set_device(dev_idx)
     if world > 1:
@@ -230,23 +306,24 @@ def run_gpu(args):
 
     wl = Workload(args.config)
     t0 = time.time()
-    nv, ids, src, dst, w = wl.graph()
     if sharded:
-        # 1D external-ID ranges balanced by edge count; this rank keeps the rows it owns
-        bounds = h2.balanced_bounds(src, world)
-        mine = np.searchsorted(bounds[1:world], src, side="right") == rank
-        rep = h2.Replica.from_edges(nv, ids, src[mine], dst[mine], w[mine], 0, device=dev_idx,
+        # 1D external-ID ranges balanced by edge count from a sample of the edge sources; each
+        # rank generates the edge list chunk by chunk and keeps the rows it owns
+        bounds = h2.balanced_bounds(wl.source_sample(), world)
+        nv, ids, src, dst, w = wl.graph_owned(lambda s: np.searchsorted(bounds[1:world], s, side="right") == rank)
+        rep = h2.Replica.from_edges(nv, ids, src, dst, w, 0, device=dev_idx,
                                     rank=rank, world=world, shard_bounds=bounds)
         eng = LibEngine(rep, f"cuda:{dev_idx}")
-        shr = ShardedReplica(eng, rank, world, f"cuda:{dev_idx}", exchange=args.exchange)
+        shr = ShardedReplica(eng, rank, world, f"cuda:{dev_idx}", exchange=args.exchange, time_exchange=True)
     else:
+        nv, ids, src, dst, w = wl.graph()
         rep = h2.Replica.from_edges(nv, ids, src, dst, w, 0, device=dev_idx, tombstone=args.tombstone)
     del src, dst, w
     setup_s = time.time() - t0
 
     n_total = args.warmup + args.steps
     # sharded: every rank draws the same global batches and takes its rank-major slice
-    # (strong scaling: the global batch is the config's); replicas: rank-distinct streams
+    # (the global batch is the config's); replicas: rank-distinct streams
     k0 = 0 if sharded else rank * 1000
 
     def my_part(b):
@@ -273,11 +350,11 @@ def run_gpu(args):
             return synth.RecordBatch(*(tens(a).cuda() for a in (rb.records, rb.inserts, rb.weights, rb.deletes)))
         return synth.Batch(*(tens(a).cuda() for a in (b.kind, b.src, b.dst, b.w, b.ts)))
 
-    def apply(b, snap):
+    def apply(r, b, snap):
         if records:
-            return rep.apply_records(b, snap)
+            return r.apply_records(b, snap)
         if not sharded:
-            return rep.apply(b, snap)
+            return r.apply(b, snap)
         l0 = eng.launches
         st = shr.apply(b, snap)
         st["n_launches"] += eng.launches - l0
@@ -285,22 +362,34 @@ def run_gpu(args):
 
     dev = [to_dev(b) for b in host]
     for k in range(args.warmup):
-        apply(dev[k], snaps[k])
+        apply(rep, dev[k], snaps[k])
     torch.cuda.synchronize()
+    # the e2e leg replays the timed batches on the same graph state: keep the state the timed
+    # region starts from (device copy of the CSR + ID map; single replica, compact IDs)
+    restore = not sharded and not args.tombstone
+    inf0 = rep.info()
+    if restore:
+        snap0 = rep.export(on_device=True)
+        snap_ts0 = inf0["snapshot_ts"]
     if world > 1:
         dist.barrier()
     stats = []
-    ev0, ev1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    evs = [torch.cuda.Event(enable_timing=True) for _ in range(args.steps + 1)]
     with ClockSampler(dev_idx) as clk:
         torch.cuda.synchronize()
-        ev0.record(stream)
-        for k in range(args.warmup, n_total):
-            stats.append(apply(dev[k], snaps[k]))
-        ev1.record(stream)
+        evs[0].record(stream)
+        for j, k in enumerate(range(args.warmup, n_total)):
+            stats.append(apply(rep, dev[k], snaps[k]))
+            evs[j + 1].record(stream)
         torch.cuda.synchronize()
     if world > 1:
         dist.barrier()
-    ms = ev0.elapsed_time(ev1)
+    ms = evs[0].elapsed_time(evs[-1])
+    step_ms = [evs[j].elapsed_time(evs[j + 1]) for j in range(args.steps)]
+    inf1 = rep.info()
+    e_steps = [inf0["n_edges"]]
+    for s_ in stats:  # I6: E' = E + NEW - DEL - CASC
+        e_steps.append(e_steps[-1] + s_["n_new"] - s_["n_del"] - s_["n_casc"])
     # updates: the global batches' ops (sharded: node ops reach every shard, count them once)
     updates = (sum(glob_n[args.warmup:]) / world if sharded else sum(s["n_visible"] for s in stats))
 
@@ -319,12 +408,19 @@ def run_gpu(args):
 
     # ---- e2e: pinned host batches through the public API, H2D inside the timed region
     pipelined = not sharded and not records
-    n_ewarm = 2 if pipelined else 0  # staging slots allocated and warm before the timed region
-    e_glob = [wl.batch(k0 + n_total + k) for k in range(args.steps + n_ewarm)]
-    e_host = [my_part(b) for b in e_glob]
-    e_snaps = [int(b.ts.max()) for b in e_glob]
-    e_glob_n = [len(b) for b in e_glob]
-    del e_glob
+    if restore:   # same graph state, same batches as the device-resident leg
+        rep.close()
+        rep = h2.Replica.from_csr(*snap0, create_ts=snap_ts0, device=dev_idx)
+        del snap0
+        e_host, e_snaps, e_glob_n = host[args.warmup:], snaps[args.warmup:], glob_n[args.warmup:]
+        e_how_state = "same graph state and batches as the device-resident leg (replica restored from a device copy)"
+    else:
+        e_glob = [wl.batch(k0 + n_total + k) for k in range(args.steps)]
+        e_host = [my_part(b) for b in e_glob]
+        e_snaps = [int(b.ts.max()) for b in e_glob]
+        e_glob_n = [len(b) for b in e_glob]
+        del e_glob
+        e_how_state = "the stream's next batches (the graph state continues from the device-resident leg)"
 
     def pinned(b):
         if records:
@@ -333,14 +429,15 @@ def run_gpu(args):
         return synth.Batch(*(tens(a).pin_memory() for a in (b.kind, b.src, b.dst, b.w, b.ts)))
 
     e_pin = [pinned(b) for b in e_host]
-    for k in range(n_ewarm):
-        apply(rep.stage(e_pin[k]), e_snaps[k])
-    e_pin, e_snaps, e_glob_n = e_pin[n_ewarm:], e_snaps[n_ewarm:], e_glob_n[n_ewarm:]
+    if pipelined:   # allocate and warm both staging slots (nothing is applied)
+        rep.stage(e_pin[0])
+        rep.stage(e_pin[min(1, len(e_pin) - 1)])
     torch.cuda.synchronize()
     if world > 1:
         dist.barrier()
     e_stats = []
     h2d0 = eng.h2d if sharded else 0
+    ev0, ev1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
     ev0.record(stream)
     if pipelined:
         # h2tap_batch_stage: the H2D copy of batch k+1 runs on the copy engine while batch k
@@ -348,11 +445,11 @@ def run_gpu(args):
         staged = rep.stage(e_pin[0])
         for k in range(args.steps):
             nxt = rep.stage(e_pin[k + 1]) if k + 1 < args.steps else None
-            e_stats.append(apply(staged, e_snaps[k]))
+            e_stats.append(apply(rep, staged, e_snaps[k]))
             staged = nxt
     else:
         for k in range(args.steps):
-            e_stats.append(apply(e_pin[k], e_snaps[k]))
+            e_stats.append(apply(rep, e_pin[k], e_snaps[k]))
     ev1.record(stream)
     torch.cuda.synchronize()
     e_ms = ev0.elapsed_time(ev1)
@@ -361,6 +458,8 @@ def run_gpu(args):
     e_updates = (sum(e_glob_n) / world if sharded else sum(s["n_visible"] for s in e_stats))
     e_ms, e_updates = reduce_max_sum(e_ms, e_updates)
     e_value = e_updates / (e_ms / 1e3)
+    if restore:
+        assert rep.info()["n_edges"] == inf1["n_edges"], "e2e replay diverged from the device-resident leg"
 
     checks = None
     if args.checks and not sharded:  # freshness checks on the final snapshot (not in updates/s)
@@ -380,6 +479,20 @@ def run_gpu(args):
             torch.cuda.synchronize()
             checks[name + "_ms"] = (time.perf_counter() - t) * 1e3
 
+    route = None
+    if sharded:
+        rb = [s.get("route_bytes", 0) for s in stats]
+        xms = [s.get("ms_exchange", 0.0) for s in stats]
+        route = {"bytes_per_step_this_rank": sum(rb) / len(rb), "ms_per_step_this_rank": sum(xms) / len(xms),
+                 "exchange": args.exchange, "backend": args.dist_backend}
+        route["achieved_gbs"] = (route["bytes_per_step_this_rank"] / (route["ms_per_step_this_rank"] / 1e3) / 1e9
+                                 if route["ms_per_step_this_rank"] > 0 else None)
+        route["peak_gbs"] = 900.0
+        route["peak_source"] = "NVLink 5 per direction per GPU (nominal, north_star)"
+        route["frac"] = route["achieved_gbs"] / 900.0 if route["achieved_gbs"] else None
+        route["note"] = ("bytes = 40-byte route records this rank sends to other ranks; time = CUDA events "
+                         "around pack + exchange on the replica stream (rank 0)")
+
     if rank == 0:
         peak, peak_src = peaks()
         mean = lambda key: sum(s[key] for s in stats) / len(stats)  # noqa: E731
@@ -389,7 +502,6 @@ def run_gpu(args):
         path_bytes = mean("bytes_alg")
         ms_step = ms / len(stats)
         path_gbs = path_bytes / (ms_step / 1e3) / 1e9
-        info = rep.info()
         try:  # DRAM bytes per launch of the same kernel from the committed ncu --set full capture
             traffic = (None if sharded else  # captured for the unsharded merge only
                        json.load(open(os.path.join(ROOT, "profiles", "traffic.json"))).get(args.config))
@@ -405,11 +517,19 @@ def run_gpu(args):
                            f"all-to-all routing over {args.dist_backend})" if args.exchange == "alltoall" else
                            "fused pack-and-store into peer CUDA-IPC windows)")
                         if sharded else "replicas" if world > 1 else "single"),
-                       "l2": "inputs larger than L2 (CSR ~%.1f GB per step)" % (path_bytes / 1e9),
-                       "replica_vertices": info["n_vertices"], "replica_edges": info["n_edges"]},
-            "roofline": {"bound": "hbm", "kernel": "k_merge", "achieved": achieved, "peak": peak,
+                       "l2": "inputs larger than L2 (CSR ~%.1f GB per step)" % (path_bytes / 1e9)
+                       if path_bytes > 2e8 else "L2-resident (C1: latency line, see step_ms)"},
+            "replica": {"vertices_start": inf0["n_vertices"], "edges_start": inf0["n_edges"],
+                        "vertices_end": inf1["n_vertices"], "edges_end": inf1["n_edges"],
+                        "edges_per_step": e_steps,
+                        "note": ("node deletes cascade (hub-first, the paper's HiDeg window): the graph shrinks "
+                                 "batch to batch" if wl.cfg["kind"] == "ldbc" else "")},
+            "step_ms": {"p10": pct(step_ms, 0.1), "p50": pct(step_ms, 0.5), "p90": pct(step_ms, 0.9),
+                        "min": min(step_ms), "max": max(step_ms),
+                        "how": "CUDA events between consecutive applies on the replica stream (rank 0)"},
+            "roofline": {"bound": "hbm", "kernel": "k_merge3", "achieved": achieved, "peak": peak,
                          "unit": "GB/s", "frac": achieved / peak, "traffic": traffic,
-                         "traffic_source": "ncu --set full, profiles/r1/summary.json (dram read+write per launch)",
+                         "traffic_source": "ncu --set full (profiles/traffic.json: dram read+write per launch)",
                          "peak_source": peak_src, "bytes_per_launch": merge_bytes,
                          "ms_per_launch": merge_ms},
             "path": {"bytes_alg_per_step": path_bytes, "achieved_gbs": path_gbs,
@@ -420,21 +540,21 @@ def run_gpu(args):
             "gpu_launches": int(sum(s["n_launches"] for s in stats)),
             "e2e": {"value": e_value, "unit": "updates/s",
                     "how": ("pinned host batches; h2tap_batch_stage copies batch k+1 while batch k is applied"
-                            if pipelined else "pinned host batches copied inside each apply"),
+                            if pipelined else "pinned host batches copied inside each apply") + "; " + e_how_state,
                     "h2d_bytes_per_step": int(sum(s["h2d_bytes"] for s in e_stats) / len(e_stats)),
                     "d2h_bytes_per_step": int(sum(s["d2h_bytes"] for s in e_stats) / len(e_stats))},
             "clocks": clk.summary(),
         }
+        if route:
+            line["nvlink"] = route
         if records:
             line["config"]["input"] = "delta records (paper §5.1 layout, h2tap_delta_apply_records)"
         if args.tombstone:
             line["config"]["id_mode"] = "tombstone rows (reading A23)"
         if checks:
             line["checks"] = checks
-        if not args.no_cpu_baseline:
-            v, sample, _ = oracle_sample(args.config, 3, 1, target_s=8.0)
-            line["cpu_baseline"] = {"value": v, "unit": "updates/s", "cores": 1, "kind": "oracle",
-                                    "sample": sample}
+        if not args.no_cpu_baseline and world == 1:
+            line["cpu_baseline"] = o3_baseline(args.config)
         print(json.dumps(line), flush=True)
     rep.close()
     if world > 1:
@@ -461,12 +581,26 @@ def cpu_baseline_dyn(scale: int = 16, records: int = 20000, cycles: int = 3):
             "sample": f"OD on RMAT-{scale} x16, {cycles} cycles of {records} records (edge-only), apply only"}
 
 
+def spawn(args) -> int:
+    """--gpus N > 1 without a launcher: start N ranks of this script (one per GPU) with
+    torch.distributed.run on 127.0.0.1; rank 0 prints the line."""
+    import socket
+    with socket.socket() as so:
+        so.bind(("127.0.0.1", 0))
+        port = so.getsockname()[1]
+    cmd = [sys.executable, "-m", "torch.distributed.run", "--nnodes=1", f"--nproc-per-node={args.gpus}",
+           "--master-addr=127.0.0.1", f"--master-port={port}", os.path.abspath(__file__)] + sys.argv[1:]
+    return subprocess.call(cmd)
+
+
 def main():
     ap = argparse.ArgumentParser()
     ap.add_argument("--gpus", type=int, default=1)
     ap.add_argument("--steps", type=int, default=20)
     ap.add_argument("--warmup", type=int, default=3)
-    ap.add_argument("--config", default="c2", choices=sorted(synth.CONFIGS))
+    ap.add_argument("--config", default=None, choices=sorted(synth.CONFIGS),
+                    help="default: c2 (BASELINE.json configs[1], the metric's config) on 1 GPU; c4 "
+                         "(configs[3], RMAT-26, the scaling config) when --gpus > 1")
     ap.add_argument("--impl", default="h2tap", choices=["h2tap", "reference"])
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--input", default="ops", choices=["ops", "records"],
@@ -488,6 +622,12 @@ def main():
     import bench_dyn
     bench_dyn.add_args(ap)
     args = ap.parse_args()
+    if args.config is None:
+        args.config = "c2" if args.gpus == 1 else "c4"
+    if args.gpus > 1 and "WORLD_SIZE" not in os.environ:
+        raise SystemExit(spawn(args))
+    if int(os.environ.get("WORLD_SIZE", "1")) != args.gpus:
+        raise SystemExit(f"bench.py: --gpus {args.gpus} but WORLD_SIZE={os.environ.get('WORLD_SIZE')}")
     if args.replica == "dyn":
         if args.impl != "h2tap" or args.gpus != 1:
             raise SystemExit("--replica dyn: single GPU, own implementation only")

@@ -30,6 +30,7 @@ constexpr int kRsSmem = kRsTile * 12;           // dynamic smem: staged keys + v
 constexpr int kRsWarps = kRsThreads / 32;
 constexpr int kRsMaxPasses = 8;
 constexpr int kRsLook = H2TAP_RS_LOOK;  // look-back: predecessor tiles read per step
+constexpr uint32_t kRsDirectTiles = 128;  // rs_coop: tiles up to which every CTA sums the count columns itself
 
 // n_dev (nullable): the key count lives in device memory (no host sync before the
 // sort); `n` is then an upper bound that only sizes the grids
@@ -302,21 +303,33 @@ __global__ void __launch_bounds__(kRsThreads, ITEMS >= 12 ? 3 : 4) rs_coop(
         s_dstart[tid] = ds;
         cnt[(uint64_t)b * 256 + tid] = c;
         rs_grid_sync(bar, target);
-        // column scans: digit d over the T tiles (exclusive, in place), total -> tot[d]
-        for (uint32_t d = b; d < 256; d += T) {
-            uint32_t carry = 0;
-            for (uint32_t t0 = 0; t0 < T; t0 += kRsThreads) {
-                const uint32_t t = t0 + tid;
-                const uint32_t x = t < T ? cnt[(uint64_t)t * 256 + d] : 0u;
-                uint32_t sum;
-                const uint32_t e = block_exclusive_scan<kRsThreads>(x, s_scan, &sum);
-                if (t < T) cnt[(uint64_t)t * 256 + d] = carry + e;
-                carry += sum;
+        if (T <= kRsDirectTiles) {
+            // few tiles: thread d of every CTA sums column d itself (T coalesced 1 KB rows):
+            // its tile's prefix and the digit total, no second barrier
+            uint32_t pre = 0, all = 0;
+            for (uint32_t t = 0; t < T; ++t) {
+                const uint32_t x = cnt[(uint64_t)t * 256 + tid];
+                pre += t < b ? x : 0u;
+                all += x;
             }
-            if (tid == 0) tot[d] = carry;
-        }
-        rs_grid_sync(bar, target);
-        {
+            uint32_t sum;
+            const uint32_t db = block_exclusive_scan<kRsThreads>(all, s_scan, &sum);
+            s_gpre[tid] = db + pre;
+        } else {
+            // column scans: digit d by CTA d mod T (exclusive over tiles, in place), total -> tot[d]
+            for (uint32_t d = b; d < 256; d += T) {
+                uint32_t carry = 0;
+                for (uint32_t t0 = 0; t0 < T; t0 += kRsThreads) {
+                    const uint32_t t = t0 + tid;
+                    const uint32_t x = t < T ? cnt[(uint64_t)t * 256 + d] : 0u;
+                    uint32_t sum;
+                    const uint32_t e = block_exclusive_scan<kRsThreads>(x, s_scan, &sum);
+                    if (t < T) cnt[(uint64_t)t * 256 + d] = carry + e;
+                    carry += sum;
+                }
+                if (tid == 0) tot[d] = carry;
+            }
+            rs_grid_sync(bar, target);
             uint32_t sum;
             const uint32_t db = block_exclusive_scan<kRsThreads>(tot[tid], s_scan, &sum);
             s_gpre[tid] = db + cnt[(uint64_t)b * 256 + tid];

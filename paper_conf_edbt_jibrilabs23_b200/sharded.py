@@ -142,7 +142,8 @@ class _Ptr:
 
 
 class ShardedReplica:
-    def __init__(self, engine, rank: int, world: int, device, group=None, exchange: str = "alltoall"):
+    def __init__(self, engine, rank: int, world: int, device, group=None, exchange: str = "alltoall",
+                 time_exchange: bool = False):
         """exchange: "alltoall" (pack, then all-to-all over the process group) or "p2p"
         (h2tap_route_pack_p2p stores every record straight into its destination's
         CUDA-IPC window: the fused pack-and-exchange kernel; world <= 16)."""
@@ -158,6 +159,8 @@ class ShardedReplica:
         # copies (tests / several ranks sharing one GPU); NCCL works on device memory
         self.coll = torch.device("cpu") if dist.get_backend(group) == "gloo" else self.device
         self.next_seq = 0
+        # CUDA events around pack + exchange (stats["ms_exchange"]; CUDA engines only)
+        self.time_exchange = time_exchange and self.device.type == "cuda"
 
     def _i64(self, vals):
         return torch.tensor(vals, dtype=torch.int64, device=self.coll)
@@ -181,6 +184,9 @@ class ShardedReplica:
         C = M[:, 2:]                                                      # C[s][d]
         seq0 = self.next_seq + sum(sizes[: self.rank])
         self.last_route_bytes = int(C[self.rank].sum() - C[self.rank][self.rank]) * ROUTE_REC_BYTES
+        if self.time_exchange:
+            ex0, ex1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+            ex0.record()
         if self.exchange == "p2p":
             recv, n_recv = self._exchange_p2p(batch, seq0, C)
         else:
@@ -192,6 +198,8 @@ class ShardedReplica:
             dist.all_to_all_single(recv, recs.to(self.coll), [c * ROUTE_REC_BYTES for c in rc],
                                    [int(c) * ROUTE_REC_BYTES for c in C[self.rank]], group=self.group)
             recv, n_recv = recv.to(recs.device), sum(rc)
+        if self.time_exchange:
+            ex1.record()
         # 4. two-phase apply: prepare everywhere, agree, then all commit or all abort
         try:
             status, stats = self.engine.prepare_routed(recv, n_recv, snapshot_ts)
@@ -208,6 +216,9 @@ class ShardedReplica:
         self.next_seq += sum(sizes)
         stats["global_batch"] = sum(sizes)
         stats["route_bytes"] = self.last_route_bytes
+        if self.time_exchange:
+            ex1.synchronize()
+            stats["ms_exchange"] = ex0.elapsed_time(ex1)
         return stats
 
     def _windows(self, need):

@@ -350,6 +350,8 @@ def test_two_phase_prepare_commit_abort(h2):
     o.apply(b, snap)
     assert_same(g.export(), o.export(), "two-phase commit")
     assert g.info()["snapshot_ts"] == snap
+    assert g.info()["n_edges"] == step.last_E[id(g)] + st["n_new"] - st["n_del"] - st["n_casc"]   # I6
+    step.last_E[id(g)] = g.info()["n_edges"]
     with pytest.raises(h2.H2tapError):
         g.commit()                                     # nothing prepared
     b2 = synth.ldbc_batch(shape, seed, 1, 3000, ts_base=snap)

@@ -9,6 +9,9 @@
 #include <vector>
 
 #include "../paper_conf_edbt_jibrilabs23_b200/csrc/radix_sort.cuh"
+#ifndef SB_ITEMS
+#define SB_ITEMS 12
+#endif
 
 using namespace h2tap;
 
@@ -57,7 +60,7 @@ int main() {
     int occ4 = 0, occ12 = 0, sms = 0;
     cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, 0);
     cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ4, rs_coop<4>, kRsThreads, 1024 * 12);
-    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ12, rs_coop<12>, kRsThreads, 3072 * 12);
+    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ12, rs_coop<SB_ITEMS>, kRsThreads, 256 * SB_ITEMS * 12);
     printf("SMs %d occ<4> %d occ<12> %d\n", sms, occ4, occ12);
     // barrier cost
     for (int g : {10, 100, 296, 444}) {
@@ -91,8 +94,11 @@ int main() {
             for (int rep = 0; rep < 5; ++rep) {
                 CK(cudaMemcpy(k0, hk.data(), n * 8, cudaMemcpyHostToDevice));
                 CK(cudaMemcpy(v0, hv.data(), n * 4, cudaMemcpyHostToDevice));
+#ifndef SB_ITEMS
+#define SB_ITEMS 12
+#endif
                 float ms = n <= (1u << 18) ? run_coop<4>(k0, v0, k1, v1, n, passes, scratch)
-                                           : run_coop<12>(k0, v0, k1, v1, n, passes, scratch);
+                                           : run_coop<SB_ITEMS>(k0, v0, k1, v1, n, passes, scratch);
                 best = std::min(best, ms);
             }
             std::vector<uint64_t> ok(n);

@@ -187,6 +187,9 @@ typedef struct {  /* all arrays caller-owned, read-only, not retained; host or d
     const h2tap_delta_record* records;
     const uint64_t* inserts; const float* weights; size_t n_inserts;
     const uint64_t* deletes; size_t n_deletes;
+    /* the paper's 8-byte weights: when non-NULL they are used instead of
+     * `weights` and narrowed to the replica's f32 by round-to-nearest-even (reading A15) */
+    const double* weights64;
 } h2tap_record_batch;
 
 /* One propagation cycle from delta records: the delta-store scan (§5.2)
@@ -199,6 +202,51 @@ typedef struct {  /* all arrays caller-owned, read-only, not retained; host or d
  * flag other than 0/1 -> E_INVAL (nothing applied). */
 h2tap_status h2tap_delta_apply_records(h2tap_replica* r, const h2tap_record_batch* batch,
         uint64_t snapshot_ts, h2tap_apply_stats* stats /* nullable */);
+
+/* ---- the append-only delta store (§5.1 "Delta Store Architecture"; Fig. 2)
+ * and the propagation cycle that scans it (§5.2-§5.3) — SURVEY.md §8(f) NEXT-1.
+ * Host side: a delta table of fixed-size chunks of h2tap_delta_record plus the inserts /
+ * weights (8-byte) / deletes arrays, chunked alike, in pinned memory.  A
+ * committing transaction appends one delta per node it changed (append-only: no lookups of
+ * other deltas, no updates); appends are thread-safe and published in index order.  The
+ * store keeps a device mirror of its unconsumed tail on `device` (copied asynchronously on
+ * the store's own copy stream).  Ownership: the store owns all its memory; appended arrays
+ * are copied in and not retained.  Errors: E_INVAL (null / bad flags / bad slices),
+ * E_NOMEM, E_CAPACITY (more than 65536 chunks), E_CUDA. */
+typedef struct h2tap_delta_store h2tap_delta_store;
+/* chunk_records: records per chunk (rounded up to a power of two, >= 1024, <= 2^24);
+ * payload chunks hold 4 x chunk_records elements. */
+h2tap_status h2tap_ds_create(int device, size_t chunk_records, h2tap_delta_store** out);
+/* one delta: transaction ts, node, inserted / deleted flags (0/1), n_ins destination IDs with
+ * their 8-byte weights, n_del deleted destination IDs; valid = 1 */
+h2tap_status h2tap_ds_append(h2tap_delta_store* s, uint64_t ts, uint64_t node, int inserted, int deleted,
+        const uint64_t* inserts, const double* weights, uint32_t n_ins, const uint64_t* deletes, uint32_t n_del);
+/* n deltas at once (one bulk commit, host arrays): records[i].ins_off / del_off index the
+ * given arrays (rebased to the store's positions); every record must have valid = 1 */
+h2tap_status h2tap_ds_append_records(h2tap_delta_store* s, const h2tap_delta_record* records, size_t n,
+        const uint64_t* inserts, const double* weights, size_t n_inserts, const uint64_t* deletes,
+        size_t n_deletes);
+/* n_records = published deltas; first_pending = index of the first delta that may still be
+ * valid (everything before it was used and its host chunks may be released); n_mirrored =
+ * deltas copied to the device; host_bytes / device_bytes = memory held (any may be NULL) */
+h2tap_status h2tap_ds_info(const h2tap_delta_store* s, uint64_t* n_records, uint64_t* first_pending,
+        uint64_t* n_mirrored, uint64_t* host_bytes, uint64_t* device_bytes);
+/* copy deltas [first, first + n) of the live window [first_pending, n_records) with their
+ * current validity flags and absolute array offsets into `out` (host) */
+h2tap_status h2tap_ds_export(h2tap_delta_store* s, uint64_t first, size_t n, h2tap_delta_record* out);
+void h2tap_ds_destroy(h2tap_delta_store* s);
+/* One propagation cycle from the store: the scan covers every published delta from
+ * first_pending on (trailing 1024-delta blocks whose deltas all have ts > snapshot_ts are
+ * invisible and left for later; their copy to the device starts now and overlaps this
+ * cycle), keeps the valid and visible ones (valid flag set, ts <= snapshot_ts),
+ * expands them as h2tap_delta_apply_records does (reading A22; weights narrowed to f32 by
+ * round-to-nearest-even) and applies them.  On success every delta it used is marked invalid
+ * ("by the end of the delta store scan" P:L721-725) and first_pending advances; on
+ * any error nothing is marked and the replica is unchanged (strong guarantee).  A valid
+ * delta with ts <= the replica's current snapshot -> E_STALE_TS (reading A20).  stats:
+ * h2d_bytes = the store's bytes copied to the device by this call. */
+h2tap_status h2tap_delta_apply_store(h2tap_replica* r, h2tap_delta_store* s, uint64_t snapshot_ts,
+        h2tap_apply_stats* stats /* nullable */);
 
 /* ---- exchange step of a sharded apply ----------------------
  * A rank holding a slice of the global batch (i) validates it (every rank must agree

@@ -19,6 +19,8 @@ input generator ``synth``, which holds none of the method's arithmetic).
 * ``OD``  (od_dynamic.py): the dynamic replica's update (Algorithm 1).
 * ``expand_records``: the delta-store scan of the paper's record layout
   (§5.1-5.2) into the flat op sequence O1 replays.
+* ``DeltaStoreModel``: the append-only delta store and its per-cycle consistency
+  check (§5.1-5.3) as a plain Python list (valid + visible deltas are used once).
 * ``checksum``: position-keyed 64-bit checksum of an exported array (the
   comparison key for large exports; written here independently of the CUDA
   export's own checksum kernel).
@@ -276,6 +278,44 @@ def expand_records(records, inserts, weights, deletes):
         if r["deleted"]:
             op(1, v, 0, 0.0, t)                                  # NODE_DELETE
     return kind, src, dst, w, ts
+
+
+class DeltaStoreModel:
+    """The delta store of §5.1 and the scan's consistency check of §5.2-5.3
+    (P:L702-769), written out plainly: an append-only list of delta records (ts, node,
+    inserted / deleted flags, validity flag, slices of the inserts / weights / deletes
+    arrays; the weights are 8-byte).  A propagation cycle with snapshot S
+    takes, in append order, every record that is valid and visible (ts <= S; an invisible
+    one waits for a later cycle, P:L763-766), expands them (expand_records, reading A22;
+    the 8-byte weights rounded to the replica's f32 by round-to-nearest-even, reading A15)
+    and marks them invalid (each delta is used once)."""
+
+    def __init__(self):
+        self.records, self.inserts, self.weights, self.deletes = [], [], [], []
+
+    def append(self, ts, node, inserts=(), weights=(), deletes=(), inserted=False, deleted=False):
+        self.records.append(dict(ts=int(ts), node=int(node), ins_off=len(self.inserts), ins_cnt=len(inserts),
+                                 del_off=len(self.deletes), del_cnt=len(deletes), valid=1,
+                                 inserted=int(bool(inserted)), deleted=int(bool(deleted))))
+        self.inserts += [int(x) for x in inserts]
+        self.weights += [float(x) for x in weights]
+        self.deletes += [int(x) for x in deletes]
+
+    def append_records(self, recs, inserts, weights, deletes):
+        for r in recs:
+            io, ic, do, dc = int(r["ins_off"]), int(r["ins_cnt"]), int(r["del_off"]), int(r["del_cnt"])
+            self.append(r["ts"], r["node"], inserts[io:io + ic], [float(x) for x in weights[io:io + ic]],
+                        deletes[do:do + dc], r["inserted"], r["deleted"])
+
+    def cycle(self, snapshot_ts):
+        """the valid and visible deltas of this cycle as flat ops (kind, src, dst, w, ts);
+        they are marked invalid"""
+        used = [r for r in self.records if r["valid"] and r["ts"] <= snapshot_ts]
+        w32 = np.asarray(self.weights, np.float64).astype(np.float32)  # RN-even narrowing
+        ops = expand_records(used, self.inserts, w32, self.deletes)
+        for r in used:
+            r["valid"] = 0
+        return ops
 
 
 def bfs(offsets, cols, source_dense: int) -> np.ndarray:

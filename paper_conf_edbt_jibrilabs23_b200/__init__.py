@@ -62,10 +62,39 @@ class _Batch(ctypes.Structure):
 class _RecordBatch(ctypes.Structure):
     _fields_ = [("n_records", ctypes.c_size_t), ("on_device", ctypes.c_int), ("records", _P),
                 ("inserts", _P), ("weights", _P), ("n_inserts", ctypes.c_size_t),
-                ("deletes", _P), ("n_deletes", ctypes.c_size_t)]
+                ("deletes", _P), ("n_deletes", ctypes.c_size_t), ("weights64", _P)]
 
 
 RECORD_BYTES = 48  # sizeof(h2tap_delta_record)
+
+
+def _is_f64(a) -> bool:
+    if a is None:
+        return False
+    if _is_torch(a):
+        import torch
+        return a.dtype == torch.float64
+    return np.asarray(a).dtype == np.float64
+
+
+def _record_batch(rb):
+    """(h2tap_record_batch, keepalive) for rb (.records .inserts .weights .deletes); f64
+    weights go through weights64 (the paper's 8-byte weights), f32 through weights."""
+    w64 = _is_f64(rb.weights)
+    pr, pi, pd = _ptr(rb.records), _ptr(rb.inserts, np.uint64), _ptr(rb.deletes, np.uint64)
+    pw = _ptr(rb.weights, np.float64 if w64 else np.float32)
+    b = _RecordBatch()
+    recs = pr[2]
+    nbytes = recs.numel() * recs.element_size() if _is_torch(recs) else recs.nbytes
+    if nbytes % RECORD_BYTES:
+        raise ValueError("records buffer is not a whole number of 48-byte records")
+    b.n_records = nbytes // RECORD_BYTES
+    b.on_device = _on_device(pr, pi, pw, pd)
+    b.records, b.inserts, b.deletes = pr[0], pi[0], pd[0]
+    b.weights, b.weights64 = (None, pw[0]) if w64 else (pw[0], None)
+    b.n_inserts = len(pi[2]) if pi[2] is not None else 0
+    b.n_deletes = len(pd[2]) if pd[2] is not None else 0
+    return b, (pr, pi, pw, pd)
 
 
 class ApplyStats(ctypes.Structure):
@@ -111,6 +140,13 @@ for _n, _a in (("h2tap_batch_stage", [_P, ctypes.POINTER(_Batch), ctypes.POINTER
                ("h2tap_delta_apply_prepare", [_P, ctypes.POINTER(_Batch), _u64, ctypes.POINTER(ApplyStats)]),
                ("h2tap_delta_apply_routed_prepare", [_P, _P, ctypes.c_size_t, _u64, ctypes.POINTER(ApplyStats)]),
                ("h2tap_delta_commit", [_P]),
+               ("h2tap_ds_create", [ctypes.c_int, ctypes.c_size_t, ctypes.POINTER(_P)]),
+               ("h2tap_ds_append", [_P, _u64, _u64, ctypes.c_int, ctypes.c_int, _P, _P, ctypes.c_uint32, _P,
+                                    ctypes.c_uint32]),
+               ("h2tap_ds_append_records", [_P, _P, ctypes.c_size_t, _P, _P, ctypes.c_size_t, _P, ctypes.c_size_t]),
+               ("h2tap_ds_info", [_P] + [ctypes.POINTER(_u64)] * 5),
+               ("h2tap_ds_export", [_P, _u64, ctypes.c_size_t, _P]),
+               ("h2tap_delta_apply_store", [_P, _P, _u64, ctypes.POINTER(ApplyStats)]),
                ("h2tap_delta_abort", [_P]),
                ("h2tap_route_pack_p2p", [_P, ctypes.POINTER(_Batch), _u64, _P, _P]),
                ("h2tap_ipc_alloc", [ctypes.c_int, ctypes.c_size_t, ctypes.POINTER(_P), _P]),
@@ -131,6 +167,8 @@ _lib.h2tap_replica_liveness.restype = ctypes.c_int
 _lib.h2tap_replica_liveness.argtypes = [_P, _P, ctypes.c_int]
 _lib.h2tap_pagerank.restype = ctypes.c_int
 _lib.h2tap_pagerank.argtypes = [_P, ctypes.c_double, ctypes.c_int, _P, ctypes.c_int]
+_lib.h2tap_ds_destroy.restype = None
+_lib.h2tap_ds_destroy.argtypes = [_P]
 _lib.h2tap_replica_destroy.restype = None
 _lib.h2tap_replica_destroy.argtypes = [_P]
 _lib.h2tap_status_str.restype = ctypes.c_char_p
@@ -394,23 +432,22 @@ class Replica:
 
     def apply_records(self, rb, snapshot_ts: int, raise_on_error: bool = True):
         """h2tap_delta_apply_records; rb has .records (48-byte records: a numpy structured
-        array, or a torch CUDA uint8 tensor) .inserts .weights .deletes."""
-        pr, pi, pw, pd = (_ptr(rb.records), _ptr(rb.inserts, np.uint64), _ptr(rb.weights, np.float32),
-                          _ptr(rb.deletes, np.uint64))
-        b = _RecordBatch()
-        recs = pr[2]
-        nbytes = recs.numel() * recs.element_size() if _is_torch(recs) else recs.nbytes
-        if nbytes % RECORD_BYTES:
-            raise ValueError("records buffer is not a whole number of 48-byte records")
-        b.n_records = nbytes // RECORD_BYTES
-        b.on_device = _on_device(pr, pi, pw, pd)
-        b.records, b.inserts, b.weights, b.deletes = pr[0], pi[0], pw[0], pd[0]
-        b.n_inserts = len(pi[2]) if pi[2] is not None else 0
-        b.n_deletes = len(pd[2]) if pd[2] is not None else 0
+        array, or a torch CUDA uint8 tensor) .inserts .weights (f32, or f64 = the paper's
+        8-byte weights) .deletes."""
+        b, keep = _record_batch(rb)
         st = ApplyStats()
         rc = _lib.h2tap_delta_apply_records(self._h, ctypes.byref(b), int(snapshot_ts), ctypes.byref(st))
         if raise_on_error:
             _check(rc, "h2tap_delta_apply_records")
+            return st.as_dict()
+        return rc, st.as_dict()
+
+    def apply_store(self, store: "DeltaStore", snapshot_ts: int, raise_on_error: bool = True):
+        """h2tap_delta_apply_store: one propagation cycle from an append-only delta store."""
+        st = ApplyStats()
+        rc = _lib.h2tap_delta_apply_store(self._h, store._h, int(snapshot_ts), ctypes.byref(st))
+        if raise_on_error:
+            _check(rc, "h2tap_delta_apply_store")
             return st.as_dict()
         return rc, st.as_dict()
 
@@ -576,18 +613,7 @@ class DynReplica:
 
     def apply_records(self, rb, raise_on_error: bool = True):
         """h2tap_dyn_apply_records on rb (.records .inserts .weights .deletes, host or device)."""
-        pr, pi, pw, pd = (_ptr(rb.records), _ptr(rb.inserts, np.uint64), _ptr(rb.weights, np.float32),
-                          _ptr(rb.deletes, np.uint64))
-        b = _RecordBatch()
-        recs = pr[2]
-        nbytes = recs.numel() * recs.element_size() if _is_torch(recs) else recs.nbytes
-        if nbytes % RECORD_BYTES:
-            raise ValueError("records buffer is not a whole number of 48-byte records")
-        b.n_records = nbytes // RECORD_BYTES
-        b.on_device = _on_device(pr, pi, pw, pd)
-        b.records, b.inserts, b.weights, b.deletes = pr[0], pi[0], pw[0], pd[0]
-        b.n_inserts = len(pi[2]) if pi[2] is not None else 0
-        b.n_deletes = len(pd[2]) if pd[2] is not None else 0
+        b, keep = _record_batch(rb)
         st = ApplyStats()
         rc = _lib.h2tap_dyn_apply_records(self._h, ctypes.byref(b), ctypes.byref(st))
         if raise_on_error:
@@ -633,3 +659,57 @@ class DynReplica:
 
     def __exit__(self, *a):
         self.close()
+
+
+class DeltaStore:
+    """The paper's append-only delta store (§5.1, Fig. 2; h2tap_ds_*): a chunked table of
+    delta records + inserts / 8-byte weights / deletes arrays on the host, mirrored to the GPU
+    by the propagation cycle (Replica.apply_store)."""
+
+    def __init__(self, device: int = 0, chunk_records: int = 1 << 16):
+        h = _P()
+        _check(_lib.h2tap_ds_create(int(device), int(chunk_records), ctypes.byref(h)), "h2tap_ds_create")
+        self._h = h
+
+    def append(self, ts: int, node: int, inserts=(), weights=(), deletes=(), inserted=False, deleted=False):
+        """one delta: transaction ts, node, its inserted (dst, 8-byte weight) and deleted dsts"""
+        i = np.ascontiguousarray(inserts, np.uint64)
+        w = np.ascontiguousarray(weights, np.float64)
+        d = np.ascontiguousarray(deletes, np.uint64)
+        if len(i) != len(w):
+            raise ValueError("inserts and weights differ in length")
+        _check(_lib.h2tap_ds_append(self._h, int(ts), int(node), int(bool(inserted)), int(bool(deleted)),
+                                    ctypes.c_void_p(i.ctypes.data), ctypes.c_void_p(w.ctypes.data), len(i),
+                                    ctypes.c_void_p(d.ctypes.data), len(d)), "h2tap_ds_append")
+
+    def append_records(self, rb):
+        """a bulk commit of host records (rb.records with valid = 1; weights f32 or f64)"""
+        rec = np.ascontiguousarray(rb.records)
+        i = np.ascontiguousarray(rb.inserts, np.uint64)
+        w = np.ascontiguousarray(rb.weights, np.float64)
+        d = np.ascontiguousarray(rb.deletes, np.uint64)
+        _check(_lib.h2tap_ds_append_records(self._h, ctypes.c_void_p(rec.ctypes.data), len(rec),
+                                            ctypes.c_void_p(i.ctypes.data), ctypes.c_void_p(w.ctypes.data), len(i),
+                                            ctypes.c_void_p(d.ctypes.data), len(d)), "h2tap_ds_append_records")
+
+    def info(self):
+        v = [_u64() for _ in range(5)]
+        _check(_lib.h2tap_ds_info(self._h, *(ctypes.byref(x) for x in v)), "h2tap_ds_info")
+        return dict(n_records=v[0].value, first_pending=v[1].value, n_mirrored=v[2].value,
+                    host_bytes=v[3].value, device_bytes=v[4].value)
+
+    def export(self, first: int, n: int):
+        """records [first, first + n) of the live window, current validity flags"""
+        from synth import RECORD_DTYPE
+        out = np.zeros(n, RECORD_DTYPE)
+        _check(_lib.h2tap_ds_export(self._h, int(first), int(n), ctypes.c_void_p(out.ctypes.data)), "h2tap_ds_export")
+        return out
+
+    def close(self):
+        if getattr(self, "_h", None):
+            _lib.h2tap_ds_destroy(self._h)
+            self._h = None
+
+    def __del__(self):
+        self.close()
+

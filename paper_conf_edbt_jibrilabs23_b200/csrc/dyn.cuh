@@ -528,6 +528,7 @@ h2tap_status dyn_apply(h2tap_dyn* d, const h2tap_record_batch* b, h2tap_apply_st
     const float* wts = b->weights;
     const uint64_t* del = b->deletes;
     if (nr && !rec) { set_err("records is NULL"); return H2TAP_E_INVAL; }
+    if (b->weights64) { set_err("the dynamic replica takes f32 weights (weights64 is for the CSR replica)"); return H2TAP_E_INVAL; }
     if ((b->n_inserts && (!ins || !wts)) || (b->n_deletes && !del)) { set_err("null inserts/weights/deletes"); return H2TAP_E_INVAL; }
     if (!b->on_device) {
         DeltaRec* xr = r->get<DeltaRec>(d->x_rec, nr);

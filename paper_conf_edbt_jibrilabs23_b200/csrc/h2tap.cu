@@ -17,7 +17,10 @@
 #include <cstdlib>
 #include <cstdio>
 #include <cstring>
+#include <atomic>
+#include <mutex>
 #include <new>
+#include <thread>
 #include <string>
 #include <vector>
 
@@ -297,6 +300,8 @@ struct BatchIn {
     uint64_t n_drec = 0;
     const uint64_t *drec_off = nullptr, *dins = nullptr, *ddel = nullptr;
     const float* dwts = nullptr;
+    const double* dwts64 = nullptr;                  // 8-byte weights (narrowed to f32)
+    uint64_t vis_ts = ~0ull, ins_base = 0, del_base = 0;  // delta-store scan: visibility, window bases
     uint64_t pre_h2d = 0, pre_d2h = 0, pre_launches = 0;  // accounting of the record pre-pass
 };
 
@@ -397,7 +402,8 @@ h2tap_status apply_core(h2tap_replica* r, const BatchIn& in, uint64_t S, bool cr
     } else if (n && in.drec) {
         const unsigned grid = (unsigned)std::min<uint64_t>(cdiv(in.n_drec * 32, 256), (uint64_t)r->n_sm * 16);
         k_rec_expand<<<grid, 256, 0, st>>>(in.drec, in.n_drec, in.drec_off, in.dins, in.dwts, in.ddel,
-                                           Wk + np, Ws + np, Wd + np, Ww + np, Wt + np);
+                                           Wk + np, Ws + np, Wd + np, Ww + np, Wt + np, in.dwts64, in.vis_ts,
+                                           in.ins_base, in.del_base);
         CKL();
         k_fill_seq<<<g1(n), 256, 0, st>>>(Wq, np, n, r->next_seq);
         CKL();
@@ -1322,11 +1328,60 @@ h2tap_status h2tap_batch_stage(h2tap_replica* r, const h2tap_batch* host, h2tap_
     });
 }
 
+}  // extern "C"
+
+namespace {
+// One cycle from delta records that are in device memory: the delta-store scan (§5.2) -
+// validity / visibility per record, op counts, placement scan, expansion into the
+// work-op SoA - then the flat pipeline.  rec / ins / w / del are device pointers; the
+// payload arrays hold absolute positions [ins_base, ins_base + n_ins) etc.
+h2tap_status apply_records_dev(h2tap_replica* r, const DeltaRec* rec, uint64_t nr, const uint64_t* ins,
+                               const float* wts, const double* wts64, uint64_t n_ins, const uint64_t* del,
+                               uint64_t n_del, uint64_t vis_ts, uint64_t ins_base, uint64_t del_base,
+                               uint64_t snapshot_ts, h2tap_apply_stats* stats) {
+    cudaStream_t st = r->st;
+    uint64_t* cnt = r->get<uint64_t>(r->xcnt, nr + 1);
+    uint64_t* off = r->get<uint64_t>(r->xoff, nr + 1);
+    unsigned long long* tb = r->get<unsigned long long>(r->misc, 2);
+    CK(cudaMemsetAsync(tb, 0, 16, st));
+    if (nr) {
+        k_rec_count<<<g1(nr), 256, 0, st>>>(rec, nr, n_ins, n_del, cnt, tb, vis_ts, ins_base, del_base);
+        CKL();
+        const uint64_t nt = cdiv(nr, kTile);
+        uint64_t* stt = r->get<uint64_t>(r->status2, nt);
+        unsigned int* ctr = reinterpret_cast<unsigned int*>(r->get<uint64_t>(r->tsum, 1));
+        CK(cudaMemsetAsync(stt, 0, nt * 8, st));
+        CK(cudaMemsetAsync(ctr, 0, 4, st));
+        k_scan_exclusive_u64<<<(unsigned)nt, kThreads, 0, st>>>(cnt, off, nr, stt, ctr);
+        CKL();
+    }
+    unsigned long long h[2] = {0, 0};
+    CK(cudaMemcpyAsync(h, tb, 16, cudaMemcpyDeviceToHost, st));
+    g_d2h += 16;
+    r->sync();  // the expanded op count sizes the work buffers
+    if (h[1] & REC_BAD_FLAG) { set_err("delta record flag other than 0/1"); return H2TAP_E_INVAL; }
+    if (h[1] & REC_BAD_SLICE) { set_err("delta record slice outside the inserts/weights/deletes arrays"); return H2TAP_E_INVAL; }
+    BatchIn in{h[0], 1, nullptr, nullptr, nullptr, nullptr, nullptr, nullptr, 0};
+    in.drec = rec; in.n_drec = nr; in.drec_off = off; in.dins = ins; in.dwts = wts; in.ddel = del;
+    in.dwts64 = wts64; in.vis_ts = vis_ts; in.ins_base = ins_base; in.del_base = del_base;
+    in.pre_h2d = g_h2d; in.pre_d2h = g_d2h; in.pre_launches = g_launches;
+    const h2tap_status s = apply_core(r, in, snapshot_ts, false, stats);
+    if (s == H2TAP_OK && stats) {  // the scan pre-pass is part of ingest
+        const float pre = ev_ms(r->ev[7], r->ev[0]);
+        stats->ms_ingest += pre;
+        stats->ms_total += pre;
+    }
+    return s;
+}
+}  // namespace
+
+extern "C" {
+
 h2tap_status h2tap_delta_apply_records(h2tap_replica* r, const h2tap_record_batch* b, uint64_t snapshot_ts,
                                        h2tap_apply_stats* stats) {
     if (!r || !b) { set_err("null argument"); return H2TAP_E_INVAL; }
     if (b->n_records && !b->records) { set_err("records must be non-NULL"); return H2TAP_E_INVAL; }
-    if ((b->n_inserts && (!b->inserts || !b->weights)) || (b->n_deletes && !b->deletes)) {
+    if ((b->n_inserts && (!b->inserts || (!b->weights && !b->weights64))) || (b->n_deletes && !b->deletes)) {
         set_err("inserts/weights/deletes must be non-NULL when their size is non-zero");
         return H2TAP_E_INVAL;
     }
@@ -1336,57 +1391,35 @@ h2tap_status h2tap_delta_apply_records(h2tap_replica* r, const h2tap_record_batc
             return H2TAP_E_SNAPSHOT_REGRESSION;
         }
         CK(cudaSetDevice(r->cfg.device));
-        cudaStream_t st = r->st;
         g_launches = g_h2d = g_d2h = 0;
         if (!r->ev[7]) CK(cudaEventCreate(&r->ev[7]));
-        CK(cudaEventRecord(r->ev[7], st));
+        CK(cudaEventRecord(r->ev[7], r->st));
         const uint64_t nr = b->n_records;
         const DeltaRec* rec = reinterpret_cast<const DeltaRec*>(b->records);
         const uint64_t *ins = b->inserts, *del = b->deletes;
-        const float* wts = b->weights;
+        const float* wts = b->weights64 ? nullptr : b->weights;
+        const double* w64 = b->weights64;
         if (!b->on_device) {  // the scan reads the records where they live: copy them in once
             DeltaRec* xr = r->get<DeltaRec>(r->xrec, nr);
             copy_in(r, xr, rec, nr, 0);
             rec = xr;
             uint64_t* xi = r->get<uint64_t>(r->xins, b->n_inserts);
-            float* xw = r->get<float>(r->xwts, b->n_inserts);
             uint64_t* xd = r->get<uint64_t>(r->xdel, b->n_deletes);
             copy_in(r, xi, ins, b->n_inserts, 0);
-            copy_in(r, xw, wts, b->n_inserts, 0);
+            if (w64) {
+                double* xw = r->get<double>(r->xwts, b->n_inserts);
+                copy_in(r, xw, w64, b->n_inserts, 0);
+                w64 = xw;
+            } else {
+                float* xw = r->get<float>(r->xwts, b->n_inserts);
+                copy_in(r, xw, wts, b->n_inserts, 0);
+                wts = xw;
+            }
             copy_in(r, xd, del, b->n_deletes, 0);
-            ins = xi; wts = xw; del = xd;
+            ins = xi; del = xd;
         }
-        uint64_t* cnt = r->get<uint64_t>(r->xcnt, nr + 1);
-        uint64_t* off = r->get<uint64_t>(r->xoff, nr + 1);
-        unsigned long long* tb = r->get<unsigned long long>(r->misc, 2);
-        CK(cudaMemsetAsync(tb, 0, 16, st));
-        if (nr) {
-            k_rec_count<<<g1(nr), 256, 0, st>>>(rec, nr, b->n_inserts, b->n_deletes, cnt, tb);
-            CKL();
-            const uint64_t nt = cdiv(nr, kTile);
-            uint64_t* stt = r->get<uint64_t>(r->status2, nt);
-            unsigned int* ctr = reinterpret_cast<unsigned int*>(r->get<uint64_t>(r->tsum, 1));
-            CK(cudaMemsetAsync(stt, 0, nt * 8, st));
-            CK(cudaMemsetAsync(ctr, 0, 4, st));
-            k_scan_exclusive_u64<<<(unsigned)nt, kThreads, 0, st>>>(cnt, off, nr, stt, ctr);
-            CKL();
-        }
-        unsigned long long h[2] = {0, 0};
-        CK(cudaMemcpyAsync(h, tb, 16, cudaMemcpyDeviceToHost, st));
-        g_d2h += 16;
-        r->sync();  // the expanded op count sizes the work buffers
-        if (h[1] & REC_BAD_FLAG) { set_err("delta record flag other than 0/1"); return H2TAP_E_INVAL; }
-        if (h[1] & REC_BAD_SLICE) { set_err("delta record slice outside the inserts/weights/deletes arrays"); return H2TAP_E_INVAL; }
-        BatchIn in{h[0], 1, nullptr, nullptr, nullptr, nullptr, nullptr, nullptr, 0};
-        in.drec = rec; in.n_drec = nr; in.drec_off = off; in.dins = ins; in.dwts = wts; in.ddel = del;
-        in.pre_h2d = g_h2d; in.pre_d2h = g_d2h; in.pre_launches = g_launches;
-        const h2tap_status s = apply_core(r, in, snapshot_ts, false, stats);
-        if (s == H2TAP_OK && stats) {  // the scan pre-pass is part of ingest
-            const float pre = ev_ms(r->ev[7], r->ev[0]);
-            stats->ms_ingest += pre;
-            stats->ms_total += pre;
-        }
-        return s;
+        return apply_records_dev(r, rec, nr, ins, wts, w64, b->n_inserts, del, b->n_deletes, ~0ull, 0, 0,
+                                 snapshot_ts, stats);
     });
 }
 
@@ -1809,3 +1842,4 @@ void h2tap_replica_destroy(h2tap_replica* r) {
 }  // extern "C"
 
 #include "dyn.cuh"  // the dynamic replica (Algorithm 1), SURVEY §8(f) NEXT-3
+#include "delta_store.cuh"  // the append-only delta store (§5.1) and the cycle from it, NEXT-1

@@ -394,8 +394,12 @@ struct DeltaRec {  // layout of h2tap_delta_record
 };
 static_assert(sizeof(DeltaRec) == 48, "delta record layout");
 enum : uint32_t { REC_BAD_SLICE = 1, REC_BAD_FLAG = 2 };
+// vis_ts: only records with ts <= vis_ts expand (the delta-store scan's visibility check,
+// §5.3; UINT64_MAX for a caller-supplied batch); ins_base / del_base: absolute
+// array position of element 0 of ins / del (a store's device mirror holds a window)
 __global__ void k_rec_count(const DeltaRec* __restrict__ rec, uint64_t n, uint64_t n_ins, uint64_t n_del,
-                            uint64_t* __restrict__ cnt, unsigned long long* __restrict__ tot_bad) {
+                            uint64_t* __restrict__ cnt, unsigned long long* __restrict__ tot_bad,
+                            uint64_t vis_ts = ~0ull, uint64_t ins_base = 0, uint64_t del_base = 0) {
     const uint64_t i = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x;
     uint64_t c = 0;
     uint32_t bad = 0;
@@ -403,9 +407,11 @@ __global__ void k_rec_count(const DeltaRec* __restrict__ rec, uint64_t n, uint64
         const DeltaRec r = rec[i];
         if (r.valid > 1 || r.deleted > 1 || r.inserted > 1) bad |= REC_BAD_FLAG;
         if (r.valid) {
-            if (r.ins_off > n_ins || r.ins_cnt > n_ins - r.ins_off || r.del_off > n_del || r.del_cnt > n_del - r.del_off)
+            if (r.ins_off < ins_base || r.del_off < del_base || r.ins_off - ins_base > n_ins ||
+                r.ins_cnt > n_ins - (r.ins_off - ins_base) || r.del_off - del_base > n_del ||
+                r.del_cnt > n_del - (r.del_off - del_base))
                 bad |= REC_BAD_SLICE;
-            c = (uint64_t)r.inserted + r.del_cnt + r.ins_cnt + r.deleted;
+            if (r.ts <= vis_ts) c = (uint64_t)r.inserted + r.del_cnt + r.ins_cnt + r.deleted;
         }
         cnt[i] = c;
     }
@@ -416,29 +422,46 @@ __global__ void k_rec_count(const DeltaRec* __restrict__ rec, uint64_t n, uint64
         if (b) atomicOr(&tot_bad[1], (unsigned long long)b);
     }
 }
-// one warp per record (a record may carry thousands of inserts of a hub node)
+// one warp per record (a record may carry thousands of inserts of a hub node).  Weights:
+// f32 (wts) or the paper's 8-byte weights (wts64) narrowed to the replica's
+// f32 by round-to-nearest-even (reading A15)
 __global__ void k_rec_expand(const DeltaRec* __restrict__ rec, uint64_t n, const uint64_t* __restrict__ off,
                              const uint64_t* __restrict__ ins, const float* __restrict__ wts,
                              const uint64_t* __restrict__ del, uint8_t* __restrict__ kind, uint64_t* __restrict__ src,
-                             uint64_t* __restrict__ dst, float* __restrict__ w, uint64_t* __restrict__ ts) {
+                             uint64_t* __restrict__ dst, float* __restrict__ w, uint64_t* __restrict__ ts,
+                             const double* __restrict__ wts64 = nullptr, uint64_t vis_ts = ~0ull,
+                             uint64_t ins_base = 0, uint64_t del_base = 0) {
     const uint64_t warp = (blockIdx.x * (uint64_t)blockDim.x + threadIdx.x) >> 5;
     const uint64_t nwarps = ((uint64_t)gridDim.x * blockDim.x) >> 5;
     for (uint64_t i = warp; i < n; i += nwarps) {
         const DeltaRec r = rec[i];
-        if (!r.valid) continue;
-        const uint64_t o = off[i];
+        if (!r.valid || r.ts > vis_ts) continue;
+        const uint64_t o = off[i], io = r.ins_off - ins_base, dq = r.del_off - del_base;
         const uint32_t a = r.inserted, b = a + r.del_cnt, c = b + r.ins_cnt, e = c + r.deleted;
         for (uint32_t j = lane_id(); j < e; j += 32) {
             uint8_t k;
             uint64_t d = 0;
             float x = 0.f;
             if (j < a) k = NODE_INSERT;
-            else if (j < b) { k = EDGE_DELETE; d = del[r.del_off + (j - a)]; }
-            else if (j < c) { k = EDGE_INSERT; d = ins[r.ins_off + (j - b)]; x = wts[r.ins_off + (j - b)]; }
-            else k = NODE_DELETE;
+            else if (j < b) { k = EDGE_DELETE; d = del[dq + (j - a)]; }
+            else if (j < c) {
+                k = EDGE_INSERT;
+                d = ins[io + (j - b)];
+                x = wts64 ? __double2float_rn(wts64[io + (j - b)]) : wts[io + (j - b)];
+            } else k = NODE_DELETE;
             kind[o + j] = k; src[o + j] = r.node; dst[o + j] = d; w[o + j] = x; ts[o + j] = r.ts;
         }
     }
+}
+// after a successful cycle from a delta store: every record the scan used is marked
+// invalid ("by the end of the delta store scan"; each delta is used once,
+// P:L615-619); first_pending = lowest index of a still-valid (not yet visible) record
+__global__ void k_rec_consume(DeltaRec* __restrict__ rec, uint64_t n, uint64_t vis_ts,
+                              unsigned long long* __restrict__ first_pending) {
+    const uint64_t i = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x;
+    if (i >= n || !rec[i].valid) return;
+    if (rec[i].ts <= vis_ts) rec[i].valid = 0;
+    else atomicMin(first_pending, (unsigned long long)i);
 }
 
 // ===================================================================== a2 ====

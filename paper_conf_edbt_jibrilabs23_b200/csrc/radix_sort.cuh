@@ -30,7 +30,10 @@ constexpr int kRsSmem = kRsTile * 12;           // dynamic smem: staged keys + v
 constexpr int kRsWarps = kRsThreads / 32;
 constexpr int kRsMaxPasses = 8;
 constexpr int kRsLook = H2TAP_RS_LOOK;  // look-back: predecessor tiles read per step
-constexpr uint32_t kRsDirectTiles = 128;  // rs_coop: tiles up to which every CTA sums the count columns itself
+#ifndef H2TAP_RS_DIRECT
+#define H2TAP_RS_DIRECT 128
+#endif
+constexpr uint32_t kRsDirectTiles = H2TAP_RS_DIRECT;  // rs_coop: tiles up to which every CTA sums the count columns itself
 
 // n_dev (nullable): the key count lives in device memory (no host sync before the
 // sort); `n` is then an upper bound that only sizes the grids

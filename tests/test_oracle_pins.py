@@ -517,3 +517,40 @@ def test_pending_is_the_invisible_ops_in_arrival_order():
     assert o.apply(Batch.of([]), 30)[0] == 0 and len(o.pending()[0]) == 0
     off, cols, ww, ids = o.export()
     assert ids.tolist() == [0, 1, 2, 3, 7] and cols.tolist() == [2, 3, 0] and ww.tolist() == [4.0, 2.0, 1.0]
+
+
+# ------------------------------------------------------- delta store model ----
+def test_delta_store_model_fig2_two_cycles():
+    """Fig. 2's transactions appended to the store model (§5.1): a cycle at ts 10 sees only
+    transaction x (y is invisible), the next cycle at 20 sees only y (x's deltas
+    were marked invalid), a third cycle sees nothing; the replica ends at the
+    Fig. 2 result (tests/golden/fig2_records.json)."""
+    g, rb = load_fig2_records()
+    m = oracle.DeltaStoreModel()
+    valid = rb.records[rb.records["valid"] == 1]
+    m.append_records(valid, rb.inserts, rb.weights.astype(np.float64), rb.deletes)
+    e = np.array(g["edges"], dtype=object)
+    o = O1.from_edges(len(g["vertices"]), np.array(g["vertices"], np.uint64), np.array(e[:, 0], np.uint64),
+                      np.array(e[:, 1], np.uint64), np.array(e[:, 2], np.float32), g["create_ts"])
+    x = m.cycle(10)
+    assert sorted(set(x[4])) == [10] and len(x[0]) == 3          # NODE_INSERT 5, 5->1, 3->5
+    assert o.apply(Batch.of(list(zip(*x))), 10)[0] == 0
+    y = m.cycle(20)
+    assert sorted(set(y[4])) == [20] and len(y[0]) == 4          # 1-/->2, 1-/->4, delete 4, 3-/->4
+    assert o.apply(Batch.of(list(zip(*y))), 20)[0] == 0
+    assert len(m.cycle(30)[0]) == 0 and all(r["valid"] == 0 for r in m.records)
+    off, cols, w, ids = o.export()
+    ex = g["expected"]
+    assert ids.tolist() == ex["ext_ids"] and off.tolist() == ex["offsets"]
+    assert cols.tolist() == ex["cols"] and w.tolist() == ex["weights"]
+
+
+def test_delta_store_model_eight_byte_weights_round_to_nearest_even():
+    """8-byte weights reach the f32 replica rounded to nearest, ties to even
+    (reading A15): 1 + 2^-24 is a tie between 1 and 1 + 2^-23 -> 1 (even); 1 + 3 * 2^-24 a tie
+    between 1 + 2^-23 and 1 + 2^-22 -> 1 + 2^-22; 1 + 2^-24 + 2^-40 is above the tie."""
+    m = oracle.DeltaStoreModel()
+    ws = [1 + 2.0 ** -24, 1 + 3 * 2.0 ** -24, 1 + 2.0 ** -24 + 2.0 ** -40, 0.1]
+    m.append(1, 7, inserts=[1, 2, 3, 4], weights=ws)
+    k, s, d, w, t = m.cycle(1)
+    assert [float(np.float32(x)) for x in w] == [1.0, 1 + 2.0 ** -22, 1 + 2.0 ** -23, float(np.float32(0.1))]

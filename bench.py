@@ -561,24 +561,32 @@ def run_gpu(args):
         dist.destroy_process_group()
 
 
-def cpu_baseline_dyn(scale: int = 16, records: int = 20000, cycles: int = 3):
-    """cpu_baseline leg of --replica dyn: OD (oracle/od_dynamic.py, as it stands) on a bounded sample: an RMAT-16 graph and
-    20 K-record cycles of the same generator, timed on this host (one thread)."""
+def cpu_baseline_dyn(args, scale: int = 16, cycles: int = 3):
+    """cpu_baseline leg of --replica dyn: OD (oracle/od_dynamic.py: Algorithm 1 on Python dicts,
+    as it stands - an oracle-only reference, not a tuned CPU implementation) on a bounded
+    sample of the SAME generator as the GPU run (bench_dyn.workload: configs[2]'s update mix as
+    delta records, plus the same share of NODE_DELETE records) on an RMAT-16 graph, one thread.
+    Updates are counted as the GPU counts n_visible (expanded inserts + deletes + node ops)."""
+    import types
+    import bench_dyn
     from oracle.od_dynamic import DynamicOracle
     n = 1 << scale
     src, dst, w = synth.rmat_edges(scale, synth.seed_of("c3"), n=16 * n)
     o = DynamicOracle(np.arange(n, dtype=np.uint64), src, dst, w)
-    xid, items, t = n - 1, 0, 0.0
+    batch = max(1000, args.batch >> (args.scale - scale))
+    nd = max(1, args.node_deletes * batch // args.batch) if args.node_deletes else 0
+    sub = types.SimpleNamespace(scale=scale, batch=batch, node_deletes=nd)
+    items, t = 0, 0.0
     for k in range(cycles):
-        rb = synth.dyn_record_batch(synth.seed_of("c3"), 1000 + k, xid, records, n_new=64, max_slice=2,
-                                    p_deleted=0.0, p_new=0.0005, p_invalid=0.0)
+        rb, _ = bench_dyn.workload(sub, n, k)
         t0 = time.perf_counter()
         o.apply_records(rb.records, rb.inserts, rb.weights, rb.deletes)
         t += time.perf_counter() - t0
-        items += int(rb.records["ins_cnt"].sum() + rb.records["del_cnt"].sum())
-        xid += 64
+        r = rb.records
+        items += int(r["ins_cnt"].sum() + r["del_cnt"].sum() + r["inserted"].sum() + r["deleted"].sum())
     return {"value": items / t, "unit": "updates/s", "cores": 1, "kind": "oracle",
-            "sample": f"OD on RMAT-{scale} x16, {cycles} cycles of {records} records (edge-only), apply only"}
+            "sample": (f"OD (Python dict oracle, as it stands) on RMAT-{scale} x16, {cycles} cycles of the GPU "
+                       f"run's generator at {batch} updates (+ {nd} node deletes) per cycle, apply only")}
 
 
 def run_store(args):
@@ -694,7 +702,7 @@ def main():
         args.warmup = max(args.warmup, 3)
         line = bench_dyn.measure(args)
         if not args.no_cpu_baseline:
-            line["cpu_baseline"] = cpu_baseline_dyn()
+            line["cpu_baseline"] = cpu_baseline_dyn(args)
         print(json.dumps(line))
         return
     if args.warmup < 3 and args.impl == "h2tap":

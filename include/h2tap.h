@@ -419,7 +419,8 @@ h2tap_status h2tap_dyn_create(const h2tap_config* cfg, size_t n_vertices, const 
  * n_launches, h2d_bytes; n_visible = expanded items (inserts + deletes + node ops). */
 h2tap_status h2tap_dyn_apply_records(h2tap_dyn* d, const h2tap_record_batch* batch,
         h2tap_apply_stats* stats);
-/* n_vertices = dense slots (live and dead), n_edges = live edges, table_slots = capacity */
+/* n_vertices = dense ids (live and dead), n_edges = live edges, table_slots = slots of the
+ * per-vertex tables in use (their live keys, tombstones and EMPTY slots; garbage excluded) */
 h2tap_status h2tap_dyn_info(const h2tap_dyn* d, uint64_t* n_vertices, uint64_t* n_edges,
         uint64_t* table_slots);
 /* Materialise the CSR (rows = dense ids, dead rows empty, columns ascending): offsets
@@ -432,6 +433,18 @@ h2tap_status h2tap_dyn_export(h2tap_dyn* d, int64_t* offsets, uint32_t* cols, fl
  * `source_ext`; level_out [n_vertices] (host or device) = hop count or -1 (unreachable or dead).
  * Unknown / dead source -> E_INVAL. */
 h2tap_status h2tap_dyn_bfs(h2tap_dyn* d, uint64_t source_ext, int32_t* level_out);
+/* PageRank (reading A18: d, fixed iterations, dangling mass spread uniformly, fp64) over the
+ * live vertices, reading the per-vertex tables in place; rank_out [n_vertices] (host or
+ * device), 0 for a dead vertex. */
+h2tap_status h2tap_dyn_pagerank(h2tap_dyn* d, double damping, int iterations, double* rank_out);
+/* SSSP (reading A21) from the live vertex source_ext over the tables in place; dist_out
+ * [n_vertices] (host or device), +inf unreachable; a negative or NaN weight -> E_INVAL. */
+h2tap_status h2tap_dyn_sssp(h2tap_dyn* d, uint64_t source_ext, double* dist_out);
+/* Staged host input (as h2tap_batch_stage): start the H2D copy of a host record batch (pinned
+ * arrays for an asynchronous copy) into one of two library slots on the copy stream and fill
+ * `staged` with the device view; pass `staged` to h2tap_dyn_apply_records, which orders the
+ * copy before its kernels.  A slot is reused two stages later. */
+h2tap_status h2tap_dyn_stage(h2tap_dyn* d, const h2tap_record_batch* host, h2tap_record_batch* staged);
 void h2tap_dyn_destroy(h2tap_dyn* d);
 
 void h2tap_replica_destroy(h2tap_replica* r);

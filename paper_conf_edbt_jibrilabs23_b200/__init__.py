@@ -147,6 +147,9 @@ for _n, _a in (("h2tap_batch_stage", [_P, ctypes.POINTER(_Batch), ctypes.POINTER
                ("h2tap_ds_info", [_P] + [ctypes.POINTER(_u64)] * 5),
                ("h2tap_ds_export", [_P, _u64, ctypes.c_size_t, _P]),
                ("h2tap_delta_apply_store", [_P, _P, _u64, ctypes.POINTER(ApplyStats)]),
+               ("h2tap_dyn_pagerank", [_P, ctypes.c_double, ctypes.c_int, _P]),
+               ("h2tap_dyn_sssp", [_P, _u64, _P]),
+               ("h2tap_dyn_stage", [_P, ctypes.POINTER(_RecordBatch), ctypes.POINTER(_RecordBatch)]),
                ("h2tap_delta_abort", [_P]),
                ("h2tap_route_pack_p2p", [_P, ctypes.POINTER(_Batch), _u64, _P, _P]),
                ("h2tap_ipc_alloc", [ctypes.c_int, ctypes.c_size_t, ctypes.POINTER(_P), _P]),
@@ -589,6 +592,13 @@ for _n, _a, _r in (("h2tap_dyn_create", [ctypes.POINTER(_Config), ctypes.c_size_
     getattr(_lib, _n).argtypes = _a
 
 
+class StagedRecords:
+    """A record batch staged by DynReplica.stage (device view of a library slot)."""
+
+    def __init__(self, b, keep):
+        self.b, self.keep = b, keep
+
+
 class DynReplica:
     """The dynamic (hash-table) replica: Algorithm 1, §5.4
     (opaque h2tap_dyn*; include/h2tap.h documents the semantics)."""
@@ -611,9 +621,18 @@ class DynReplica:
                                      ctypes.byref(h)), "h2tap_dyn_create")
         return cls(h, keep + [cfg])
 
-    def apply_records(self, rb, raise_on_error: bool = True):
-        """h2tap_dyn_apply_records on rb (.records .inserts .weights .deletes, host or device)."""
+    def stage(self, rb) -> "StagedRecords":
+        """h2tap_dyn_stage: start the H2D copy of a host record batch (pinned for an
+        asynchronous copy) into a library slot; apply_records() the returned handle later."""
         b, keep = _record_batch(rb)
+        out = _RecordBatch()
+        _check(_lib.h2tap_dyn_stage(self._h, ctypes.byref(b), ctypes.byref(out)), "h2tap_dyn_stage")
+        return StagedRecords(out, keep)
+
+    def apply_records(self, rb, raise_on_error: bool = True):
+        """h2tap_dyn_apply_records on rb (.records .inserts .weights .deletes, host or device),
+        or on a StagedRecords from stage()."""
+        b, keep = (rb.b, rb.keep) if isinstance(rb, StagedRecords) else _record_batch(rb)
         st = ApplyStats()
         rc = _lib.h2tap_dyn_apply_records(self._h, ctypes.byref(b), ctypes.byref(st))
         if raise_on_error:
@@ -642,6 +661,19 @@ class DynReplica:
         lv = np.empty(self.info()["n_vertices"], np.int32)
         _check(_lib.h2tap_dyn_bfs(self._h, int(source_ext), ctypes.c_void_p(lv.ctypes.data)), "h2tap_dyn_bfs")
         return lv
+
+    def pagerank(self, damping: float = 0.85, iterations: int = 20) -> np.ndarray:
+        """PageRank (fp64) over the live vertices, 0 for a dead one, tables read in place."""
+        pr = np.empty(self.info()["n_vertices"], np.float64)
+        _check(_lib.h2tap_dyn_pagerank(self._h, float(damping), int(iterations), ctypes.c_void_p(pr.ctypes.data)),
+               "h2tap_dyn_pagerank")
+        return pr
+
+    def sssp(self, source_ext: int) -> np.ndarray:
+        """SSSP distances (fp64, +inf unreachable) from a live ext id, tables read in place."""
+        dist = np.empty(self.info()["n_vertices"], np.float64)
+        _check(_lib.h2tap_dyn_sssp(self._h, int(source_ext), ctypes.c_void_p(dist.ctypes.data)), "h2tap_dyn_sssp")
+        return dist
 
     def close(self):
         if getattr(self, "_h", None):

@@ -1,14 +1,19 @@
 // dyn.cuh - the dynamic replica: Algorithm 1 (§5.4 "Dynamic
-// Data Structures") ingesting one cycle's delta records into a GPU hash-table
-// graph, included by h2tap.cu (shares its allocator, stream, radix sort and record layout).
+// Data Structures") ingesting one cycle's delta records into a GPU graph of
+// per-vertex hash tables - "a hash table per node to store edges" ([7]) - included
+// by h2tap.cu (shares its allocator, stream, radix sort and record layout).
 //
-// Storage: one open-addressing table over packed edge keys
-//   key = src_dense << 32 | dst_dense  (u64; EMPTY = ~0, TOMB = ~0 - 1), value f32
-// linear probing from fmix64(key), load (live + tombstones) <= 0.7 (re-hashed into a table of
-// twice the needed size when a cycle would pass it); inserts only ever claim EMPTY slots, so a
-// CAS on the key word is the whole synchronisation.  Vertices: ext ids ascending (new IDs are
-// > xid, Alg. 1 line 5/8, so they append) and a u32 liveness word per dense id (D3: dense ids
-// never move, dead ones keep an empty row).
+// Storage: one slab of u32 destination keys (EMPTY = ~0, TOMB = ~0 - 1) and a
+// parallel slab of f32 weights.  Vertex v owns the slots [base[v], base[v] + cap[v]) - an
+// open-addressing table (linear probing from a 32-bit mix of the key), cap a power of two
+// (>= 4, 16-byte aligned) or 0 - with cnt[v] live keys and used[v] = live + tombstones.  A
+// table grows (into fresh slots at the slab's tail, the old slots becoming garbage) when a
+// cycle would push used over 3/4 of cap; the new cap keeps the load at or below 1/2.  The
+// slab is rebuilt (every vertex's live keys re-hashed into tables sized for load 1/2,
+// garbage dropped) when it runs out of room.  Inserts claim only EMPTY slots (a CAS on the
+// key word); a key is unique within a launch (the items were sorted first).  Vertices: ext ids
+// ascending (new IDs are > xid, Alg. 1 line 5/8, so they append) and a u32 liveness word per
+// dense id (D3: dense ids never move, dead ones keep an empty table).
 //
 // One cycle (h2tap_dyn_apply_records), all on the replica stream:
 //   k_dyn_rec        classify records (lines 2-9): deletion / new-node queues, per-record
@@ -18,19 +23,21 @@
 //                    cycle: D3), k_dyn_heads + scan + k_dyn_append (line 10)
 //   k_dyn_expand_ins thread per record (warp per large record): resolve endpoints, gate (D2), pack keys
 //   radix sort       (key, item) - stable, so the last item of a key is the latest (D1)
-//   k_dyn_upsert     last item of each key: CAS-insert or overwrite (lines 6, 10)
+//   k_dyn_inc / k_dyn_plan / k_dyn_grow   per source: incoming keys, tables that must grow
+//                    (+ one read-back to place them in the slab), re-hash into the new tables
+//   k_dyn_upsert     last item of each key: overwrite, or CAS-claim an EMPTY slot (lines 6, 10)
 //   k_dyn_delete     thread per record (warp per large record): probe + CAS to TOMB (line 7)
-//   k_dyn_node_del   liveness off (line 11) + k_dyn_cascade over the table if any died
-// Export materialises the CSR: k_dyn_compact (warp-aggregated) + radix sort + k_dyn_emit +
-// k_dyn_offsets.  The cost of a cycle is O(batch) plus O(table) only for node deletes.
+//   k_dyn_node_del   liveness off (line 11) + k_dyn_cascade over every table if any died
+// Reads traverse the tables in place (no materialisation): BFS, PageRank and SSSP scan a
+// vertex's slots and skip EMPTY / TOMB.  Export (tests, checkpoints) materialises a CSR.
 
 namespace dyn {
 
-constexpr uint64_t kEmpty = ~0ull, kTomb = ~0ull - 1;
 constexpr uint32_t kFilterBits = 1u << 18;   // cascade filter: 32 KB of shared memory
 
 struct Ctr {
     unsigned long long n_new_ids, n_del_ids, bad, max_new, n_new, n_upd, n_del, n_casc, n_gated, n_vdel, n_out, last_ext, n_big_ins, n_big_del, sum_ins, sum_del;
+    unsigned long long n_grow, grow_slots, alloc_tail, garbage, n_big_casc, n_front, bad_w;
 };
 
 __device__ __forceinline__ uint64_t hmix(uint64_t k) {
@@ -176,58 +183,143 @@ __global__ void __launch_bounds__(256) k_dyn_expand_ins(const DeltaRec* __restri
     if ((threadIdx.x & 31) == 0 && gated) atomicAdd(&c->n_gated, gated);
 }
 
-// insert-only probe into EMPTY slots; keys are unique within a launch
-__device__ __forceinline__ bool table_put(uint64_t* hk, float* hv, uint64_t mask, uint64_t k, float w) {
-    uint64_t h = hmix(k) & mask;
-    while (true) {
-        uint64_t cur = *((volatile uint64_t*)&hk[h]);
-        if (cur == k) { hv[h] = w; return false; }
-        if (cur == kEmpty) {
-            cur = atomicCAS((unsigned long long*)&hk[h], (unsigned long long)kEmpty, (unsigned long long)k);
-            if (cur == kEmpty || cur == k) { hv[h] = w; return cur == kEmpty; }
-        }
-        h = (h + 1) & mask;
-    }
+// ---- per-vertex hash tables over the slab
+constexpr uint32_t kKEmpty = 0xFFFFFFFFu, kKTomb = 0xFFFFFFFEu;
+__device__ __forceinline__ uint32_t hmix32(uint32_t x) {
+    x ^= x >> 16; x *= 0x7feb352du; x ^= x >> 15; x *= 0x846ca68bu; x ^= x >> 16;
+    return x;
+}
+struct Tabs {
+    uint64_t* base;   // first slot of vertex v's table
+    uint32_t* cap;    // slots (power of two >= 4, or 0)
+    uint32_t* cnt;    // live keys
+    uint32_t* used;   // live keys + tombstones
+    uint32_t* key;    // slab: destination dense ids, EMPTY / TOMB
+    float* val;       // slab: weights
+};
+__device__ __forceinline__ uint32_t pow2_cap(uint64_t live) {  // load <= 1/2, >= 4 slots
+    uint32_t c = 4;
+    while ((uint64_t)c < 2 * live) c <<= 1;
+    return c;
+}
+// insert a key that is not in the table (re-hash / first insert): claim the first EMPTY slot
+__device__ __forceinline__ void tab_claim(uint32_t* key, float* val, uint64_t b, uint32_t mask, uint32_t k, float w) {
+    uint32_t h = hmix32(k) & mask;
+    while (atomicCAS(&key[b + h], kKEmpty, k) != kKEmpty) h = (h + 1) & mask;
+    val[b + h] = w;
 }
 
+// per source: the distinct keys this cycle upserts (the latest item of every key)
+__global__ void k_dyn_inc(const uint64_t* __restrict__ sk, uint64_t n, uint64_t V, uint32_t* __restrict__ inc) {
+    const uint64_t i = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x;
+    if (i >= n) return;
+    const uint64_t k = sk[i];
+    if (k >= V * V || (i + 1 < n && sk[i + 1] == k)) return;
+    atomicAdd(&inc[k / V], 1u);
+}
+// the first key of every source decides: the table grows when used + incoming would pass 3/4
+// of its slots (a missing table always "grows"); the new size keeps the load <= 1/2
+__global__ void k_dyn_plan(const uint64_t* __restrict__ sk, uint64_t n, uint64_t V, Tabs T, uint32_t* __restrict__ inc,
+                           uint32_t* __restrict__ grow_v, uint32_t* __restrict__ grow_cap, Ctr* __restrict__ c) {
+    const uint64_t i = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x;
+    if (i >= n) return;
+    const uint64_t k = sk[i];
+    if (k >= V * V) return;
+    const uint64_t s = k / V;
+    if (i > 0 && sk[i - 1] / V == s) return;
+    const uint32_t in = inc[s];
+    inc[s] = 0;
+    const uint32_t cap = T.cap[s];
+    if (cap && 4ull * ((uint64_t)T.used[s] + in) <= 3ull * cap) return;
+    const uint32_t nc = pow2_cap((uint64_t)T.cnt[s] + in);
+    const uint64_t g = atomicAdd(&c->n_grow, 1ull);
+    grow_v[g] = (uint32_t)s;
+    grow_cap[g] = nc;
+    atomicAdd(&c->grow_slots, (unsigned long long)nc);
+}
+// warp per growing table: fresh slots at the slab tail, live keys re-hashed, old slots -> garbage
+__global__ void k_dyn_grow(const uint32_t* __restrict__ grow_v, const uint32_t* __restrict__ grow_cap, Tabs T,
+                           uint64_t tail0, Ctr* __restrict__ c) {
+    const uint64_t ng = c->n_grow;
+    const uint64_t nw = ((uint64_t)gridDim.x * blockDim.x) >> 5;
+    const uint32_t lane = threadIdx.x & 31;
+    for (uint64_t g = (blockIdx.x * (uint64_t)blockDim.x + threadIdx.x) >> 5; g < ng; g += nw) {
+        const uint32_t v = grow_v[g], nc = grow_cap[g];
+        unsigned long long nb = 0;
+        if (lane == 0) nb = tail0 + atomicAdd(&c->alloc_tail, (unsigned long long)nc);
+        nb = __shfl_sync(0xffffffffu, nb, 0);
+        const uint64_t ob = T.base[v];
+        const uint32_t oc = T.cap[v];
+        for (uint32_t j = lane; j < oc; j += 32) {
+            const uint32_t k = T.key[ob + j];
+            if (k < kKTomb) tab_claim(T.key, T.val, nb, nc - 1, k, T.val[ob + j]);
+        }
+        __syncwarp();
+        if (lane == 0) {
+            T.base[v] = nb;
+            T.cap[v] = nc;
+            T.used[v] = T.cnt[v];
+            if (oc) atomicAdd(&c->garbage, (unsigned long long)oc);
+        }
+    }
+}
+// lines 6 + 10: the latest item of every key overwrites its weight, or claims an EMPTY slot
 __global__ void k_dyn_upsert(const uint64_t* __restrict__ sk, const uint32_t* __restrict__ sv, uint64_t n,
-                             const float* __restrict__ witem, uint64_t V, uint64_t* hk, float* hv, uint64_t mask,
-                             Ctr* __restrict__ c) {
-    const uint64_t key_bad = V * V;
+                             const float* __restrict__ witem, uint64_t V, Tabs T, Ctr* __restrict__ c) {
     const uint64_t i = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x;
     bool nw = false, up = false;
     if (i < n) {
         const uint64_t k = sk[i];
-        if (k < key_bad && (i + 1 == n || sk[i + 1] != k)) {   // D1: the latest item of its key
+        if (k < V * V && (i + 1 == n || sk[i + 1] != k)) {   // D1: the latest item of its key
             const uint64_t s = k / V;
-            nw = table_put(hk, hv, mask, s << 32 | (k - s * V), witem[sv[i]]);
-            up = !nw;
+            const uint32_t d = (uint32_t)(k - s * V), mask = T.cap[s] - 1;
+            const uint64_t b = T.base[s];
+            const float w = witem[sv[i]];
+            uint32_t h = hmix32(d) & mask;
+            while (true) {
+                uint32_t cur = *((volatile uint32_t*)&T.key[b + h]);
+                if (cur == d) { T.val[b + h] = w; up = true; break; }
+                if (cur == kKEmpty) {
+                    cur = atomicCAS(&T.key[b + h], kKEmpty, d);
+                    if (cur == kKEmpty) {
+                        T.val[b + h] = w;
+                        atomicAdd(&T.cnt[s], 1u);
+                        atomicAdd(&T.used[s], 1u);
+                        nw = true;
+                        break;
+                    }
+                    continue;   // another key took the slot: look at it again
+                }
+                h = (h + 1) & mask;
+            }
         }
     }
     wadd(&c->n_new, nw);
     wadd(&c->n_upd, up);
 }
 
-__device__ __forceinline__ bool del_item(int64_t s, uint64_t x, const uint64_t* __restrict__ ext, uint64_t V,
-                                         uint64_t* hk, uint64_t mask) {
+__device__ __forceinline__ bool del_item(int64_t s, uint64_t x, const uint64_t* __restrict__ ext, uint64_t V, Tabs T) {
     const int64_t d = find_ext(ext, V, x);
-    if (d < 0) return false;
-    const uint64_t k = (uint64_t)s << 32 | (uint64_t)d;
-    uint64_t h = hmix(k) & mask;
-    while (true) {
-        const uint64_t cur = *((volatile uint64_t*)&hk[h]);
-        if (cur == k)
-            return atomicCAS((unsigned long long*)&hk[h], (unsigned long long)k, (unsigned long long)kTomb) == k;
-        if (cur == kEmpty) return false;
-        h = (h + 1) & mask;
+    const uint32_t cap = T.cap[s];
+    if (d < 0 || cap == 0) return false;
+    const uint64_t b = T.base[s];
+    uint32_t h = hmix32((uint32_t)d) & (cap - 1);
+    while (true) {   // at least a quarter of the slots are EMPTY: the probe ends
+        const uint32_t cur = *((volatile uint32_t*)&T.key[b + h]);
+        if (cur == (uint32_t)d) {
+            if (atomicCAS(&T.key[b + h], (uint32_t)d, kKTomb) != (uint32_t)d) return false;
+            atomicSub(&T.cnt[s], 1u);
+            return true;
+        }
+        if (cur == kKEmpty) return false;
+        h = (h + 1) & (cap - 1);
     }
 }
 // line 7: the records' deleted edges to TOMB; passes as in k_dyn_expand_ins
 template <int kPass>
 __global__ void __launch_bounds__(256) k_dyn_delete(const DeltaRec* __restrict__ rec, uint64_t nr,
         const uint64_t* __restrict__ off, const uint64_t* __restrict__ del, const uint64_t* __restrict__ ext,
-        uint64_t V, uint64_t* hk, uint64_t mask, uint64_t* __restrict__ big, unsigned long long* __restrict__ n_big,
-        Ctr* __restrict__ c) {
+        uint64_t V, Tabs T, uint64_t* __restrict__ big, unsigned long long* __restrict__ n_big, Ctr* __restrict__ c) {
     unsigned long long hits = 0;
     if (kPass == 0) {
         const uint64_t i = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x;
@@ -238,7 +330,7 @@ __global__ void __launch_bounds__(256) k_dyn_delete(const DeltaRec* __restrict__
                 const DeltaRec r = rec[i];
                 const int64_t s = find_ext(ext, V, r.node);
                 if (s >= 0)                                      // D4
-                    for (uint64_t j = 0; j < n; ++j) hits += del_item(s, del[r.del_off + j], ext, V, hk, mask);
+                    for (uint64_t j = 0; j < n; ++j) hits += del_item(s, del[r.del_off + j], ext, V, T);
             }
         }
     } else {
@@ -250,11 +342,33 @@ __global__ void __launch_bounds__(256) k_dyn_delete(const DeltaRec* __restrict__
             s = __shfl_sync(0xffffffffu, s, 0);
             if (s < 0) continue;
             const uint64_t dO = rec[i].del_off;
-            for (uint64_t j = lane; j < n; j += 32) hits += del_item(s, del[dO + j], ext, V, hk, mask);
+            for (uint64_t j = lane; j < n; j += 32) hits += del_item(s, del[dO + j], ext, V, T);
         }
     }
     hits = warp_sum<unsigned long long>(hits);
     if ((threadIdx.x & 31) == 0 && hits) atomicAdd(&c->n_del, hits);
+}
+
+// slab rebuild: every vertex's table re-sized for load <= 1/2 (live keys only) into a new slab
+__global__ void k_dyn_caps(const uint32_t* __restrict__ cnt, uint64_t V, uint64_t* __restrict__ capn) {
+    const uint64_t v = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x;
+    if (v < V) capn[v] = cnt[v] ? pow2_cap(cnt[v]) : 0;
+    else if (v == V) capn[V] = 0;
+}
+__global__ void k_dyn_rebuild(Tabs T, uint64_t V, const uint64_t* __restrict__ capn, const uint64_t* __restrict__ nbase,
+                              uint32_t* __restrict__ nkey, float* __restrict__ nval) {
+    const uint64_t nw = ((uint64_t)gridDim.x * blockDim.x) >> 5;
+    const uint32_t lane = threadIdx.x & 31;
+    for (uint64_t v = (blockIdx.x * (uint64_t)blockDim.x + threadIdx.x) >> 5; v < V; v += nw) {
+        const uint32_t oc = T.cap[v], nc = (uint32_t)capn[v];
+        const uint64_t ob = T.base[v], nb = nbase[v];
+        for (uint32_t j = lane; j < oc; j += 32) {
+            const uint32_t k = T.key[ob + j];
+            if (k < kKTomb) tab_claim(nkey, nval, nb, nc - 1, k, T.val[ob + j]);
+        }
+        __syncwarp();
+        if (lane == 0) { T.base[v] = nb; T.cap[v] = nc; T.used[v] = T.cnt[v]; }
+    }
 }
 
 __global__ void k_dyn_node_del(const uint64_t* __restrict__ del_ids, uint64_t nd, const uint64_t* __restrict__ ext,
@@ -274,56 +388,74 @@ __global__ void k_dyn_node_del(const uint64_t* __restrict__ del_ids, uint64_t nd
     wadd(&c->n_vdel, died);
 }
 
-// every table key had two live endpoints before this cycle's node deletes, so a key is
-// removed iff an endpoint died this cycle (bitmap, V/8 bytes, L2-resident); 2 slots/thread
-// a 32 KB filter (bit v mod 2^18 of every dead vertex) in shared memory screens the keys;
-// the exact bitmap is read only on a filter hit
-__device__ __forceinline__ bool died_of(const uint32_t* __restrict__ b, const uint32_t* __restrict__ filt, uint64_t k) {
-    const uint64_t s = k >> 32, d = k & 0xffffffffu;
-    const uint32_t fs = (uint32_t)s & (kFilterBits - 1), fd = (uint32_t)d & (kFilterBits - 1);
-    if ((((filt[fs >> 5] >> (fs & 31)) | (filt[fd >> 5] >> (fd & 31))) & 1u) == 0) return false;
-    return ((__ldg(b + (s >> 5)) >> (s & 31)) | (__ldg(b + (d >> 5)) >> (d & 31))) & 1u;
+// line 11's cascade: a key is removed iff an endpoint died this cycle (bitmap, V/8 bytes,
+// L2-resident).  A 32 KB filter (bit v mod 2^18 of every dead vertex) in shared memory
+// screens the keys; the exact bitmap is read only on a filter hit.  Pass 0: thread per
+// vertex for tables of <= 32 slots (16-byte loads); larger tables are queued for pass 1
+// (warp per table).  A dead vertex's own table is dropped (its keys are cascaded).
+__device__ __forceinline__ bool died_of(const uint32_t* __restrict__ b, const uint32_t* __restrict__ filt, uint32_t d) {
+    const uint32_t fd = d & (kFilterBits - 1);
+    if (((filt[fd >> 5] >> (fd & 31)) & 1u) == 0) return false;
+    return (__ldg(b + (d >> 5)) >> (d & 31)) & 1u;
 }
-__global__ void __launch_bounds__(256, 4) k_dyn_cascade(uint64_t* __restrict__ hk, uint64_t cap,
-        const uint32_t* __restrict__ died_bits, const uint32_t* __restrict__ filter, Ctr* __restrict__ c) {
+template <int kPass>
+__global__ void __launch_bounds__(256) k_dyn_cascade(Tabs T, uint64_t V, const uint32_t* __restrict__ died_bits,
+        const uint32_t* __restrict__ filter, uint32_t* __restrict__ big, Ctr* __restrict__ c) {
     if (*(volatile unsigned long long*)&c->n_vdel == 0) return;   // nobody died this cycle (no host sync)
     extern __shared__ uint32_t filt[];
     for (uint32_t t = threadIdx.x; t < kFilterBits / 32; t += blockDim.x) filt[t] = filter[t];
     __syncthreads();
-    const uint64_t stride = (uint64_t)gridDim.x * blockDim.x, half = cap >> 1;
-    ulonglong2* h2 = reinterpret_cast<ulonglong2*>(hk);
-    unsigned long long gone = 0;
-    constexpr int U = 4;   // 4 independent 16-byte loads in flight per thread
-    uint64_t i = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x;
-    for (; i + (U - 1) * stride < half; i += U * stride) {
-        ulonglong2 k[U];
+    unsigned long long gone = 0, garb = 0;
+    if (kPass == 0) {
+        const uint64_t stride = (uint64_t)gridDim.x * blockDim.x;
+        for (uint64_t u = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; u < V; u += stride) {
+            const uint32_t cap = T.cap[u];
+            if (!cap) continue;
+            if ((__ldg(died_bits + (u >> 5)) >> (u & 31)) & 1u) {   // its out-edges go with it
+                gone += T.cnt[u];
+                garb += cap;
+                T.cap[u] = 0; T.cnt[u] = 0; T.used[u] = 0;
+                continue;
+            }
+            if (cap > 32) { big[atomicAdd(&c->n_big_casc, 1ull)] = (uint32_t)u; continue; }
+            uint4* q = reinterpret_cast<uint4*>(T.key + T.base[u]);
+            uint32_t hits = 0;
+            for (uint32_t j = 0; j < cap / 4; ++j) {
+                uint4 k = q[j];
+                bool w = false;
+                uint32_t* kk = reinterpret_cast<uint32_t*>(&k);
 #pragma unroll
-        for (int u = 0; u < U; ++u) k[u] = __ldcs(h2 + i + u * stride);
+                for (int e = 0; e < 4; ++e)
+                    if (kk[e] < kKTomb && died_of(died_bits, filt, kk[e])) { kk[e] = kKTomb; w = true; ++hits; }
+                if (w) q[j] = k;
+            }
+            if (hits) { T.cnt[u] -= hits; gone += hits; }
+        }
+    } else {
+        const uint64_t nb = c->n_big_casc, nw = ((uint64_t)gridDim.x * blockDim.x) >> 5;
+        const uint32_t lane = threadIdx.x & 31;
+        for (uint64_t q = (blockIdx.x * (uint64_t)blockDim.x + threadIdx.x) >> 5; q < nb; q += nw) {
+            const uint32_t u = big[q], cap = T.cap[u];
+            uint4* p = reinterpret_cast<uint4*>(T.key + T.base[u]);
+            uint32_t hits = 0;
+            for (uint32_t j = lane; j < cap / 4; j += 32) {
+                uint4 k = p[j];
+                bool w = false;
+                uint32_t* kk = reinterpret_cast<uint32_t*>(&k);
 #pragma unroll
-        for (int u = 0; u < U; ++u) {
-            bool w = false;
-            if (k[u].x < kTomb && died_of(died_bits, filt, k[u].x)) { k[u].x = kTomb; w = true; ++gone; }
-            if (k[u].y < kTomb && died_of(died_bits, filt, k[u].y)) { k[u].y = kTomb; w = true; ++gone; }
-            if (w) h2[i + u * stride] = k[u];
+                for (int e = 0; e < 4; ++e)
+                    if (kk[e] < kKTomb && died_of(died_bits, filt, kk[e])) { kk[e] = kKTomb; w = true; ++hits; }
+                if (w) p[j] = k;
+            }
+            hits = warp_sum<uint32_t>(hits);
+            if (lane == 0 && hits) { T.cnt[u] -= hits; gone += hits; }
         }
     }
-    for (; i < half; i += stride) {
-        ulonglong2 k = h2[i];
-        bool w = false;
-        if (k.x < kTomb && died_of(died_bits, filt, k.x)) { k.x = kTomb; w = true; ++gone; }
-        if (k.y < kTomb && died_of(died_bits, filt, k.y)) { k.y = kTomb; w = true; ++gone; }
-        if (w) h2[i] = k;
-    }
     gone = warp_sum<unsigned long long>(gone);
-    if ((threadIdx.x & 31) == 0 && gone) atomicAdd(&c->n_casc, gone);
-}
-
-__global__ void k_dyn_rehash(const uint64_t* __restrict__ ok, const float* __restrict__ ov, uint64_t ocap,
-                             uint64_t* hk, float* hv, uint64_t mask) {
-    const uint64_t stride = (uint64_t)gridDim.x * blockDim.x;
-    for (uint64_t i = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; i < ocap; i += stride) {
-        const uint64_t k = ok[i];
-        if (k < kTomb) table_put(hk, hv, mask, k, ov[i]);
+    garb = warp_sum<unsigned long long>(garb);
+    if ((threadIdx.x & 31) == 0) {
+        if (gone) atomicAdd(&c->n_casc, gone);
+        if (garb) atomicAdd(&c->garbage, garb);
     }
 }
 
@@ -354,28 +486,123 @@ __global__ void k_dyn_fill_u32(uint32_t* p, uint64_t n, uint32_t v) {
     if (i < n) p[i] = v;
 }
 
-// export
-__global__ void k_dyn_compact(const uint64_t* __restrict__ hk, const float* __restrict__ hv, uint64_t cap,
-                              uint64_t V, uint64_t* __restrict__ ok, uint32_t* __restrict__ oi, float* __restrict__ ow,
-                              Ctr* __restrict__ c) {
+// export: every live key as a sort key s * V + d (thread per vertex, warp-aggregated output)
+__global__ void k_dyn_compact(Tabs T, uint64_t V, uint64_t* __restrict__ ok, uint32_t* __restrict__ oi,
+                              float* __restrict__ ow, Ctr* __restrict__ c) {
     const uint64_t stride = (uint64_t)gridDim.x * blockDim.x;
-    const unsigned lane = threadIdx.x & 31;
-    for (uint64_t i0 = blockIdx.x * (uint64_t)blockDim.x; i0 < cap; i0 += stride) {
-        const uint64_t i = i0 + threadIdx.x;
-        const uint64_t k = i < cap ? hk[i] : kEmpty;
-        const bool keep = k < kTomb;
-        const unsigned m = __ballot_sync(0xffffffffu, keep);
+    for (uint64_t u0 = blockIdx.x * (uint64_t)blockDim.x; u0 < V; u0 += stride) {
+        const uint64_t u = u0 + threadIdx.x;
+        const uint32_t n = u < V ? T.cnt[u] : 0u;
+        const uint32_t lane = threadIdx.x & 31;
+        uint32_t inc = n;
+#pragma unroll
+        for (int o = 1; o < 32; o <<= 1) {
+            const uint32_t y = __shfl_up_sync(0xffffffffu, inc, o);
+            if ((int)lane >= o) inc += y;
+        }
+        const uint32_t tot = __shfl_sync(0xffffffffu, inc, 31);
         unsigned long long base = 0;
-        if (lane == 0 && m) base = atomicAdd(&c->n_out, (unsigned long long)__popc(m));
-        base = __shfl_sync(0xffffffffu, base, 0);
-        if (keep) {
-            const uint64_t p = base + __popc(m & ((1u << lane) - 1));
-            ok[p] = (k >> 32) * V + (k & 0xffffffffu);   // sort key
-            oi[p] = (uint32_t)p;
-            ow[p] = hv[i];
+        if (lane == 0 && tot) base = atomicAdd(&c->n_out, (unsigned long long)tot);
+        base = __shfl_sync(0xffffffffu, base, 0) + inc - n;
+        if (!n) continue;
+        const uint64_t b = T.base[u];
+        const uint32_t cap = T.cap[u];
+        for (uint32_t j = 0; j < cap; ++j) {
+            const uint32_t k = T.key[b + j];
+            if (k < kKTomb) {
+                ok[base] = u * V + k;
+                oi[base] = (uint32_t)base;
+                ow[base] = T.val[b + j];
+                ++base;
+            }
         }
     }
 }
+
+// ---- reads on the tables in place (Table 1's BFS / PageRank / SSSP)
+__global__ void k_dyn_bfs_expand(Tabs T, const uint32_t* __restrict__ front, uint64_t nf, int32_t* __restrict__ level,
+                                 int32_t depth, uint32_t* __restrict__ next, unsigned long long* __restrict__ n_next) {
+    const uint64_t nw = ((uint64_t)gridDim.x * blockDim.x) >> 5;
+    for (uint64_t f = (blockIdx.x * (uint64_t)blockDim.x + threadIdx.x) >> 5; f < nf; f += nw) {
+        const uint32_t u = front[f], cap = T.cap[u];
+        const uint64_t b = T.base[u];
+        for (uint32_t j = lane_id(); j < cap; j += 32) {
+            const uint32_t v = T.key[b + j];
+            bool claim = false;
+            if (v < kKTomb && level[v] < 0) claim = atomicCAS(&level[v], -1, depth + 1) == -1;
+            const uint32_t m = __ballot_sync(__activemask(), claim);
+            if (claim) {
+                const uint32_t leader = __ffs(m) - 1;
+                unsigned long long o = 0;
+                if (lane_id() == leader) o = atomicAdd(n_next, (unsigned long long)__popc(m));
+                o = __shfl_sync(m, o, leader);
+                next[o + __popc(m & lanemask_lt())] = v;
+            }
+        }
+    }
+}
+__global__ void k_dyn_pr_dangling(const uint32_t* __restrict__ cnt, const uint32_t* __restrict__ live,
+                                  const double* __restrict__ pr, uint64_t V, double* __restrict__ out) {
+    double acc = 0;
+    for (uint64_t u = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; u < V; u += (uint64_t)gridDim.x * blockDim.x)
+        if (live[u] && cnt[u] == 0) acc += pr[u];
+    acc = warp_sum(acc);
+    if (lane_id() == 0 && acc != 0.0) atomicAdd(out, acc);
+}
+__global__ void k_dyn_pr_push(Tabs T, const double* __restrict__ pr, uint64_t V, double* __restrict__ nxt) {
+    const uint64_t nw = ((uint64_t)gridDim.x * blockDim.x) >> 5;
+    for (uint64_t u = (blockIdx.x * (uint64_t)blockDim.x + threadIdx.x) >> 5; u < V; u += nw) {
+        const uint32_t n = T.cnt[u];
+        if (!n) continue;
+        const uint32_t cap = T.cap[u];
+        const uint64_t b = T.base[u];
+        const double cu = pr[u] / (double)n;
+        for (uint32_t j = lane_id(); j < cap; j += 32) {
+            const uint32_t v = T.key[b + j];
+            if (v < kKTomb) atomicAdd(&nxt[v], cu);
+        }
+    }
+}
+__global__ void k_dyn_check_w(Tabs T, uint64_t V, Ctr* __restrict__ c) {
+    const uint64_t nw = ((uint64_t)gridDim.x * blockDim.x) >> 5;
+    bool bad = false;
+    for (uint64_t u = (blockIdx.x * (uint64_t)blockDim.x + threadIdx.x) >> 5; u < V; u += nw) {
+        const uint32_t cap = T.cap[u];
+        const uint64_t b = T.base[u];
+        for (uint32_t j = lane_id(); j < cap; j += 32)
+            if (T.key[b + j] < kKTomb) { const float x = T.val[b + j]; bad |= !(x >= 0.0f); }
+    }
+    if (__any_sync(0xffffffffu, bad) && lane_id() == 0) atomicOr(&c->bad_w, 1ull);
+}
+__global__ void k_dyn_sssp_relax(Tabs T, const uint32_t* __restrict__ front, uint64_t nf, unsigned long long* dist,
+                                 uint32_t* __restrict__ stamp, uint32_t round, uint32_t* __restrict__ next,
+                                 unsigned long long* __restrict__ n_next) {
+    const uint64_t nw = ((uint64_t)gridDim.x * blockDim.x) >> 5;
+    for (uint64_t f = (blockIdx.x * (uint64_t)blockDim.x + threadIdx.x) >> 5; f < nf; f += nw) {
+        const uint32_t u = front[f], cap = T.cap[u];
+        const uint64_t b = T.base[u];
+        const double du = __longlong_as_double((long long)ld_volatile(reinterpret_cast<const uint64_t*>(dist + u)));
+        for (uint32_t j = lane_id(); j < cap; j += 32) {
+            const uint32_t v = T.key[b + j];
+            bool push = false;
+            if (v < kKTomb) {
+                const double nd = du + (double)T.val[b + j];
+                const unsigned long long nb = (unsigned long long)__double_as_longlong(nd);
+                if (nb < ld_volatile(reinterpret_cast<const uint64_t*>(dist + v)) && atomicMin(dist + v, nb) > nb)
+                    push = atomicExch(stamp + v, round) != round;
+            }
+            const uint32_t m = __ballot_sync(__activemask(), push);
+            if (push) {
+                const uint32_t leader = __ffs(m) - 1;
+                unsigned long long o = 0;
+                if (lane_id() == leader) o = atomicAdd(n_next, (unsigned long long)__popc(m));
+                o = __shfl_sync(m, o, leader);
+                next[o + __popc(m & lanemask_lt())] = v;
+            }
+        }
+    }
+}
+
 __global__ void k_dyn_emit(const uint64_t* __restrict__ sk, const uint32_t* __restrict__ si, const float* __restrict__ cw,
                            uint64_t E, uint64_t V, uint32_t* __restrict__ cols, float* __restrict__ w) {
     const uint64_t i = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x;
@@ -410,22 +637,41 @@ __global__ void k_dyn_live_u8(const uint32_t* __restrict__ live, uint64_t V, uin
 
 struct h2tap_dyn {
     h2tap_replica* r = nullptr;   // stream, allocator, radix-sort scratch
-    uint64_t V = 0, n_live = 0, n_tomb = 0, cap = 0, xid = 0;   // xid = ext[V - 1] (host copy)
-    Buf ext, live, hk, hv, died, big;
+    uint64_t V = 0, n_live = 0, xid = 0;   // xid = ext[V - 1] (host copy)
+    uint64_t slab_cap = 0, tail = 0, garbage = 0;   // slab slots, allocated slots, garbage slots
+    Buf ext, live, base, cap, cnt, used, key, val, inc, grow_v, grow_cap, died, big;
     Buf cin, oin, new_ids, del_ids, kill, flag, fpos, keys, vals, keys2, vals2, witem, ctr, xo;
-    Buf x_rec, x_ins, x_wts, x_del;
+    Buf x_rec, x_ins, x_wts, x_del, live8, fa, fb, lvl, da, db;
+    struct Stage {
+        Buf rec, ins, wts, del;
+        cudaEvent_t ev = nullptr;
+        uint64_t bytes = 0;
+    } stg[2];
+    int stg_next = 0;
     dyn::Ctr* hctr = nullptr;     // pinned host mirror
 };
 
 namespace {
 
+dyn::Tabs dyn_tabs(h2tap_dyn* d) {
+    return dyn::Tabs{static_cast<uint64_t*>(d->base.p), static_cast<uint32_t*>(d->cap.p),
+                     static_cast<uint32_t*>(d->cnt.p), static_cast<uint32_t*>(d->used.p),
+                     static_cast<uint32_t*>(d->key.p), static_cast<float*>(d->val.p)};
+}
+
 void dyn_free(h2tap_dyn* d) {
     if (!d) return;
     if (d->r) {
-        for (Buf* b : {&d->ext, &d->live, &d->died, &d->big, &d->hk, &d->hv, &d->cin, &d->oin, &d->new_ids,
-                       &d->del_ids, &d->kill, &d->flag, &d->fpos, &d->keys, &d->vals, &d->keys2, &d->vals2,
-                       &d->witem, &d->ctr, &d->xo, &d->x_rec, &d->x_ins, &d->x_wts, &d->x_del})
+        for (Buf* b : {&d->ext, &d->live, &d->base, &d->cap, &d->cnt, &d->used, &d->key, &d->val, &d->inc,
+                       &d->grow_v, &d->grow_cap, &d->died, &d->big, &d->cin, &d->oin, &d->new_ids, &d->del_ids,
+                       &d->kill, &d->flag, &d->fpos, &d->keys, &d->vals, &d->keys2, &d->vals2, &d->witem, &d->ctr,
+                       &d->xo, &d->x_rec, &d->x_ins, &d->x_wts, &d->x_del, &d->live8, &d->fa, &d->fb, &d->lvl,
+                       &d->da, &d->db})
             if (b->p) d->r->dfree(b->p);
+        for (auto& g : d->stg) {
+            for (Buf* b : {&g.rec, &g.ins, &g.wts, &g.del}) if (b->p) d->r->dfree(b->p);
+            if (g.ev) cudaEventDestroy(g.ev);
+        }
         free_replica(d->r);
     }
     if (d->hctr) cudaFreeHost(d->hctr);
@@ -444,67 +690,105 @@ void dyn_ctr_read(h2tap_dyn* d) {
     d->r->sync();
 }
 
-// grow ext / live to hold n dense ids (contents kept)
+// grow the per-vertex arrays to hold n dense ids (contents kept, new entries: no table)
 void dyn_reserve_vertices(h2tap_dyn* d, uint64_t n) {
     h2tap_replica* r = d->r;
     if (d->ext.cap >= (n + 16) * 8 && d->live.cap >= (n + 16) * 4) return;
     const uint64_t want = std::max<uint64_t>(n, 2 * d->V) + 1024;
-    Buf e2, l2;
-    r->get<uint64_t>(e2, want);
-    r->get<uint32_t>(l2, want);
-    if (d->V) {
-        CK(cudaMemcpyAsync(e2.p, d->ext.p, d->V * 8, cudaMemcpyDeviceToDevice, r->st));
-        CK(cudaMemcpyAsync(l2.p, d->live.p, d->V * 4, cudaMemcpyDeviceToDevice, r->st));
-    }
-    r->release(d->ext);
-    r->release(d->live);
-    d->ext = e2;
-    d->live = l2;
+    auto regrow = [&](Buf& b, size_t el) {
+        Buf b2;
+        r->get<uint8_t>(b2, want * el);
+        CK(cudaMemsetAsync(b2.p, 0, (want + 16) * el, r->st));
+        if (d->V) CK(cudaMemcpyAsync(b2.p, b.p, d->V * el, cudaMemcpyDeviceToDevice, r->st));
+        r->release(b);
+        b = b2;
+    };
+    regrow(d->ext, 8);
+    regrow(d->live, 4);
+    regrow(d->base, 8);
+    regrow(d->cap, 4);
+    regrow(d->cnt, 4);
+    regrow(d->used, 4);
+    regrow(d->inc, 4);
 }
 
-uint64_t pow2_at_least(uint64_t x) {
-    uint64_t c = 1024;
-    while (c < x) c <<= 1;
-    return c;
-}
-
-// make room for `incoming` more keys at load <= 0.7 (tombstones count as used); a re-hash
-// sizes for load <= 0.7 as well, so after it the load is 0.35-0.7 (the cascade pass of a
-// node delete streams the whole table: a denser table is a shorter pass)
-void dyn_reserve_table(h2tap_dyn* d, uint64_t incoming) {
+// rebuild the slab: every table re-sized for load <= 1/2 into a slab with `extra` free slots
+void dyn_rebuild(h2tap_dyn* d, uint64_t extra) {
     h2tap_replica* r = d->r;
-    if (d->cap && 10 * (d->n_live + d->n_tomb + incoming) <= 7 * d->cap) return;
-    const uint64_t nc = pow2_at_least((10 * (d->n_live + incoming)) / 7 + 1);
+    cudaStream_t st = r->st;
+    const uint64_t V = d->V;
+    Buf bc, bb;
+    uint64_t* capn = r->get<uint64_t>(bc, V + 1);
+    uint64_t* nbase = r->get<uint64_t>(bb, V + 1);
+    dyn::k_dyn_caps<<<g1(V + 1), 256, 0, st>>>(static_cast<const uint32_t*>(d->cnt.p), V, capn);
+    CKL();
+    const uint64_t nt = cdiv(V + 1, kTile);
+    uint64_t* stt = r->get<uint64_t>(r->status2, nt);
+    unsigned int* sc = reinterpret_cast<unsigned int*>(r->get<uint64_t>(d->xo, 2));
+    CK(cudaMemsetAsync(stt, 0, nt * 8, st));
+    CK(cudaMemsetAsync(sc, 0, 4, st));
+    k_scan_exclusive_u64<<<(unsigned)nt, kThreads, 0, st>>>(capn, nbase, V + 1, stt, sc);
+    CKL();
+    uint64_t total = 0;
+    CK(cudaMemcpyAsync(&total, nbase + V, 8, cudaMemcpyDeviceToHost, st));
+    r->sync();
+    const uint64_t ncap = ((total + extra) * 5 / 4 + 1023) & ~1023ull;
     Buf k2, v2;
-    uint64_t* nk = r->get<uint64_t>(k2, nc);
-    float* nv = r->get<float>(v2, nc);
-    CK(cudaMemsetAsync(nk, 0xFF, nc * 8, r->st));
-    if (d->cap && d->n_live) {
-        const unsigned grid = (unsigned)std::min<uint64_t>(g1(d->cap), (uint64_t)r->n_sm * 8);
-        dyn::k_dyn_rehash<<<grid, 256, 0, r->st>>>(static_cast<uint64_t*>(d->hk.p), static_cast<float*>(d->hv.p),
-                                                   d->cap, nk, nv, nc - 1);
+    uint32_t* nk = r->get<uint32_t>(k2, ncap);
+    float* nv = r->get<float>(v2, ncap);
+    CK(cudaMemsetAsync(nk, 0xFF, (ncap + 16) * 4, st));
+    if (V) {
+        const unsigned grid = (unsigned)std::min<uint64_t>(cdiv(V * 32, 256), (uint64_t)r->n_sm * 16);
+        dyn::k_dyn_rebuild<<<grid, 256, 0, st>>>(dyn_tabs(d), V, capn, nbase, nk, nv);
         CKL();
     }
-    r->release(d->hk);
-    r->release(d->hv);
-    d->hk = k2;
-    d->hv = v2;
-    d->cap = nc;
-    d->n_tomb = 0;
+    r->release(d->key);
+    r->release(d->val);
+    r->release(bc);
+    r->release(bb);
+    d->key = k2;
+    d->val = v2;
+    d->slab_cap = ncap;
+    d->tail = total;
+    d->garbage = 0;
 }
 
-// sort (keys, item) items and upsert the latest item of every key; n items, keys < V' << 32
+// sort (key, item) items and upsert the latest item of every key; tables grow first
 void dyn_upsert_items(h2tap_dyn* d, uint64_t n, dyn::Ctr* c) {
     h2tap_replica* r = d->r;
+    cudaStream_t st = r->st;
     if (!n) return;
     uint64_t* k = static_cast<uint64_t*>(d->keys.p);
     uint32_t* v = static_cast<uint32_t*>(d->vals.p);
     uint64_t* k2 = static_cast<uint64_t*>(d->keys2.p);
     uint32_t* v2 = static_cast<uint32_t*>(d->vals2.p);
     radix_sort(r, k, v, k2, v2, n, bits_for(d->V * d->V));
-    dyn::k_dyn_upsert<<<g1(n), 256, 0, r->st>>>(k, v, n, static_cast<float*>(d->witem.p), d->V,
-                                                static_cast<uint64_t*>(d->hk.p), static_cast<float*>(d->hv.p),
-                                                d->cap - 1, c);
+    uint32_t* grow_v = r->get<uint32_t>(d->grow_v, n);
+    uint32_t* grow_cap = r->get<uint32_t>(d->grow_cap, n);
+    for (int attempt = 0;; ++attempt) {
+        CK(cudaMemsetAsync(&c->n_grow, 0, 24, st));   // n_grow, grow_slots, alloc_tail
+        dyn::k_dyn_inc<<<g1(n), 256, 0, st>>>(k, n, d->V, static_cast<uint32_t*>(d->inc.p));
+        CKL();
+        dyn::k_dyn_plan<<<g1(n), 256, 0, st>>>(k, n, d->V, dyn_tabs(d), static_cast<uint32_t*>(d->inc.p), grow_v,
+                                               grow_cap, c);
+        CKL();
+        dyn_ctr_read(d);
+        const uint64_t ng = d->hctr->n_grow, slots = d->hctr->grow_slots;
+        if (d->tail + slots <= d->slab_cap) {
+            if (ng) {
+                CK(cudaMemsetAsync(static_cast<uint32_t*>(d->key.p) + d->tail, 0xFF, slots * 4, st));
+                const unsigned grid = (unsigned)std::min<uint64_t>(cdiv(ng * 32, 256), (uint64_t)r->n_sm * 16);
+                dyn::k_dyn_grow<<<grid, 256, 0, st>>>(grow_v, grow_cap, dyn_tabs(d), d->tail, c);
+                CKL();
+                d->tail += slots;
+            }
+            break;
+        }
+        if (attempt) { set_err("slab rebuild did not make room"); throw Fail{H2TAP_E_CUDA}; }
+        // out of slab: rebuild (garbage dropped, room for this cycle's growth), then plan again
+        dyn_rebuild(d, slots + d->slab_cap / 4);
+    }
+    dyn::k_dyn_upsert<<<g1(n), 256, 0, st>>>(k, v, n, static_cast<float*>(d->witem.p), d->V, dyn_tabs(d), c);
     CKL();
 }
 
@@ -530,6 +814,12 @@ h2tap_status dyn_apply(h2tap_dyn* d, const h2tap_record_batch* b, h2tap_apply_st
     if (nr && !rec) { set_err("records is NULL"); return H2TAP_E_INVAL; }
     if (b->weights64) { set_err("the dynamic replica takes f32 weights (weights64 is for the CSR replica)"); return H2TAP_E_INVAL; }
     if ((b->n_inserts && (!ins || !wts)) || (b->n_deletes && !del)) { set_err("null inserts/weights/deletes"); return H2TAP_E_INVAL; }
+    for (auto& g : d->stg)  // a batch staged by h2tap_dyn_stage: its copy is ordered first
+        if (nr && b->on_device && b->records == g.rec.p) {
+            CK(cudaStreamWaitEvent(st, g.ev, 0));
+            g_h2d += g.bytes;
+            g.bytes = 0;
+        }
     if (!b->on_device) {
         DeltaRec* xr = r->get<DeltaRec>(d->x_rec, nr);
         uint64_t* xi = r->get<uint64_t>(d->x_ins, b->n_inserts);
@@ -646,16 +936,14 @@ h2tap_status dyn_apply(h2tap_dyn* d, const h2tap_record_batch* b, h2tap_apply_st
                                                        static_cast<uint64_t*>(d->keys.p), static_cast<uint32_t*>(d->vals.p),
                                                        static_cast<float*>(d->witem.p), big, nbig, c);
         CKL();
-        dyn_reserve_table(d, n_ins);
         dyn_upsert_items(d, n_ins, c);
     }
     // ---- line 7: delete batch
-    if (tot[1] && d->cap) {
+    if (tot[1]) {
         uint64_t* big = r->get<uint64_t>(d->big, nr);
-        uint64_t* hk = static_cast<uint64_t*>(d->hk.p);
-        dyn::k_dyn_delete<0><<<g1(nr), 256, 0, st>>>(rec, nr, odel, del, ext, d->V, hk, d->cap - 1, big, &c->n_big_del, c);
+        dyn::k_dyn_delete<0><<<g1(nr), 256, 0, st>>>(rec, nr, odel, del, ext, d->V, dyn_tabs(d), big, &c->n_big_del, c);
         CKL();
-        dyn::k_dyn_delete<1><<<wgrid, 256, 0, st>>>(rec, nr, odel, del, ext, d->V, hk, d->cap - 1, big, &c->n_big_del, c);
+        dyn::k_dyn_delete<1><<<wgrid, 256, 0, st>>>(rec, nr, odel, del, ext, d->V, dyn_tabs(d), big, &c->n_big_del, c);
         CKL();
     }
     // ---- line 11: node deletes + cascade
@@ -667,12 +955,16 @@ h2tap_status dyn_apply(h2tap_dyn* d, const h2tap_record_batch* b, h2tap_apply_st
         CK(cudaMemsetAsync(died, 0, (nwd + nwf) * 4, st));
         dyn::k_dyn_node_del<<<g1(h0.n_del_ids), 256, 0, st>>>(del_ids, h0.n_del_ids, ext, d->V, live, died, filter, c);
         CKL();
-        if (d->cap) {
+        if (d->V) {
             constexpr int smem = dyn::kFilterBits / 8;
-            CK(cudaFuncSetAttribute(dyn::k_dyn_cascade, cudaFuncAttributeMaxDynamicSharedMemorySize, smem));
-            const unsigned grid = (unsigned)std::min<uint64_t>(g1(d->cap / 2), (uint64_t)r->n_sm * 4);  // 4 CTAs/SM
+            CK(cudaFuncSetAttribute(dyn::k_dyn_cascade<0>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem));
+            CK(cudaFuncSetAttribute(dyn::k_dyn_cascade<1>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem));
+            uint32_t* bigv = r->get<uint32_t>(d->grow_v, d->V);
+            const unsigned grid = (unsigned)std::min<uint64_t>(g1(d->V), (uint64_t)r->n_sm * 4);  // 4 CTAs/SM
             CK(cudaEventRecord(r->ev[2], st));
-            dyn::k_dyn_cascade<<<grid, 256, smem, st>>>(static_cast<uint64_t*>(d->hk.p), d->cap, died, filter, c);
+            dyn::k_dyn_cascade<0><<<grid, 256, smem, st>>>(dyn_tabs(d), d->V, died, filter, bigv, c);
+            CKL();
+            dyn::k_dyn_cascade<1><<<(unsigned)r->n_sm * 4, 256, smem, st>>>(dyn_tabs(d), d->V, died, filter, bigv, c);
             CKL();
             CK(cudaEventRecord(r->ev[3], st));
             casc_timed = true;
@@ -682,7 +974,7 @@ h2tap_status dyn_apply(h2tap_dyn* d, const h2tap_record_batch* b, h2tap_apply_st
     dyn_ctr_read(d);
     const dyn::Ctr& h = *d->hctr;
     d->n_live = d->n_live + h.n_new - h.n_del - h.n_casc;
-    d->n_tomb += h.n_del + h.n_casc;
+    d->garbage += h.garbage;
     if (n_vins) d->xid = h.last_ext;
     if (stats) {
         std::memset(stats, 0, sizeof(*stats));
@@ -697,10 +989,10 @@ h2tap_status dyn_apply(h2tap_dyn* d, const h2tap_record_batch* b, h2tap_apply_st
         stats->ms_total = ev_ms(r->ev[0], r->ev[1]);
         if (casc_timed && h.n_vdel) {   // the cascade pass: its launch time and the table bytes it streams
             stats->ms_merge = ev_ms(r->ev[2], r->ev[3]);
-            stats->bytes_merge = d->cap * 8;
+            stats->bytes_merge = (d->tail - d->garbage) * 4 + d->V * 16;
         }
-        // algorithmic bytes: records + slices read, one 12-byte slot touch per item
-        stats->bytes_alg = nr * sizeof(DeltaRec) + n_ins * 12 + tot[1] * 8 + (n_ins + tot[1]) * 12;
+        // algorithmic bytes: records + slices read, one probe (4-byte key + 4-byte weight) per item
+        stats->bytes_alg = nr * sizeof(DeltaRec) + n_ins * 12 + tot[1] * 8 + (n_ins + tot[1]) * 8;
         stats->n_launches = g_launches;
         stats->h2d_bytes = g_h2d;
         stats->d2h_bytes = g_d2h;
@@ -708,7 +1000,7 @@ h2tap_status dyn_apply(h2tap_dyn* d, const h2tap_record_batch* b, h2tap_apply_st
     return H2TAP_OK;
 }
 
-// the CSR of the table (rows = dense ids, columns ascending) into caller-owned scratch Bufs
+// the CSR of the tables (rows = dense ids, columns ascending) into caller-owned scratch Bufs
 h2tap_status dyn_materialise(h2tap_dyn* d, Buf& bo, Buf& bc, Buf& bw) {
     h2tap_replica* r = d->r;
     cudaStream_t st = r->st;
@@ -720,10 +1012,9 @@ h2tap_status dyn_materialise(h2tap_dyn* d, Buf& bo, Buf& bc, Buf& bw) {
     uint64_t* k2 = static_cast<uint64_t*>(d->keys2.p);
     uint32_t* v2 = static_cast<uint32_t*>(d->vals2.p);
     float* cw = static_cast<float*>(d->witem.p);
-    if (d->cap) {
-        const unsigned grid = (unsigned)std::min<uint64_t>(g1(d->cap), (uint64_t)r->n_sm * 8);
-        dyn::k_dyn_compact<<<grid, 256, 0, st>>>(static_cast<uint64_t*>(d->hk.p), static_cast<float*>(d->hv.p),
-                                                 d->cap, V, k, v, cw, c);
+    if (V) {
+        const unsigned grid = (unsigned)std::min<uint64_t>(g1(V), (uint64_t)r->n_sm * 16);
+        dyn::k_dyn_compact<<<grid, 256, 0, st>>>(dyn_tabs(d), V, k, v, cw, c);
         CKL();
     }
     radix_sort(r, k, v, k2, v2, E, bits_for(V * V));
@@ -735,9 +1026,22 @@ h2tap_status dyn_materialise(h2tap_dyn* d, Buf& bo, Buf& bc, Buf& bw) {
     CKL();
     dyn_ctr_read(d);
     if (d->hctr->n_out != E) {
-        set_err("table holds %llu live keys, expected %llu", d->hctr->n_out, (unsigned long long)E);
+        set_err("tables hold %llu live keys, expected %llu", d->hctr->n_out, (unsigned long long)E);
         return H2TAP_E_CUDA;
     }
+    return H2TAP_OK;
+}
+
+// dense id of a live vertex (or an error)
+h2tap_status dyn_source(h2tap_dyn* d, uint64_t source_ext, uint64_t* out) {
+    h2tap_replica* r = d->r;
+    dyn::Ctr* c = dyn_ctr_reset(d);
+    dyn::k_dyn_lookup<<<1, 32, 0, r->st>>>(static_cast<const uint64_t*>(d->ext.p),
+                                           static_cast<const uint32_t*>(d->live.p), d->V, source_ext, c);
+    CKL();
+    dyn_ctr_read(d);
+    if (!d->hctr->bad) { set_err("source %llu is not a live vertex", (unsigned long long)source_ext); return H2TAP_E_INVAL; }
+    *out = d->hctr->bad - 1;
     return H2TAP_OK;
 }
 
@@ -751,7 +1055,7 @@ h2tap_status h2tap_dyn_create(const h2tap_config* cfg, size_t n_vertices, const 
     if (!out) { set_err("out is NULL"); return H2TAP_E_INVAL; }
     *out = nullptr;
     if (n_edges && (!src || !dst)) { set_err("src/dst NULL"); return H2TAP_E_INVAL; }
-    if (n_vertices >= 0xFFFFFFFFull || n_edges >= 0xFFFFFFFFull) { set_err("more than 2^32 - 2 vertices or edges"); return H2TAP_E_CAPACITY; }
+    if (n_vertices >= 0xFFFFFFFEull || n_edges >= 0xFFFFFFFFull) { set_err("more than 2^32 - 3 vertices or 2^32 - 2 edges"); return H2TAP_E_CAPACITY; }
     if (cfg && (cfg->world > 1 || cfg->id_mode != H2TAP_ID_COMPACT)) {
         set_err("the dynamic replica is single-GPU with fixed dense ids (leave world / id_mode at 0)");
         return H2TAP_E_INVAL;
@@ -763,9 +1067,9 @@ h2tap_status h2tap_dyn_create(const h2tap_config* cfg, size_t n_vertices, const 
         d->r = new_replica(cfg);
         h2tap_replica* r = d->r;
         CK(cudaHostAlloc(reinterpret_cast<void**>(&d->hctr), sizeof(dyn::Ctr), cudaHostAllocDefault));
-        if (!r->ev[0]) CK(cudaEventCreate(&r->ev[0]));
-        for (int e = 1; e < 4; ++e)
+        for (int e = 0; e < 4; ++e)
             if (!r->ev[e]) CK(cudaEventCreate(&r->ev[e]));
+        for (auto& g : d->stg) CK(cudaEventCreateWithFlags(&g.ev, cudaEventDisableTiming));
         dyn_reserve_vertices(d, n_vertices);
         uint64_t* ext = static_cast<uint64_t*>(d->ext.p);
         if (vertex_ids) copy_in(r, ext, vertex_ids, n_vertices, on_device);
@@ -784,7 +1088,7 @@ h2tap_status h2tap_dyn_create(const h2tap_config* cfg, size_t n_vertices, const 
             CK(cudaMemcpyAsync(&d->xid, ext + n_vertices - 1, 8, cudaMemcpyDeviceToHost, r->st));
             r->sync();
         }
-        dyn_reserve_table(d, n_edges);
+        dyn_rebuild(d, n_edges);   // an empty slab with room for the edges' tables
         if (n_edges) {
             dyn_item_bufs(d, n_edges);
             const uint64_t *s2 = src, *d2 = dst;
@@ -809,6 +1113,7 @@ h2tap_status h2tap_dyn_create(const h2tap_config* cfg, size_t n_vertices, const 
             dyn_upsert_items(d, n_edges, c);
             dyn_ctr_read(d);
             d->n_live = d->hctr->n_new;
+            d->garbage = d->hctr->garbage;
         }
         r->sync();
         return H2TAP_OK;
@@ -826,11 +1131,52 @@ h2tap_status h2tap_dyn_apply_records(h2tap_dyn* d, const h2tap_record_batch* bat
     return run_guarded(d->r, [&]() { return dyn_apply(d, batch, stats); });
 }
 
+h2tap_status h2tap_dyn_stage(h2tap_dyn* d, const h2tap_record_batch* host, h2tap_record_batch* staged) {
+    if (!d || !host || !staged) { set_err("null argument"); return H2TAP_E_INVAL; }
+    if (host->on_device) { set_err("h2tap_dyn_stage takes a host batch"); return H2TAP_E_INVAL; }
+    if (host->weights64) { set_err("the dynamic replica takes f32 weights"); return H2TAP_E_INVAL; }
+    if ((host->n_records && !host->records) || (host->n_inserts && (!host->inserts || !host->weights)) ||
+        (host->n_deletes && !host->deletes)) {
+        set_err("null records/inserts/weights/deletes");
+        return H2TAP_E_INVAL;
+    }
+    return run_guarded(d->r, [&]() -> h2tap_status {
+        h2tap_replica* r = d->r;
+        CK(cudaSetDevice(r->cfg.device));
+        auto& g = d->stg[d->stg_next];
+        d->stg_next ^= 1;
+        CK(cudaEventSynchronize(g.ev));   // the slot's previous copy is done before a regrow
+        DeltaRec* xr = r->get<DeltaRec>(g.rec, host->n_records);
+        uint64_t* xi = r->get<uint64_t>(g.ins, host->n_inserts);
+        float* xw = r->get<float>(g.wts, host->n_inserts);
+        uint64_t* xd = r->get<uint64_t>(g.del, host->n_deletes);
+        CK(cudaStreamSynchronize(r->st));   // slot buffers (re)allocated on the replica stream are ready
+        cudaStream_t cs = r->st_copy;
+        uint64_t bytes = 0;
+        auto cp = [&](void* dst, const void* src, uint64_t nb) {
+            if (!nb) return;
+            CK(cudaMemcpyAsync(dst, src, nb, cudaMemcpyHostToDevice, cs));
+            bytes += nb;
+        };
+        cp(xr, host->records, host->n_records * sizeof(DeltaRec));
+        cp(xi, host->inserts, host->n_inserts * 8);
+        cp(xw, host->weights, host->n_inserts * 4);
+        cp(xd, host->deletes, host->n_deletes * 8);
+        CK(cudaEventRecord(g.ev, cs));
+        g.bytes = bytes;
+        *staged = *host;
+        staged->on_device = 1;
+        staged->records = reinterpret_cast<const h2tap_delta_record*>(xr);
+        staged->inserts = xi; staged->weights = xw; staged->deletes = xd;
+        return H2TAP_OK;
+    });
+}
+
 h2tap_status h2tap_dyn_info(const h2tap_dyn* d, uint64_t* n_vertices, uint64_t* n_edges, uint64_t* table_slots) {
     if (!d) { set_err("null argument"); return H2TAP_E_INVAL; }
     if (n_vertices) *n_vertices = d->V;
     if (n_edges) *n_edges = d->n_live;
-    if (table_slots) *table_slots = d->cap;
+    if (table_slots) *table_slots = d->tail - d->garbage;
     return H2TAP_OK;
 }
 
@@ -863,21 +1209,12 @@ h2tap_status h2tap_dyn_bfs(h2tap_dyn* d, uint64_t source_ext, int32_t* level_out
         h2tap_replica* r = d->r;
         cudaStream_t st = r->st;
         const uint64_t V = d->V;
-        const uint64_t* ext = static_cast<const uint64_t*>(d->ext.p);
-        // source: dense id of a live vertex (host binary search over a copy is avoided:
-        // one device lookup through the counters block)
-        dyn::Ctr* c = dyn_ctr_reset(d);
-        dyn::k_dyn_lookup<<<1, 32, 0, st>>>(ext, static_cast<const uint32_t*>(d->live.p), V, source_ext, c);
-        CKL();
-        dyn_ctr_read(d);
-        if (!d->hctr->bad) { set_err("BFS source %llu is not a live vertex", (unsigned long long)source_ext); return H2TAP_E_INVAL; }
-        const uint64_t src = d->hctr->bad - 1;
-        Buf bo, bc, bw, bl, fa_, fb_;
-        const h2tap_status s = dyn_materialise(d, bo, bc, bw);
-        if (s != H2TAP_OK) return s;
-        int32_t* level = r->get<int32_t>(bl, V);
-        uint32_t* fa = r->get<uint32_t>(fa_, V);
-        uint32_t* fb = r->get<uint32_t>(fb_, V);
+        uint64_t src = 0;
+        const h2tap_status e = dyn_source(d, source_ext, &src);
+        if (e != H2TAP_OK) return e;
+        int32_t* level = r->get<int32_t>(d->lvl, V);
+        uint32_t* fa = r->get<uint32_t>(d->fa, V);
+        uint32_t* fb = r->get<uint32_t>(d->fb, V);
         unsigned long long* cnt = r->get<unsigned long long>(r->misc, 1);
         k_fill_i32<<<g1(V), 256, 0, st>>>(level, V, -1);
         CKL();
@@ -886,11 +1223,10 @@ h2tap_status h2tap_dyn_bfs(h2tap_dyn* d, uint64_t source_ext, int32_t* level_out
         CK(cudaMemcpyAsync(level + src, &zero, 4, cudaMemcpyHostToDevice, st));
         CK(cudaMemcpyAsync(fa, &s32, 4, cudaMemcpyHostToDevice, st));
         uint64_t nf = 1;
-        for (int32_t depth = 0; nf; ++depth) {   // the CSR path's level-synchronous expansion
+        for (int32_t depth = 0; nf; ++depth) {   // level-synchronous, the tables read in place
             CK(cudaMemsetAsync(cnt, 0, 8, st));
-            const unsigned grid = (unsigned)std::min<uint64_t>(cdiv(nf * 32, 256), 148 * 32);
-            k_bfs_expand<<<grid, 256, 0, st>>>(static_cast<const int64_t*>(bo.p), static_cast<const uint32_t*>(bc.p),
-                                               fa, nf, level, depth, fb, cnt);
+            const unsigned grid = (unsigned)std::min<uint64_t>(cdiv(nf * 32, 256), (uint64_t)r->n_sm * 32);
+            dyn::k_dyn_bfs_expand<<<grid, 256, 0, st>>>(dyn_tabs(d), fa, nf, level, depth, fb, cnt);
             CKL();
             unsigned long long h = 0;
             CK(cudaMemcpyAsync(&h, cnt, 8, cudaMemcpyDeviceToHost, st));
@@ -900,7 +1236,97 @@ h2tap_status h2tap_dyn_bfs(h2tap_dyn* d, uint64_t source_ext, int32_t* level_out
         }
         CK(cudaMemcpyAsync(level_out, level, V * 4, cudaMemcpyDefault, st));
         r->sync();
-        for (Buf* b : {&bo, &bc, &bw, &bl, &fa_, &fb_}) r->release(*b);
+        return H2TAP_OK;
+    });
+}
+
+h2tap_status h2tap_dyn_pagerank(h2tap_dyn* d, double damping, int iterations, double* rank_out) {
+    if (!d || !rank_out || iterations < 0) { set_err("bad argument"); return H2TAP_E_INVAL; }
+    return run_guarded(d->r, [&]() -> h2tap_status {
+        h2tap_replica* r = d->r;
+        cudaStream_t st = r->st;
+        const uint64_t V = d->V;
+        if (V == 0) return H2TAP_OK;
+        // the graph is the live vertices (dead ones keep an empty table and rank 0, D3)
+        uint8_t* l8 = r->get<uint8_t>(d->live8, V);
+        dyn::k_dyn_live_u8<<<g1(V), 256, 0, st>>>(static_cast<const uint32_t*>(d->live.p), V, l8);
+        CKL();
+        unsigned long long* c = r->get<unsigned long long>(r->misc, 2);
+        CK(cudaMemsetAsync(c, 0, 16, st));
+        k_count_u8<<<(unsigned)std::min<uint64_t>(g1(V), (uint64_t)r->n_sm * 8), 256, 0, st>>>(l8, V, c);
+        CKL();
+        unsigned long long nl = 0;
+        CK(cudaMemcpyAsync(&nl, c, 8, cudaMemcpyDeviceToHost, st));
+        r->sync();
+        double* a = r->get<double>(d->da, V);
+        double* b = r->get<double>(d->db, V);
+        double* ds = reinterpret_cast<double*>(c + 1);
+        if (nl == 0) {
+            CK(cudaMemsetAsync(a, 0, V * 8, st));
+        } else {
+            k_pr_init<<<g1(V), 256, 0, st>>>(a, V, l8, nl);
+            CKL();
+            const unsigned gs = (unsigned)std::min<uint64_t>(g1(V), (uint64_t)r->n_sm * 8);
+            const unsigned gw = (unsigned)std::min<uint64_t>(cdiv(V * 32, 256), (uint64_t)r->n_sm * 32);
+            for (int it = 0; it < iterations; ++it) {
+                CK(cudaMemsetAsync(ds, 0, 8, st));
+                CK(cudaMemsetAsync(b, 0, V * 8, st));
+                dyn::k_dyn_pr_dangling<<<gs, 256, 0, st>>>(static_cast<const uint32_t*>(d->cnt.p),
+                                                           static_cast<const uint32_t*>(d->live.p), a, V, ds);
+                dyn::k_dyn_pr_push<<<gw, 256, 0, st>>>(dyn_tabs(d), a, V, b);
+                k_pr_finish<<<g1(V), 256, 0, st>>>(b, V, damping, ds, l8, nl);
+                CKL();
+                std::swap(a, b);
+            }
+        }
+        CK(cudaMemcpyAsync(rank_out, a, V * 8, cudaMemcpyDefault, st));
+        r->sync();
+        return H2TAP_OK;
+    });
+}
+
+h2tap_status h2tap_dyn_sssp(h2tap_dyn* d, uint64_t source_ext, double* dist_out) {
+    if (!d || !dist_out) { set_err("null argument"); return H2TAP_E_INVAL; }
+    return run_guarded(d->r, [&]() -> h2tap_status {
+        h2tap_replica* r = d->r;
+        cudaStream_t st = r->st;
+        const uint64_t V = d->V;
+        uint64_t src = 0;
+        const h2tap_status e = dyn_source(d, source_ext, &src);
+        if (e != H2TAP_OK) return e;
+        dyn::Ctr* c = dyn_ctr_reset(d);
+        dyn::k_dyn_check_w<<<(unsigned)std::min<uint64_t>(cdiv(V * 32, 256), (uint64_t)r->n_sm * 16), 256, 0, st>>>(
+            dyn_tabs(d), V, c);
+        CKL();
+        dyn_ctr_read(d);
+        if (d->hctr->bad_w) { set_err("h2tap_dyn_sssp: negative or NaN edge weight"); return H2TAP_E_INVAL; }
+        double* dist = r->get<double>(d->da, V);
+        uint32_t* stamp = reinterpret_cast<uint32_t*>(r->get<double>(d->db, V));
+        uint32_t* fa = r->get<uint32_t>(d->fa, V);
+        uint32_t* fb = r->get<uint32_t>(d->fb, V);
+        unsigned long long* cnt = r->get<unsigned long long>(r->misc, 1);
+        k_fill_u64<<<g1(V), 256, 0, st>>>(reinterpret_cast<uint64_t*>(dist), V, 0x7FF0000000000000ull);  // +inf
+        CKL();
+        CK(cudaMemsetAsync(stamp, 0, V * 4, st));
+        const double zero = 0.0;
+        const uint32_t s32 = (uint32_t)src;
+        CK(cudaMemcpyAsync(dist + src, &zero, 8, cudaMemcpyHostToDevice, st));
+        CK(cudaMemcpyAsync(fa, &s32, 4, cudaMemcpyHostToDevice, st));
+        uint64_t nf = 1;
+        for (uint32_t round = 1; nf; ++round) {
+            CK(cudaMemsetAsync(cnt, 0, 8, st));
+            const unsigned grid = (unsigned)std::min<uint64_t>(cdiv(nf * 32, 256), (uint64_t)r->n_sm * 32);
+            dyn::k_dyn_sssp_relax<<<grid, 256, 0, st>>>(dyn_tabs(d), fa, nf, reinterpret_cast<unsigned long long*>(dist),
+                                                        stamp, round, fb, cnt);
+            CKL();
+            unsigned long long h = 0;
+            CK(cudaMemcpyAsync(&h, cnt, 8, cudaMemcpyDeviceToHost, st));
+            r->sync();
+            nf = h;
+            std::swap(fa, fb);
+        }
+        CK(cudaMemcpyAsync(dist_out, dist, V * 8, cudaMemcpyDefault, st));
+        r->sync();
         return H2TAP_OK;
     });
 }

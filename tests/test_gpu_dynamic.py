@@ -84,13 +84,53 @@ def test_bfs_after_cycles(h2):
                                                     rb.inserts), rb.weights,
                                ids[(rb.deletes % n).astype(np.int64)])
         cycle(g, o, rb, f"bfs cycle {cyc}")
-    off, cols, _, ext, live = o.export()
+    off, cols, ww, ext, live = o.export()
     for s_dense in np.flatnonzero(live)[:5]:
         assert np.array_equal(g.bfs(int(ext[s_dense])), oracle.bfs(off, cols, int(s_dense)))
+        # SSSP over the tables in place vs Dijkstra on OD's export (dead: unreachable)
+        assert np.array_equal(g.sssp(int(ext[s_dense])), oracle.sssp(off, cols, ww, int(s_dense)))
     dead = np.flatnonzero(live == 0)
-    if len(dead):
-        with pytest.raises(Exception):
-            g.bfs(int(ext[dead[0]]))
+    assert len(dead)
+    with pytest.raises(Exception):
+        g.bfs(int(ext[dead[0]]))
+    # PageRank over the live vertices (reading A18 on the live subgraph, D3: a dead vertex keeps
+    # an empty table and rank 0) vs the oracle on the compacted live part of OD's export
+    from test_oracle_pins import compact_view
+    coff, ccols, _, _ = compact_view(off, cols, ww, ext, live)
+    ref = np.zeros(len(live))
+    ref[np.flatnonzero(live)] = oracle.pagerank(coff, ccols, 0.85, 20)
+    pr = g.pagerank(0.85, 20)
+    assert np.all(pr[live == 0] == 0)
+    assert np.max(np.abs(pr - ref)[live == 1] / ref[live == 1]) <= 1e-6
+
+
+def test_staged_host_records_pipeline(h2):
+    """h2tap_dyn_stage: batch k+1 is copied on the copy stream while batch k is applied; the
+    result equals OD after every cycle (pinned host records)."""
+    import torch
+    rng = np.random.default_rng(11)
+    n = 2000
+    ids = np.arange(n, dtype=np.uint64)
+    m = 9000
+    g, o = pair(h2, ids, ids[rng.integers(0, n, m)], ids[rng.integers(0, n, m)], rng.random(m))
+    pin = lambda a: torch.from_numpy(a.view(np.uint8) if a.dtype.fields else a.view(np.int64) if a.dtype == np.uint64 else a).pin_memory()  # noqa: E731
+    rbs = []
+    xid = n - 1
+    for cyc in range(5):
+        rb = synth.dyn_record_batch(31, cyc, xid, 3000, n_new=30, max_slice=4, p_deleted=0.01)
+        rbs.append(rb)
+        xid += 30
+    host = [synth.RecordBatch(pin(r.records), pin(r.inserts), pin(r.weights), pin(r.deletes)) for r in rbs]
+    staged = g.stage(host[0])
+    for k in range(5):
+        nxt = g.stage(host[k + 1]) if k + 1 < 5 else None
+        st = g.apply_records(staged)
+        ost = o.apply_records(rbs[k].records, rbs[k].inserts, rbs[k].weights, rbs[k].deletes)
+        for key in KEYS:
+            assert st[key] == ost[key], f"staged cycle {k}: {key}"
+        assert st["h2d_bytes"] > 0
+        same(g, o, f"staged cycle {k}")
+        staged = nxt
 
 
 def test_multi_tile_cycles_with_rehash_and_device_inputs(h2):

@@ -560,9 +560,12 @@ h2tap_status apply_core(h2tap_replica* r, const BatchIn& in, uint64_t S, bool cr
         // phase below (latency-bound sort / classify) reads its output, so it runs on the
         // side stream with a grid of 4 CTAs per SM, leaving most of every SM to the edge-op
         // kernels; the row pass joins it (casc_join) before reading the cascade tables.
+#ifndef H2TAP_CASC_MAIN
+#define H2TAP_CASC_MAIN 0
+#endif
         CK(cudaEventRecord(r->evA, st));
         CK(cudaStreamWaitEvent(r->st2, r->evA, 0));
-        cudaStream_t cs = r->st2;
+        cudaStream_t cs = H2TAP_CASC_MAIN ? st : r->st2;
         if (nblk_c) {
             const unsigned gc = (unsigned)std::min<uint64_t>(cdiv(nblk_c, 2), (uint64_t)r->n_sm * kCascCtasPerSm);
             k_casc_cols<<<gc, kThreads, 0, cs>>>(old_cols_nc, E, hd_bits, hd_rows, dc, casc_mask);

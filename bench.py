@@ -544,6 +544,13 @@ def run_gpu(args):
                     "h2d_bytes_per_step": int(sum(s["h2d_bytes"] for s in e_stats) / len(e_stats)),
                     "d2h_bytes_per_step": int(sum(s["d2h_bytes"] for s in e_stats) / len(e_stats))},
             "clocks": clk.summary(),
+            "host": host_info(),
+            "paper_context": {"what": "the paper's propagation of 2,014,347 SF10 deltas: scan 2595.95 ms + Algorithm 2 "
+                                      "merge into the CPU CSR 2064.44 ms = 4660.39 ms (~432 K deltas/s), then 720.64 ms "
+                                      "to copy the CSR to an A100 over PCIe 4.0",
+                              "hardware": "2x AMD EPYC 7F52 + 1x A100 40 GB", "source": "PAPER.md P:L1899, "
+                              "P:L1913, P:L1933-1936", "note": "context, not a target: other hardware, deltas "
+                                                               "not flat ops"},
         }
         if route:
             line["nvlink"] = route

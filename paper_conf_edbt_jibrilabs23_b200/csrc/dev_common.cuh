@@ -2,7 +2,7 @@
 //
 //  * block-wide exclusive scans over per-thread item counts (warp shuffles + smem)
 //  * decoupled look-back (Merrill & Garland single-pass scan): each tile publishes
-//    its aggregate, then one warp inspects 32 predecessors at a time until it
+//    its aggregate, then one warp inspects 128 predecessors at a time until it
 //    meets an inclusive prefix.  Status word: 2-bit flag | 62-bit value.
 //    Tiles take their index from an atomic counter, so every predecessor of a
 //    spinning tile has already been scheduled (forward progress).
@@ -81,7 +81,15 @@ __device__ __forceinline__ void st_volatile(uint64_t* p, uint64_t v) {
 
 // Called by ONE full warp of the tile.  Publishes `aggregate` for `tile`, looks
 // back over predecessors, publishes the inclusive prefix, returns the exclusive
-// prefix (identical in all lanes).
+// prefix (identical in all lanes).  Each step reads 128 predecessors (4 per lane,
+// nearest first): when every tile of a grid publishes at about the same time, the
+// frontier of resolved prefixes advances one step-window per L2 round trip, so the
+// window width - not the tile work - bounds how fast a grid of thousands of tiles
+// drains (32 per step made it the critical path of the select / classify kernels).
+#ifndef H2TAP_LOOKQ
+#define H2TAP_LOOKQ 4
+#endif
+constexpr int kLookQ = H2TAP_LOOKQ;
 __device__ __forceinline__ uint64_t lookback_warp(uint64_t* status, uint32_t tile, uint64_t aggregate) {
     if (tile == 0) {
         if (lane_id() == 0) st_volatile(&status[0], kFlagPrefix | aggregate);
@@ -91,17 +99,28 @@ __device__ __forceinline__ uint64_t lookback_warp(uint64_t* status, uint32_t til
     uint64_t excl = 0;
     int64_t t = (int64_t)tile - 1;
     while (true) {
-        int64_t idx = t - (int64_t)lane_id();  // lane 0 = nearest predecessor
-        uint64_t s = (idx >= 0) ? ld_volatile(&status[idx]) : kFlagPrefix;  // virtual prefix 0 before tile 0
-        uint32_t not_ready = __ballot_sync(0xffffffffu, (s >> 62) == 0);
-        if (not_ready) { continue; }  // spin until all 32 visible (predecessors are scheduled)
-        uint32_t is_prefix = __ballot_sync(0xffffffffu, (s >> 62) == 2);
-        // nearest prefix lane (smallest lane index with prefix)
-        int first = is_prefix ? (__ffs(is_prefix) - 1) : 32;
-        uint64_t v = ((int)lane_id() <= first) ? (s & kValMask) : 0;
+        uint64_t s[kLookQ];
+        bool not_ready = false;
+#pragma unroll
+        for (int q = 0; q < kLookQ; ++q) {
+            const int64_t idx = t - (int64_t)(lane_id() * kLookQ + q);   // lane 0, q 0 = nearest
+            s[q] = (idx >= 0) ? ld_volatile(&status[idx]) : kFlagPrefix;  // virtual prefix 0 before tile 0
+            not_ready |= (s[q] >> 62) == 0;
+        }
+        if (__any_sync(0xffffffffu, not_ready)) continue;  // spin until all are visible (predecessors are scheduled)
+        int fq = kLookQ;  // this lane's nearest prefix
+#pragma unroll
+        for (int q = kLookQ - 1; q >= 0; --q)
+            if ((s[q] >> 62) == 2) fq = q;
+        const uint32_t has = __ballot_sync(0xffffffffu, fq < kLookQ);
+        const int first = has ? (__ffs(has) - 1) : 32;  // lane holding the nearest prefix
+        uint64_t v = 0;
+#pragma unroll
+        for (int q = 0; q < kLookQ; ++q)
+            if ((int)lane_id() < first || ((int)lane_id() == first && q <= fq)) v += s[q] & kValMask;
         excl += warp_sum(v);
-        if (is_prefix) break;
-        t -= 32;
+        if (has) break;
+        t -= 32 * kLookQ;
     }
     if (lane_id() == 0) st_volatile(&status[tile], kFlagPrefix | (excl + aggregate));
     return excl;

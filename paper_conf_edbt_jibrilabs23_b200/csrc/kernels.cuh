@@ -154,7 +154,16 @@ __global__ void __launch_bounds__(kThreads) k_partition(
         }
     }
     if (bad) atomicOr(&c->status, (unsigned long long)bad);
-    if (tmin != ~0ull) {
+    // node-op ranges: reduced per warp first (one atomic per warp, not per thread: a node-heavy
+    // batch would otherwise serialise thousands of atomics on four addresses)
+#pragma unroll
+    for (int o = 16; o > 0; o >>= 1) {
+        tmin = min(tmin, (uint64_t)__shfl_xor_sync(0xffffffffu, tmin, o));
+        tmax = max(tmax, (uint64_t)__shfl_xor_sync(0xffffffffu, tmax, o));
+        vmin = min(vmin, (uint64_t)__shfl_xor_sync(0xffffffffu, vmin, o));
+        vmax = max(vmax, (uint64_t)__shfl_xor_sync(0xffffffffu, vmax, o));
+    }
+    if (lane_id() == 0 && tmin != ~0ull) {
         atomicMin(&c->ts_min, tmin); atomicMax(&c->ts_max, tmax);
         atomicMin(&c->v_min, vmin); atomicMax(&c->v_max, vmax);
     }
@@ -459,9 +468,13 @@ __global__ void k_rec_expand(const DeltaRec* __restrict__ rec, uint64_t n, const
 __global__ void k_rec_consume(DeltaRec* __restrict__ rec, uint64_t n, uint64_t vis_ts,
                               unsigned long long* __restrict__ first_pending) {
     const uint64_t i = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x;
-    if (i >= n || !rec[i].valid) return;
-    if (rec[i].ts <= vis_ts) rec[i].valid = 0;
-    else atomicMin(first_pending, (unsigned long long)i);
+    bool pend = false;
+    if (i < n && rec[i].valid) {
+        if (rec[i].ts <= vis_ts) rec[i].valid = 0;
+        else pend = true;
+    }
+    const uint32_t m = __ballot_sync(0xffffffffu, pend);   // the warp's lowest pending index
+    if (m && lane_id() == (uint32_t)(__ffs(m) - 1)) atomicMin(first_pending, (unsigned long long)i);
 }
 
 // ===================================================================== a2 ====

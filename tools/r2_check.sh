@@ -1,6 +1,7 @@
 #!/bin/bash
 # round-2 GPU check: new tests, variant benches, dyn and store benches -> gpurun_out/<tag>/
 tag=${1:-r2check}; out=gpurun_out/$tag; mkdir -p $out
+python -c "import __graft_entry__ as g; g.smoke()" > $out/smoke.txt 2>&1
 timeout 1500 python -m pytest tests/test_gpu_store.py tests/test_gpu_dynamic.py tests/test_gpu_parity.py \
     tests/test_gpu_records.py tests/test_gpu_sharded.py tests/test_gpu_sharded_mp.py tests/test_gpu_tombstone.py \
     -x -q --durations=10 > $out/pytest.txt 2>&1
@@ -20,3 +21,4 @@ for v in base rslook16; do
   lib=""; [ $v != base ] && lib="H2TAP_LIB=build/libh2tap_$v.so"
   env $lib timeout 600 python bench.py --config c4 --steps 5 --no-cpu-baseline > $out/bench_c4_$v.json 2> $out/bench_c4_$v.err
 done
+python -c 'import __graft_entry__ as g; g.smoke()' > $out/smoke.txt 2>&1

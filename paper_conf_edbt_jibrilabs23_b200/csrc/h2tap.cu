@@ -202,6 +202,9 @@ struct h2tap_replica {
             size_t nc = need + need / 8;
             b.p = dalloc(nc);
             b.cap = nc;
+            // defined contents once: 128-bit loads and sector probes may read the slack past
+            // the live elements (masked off, never used) - compute-sanitizer initcheck clean
+            CK(cudaMemsetAsync(b.p, 0, nc, st));
         }
         return static_cast<T*>(b.p);
     }

@@ -45,6 +45,9 @@ struct h2tap_delta_store {
     uint64_t freed_r = 0, freed_i = 0, freed_d = 0;   // host chunks released below these
     cudaStream_t cs = nullptr;
     cudaEvent_t ev = nullptr;
+    std::mutex free_mu;                 // recycled pinned chunks by size class:
+    std::vector<void*> free_chunks[3];  // records, 8-byte payload, (unused)
+    int chunk_class(size_t bytes) const { return bytes == crec * sizeof(DeltaRec) ? 0 : 1; }
     h2tap_delta_store() {
         for (uint64_t i = 0; i < kMaxChunks; ++i) { rch[i] = nullptr; bmin[i] = nullptr; ich[i] = nullptr; wch[i] = nullptr; dch[i] = nullptr; }
     }
@@ -52,11 +55,23 @@ struct h2tap_delta_store {
 
 namespace {
 
+// pinned chunks are recycled (cudaHostAlloc / cudaFreeHost cost milliseconds and synchronise):
+// a released chunk goes to its size class's free list and the next reservation takes it
 template <typename T>
-T* host_chunk(uint64_t n) {
+T* host_chunk(h2tap_delta_store* s, uint64_t n) {
     void* p = nullptr;
-    CK(cudaHostAlloc(&p, n * sizeof(T), cudaHostAllocPortable));
+    {
+        std::lock_guard<std::mutex> g(s->free_mu);
+        std::vector<void*>& f = s->free_chunks[s->chunk_class(n * sizeof(T))];
+        if (!f.empty()) { p = f.back(); f.pop_back(); }
+    }
+    if (!p) CK(cudaHostAlloc(&p, n * sizeof(T), cudaHostAllocPortable));
     return static_cast<T*>(p);
+}
+void release_chunk(h2tap_delta_store* s, void* p, size_t bytes) {
+    if (!p) return;
+    std::lock_guard<std::mutex> g(s->free_mu);
+    s->free_chunks[s->chunk_class(bytes)].push_back(p);
 }
 
 // under s->mu: chunks for records [r0, r1) and payload [i0, i1), [d0, d1)
@@ -73,12 +88,12 @@ void ds_reserve_chunks(h2tap_delta_store* s, uint64_t r0, uint64_t r1, uint64_t 
             auto* bm = new std::atomic<uint64_t>[nb];
             for (uint64_t b = 0; b < nb; ++b) bm[b] = ~0ull;
             s->bmin[c].store(bm);
-            s->rch[c].store(host_chunk<DeltaRec>(s->crec));
+            s->rch[c].store(host_chunk<DeltaRec>(s, s->crec));
         }
     for (uint64_t c = i0 / s->cpay; c * s->cpay < i1; ++c)
-        if (!s->ich[c].load()) { s->ich[c].store(host_chunk<uint64_t>(s->cpay)); s->wch[c].store(host_chunk<double>(s->cpay)); }
+        if (!s->ich[c].load()) { s->ich[c].store(host_chunk<uint64_t>(s, s->cpay)); s->wch[c].store(host_chunk<double>(s, s->cpay)); }
     for (uint64_t c = d0 / s->cpay; c * s->cpay < d1; ++c)
-        if (!s->dch[c].load()) s->dch[c].store(host_chunk<uint64_t>(s->cpay));
+        if (!s->dch[c].load()) s->dch[c].store(host_chunk<uint64_t>(s, s->cpay));
 }
 
 // copy n elements starting at absolute position a of a chunked host array into dst
@@ -161,14 +176,15 @@ void ds_pos(const h2tap_delta_store* s, uint64_t i, uint64_t n_pub, uint64_t pin
 
 void ds_release_below(h2tap_delta_store* s, uint64_t rec_lo, uint64_t ins_lo, uint64_t del_lo) {
     for (; (s->freed_r + 1) * s->crec <= rec_lo; ++s->freed_r) {
-        cudaFreeHost(s->rch[s->freed_r].exchange(nullptr));
+        release_chunk(s, s->rch[s->freed_r].exchange(nullptr), s->crec * sizeof(DeltaRec));
         delete[] s->bmin[s->freed_r].exchange(nullptr);
     }
     for (; (s->freed_i + 1) * s->cpay <= ins_lo; ++s->freed_i) {
-        cudaFreeHost(s->ich[s->freed_i].exchange(nullptr));
-        cudaFreeHost(s->wch[s->freed_i].exchange(nullptr));
+        release_chunk(s, s->ich[s->freed_i].exchange(nullptr), s->cpay * 8);
+        release_chunk(s, s->wch[s->freed_i].exchange(nullptr), s->cpay * 8);
     }
-    for (; (s->freed_d + 1) * s->cpay <= del_lo; ++s->freed_d) cudaFreeHost(s->dch[s->freed_d].exchange(nullptr));
+    for (; (s->freed_d + 1) * s->cpay <= del_lo; ++s->freed_d)
+        release_chunk(s, s->dch[s->freed_d].exchange(nullptr), s->cpay * 8);
 }
 
 }  // namespace
@@ -325,6 +341,8 @@ void h2tap_ds_destroy(h2tap_delta_store* s) {
         if (double* p = s->wch[c].load()) cudaFreeHost(p);
         if (uint64_t* p = s->dch[c].load()) cudaFreeHost(p);
     }
+    for (auto& f : s->free_chunks)
+        for (void* p : f) cudaFreeHost(p);
     for (void* p : {(void*)s->m_rec, (void*)s->m_ins, (void*)s->m_w, (void*)s->m_del}) if (p) cudaFree(p);
     if (s->ev) cudaEventDestroy(s->ev);
     if (s->cs) cudaStreamDestroy(s->cs);

@@ -81,13 +81,12 @@ __device__ __forceinline__ void st_volatile(uint64_t* p, uint64_t v) {
 
 // Called by ONE full warp of the tile.  Publishes `aggregate` for `tile`, looks
 // back over predecessors, publishes the inclusive prefix, returns the exclusive
-// prefix (identical in all lanes).  Each step reads 128 predecessors (4 per lane,
-// nearest first): when every tile of a grid publishes at about the same time, the
-// frontier of resolved prefixes advances one step-window per L2 round trip, so the
-// window width - not the tile work - bounds how fast a grid of thousands of tiles
-// drains (32 per step made it the critical path of the select / classify kernels).
+// prefix (identical in all lanes).  Each step reads 32 * kLookQ predecessors
+// (kLookQ per lane, nearest first).  Measured on B200 (round 2): 4 or 8 per lane made
+// the 1M-item select / classify kernels slower (more L2 traffic while spinning on
+// predecessors that have not published yet), so the default stays at 1.
 #ifndef H2TAP_LOOKQ
-#define H2TAP_LOOKQ 4
+#define H2TAP_LOOKQ 1
 #endif
 constexpr int kLookQ = H2TAP_LOOKQ;
 __device__ __forceinline__ uint64_t lookback_warp(uint64_t* status, uint32_t tile, uint64_t aggregate) {

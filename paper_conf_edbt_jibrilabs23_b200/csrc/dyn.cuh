@@ -196,7 +196,9 @@ struct Tabs {
     uint32_t* used;   // live keys + tombstones
     uint32_t* key;    // slab: destination dense ids, EMPTY / TOMB
     float* val;       // slab: weights
+    uint32_t* own;    // slab: owner vertex of every 4-slot group (kNoOwner: free or garbage)
 };
+constexpr uint32_t kNoOwner = 0xFFFFFFFFu;
 __device__ __forceinline__ uint32_t pow2_cap(uint64_t live) {  // load <= 1/2, >= 4 slots
     uint32_t c = 4;
     while ((uint64_t)c < 2 * live) c <<= 1;
@@ -254,6 +256,8 @@ __global__ void k_dyn_grow(const uint32_t* __restrict__ grow_v, const uint32_t* 
             const uint32_t k = T.key[ob + j];
             if (k < kKTomb) tab_claim(T.key, T.val, nb, nc - 1, k, T.val[ob + j]);
         }
+        for (uint32_t q = lane; q < nc / 4; q += 32) T.own[nb / 4 + q] = v;
+        for (uint32_t q = lane; q < oc / 4; q += 32) T.own[ob / 4 + q] = kNoOwner;
         __syncwarp();
         if (lane == 0) {
             T.base[v] = nb;
@@ -356,7 +360,7 @@ __global__ void k_dyn_caps(const uint32_t* __restrict__ cnt, uint64_t V, uint64_
     else if (v == V) capn[V] = 0;
 }
 __global__ void k_dyn_rebuild(Tabs T, uint64_t V, const uint64_t* __restrict__ capn, const uint64_t* __restrict__ nbase,
-                              uint32_t* __restrict__ nkey, float* __restrict__ nval) {
+                              uint32_t* __restrict__ nkey, float* __restrict__ nval, uint32_t* __restrict__ nown) {
     const uint64_t nw = ((uint64_t)gridDim.x * blockDim.x) >> 5;
     const uint32_t lane = threadIdx.x & 31;
     for (uint64_t v = (blockIdx.x * (uint64_t)blockDim.x + threadIdx.x) >> 5; v < V; v += nw) {
@@ -366,6 +370,7 @@ __global__ void k_dyn_rebuild(Tabs T, uint64_t V, const uint64_t* __restrict__ c
             const uint32_t k = T.key[ob + j];
             if (k < kKTomb) tab_claim(nkey, nval, nb, nc - 1, k, T.val[ob + j]);
         }
+        for (uint32_t q = lane; q < nc / 4; q += 32) nown[nb / 4 + q] = (uint32_t)v;
         __syncwarp();
         if (lane == 0) { T.base[v] = nb; T.cap[v] = nc; T.used[v] = T.cnt[v]; }
     }
@@ -388,75 +393,66 @@ __global__ void k_dyn_node_del(const uint64_t* __restrict__ del_ids, uint64_t nd
     wadd(&c->n_vdel, died);
 }
 
-// line 11's cascade: a key is removed iff an endpoint died this cycle (bitmap, V/8 bytes,
-// L2-resident).  A 32 KB filter (bit v mod 2^18 of every dead vertex) in shared memory
-// screens the keys; the exact bitmap is read only on a filter hit.  Pass 0: thread per
-// vertex for tables of <= 32 slots (16-byte loads); larger tables are queued for pass 1
-// (warp per table).  A dead vertex's own table is dropped (its keys are cascaded).
+// line 11's cascade.  First the dead vertices' own tables are dropped (their keys are
+// cascaded; the slots become garbage).  Then one linear pass over the slab: a key is removed
+// iff its destination died this cycle (bitmap, V/8 bytes, L2-resident; a 32 KB shared-memory
+// filter of the dead ids screens the keys before the bitmap is read).  16-byte loads of 4-slot
+// groups, coalesced; only a group with a hit reads its owner (garbage groups have none and are
+// skipped) to turn the keys into tombstones and lower the owner's live count.
 __device__ __forceinline__ bool died_of(const uint32_t* __restrict__ b, const uint32_t* __restrict__ filt, uint32_t d) {
     const uint32_t fd = d & (kFilterBits - 1);
     if (((filt[fd >> 5] >> (fd & 31)) & 1u) == 0) return false;
     return (__ldg(b + (d >> 5)) >> (d & 31)) & 1u;
 }
-template <int kPass>
-__global__ void __launch_bounds__(256) k_dyn_cascade(Tabs T, uint64_t V, const uint32_t* __restrict__ died_bits,
-        const uint32_t* __restrict__ filter, uint32_t* __restrict__ big, Ctr* __restrict__ c) {
+__global__ void k_dyn_drop_dead(const uint64_t* __restrict__ del_ids, uint64_t nd, const uint64_t* __restrict__ ext,
+                                uint64_t V, const uint32_t* __restrict__ died_bits, Tabs T, Ctr* __restrict__ c) {
+    const uint64_t i = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x;
+    if (i >= nd) return;
+    const int64_t d = find_ext(ext, V, del_ids[i]);
+    if (d < 0 || !((died_bits[d >> 5] >> (d & 31)) & 1u)) return;
+    const uint32_t cap = atomicExch(&T.cap[d], 0u);   // a vertex listed twice is dropped once
+    if (!cap) return;
+    const uint64_t b = T.base[d];
+    for (uint32_t q = 0; q < cap / 4; ++q) T.own[b / 4 + q] = kNoOwner;
+    atomicAdd(&c->n_casc, (unsigned long long)T.cnt[d]);
+    atomicAdd(&c->garbage, (unsigned long long)cap);
+    T.cnt[d] = 0;
+    T.used[d] = 0;
+}
+__global__ void __launch_bounds__(256, 4) k_dyn_cascade(Tabs T, uint64_t groups, const uint32_t* __restrict__ died_bits,
+                                                        const uint32_t* __restrict__ filter, Ctr* __restrict__ c) {
     if (*(volatile unsigned long long*)&c->n_vdel == 0) return;   // nobody died this cycle (no host sync)
     extern __shared__ uint32_t filt[];
     for (uint32_t t = threadIdx.x; t < kFilterBits / 32; t += blockDim.x) filt[t] = filter[t];
     __syncthreads();
-    unsigned long long gone = 0, garb = 0;
-    if (kPass == 0) {
-        const uint64_t stride = (uint64_t)gridDim.x * blockDim.x;
-        for (uint64_t u = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; u < V; u += stride) {
-            const uint32_t cap = T.cap[u];
-            if (!cap) continue;
-            if ((__ldg(died_bits + (u >> 5)) >> (u & 31)) & 1u) {   // its out-edges go with it
-                gone += T.cnt[u];
-                garb += cap;
-                T.cap[u] = 0; T.cnt[u] = 0; T.used[u] = 0;
-                continue;
-            }
-            if (cap > 32) { big[atomicAdd(&c->n_big_casc, 1ull)] = (uint32_t)u; continue; }
-            uint4* q = reinterpret_cast<uint4*>(T.key + T.base[u]);
-            uint32_t hits = 0;
-            for (uint32_t j = 0; j < cap / 4; ++j) {
-                uint4 k = q[j];
-                bool w = false;
-                uint32_t* kk = reinterpret_cast<uint32_t*>(&k);
+    const uint64_t stride = (uint64_t)gridDim.x * blockDim.x;
+    uint4* g4 = reinterpret_cast<uint4*>(T.key);
+    unsigned long long gone = 0;
+    constexpr int U = 4;   // 4 independent 16-byte loads in flight per thread
+    uint64_t g = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x;
+    auto visit = [&](uint64_t q, uint4 k) {
+        uint32_t* kk = reinterpret_cast<uint32_t*>(&k);
+        uint32_t hits = 0;
 #pragma unroll
-                for (int e = 0; e < 4; ++e)
-                    if (kk[e] < kKTomb && died_of(died_bits, filt, kk[e])) { kk[e] = kKTomb; w = true; ++hits; }
-                if (w) q[j] = k;
-            }
-            if (hits) { T.cnt[u] -= hits; gone += hits; }
-        }
-    } else {
-        const uint64_t nb = c->n_big_casc, nw = ((uint64_t)gridDim.x * blockDim.x) >> 5;
-        const uint32_t lane = threadIdx.x & 31;
-        for (uint64_t q = (blockIdx.x * (uint64_t)blockDim.x + threadIdx.x) >> 5; q < nb; q += nw) {
-            const uint32_t u = big[q], cap = T.cap[u];
-            uint4* p = reinterpret_cast<uint4*>(T.key + T.base[u]);
-            uint32_t hits = 0;
-            for (uint32_t j = lane; j < cap / 4; j += 32) {
-                uint4 k = p[j];
-                bool w = false;
-                uint32_t* kk = reinterpret_cast<uint32_t*>(&k);
+        for (int e = 0; e < 4; ++e)
+            if (kk[e] < kKTomb && died_of(died_bits, filt, kk[e])) { kk[e] = kKTomb; ++hits; }
+        if (!hits) return;
+        const uint32_t o = T.own[q];
+        if (o == kNoOwner) return;   // garbage: stale keys of a moved or dropped table
+        g4[q] = k;
+        atomicSub(&T.cnt[o], hits);
+        gone += hits;
+    };
+    for (; g + (U - 1) * stride < groups; g += U * stride) {
+        uint4 k[U];
 #pragma unroll
-                for (int e = 0; e < 4; ++e)
-                    if (kk[e] < kKTomb && died_of(died_bits, filt, kk[e])) { kk[e] = kKTomb; w = true; ++hits; }
-                if (w) p[j] = k;
-            }
-            hits = warp_sum<uint32_t>(hits);
-            if (lane == 0 && hits) { T.cnt[u] -= hits; gone += hits; }
-        }
+        for (int u = 0; u < U; ++u) k[u] = __ldcs(g4 + g + u * stride);
+#pragma unroll
+        for (int u = 0; u < U; ++u) visit(g + u * stride, k[u]);
     }
+    for (; g < groups; g += stride) visit(g, g4[g]);
     gone = warp_sum<unsigned long long>(gone);
-    garb = warp_sum<unsigned long long>(garb);
-    if ((threadIdx.x & 31) == 0) {
-        if (gone) atomicAdd(&c->n_casc, gone);
-        if (garb) atomicAdd(&c->garbage, garb);
-    }
+    if ((threadIdx.x & 31) == 0 && gone) atomicAdd(&c->n_casc, gone);
 }
 
 // create: flat edge list -> packed keys (an endpoint that is no vertex -> bad)
@@ -639,7 +635,7 @@ struct h2tap_dyn {
     h2tap_replica* r = nullptr;   // stream, allocator, radix-sort scratch
     uint64_t V = 0, n_live = 0, xid = 0;   // xid = ext[V - 1] (host copy)
     uint64_t slab_cap = 0, tail = 0, garbage = 0;   // slab slots, allocated slots, garbage slots
-    Buf ext, live, base, cap, cnt, used, key, val, inc, grow_v, grow_cap, died, big;
+    Buf ext, live, base, cap, cnt, used, key, val, own, inc, grow_v, grow_cap, died, big;
     Buf cin, oin, new_ids, del_ids, kill, flag, fpos, keys, vals, keys2, vals2, witem, ctr, xo;
     Buf x_rec, x_ins, x_wts, x_del, live8, fa, fb, lvl, da, db;
     struct Stage {
@@ -656,13 +652,14 @@ namespace {
 dyn::Tabs dyn_tabs(h2tap_dyn* d) {
     return dyn::Tabs{static_cast<uint64_t*>(d->base.p), static_cast<uint32_t*>(d->cap.p),
                      static_cast<uint32_t*>(d->cnt.p), static_cast<uint32_t*>(d->used.p),
-                     static_cast<uint32_t*>(d->key.p), static_cast<float*>(d->val.p)};
+                     static_cast<uint32_t*>(d->key.p), static_cast<float*>(d->val.p),
+                     static_cast<uint32_t*>(d->own.p)};
 }
 
 void dyn_free(h2tap_dyn* d) {
     if (!d) return;
     if (d->r) {
-        for (Buf* b : {&d->ext, &d->live, &d->base, &d->cap, &d->cnt, &d->used, &d->key, &d->val, &d->inc,
+        for (Buf* b : {&d->ext, &d->live, &d->base, &d->cap, &d->cnt, &d->used, &d->key, &d->val, &d->own, &d->inc,
                        &d->grow_v, &d->grow_cap, &d->died, &d->big, &d->cin, &d->oin, &d->new_ids, &d->del_ids,
                        &d->kill, &d->flag, &d->fpos, &d->keys, &d->vals, &d->keys2, &d->vals2, &d->witem, &d->ctr,
                        &d->xo, &d->x_rec, &d->x_ins, &d->x_wts, &d->x_del, &d->live8, &d->fa, &d->fb, &d->lvl,
@@ -733,17 +730,21 @@ void dyn_rebuild(h2tap_dyn* d, uint64_t extra) {
     CK(cudaMemcpyAsync(&total, nbase + V, 8, cudaMemcpyDeviceToHost, st));
     r->sync();
     const uint64_t ncap = ((total + extra) * 5 / 4 + 1023) & ~1023ull;
-    Buf k2, v2;
+    Buf k2, v2, o2;
     uint32_t* nk = r->get<uint32_t>(k2, ncap);
     float* nv = r->get<float>(v2, ncap);
+    uint32_t* no = r->get<uint32_t>(o2, ncap / 4);
     CK(cudaMemsetAsync(nk, 0xFF, (ncap + 16) * 4, st));
+    CK(cudaMemsetAsync(no, 0xFF, (ncap / 4 + 16) * 4, st));
     if (V) {
         const unsigned grid = (unsigned)std::min<uint64_t>(cdiv(V * 32, 256), (uint64_t)r->n_sm * 16);
-        dyn::k_dyn_rebuild<<<grid, 256, 0, st>>>(dyn_tabs(d), V, capn, nbase, nk, nv);
+        dyn::k_dyn_rebuild<<<grid, 256, 0, st>>>(dyn_tabs(d), V, capn, nbase, nk, nv, no);
         CKL();
     }
     r->release(d->key);
     r->release(d->val);
+    r->release(d->own);
+    d->own = o2;
     r->release(bc);
     r->release(bb);
     d->key = k2;
@@ -955,16 +956,15 @@ h2tap_status dyn_apply(h2tap_dyn* d, const h2tap_record_batch* b, h2tap_apply_st
         CK(cudaMemsetAsync(died, 0, (nwd + nwf) * 4, st));
         dyn::k_dyn_node_del<<<g1(h0.n_del_ids), 256, 0, st>>>(del_ids, h0.n_del_ids, ext, d->V, live, died, filter, c);
         CKL();
-        if (d->V) {
+        dyn::k_dyn_drop_dead<<<g1(h0.n_del_ids), 256, 0, st>>>(del_ids, h0.n_del_ids, ext, d->V, died, dyn_tabs(d), c);
+        CKL();
+        if (d->tail) {
             constexpr int smem = dyn::kFilterBits / 8;
-            CK(cudaFuncSetAttribute(dyn::k_dyn_cascade<0>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem));
-            CK(cudaFuncSetAttribute(dyn::k_dyn_cascade<1>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem));
-            uint32_t* bigv = r->get<uint32_t>(d->grow_v, d->V);
-            const unsigned grid = (unsigned)std::min<uint64_t>(g1(d->V), (uint64_t)r->n_sm * 4);  // 4 CTAs/SM
+            CK(cudaFuncSetAttribute(dyn::k_dyn_cascade, cudaFuncAttributeMaxDynamicSharedMemorySize, smem));
+            const uint64_t groups = d->tail / 4;
+            const unsigned grid = (unsigned)std::min<uint64_t>(g1(groups), (uint64_t)r->n_sm * 4);  // 4 CTAs/SM
             CK(cudaEventRecord(r->ev[2], st));
-            dyn::k_dyn_cascade<0><<<grid, 256, smem, st>>>(dyn_tabs(d), d->V, died, filter, bigv, c);
-            CKL();
-            dyn::k_dyn_cascade<1><<<(unsigned)r->n_sm * 4, 256, smem, st>>>(dyn_tabs(d), d->V, died, filter, bigv, c);
+            dyn::k_dyn_cascade<<<grid, 256, smem, st>>>(dyn_tabs(d), groups, died, filter, c);
             CKL();
             CK(cudaEventRecord(r->ev[3], st));
             casc_timed = true;
@@ -989,7 +989,7 @@ h2tap_status dyn_apply(h2tap_dyn* d, const h2tap_record_batch* b, h2tap_apply_st
         stats->ms_total = ev_ms(r->ev[0], r->ev[1]);
         if (casc_timed && h.n_vdel) {   // the cascade pass: its launch time and the table bytes it streams
             stats->ms_merge = ev_ms(r->ev[2], r->ev[3]);
-            stats->bytes_merge = (d->tail - d->garbage) * 4 + d->V * 16;
+            stats->bytes_merge = d->tail * 4;   // the linear pass reads every allocated slot once
         }
         // algorithmic bytes: records + slices read, one probe (4-byte key + 4-byte weight) per item
         stats->bytes_alg = nr * sizeof(DeltaRec) + n_ins * 12 + tot[1] * 8 + (n_ins + tot[1]) * 8;
@@ -1088,7 +1088,7 @@ h2tap_status h2tap_dyn_create(const h2tap_config* cfg, size_t n_vertices, const 
             CK(cudaMemcpyAsync(&d->xid, ext + n_vertices - 1, 8, cudaMemcpyDeviceToHost, r->st));
             r->sync();
         }
-        dyn_rebuild(d, n_edges);   // an empty slab with room for the edges' tables
+        dyn_rebuild(d, 3 * n_edges);   // an empty slab with room for the edges' tables (load >= 1/4)
         if (n_edges) {
             dyn_item_bufs(d, n_edges);
             const uint64_t *s2 = src, *d2 = dst;

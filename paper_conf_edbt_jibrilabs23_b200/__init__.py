@@ -698,7 +698,7 @@ class DeltaStore:
     delta records + inserts / 8-byte weights / deletes arrays on the host, mirrored to the GPU
     by the propagation cycle (Replica.apply_store)."""
 
-    def __init__(self, device: int = 0, chunk_records: int = 1 << 16):
+    def __init__(self, device: int = 0, chunk_records: int = 1 << 20):
         h = _P()
         _check(_lib.h2tap_ds_create(int(device), int(chunk_records), ctypes.byref(h)), "h2tap_ds_create")
         self._h = h

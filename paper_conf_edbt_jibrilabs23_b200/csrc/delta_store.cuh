@@ -386,11 +386,15 @@ h2tap_status h2tap_delta_apply_store(h2tap_replica* r, h2tap_delta_store* s, uin
         uint64_t h2d = ds_mirror(s, end, ie, de);
         CK(cudaEventRecord(s->ev, s->cs));
         CK(cudaStreamWaitEvent(st, s->ev, 0));
-        h2d += ds_mirror(s, np, pins, pdel);  // read-ahead: overlaps the cycle below
         const uint64_t nr = end - s->cursor;
         DeltaRec* rec = s->m_rec + (s->cursor - s->mbase);
+        // read-ahead: the copies of the not-yet-needed deltas are issued while the scan kernels run
+        // and overlap the rest of the cycle (the mirror's capacity was reserved above)
+        uint64_t ra = 0;
         h2tap_status rc = apply_records_dev(r, rec, nr, s->m_ins, nullptr, s->m_w, ie - s->ibase, s->m_del,
-                                            de - s->dbase, snapshot_ts, s->ibase, s->dbase, snapshot_ts, stats);
+                                            de - s->dbase, snapshot_ts, s->ibase, s->dbase, snapshot_ts, stats,
+                                            [&] { ra = ds_mirror(s, np, pins, pdel); });
+        h2d += ra;
         if (stats) stats->h2d_bytes += h2d;
         if (rc != H2TAP_OK) return rc;
         // consumed records -> invalid; the first still-pending record becomes the cursor

@@ -17,6 +17,7 @@
 #include <cstdlib>
 #include <cstdio>
 #include <cstring>
+#include <functional>
 #include <atomic>
 #include <mutex>
 #include <new>
@@ -1347,7 +1348,8 @@ namespace {
 h2tap_status apply_records_dev(h2tap_replica* r, const DeltaRec* rec, uint64_t nr, const uint64_t* ins,
                                const float* wts, const double* wts64, uint64_t n_ins, const uint64_t* del,
                                uint64_t n_del, uint64_t vis_ts, uint64_t ins_base, uint64_t del_base,
-                               uint64_t snapshot_ts, h2tap_apply_stats* stats) {
+                               uint64_t snapshot_ts, h2tap_apply_stats* stats,
+                               const std::function<void()>& overlap = {}) {
     cudaStream_t st = r->st;
     uint64_t* cnt = r->get<uint64_t>(r->xcnt, nr + 1);
     uint64_t* off = r->get<uint64_t>(r->xoff, nr + 1);
@@ -1367,6 +1369,7 @@ h2tap_status apply_records_dev(h2tap_replica* r, const DeltaRec* rec, uint64_t n
     unsigned long long h[2] = {0, 0};
     CK(cudaMemcpyAsync(h, tb, 16, cudaMemcpyDeviceToHost, st));
     g_d2h += 16;
+    if (overlap) overlap();  // host work that can run while the scan kernels execute
     r->sync();  // the expanded op count sizes the work buffers
     if (h[1] & REC_BAD_FLAG) { set_err("delta record flag other than 0/1"); return H2TAP_E_INVAL; }
     if (h[1] & REC_BAD_SLICE) { set_err("delta record slice outside the inserts/weights/deletes arrays"); return H2TAP_E_INVAL; }

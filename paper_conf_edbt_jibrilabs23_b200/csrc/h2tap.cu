@@ -119,7 +119,7 @@ struct h2tap_replica {
         uint64_t bytes = 0;  // staged H2D bytes not yet accounted to an apply
     } stg[2];
     int stg_next = 0;
-    cudaEvent_t evA = nullptr, evB = nullptr, evC = nullptr;
+    cudaEvent_t evA = nullptr, evB = nullptr, evC = nullptr, evD = nullptr;
     uint64_t V = 0, E = 0, snap = 0, next_seq = 0, n_pend = 0;
     // sharding: V = global live vertices (the replicated ID map), the CSR holds the Vr rows
     // of the owned external-ID range starting at global dense id row_lo
@@ -137,7 +137,7 @@ struct h2tap_replica {
     Buf keyA, keyB, valA, valB, hist, dbase, rs_status, rs_ctr, rs_coop;
     Buf nv, nv_ext, dropped, ins_q, ins_oldpos, hd_rows, hd_bits;
     Buf op_flags, op_ou, op_ow;
-    Buf ins_pos, ins_row, ins_col, ins_w, del_pos, upd_pos, upd_w, KR;
+    Buf ins_pos, ins_row, ins_col, ins_w, del_pos, upd_pos, upd_w, KR, cls_cat, cls_pos, cls_w;
     Buf misc, nsorted, part, opart, deg, tsum, remap_shift, remap32, casc_wrel, tile_emit, tile_base, del_row, casc_mask, status2, bfs_a, bfs_b, pr_a, pr_b;
     Buf xrec, xins, xwts, xdel, xcnt, xoff;  // delta-record input (h2tap_delta_apply_records)
     bool tomb = false;  // tombstone-row mode (reading A23)
@@ -379,6 +379,7 @@ h2tap_status apply_core(h2tap_replica* r, const BatchIn& in, uint64_t S, bool cr
     for (int i = 0; i < 8; ++i)
         if (!r->ev[i]) CK(cudaEventCreate(&r->ev[i]));
     CK(cudaStreamWaitEvent(st, r->evB, 0));  // a cascade pass of an earlier (failed) cycle is done
+    CK(cudaStreamWaitEvent(st, r->evD, 0));  // and so is its merge partition (side stream)
     CK(cudaEventRecord(r->ev[0], st));
     TR("start");
 
@@ -654,19 +655,58 @@ h2tap_status apply_core(h2tap_replica* r, const BatchIn& in, uint64_t S, bool cr
         ca.del_pos = del_pos;
         ca.del_row = del_row;
         ca.upd_pos = upd_pos; ca.upd_w = upd_w;
-        uint64_t nt2 = cdiv(n_edge, kCTile);
-        ca.status3 = r->get<uint64_t>(r->status2, 3 * nt2);
-        CK(cudaMemsetAsync(ca.status3, 0, 3 * nt2 * 8, st));
-        ca.n_tiles = nt2;
+#ifndef H2TAP_CLASSIFY_SPLIT
+#define H2TAP_CLASSIFY_SPLIT 1
+#endif
         ca.c = dc;
-        k_reduce_classify<<<(unsigned)nt2, kThreads, 0, st>>>(ca);
-        CKL();
+        if (H2TAP_CLASSIFY_SPLIT) {
+            ca.kcat = r->get<uint8_t>(r->cls_cat, n_edge);
+            ca.kpos = r->get<uint64_t>(r->cls_pos, n_edge);
+            ca.kw = r->get<float>(r->cls_w, n_edge);
+            k_reduce_classify<1><<<(unsigned)cdiv(n_edge, kCTile), kThreads, 0, st>>>(ca);
+            CKL();
+            const uint64_t nt3 = cdiv(n_edge, kTile);
+            ca.status3 = r->get<uint64_t>(r->status2, 3 * nt3);
+            CK(cudaMemsetAsync(ca.status3, 0, 3 * nt3 * 8, st));
+            ca.n_tiles = nt3;
+            k_classify_compact<<<(unsigned)nt3, kThreads, 0, st>>>(ca);
+            CKL();
+        } else {
+            uint64_t nt2 = cdiv(n_edge, kCTile);
+            ca.status3 = r->get<uint64_t>(r->status2, 3 * nt2);
+            CK(cudaMemsetAsync(ca.status3, 0, 3 * nt2 * 8, st));
+            ca.n_tiles = nt2;
+            k_reduce_classify<0><<<(unsigned)nt2, kThreads, 0, st>>>(ca);
+            CKL();
+        }
         TR("classify");
     }
     CK(cudaEventRecord(r->ev[3], st));
 
-    // ---- a6: merge into the back buffer (skipped when no op can change the CSR)
+    // ---- a6 prerequisite: the merge-path partition depends only on the outcome lists (and the
+    // cascade tables, which the side stream already produces), so it runs on the side stream
+    // beside the row-offset / ID-map pass of the main stream
     const bool csr_changed = node_mode || n_edge;
+    const uint64_t Ecap_ = E + n_edge;
+    TilePart* part = nullptr;
+    MergeArgs mp{};
+    if (csr_changed && Ecap_) {
+        mp.E_old = E;
+        mp.ins_pos = ins_pos;
+        mp.del_pos = del_pos;
+        mp.upd_pos = upd_pos;
+        mp.n_tiles = cdiv(Ecap_, kMergeTile);  // upper bound; the kernels use E + n_ins
+        mp.c = dc;
+        if (node_mode) { mp.casc_mask = casc_mask; mp.casc_pre = casc_pre; }
+        part = r->get<TilePart>(r->part, mp.n_tiles + 1);
+        CK(cudaEventRecord(r->evC, st));
+        CK(cudaStreamWaitEvent(r->st2, r->evC, 0));
+        k_merge_partition<<<g1(mp.n_tiles + 1), 256, 0, r->st2>>>(mp, part);
+        CKL();
+        CK(cudaEventRecord(r->evD, r->st2));
+    }
+
+    // ---- a6: merge into the back buffer (skipped when no op can change the CSR)
     const int nb = csr_changed ? (r->cur ^ 1) : r->cur;
     int64_t* new_off = nullptr;
     const bool casc = node_mode;
@@ -751,9 +791,8 @@ h2tap_status apply_core(h2tap_replica* r, const BatchIn& in, uint64_t S, bool cr
             ma.casc_mask = casc_mask;
             ma.casc_pre = casc_pre;
         }
-        TilePart* part = r->get<TilePart>(r->part, ma.n_tiles + 1);
-        k_merge_partition<<<g1(ma.n_tiles + 1), 256, 0, st>>>(ma, part);
-        CKL();
+        CK(cudaStreamWaitEvent(st, r->evD, 0));  // the partition (side stream) is complete
+        if (casc_pending) { CK(cudaStreamWaitEvent(st, r->evB, 0)); casc_pending = false; }
         CK(cudaEventRecord(r->ev[6], st));  // merge kernel starts here (after its prerequisites)
         TR("merge_prep+casc_join");
         auto launch = [&](auto kern) {
@@ -924,6 +963,7 @@ h2tap_replica* new_replica(const h2tap_config* cfg) {
     CK(cudaEventCreateWithFlags(&r->evA, cudaEventDisableTiming));
     CK(cudaEventCreateWithFlags(&r->evB, cudaEventDisableTiming));
     CK(cudaEventCreateWithFlags(&r->evC, cudaEventDisableTiming));
+    CK(cudaEventCreateWithFlags(&r->evD, cudaEventDisableTiming));
     CK(cudaHostAlloc(reinterpret_cast<void**>(&r->hc), sizeof(Counters), cudaHostAllocMapped));
     CK(cudaHostGetDevicePointer(reinterpret_cast<void**>(&r->hc_dev), r->hc, 0));
     r->get<Counters>(r->ctr, 1);
@@ -939,7 +979,7 @@ void free_replica(h2tap_replica* r) {
                    &r->hist, &r->dbase, &r->rs_status, &r->rs_ctr, &r->rs_coop, &r->nv, &r->nv_ext, &r->dropped, &r->ins_q,
                    &r->ins_oldpos, &r->hd_rows, &r->hd_bits, &r->op_flags, &r->op_ou, &r->op_ow,
                    &r->ins_pos, &r->ins_row, &r->ins_col, &r->ins_w, &r->del_pos, &r->upd_pos, &r->upd_w,
-                   &r->KR, &r->misc, &r->nsorted, &r->part, &r->opart, &r->deg, &r->tsum, &r->remap_shift, &r->remap32, &r->casc_wrel, &r->tile_emit, &r->tile_base, &r->del_row, &r->casc_mask, &r->status2, &r->bounds_dev, &r->fence[0], &r->fence[1], &r->bfs_a, &r->bfs_b, &r->pr_a, &r->pr_b, &r->ctr,
+                   &r->KR, &r->cls_cat, &r->cls_pos, &r->cls_w, &r->misc, &r->nsorted, &r->part, &r->opart, &r->deg, &r->tsum, &r->remap_shift, &r->remap32, &r->casc_wrel, &r->tile_emit, &r->tile_base, &r->del_row, &r->casc_mask, &r->status2, &r->bounds_dev, &r->fence[0], &r->fence[1], &r->bfs_a, &r->bfs_b, &r->pr_a, &r->pr_b, &r->ctr,
                    &r->xrec, &r->xins, &r->xwts, &r->xdel, &r->xcnt, &r->xoff, &r->live[0], &r->live[1], &r->casc_status};
     for (Buf* b : bufs) if (b->p) r->dfree(b->p);
     cudaStreamSynchronize(r->st);
@@ -947,6 +987,7 @@ void free_replica(h2tap_replica* r) {
     if (r->evA) cudaEventDestroy(r->evA);
     if (r->evB) cudaEventDestroy(r->evB);
     if (r->evC) cudaEventDestroy(r->evC);
+    if (r->evD) cudaEventDestroy(r->evD);
     if (r->st2) { cudaStreamSynchronize(r->st2); cudaStreamDestroy(r->st2); }
     if (r->st_copy) { cudaStreamSynchronize(r->st_copy); cudaStreamDestroy(r->st_copy); }
     for (auto& g : r->stg) {

@@ -856,6 +856,9 @@ struct ClassArgs {
     uint64_t* status3;
     uint64_t n_tiles;
     Counters* c;
+    uint8_t* kcat;    // split mode: per sorted item, 0 none / 1 insert / 2 delete / 3 weight update
+    uint64_t* kpos;   //             its old position (lower bound of the key in its old row)
+    float* kw;        //             its weight
 };
 
 #ifndef H2TAP_CITEMS
@@ -863,13 +866,18 @@ struct ClassArgs {
 #endif
 constexpr int kCItems = H2TAP_CITEMS;  // classify: items per thread (occupancy over ILP)
 constexpr int kCTile = kThreads * kCItems;
+// SPLIT = 1: the classification alone (no compaction, no look-back), one item per thread in
+// launch order: its outcome goes to kcat / kpos / kw and k_classify_compact builds the three
+// lists.  The fused form (SPLIT = 0) compacts in the same kernel; there a tile holding a slow
+// dependent chain (gather -> row bounds -> probes) delays every later tile's look-back.
+template <int SPLIT>
 __global__ void __launch_bounds__(kThreads) k_reduce_classify(ClassArgs a) {
     __shared__ uint32_t s_tile;
     __shared__ uint32_t s_cmp[3][kCItems * kThreads / 32 + 1];
     __shared__ uint64_t s_base[3];
-    if (threadIdx.x == 0) s_tile = atomicAdd(&a.c->tiles[4], 1u);
-    __syncthreads();
-    const uint32_t tile = s_tile;
+    if (!SPLIT && threadIdx.x == 0) s_tile = atomicAdd(&a.c->tiles[4], 1u);
+    if (!SPLIT) __syncthreads();
+    const uint32_t tile = SPLIT ? blockIdx.x : s_tile;
     const uint64_t n = min(a.n, (uint64_t)a.c->n_valid);  // a.n: the grid's upper bound
     const uint64_t n_tiles = (n + kCTile - 1) / kCTile;
     if (tile >= n_tiles) return;
@@ -995,6 +1003,18 @@ __global__ void __launch_bounds__(kThreads) k_reduce_classify(ClassArgs a) {
         cat[j] = ct;
         f0[j] = ct == 1; f1[j] = ct == 2; f2[j] = ct == 3;
     }
+    if (SPLIT) {
+#pragma unroll
+        for (int j = 0; j < kCItems; ++j) {
+            const uint64_t i = i0 + (uint64_t)j * kThreads;
+            if (i < n) {
+                a.kcat[i] = cat[j];
+                a.kpos[i] = lo[j];
+                a.kw[i] = wv[j];
+            }
+        }
+        return;
+    }
     uint32_t rk0[kCItems], rk1[kCItems], rk2[kCItems];
     const uint32_t t0 = striped_compact<kThreads, kCItems>(f0, rk0, s_cmp[0]);
     const uint32_t t1 = striped_compact<kThreads, kCItems>(f1, rk1, s_cmp[1]);
@@ -1029,6 +1049,69 @@ __global__ void __launch_bounds__(kThreads) k_reduce_classify(ClassArgs a) {
             const uint64_t ou = s_base[2] + rk2[j];
             a.upd_pos[ou] = lo[j];
             a.upd_w[ou] = wv[j];
+        }
+    }
+}
+
+// the three outcome lists from the split classification: stable 3-way compaction of the
+// classified items (key order), decoupled look-back; the item fields are read only for
+// items that go to a list
+__global__ void __launch_bounds__(kThreads) k_classify_compact(ClassArgs a) {
+    __shared__ uint32_t s_tile;
+    __shared__ uint32_t s_cmp[3][kItems * kThreads / 32 + 1];
+    __shared__ uint64_t s_base[3];
+    if (threadIdx.x == 0) s_tile = atomicAdd(&a.c->tiles[4], 1u);
+    __syncthreads();
+    const uint32_t tile = s_tile;
+    const uint64_t n = min(a.n, (uint64_t)a.c->n_valid);
+    const uint64_t n_tiles = (n + kTile - 1) / kTile;
+    if (tile >= n_tiles) return;
+    const uint64_t i0 = (uint64_t)tile * kTile + threadIdx.x;
+    uint8_t cat[kItems];
+    bool f0[kItems], f1[kItems], f2[kItems];
+#pragma unroll
+    for (int j = 0; j < kItems; ++j) {
+        const uint64_t i = i0 + (uint64_t)j * kThreads;
+        cat[j] = i < n ? a.kcat[i] : 0;
+        f0[j] = cat[j] == 1; f1[j] = cat[j] == 2; f2[j] = cat[j] == 3;
+    }
+    uint32_t rk0[kItems], rk1[kItems], rk2[kItems];
+    const uint32_t t0 = striped_compact<kThreads, kItems>(f0, rk0, s_cmp[0]);
+    const uint32_t t1 = striped_compact<kThreads, kItems>(f1, rk1, s_cmp[1]);
+    const uint32_t t2 = striped_compact<kThreads, kItems>(f2, rk2, s_cmp[2]);
+    const int wid = threadIdx.x >> 5;
+    if (wid < 3) {
+        const uint32_t tw = wid == 0 ? t0 : (wid == 1 ? t1 : t2);
+        uint64_t b = lookback_warp(a.status3 + (uint64_t)wid * a.n_tiles, tile, tw);
+        if (lane_id() == 0) {
+            s_base[wid] = b;
+            if (tile == n_tiles - 1) {
+                unsigned long long* d = wid == 0 ? &a.c->n_ins : (wid == 1 ? &a.c->n_del : &a.c->n_upd);
+                *d = b + tw;
+            }
+        }
+    }
+    __syncthreads();
+    const uint64_t mask = (1ull << a.bits) - 1;
+#pragma unroll
+    for (int j = 0; j < kItems; ++j) {
+        if (!cat[j]) continue;
+        const uint64_t i = i0 + (uint64_t)j * kThreads;
+        const uint64_t key = a.keys[i], pos = a.kpos[i];
+        if (cat[j] == 1) {
+            const uint64_t oi = s_base[0] + rk0[j];
+            a.ins_pos[oi] = pos;
+            a.ins_row[oi] = (uint32_t)(key >> a.bits);
+            a.ins_col[oi] = (uint32_t)(key & mask);
+            a.ins_w[oi] = a.kw[i];
+        } else if (cat[j] == 2) {
+            const uint64_t od = s_base[1] + rk1[j];
+            a.del_pos[od] = pos;
+            a.del_row[od] = (uint32_t)(key >> a.bits);
+        } else {
+            const uint64_t ou = s_base[2] + rk2[j];
+            a.upd_pos[ou] = pos;
+            a.upd_w[ou] = a.kw[i];
         }
     }
 }

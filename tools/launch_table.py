@@ -7,7 +7,7 @@ rows = [r for r in csv.reader(open(sys.argv[1])) if len(r) > 10]
 h = rows[0]
 ki, mi, vi, ui, ii = (h.index("Kernel Name"), h.index("Metric Name"), h.index("Metric Value"),
                       h.index("Metric Unit"), h.index("ID"))
-sc = {"nsecond": 1e-3, "usecond": 1.0, "msecond": 1e3, "second": 1e6, "byte": 1, "Kbyte": 1e3, "Mbyte": 1e6,
+sc = {"ns": 1e-3, "us": 1.0, "ms": 1e3, "nsecond": 1e-3, "usecond": 1.0, "msecond": 1e3, "second": 1e6, "byte": 1, "Kbyte": 1e3, "Mbyte": 1e6,
       "Gbyte": 1e9}
 k = {}
 order = []

@@ -350,19 +350,35 @@ def run_gpu(args):
             return synth.RecordBatch(*(tens(a).cuda() for a in (rb.records, rb.inserts, rb.weights, rb.deletes)))
         return synth.Batch(*(tens(a).cuda() for a in (b.kind, b.src, b.dst, b.w, b.ts)))
 
-    def apply(r, b, snap):
+    # single replica, flat ops: h2tap_delta_apply_async (cycles enqueued back to back; the stats of
+    # cycle k come back from call k+1 or from the final sync, which is inside the timed region)
+    use_async = not sharded and not records and not args.sync_apply
+
+    def apply(r, b, snap, out=None):
         if records:
-            return r.apply_records(b, snap)
-        if not sharded:
-            return r.apply(b, snap)
-        l0 = eng.launches
-        st = shr.apply(b, snap)
-        st["n_launches"] += eng.launches - l0
+            st = r.apply_records(b, snap)
+        elif use_async:
+            st = r.apply_async(b, snap)
+        elif not sharded:
+            st = r.apply(b, snap)
+        else:
+            l0 = eng.launches
+            st = shr.apply(b, snap)
+            st["n_launches"] += eng.launches - l0
+        if st is not None and out is not None:
+            out.append(st)
         return st
+
+    def drain(r, out):
+        if use_async:
+            st = r.sync()
+            if st is not None:
+                out.append(st)
 
     dev = [to_dev(b) for b in host]
     for k in range(args.warmup):
         apply(rep, dev[k], snaps[k])
+    drain(rep, [])
     torch.cuda.synchronize()
     # the e2e leg replays the timed batches on the same graph state: keep the state the timed
     # region starts from (device copy of the CSR + ID map; single replica, compact IDs)
@@ -379,8 +395,10 @@ def run_gpu(args):
         torch.cuda.synchronize()
         evs[0].record(stream)
         for j, k in enumerate(range(args.warmup, n_total)):
-            stats.append(apply(rep, dev[k], snaps[k]))
+            apply(rep, dev[k], snaps[k], stats)
             evs[j + 1].record(stream)
+        drain(rep, stats)
+        evs[-1].record(stream)
         torch.cuda.synchronize()
     if world > 1:
         dist.barrier()
@@ -417,6 +435,7 @@ def run_gpu(args):
         rc, _ = rep.prepare(dev[args.warmup], snaps[args.warmup])
         assert rc == 0
         rep.abort()
+        rep.sync()
         e_host, e_snaps, e_glob_n = host[args.warmup:], snaps[args.warmup:], glob_n[args.warmup:]
         e_how_state = "same graph state and batches as the device-resident leg (replica restored from a device copy)"
     else:
@@ -437,6 +456,7 @@ def run_gpu(args):
     if pipelined:   # allocate and warm both staging slots (nothing is applied)
         rep.stage(e_pin[0])
         rep.stage(e_pin[min(1, len(e_pin) - 1)])
+    drain(rep, [])
     torch.cuda.synchronize()
     if world > 1:
         dist.barrier()
@@ -450,11 +470,12 @@ def run_gpu(args):
         staged = rep.stage(e_pin[0])
         for k in range(args.steps):
             nxt = rep.stage(e_pin[k + 1]) if k + 1 < args.steps else None
-            e_stats.append(apply(rep, staged, e_snaps[k]))
+            apply(rep, staged, e_snaps[k], e_stats)
             staged = nxt
     else:
         for k in range(args.steps):
-            e_stats.append(apply(rep, e_pin[k], e_snaps[k]))
+            apply(rep, e_pin[k], e_snaps[k], e_stats)
+    drain(rep, e_stats)
     ev1.record(stream)
     torch.cuda.synchronize()
     e_ms = ev0.elapsed_time(ev1)
@@ -689,6 +710,9 @@ def main():
     ap.add_argument("--exchange", default="alltoall", choices=["alltoall", "p2p"],
                     help="sharded exchange: pack + all-to-all (NCCL), or the fused pack-and-store kernel "
                          "into peers' CUDA-IPC windows (h2tap_route_pack_p2p)")
+    ap.add_argument("--sync-apply", action="store_true",
+                    help="time h2tap_delta_apply (each call returns after its cycle) instead of "
+                         "h2tap_delta_apply_async (cycles enqueued back to back)")
     ap.add_argument("--tombstone", action="store_true",
                     help="tombstone-row replica (deleted nodes keep an empty row; reading A23)")
     ap.add_argument("--checks", action="store_true",

@@ -312,6 +312,21 @@ h2tap_status h2tap_delta_apply_routed_prepare(h2tap_replica* r, const h2tap_rout
 h2tap_status h2tap_delta_commit(h2tap_replica* r);  /* E_INVAL if nothing is prepared */
 h2tap_status h2tap_delta_abort(h2tap_replica* r);   /* no-op if nothing is prepared */
 
+/* Asynchronous apply (throughput mode): the whole cycle of h2tap_delta_apply is enqueued on
+ * the replica's stream and the call returns after the cycle's first read-back (a1), without
+ * waiting for the merge; the new snapshot is visible to every later call, which completes the
+ * cycle first (export / info / checks synchronise; the next apply reads the cycle's final sizes
+ * when its own first read-back has passed them, so consecutive cycles leave the GPU no idle gap).
+ * *has_completed = 1 and *completed = the stats of the cycle completed during this call (the
+ * previous one), else 0.  h2tap_replica_sync completes the last cycle and hands out its stats.
+ * Errors detected before the return are those of h2tap_delta_apply (strong guarantee); the
+ * asynchronous path is not taken for sharded replicas or two-phase cycles (they run
+ * synchronously). */
+h2tap_status h2tap_delta_apply_async(h2tap_replica* r, const h2tap_batch* batch, uint64_t snapshot_ts,
+        h2tap_apply_stats* completed /* nullable */, int* has_completed /* nullable */);
+h2tap_status h2tap_replica_sync(h2tap_replica* r, h2tap_apply_stats* completed /* nullable */,
+        int* has_completed /* nullable */);
+
 /* Sizes of the current replica (any pointer may be NULL). */
 h2tap_status h2tap_replica_info(const h2tap_replica* r, uint64_t* n_vertices, uint64_t* n_edges,
         uint64_t* snapshot_ts, uint64_t* n_pending, uint64_t* shard_vertex_base,

@@ -140,6 +140,9 @@ for _n, _a in (("h2tap_batch_stage", [_P, ctypes.POINTER(_Batch), ctypes.POINTER
                ("h2tap_delta_apply_prepare", [_P, ctypes.POINTER(_Batch), _u64, ctypes.POINTER(ApplyStats)]),
                ("h2tap_delta_apply_routed_prepare", [_P, _P, ctypes.c_size_t, _u64, ctypes.POINTER(ApplyStats)]),
                ("h2tap_delta_commit", [_P]),
+               ("h2tap_delta_apply_async", [_P, ctypes.POINTER(_Batch), _u64, ctypes.POINTER(ApplyStats),
+                                            ctypes.POINTER(ctypes.c_int)]),
+               ("h2tap_replica_sync", [_P, ctypes.POINTER(ApplyStats), ctypes.POINTER(ctypes.c_int)]),
                ("h2tap_ds_create", [ctypes.c_int, ctypes.c_size_t, ctypes.POINTER(_P)]),
                ("h2tap_ds_append", [_P, _u64, _u64, ctypes.c_int, ctypes.c_int, _P, _P, ctypes.c_uint32, _P,
                                     ctypes.c_uint32]),
@@ -432,6 +435,24 @@ class Replica:
             _check(rc, "h2tap_delta_apply")
             return st.as_dict()
         return rc, st.as_dict()
+
+    def apply_async(self, batch, snapshot_ts: int):
+        """h2tap_delta_apply_async: enqueue the cycle and return; returns the stats dict of the
+        cycle completed during this call (the previous one) or None."""
+        if isinstance(batch, StagedBatch):
+            b, keep = batch.b, batch.keep
+        else:
+            b, keep = self._batch(batch)
+        st, has = ApplyStats(), ctypes.c_int(0)
+        _check(_lib.h2tap_delta_apply_async(self._h, ctypes.byref(b), int(snapshot_ts), ctypes.byref(st),
+                                            ctypes.byref(has)), "h2tap_delta_apply_async")
+        return st.as_dict() if has.value else None
+
+    def sync(self):
+        """h2tap_replica_sync: complete the last asynchronous cycle; its stats dict or None."""
+        st, has = ApplyStats(), ctypes.c_int(0)
+        _check(_lib.h2tap_replica_sync(self._h, ctypes.byref(st), ctypes.byref(has)), "h2tap_replica_sync")
+        return st.as_dict() if has.value else None
 
     def apply_records(self, rb, snapshot_ts: int, raise_on_error: bool = True):
         """h2tap_delta_apply_records; rb has .records (48-byte records: a numpy structured

@@ -115,7 +115,8 @@ struct h2tap_replica {
     cudaStream_t st_copy = nullptr;            // host->device staging of the next batch
     struct Stage {
         Buf k, s, d, w, t;
-        cudaEvent_t ev = nullptr;
+        cudaEvent_t ev = nullptr;    // its H2D copy is complete
+        cudaEvent_t done = nullptr;  // the cycle that read it has finished (the slot may be refilled)
         uint64_t bytes = 0;  // staged H2D bytes not yet accounted to an apply
     } stg[2];
     int stg_next = 0;
@@ -149,6 +150,21 @@ struct h2tap_replica {
         uint64_t V = 0, E = 0, row_lo = 0, Vr = 0, n_pend = 0, n = 0, S = 0;
     } prep;
     bool defer_commit = false;  // apply_core leaves the result prepared instead of swapping
+    // asynchronous apply (h2tap_delta_apply_async): the cycle is enqueued and the call returns;
+    // the counters that size the next cycle (V, E, row range, identity) are read when the next
+    // cycle's first read-back has passed them (or at h2tap_replica_sync / any read call)
+    bool async_req = false;
+    struct Inflight {
+        bool on = false, node_mode = false, csr_changed = false;
+        cudaEvent_t ev[8];
+        uint64_t n = 0, n_node = 0, n_edge = 0, n_pend_new = 0, V = 0, Vr = 0, E = 0, row_lo = 0;
+        uint64_t launches = 0, h2d = 0, d2h = 0;
+    } infl;
+    bool fin_ready = false;       // stats of a finalised asynchronous cycle, not yet handed out
+    h2tap_apply_stats fin_stats{};
+    Counters* hcf = nullptr;      // mapped host slot of an asynchronous cycle's final counters
+    Counters* hcf_dev = nullptr;
+    cudaEvent_t evx[8]{};         // the other event set (alternates with ev across async cycles)
     void commit() {             // a7: the pointer flip
         cur = prep.nb;
         if (prep.node_mode) {
@@ -366,6 +382,56 @@ ExtIndex ext_index(h2tap_replica* r) {
 #endif
 constexpr int kCascCtasPerSm = H2TAP_CASC_CTAS;  // cascade pass beside the edge-op phase
 
+// An asynchronous cycle's end: the sizes of the new replica from its final counters (the
+// stream has passed their store), its stats kept for h2tap_delta_apply_async /
+// h2tap_replica_sync.  The counter-independent part of the swap happened at enqueue time.
+void finalize_inflight(h2tap_replica* r) {
+    h2tap_replica::Inflight& f = r->infl;
+    const Counters& fc = *r->hcf;
+    r->V = fc.Vn;
+    r->E = fc.En;
+    r->Vr = fc.Vr_new;
+    if (f.node_mode) r->identity = fc.new_identity == 1;
+    h2tap_apply_stats& st = r->fin_stats;
+    memset(&st, 0, sizeof st);
+    st.n_visible = f.n_node + f.n_edge;
+    st.n_deferred = f.n_pend_new;
+    st.n_gated = fc.n_gated;
+    st.n_new = fc.n_ins;
+    st.n_del = fc.n_del;
+    st.n_upd = fc.n_upd;
+    st.n_casc = fc.n_casc;
+    st.n_vertex_inserted = fc.n_inserted;
+    st.n_vertex_deleted = fc.n_killed;
+    st.ms_ingest = ev_ms(f.ev[0], f.ev[1]);
+    st.ms_nodeops = ev_ms(f.ev[1], f.ev[2]);
+    st.ms_sort_reduce = ev_ms(f.ev[2], f.ev[3]);
+    st.ms_merge = ev_ms(f.ev[6], f.ev[4]);
+    st.ms_degree_scan = ev_ms(f.ev[3], f.ev[6]) + ev_ms(f.ev[4], f.ev[5]);
+    st.ms_total = ev_ms(f.ev[0], f.ev[5]);
+    uint64_t b = 8 * (f.Vr + 1) + 8 * f.E + 8 * (fc.Vr_new + 1) + 8 * fc.En + 29 * f.n;
+    if (f.node_mode) b += 16 * f.V + 4 * f.E + 4 * f.V;
+    st.bytes_alg = b;
+    uint64_t bm = 0;
+    if (f.csr_changed && f.E + fc.n_ins) {
+        bm = 8 * f.E + 8 * fc.En + 20 * fc.n_ins + 8 * fc.n_del + 12 * fc.n_upd;
+        if (f.node_mode) bm += f.E / 8;
+    }
+    st.bytes_merge = bm;
+    st.n_launches = f.launches;
+    st.h2d_bytes = f.h2d;
+    st.d2h_bytes = f.d2h;
+    r->fin_ready = true;
+    f.on = false;
+}
+// every call that reads the replica's sizes or contents first completes an asynchronous cycle
+void ensure_final(const h2tap_replica* rc) {
+    h2tap_replica* r = const_cast<h2tap_replica*>(rc);
+    if (!r || !r->infl.on) return;
+    CK(cudaStreamSynchronize(r->st));
+    finalize_inflight(r);
+}
+
 // One propagation cycle.  Nothing visible changes until the final swap.
 h2tap_status apply_core(h2tap_replica* r, const BatchIn& in, uint64_t S, bool create, h2tap_apply_stats* stats) {
     cudaStream_t st = r->st;
@@ -376,8 +442,14 @@ h2tap_status apply_core(h2tap_replica* r, const BatchIn& in, uint64_t S, bool cr
     g_h2d = in.pre_h2d;
     g_d2h = in.pre_d2h;
     g_tr.init();
+    const bool async = r->async_req && !create && !r->sharded && !r->defer_commit && !g_tr.on;
     for (int i = 0; i < 8; ++i)
         if (!r->ev[i]) CK(cudaEventCreate(&r->ev[i]));
+    if (async || r->infl.on) {  // the in-flight cycle keeps its event set until it is finalised
+        for (int i = 0; i < 8; ++i)
+            if (!r->evx[i]) CK(cudaEventCreate(&r->evx[i]));
+        std::swap(r->ev, r->evx);
+    }
     CK(cudaStreamWaitEvent(st, r->evB, 0));  // a cascade pass of an earlier (failed) cycle is done
     CK(cudaStreamWaitEvent(st, r->evD, 0));  // and so is its merge partition (side stream)
     CK(cudaEventRecord(r->ev[0], st));
@@ -449,6 +521,7 @@ h2tap_status apply_core(h2tap_replica* r, const BatchIn& in, uint64_t S, bool cr
     TR("assemble+partition");
     r->read_counters();
     TR("sync1");
+    if (r->infl.on) finalize_inflight(r);  // the previous (asynchronous) cycle's counters precede this read-back
     Counters hc = *r->hc;
     if (hc.status & ST_BAD_KIND) { set_err("unknown op kind in batch"); return H2TAP_E_INVAL; }
     if (hc.status & ST_STALE) {
@@ -830,6 +903,26 @@ h2tap_status apply_core(h2tap_replica* r, const BatchIn& in, uint64_t S, bool cr
     CKL();
     CK(cudaEventRecord(r->ev[5], st));
     TR("offsets+pending");
+    if (async) {  // enqueue the final read-back and return; finalize_inflight completes the cycle
+        k_store_counters<<<1, 32, 0, st>>>(dc, r->hcf_dev);
+        CKL();
+        h2tap_replica::Inflight& f = r->infl;
+        f.on = true;
+        for (int i = 0; i < 8; ++i) f.ev[i] = r->ev[i];
+        f.node_mode = node_mode; f.csr_changed = csr_changed;
+        f.n = n; f.n_node = n_node; f.n_edge = n_edge; f.n_pend_new = n_pend_new;
+        f.V = V; f.Vr = Vr; f.E = E; f.row_lo = row_lo;
+        f.launches = g_launches; f.h2d = g_h2d; f.d2h = g_d2h + sizeof(Counters);
+        // the part of the swap that needs no counter (what the next cycle reads first)
+        r->cur = nb;
+        if (node_mode) r->ext_cur = ec ^ 1;
+        r->pcur = pc ^ 1;
+        r->n_pend = n_pend_new;
+        r->next_seq += n;
+        r->snap = S;
+        if (stats) memset(stats, 0, sizeof *stats);
+        return H2TAP_OK;
+    }
     r->read_counters();  // the one read-back of the cycle's device-side sizes
     TR("end");
     g_tr.dump();
@@ -958,7 +1051,10 @@ h2tap_replica* new_replica(const h2tap_config* cfg) {
         CK(cudaDeviceGetStreamPriorityRange(&lo, &hi));
         CK(cudaStreamCreateWithPriority(&r->st2, cudaStreamNonBlocking, lo));
         CK(cudaStreamCreateWithFlags(&r->st_copy, cudaStreamNonBlocking));
-        for (auto& g : r->stg) CK(cudaEventCreateWithFlags(&g.ev, cudaEventDisableTiming));
+        for (auto& g : r->stg) {
+            CK(cudaEventCreateWithFlags(&g.ev, cudaEventDisableTiming));
+            CK(cudaEventCreateWithFlags(&g.done, cudaEventDisableTiming));
+        }
     }
     CK(cudaEventCreateWithFlags(&r->evA, cudaEventDisableTiming));
     CK(cudaEventCreateWithFlags(&r->evB, cudaEventDisableTiming));
@@ -966,6 +1062,8 @@ h2tap_replica* new_replica(const h2tap_config* cfg) {
     CK(cudaEventCreateWithFlags(&r->evD, cudaEventDisableTiming));
     CK(cudaHostAlloc(reinterpret_cast<void**>(&r->hc), sizeof(Counters), cudaHostAllocMapped));
     CK(cudaHostGetDevicePointer(reinterpret_cast<void**>(&r->hc_dev), r->hc, 0));
+    CK(cudaHostAlloc(reinterpret_cast<void**>(&r->hcf), sizeof(Counters), cudaHostAllocMapped));
+    CK(cudaHostGetDevicePointer(reinterpret_cast<void**>(&r->hcf_dev), r->hcf, 0));
     r->get<Counters>(r->ctr, 1);
     return r;
 }
@@ -993,8 +1091,11 @@ void free_replica(h2tap_replica* r) {
     for (auto& g : r->stg) {
         for (Buf* b : {&g.k, &g.s, &g.d, &g.w, &g.t}) if (b->p) r->dfree(b->p);
         if (g.ev) cudaEventDestroy(g.ev);
+        if (g.done) cudaEventDestroy(g.done);
     }
     if (r->hc) cudaFreeHost(r->hc);
+    if (r->hcf) cudaFreeHost(r->hcf);
+    for (auto& e : r->evx) if (e) cudaEventDestroy(e);
     delete r;
 }
 
@@ -1164,13 +1265,17 @@ h2tap_status h2tap_delta_apply(h2tap_replica* r, const h2tap_batch* b, uint64_t 
         }
         CK(cudaSetDevice(r->cfg.device));
         BatchIn in{b->n, b->on_device, b->seq, b->kind, b->src, b->dst, b->weight, b->ts, 0};
+        h2tap_replica::Stage* used = nullptr;
         for (auto& g : r->stg)  // a batch staged by h2tap_batch_stage: its copy is ordered first
             if (b->n && b->on_device && b->kind == g.k.p) {
                 CK(cudaStreamWaitEvent(r->st, g.ev, 0));
                 in.pre_h2d = g.bytes;
                 g.bytes = 0;
+                used = &g;
             }
-        return apply_core(r, in, snapshot_ts, false, stats);
+        const h2tap_status s = apply_core(r, in, snapshot_ts, false, stats);
+        if (used) CK(cudaEventRecord(used->done, r->st));  // after every kernel that reads the slot
+        return s;
     });
 }
 
@@ -1350,13 +1455,16 @@ h2tap_status h2tap_batch_stage(h2tap_replica* r, const h2tap_batch* host, h2tap_
         // the slot's previous copy (a staged batch that was never applied) may still be
         // running: wait for it before get() can free and re-allocate the slot's buffers
         CK(cudaEventSynchronize(g.ev));
+        const size_t caps = g.k.cap + g.s.cap + g.d.cap + g.w.cap + g.t.cap;
         uint8_t* k = r->get<uint8_t>(g.k, n);
         uint64_t* s = r->get<uint64_t>(g.s, n);
         uint64_t* d = r->get<uint64_t>(g.d, n);
         float* w = r->get<float>(g.w, n);
         uint64_t* t = r->get<uint64_t>(g.t, n);
-        CK(cudaStreamSynchronize(r->st));  // buffers (re)allocated on the replica stream are ready
+        if (caps != g.k.cap + g.s.cap + g.d.cap + g.w.cap + g.t.cap)
+            CK(cudaStreamSynchronize(r->st));  // buffers (re)allocated on the replica stream are ready
         cudaStream_t cs = r->st_copy;
+        CK(cudaStreamWaitEvent(cs, g.done, 0));  // the cycle that read this slot (asynchronous apply) is done
         uint64_t bytes = 0;
         auto cp = [&](void* dst, const void* src, uint64_t nb) {
             if (!nb) return;
@@ -1490,6 +1598,29 @@ h2tap_status h2tap_delta_apply_routed(h2tap_replica* r, const h2tap_route_rec* r
     });
 }
 
+h2tap_status h2tap_delta_apply_async(h2tap_replica* r, const h2tap_batch* b, uint64_t snapshot_ts,
+                                     h2tap_apply_stats* completed, int* has_completed) {
+    if (!r) { set_err("null replica"); return H2TAP_E_INVAL; }
+    r->async_req = true;
+    const h2tap_status s = h2tap_delta_apply(r, b, snapshot_ts, nullptr);
+    r->async_req = false;
+    if (has_completed) *has_completed = r->fin_ready ? 1 : 0;
+    if (r->fin_ready && completed) *completed = r->fin_stats;
+    r->fin_ready = false;
+    return s;
+}
+
+h2tap_status h2tap_replica_sync(h2tap_replica* r, h2tap_apply_stats* completed, int* has_completed) {
+    if (!r) { set_err("null replica"); return H2TAP_E_INVAL; }
+    return run_guarded(r, [&]() -> h2tap_status {
+        ensure_final(r);
+        if (has_completed) *has_completed = r->fin_ready ? 1 : 0;
+        if (r->fin_ready && completed) *completed = r->fin_stats;
+        r->fin_ready = false;
+        return H2TAP_OK;
+    });
+}
+
 h2tap_status h2tap_delta_apply_prepare(h2tap_replica* r, const h2tap_batch* b, uint64_t snapshot_ts,
                                        h2tap_apply_stats* stats) {
     if (!r) { set_err("null replica"); return H2TAP_E_INVAL; }
@@ -1525,6 +1656,13 @@ h2tap_status h2tap_delta_abort(h2tap_replica* r) {
 h2tap_status h2tap_replica_info(const h2tap_replica* r, uint64_t* nv, uint64_t* ne, uint64_t* snap, uint64_t* npend,
                                 uint64_t* vbase, uint64_t* ebase) {
     if (!r) { set_err("null replica"); return H2TAP_E_INVAL; }
+    if (r->infl.on) {
+        const h2tap_status st = run_guarded(const_cast<h2tap_replica*>(r), [&]() -> h2tap_status {
+            ensure_final(r);
+            return H2TAP_OK;
+        });
+        if (st != H2TAP_OK) return st;
+    }
     if (nv) *nv = r->Vr;  // rows of this shard (= all vertices when not sharded)
     if (ne) *ne = r->E;
     if (snap) *snap = r->snap;
@@ -1539,6 +1677,7 @@ h2tap_status h2tap_replica_export(const h2tap_replica* rc, int64_t* offsets, uin
     h2tap_replica* r = const_cast<h2tap_replica*>(rc);
     if (!r) { set_err("null replica"); return H2TAP_E_INVAL; }
     return run_guarded(r, [&]() -> h2tap_status {
+        ensure_final(r);
         CK(cudaSetDevice(r->cfg.device));
         cudaMemcpyKind k = on_device ? cudaMemcpyDeviceToDevice : cudaMemcpyDeviceToHost;
         const int c = r->cur;
@@ -1592,6 +1731,7 @@ h2tap_status h2tap_bfs(const h2tap_replica* rc, uint64_t source_ext, int32_t* le
     if (!r || !level_out) { set_err("null argument"); return H2TAP_E_INVAL; }
     if (r->sharded) { set_err("h2tap_bfs: not available on a sharded replica in this build"); return H2TAP_E_INVAL; }
     return run_guarded(r, [&]() -> h2tap_status {
+        ensure_final(r);
         CK(cudaSetDevice(r->cfg.device));
         const uint64_t V = r->V;
         const uint64_t src = dense_of(r, source_ext);
@@ -1631,6 +1771,7 @@ h2tap_status h2tap_sssp(const h2tap_replica* rc, uint64_t source_ext, double* di
     if (!r || !dist_out) { set_err("null argument"); return H2TAP_E_INVAL; }
     if (r->sharded) { set_err("h2tap_sssp: not available on a sharded replica in this build"); return H2TAP_E_INVAL; }
     return run_guarded(r, [&]() -> h2tap_status {
+        ensure_final(r);
         CK(cudaSetDevice(r->cfg.device));
         const uint64_t V = r->V, E = r->E;
         const uint64_t src = dense_of(r, source_ext);
@@ -1700,6 +1841,7 @@ h2tap_status h2tap_replica_lookup(const h2tap_replica* rc, uint64_t ext_id, uint
     h2tap_replica* r = const_cast<h2tap_replica*>(rc);
     if (!r || !dense_out) { set_err("null argument"); return H2TAP_E_INVAL; }
     return run_guarded(r, [&]() -> h2tap_status {
+        ensure_final(r);
         CK(cudaSetDevice(r->cfg.device));
         const uint64_t k = dense_of(r, ext_id);
         if (k >= r->V) { set_err("%llu is not a live vertex", (unsigned long long)ext_id); return H2TAP_E_INVAL; }
@@ -1819,6 +1961,7 @@ h2tap_status h2tap_replica_liveness(const h2tap_replica* rc, uint8_t* live_out, 
     h2tap_replica* r = const_cast<h2tap_replica*>(rc);
     if (!r || !live_out) { set_err("null argument"); return H2TAP_E_INVAL; }
     return run_guarded(r, [&]() -> h2tap_status {
+        ensure_final(r);
         CK(cudaSetDevice(r->cfg.device));
         const uint64_t V = r->V;
         if (!r->tomb) {  // compacting replica: every vertex in the ID map is live
@@ -1840,6 +1983,7 @@ h2tap_status h2tap_pagerank(const h2tap_replica* rc, double damping, int iterati
     if (!r || !rank_out || iterations < 0) { set_err("bad argument"); return H2TAP_E_INVAL; }
     if (r->sharded) { set_err("h2tap_pagerank: not available on a sharded replica in this build"); return H2TAP_E_INVAL; }
     return run_guarded(r, [&]() -> h2tap_status {
+        ensure_final(r);
         CK(cudaSetDevice(r->cfg.device));
         const uint64_t V = r->V;
         if (V == 0) return H2TAP_OK;

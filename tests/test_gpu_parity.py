@@ -356,3 +356,42 @@ def test_two_phase_prepare_commit_abort(h2):
         g.commit()                                     # nothing prepared
     b2 = synth.ldbc_batch(shape, seed, 1, 3000, ts_base=snap)
     step(g, o, b2, int(b2.ts.max()), "after two-phase")
+
+
+def test_async_apply_stream(h2):
+    """h2tap_delta_apply_async: cycles enqueued back to back (the next one reads the previous
+    cycle's sizes at its first read-back) give the same replica as the synchronous path, with
+    node ops, deferral and sparse ids; stats come out one call late and at h2tap_replica_sync;
+    a read call (export) completes the in-flight cycle; a refused batch leaves the committed
+    cycles in place."""
+    shape = synth.LdbcShape(n_person=256, n_msg=6000, e_person=9000)
+    seed = synth.seed_of("c2")
+    ids = synth.ldbc_vertices(shape)
+    src, dst, w = synth.ldbc_edges(shape, seed)
+    g, o = pair_from_edges(h2, len(ids), ids, src, dst, w)
+    ts, seen = 1, []
+    for k in range(6):
+        b = synth.ldbc_batch(shape, seed, k, 2500, ts_base=ts)
+        snap = int(np.quantile(b.ts, 0.9)) if k % 2 else int(b.ts.max())   # some ops deferred
+        st = g.apply_async(b, snap)
+        if st is not None:
+            seen.append(st)
+        rc, _ = o.apply(b, snap)
+        assert rc == 0
+        ts = int(b.ts.max()) + 1
+        if k == 2:                                       # a read completes the in-flight cycle
+            assert_same(g.export(), o.export(), "async, read in the middle")
+    last = g.sync()
+    assert last is not None and g.sync() is None
+    seen.append(last)
+    assert len(seen) == 6
+    assert_same(g.export(), o.export(), "async stream")
+    assert g.info()["n_pending"] == o.info()["n_pending"]
+    # a stale op refused by an asynchronous call: the earlier cycles stay committed
+    before = g.export(checksums=True)
+    with pytest.raises(h2.H2tapError):
+        g.apply_async(Batch.of([(EDGE_INSERT, int(ids[0]), int(ids[1]), 1.0, 1)]), ts + 5)
+    assert g.export(checksums=True)[4] == before[4]
+    g.apply(Batch.empty(0), ts + 100)
+    o.apply(Batch.empty(0), ts + 100)
+    assert_same(g.export(), o.export(), "sync after async")

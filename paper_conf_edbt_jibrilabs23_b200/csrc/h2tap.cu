@@ -154,6 +154,7 @@ struct h2tap_replica {
     // the counters that size the next cycle (V, E, row range, identity) are read when the next
     // cycle's first read-back has passed them (or at h2tap_replica_sync / any read call)
     bool async_req = false;
+    bool last_node_mode = false;  // the previous cycle had node ops (speculation predictor)
     struct Inflight {
         bool on = false, node_mode = false, csr_changed = false;
         cudaEvent_t ev[8];
@@ -518,6 +519,45 @@ h2tap_status apply_core(h2tap_replica* r, const BatchIn& in, uint64_t S, bool cr
                                                        stt, nt, dc);
         CKL();
     }
+    // Speculation: when this replica's last cycles had no node ops (and the ID map is the
+    // identity), the edge-op keys and their sort do not depend on anything the read-back below
+    // returns - they are launched now, sized by upper bounds with the counts read on the device,
+    // so the GPU keeps working while the host waits; a batch that does carry node ops discards
+    // them and redoes both in node mode.
+#ifndef H2TAP_SPECULATE
+#define H2TAP_SPECULATE 1
+#endif
+    const bool spec = H2TAP_SPECULATE && m && !create && !r->sharded && r->identity && !r->last_node_mode &&
+                      !(r->infl.on && r->infl.node_mode);
+    uint64_t *sk = nullptr, *sk2 = nullptr;
+    uint32_t *sv = nullptr, *sv2 = nullptr;
+    if (spec) {
+        sk = r->get<uint64_t>(r->keyA, m);
+        sk2 = r->get<uint64_t>(r->keyB, m);
+        sv = r->get<uint32_t>(r->valA, m);
+        sv2 = r->get<uint32_t>(r->valB, m);
+        const uint64_t Vs = r->V;  // no node ops in flight: the vertex count is final
+        const int sbits = std::max(1, bits_for(Vs > 1 ? Vs - 1 : 1));
+        PrepArgs pa{};
+        pa.ops = ops;
+        pa.edge_idx = idx_e;
+        pa.n_edge = m;
+        pa.count_dev = 1;
+        pa.X = ext_index(r);
+        pa.bits = sbits;
+        pa.own = r->own;
+        pa.keys = sk;
+        pa.vals = sv;
+        pa.recs = r->get<EdgeRec>(r->op_flags, m);
+        const uint64_t nts = cdiv(m, (uint64_t)kThreads * 4);
+        pa.status = r->get<uint64_t>(r->status2, nts);
+        CK(cudaMemsetAsync(pa.status, 0, nts * 8, st));
+        pa.n_tiles = nts;
+        pa.c = dc;
+        k_edge_prep<4><<<(unsigned)nts, kThreads, 0, st>>>(pa);
+        CKL();
+        radix_sort(r, sk, sv, sk2, sv2, m, 2 * sbits, &dc->n_valid);
+    }
     TR("assemble+partition");
     r->read_counters();
     TR("sync1");
@@ -682,6 +722,7 @@ h2tap_status apply_core(h2tap_replica* r, const BatchIn& in, uint64_t S, bool cr
         uint64_t* kB = r->get<uint64_t>(r->keyB, n_edge);
         uint32_t* vA = r->get<uint32_t>(r->valA, n_edge);
         uint32_t* vB = r->get<uint32_t>(r->valB, n_edge);
+        const bool spec_ok = spec && !node_mode;  // the speculative keys are this cycle's keys
         PrepArgs pa{};
         pa.ops = ops;
         pa.edge_idx = idx_e;
@@ -707,11 +748,20 @@ h2tap_status apply_core(h2tap_replica* r, const BatchIn& in, uint64_t S, bool cr
         CK(cudaMemsetAsync(pa.status, 0, nt * 8, st));
         pa.n_tiles = nt;
         pa.c = dc;
-        if (lookups_direct) k_edge_prep<H2TAP_EI_DIRECT><<<(unsigned)nt, kThreads, 0, st>>>(pa);
-        else k_edge_prep<1><<<(unsigned)nt, kThreads, 0, st>>>(pa);
-        CKL();
-        TR("edge_prep");
-        radix_sort(r, kA, vA, kB, vB, n_edge, 2 * bits, &dc->n_valid);
+        if (spec_ok) {
+            kA = sk; vA = sv;
+        } else {
+            if (spec) {  // discard the speculative keys: counters and the tile ticket start over
+                CK(cudaMemsetAsync(&dc->n_valid, 0, 8, st));
+                CK(cudaMemsetAsync(&dc->n_gated, 0, 8, st));
+                CK(cudaMemsetAsync(&dc->tiles[3], 0, 4, st));
+            }
+            if (lookups_direct) k_edge_prep<H2TAP_EI_DIRECT><<<(unsigned)nt, kThreads, 0, st>>>(pa);
+            else k_edge_prep<1><<<(unsigned)nt, kThreads, 0, st>>>(pa);
+            CKL();
+            TR("edge_prep");
+            radix_sort(r, kA, vA, kB, vB, n_edge, 2 * bits, &dc->n_valid);
+        }
         TR("edge_sort");
         ClassArgs ca{};
         ca.ops = ops;
@@ -920,6 +970,7 @@ h2tap_status apply_core(h2tap_replica* r, const BatchIn& in, uint64_t S, bool cr
         r->n_pend = n_pend_new;
         r->next_seq += n;
         r->snap = S;
+        r->last_node_mode = node_mode;
         if (stats) memset(stats, 0, sizeof *stats);
         return H2TAP_OK;
     }
@@ -947,6 +998,7 @@ h2tap_status apply_core(h2tap_replica* r, const BatchIn& in, uint64_t S, bool cr
     pr.V = Vn; pr.E = En; pr.row_lo = row_lo_new; pr.Vr = Vr_new; pr.n_pend = n_pend_new; pr.n = n; pr.S = S;
     pr.on = true;
     if (!r->defer_commit) r->commit();
+    r->last_node_mode = node_mode;
     if (stats) {
         memset(stats, 0, sizeof *stats);
         stats->n_visible = n_node + n_edge;

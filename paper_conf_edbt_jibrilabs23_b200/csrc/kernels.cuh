@@ -684,6 +684,7 @@ struct PrepArgs {
     uint64_t* status;
     uint64_t n_tiles;
     Counters* c;
+    int count_dev;                // 1: n_edge is an upper bound, the count is c->n_edge (speculative launch)
 };
 
 __device__ __forceinline__ Lookup do_lookup(const PrepArgs& a, uint64_t U, uint64_t x) {
@@ -743,6 +744,11 @@ __global__ void __launch_bounds__(kThreads) k_edge_prep(PrepArgs a) {
     if (threadIdx.x == 0) s_tile = atomicAdd(&a.c->tiles[3], 1u);
     __syncthreads();
     const uint32_t tile = s_tile;
+    if (a.count_dev) {   // launched before the host knew the count: the partition wrote it
+        a.n_edge = min(a.n_edge, (uint64_t)a.c->n_edge);
+        a.n_tiles = (a.n_edge + kETile - 1) / kETile;
+        if (tile >= a.n_tiles) return;   // beyond the last tile: no later tile depends on it
+    }
     const uint64_t i0 = (uint64_t)tile * kETile + threadIdx.x;
     const uint64_t U = a.nv ? a.c->n_unique : 0;
     uint64_t key[kEItems];

@@ -120,7 +120,7 @@ struct h2tap_replica {
         uint64_t bytes = 0;  // staged H2D bytes not yet accounted to an apply
     } stg[2];
     int stg_next = 0;
-    cudaEvent_t evA = nullptr, evB = nullptr, evC = nullptr, evD = nullptr;
+    cudaEvent_t evA = nullptr, evB = nullptr, evC = nullptr, evD = nullptr, evS = nullptr;
     uint64_t V = 0, E = 0, snap = 0, next_seq = 0, n_pend = 0;
     // sharding: V = global live vertices (the replicated ID map), the CSR holds the Vr rows
     // of the owned external-ID range starting at global dense id row_lo
@@ -531,6 +531,13 @@ h2tap_status apply_core(h2tap_replica* r, const BatchIn& in, uint64_t S, bool cr
                       !(r->infl.on && r->infl.node_mode);
     uint64_t *sk = nullptr, *sk2 = nullptr;
     uint32_t *sv = nullptr, *sv2 = nullptr;
+    // the first read-back: its store is enqueued before the speculative kernels and the host
+    // waits for an event behind the store only, not for the stream
+    g_d2h += sizeof(Counters);
+    k_store_counters<<<1, 32, 0, st>>>(dc, r->hc_dev);
+    CKL();
+    if (!r->evS) CK(cudaEventCreateWithFlags(&r->evS, cudaEventDisableTiming));
+    CK(cudaEventRecord(r->evS, st));
     if (spec) {
         sk = r->get<uint64_t>(r->keyA, m);
         sk2 = r->get<uint64_t>(r->keyB, m);
@@ -559,7 +566,7 @@ h2tap_status apply_core(h2tap_replica* r, const BatchIn& in, uint64_t S, bool cr
         radix_sort(r, sk, sv, sk2, sv2, m, 2 * sbits, &dc->n_valid);
     }
     TR("assemble+partition");
-    r->read_counters();
+    CK(cudaEventSynchronize(r->evS));
     TR("sync1");
     if (r->infl.on) finalize_inflight(r);  // the previous (asynchronous) cycle's counters precede this read-back
     Counters hc = *r->hc;
@@ -1138,6 +1145,7 @@ void free_replica(h2tap_replica* r) {
     if (r->evB) cudaEventDestroy(r->evB);
     if (r->evC) cudaEventDestroy(r->evC);
     if (r->evD) cudaEventDestroy(r->evD);
+    if (r->evS) cudaEventDestroy(r->evS);
     if (r->st2) { cudaStreamSynchronize(r->st2); cudaStreamDestroy(r->st2); }
     if (r->st_copy) { cudaStreamSynchronize(r->st_copy); cudaStreamDestroy(r->st_copy); }
     for (auto& g : r->stg) {

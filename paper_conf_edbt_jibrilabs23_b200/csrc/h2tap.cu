@@ -111,8 +111,7 @@ inline int bits_for(uint64_t range) { return range == 0 ? 0 : 64 - __builtin_clz
 
 struct h2tap_replica {
     h2tap_config cfg{};
-    cudaStream_t st = nullptr, st2 = nullptr;  // st2: side stream (cascade pass, merge partition)
-    cudaStream_t st3 = nullptr;                // third stream (ID map of a node-op cycle)
+    cudaStream_t st = nullptr, st2 = nullptr;  // st2: side stream (cascade pass)
     cudaStream_t st_copy = nullptr;            // host->device staging of the next batch
     struct Stage {
         Buf k, s, d, w, t;
@@ -121,7 +120,7 @@ struct h2tap_replica {
         uint64_t bytes = 0;  // staged H2D bytes not yet accounted to an apply
     } stg[2];
     int stg_next = 0;
-    cudaEvent_t evA = nullptr, evB = nullptr, evC = nullptr, evD = nullptr, evS = nullptr, evE = nullptr;
+    cudaEvent_t evA = nullptr, evB = nullptr, evC = nullptr, evD = nullptr, evS = nullptr;
     uint64_t V = 0, E = 0, snap = 0, next_seq = 0, n_pend = 0;
     // sharding: V = global live vertices (the replicated ID map), the CSR holds the Vr rows
     // of the owned external-ID range starting at global dense id row_lo
@@ -454,7 +453,6 @@ h2tap_status apply_core(h2tap_replica* r, const BatchIn& in, uint64_t S, bool cr
     }
     CK(cudaStreamWaitEvent(st, r->evB, 0));  // a cascade pass of an earlier (failed) cycle is done
     CK(cudaStreamWaitEvent(st, r->evD, 0));  // and so is its merge partition (side stream)
-    CK(cudaStreamWaitEvent(st, r->evE, 0));  // and its ID-map pass (third stream)
     CK(cudaEventRecord(r->ev[0], st));
     TR("start");
 
@@ -601,7 +599,6 @@ h2tap_status apply_core(h2tap_replica* r, const BatchIn& in, uint64_t S, bool cr
     uint64_t* new_ext = nullptr;
     uint32_t* casc_mask = nullptr;
     bool casc_pending = false;  // cascade pass in flight on the side stream
-    bool idmap_pending = false; // ID-map pass in flight on the third stream
     uint64_t *casc_cnt = nullptr, *casc_pre = nullptr;
     uint16_t* casc_wrel = nullptr;
     const int64_t* old_off_nc = static_cast<const int64_t*>(r->off[r->cur].p);
@@ -671,32 +668,6 @@ h2tap_status apply_core(h2tap_replica* r, const BatchIn& in, uint64_t S, bool cr
         if (r->sharded) {
             k_row_range_new<<<1, 1, 0, st>>>(dropped, ins_q, nv_ext, row_lo, row_lo + Vr, r->own, dc);
             CKL();
-        }
-        // the survivors' ID-map entries (+ liveness) and the new map's fences need nothing from
-        // the edge-op phase: a third stream builds them beside it, joined at the cycle's end
-        {
-            RowArgs ia{};
-            ia.V_old = V; ia.R = R; ia.c = dc;
-            ia.old_ext = old_ext; ia.new_ext = new_ext; ia.identity = r->identity ? 1 : 0;
-            if (r->tomb) {
-                ia.old_live = static_cast<const uint8_t*>(r->live[ec].p);
-                ia.new_live = r->get<uint8_t>(r->live[ec ^ 1], Vn_ub);
-            }
-            uint64_t* fnc = r->get<uint64_t>(r->fence[ec ^ 1], n_fence(Vn_ub));
-            CK(cudaEventRecord(r->evE, st));
-            CK(cudaStreamWaitEvent(r->st3, r->evE, 0));
-            if (V) {
-                k_rows_fused<1><<<(unsigned)cdiv(V, kRowTile), kThreads, 0, r->st3>>>(ia);
-                CKL();
-            }
-            if (ia.new_live) {  // node-op vertices' final liveness over the carried flags
-                k_nv_live<<<g1(n_node), 256, 0, r->st3>>>(nv, dc, R, ia.new_live);
-                CKL();
-            }
-            k_build_fence_dev<<<g1(n_fence(Vn_ub)), 256, 0, r->st3>>>(new_ext, dc, fnc);
-            CKL();
-            CK(cudaEventRecord(r->evE, r->st3));
-            idmap_pending = true;
         }
         // cascade pass (a4, reading A8): one bit per old element removed by a node delete
         hd_bits = r->get<uint32_t>(r->hd_bits, cdiv(V, 32));
@@ -887,6 +858,11 @@ h2tap_status apply_core(h2tap_replica* r, const BatchIn& in, uint64_t S, bool cr
         ra.new_off = new_off;
         ra.c = dc;
         ra.old_ext = old_ext; ra.new_ext = new_ext; ra.identity = r->identity ? 1 : 0;
+        uint8_t* new_live = nullptr;
+        if (r->tomb) {
+            ra.old_live = static_cast<const uint8_t*>(r->live[ec].p);
+            ra.new_live = new_live = r->get<uint8_t>(r->live[ec ^ 1], Vn_ub);
+        }
         const uint64_t ncta = cdiv(V, kRowTile);
         ra.part = r->get<uint64_t>(r->opart, 2 * (ncta + 1));
         if (V) {
@@ -899,10 +875,17 @@ h2tap_status apply_core(h2tap_replica* r, const BatchIn& in, uint64_t S, bool cr
             TR("casc_join");
         }
         if (V) {
-            k_rows_fused<2><<<(unsigned)ncta, kThreads, 0, st>>>(ra);  // survivors' row offsets
+            k_rows_fused<<<(unsigned)ncta, kThreads, 0, st>>>(ra);  // survivors: ID map + row offsets
             CKL();
         }
         k_offsets_inserted<<<g1(n_node), 256, 0, st>>>(nv, ins_q, ra);
+        CKL();
+        if (new_live) {  // node-op vertices' final liveness over the carried flags
+            k_nv_live<<<g1(n_node), 256, 0, st>>>(nv, dc, R, new_live);
+            CKL();
+        }
+        uint64_t* f = r->get<uint64_t>(r->fence[ec ^ 1], n_fence(Vn_ub));
+        k_build_fence_dev<<<g1(n_fence(Vn_ub)), 256, 0, st>>>(new_ext, dc, f);
         CKL();
     }
     // ---- a4/a5 without node ops: row offsets (while the outcome lists are L2-resident)
@@ -973,7 +956,6 @@ h2tap_status apply_core(h2tap_replica* r, const BatchIn& in, uint64_t S, bool cr
             r->get<uint64_t>(r->pt[pn], n_pend_new), r->get<uint64_t>(r->pq[pn], n_pend_new));
         CKL();
     }
-    if (idmap_pending) CK(cudaStreamWaitEvent(st, r->evE, 0));  // the ID map (third stream) is complete
     k_finish<<<1, 1, 0, st>>>(dc, V, Vr, E, node_mode ? 1 : 0, r->sharded ? 1 : 0, new_ext, new_off);
     CKL();
     CK(cudaEventRecord(r->ev[5], st));
@@ -1127,7 +1109,6 @@ h2tap_replica* new_replica(const h2tap_config* cfg) {
         int lo = 0, hi = 0;
         CK(cudaDeviceGetStreamPriorityRange(&lo, &hi));
         CK(cudaStreamCreateWithPriority(&r->st2, cudaStreamNonBlocking, lo));
-        CK(cudaStreamCreateWithPriority(&r->st3, cudaStreamNonBlocking, lo));
         CK(cudaStreamCreateWithFlags(&r->st_copy, cudaStreamNonBlocking));
         for (auto& g : r->stg) {
             CK(cudaEventCreateWithFlags(&g.ev, cudaEventDisableTiming));
@@ -1138,7 +1119,6 @@ h2tap_replica* new_replica(const h2tap_config* cfg) {
     CK(cudaEventCreateWithFlags(&r->evB, cudaEventDisableTiming));
     CK(cudaEventCreateWithFlags(&r->evC, cudaEventDisableTiming));
     CK(cudaEventCreateWithFlags(&r->evD, cudaEventDisableTiming));
-    CK(cudaEventCreateWithFlags(&r->evE, cudaEventDisableTiming));
     CK(cudaHostAlloc(reinterpret_cast<void**>(&r->hc), sizeof(Counters), cudaHostAllocMapped));
     CK(cudaHostGetDevicePointer(reinterpret_cast<void**>(&r->hc_dev), r->hc, 0));
     CK(cudaHostAlloc(reinterpret_cast<void**>(&r->hcf), sizeof(Counters), cudaHostAllocMapped));
@@ -1166,9 +1146,7 @@ void free_replica(h2tap_replica* r) {
     if (r->evC) cudaEventDestroy(r->evC);
     if (r->evD) cudaEventDestroy(r->evD);
     if (r->evS) cudaEventDestroy(r->evS);
-    if (r->evE) cudaEventDestroy(r->evE);
     if (r->st2) { cudaStreamSynchronize(r->st2); cudaStreamDestroy(r->st2); }
-    if (r->st3) { cudaStreamSynchronize(r->st3); cudaStreamDestroy(r->st3); }
     if (r->st_copy) { cudaStreamSynchronize(r->st_copy); cudaStreamDestroy(r->st_copy); }
     for (auto& g : r->stg) {
         for (Buf* b : {&g.k, &g.s, &g.d, &g.w, &g.t}) if (b->p) r->dfree(b->p);

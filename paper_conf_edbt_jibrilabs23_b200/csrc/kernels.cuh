@@ -1434,15 +1434,11 @@ __global__ void k_rows_partition(RowArgs a_) {
 #ifndef H2TAP_ROWS_MINB
 #define H2TAP_ROWS_MINB 6
 #endif
-// PART 1: the ID map (and liveness) only - it needs nothing from the edge-op phase and runs
-// beside it on a third stream; PART 2: the row offsets only; PART 3: both
-template <int PART>
 __global__ void __launch_bounds__(kThreads, H2TAP_ROWS_MINB) k_rows_fused(RowArgs a_) {
     const RowArgs a = row_counts(a_);
     const uint64_t k0 = (uint64_t)blockIdx.x * kRowTile, k1 = min(k0 + kRowTile, a.V_old);
     const uint64_t* pp = a.part + 2 * blockIdx.x;  // this CTA's slices of the delete / insert-row lists
-    uint64_t da = 0, ia = 0, db = 0, ib = 0;
-    if (PART & 2) { da = pp[0]; ia = pp[1]; db = pp[2]; ib = pp[3]; }
+    const uint64_t da = pp[0], ia = pp[1], db = pp[2], ib = pp[3];
     constexpr int PER = kRowTile / kThreads;  // ids per thread, all loads issued together
     uint32_t u[PER];
     uint64_t x[PER], ext[PER];
@@ -1456,9 +1452,9 @@ __global__ void __launch_bounds__(kThreads, H2TAP_ROWS_MINB) k_rows_fused(RowArg
         row[j] = false;
         if (k < k1) {
             u[j] = remap_of(a.R, (uint32_t)k);
-            if ((PART & 1) && !a.identity) ext[j] = a.old_ext[k];
-            if ((PART & 1) && a.new_live && u[j] != kNone32) a.new_live[u[j]] = a.old_live[k];
-            row[j] = (PART & 2) && k >= a.row_lo && k < a.row_hi;
+            if (!a.identity) ext[j] = a.old_ext[k];
+            if (a.new_live && u[j] != kNone32) a.new_live[u[j]] = a.old_live[k];
+            row[j] = k >= a.row_lo && k < a.row_hi;
             if (row[j]) x[j] = (uint64_t)a.old_off[k];
         }
     }
@@ -1468,7 +1464,7 @@ __global__ void __launch_bounds__(kThreads, H2TAP_ROWS_MINB) k_rows_fused(RowArg
 #pragma unroll
     for (int j = 0; j < PER; ++j) {
         if (u[j] == kNone32) continue;
-        if (PART & 1) a.new_ext[u[j]] = ext[j];
+        a.new_ext[u[j]] = ext[j];
         if (!row[j]) continue;
         const uint64_t kept = x[j] - cb[j] - lower_bound_dev(a.del_pos, da, db, x[j]);
         a.new_off[u[j] - a.row_lo_new] = (int64_t)(kept + lower_bound_dev(a.ins_row, ia, ib, u[j]));

@@ -327,6 +327,15 @@ h2tap_status h2tap_delta_apply_async(h2tap_replica* r, const h2tap_batch* batch,
 h2tap_status h2tap_replica_sync(h2tap_replica* r, h2tap_apply_stats* completed /* nullable */,
         int* has_completed /* nullable */);
 
+/* The pending set (ops committed after the current snapshot, kept for a later cycle, reading
+ * A6) in arrival order with their arrival numbers - the part of a checkpoint the CSR
+ * export does not hold (cf. the paper's persistent copy).  Arrays of n_pending
+ * entries (h2tap_replica_info), host or device (on_device), any may be NULL.  Restore:
+ * h2tap_replica_create_from_csr(create_ts = snapshot_ts) + h2tap_delta_apply of these ops at the
+ * same snapshot_ts (they stay pending, in the same relative order). */
+h2tap_status h2tap_pending_export(const h2tap_replica* r, uint8_t* kind, uint64_t* src, uint64_t* dst,
+        float* w, uint64_t* ts, uint64_t* seq, int on_device);
+
 /* Sizes of the current replica (any pointer may be NULL). */
 h2tap_status h2tap_replica_info(const h2tap_replica* r, uint64_t* n_vertices, uint64_t* n_edges,
         uint64_t* snapshot_ts, uint64_t* n_pending, uint64_t* shard_vertex_base,

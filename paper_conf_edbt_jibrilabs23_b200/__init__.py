@@ -143,6 +143,7 @@ for _n, _a in (("h2tap_batch_stage", [_P, ctypes.POINTER(_Batch), ctypes.POINTER
                ("h2tap_delta_apply_async", [_P, ctypes.POINTER(_Batch), _u64, ctypes.POINTER(ApplyStats),
                                             ctypes.POINTER(ctypes.c_int)]),
                ("h2tap_replica_sync", [_P, ctypes.POINTER(ApplyStats), ctypes.POINTER(ctypes.c_int)]),
+               ("h2tap_pending_export", [_P, _P, _P, _P, _P, _P, _P, ctypes.c_int]),
                ("h2tap_ds_create", [ctypes.c_int, ctypes.c_size_t, ctypes.POINTER(_P)]),
                ("h2tap_ds_append", [_P, _u64, _u64, ctypes.c_int, ctypes.c_int, _P, _P, ctypes.c_uint32, _P,
                                     ctypes.c_uint32]),
@@ -447,6 +448,14 @@ class Replica:
         _check(_lib.h2tap_delta_apply_async(self._h, ctypes.byref(b), int(snapshot_ts), ctypes.byref(st),
                                             ctypes.byref(has)), "h2tap_delta_apply_async")
         return st.as_dict() if has.value else None
+
+    def pending(self):
+        """h2tap_pending_export: (kind, src, dst, w, ts, seq) numpy arrays of the pending ops"""
+        n = self.info()["n_pending"]
+        a = [np.empty(n, dt) for dt in (np.uint8, np.uint64, np.uint64, np.float32, np.uint64, np.uint64)]
+        _check(_lib.h2tap_pending_export(self._h, *(ctypes.c_void_p(x.ctypes.data) for x in a), 0),
+               "h2tap_pending_export")
+        return a
 
     def sync(self):
         """h2tap_replica_sync: complete the last asynchronous cycle; its stats dict or None."""

@@ -12,6 +12,7 @@
 //   a7 swap                front <-> back at snapshot_ts (host pointer flip)
 // Host syncs read small counters between steps (sizes of the next launches).
 #include <cuda_runtime.h>
+#include <nvtx3/nvToolsExt.h>
 
 #include <cstdarg>
 #include <cstdlib>
@@ -104,8 +105,15 @@ struct Trace {
     Trace() { for (auto& x : ev) x = nullptr; }
 };
 thread_local Trace g_tr;
-#define TR(nm) g_tr.mark(nm, st)
+#define TR(nm) (g_tr.mark(nm, st), nvtxMarkA("h2tap " nm))
 inline int bits_for(uint64_t range) { return range == 0 ? 0 : 64 - __builtin_clzll(range); }
+
+// NVTX ranges (host timeline of nsys / ncu --nvtx): one per cycle and one per step of the path;
+// header-only NVTX 3, a no-op unless a tool is attached
+struct NvtxRange {
+    explicit NvtxRange(const char* name) { nvtxRangePushA(name); }
+    ~NvtxRange() { nvtxRangePop(); }
+};
 
 }  // namespace
 
@@ -439,6 +447,7 @@ h2tap_status apply_core(h2tap_replica* r, const BatchIn& in, uint64_t S, bool cr
     const uint64_t n = in.n, np = r->n_pend, m = np + n;
     if (r->prep.on) { set_err("a prepared cycle must be committed or aborted first"); return H2TAP_E_INVAL; }
     if (m >= 0xFFFFFFFFull) { set_err("batch + pending = %llu ops exceeds 2^32-1", (unsigned long long)m); return H2TAP_E_CAPACITY; }
+    NvtxRange nv_cycle(create ? "h2tap create" : "h2tap cycle");
     g_launches = in.pre_launches;
     g_h2d = in.pre_h2d;
     g_d2h = in.pre_d2h;
@@ -1711,6 +1720,30 @@ h2tap_status h2tap_delta_abort(h2tap_replica* r) {
     if (!r) { set_err("null replica"); return H2TAP_E_INVAL; }
     r->prep.on = false;  // the back buffers are simply overwritten by the next cycle
     return H2TAP_OK;
+}
+
+h2tap_status h2tap_pending_export(const h2tap_replica* rc, uint8_t* kind, uint64_t* src, uint64_t* dst, float* w,
+                                  uint64_t* ts, uint64_t* seq, int on_device) {
+    h2tap_replica* r = const_cast<h2tap_replica*>(rc);
+    if (!r) { set_err("null replica"); return H2TAP_E_INVAL; }
+    return run_guarded(r, [&]() -> h2tap_status {
+        ensure_final(r);
+        CK(cudaSetDevice(r->cfg.device));
+        const uint64_t n = r->n_pend;
+        const int pc = r->pcur;
+        const cudaMemcpyKind kd = on_device ? cudaMemcpyDeviceToDevice : cudaMemcpyDeviceToHost;
+        auto cp = [&](void* dst_, const Buf& b, size_t el) {
+            if (dst_ && n) CK(cudaMemcpyAsync(dst_, b.p, n * el, kd, r->st));
+        };
+        cp(kind, r->pk[pc], 1);
+        cp(src, r->ps[pc], 8);
+        cp(dst, r->pd[pc], 8);
+        cp(w, r->pw[pc], 4);
+        cp(ts, r->pt[pc], 8);
+        cp(seq, r->pq[pc], 8);
+        r->sync();
+        return H2TAP_OK;
+    });
 }
 
 h2tap_status h2tap_replica_info(const h2tap_replica* r, uint64_t* nv, uint64_t* ne, uint64_t* snap, uint64_t* npend,

@@ -395,3 +395,39 @@ def test_async_apply_stream(h2):
     g.apply(Batch.empty(0), ts + 100)
     o.apply(Batch.empty(0), ts + 100)
     assert_same(g.export(), o.export(), "sync after async")
+
+
+def test_pending_export_and_checkpoint_restore(h2):
+    """h2tap_pending_export equals O1's pending set (pinned in test_oracle_pins.py) after cycles
+    with deferral; a checkpoint (CSR export + pending ops) restored through create_from_csr and
+    one apply of the pending ops at the same snapshot continues exactly like the original."""
+    scale, seed = 10, 21
+    n = 1 << scale
+    src, dst, w = synth.rmat_edges(scale, seed)
+    g, o = pair_from_edges(h2, n, None, src, dst, w)
+    ts = 0
+    for k in range(3):
+        b = synth.rmat_batch(scale, seed, k, 3000, len(src), p_insert=0.7, p_weight=0.1, ts_base=ts)
+        snap = int(np.quantile(b.ts, 0.7))
+        step(g, o, b, snap, f"pending {k}")
+        ts = int(b.ts.max())
+        got, ref = g.pending(), o.pending()
+        for name, x, y in zip(("kind", "src", "dst", "w", "ts"), got[:5], ref[:5]):
+            assert np.array_equal(x.view(np.uint32) if x.dtype == np.float32 else x,
+                                  y.view(np.uint32) if y.dtype == np.float32 else y), f"pending {name}"
+        # arrival numbers: the same order and spacing (the replica also numbered its create edges)
+        assert len(got[5]) == len(ref[5])
+        if len(got[5]):
+            assert np.array_equal(got[5] - got[5][0], ref[5] - ref[5][0])
+    # checkpoint -> restore
+    off, cols, ww, ext = g.export()
+    kind, s_, d_, w_, t_, q_ = g.pending()
+    S = g.info()["snapshot_ts"]
+    h = h2.Replica.from_csr(off, cols, ww, ext, create_ts=S)
+    h.apply(Batch(kind, s_, d_, w_, t_), S)
+    assert h.info()["n_pending"] == len(kind)
+    b = synth.rmat_batch(scale, seed, 9, 3000, len(src), p_insert=0.7, p_weight=0.1, ts_base=ts)
+    last = int(b.ts.max())
+    g.apply(b, last)
+    h.apply(b, last)
+    assert_same(h.export(), g.export(), "restored checkpoint")

@@ -148,7 +148,7 @@ struct h2tap_replica {
     Buf op_flags, op_ou, op_ow;
     Buf ins_pos, ins_row, ins_col, ins_w, del_pos, upd_pos, upd_w, KR, cls_cat, cls_pos, cls_w;
     Buf misc, nsorted, part, opart, deg, tsum, remap_shift, remap32, casc_wrel, tile_emit, tile_base, del_row, casc_mask, status2, bfs_a, bfs_b, pr_a, pr_b;
-    Buf xrec, xins, xwts, xdel, xcnt, xoff;  // delta-record input (h2tap_delta_apply_records)
+    Buf xrec, xins, xwts, xdel, xcnt, xoff, xbig, xnbig;  // delta-record input (h2tap_delta_apply_records)
     bool tomb = false;  // tombstone-row mode (reading A23)
     // a finished cycle waiting for the swap (two-phase apply of a sharded replica: every
     // rank prepares, the ranks agree on the status, then all commit or all abort)
@@ -490,10 +490,17 @@ h2tap_status apply_core(h2tap_replica* r, const BatchIn& in, uint64_t S, bool cr
         k_unpack_recs<<<g1(n), 256, 0, st>>>(in.recs, n, Wk + np, Ws + np, Wd + np, Ww + np, Wt + np, Wq + np);
         CKL();
     } else if (n && in.drec) {
-        const unsigned grid = (unsigned)std::min<uint64_t>(cdiv(in.n_drec * 32, 256), (uint64_t)r->n_sm * 16);
-        k_rec_expand<<<grid, 256, 0, st>>>(in.drec, in.n_drec, in.drec_off, in.dins, in.dwts, in.ddel,
-                                           Wk + np, Ws + np, Wd + np, Ww + np, Wt + np, in.dwts64, in.vis_ts,
-                                           in.ins_base, in.del_base);
+        uint32_t* bigq = r->get<uint32_t>(r->xbig, in.n_drec);
+        unsigned long long* nbig = reinterpret_cast<unsigned long long*>(r->get<uint64_t>(r->xnbig, 1));
+        CK(cudaMemsetAsync(nbig, 0, 8, st));
+        k_rec_expand<0><<<g1(in.n_drec), 256, 0, st>>>(in.drec, in.n_drec, in.drec_off, in.dins, in.dwts, in.ddel,
+                                                      Wk + np, Ws + np, Wd + np, Ww + np, Wt + np, in.dwts64,
+                                                      in.vis_ts, in.ins_base, in.del_base, bigq, nbig);
+        CKL();
+        k_rec_expand<1><<<(unsigned)r->n_sm * 8, 256, 0, st>>>(in.drec, in.n_drec, in.drec_off, in.dins, in.dwts,
+                                                               in.ddel, Wk + np, Ws + np, Wd + np, Ww + np, Wt + np,
+                                                               in.dwts64, in.vis_ts, in.ins_base, in.del_base, bigq,
+                                                               nbig);
         CKL();
         k_fill_seq<<<g1(n), 256, 0, st>>>(Wq, np, n, r->next_seq);
         CKL();
@@ -1146,7 +1153,7 @@ void free_replica(h2tap_replica* r) {
                    &r->ins_oldpos, &r->hd_rows, &r->hd_bits, &r->op_flags, &r->op_ou, &r->op_ow,
                    &r->ins_pos, &r->ins_row, &r->ins_col, &r->ins_w, &r->del_pos, &r->upd_pos, &r->upd_w,
                    &r->KR, &r->cls_cat, &r->cls_pos, &r->cls_w, &r->misc, &r->nsorted, &r->part, &r->opart, &r->deg, &r->tsum, &r->remap_shift, &r->remap32, &r->casc_wrel, &r->tile_emit, &r->tile_base, &r->del_row, &r->casc_mask, &r->status2, &r->bounds_dev, &r->fence[0], &r->fence[1], &r->bfs_a, &r->bfs_b, &r->pr_a, &r->pr_b, &r->ctr,
-                   &r->xrec, &r->xins, &r->xwts, &r->xdel, &r->xcnt, &r->xoff, &r->live[0], &r->live[1], &r->casc_status};
+                   &r->xrec, &r->xins, &r->xwts, &r->xdel, &r->xcnt, &r->xoff, &r->xbig, &r->xnbig, &r->live[0], &r->live[1], &r->casc_status};
     for (Buf* b : bufs) if (b->p) r->dfree(b->p);
     cudaStreamSynchronize(r->st);
     for (auto& e : r->ev) if (e) cudaEventDestroy(e);
@@ -1569,6 +1576,7 @@ h2tap_status apply_records_dev(h2tap_replica* r, const DeltaRec* rec, uint64_t n
                                uint64_t snapshot_ts, h2tap_apply_stats* stats,
                                const std::function<void()>& overlap = {}) {
     cudaStream_t st = r->st;
+    if (nr >= 0xFFFFFFFFull) { set_err("%llu delta records in one cycle (limit 2^32 - 2)", (unsigned long long)nr); return H2TAP_E_CAPACITY; }
     uint64_t* cnt = r->get<uint64_t>(r->xcnt, nr + 1);
     uint64_t* off = r->get<uint64_t>(r->xoff, nr + 1);
     unsigned long long* tb = r->get<unsigned long long>(r->misc, 2);

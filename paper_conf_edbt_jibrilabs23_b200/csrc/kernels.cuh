@@ -431,18 +431,47 @@ __global__ void k_rec_count(const DeltaRec* __restrict__ rec, uint64_t n, uint64
         if (b) atomicOr(&tot_bad[1], (unsigned long long)b);
     }
 }
-// one warp per record (a record may carry thousands of inserts of a hub node).  Weights:
-// f32 (wts) or the paper's 8-byte weights (wts64) narrowed to the replica's
-// f32 by round-to-nearest-even (reading A15)
+// Expansion: pass 0 (BIG = 0) one thread per record for records of <= kRecSmall ops (most
+// deltas are one transaction's change to one node); larger records are queued and pass 1
+// (BIG = 1) gives each one warp (a hub's record may carry thousands of inserts).  Weights: f32
+// (wts) or the paper's 8-byte weights (wts64) narrowed to the replica's f32 by
+// round-to-nearest-even (reading A15).
+constexpr uint32_t kRecSmall = 8;
+template <int BIG>
 __global__ void k_rec_expand(const DeltaRec* __restrict__ rec, uint64_t n, const uint64_t* __restrict__ off,
                              const uint64_t* __restrict__ ins, const float* __restrict__ wts,
                              const uint64_t* __restrict__ del, uint8_t* __restrict__ kind, uint64_t* __restrict__ src,
                              uint64_t* __restrict__ dst, float* __restrict__ w, uint64_t* __restrict__ ts,
-                             const double* __restrict__ wts64 = nullptr, uint64_t vis_ts = ~0ull,
-                             uint64_t ins_base = 0, uint64_t del_base = 0) {
+                             const double* __restrict__ wts64, uint64_t vis_ts, uint64_t ins_base, uint64_t del_base,
+                             uint32_t* __restrict__ big, unsigned long long* __restrict__ n_big) {
+    if (!BIG) {
+        const uint64_t i = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x;
+        if (i >= n) return;
+        const DeltaRec r = rec[i];
+        if (!r.valid || r.ts > vis_ts) return;
+        const uint32_t a = r.inserted, b = a + r.del_cnt, c = b + r.ins_cnt, e = c + r.deleted;
+        if (e > kRecSmall) { big[atomicAdd(n_big, 1ull)] = (uint32_t)i; return; }
+        const uint64_t o = off[i], io = r.ins_off - ins_base, dq = r.del_off - del_base;
+        for (uint32_t j = 0; j < e; ++j) {
+            uint8_t k;
+            uint64_t d = 0;
+            float x = 0.f;
+            if (j < a) k = NODE_INSERT;
+            else if (j < b) { k = EDGE_DELETE; d = del[dq + (j - a)]; }
+            else if (j < c) {
+                k = EDGE_INSERT;
+                d = ins[io + (j - b)];
+                x = wts64 ? __double2float_rn(wts64[io + (j - b)]) : wts[io + (j - b)];
+            } else k = NODE_DELETE;
+            kind[o + j] = k; src[o + j] = r.node; dst[o + j] = d; w[o + j] = x; ts[o + j] = r.ts;
+        }
+        return;
+    }
     const uint64_t warp = (blockIdx.x * (uint64_t)blockDim.x + threadIdx.x) >> 5;
     const uint64_t nwarps = ((uint64_t)gridDim.x * blockDim.x) >> 5;
-    for (uint64_t i = warp; i < n; i += nwarps) {
+    const uint64_t nb = *n_big;
+    for (uint64_t q = warp; q < nb; q += nwarps) {
+        const uint64_t i = big[q];
         const DeltaRec r = rec[i];
         if (!r.valid || r.ts > vis_ts) continue;
         const uint64_t o = off[i], io = r.ins_off - ins_base, dq = r.del_off - del_base;

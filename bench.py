@@ -382,7 +382,7 @@ def run_gpu(args):
     torch.cuda.synchronize()
     # the e2e leg replays the timed batches on the same graph state: keep the state the timed
     # region starts from (device copy of the CSR + ID map; single replica, compact IDs)
-    restore = not sharded and not args.tombstone
+    restore = not sharded and not args.tombstone and not records
     inf0 = rep.info()
     if restore:
         snap0 = rep.export(on_device=True)

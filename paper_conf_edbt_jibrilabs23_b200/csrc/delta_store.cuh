@@ -39,9 +39,9 @@ struct h2tap_delta_store {
     uint64_t snap = 0;                                // snapshot of the last successful scan
     uint64_t mbase = 0, mlen = 0, mcap = 0;           // mirror holds records [mbase, mbase + mlen)
     uint64_t ibase = 0, ilen = 0, icap = 0, wcap = 0, dbase = 0, dlen = 0, dcap = 0;
-    DeltaRec* m_rec = nullptr;
-    uint64_t *m_ins = nullptr, *m_del = nullptr;
-    double* m_w = nullptr;
+    DeltaRec* m_rec = nullptr, *m_rec2 = nullptr;
+    uint64_t *m_ins = nullptr, *m_del = nullptr, *m_ins2 = nullptr, *m_del2 = nullptr;
+    double* m_w = nullptr, *m_w2 = nullptr;
     uint64_t freed_r = 0, freed_i = 0, freed_d = 0;   // host chunks released below these
     cudaStream_t cs = nullptr;
     cudaEvent_t ev = nullptr;
@@ -130,15 +130,18 @@ void ds_note_ts(h2tap_delta_store* s, uint64_t idx, uint64_t ts) {
     while (ts < cur && !m.compare_exchange_weak(cur, ts, std::memory_order_relaxed)) {}
 }
 
+// device mirror array + its compaction twin (the window moves between the two): grown 2x, rarely
 template <typename T>
-void ds_grow(T*& p, uint64_t& cap, uint64_t keep, uint64_t need) {  // device mirror array
+void ds_grow(T*& p, T*& p2, uint64_t& cap, uint64_t keep, uint64_t need) {
     if (need <= cap) return;
-    const uint64_t nc = std::max<uint64_t>(need + need / 2, 1024);
+    const uint64_t nc = std::max<uint64_t>(2 * need, 1024);
     T* q = nullptr;
     CK(cudaMalloc(&q, nc * sizeof(T)));
     if (keep) CK(cudaMemcpy(q, p, keep * sizeof(T), cudaMemcpyDeviceToDevice));
     if (p) CK(cudaFree(p));
+    if (p2) CK(cudaFree(p2));
     p = q;
+    CK(cudaMalloc(&p2, nc * sizeof(T)));
     cap = nc;
 }
 
@@ -343,7 +346,9 @@ void h2tap_ds_destroy(h2tap_delta_store* s) {
     }
     for (auto& f : s->free_chunks)
         for (void* p : f) cudaFreeHost(p);
-    for (void* p : {(void*)s->m_rec, (void*)s->m_ins, (void*)s->m_w, (void*)s->m_del}) if (p) cudaFree(p);
+    for (void* p : {(void*)s->m_rec, (void*)s->m_ins, (void*)s->m_w, (void*)s->m_del, (void*)s->m_rec2,
+                    (void*)s->m_ins2, (void*)s->m_w2, (void*)s->m_del2})
+        if (p) cudaFree(p);
     if (s->ev) cudaEventDestroy(s->ev);
     if (s->cs) cudaStreamDestroy(s->cs);
     delete s;
@@ -378,11 +383,15 @@ h2tap_status h2tap_delta_apply_store(h2tap_replica* r, h2tap_delta_store* s, uin
         ds_pos(s, end, np, pins, pdel, &ie, &de);
         // mirror capacity for everything published (read-ahead included), then the copies the
         // scan needs; the replica stream waits for them
-        CK(cudaStreamSynchronize(s->cs));  // earlier read-ahead copies: done before any regrow
-        ds_grow(s->m_rec, s->mcap, s->mlen, np - s->mbase);
-        ds_grow(s->m_ins, s->icap, s->ilen, pins - s->ibase);
-        ds_grow(s->m_w, s->wcap, s->ilen, pins - s->ibase);
-        ds_grow(s->m_del, s->dcap, s->dlen, pdel - s->dbase);
+        if (np - s->mbase > s->mcap || pins - s->ibase > s->icap || pins - s->ibase > s->wcap ||
+            pdel - s->dbase > s->dcap) {
+            CK(cudaStreamSynchronize(s->cs));  // earlier copies are done before a regrow
+            CK(cudaStreamSynchronize(st));
+            ds_grow(s->m_rec, s->m_rec2, s->mcap, s->mlen, np - s->mbase);
+            ds_grow(s->m_ins, s->m_ins2, s->icap, s->ilen, pins - s->ibase);
+            ds_grow(s->m_w, s->m_w2, s->wcap, s->ilen, pins - s->ibase);
+            ds_grow(s->m_del, s->m_del2, s->dcap, s->dlen, pdel - s->dbase);
+        }
         uint64_t h2d = ds_mirror(s, end, ie, de);
         CK(cudaEventRecord(s->ev, s->cs));
         CK(cudaStreamWaitEvent(st, s->ev, 0));
@@ -411,19 +420,20 @@ h2tap_status h2tap_delta_apply_store(h2tap_replica* r, h2tap_delta_store* s, uin
         s->cursor = cur; s->cur_ins = ci; s->cur_del = cd;
         s->snap = snapshot_ts;
         ds_release_below(s, cur, ci, cd);
-        // compact the mirror window when the consumed prefix is at least as long as what is kept
+        // move the mirror window to the twin buffers: what is still pending starts at slot 0 again
         const uint64_t rs = cur - s->mbase, is = ci - s->ibase, dsh = cd - s->dbase;
-        if (rs && rs >= s->mlen - rs && is >= s->ilen - is && dsh >= s->dlen - dsh) {
+        if (rs) {
             CK(cudaEventRecord(s->ev, st));  // the consume kernel ran on the replica stream
             CK(cudaStreamWaitEvent(s->cs, s->ev, 0));
-            auto shift = [&](void* p, uint64_t by, uint64_t len, size_t el) {
+            auto move = [&](auto*& p, auto*& p2, uint64_t by, uint64_t len) {
                 if (len > by)
-                    CK(cudaMemcpyAsync(p, (char*)p + by * el, (len - by) * el, cudaMemcpyDeviceToDevice, s->cs));
+                    CK(cudaMemcpyAsync(p2, p + by, (len - by) * sizeof(*p), cudaMemcpyDeviceToDevice, s->cs));
+                std::swap(p, p2);
             };
-            shift(s->m_rec, rs, s->mlen, sizeof(DeltaRec));
-            shift(s->m_ins, is, s->ilen, 8);
-            shift(s->m_w, is, s->ilen, 8);
-            shift(s->m_del, dsh, s->dlen, 8);
+            move(s->m_rec, s->m_rec2, rs, s->mlen);
+            move(s->m_ins, s->m_ins2, is, s->ilen);
+            move(s->m_w, s->m_w2, is, s->ilen);
+            move(s->m_del, s->m_del2, dsh, s->dlen);
             s->mbase = cur; s->mlen -= rs;
             s->ibase = ci; s->ilen -= is;
             s->dbase = cd; s->dlen -= dsh;

@@ -260,26 +260,52 @@ h2tap_status h2tap_ds_append_records(h2tap_delta_store* s, const h2tap_delta_rec
         }
     }
     return run_guarded(nullptr, [&]() -> h2tap_status {
+        uint64_t si = 0, sd = 0;   // the records' slices (a caller array may hold unused entries)
+        for (size_t i = 0; i < n; ++i) { si += in[i].ins_cnt; sd += in[i].del_cnt; }
         uint64_t idx, io, dq;
         {
             std::lock_guard<std::mutex> g(s->mu);
-            ds_reserve_chunks(s, s->n_res, s->n_res + n, s->ins_res, s->ins_res + n_ins, s->del_res, s->del_res + n_del);
+            ds_reserve_chunks(s, s->n_res, s->n_res + n, s->ins_res, s->ins_res + si, s->del_res, s->del_res + sd);
             idx = s->n_res; s->n_res += n;
-            io = s->ins_res; s->ins_res += n_ins;
-            dq = s->del_res; s->del_res += n_del;
+            io = s->ins_res; s->ins_res += si;
+            dq = s->del_res; s->del_res += sd;
         }
-        ds_scatter(s, s->ich, s->cpay, io, n_ins, inserts);
-        ds_scatter(s, s->wch, s->cpay, io, n_ins, weights);
-        ds_scatter(s, s->dch, s->cpay, dq, n_del, deletes);
+        n_ins = si;   // what is copied below
+        n_del = sd;
+        // The store keeps every record's slices in record order (payload offsets grow with the
+        // record index; an empty slice sits at the running position): a caller layout that is
+        // already back to back goes in with one copy per array, any other is gathered per record.
+        bool packed = true;
+        for (uint64_t i = 0, pi = 0, pd = 0; i < n && packed; ++i) {
+            packed = (in[i].ins_cnt == 0 || in[i].ins_off == pi) && (in[i].del_cnt == 0 || in[i].del_off == pd);
+            pi += in[i].ins_cnt;
+            pd += in[i].del_cnt;
+        }
+        if (packed) {
+            ds_scatter(s, s->ich, s->cpay, io, n_ins, inserts);
+            ds_scatter(s, s->wch, s->cpay, io, n_ins, weights);
+            ds_scatter(s, s->dch, s->cpay, dq, n_del, deletes);
+        } else {
+            for (uint64_t i = 0, pi = io, pd = dq; i < n; ++i) {
+                ds_scatter(s, s->ich, s->cpay, pi, in[i].ins_cnt, inserts + in[i].ins_off);
+                ds_scatter(s, s->wch, s->cpay, pi, in[i].ins_cnt, weights + in[i].ins_off);
+                ds_scatter(s, s->dch, s->cpay, pd, in[i].del_cnt, deletes + in[i].del_off);
+                pi += in[i].ins_cnt;
+                pd += in[i].del_cnt;
+            }
+        }
         const uint64_t bs = 1u << 14;
         std::vector<DeltaRec> tmp(std::min<uint64_t>(n, bs));
-        for (uint64_t a = 0; a < n; a += bs) {  // rebased to the store's array positions
+        uint64_t pi = io, pd = dq;   // running positions (the records' slices, in record order)
+        for (uint64_t a = 0; a < n; a += bs) {
             const uint64_t k = std::min<uint64_t>(bs, n - a);
             uint64_t mn = ~0ull;
             for (uint64_t i = 0; i < k; ++i) {
                 tmp[i] = in[a + i];
-                tmp[i].ins_off += io;
-                tmp[i].del_off += dq;
+                tmp[i].ins_off = pi;
+                tmp[i].del_off = pd;
+                pi += tmp[i].ins_cnt;
+                pd += tmp[i].del_cnt;
             }
             ds_scatter(s, s->rch, s->crec, idx + a, k, tmp.data());
             for (uint64_t i = 0; i < k; ++i) {
@@ -287,7 +313,7 @@ h2tap_status h2tap_ds_append_records(h2tap_delta_store* s, const h2tap_delta_rec
                 if (((idx + a + i + 1) % s->kBlock) == 0 || i + 1 == k) { ds_note_ts(s, idx + a + i, mn); mn = ~0ull; }
             }
         }
-        ds_publish(s, idx, n, io + n_ins, dq + n_del);
+        ds_publish(s, idx, n, io + si, dq + sd);
         return H2TAP_OK;
     });
 }

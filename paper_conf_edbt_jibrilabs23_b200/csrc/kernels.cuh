@@ -415,10 +415,11 @@ __global__ void k_rec_count(const DeltaRec* __restrict__ rec, uint64_t n, uint64
     if (i < n) {
         const DeltaRec r = rec[i];
         if (r.valid > 1 || r.deleted > 1 || r.inserted > 1) bad |= REC_BAD_FLAG;
-        if (r.valid) {
-            if (r.ins_off < ins_base || r.del_off < del_base || r.ins_off - ins_base > n_ins ||
-                r.ins_cnt > n_ins - (r.ins_off - ins_base) || r.del_off - del_base > n_del ||
-                r.del_cnt > n_del - (r.del_off - del_base))
+        if (r.valid) {   // an empty slice's offset is never read
+            if ((r.ins_cnt && (r.ins_off < ins_base || r.ins_off - ins_base > n_ins ||
+                               r.ins_cnt > n_ins - (r.ins_off - ins_base))) ||
+                (r.del_cnt && (r.del_off < del_base || r.del_off - del_base > n_del ||
+                               r.del_cnt > n_del - (r.del_off - del_base))))
                 bad |= REC_BAD_SLICE;
             if (r.ts <= vis_ts) c = (uint64_t)r.inserted + r.del_cnt + r.ins_cnt + r.deleted;
         }

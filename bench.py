@@ -639,6 +639,7 @@ def run_store(args):
     store = h2.DeltaStore(0)
     n_total = args.warmup + args.steps
     batches = [wl.batch(k) for k in range(n_total + 1)]
+    snaps = [int(b.ts.max()) for b in batches]  # (a max over the batch: outside the timed region)
     rbs = []
     for b in batches:
         rb = synth.records_from_ops(b)
@@ -651,7 +652,8 @@ def run_store(args):
             e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
             torch.cuda.synchronize()
             e0.record(stream)
-            st = rep.apply_store(store, int(batches[k].ts.max()))
+            st = rep.apply_store(store, snaps[k])
+            store.join(stream)                      # the cycle's read-ahead copy is inside the timing
             e1.record(stream)
             torch.cuda.synchronize()
             if k >= args.warmup:
@@ -671,7 +673,8 @@ def run_store(args):
                     "h2d_bytes_per_step": int(sum(s["h2d_bytes"] for s in stats) / len(stats)),
                     "d2h_bytes_per_step": int(sum(s["d2h_bytes"] for s in stats) / len(stats)),
                     "how": "store on the host; every byte of it crosses to the GPU inside the timed cycles "
-                           "(read-ahead of batch k+1 overlaps cycle k)"},
+                           "(read-ahead of batch k+1 overlaps cycle k; a cycle's timing ends when both "
+                           "its replica work and its read-ahead copy are complete)"},
             "store_bytes_per_batch": rec_bytes,
             "gpu_launches": int(sum(s["n_launches"] for s in stats)),
             "phase_ms": {k: sum(s[k] for s in stats) / len(stats) for k in ("ms_ingest", "ms_merge", "ms_total")},

@@ -247,6 +247,11 @@ void h2tap_ds_destroy(h2tap_delta_store* s);
  * h2d_bytes = the store's bytes copied to the device by this call. */
 h2tap_status h2tap_delta_apply_store(h2tap_replica* r, h2tap_delta_store* s, uint64_t snapshot_ts,
         h2tap_apply_stats* stats /* nullable */);
+/* Make `stream` (a cudaStream_t of the store's device; NULL = the legacy default stream) wait
+ * for every host-to-device copy the store has issued so far - the read-ahead of the deltas a
+ * cycle left for later keeps running after h2tap_delta_apply_store returns; an event recorded
+ * on `stream` after this call completes only when those copies have.  Nothing blocks the host. */
+h2tap_status h2tap_ds_join(h2tap_delta_store* s, void* stream);
 
 /* ---- exchange step of a sharded apply ----------------------
  * A rank holding a slice of the global batch (i) validates it (every rank must agree

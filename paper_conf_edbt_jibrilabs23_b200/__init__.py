@@ -151,6 +151,7 @@ for _n, _a in (("h2tap_batch_stage", [_P, ctypes.POINTER(_Batch), ctypes.POINTER
                ("h2tap_ds_info", [_P] + [ctypes.POINTER(_u64)] * 5),
                ("h2tap_ds_export", [_P, _u64, ctypes.c_size_t, _P]),
                ("h2tap_delta_apply_store", [_P, _P, _u64, ctypes.POINTER(ApplyStats)]),
+               ("h2tap_ds_join", [_P, _P]),
                ("h2tap_dyn_pagerank", [_P, ctypes.c_double, ctypes.c_int, _P]),
                ("h2tap_dyn_sssp", [_P, _u64, _P]),
                ("h2tap_dyn_stage", [_P, ctypes.POINTER(_RecordBatch), ctypes.POINTER(_RecordBatch)]),
@@ -759,6 +760,15 @@ class DeltaStore:
         _check(_lib.h2tap_ds_info(self._h, *(ctypes.byref(x) for x in v)), "h2tap_ds_info")
         return dict(n_records=v[0].value, first_pending=v[1].value, n_mirrored=v[2].value,
                     host_bytes=v[3].value, device_bytes=v[4].value)
+
+    def join(self, stream=None):
+        """h2tap_ds_join: `stream` (a torch.cuda.Stream or raw handle; None = the current torch
+        stream) waits for the store's outstanding host-to-device copies (the read-ahead)"""
+        if stream is None:
+            import torch
+            stream = torch.cuda.current_stream()
+        h = getattr(stream, "cuda_stream", stream)
+        _check(_lib.h2tap_ds_join(self._h, ctypes.c_void_p(int(h or 0))), "h2tap_ds_join")
 
     def export(self, first: int, n: int):
         """records [first, first + n) of the live window, current validity flags"""

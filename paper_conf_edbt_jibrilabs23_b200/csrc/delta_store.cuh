@@ -55,6 +55,21 @@ struct h2tap_delta_store {
 
 namespace {
 
+// the mirror's compaction: up to four arrays (records, inserts, weights, deletes) moved to
+// their twin buffers in one launch, 8-byte words, grid-stride
+struct DsMove {
+    const uint64_t* src[4];
+    uint64_t* dst[4];
+    uint64_t words[4];
+};
+__global__ void k_ds_move(DsMove m) {
+    const uint64_t stride = (uint64_t)gridDim.x * blockDim.x;
+#pragma unroll
+    for (int k = 0; k < 4; ++k)
+        for (uint64_t i = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; i < m.words[k]; i += stride)
+            m.dst[k][i] = __ldcs(m.src[k] + i);
+}
+
 // pinned chunks are recycled (cudaHostAlloc / cudaFreeHost cost milliseconds and synchronise):
 // a released chunk goes to its size class's free list and the next reservation takes it
 template <typename T>
@@ -359,6 +374,18 @@ h2tap_status h2tap_ds_export(h2tap_delta_store* s, uint64_t first, size_t n, h2t
     });
 }
 
+h2tap_status h2tap_ds_join(h2tap_delta_store* s, void* stream) {
+    if (!s) { set_err("null argument"); return H2TAP_E_INVAL; }
+    try {
+        CK(cudaSetDevice(s->device));
+        CK(cudaEventRecord(s->ev, s->cs));
+        CK(cudaStreamWaitEvent(static_cast<cudaStream_t>(stream), s->ev, 0));
+    } catch (const Fail& e) {
+        return e.st;
+    }
+    return H2TAP_OK;
+}
+
 void h2tap_ds_destroy(h2tap_delta_store* s) {
     if (!s) return;
     cudaSetDevice(s->device);
@@ -390,6 +417,8 @@ h2tap_status h2tap_delta_apply_store(h2tap_replica* r, h2tap_delta_store* s, uin
             set_err("snapshot_ts %llu < current %llu", (unsigned long long)snapshot_ts, (unsigned long long)r->snap);
             return H2TAP_E_SNAPSHOT_REGRESSION;
         }
+        g_ht.init();
+        g_ht.mark("entry");
         CK(cudaSetDevice(r->cfg.device));
         cudaStream_t st = r->st;
         g_launches = g_h2d = g_d2h = 0;
@@ -405,6 +434,7 @@ h2tap_status h2tap_delta_apply_store(h2tap_replica* r, h2tap_delta_store* s, uin
             if (s->bmin[b0 / s->crec].load()[(b0 % s->crec) / s->kBlock].load() <= snapshot_ts) break;
             end = b0;
         }
+        g_ht.mark("visible_end");
         uint64_t ie, de;  // payload positions at the scan's end
         ds_pos(s, end, np, pins, pdel, &ie, &de);
         // mirror capacity for everything published (read-ahead included), then the copies the
@@ -418,28 +448,43 @@ h2tap_status h2tap_delta_apply_store(h2tap_replica* r, h2tap_delta_store* s, uin
             ds_grow(s->m_w, s->m_w2, s->wcap, s->ilen, pins - s->ibase);
             ds_grow(s->m_del, s->m_del2, s->dcap, s->dlen, pdel - s->dbase);
         }
+        g_ht.mark("grow");
         uint64_t h2d = ds_mirror(s, end, ie, de);
         CK(cudaEventRecord(s->ev, s->cs));
         CK(cudaStreamWaitEvent(st, s->ev, 0));
+        g_ht.mark("mirror");
         const uint64_t nr = end - s->cursor;
         DeltaRec* rec = s->m_rec + (s->cursor - s->mbase);
         // read-ahead: the copies of the not-yet-needed deltas are issued while the scan kernels run
         // and overlap the rest of the cycle (the mirror's capacity was reserved above)
         uint64_t ra = 0;
+        // consumed records -> invalid, enqueued behind the cycle's last kernel so that the
+        // first still-pending record comes back with the cycle's own read-back (Counters);
+        // the kernel marks nothing when the cycle's status carries an error
+        bool consumed = false;
+        const std::function<void()> consume = [&] {
+            if (nr) {
+                k_rec_consume<<<g1(nr), 256, 0, st>>>(rec, nr, snapshot_ts, r->dctr(), ST_NOT_OWNED | ST_CREATE_ENDPOINT);
+                CK(cudaGetLastError());
+            }
+            consumed = true;
+        };
         h2tap_status rc = apply_records_dev(r, rec, nr, s->m_ins, nullptr, s->m_w, ie - s->ibase, s->m_del,
                                             de - s->dbase, snapshot_ts, s->ibase, s->dbase, snapshot_ts, stats,
-                                            [&] { ra = ds_mirror(s, np, pins, pdel); });
+                                            [&] { ra = ds_mirror(s, np, pins, pdel); }, &consume);
+        g_ht.mark("apply");
         h2d += ra;
         if (stats) stats->h2d_bytes += h2d;
         if (rc != H2TAP_OK) return rc;
-        // consumed records -> invalid; the first still-pending record becomes the cursor
-        unsigned long long* fp = r->get<unsigned long long>(r->misc, 2);
-        CK(cudaMemsetAsync(fp, 0xFF, 8, st));
-        if (nr) { k_rec_consume<<<g1(nr), 256, 0, st>>>(rec, nr, snapshot_ts, fp); CK(cudaGetLastError()); }
-        unsigned long long first = 0;
-        CK(cudaMemcpyAsync(&first, fp, 8, cudaMemcpyDeviceToHost, st));
-        CK(cudaStreamSynchronize(st));
-        if (stats) { stats->d2h_bytes += 8; stats->n_launches += nr ? 1 : 0; }
+        unsigned long long first = r->hc->first_pend;
+        if (!consumed) {  // the cycle ended before its final read-back (nothing visible): mark here
+            k_init_counters<<<1, 32, 0, st>>>(r->dctr());
+            consume();
+            r->read_counters();
+            first = r->hc->first_pend;
+        }
+        g_ht.mark("consume");
+        if (stats) stats->n_launches += nr ? 1 : 0;
         const uint64_t cur = s->cursor + std::min<uint64_t>(first, nr);
         uint64_t ci, cd;
         ds_pos(s, cur, np, pins, pdel, &ci, &cd);
@@ -451,19 +496,31 @@ h2tap_status h2tap_delta_apply_store(h2tap_replica* r, h2tap_delta_store* s, uin
         if (rs) {
             CK(cudaEventRecord(s->ev, st));  // the consume kernel ran on the replica stream
             CK(cudaStreamWaitEvent(s->cs, s->ev, 0));
-            auto move = [&](auto*& p, auto*& p2, uint64_t by, uint64_t len) {
-                if (len > by)
-                    CK(cudaMemcpyAsync(p2, p + by, (len - by) * sizeof(*p), cudaMemcpyDeviceToDevice, s->cs));
+            DsMove mv{};
+            int k = 0;
+            auto seg = [&](auto*& p, auto*& p2, uint64_t by, uint64_t len) {
+                if (len > by) {
+                    mv.src[k] = reinterpret_cast<const uint64_t*>(p + by);
+                    mv.dst[k] = reinterpret_cast<uint64_t*>(p2);
+                    mv.words[k] = (len - by) * sizeof(*p) / 8;
+                    ++k;
+                }
                 std::swap(p, p2);
             };
-            move(s->m_rec, s->m_rec2, rs, s->mlen);
-            move(s->m_ins, s->m_ins2, is, s->ilen);
-            move(s->m_w, s->m_w2, is, s->ilen);
-            move(s->m_del, s->m_del2, dsh, s->dlen);
+            seg(s->m_rec, s->m_rec2, rs, s->mlen);
+            seg(s->m_ins, s->m_ins2, is, s->ilen);
+            seg(s->m_w, s->m_w2, is, s->ilen);
+            seg(s->m_del, s->m_del2, dsh, s->dlen);
+            if (k) {
+                k_ds_move<<<(unsigned)(r->n_sm * 4), 256, 0, s->cs>>>(mv);
+                CK(cudaGetLastError());
+            }
             s->mbase = cur; s->mlen -= rs;
             s->ibase = ci; s->ilen -= is;
             s->dbase = cd; s->dlen -= dsh;
         }
+        g_ht.mark("release+move");
+        g_ht.dump("store cycle");
         return H2TAP_OK;
     });
 }

@@ -16,6 +16,7 @@
 
 #include <cstdarg>
 #include <cstdlib>
+#include <chrono>
 #include <cstdio>
 #include <cstring>
 #include <functional>
@@ -106,6 +107,23 @@ struct Trace {
 };
 thread_local Trace g_tr;
 #define TR(nm) (g_tr.mark(nm, st), nvtxMarkA("h2tap " nm))
+// host-side timestamps of the same opt-in trace (host stalls vs device time)
+struct HostTrace {
+    bool on = false;
+    int n = 0;
+    const char* name[32];
+    std::chrono::steady_clock::time_point t[32];
+    void init() { const char* e = getenv("H2TAP_TRACE"); on = e && *e && *e != '0'; n = 0; }
+    void mark(const char* nm) { if (on && n < 32) { name[n] = nm; t[n++] = std::chrono::steady_clock::now(); } }
+    void dump(const char* what) {
+        if (!on || n < 2) return;
+        fprintf(stderr, "[h2tap host %s]", what);
+        for (int i = 1; i < n; ++i)
+            fprintf(stderr, " %s=%.1fus", name[i], std::chrono::duration<double, std::micro>(t[i] - t[i - 1]).count());
+        fprintf(stderr, " | total=%.1fus\n", std::chrono::duration<double, std::micro>(t[n - 1] - t[0]).count());
+    }
+};
+thread_local HostTrace g_ht;
 inline int bits_for(uint64_t range) { return range == 0 ? 0 : 64 - __builtin_clzll(range); }
 
 // NVTX ranges (host timeline of nsys / ncu --nvtx): one per cycle and one per step of the path;
@@ -195,6 +213,8 @@ struct h2tap_replica {
     Buf ctr;
     Counters* hc = nullptr;      // pinned, device-mapped host mirror
     Counters* hc_dev = nullptr;  // its device address: a kernel writes it (no copy engine)
+    unsigned long long* hx = nullptr;      // mapped host words of the record pre-pass read-back
+    unsigned long long* hx_dev = nullptr;
     cudaEvent_t ev[8]{};
 
     void* dalloc(size_t bytes) {
@@ -335,6 +355,8 @@ struct BatchIn {
     const double* dwts64 = nullptr;                  // 8-byte weights (narrowed to f32)
     uint64_t vis_ts = ~0ull, ins_base = 0, del_base = 0;  // delta-store scan: visibility, window bases
     uint64_t pre_h2d = 0, pre_d2h = 0, pre_launches = 0;  // accounting of the record pre-pass
+    const std::function<void()>* after_merge_launch = nullptr;  // host work issued behind the merge
+    const std::function<void()>* before_readback = nullptr;     // kernels enqueued before the final read-back
 };
 
 template <typename T>
@@ -452,6 +474,7 @@ h2tap_status apply_core(h2tap_replica* r, const BatchIn& in, uint64_t S, bool cr
     g_h2d = in.pre_h2d;
     g_d2h = in.pre_d2h;
     g_tr.init();
+    g_ht.mark("core_start");
     const bool async = r->async_req && !create && !r->sharded && !r->defer_commit && !g_tr.on;
     for (int i = 0; i < 8; ++i)
         if (!r->ev[i]) CK(cudaEventCreate(&r->ev[i]));
@@ -582,10 +605,13 @@ h2tap_status apply_core(h2tap_replica* r, const BatchIn& in, uint64_t S, bool cr
         radix_sort(r, sk, sv, sk2, sv2, m, 2 * sbits, &dc->n_valid);
     }
     TR("assemble+partition");
+    g_ht.mark("a1_issued");
     CK(cudaEventSynchronize(r->evS));
+    g_ht.mark("sync1");
     TR("sync1");
     if (r->infl.on) finalize_inflight(r);  // the previous (asynchronous) cycle's counters precede this read-back
     Counters hc = *r->hc;
+    g_ht.mark("hc_read");
     if (hc.status & ST_BAD_KIND) { set_err("unknown op kind in batch"); return H2TAP_E_INVAL; }
     if (hc.status & ST_STALE) {
         set_err("op with ts <= current snapshot_ts %llu (reading A7)", (unsigned long long)r->snap);
@@ -725,6 +751,7 @@ h2tap_status apply_core(h2tap_replica* r, const BatchIn& in, uint64_t S, bool cr
         casc_pending = true;
     }
     CK(cudaEventRecord(r->ev[2], st));
+    g_ht.mark("idmap");
     TR("idmap+remap");
 
     // ---- a3: edge ops -> keys, sort, segmented reduce + classify
@@ -952,6 +979,7 @@ h2tap_status apply_core(h2tap_replica* r, const BatchIn& in, uint64_t S, bool cr
         if (node_mode) launch(k_merge3<true, true>);
         else launch(k_merge3<false, false>);
         CKL();
+        if (in.after_merge_launch) (*in.after_merge_launch)();
     } else {
         CK(cudaEventRecord(r->ev[6], st));
     }
@@ -997,8 +1025,11 @@ h2tap_status apply_core(h2tap_replica* r, const BatchIn& in, uint64_t S, bool cr
         if (stats) memset(stats, 0, sizeof *stats);
         return H2TAP_OK;
     }
+    if (in.before_readback) (*in.before_readback)();
+    g_ht.mark("issued");
     r->read_counters();  // the one read-back of the cycle's device-side sizes
     TR("end");
+    g_ht.mark("core_end");
     g_tr.dump();
     const Counters& fc = *r->hc;
     if (create && (fc.status & ST_CREATE_ENDPOINT)) {
@@ -1139,6 +1170,8 @@ h2tap_replica* new_replica(const h2tap_config* cfg) {
     CK(cudaHostGetDevicePointer(reinterpret_cast<void**>(&r->hc_dev), r->hc, 0));
     CK(cudaHostAlloc(reinterpret_cast<void**>(&r->hcf), sizeof(Counters), cudaHostAllocMapped));
     CK(cudaHostGetDevicePointer(reinterpret_cast<void**>(&r->hcf_dev), r->hcf, 0));
+    CK(cudaHostAlloc(reinterpret_cast<void**>(&r->hx), 64, cudaHostAllocMapped));
+    CK(cudaHostGetDevicePointer(reinterpret_cast<void**>(&r->hx_dev), r->hx, 0));
     r->get<Counters>(r->ctr, 1);
     return r;
 }
@@ -1171,6 +1204,7 @@ void free_replica(h2tap_replica* r) {
     }
     if (r->hc) cudaFreeHost(r->hc);
     if (r->hcf) cudaFreeHost(r->hcf);
+    if (r->hx) cudaFreeHost(r->hx);
     for (auto& e : r->evx) if (e) cudaEventDestroy(e);
     delete r;
 }
@@ -1574,7 +1608,8 @@ h2tap_status apply_records_dev(h2tap_replica* r, const DeltaRec* rec, uint64_t n
                                const float* wts, const double* wts64, uint64_t n_ins, const uint64_t* del,
                                uint64_t n_del, uint64_t vis_ts, uint64_t ins_base, uint64_t del_base,
                                uint64_t snapshot_ts, h2tap_apply_stats* stats,
-                               const std::function<void()>& overlap = {}) {
+                               const std::function<void()>& overlap = {},
+                               const std::function<void()>* before_readback = nullptr) {
     cudaStream_t st = r->st;
     if (nr >= 0xFFFFFFFFull) { set_err("%llu delta records in one cycle (limit 2^32 - 2)", (unsigned long long)nr); return H2TAP_E_CAPACITY; }
     uint64_t* cnt = r->get<uint64_t>(r->xcnt, nr + 1);
@@ -1592,18 +1627,35 @@ h2tap_status apply_records_dev(h2tap_replica* r, const DeltaRec* rec, uint64_t n
         k_scan_exclusive_u64<<<(unsigned)nt, kThreads, 0, st>>>(cnt, off, nr, stt, ctr);
         CKL();
     }
-    unsigned long long h[2] = {0, 0};
-    CK(cudaMemcpyAsync(h, tb, 16, cudaMemcpyDeviceToHost, st));
+    // the op count and flags come back through mapped host words (a one-warp kernel store: no
+    // pageable copy, no copy-engine queue behind an H2D transfer)
+    k_store_words<<<1, 32, 0, st>>>(tb, 2, r->hx_dev);
+    CKL();
     g_d2h += 16;
-    if (overlap) overlap();  // host work that can run while the scan kernels execute
+    g_ht.mark("count_issued");
+    // host work that overlaps the cycle (the delta store's read-ahead copies): issued behind
+    // the merge launch by default.  While a host-to-device DMA runs, the short kernels of the
+    // cycle start late (measured: the sort / classify / partition segments of a C3 cycle grow
+    // by ~0.25 ms), so the copy is issued where one long kernel follows.  H2TAP_RA=0: behind
+    // the scan kernels instead; 2: after the cycle (profiles/r2/store/README.md)
+    static const int ra_mode = [] { const char* e = getenv("H2TAP_RA"); return e ? atoi(e) : 1; }();
+    bool ran = false;
+    const std::function<void()> late = [&] { if (!ran && overlap) { ran = true; overlap(); } };
+    if (ra_mode == 0) late();
+    g_ht.mark("overlap");
     r->sync();  // the expanded op count sizes the work buffers
+    const unsigned long long h[2] = {r->hx[0], r->hx[1]};
+    g_ht.mark("count_sync");
     if (h[1] & REC_BAD_FLAG) { set_err("delta record flag other than 0/1"); return H2TAP_E_INVAL; }
     if (h[1] & REC_BAD_SLICE) { set_err("delta record slice outside the inserts/weights/deletes arrays"); return H2TAP_E_INVAL; }
     BatchIn in{h[0], 1, nullptr, nullptr, nullptr, nullptr, nullptr, nullptr, 0};
     in.drec = rec; in.n_drec = nr; in.drec_off = off; in.dins = ins; in.dwts = wts; in.ddel = del;
     in.dwts64 = wts64; in.vis_ts = vis_ts; in.ins_base = ins_base; in.del_base = del_base;
     in.pre_h2d = g_h2d; in.pre_d2h = g_d2h; in.pre_launches = g_launches;
+    if (ra_mode == 1) in.after_merge_launch = &late;
+    in.before_readback = before_readback;
     const h2tap_status s = apply_core(r, in, snapshot_ts, false, stats);
+    if (s == H2TAP_OK) late();  // no merge this cycle (or H2TAP_RA=2): after it
     if (s == H2TAP_OK && stats) {  // the scan pre-pass is part of ingest
         const float pre = ev_ms(r->ev[7], r->ev[0]);
         stats->ms_ingest += pre;
@@ -1628,6 +1680,8 @@ h2tap_status h2tap_delta_apply_records(h2tap_replica* r, const h2tap_record_batc
             set_err("snapshot_ts %llu < current %llu", (unsigned long long)snapshot_ts, (unsigned long long)r->snap);
             return H2TAP_E_SNAPSHOT_REGRESSION;
         }
+        g_ht.init();
+        g_ht.mark("entry");
         CK(cudaSetDevice(r->cfg.device));
         g_launches = g_h2d = g_d2h = 0;
         if (!r->ev[7]) CK(cudaEventCreate(&r->ev[7]));
@@ -1656,8 +1710,11 @@ h2tap_status h2tap_delta_apply_records(h2tap_replica* r, const h2tap_record_batc
             copy_in(r, xd, del, b->n_deletes, 0);
             ins = xi; del = xd;
         }
-        return apply_records_dev(r, rec, nr, ins, wts, w64, b->n_inserts, del, b->n_deletes, ~0ull, 0, 0,
-                                 snapshot_ts, stats);
+        const h2tap_status rc = apply_records_dev(r, rec, nr, ins, wts, w64, b->n_inserts, del, b->n_deletes,
+                                                  ~0ull, 0, 0, snapshot_ts, stats);
+        g_ht.mark("return");
+        g_ht.dump("records cycle");
+        return rc;
     });
 }
 

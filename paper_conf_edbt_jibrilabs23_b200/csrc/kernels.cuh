@@ -40,7 +40,7 @@ struct Counters {
     unsigned long long row_lo_new, row_hi_new;  // sharded: the shard's row range in the new ID map
     unsigned long long Vn, Vr_new, En, new_identity;  // written by k_finish
     unsigned long long n_killed;  // vertices live before the cycle and dead after it (stats)
-    unsigned long long pad_;
+    unsigned long long first_pend;  // delta-store scan: first record left valid (k_rec_consume)
     unsigned int tiles[16];
 };
 
@@ -49,12 +49,15 @@ __global__ void k_store_counters(const Counters* __restrict__ c, Counters* host_
     for (int i = threadIdx.x; i < nw; i += blockDim.x)
         reinterpret_cast<volatile unsigned long long*>(host_mapped)[i] = reinterpret_cast<const unsigned long long*>(c)[i];
 }
+__global__ void k_store_words(const unsigned long long* __restrict__ src, int n, unsigned long long* host_mapped) {
+    for (int i = threadIdx.x; i < n; i += blockDim.x) reinterpret_cast<volatile unsigned long long*>(host_mapped)[i] = src[i];
+}
 __global__ void k_init_counters(Counters* c) {  // zero, with the two minima at their identity
     constexpr int nw = sizeof(Counters) / 8;
     static_assert(sizeof(Counters) % 8 == 0, "Counters is zeroed in 8-byte words");
     for (int i = threadIdx.x; i < nw; i += blockDim.x) reinterpret_cast<unsigned long long*>(c)[i] = 0;
     __syncwarp();
-    if (threadIdx.x == 0) { c->ts_min = ~0ull; c->v_min = ~0ull; }
+    if (threadIdx.x == 0) { c->ts_min = ~0ull; c->v_min = ~0ull; c->first_pend = ~0ull; }
 }
 
 // owned external-ID range of a shard: [lo, hi), hi == ~0 means "through UINT64_MAX"
@@ -495,8 +498,11 @@ __global__ void k_rec_expand(const DeltaRec* __restrict__ rec, uint64_t n, const
 // after a successful cycle from a delta store: every record the scan used is marked
 // invalid ("by the end of the delta store scan"; each delta is used once,
 // P:L615-619); first_pending = lowest index of a still-valid (not yet visible) record
-__global__ void k_rec_consume(DeltaRec* __restrict__ rec, uint64_t n, uint64_t vis_ts,
-                              unsigned long long* __restrict__ first_pending) {
+__global__ void k_rec_consume(DeltaRec* __restrict__ rec, uint64_t n, uint64_t vis_ts, Counters* __restrict__ c,
+                              unsigned long long fail_mask) {
+    // runs behind the cycle's last kernel, before its read-back: a cycle whose status carries
+    // an error bit marks nothing (the host then reports the error and keeps every delta)
+    if (c->status & fail_mask) return;
     const uint64_t i = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x;
     bool pend = false;
     if (i < n && rec[i].valid) {
@@ -504,7 +510,7 @@ __global__ void k_rec_consume(DeltaRec* __restrict__ rec, uint64_t n, uint64_t v
         else pend = true;
     }
     const uint32_t m = __ballot_sync(0xffffffffu, pend);   // the warp's lowest pending index
-    if (m && lane_id() == (uint32_t)(__ffs(m) - 1)) atomicMin(first_pending, (unsigned long long)i);
+    if (m && lane_id() == (uint32_t)(__ffs(m) - 1)) atomicMin(&c->first_pend, (unsigned long long)i);
 }
 
 // ===================================================================== a2 ====

@@ -65,6 +65,7 @@ def test_fig2_two_cycles_and_validity(h2):
     assert ids.tolist() == ex["ext_ids"] and cols.tolist() == ex["cols"] and w.tolist() == ex["weights"]
     st = cycle(g, store, o, model, 30, "empty")
     assert st["n_visible"] == 0
+    store.join()                      # no copy outstanding: returns at once
     store.close()
 
 

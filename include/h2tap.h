@@ -112,7 +112,7 @@ typedef struct {
 typedef struct {
     int device;                  /* CUDA device ordinal */
     int rank, world;             /* world == 1 for a single replica */
-    const void* nccl_unique_id;  /* ncclUniqueId bytes (collective mode), else NULL */
+    const void* nccl_unique_id;  /* ncclUniqueId bytes (collective mode, see below), else NULL */
     const uint64_t* shard_bounds;/* world + 1 non-decreasing external-ID split points (host),
                                     NULL if world == 1; world <= 4096, else H2TAP_E_INVAL */
     uint64_t expected_batch;     /* capacity hint (ops per batch); 0 = none */
@@ -265,6 +265,32 @@ typedef struct {
     uint8_t kind;
     uint8_t pad[3];
 } h2tap_route_rec;
+
+/* ---- collective mode ("every multi-GPU call is collective"; north_star:
+ * ops routed to the owner of their source with an NCCL all-to-all, global offsets from
+ * all-gathered per-shard counts).  A replica created with cfg.nccl_unique_id != NULL (the
+ * same 128-byte id on every rank, from h2tap_nccl_unique_id on one rank; world >= 1,
+ * shard_bounds may be NULL when world == 1) owns an NCCL communicator; creating it is
+ * collective.  On such a replica:
+ *   h2tap_delta_apply(slice, snapshot_ts): every rank passes ITS slice of the global batch
+ *     (rank-major arrival order, reading A5; host or device) and the same snapshot_ts.  Inside:
+ *     validation + destination counts, one ncclAllGather (host round trip 1: any rank's bad
+ *     slice -> every rank returns the same E_INVAL / E_STALE_TS, nothing applied), the
+ *     route records exchanged with grouped ncclSend/ncclRecv, the cycle prepared in the back
+ *     buffers, one ncclAllGather of the prepare statuses and shard edge counts (round trip 2):
+ *     every rank commits, or every rank aborts and returns the lowest (worst) status.
+ *     h2tap_replica_info's ebase is then the shard's first global edge.  Prepare / async are
+ *     refused (E_INVAL) on a collective replica: the call agrees and swaps itself.
+ *   h2tap_bfs / h2tap_sssp / h2tap_pagerank: collective; the per-shard kernels plus one
+ *     ncclAllReduce per step (MAX of the u8 frontier marks, SUM of the PageRank
+ *     contributions and dangling mass, MIN of the fp64 distances); results are global
+ *     (V entries, dense order) on every rank.
+ * NCCL is loaded at run time (dlopen libnccl.so.2); unavailable -> E_INVAL at create.
+ * A failure inside an NCCL call is E_NCCL. */
+h2tap_status h2tap_nccl_unique_id(void* id_out /* >= 128 bytes */, size_t cap);
+/* global arrival number of the next slice base; route bytes this rank sent to other
+ * ranks in the last collective apply (40 B per record).  E_INVAL without a communicator. */
+h2tap_status h2tap_collective_stats(const h2tap_replica* r, uint64_t* global_seq, uint64_t* route_bytes);
 
 /* E_INVAL (unknown kind) / E_STALE_TS (ts <= snapshot) / OK for a batch slice. */
 h2tap_status h2tap_batch_validate(const h2tap_replica* r, const h2tap_batch* batch);

@@ -293,6 +293,16 @@ def _close_live():
         r.close()
 
 
+NCCL_ID_BYTES = 128  # sizeof(ncclUniqueId)
+
+
+def nccl_unique_id() -> bytes:
+    """h2tap_nccl_unique_id: a fresh NCCL id (call on one rank, broadcast the bytes)"""
+    buf = ctypes.create_string_buffer(NCCL_ID_BYTES)
+    _check(_lib.h2tap_nccl_unique_id(buf, NCCL_ID_BYTES), "h2tap_nccl_unique_id")
+    return buf.raw
+
+
 class Replica:
     """A CSR replica in device memory (opaque h2tap_replica*)."""
 
@@ -303,13 +313,18 @@ class Replica:
 
     # ---------------------------------------------------------------- create
     @staticmethod
-    def _config(device, stream, torch_allocator, rank=0, world=1, shard_bounds=None, tombstone=False):
+    def _config(device, stream, torch_allocator, rank=0, world=1, shard_bounds=None, tombstone=False,
+                nccl_id=None):
         cfg = _Config()
         cfg.device = device
         cfg.id_mode = 1 if tombstone else 0  # H2TAP_ID_TOMBSTONE / H2TAP_ID_COMPACT
         cfg.rank, cfg.world = rank, world
         keep = []
-        if world > 1:
+        if nccl_id is not None:  # collective mode: the library owns an NCCL communicator
+            idb = ctypes.create_string_buffer(bytes(nccl_id), NCCL_ID_BYTES)
+            cfg.nccl_unique_id = ctypes.cast(idb, ctypes.c_void_p)
+            keep.append(idb)
+        if world > 1 or (nccl_id is not None and shard_bounds is not None):
             sb = np.ascontiguousarray(shard_bounds, dtype=np.uint64)
             if sb.shape != (world + 1,):
                 raise ValueError("shard_bounds must have world + 1 entries")
@@ -330,10 +345,14 @@ class Replica:
 
     @classmethod
     def from_edges(cls, n_vertices, vertex_ids, src, dst, w, create_ts=0, device=0, stream=None,
-                   torch_allocator=True, rank=0, world=1, shard_bounds=None, tombstone=False) -> "Replica":
+                   torch_allocator=True, rank=0, world=1, shard_bounds=None, tombstone=False,
+                   nccl_id=None) -> "Replica":
         """Create a replica (world > 1: shard `rank` of a vertex-range sharded graph; pass
-        the GLOBAL vertex set and only the edges whose source this shard owns)."""
-        cfg, keep = cls._config(device, stream, torch_allocator, rank, world, shard_bounds, tombstone)
+        the GLOBAL vertex set and only the edges whose source this shard owns).  nccl_id
+        (bytes from nccl_unique_id() on one rank, the same on every rank): collective mode -
+        apply() takes this rank's slice of the global batch and routes / agrees inside the
+        library; bfs / sssp / pagerank are collective (include/h2tap.h)."""
+        cfg, keep = cls._config(device, stream, torch_allocator, rank, world, shard_bounds, tombstone, nccl_id)
         pi, ps, pd, pw = (_ptr(vertex_ids, np.uint64), _ptr(src, np.uint64), _ptr(dst, np.uint64),
                           _ptr(w, np.float32))
         ond = _on_device(pi, ps, pd, pw)
@@ -484,6 +503,12 @@ class Replica:
             _check(rc, "h2tap_delta_apply_store")
             return st.as_dict()
         return rc, st.as_dict()
+
+    def collective_stats(self):
+        """h2tap_collective_stats: {global_seq, route_bytes} of a collective-mode replica"""
+        a, b = _u64(), _u64()
+        _check(_lib.h2tap_collective_stats(self._h, ctypes.byref(a), ctypes.byref(b)), "h2tap_collective_stats")
+        return dict(global_seq=a.value, route_bytes=b.value)
 
     # ------------------------------------------------------------- read back
     def info(self):

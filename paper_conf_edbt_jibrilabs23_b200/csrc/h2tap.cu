@@ -197,6 +197,7 @@ struct h2tap_replica {
         if (prep.node_mode) {
             ext_cur = prep.ext_new;
             identity = prep.identity;
+            idmap_swapped();
         }
         V = prep.V;
         E = prep.E;
@@ -208,6 +209,13 @@ struct h2tap_replica {
         snap = prep.S;
         prep.on = false;
     }
+    // collective mode (library-owned NCCL communicator, csrc/collective.cuh)
+    void* comm = nullptr;                 // ncclComm_t
+    Buf coll, coll_send, coll_recv;       // gather words, route records out / in
+    uint64_t coll_seq = 0;                // global arrival number of the next slice base
+    uint64_t edge_base = 0;               // first global edge of this shard
+    uint64_t last_route_bytes = 0;        // records sent to other ranks by the last apply
+    Buf idsame;         // 2 words: back ID-map buffer == front on [0, [0]); [1] = [0] after the swap
     Buf casc_status;    // look-back words of the cascade scan (runs beside the edge-op phase)
     Buf live[2];        // tombstone mode: u8 liveness per dense id, double-buffered with ext
     Buf ctr;
@@ -255,6 +263,11 @@ struct h2tap_replica {
         return static_cast<T*>(b.p);
     }
     void release(Buf& b) { dfree(b.p); b.p = nullptr; b.cap = 0; }
+    // the two ID-map buffers traded places: they now hold consecutive snapshots
+    void idmap_swapped() {
+        k_idmap_commit<<<1, 1, 0, st>>>(get<unsigned long long>(idsame, 2));
+        CK(cudaGetLastError());
+    }
     void sync() { CK(cudaStreamSynchronize(st)); }
     bool identity_pending = false;  // identity flag of the ext buffer being built
     bool identity_of(int which) const { return which == ext_cur ? identity : identity_pending; }
@@ -270,6 +283,15 @@ struct h2tap_replica {
     template <typename T>
     void zero(Buf& b, uint64_t count) { CK(cudaMemsetAsync(b.p, 0, count * sizeof(T), st)); }
 };
+
+namespace coll {  // csrc/collective.cuh
+void init_comm(h2tap_replica* r);
+void destroy_comm(h2tap_replica* r);
+h2tap_status apply(h2tap_replica* r, const h2tap_batch* b, uint64_t S, h2tap_apply_stats* stats);
+h2tap_status bfs(h2tap_replica* r, uint64_t source_ext, int32_t* level_out, int on_device);
+h2tap_status pagerank(h2tap_replica* r, double damping, int iterations, double* rank_out, int on_device);
+h2tap_status sssp(h2tap_replica* r, uint64_t source_ext, double* dist_out, int on_device);
+}  // namespace coll
 
 namespace {
 
@@ -408,6 +430,9 @@ ExtIndex ext_index(h2tap_replica* r) {
 #ifndef H2TAP_MERGE_CTAS
 #define H2TAP_MERGE_CTAS 0
 #endif
+#ifndef H2TAP_IDMAP_KEEP
+#define H2TAP_IDMAP_KEEP 1  // node mode: leave the ID-map prefix both buffers already share
+#endif
 #ifndef H2TAP_CASC_CTAS
 #define H2TAP_CASC_CTAS 4
 #endif
@@ -441,7 +466,7 @@ void finalize_inflight(h2tap_replica* r) {
     st.ms_degree_scan = ev_ms(f.ev[3], f.ev[6]) + ev_ms(f.ev[4], f.ev[5]);
     st.ms_total = ev_ms(f.ev[0], f.ev[5]);
     uint64_t b = 8 * (f.Vr + 1) + 8 * f.E + 8 * (fc.Vr_new + 1) + 8 * fc.En + 29 * f.n;
-    if (f.node_mode) b += 16 * f.V + 4 * f.E + 4 * f.V;
+    if (f.node_mode) b += 16 * (f.V - fc.idmap_keep) + 4 * f.E + 4 * f.V;
     st.bytes_alg = b;
     uint64_t bm = 0;
     if (f.csr_changed && f.E + fc.n_ins) {
@@ -639,6 +664,7 @@ h2tap_status apply_core(h2tap_replica* r, const BatchIn& in, uint64_t S, bool cr
     uint32_t *dropped = nullptr, *ins_q = nullptr, *ins_oldpos = nullptr, *hd_rows = nullptr,
              *hd_bits = nullptr, *node_sorted = nullptr;
     uint64_t* new_ext = nullptr;
+    unsigned long long* idsame = nullptr;
     uint32_t* casc_mask = nullptr;
     bool casc_pending = false;  // cascade pass in flight on the side stream
     uint64_t *casc_cnt = nullptr, *casc_pre = nullptr;
@@ -692,7 +718,10 @@ h2tap_status apply_core(h2tap_replica* r, const BatchIn& in, uint64_t S, bool cr
         TR("node_lists");
         // ID-map compaction: remap tables (64K-id block shifts, 32-id groups, the
         // unchanged / uniformly shifted id ranges), then the survivors and the inserted
+        const size_t ext_cap = r->ext[ec ^ 1].cap;  // a regrow (even at the same address) zeroes it
         new_ext = r->get<uint64_t>(r->ext[ec ^ 1], Vn_ub);
+        idsame = r->get<unsigned long long>(r->idsame, 2);
+        if (r->ext[ec ^ 1].cap != ext_cap) CK(cudaMemsetAsync(idsame, 0, 16, st));  // fresh back buffer
         const uint64_t nblk = cdiv(V, 1ull << kRemapBlockShift), ng = cdiv(V, 32);
         int32_t* rs = r->get<int32_t>(r->remap_shift, nblk + 8);  // + lohi (6 entries)
         uint2* r32 = r->get<uint2>(r->remap32, ng);
@@ -901,6 +930,7 @@ h2tap_status apply_core(h2tap_replica* r, const BatchIn& in, uint64_t S, bool cr
         ra.new_off = new_off;
         ra.c = dc;
         ra.old_ext = old_ext; ra.new_ext = new_ext; ra.identity = r->identity ? 1 : 0;
+        ra.same = H2TAP_IDMAP_KEEP ? idsame : nullptr;
         uint8_t* new_live = nullptr;
         if (r->tomb) {
             ra.old_live = static_cast<const uint8_t*>(r->live[ec].p);
@@ -920,6 +950,10 @@ h2tap_status apply_core(h2tap_replica* r, const BatchIn& in, uint64_t S, bool cr
         if (V) {
             k_rows_fused<<<(unsigned)ncta, kThreads, 0, st>>>(ra);  // survivors: ID map + row offsets
             CKL();
+            k_idmap_mark<<<1, 1, 0, st>>>(idsame, R.lohi, dc, (r->tomb || !H2TAP_IDMAP_KEEP) ? 1 : 0);
+            CKL();
+        } else {
+            CK(cudaMemsetAsync(idsame, 0, 16, st));
         }
         k_offsets_inserted<<<g1(n_node), 256, 0, st>>>(nv, ins_q, ra);
         CKL();
@@ -1016,7 +1050,7 @@ h2tap_status apply_core(h2tap_replica* r, const BatchIn& in, uint64_t S, bool cr
         f.launches = g_launches; f.h2d = g_h2d; f.d2h = g_d2h + sizeof(Counters);
         // the part of the swap that needs no counter (what the next cycle reads first)
         r->cur = nb;
-        if (node_mode) r->ext_cur = ec ^ 1;
+        if (node_mode) { r->ext_cur = ec ^ 1; r->idmap_swapped(); }
         r->pcur = pc ^ 1;
         r->n_pend = n_pend_new;
         r->next_seq += n;
@@ -1073,7 +1107,7 @@ h2tap_status apply_core(h2tap_replica* r, const BatchIn& in, uint64_t S, bool cr
         stats->ms_degree_scan = ev_ms(r->ev[3], r->ev[6]) + ev_ms(r->ev[4], r->ev[5]);
         stats->ms_total = ev_ms(r->ev[0], r->ev[5]);
         uint64_t b = 8 * (Vr + 1) + 8 * E + 8 * (Vr_new + 1) + 8 * En + 29 * n;
-        if (node_mode) b += 16 * V + 4 * E + 4 * V;
+        if (node_mode) b += 16 * (V - fc.idmap_keep) + 4 * E + 4 * V;
         stats->bytes_alg = b;
         // merge launch: stream old cols+weights, write new ones, read the outcome lists
         // (+ remap table and cascade bitmap when node ops changed the ID map)
@@ -1125,7 +1159,9 @@ h2tap_replica* new_replica(const h2tap_config* cfg) {
         set_err("tombstone-row mode is single-replica only in this build");
         throw Fail{H2TAP_E_INVAL};
     }
-    if (r->cfg.world > 1) {
+    static const uint64_t kOneShard[2] = {0, ~0ull};
+    if (r->cfg.nccl_unique_id && r->cfg.world == 1 && !r->cfg.shard_bounds) r->cfg.shard_bounds = kOneShard;
+    if (r->cfg.world > 1 || r->cfg.nccl_unique_id) {
         if (!r->cfg.shard_bounds || r->cfg.rank < 0 || r->cfg.rank >= r->cfg.world) {
             set_err("sharded replica needs shard_bounds[world+1] and 0 <= rank < world");
             throw Fail{H2TAP_E_INVAL};
@@ -1136,11 +1172,6 @@ h2tap_replica* new_replica(const h2tap_config* cfg) {
                 set_err("shard_bounds must be non-decreasing");
                 throw Fail{H2TAP_E_INVAL};
             }
-        if (r->cfg.nccl_unique_id) {
-            set_err("collective mode (NCCL communicator inside the library) is not in this build; "
-                    "use caller-routed sharding (nccl_unique_id = NULL)");
-            throw Fail{H2TAP_E_INVAL};
-        }
         r->sharded = true;
         uint64_t* bd = r->get<uint64_t>(r->bounds_dev, r->cfg.world + 1);
         CK(cudaMemcpy(bd, r->cfg.shard_bounds, (r->cfg.world + 1) * 8, cudaMemcpyHostToDevice));
@@ -1149,6 +1180,7 @@ h2tap_replica* new_replica(const h2tap_config* cfg) {
         r->cfg.shard_bounds = nullptr;  // not retained
     }
     CK(cudaSetDevice(r->cfg.device));
+    if (r->cfg.nccl_unique_id) coll::init_comm(r);  // collective: every rank creates its shard
     CK(cudaDeviceGetAttribute(&r->n_sm, cudaDevAttrMultiProcessorCount, r->cfg.device));
     r->st = static_cast<cudaStream_t>(r->cfg.stream);
     {   // side stream at the lowest priority: its streaming work fills gaps left by the
@@ -1178,6 +1210,7 @@ h2tap_replica* new_replica(const h2tap_config* cfg) {
 
 void free_replica(h2tap_replica* r) {
     if (!r) return;
+    if (r->comm) coll::destroy_comm(r);
     Buf* bufs[] = {&r->off[0], &r->off[1], &r->cols[0], &r->cols[1], &r->w[0], &r->w[1], &r->ext[0], &r->ext[1],
                    &r->pk[0], &r->pk[1], &r->ps[0], &r->ps[1], &r->pd[0], &r->pd[1], &r->pw[0], &r->pw[1],
                    &r->pt[0], &r->pt[1], &r->pq[0], &r->pq[1], &r->Wk, &r->Ws, &r->Wd, &r->Ww, &r->Wt, &r->Wq,
@@ -1186,7 +1219,7 @@ void free_replica(h2tap_replica* r) {
                    &r->ins_oldpos, &r->hd_rows, &r->hd_bits, &r->op_flags, &r->op_ou, &r->op_ow,
                    &r->ins_pos, &r->ins_row, &r->ins_col, &r->ins_w, &r->del_pos, &r->upd_pos, &r->upd_w,
                    &r->KR, &r->cls_cat, &r->cls_pos, &r->cls_w, &r->misc, &r->nsorted, &r->part, &r->opart, &r->deg, &r->tsum, &r->remap_shift, &r->remap32, &r->casc_wrel, &r->tile_emit, &r->tile_base, &r->del_row, &r->casc_mask, &r->status2, &r->bounds_dev, &r->fence[0], &r->fence[1], &r->bfs_a, &r->bfs_b, &r->pr_a, &r->pr_b, &r->ctr,
-                   &r->xrec, &r->xins, &r->xwts, &r->xdel, &r->xcnt, &r->xoff, &r->xbig, &r->xnbig, &r->live[0], &r->live[1], &r->casc_status};
+                   &r->xrec, &r->xins, &r->xwts, &r->xdel, &r->xcnt, &r->xoff, &r->xbig, &r->xnbig, &r->live[0], &r->live[1], &r->casc_status, &r->idsame, &r->coll, &r->coll_send, &r->coll_recv};
     for (Buf* b : bufs) if (b->p) r->dfree(b->p);
     cudaStreamSynchronize(r->st);
     for (auto& e : r->ev) if (e) cudaEventDestroy(e);
@@ -1214,6 +1247,7 @@ void init_vertices(h2tap_replica* r, uint64_t nv, const uint64_t* ids, int on_de
     r->V = nv;
     r->E = 0;
     uint64_t* ext = r->get<uint64_t>(r->ext[0], nv);
+    CK(cudaMemsetAsync(r->get<unsigned long long>(r->idsame, 2), 0, 16, r->st));  // back buffer unknown
     if (ids) copy_in(r, ext, ids, nv, on_device);
     else if (nv) { k_iota_u64<<<g1(nv), 256, 0, r->st>>>(ext, nv); CKL(); }
     int64_t* off = r->get<int64_t>(r->off[0], nv + 1);
@@ -1374,6 +1408,10 @@ h2tap_status h2tap_delta_apply(h2tap_replica* r, const h2tap_batch* b, uint64_t 
             return H2TAP_E_SNAPSHOT_REGRESSION;
         }
         CK(cudaSetDevice(r->cfg.device));
+        if (r->comm) {  // collective: every rank calls; the swap is agreed inside
+            if (r->defer_commit) { set_err("collective replica: apply agrees and commits itself (no prepare)"); return H2TAP_E_INVAL; }
+            return coll::apply(r, b, snapshot_ts, stats);
+        }
         BatchIn in{b->n, b->on_device, b->seq, b->kind, b->src, b->dst, b->weight, b->ts, 0};
         h2tap_replica::Stage* used = nullptr;
         for (auto& g : r->stg)  // a batch staged by h2tap_batch_stage: its copy is ordered first
@@ -1826,7 +1864,7 @@ h2tap_status h2tap_replica_info(const h2tap_replica* r, uint64_t* nv, uint64_t* 
     if (snap) *snap = r->snap;
     if (npend) *npend = r->n_pend;
     if (vbase) *vbase = r->row_lo;
-    if (ebase) *ebase = 0;  // caller-routed sharding: the caller sums the shards' edge counts
+    if (ebase) *ebase = r->edge_base;  // collective mode; 0 when the caller routes (it sums the shards)
     return H2TAP_OK;
 }
 
@@ -1887,10 +1925,11 @@ static uint64_t dense_of(h2tap_replica* r, uint64_t x_ext) {
 h2tap_status h2tap_bfs(const h2tap_replica* rc, uint64_t source_ext, int32_t* level_out, int on_device) {
     h2tap_replica* r = const_cast<h2tap_replica*>(rc);
     if (!r || !level_out) { set_err("null argument"); return H2TAP_E_INVAL; }
-    if (r->sharded) { set_err("h2tap_bfs: not available on a sharded replica in this build"); return H2TAP_E_INVAL; }
+    if (r->sharded && !r->comm) { set_err("h2tap_bfs: caller-routed sharded replica (use the shard steps)"); return H2TAP_E_INVAL; }
     return run_guarded(r, [&]() -> h2tap_status {
         ensure_final(r);
         CK(cudaSetDevice(r->cfg.device));
+        if (r->comm) return coll::bfs(r, source_ext, level_out, on_device);
         const uint64_t V = r->V;
         const uint64_t src = dense_of(r, source_ext);
         if (src >= V) { set_err("BFS source %llu is not a live vertex", (unsigned long long)source_ext); return H2TAP_E_INVAL; }
@@ -1927,10 +1966,11 @@ h2tap_status h2tap_bfs(const h2tap_replica* rc, uint64_t source_ext, int32_t* le
 h2tap_status h2tap_sssp(const h2tap_replica* rc, uint64_t source_ext, double* dist_out, int on_device) {
     h2tap_replica* r = const_cast<h2tap_replica*>(rc);
     if (!r || !dist_out) { set_err("null argument"); return H2TAP_E_INVAL; }
-    if (r->sharded) { set_err("h2tap_sssp: not available on a sharded replica in this build"); return H2TAP_E_INVAL; }
+    if (r->sharded && !r->comm) { set_err("h2tap_sssp: caller-routed sharded replica (use the shard steps)"); return H2TAP_E_INVAL; }
     return run_guarded(r, [&]() -> h2tap_status {
         ensure_final(r);
         CK(cudaSetDevice(r->cfg.device));
+        if (r->comm) return coll::sssp(r, source_ext, dist_out, on_device);
         const uint64_t V = r->V, E = r->E;
         const uint64_t src = dense_of(r, source_ext);
         if (src >= V) { set_err("SSSP source %llu is not a live vertex", (unsigned long long)source_ext); return H2TAP_E_INVAL; }
@@ -1994,6 +2034,30 @@ unsigned warp_grid(h2tap_replica* r, uint64_t rows) {
     return (unsigned)std::max<uint64_t>(1, std::min<uint64_t>(cdiv(rows * 32, 256), (uint64_t)r->n_sm * 32));
 }
 }  // namespace
+}  // extern "C"
+
+#include "collective.cuh"
+
+extern "C" {
+
+h2tap_status h2tap_nccl_unique_id(void* id_out, size_t cap) {
+    if (!id_out || cap < sizeof(ncclUniqueId)) { set_err("h2tap_nccl_unique_id: need %zu bytes", sizeof(ncclUniqueId)); return H2TAP_E_INVAL; }
+    const coll::Api* A = coll::api();
+    if (!A) return H2TAP_E_INVAL;
+    ncclUniqueId id;
+    const ncclResult_t e = A->GetUniqueId(&id);
+    if (e != ncclSuccess) { set_err("ncclGetUniqueId: %s", A->GetErrorString(e)); return H2TAP_E_CUDA; }
+    std::memcpy(id_out, &id, sizeof id);
+    return H2TAP_OK;
+}
+
+h2tap_status h2tap_collective_stats(const h2tap_replica* r, uint64_t* global_seq, uint64_t* route_bytes) {
+    if (!r) { set_err("null replica"); return H2TAP_E_INVAL; }
+    if (!r->comm) { set_err("replica has no communicator (collective mode off)"); return H2TAP_E_INVAL; }
+    if (global_seq) *global_seq = r->coll_seq;
+    if (route_bytes) *route_bytes = r->last_route_bytes;
+    return H2TAP_OK;
+}
 
 h2tap_status h2tap_replica_lookup(const h2tap_replica* rc, uint64_t ext_id, uint64_t* dense_out) {
     h2tap_replica* r = const_cast<h2tap_replica*>(rc);
@@ -2139,10 +2203,11 @@ h2tap_status h2tap_replica_liveness(const h2tap_replica* rc, uint8_t* live_out, 
 h2tap_status h2tap_pagerank(const h2tap_replica* rc, double damping, int iterations, double* rank_out, int on_device) {
     h2tap_replica* r = const_cast<h2tap_replica*>(rc);
     if (!r || !rank_out || iterations < 0) { set_err("bad argument"); return H2TAP_E_INVAL; }
-    if (r->sharded) { set_err("h2tap_pagerank: not available on a sharded replica in this build"); return H2TAP_E_INVAL; }
+    if (r->sharded && !r->comm) { set_err("h2tap_pagerank: caller-routed sharded replica (use the shard steps)"); return H2TAP_E_INVAL; }
     return run_guarded(r, [&]() -> h2tap_status {
         ensure_final(r);
         CK(cudaSetDevice(r->cfg.device));
+        if (r->comm) return coll::pagerank(r, damping, iterations, rank_out, on_device);
         const uint64_t V = r->V;
         if (V == 0) return H2TAP_OK;
         double* a = r->get<double>(r->pr_a, V);

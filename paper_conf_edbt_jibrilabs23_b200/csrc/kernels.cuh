@@ -41,6 +41,8 @@ struct Counters {
     unsigned long long Vn, Vr_new, En, new_identity;  // written by k_finish
     unsigned long long n_killed;  // vertices live before the cycle and dead after it (stats)
     unsigned long long first_pend;  // delta-store scan: first record left valid (k_rec_consume)
+    unsigned long long idmap_lo;    // node mode: ids below it keep their id and external id
+    unsigned long long idmap_keep;  // node mode: ID-map prefix the survivor pass did not rewrite
     unsigned int tiles[16];
 };
 
@@ -1423,6 +1425,7 @@ struct RowArgs {
     int identity;
     const uint8_t* old_live;  // tombstone mode: liveness carried to the new slots
     uint8_t* new_live;
+    const unsigned long long* same;  // back ID-map buffer == front on [0, *same) (nullptr: unknown)
 };
 __device__ __forceinline__ RowArgs row_counts(RowArgs a) {
     a.n_del = a.c->n_del;
@@ -1475,10 +1478,13 @@ __global__ void __launch_bounds__(kThreads, H2TAP_ROWS_MINB) k_rows_fused(RowArg
     const uint64_t k0 = (uint64_t)blockIdx.x * kRowTile, k1 = min(k0 + kRowTile, a.V_old);
     const uint64_t* pp = a.part + 2 * blockIdx.x;  // this CTA's slices of the delete / insert-row lists
     const uint64_t da = pp[0], ia = pp[1], db = pp[2], ib = pp[3];
+    // ID-map prefix already in place: ids below R.lohi[0] keep their dense id (u = k) and
+    // external id, and the back buffer equals the front one on [0, *same)
+    const uint64_t keep = (a.same && !a.new_live) ? min((uint64_t)*a.same, (uint64_t)(uint32_t)a.R.lohi[0]) : 0;
     constexpr int PER = kRowTile / kThreads;  // ids per thread, all loads issued together
     uint32_t u[PER];
     uint64_t x[PER], ext[PER];
-    bool row[PER];
+    bool row[PER], wext[PER];
 #pragma unroll
     for (int j = 0; j < PER; ++j) {
         const uint64_t k = k0 + threadIdx.x + (uint64_t)j * kThreads;
@@ -1486,9 +1492,10 @@ __global__ void __launch_bounds__(kThreads, H2TAP_ROWS_MINB) k_rows_fused(RowArg
         x[j] = 0;
         ext[j] = k;
         row[j] = false;
+        wext[j] = k >= keep;
         if (k < k1) {
             u[j] = remap_of(a.R, (uint32_t)k);
-            if (!a.identity) ext[j] = a.old_ext[k];
+            if (!a.identity && wext[j]) ext[j] = a.old_ext[k];
             if (a.new_live && u[j] != kNone32) a.new_live[u[j]] = a.old_live[k];
             row[j] = k >= a.row_lo && k < a.row_hi;
             if (row[j]) x[j] = (uint64_t)a.old_off[k];
@@ -1500,12 +1507,25 @@ __global__ void __launch_bounds__(kThreads, H2TAP_ROWS_MINB) k_rows_fused(RowArg
 #pragma unroll
     for (int j = 0; j < PER; ++j) {
         if (u[j] == kNone32) continue;
-        a.new_ext[u[j]] = ext[j];
+        if (wext[j]) a.new_ext[u[j]] = ext[j];
         if (!row[j]) continue;
         const uint64_t kept = x[j] - cb[j] - lower_bound_dev(a.del_pos, da, db, x[j]);
         a.new_off[u[j] - a.row_lo_new] = (int64_t)(kept + lower_bound_dev(a.ins_row, ia, ib, u[j]));
     }
 }
+
+// ID-map prefix bookkeeping (node mode).  *same: the back ID-map buffer equals the front
+// one on [0, *same).  The survivor pass rewrote the back buffer from min(*same, lo) on, so
+// it now equals the front one only below that (what an abort leaves); after the swap the
+// two buffers hold consecutive snapshots, equal below this cycle's lo.
+__global__ void k_idmap_mark(unsigned long long* same, const int32_t* __restrict__ lohi, Counters* c, int tomb) {
+    const unsigned long long lo = (unsigned long long)(uint32_t)lohi[0];
+    c->idmap_lo = lo;
+    c->idmap_keep = tomb ? 0ull : min(same[0], lo);
+    same[0] = min(same[0], lo);
+    same[1] = lo;  // what the swap makes of same[0]
+}
+__global__ void k_idmap_commit(unsigned long long* same) { same[0] = same[1]; }
 
 // Row offsets without node ops (a4/a5; identity remap, no cascade): the exclusive
 // scan of the per-row degree delta at row k is a difference of two ranks in the

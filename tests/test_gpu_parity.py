@@ -431,3 +431,61 @@ def test_pending_export_and_checkpoint_restore(h2):
     g.apply(b, last)
     h.apply(b, last)
     assert_same(h.export(), g.export(), "restored checkpoint")
+
+
+def test_idmap_prefix_reuse_across_cycles(h2):
+    """Node-mode cycles leave the ID-map prefix the two buffers already share:
+    node ops alternate between the top, the bottom and the middle of the id space, prepared
+    cycles are aborted in between (the back buffer then holds a partial rewrite), and the
+    asynchronous path swaps buffers without a host read-back - the ID map and the CSR stay
+    bit-exact with O1 after every cycle."""
+    n = 1 << 12
+    src, dst, w = synth.rmat_edges(12, 11, n=8 * n)
+    ids = np.arange(n, dtype=np.uint64) * 4 + 100          # gaps: new ids fit anywhere
+    g, o = pair_from_edges(h2, n, ids, ids[src], ids[dst], w)
+    rng = np.random.default_rng(5)
+    live = set(int(x) for x in ids)
+    ts = 0
+
+    def batch(lo_frac, hi_frac, k):
+        nonlocal ts
+        ops = []
+        cand = sorted(x for x in live if lo_frac * 4 * n <= x - 100 < hi_frac * 4 * n)
+        for v in rng.choice(cand, size=min(6, len(cand)), replace=False):
+            ts += 1
+            ops.append((NODE_DELETE, int(v), 0, 0.0, ts))
+            live.discard(int(v))
+        for j in range(5):   # new ids inside the region (odd offsets: never an old id)
+            v = 100 + int(rng.integers(int(lo_frac * 4 * n), int(hi_frac * 4 * n))) | 1
+            if v in live:
+                continue
+            ts += 1
+            ops.append((NODE_INSERT, v, 0, 0.0, ts))
+            live.add(v)
+            u = int(rng.choice(sorted(live)))
+            ops.append((EDGE_INSERT, v, u, float(j), ts))
+            ops.append((EDGE_INSERT, u, v, float(k), ts))
+        for _ in range(40):  # edge ops over the whole graph
+            ts += 1
+            a, b = (int(x) for x in rng.choice(sorted(live), 2))
+            ops.append((EDGE_INSERT if rng.random() < 0.7 else EDGE_DELETE, a, b, float(rng.random()), ts))
+        return Batch.of(ops)
+
+    regions = [(0.9, 1.0), (0.0, 0.1), (0.45, 0.55), (0.95, 1.0), (0.95, 1.0), (0.0, 0.05)]
+    for k, (lo, hi) in enumerate(regions):
+        if k % 2 == 1:  # a prepared cycle that is thrown away (its ops never happened)
+            saved_live, saved_ts = set(live), ts
+            bad = batch(0.0, 1.0, 100 + k)
+            rc, _ = g.prepare(bad, ts)
+            assert rc == 0
+            g.abort()
+            live, ts = saved_live, saved_ts
+        b = batch(lo, hi, k)
+        step(g, o, b, ts, f"region {lo}-{hi} cycle {k}")
+    # asynchronous cycles: the swap is enqueued, the next cycle reads the ID map it left
+    for k, (lo, hi) in enumerate(regions[:4]):
+        b = batch(lo, hi, 50 + k)
+        g.apply_async(b, ts)
+        o.apply(b, ts)
+    g.sync()
+    assert_same(g.export(), o.export(), "async node-mode cycles")

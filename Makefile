@@ -11,7 +11,7 @@ NVFLAGS := -gencode arch=compute_100a,code=sm_100a -O3 -lineinfo -std=c++17 \
 all: lib oracle synth
 
 lib: $(PKG)/libh2tap.so
-$(PKG)/libh2tap.so: $(CSRC)/h2tap.cu $(CSRC)/kernels.cuh $(CSRC)/radix_sort.cuh $(CSRC)/dev_common.cuh $(CSRC)/dyn.cuh $(CSRC)/delta_store.cuh include/h2tap.h
+$(PKG)/libh2tap.so: $(CSRC)/h2tap.cu $(CSRC)/kernels.cuh $(CSRC)/radix_sort.cuh $(CSRC)/dev_common.cuh $(CSRC)/dyn.cuh $(CSRC)/delta_store.cuh $(CSRC)/collective.cuh include/h2tap.h
 	$(NVCC) $(NVFLAGS) -o $@ $(CSRC)/h2tap.cu 2> $(CSRC)/ptxas.log || (cat $(CSRC)/ptxas.log; false)
 
 oracle: oracle/liboracle.so oracle/libo3.so

@@ -489,3 +489,27 @@ def test_idmap_prefix_reuse_across_cycles(h2):
         o.apply(b, ts)
     g.sync()
     assert_same(g.export(), o.export(), "async node-mode cycles")
+
+
+def test_sort_heavy_duplicate_keys(h2):
+    """The edge-key sort's sample-sort path puts equal keys in one bucket: a batch where one
+    (src, dst) pair carries 20K ops (a bucket far above the 8K a CTA sorts in shared memory,
+    so its chunked global-memory path runs) and another 9K, around 30K other ops, all with
+    interleaved timestamps - latest commit wins must still come out of a stable sort."""
+    n = 1 << 12
+    src, dst, w = synth.rmat_edges(12, 21, n=8 * n)
+    g, o = pair_from_edges(h2, n, None, src, dst, w)
+    rng = np.random.default_rng(9)
+    m = 60000
+    kind = rng.choice([EDGE_INSERT, EDGE_DELETE, EDGE_WEIGHT], size=m, p=[0.6, 0.2, 0.2]).astype(np.uint8)
+    s = rng.integers(0, n, m).astype(np.uint64)
+    d = rng.integers(0, n, m).astype(np.uint64)
+    s[:20000], d[:20000] = 7, 9            # one heavy key
+    s[20000:29000], d[20000:29000] = 4095, 0
+    perm = rng.permutation(m)
+    b = Batch(kind[perm], s[perm], d[perm], rng.random(m).astype(np.float32),
+              rng.integers(1, 5000, m).astype(np.uint64))
+    step(g, o, b, 5000, "heavy duplicate keys")
+    b2 = synth.rmat_batch(12, 21, 1, 30000, len(src))
+    b2.ts += 5000
+    step(g, o, b2, int(b2.ts.max()), "after heavy keys")

@@ -433,6 +433,9 @@ ExtIndex ext_index(h2tap_replica* r) {
 #ifndef H2TAP_IDMAP_KEEP
 #define H2TAP_IDMAP_KEEP 1  // node mode: leave the ID-map prefix both buffers already share
 #endif
+#ifndef H2TAP_CASC_TMA
+#define H2TAP_CASC_TMA 1  // cascade column pass streamed by TMA, one small CTA per SM
+#endif
 #ifndef H2TAP_CASC_CTAS
 #define H2TAP_CASC_CTAS 4
 #endif
@@ -727,7 +730,7 @@ h2tap_status apply_core(h2tap_replica* r, const BatchIn& in, uint64_t S, bool cr
         uint2* r32 = r->get<uint2>(r->remap32, ng);
         k_remap_blocks<<<g1(nblk), 256, 0, st>>>(V, dropped, ins_oldpos, dc, rs, rs + nblk);  // also writes c->Vn
         CKL();
-        if (ng) { k_remap32<<<g1(ng), 256, 0, st>>>(V, dropped, ins_oldpos, dc, r32); CKL(); }
+        if (ng) { k_remap32<<<g1(ng), 256, 0, st>>>(V, dropped, ins_oldpos, dc, rs + nblk, r32); CKL(); }
         R.shift = rs; R.g32 = r32; R.ins_oldpos = ins_oldpos; R.n_vins = &dc->n_inserted; R.lohi = rs + nblk;
         TR("remap_tables");
         // the inserted vertices' ID-map entries now; the survivors' entries are written
@@ -766,8 +769,15 @@ h2tap_status apply_core(h2tap_replica* r, const BatchIn& in, uint64_t S, bool cr
         CK(cudaStreamWaitEvent(r->st2, r->evA, 0));
         cudaStream_t cs = H2TAP_CASC_MAIN ? st : r->st2;
         if (nblk_c) {
-            const unsigned gc = (unsigned)std::min<uint64_t>(cdiv(nblk_c, 2), (uint64_t)r->n_sm * kCascCtasPerSm);
-            k_casc_cols<<<gc, kThreads, 0, cs>>>(old_cols_nc, E, hd_bits, hd_rows, dc, casc_mask);
+            if (H2TAP_CASC_TMA) {
+                static bool attr = false;
+                if (!attr) { CK(cudaFuncSetAttribute(k_casc_cols_tma, cudaFuncAttributeMaxDynamicSharedMemorySize, kCcSmem)); attr = true; }
+                const unsigned gc = (unsigned)std::min<uint64_t>(cdiv(E, kCcChunk), (uint64_t)r->n_sm);
+                k_casc_cols_tma<<<gc, kCcThreads, kCcSmem, cs>>>(old_cols_nc, E, hd_bits, hd_rows, dc, casc_mask);
+            } else {
+                const unsigned gc = (unsigned)std::min<uint64_t>(cdiv(nblk_c, 2), (uint64_t)r->n_sm * kCascCtasPerSm);
+                k_casc_cols<<<gc, kThreads, 0, cs>>>(old_cols_nc, E, hd_bits, hd_rows, dc, casc_mask);
+            }
             CKL();
             k_casc_rows<<<rg, 256, 0, cs>>>(old_off_nc, hd_rows, dc, row_lo, row_lo + Vr, casc_mask);
             CKL();

@@ -248,6 +248,9 @@ __device__ __forceinline__ uint64_t old_lookup(const ExtIndex& X, uint64_t x, bo
     uint64_t i = upper_bound_dev(X.fence, 0, X.nf, x);
     if (i == 0) { *present = false; return 0; }
     uint64_t lo = (i - 1) << kFenceShift, hi = min(lo + (uint64_t)(1u << kFenceShift), (uint64_t)X.V);
+    // a dense run of ids (ext[lo + d] = ext[lo] + d) answers with one probe
+    const uint64_t d = x - X.fence[i - 1];
+    if (d < hi - lo && X.ext[lo + d] == x) { *present = true; return lo + d; }
     uint64_t k = lower_bound_dev(X.ext, lo, hi, x);
     *present = (k < X.V && X.ext[k] == x);
     return k;
@@ -1330,6 +1333,94 @@ __global__ void __launch_bounds__(kThreads) k_casc_cols(const uint32_t* __restri
     }
 }
 
+// The same pass streamed with TMA: one CTA of 256 threads per SM, the columns arriving in
+// 32 KB bulk copies (2 buffers in flight per SM, ~9.5 MB across the GPU) signalled on
+// mbarriers, and the deleted-vertex bits of [hd_lo, hd_lo + span] copied into shared memory
+// when they fit (32 KB), so the pass runs near HBM speed while leaving 7/8 of every SM's
+// threads to the latency-bound edge-op kernels it overlaps.  Warp w turns kCcSub staged
+// columns into kCcSub / 32 mask words (lane-interleaved reads, one ballot per word) and
+// stores them with one coalesced store.
+constexpr int kCcChunk = 8192;                 // columns per bulk copy
+constexpr int kCcBuf = 2;
+#ifndef H2TAP_CC_THREADS
+#define H2TAP_CC_THREADS 256
+#endif
+constexpr int kCcThreads = H2TAP_CC_THREADS;
+constexpr int kCcSub = kCcChunk / (kCcThreads / 32);  // columns per warp per chunk (<= 1024)
+static_assert(kCcSub % 32 == 0 && kCcSub <= 1024, "a warp turns kCcSub columns into kCcSub / 32 mask words");
+constexpr int kCcHdWords = 8192;               // deleted-vertex bitmap window in shared memory
+constexpr int kCcSmem = kCcBuf * kCcChunk * 4 + kCcHdWords * 4;  // dynamic shared memory
+__global__ void __launch_bounds__(kCcThreads, 1) k_casc_cols_tma(const uint32_t* __restrict__ old_cols, uint64_t E,
+        const uint32_t* __restrict__ hd_bits, const uint32_t* __restrict__ hd_rows, const Counters* __restrict__ cn,
+        uint32_t* __restrict__ mask) {
+    extern __shared__ __align__(128) uint8_t cc_dsm[];
+    uint32_t* sb = reinterpret_cast<uint32_t*>(cc_dsm);
+    uint32_t* s_hd = sb + kCcBuf * kCcChunk;
+    __shared__ __align__(8) uint64_t bar[kCcBuf];
+    const uint64_t n_hd = cn->n_hd;
+    const uint32_t hd_lo = n_hd ? hd_rows[0] : 1u;
+    const uint32_t span = n_hd ? hd_rows[n_hd - 1] - hd_lo : 0u;
+    const uint64_t nch = (E + kCcChunk - 1) / kCcChunk;
+    const uint64_t wend = ((E + 31) >> 5) + 2 * kCascBlock / 32;  // mask words past E are written as 0
+    const int tid = threadIdx.x, w = tid >> 5;
+    const uint32_t lane = lane_id();
+    const uint64_t G = gridDim.x;
+    if (n_hd == 0) {  // no deleted vertex: an all-zero mask
+        for (uint64_t q = blockIdx.x * (uint64_t)kCcThreads + tid; q < wend; q += G * kCcThreads) mask[q] = 0u;
+        return;
+    }
+    auto issue = [&](uint64_t c, int b) {  // thread 0
+        const uint64_t c0 = c * kCcChunk;
+        const uint32_t nc = (uint32_t)min((uint64_t)kCcChunk, E - c0);
+        const uint32_t bytes = ((nc + 3) & ~3u) * 4;  // 16-byte multiple (the buffers have slack)
+        mbar_expect_tx(&bar[b], bytes);
+        bulk_g2s(sb + b * kCcChunk, old_cols + c0, bytes, &bar[b]);
+    };
+    if (tid == 0) {
+        for (int b = 0; b < kCcBuf; ++b) mbar_init(&bar[b], 1);
+        fence_mbar_init();
+        for (int b = 0; b < kCcBuf; ++b)
+            if (blockIdx.x + b * G < nch) issue(blockIdx.x + b * G, b);
+    }
+    // the bitmap words of ids hd_lo .. hd_lo + span (word-aligned window)
+    const uint32_t hw0 = hd_lo >> 5, hwn = ((hd_lo + span) >> 5) - hw0 + 1;
+    const bool hd_smem = hwn <= (uint32_t)kCcHdWords;
+    if (hd_smem)
+        for (uint32_t q = tid; q < hwn; q += kCcThreads) s_hd[q] = hd_bits[hw0 + q];
+    __syncthreads();
+    uint64_t i = 0;
+    for (uint64_t c = blockIdx.x; c < nch; c += G, ++i) {
+        const int b = (int)(i % kCcBuf);
+        mbar_wait(&bar[b], (uint32_t)((i / kCcBuf) & 1));
+        const uint32_t* s = sb + b * kCcChunk;
+        const uint64_t c0 = c * kCcChunk;
+        const uint32_t nc = (uint32_t)min((uint64_t)kCcChunk, E - c0);
+        {
+            const int sub = w;
+            uint32_t mine = 0;
+#pragma unroll 8
+            for (int q = 0; q < kCcSub / 32; ++q) {
+                const uint32_t j = sub * kCcSub + q * 32 + lane;
+                const uint32_t v = s[j], d = v - hd_lo;
+                bool hit = false;
+                if (j < nc && d <= span)
+                    hit = hd_smem ? (s_hd[(v >> 5) - hw0] >> (v & 31)) & 1u : (hd_bits[v >> 5] >> (v & 31)) & 1u;
+                const uint32_t word = __ballot_sync(0xffffffffu, hit);
+                if (lane == (uint32_t)q) mine = word;
+            }
+            const uint64_t q = ((c0 + sub * kCcSub) >> 5) + lane;
+            if (lane < kCcSub / 32 && q < wend) mask[q] = mine;
+        }
+        __syncthreads();  // buffer b fully consumed
+        if (tid == 0 && c + kCcBuf * G < nch) {
+            fence_proxy_async();
+            issue(c + kCcBuf * G, b);
+        }
+    }
+    if (blockIdx.x == 0)  // words past the last chunk
+        for (uint64_t q = nch * (kCcChunk / 32) + tid; q < wend; q += kCcThreads) mask[q] = 0u;
+}
+
 // rows of deleted vertices -> whole bit ranges (warp per row), OR-ed into the mask
 __global__ void k_casc_rows(const int64_t* __restrict__ old_off, const uint32_t* __restrict__ hd_rows,
                             const Counters* __restrict__ cn, uint64_t row_lo, uint64_t row_hi, uint32_t* __restrict__ mask) {
@@ -1981,14 +2072,20 @@ __global__ void k_offsets_inserted(const NodeVtx* __restrict__ nv, const uint32_
 }
 
 // per 32 old ids: {new id of the group's first id (as if it survived) | exact << 31,
-// dropped bitmask}; exact = an insertion point lies strictly inside the group
+// dropped bitmask}; exact = an insertion point lies strictly inside the group.  Only the
+// groups of the 64K-id blocks overlapping [lohi[0], lohi[1]) are written: every reader
+// (k_merge3's table path, remap_of on a mixed 64K block) looks up ids there only
 __global__ void k_remap32(uint64_t V, const uint32_t* __restrict__ dropped, const uint32_t* __restrict__ ins_oldpos,
-                          const Counters* __restrict__ c, uint2* __restrict__ out) {
+                          const Counters* __restrict__ c, const int32_t* __restrict__ lohi, uint2* __restrict__ out) {
     // the CTA's id range narrows both sorted lists once (4 searches), then every group
     // searches only its CTA's slices (empty for most CTAs)
     __shared__ uint64_t s_rng[4];
     const uint64_t n_dropped = c->n_dropped, n_vins = c->n_inserted, ng = (V + 31) / 32;
     const uint64_t gb = (uint64_t)blockIdx.x * blockDim.x;
+    // [lo, hi) widened to whole 64K-id blocks: remap_of reads the groups of a mixed block
+    constexpr uint64_t B = 1ull << kRemapBlockShift;
+    const uint64_t lo = (uint64_t)(uint32_t)lohi[0] & ~(B - 1), hi = ((uint64_t)(uint32_t)lohi[1] + B - 1) & ~(B - 1);
+    if ((gb + blockDim.x) * 32 <= lo || gb * 32 >= hi) return;  // CTA-uniform
     if (threadIdx.x < 4) {
         const uint64_t lo = gb * 32, hi = min((gb + blockDim.x) * 32, (uint64_t)0xFFFFFFFFull);
         const uint32_t x = (uint32_t)((threadIdx.x & 1) ? hi : lo);

@@ -1485,7 +1485,7 @@ __global__ void __launch_bounds__(kThreads) k_casc_scan(const uint32_t* __restri
 //   new_off[u'] = x - (cascaded before x) - (deleted before x) + (inserted records in rows < u')
 // with x = old_off[k]; the CTA narrows the sorted delete / insert-row lists first.
 #ifndef H2TAP_ROW_TILE
-#define H2TAP_ROW_TILE 512
+#define H2TAP_ROW_TILE 256
 #endif
 constexpr int kRowTile = H2TAP_ROW_TILE;  // old ids per CTA of the node-mode row pass
 struct RowArgs {
@@ -1562,7 +1562,7 @@ __global__ void k_rows_partition(RowArgs a_) {
 //   new_off[u] = x - (cascaded before x) - (deleted before x) + (inserted records in rows < u)
 // with x = old_off[k].  The CTA narrows the sorted delete / insert-row lists first.
 #ifndef H2TAP_ROWS_MINB
-#define H2TAP_ROWS_MINB 6
+#define H2TAP_ROWS_MINB 8
 #endif
 __global__ void __launch_bounds__(kThreads, H2TAP_ROWS_MINB) k_rows_fused(RowArgs a_) {
     const RowArgs a = row_counts(a_);

@@ -305,7 +305,10 @@ bool radix_sort_coop(h2tap_replica* r, uint64_t*& k, uint32_t*& v, uint64_t*& k2
                      int passes, const unsigned long long* n_dev) {
     constexpr int tile = kRsThreads * ITEMS, smem = tile * 12;
     static int occ = -1;  // per process: one device type
-    if (occ < 0) CK(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, rs_coop<ITEMS>, kRsThreads, smem));
+    if (occ < 0) {
+        CK(cudaFuncSetAttribute(rs_coop<ITEMS>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem));
+        CK(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, rs_coop<ITEMS>, kRsThreads, smem));
+    }
     const uint64_t T = cdiv(n, tile);
     if (T > (uint64_t)occ * r->n_sm) return false;
     uint32_t* cnt = r->get<uint32_t>(r->rs_coop, T * 256 + 256 + 32);
@@ -868,10 +871,10 @@ h2tap_status apply_core(h2tap_replica* r, const BatchIn& in, uint64_t S, bool cr
         ca.del_row = del_row;
         ca.upd_pos = upd_pos; ca.upd_w = upd_w;
 #ifndef H2TAP_CLASSIFY_SPLIT
-#define H2TAP_CLASSIFY_SPLIT 1
+#define H2TAP_CLASSIFY_SPLIT (1u << 16)  // edge ops from which classification and compaction are split
 #endif
         ca.c = dc;
-        if (H2TAP_CLASSIFY_SPLIT) {
+        if (n_edge >= H2TAP_CLASSIFY_SPLIT) {
             ca.kcat = r->get<uint8_t>(r->cls_cat, n_edge);
             ca.kpos = r->get<uint64_t>(r->cls_pos, n_edge);
             ca.kw = r->get<float>(r->cls_w, n_edge);

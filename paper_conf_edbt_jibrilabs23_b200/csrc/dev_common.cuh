@@ -89,6 +89,10 @@ __device__ __forceinline__ void st_volatile(uint64_t* p, uint64_t v) {
 #define H2TAP_LOOKQ 1
 #endif
 constexpr int kLookQ = H2TAP_LOOKQ;
+#ifndef H2TAP_LOOK_BACKOFF
+#define H2TAP_LOOK_BACKOFF 32
+#endif
+constexpr unsigned kLookBackoffNs = H2TAP_LOOK_BACKOFF;  // look-back re-poll delay (ns)
 __device__ __forceinline__ uint64_t lookback_warp(uint64_t* status, uint32_t tile, uint64_t aggregate) {
     if (tile == 0) {
         if (lane_id() == 0) st_volatile(&status[0], kFlagPrefix | aggregate);
@@ -106,7 +110,10 @@ __device__ __forceinline__ uint64_t lookback_warp(uint64_t* status, uint32_t til
             s[q] = (idx >= 0) ? ld_volatile(&status[idx]) : kFlagPrefix;  // virtual prefix 0 before tile 0
             not_ready |= (s[q] >> 62) == 0;
         }
-        if (__any_sync(0xffffffffu, not_ready)) continue;  // spin until all are visible (predecessors are scheduled)
+        if (__any_sync(0xffffffffu, not_ready)) {  // spin until all are visible (predecessors are scheduled),
+            __nanosleep(kLookBackoffNs);             // backing off so the polls leave L2 bandwidth to them
+            continue;
+        }
         int fq = kLookQ;  // this lane's nearest prefix
 #pragma unroll
         for (int q = kLookQ - 1; q >= 0; --q)

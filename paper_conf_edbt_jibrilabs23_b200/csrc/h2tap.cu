@@ -381,6 +381,7 @@ struct BatchIn {
     uint64_t vis_ts = ~0ull, ins_base = 0, del_base = 0;  // delta-store scan: visibility, window bases
     uint64_t pre_h2d = 0, pre_d2h = 0, pre_launches = 0;  // accounting of the record pre-pass
     const std::function<void()>* after_merge_launch = nullptr;  // host work issued behind the merge
+    cudaEvent_t input_done = nullptr;  // recorded once no kernel of the cycle reads the input arrays
     const std::function<void()>* before_readback = nullptr;     // kernels enqueued before the final read-back
 };
 
@@ -897,6 +898,18 @@ h2tap_status apply_core(h2tap_replica* r, const BatchIn& in, uint64_t S, bool cr
         TR("classify");
     }
     CK(cudaEventRecord(r->ev[3], st));
+    // ---- new pending set (double-buffered so an error above leaves the old one intact): the
+    // last reader of the input arrays, so a staged batch's slot may be refilled from here on
+    // (the next-but-one batch's H2D copy then overlaps this cycle's merge)
+    const int pn = pc ^ 1;
+    if (n_pend_new) {
+        k_gather_ops<<<g1(n_pend_new), 256, 0, st>>>(
+            ops, idx_p, n_pend_new, r->get<uint8_t>(r->pk[pn], n_pend_new), r->get<uint64_t>(r->ps[pn], n_pend_new),
+            r->get<uint64_t>(r->pd[pn], n_pend_new), r->get<float>(r->pw[pn], n_pend_new),
+            r->get<uint64_t>(r->pt[pn], n_pend_new), r->get<uint64_t>(r->pq[pn], n_pend_new));
+        CKL();
+    }
+    if (in.input_done) CK(cudaEventRecord(in.input_done, st));
 
     // ---- a6 prerequisite: the merge-path partition depends only on the outcome lists (and the
     // cascade tables, which the side stream already produces), so it runs on the side stream
@@ -1038,15 +1051,6 @@ h2tap_status apply_core(h2tap_replica* r, const BatchIn& in, uint64_t S, bool cr
         CK(cudaEventRecord(r->ev[4], st));
     }
 
-    // ---- new pending set (double-buffered so an error above leaves the old one intact)
-    const int pn = pc ^ 1;
-    if (n_pend_new) {
-        k_gather_ops<<<g1(n_pend_new), 256, 0, st>>>(
-            ops, idx_p, n_pend_new, r->get<uint8_t>(r->pk[pn], n_pend_new), r->get<uint64_t>(r->ps[pn], n_pend_new),
-            r->get<uint64_t>(r->pd[pn], n_pend_new), r->get<float>(r->pw[pn], n_pend_new),
-            r->get<uint64_t>(r->pt[pn], n_pend_new), r->get<uint64_t>(r->pq[pn], n_pend_new));
-        CKL();
-    }
     k_finish<<<1, 1, 0, st>>>(dc, V, Vr, E, node_mode ? 1 : 0, r->sharded ? 1 : 0, new_ext, new_off);
     CKL();
     CK(cudaEventRecord(r->ev[5], st));
@@ -1434,8 +1438,9 @@ h2tap_status h2tap_delta_apply(h2tap_replica* r, const h2tap_batch* b, uint64_t 
                 g.bytes = 0;
                 used = &g;
             }
+        if (used) in.input_done = used->done;  // recorded by the cycle after its last read of the slot
         const h2tap_status s = apply_core(r, in, snapshot_ts, false, stats);
-        if (used) CK(cudaEventRecord(used->done, r->st));  // after every kernel that reads the slot
+        if (used && s != H2TAP_OK) CK(cudaEventRecord(used->done, r->st));  // a refused cycle: after all it enqueued
         return s;
     });
 }

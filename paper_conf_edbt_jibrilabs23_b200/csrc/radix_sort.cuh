@@ -189,6 +189,7 @@ __global__ void __launch_bounds__(kRsThreads) rs_onesweep(
                     if (f == 2) done = true;
                 }
                 if (done) break;
+                if (q == 0) __nanosleep(kLookBackoffNs);  // nearest predecessor not published yet
                 t -= q;
             }
             st_volatile(st, kFlagPrefix | (excl + c));

@@ -311,6 +311,51 @@ def test_staged_batches_pipeline(h2):
         staged = nxt
 
 
+def test_staged_copy_behind_merge_launches(h2):
+    """A staged batch's copy waits for the latest merge launch (and for the last read of its
+    slot): staged batches interleaved with device-resident and host batches, a cycle with no
+    merge, a staged batch applied right away, and two staged at once - all as the oracle"""
+    import torch
+    src, dst, w = synth.rmat_edges(11, 35)
+    g, o = pair_from_edges(h2, 1 << 11, None, src, dst, w)
+    ts = 0
+    bs = []
+    for k in range(8):
+        b = synth.rmat_batch(11, 35, k, 3000, len(src), p_weight=0.1, ts_base=ts)
+        ts = int(b.ts.max())
+        bs.append(b)
+
+    def pin(b):
+        return Batch(*(torch.from_numpy(a.view(np.int64) if a.dtype == np.uint64 else a).pin_memory()
+                       for a in (b.kind, b.src, b.dst, b.w, b.ts)))
+
+    def dev(b):
+        return Batch(*(torch.from_numpy(a.view(np.int64) if a.dtype == np.uint64 else a).cuda()
+                       for a in (b.kind, b.src, b.dst, b.w, b.ts)))
+
+    def both(x, b):
+        st = g.apply(x, int(b.ts.max()))
+        rc, _ = o.apply(b, int(b.ts.max()))
+        assert rc == 0
+        return st
+
+    p = [pin(b) for b in bs]
+    s1 = g.stage(p[1])                      # deferred ...
+    both(dev(bs[0]), bs[0])                 # ... its copy starts behind this merge launch
+    both(s1, bs[1])
+    both(g.stage(p[2]), bs[2])              # staged and applied at once: copied by the apply
+    s3, s4 = g.stage(p[3]), g.stage(p[4])   # two outstanding
+    empty = Batch.empty(0)
+    g.apply(empty, int(bs[2].ts.max()))     # a cycle with no merge: s3 starts at its end
+    o.apply(empty, int(bs[2].ts.max()))
+    both(s3, bs[3])
+    both(s4, bs[4])
+    both(bs[5], bs[5])                      # host batch (copied inside the call)
+    s6 = g.stage(p[6])
+    both(s6, bs[6])
+    assert_same(g.export(), o.export(), "deferred staging")
+
+
 def test_chunked_create_last_duplicate_wins(h2, monkeypatch):
     """create_from_edges goes in as insert batches of H2TAP_CREATE_CHUNK edges (2^28 by
     default); duplicates across chunks: the last one wins, as in one batch"""

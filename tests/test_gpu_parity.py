@@ -311,10 +311,10 @@ def test_staged_batches_pipeline(h2):
         staged = nxt
 
 
-def test_staged_copy_behind_merge_launches(h2):
-    """A staged batch's copy waits for the latest merge launch (and for the last read of its
-    slot): staged batches interleaved with device-resident and host batches, a cycle with no
-    merge, a staged batch applied right away, and two staged at once - all as the oracle"""
+def test_staged_slots_interleaved(h2):
+    """A staged slot is refilled once the cycle that used it passed its last read of it:
+    staged batches interleaved with device-resident and host batches, a cycle with no merge,
+    a staged batch applied right away, and two staged at once - all as the oracle"""
     import torch
     src, dst, w = synth.rmat_edges(11, 35)
     g, o = pair_from_edges(h2, 1 << 11, None, src, dst, w)
@@ -340,13 +340,13 @@ def test_staged_copy_behind_merge_launches(h2):
         return st
 
     p = [pin(b) for b in bs]
-    s1 = g.stage(p[1])                      # deferred ...
-    both(dev(bs[0]), bs[0])                 # ... its copy starts behind this merge launch
+    s1 = g.stage(p[1])
+    both(dev(bs[0]), bs[0])
     both(s1, bs[1])
-    both(g.stage(p[2]), bs[2])              # staged and applied at once: copied by the apply
+    both(g.stage(p[2]), bs[2])              # staged and applied at once
     s3, s4 = g.stage(p[3]), g.stage(p[4])   # two outstanding
     empty = Batch.empty(0)
-    g.apply(empty, int(bs[2].ts.max()))     # a cycle with no merge: s3 starts at its end
+    g.apply(empty, int(bs[2].ts.max()))     # a cycle with no merge
     o.apply(empty, int(bs[2].ts.max()))
     both(s3, bs[3])
     both(s4, bs[4])

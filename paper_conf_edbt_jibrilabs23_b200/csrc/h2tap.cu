@@ -330,11 +330,15 @@ void radix_sort(h2tap_replica* r, uint64_t*& k, uint32_t*& v, uint64_t*& k2, uin
     if (n <= 1 || bits <= 0) return;
     const int passes = (bits + 7) / 8;
     if (passes <= kRsMaxPasses) {
+#ifndef H2TAP_RS_TINY
+#define H2TAP_RS_TINY (1u << 15)  // rs_coop tile: 512 keys up to here
+#endif
 #ifndef H2TAP_RS_SMALL
 #define H2TAP_RS_SMALL (1u << 18)
 #endif
-        if (n <= H2TAP_RS_SMALL ? radix_sort_coop<4>(r, k, v, k2, v2, n, passes, n_dev)
-                                : radix_sort_coop<12>(r, k, v, k2, v2, n, passes, n_dev))
+        if (n <= H2TAP_RS_TINY ? radix_sort_coop<2>(r, k, v, k2, v2, n, passes, n_dev)
+            : n <= H2TAP_RS_SMALL ? radix_sort_coop<4>(r, k, v, k2, v2, n, passes, n_dev)
+                                  : radix_sort_coop<12>(r, k, v, k2, v2, n, passes, n_dev))
             return;
     }
     const uint64_t ntiles = cdiv(n, kRsTile);

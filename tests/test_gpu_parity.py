@@ -558,3 +558,28 @@ def test_sort_heavy_duplicate_keys(h2):
     b2 = synth.rmat_batch(12, 21, 1, 30000, len(src))
     b2.ts += 5000
     step(g, o, b2, int(b2.ts.max()), "after heavy keys")
+
+
+def test_cascade_deleted_ids_spread_wide(h2):
+    """Node deletes whose ids span more than the cascade pass's shared-memory bitmap window
+    (8192 words = 262,144 ids): the pass reads the global deleted-vertex bitmap instead; and a
+    second batch whose deletes sit close together (the shared-memory window)"""
+    scale = 20
+    n = 1 << scale
+    src, dst, w = synth.rmat_edges(scale, 17, n=2 * n)
+    g, o = pair_from_edges(h2, n, None, src, dst, w)
+    deg = np.bincount(dst.astype(np.int64), minlength=n)        # vertices with in-edges
+    hubs = np.argsort(-deg)[:40]
+    ts = 1
+    ops = []
+    for v in sorted(int(x) for x in hubs) + [3, n - 5]:         # ids from 3 to n - 5
+        ops.append((NODE_DELETE, v, 0, 0.0, ts))
+        ts += 1
+    b = Batch.of(ops).concat(synth.rmat_batch(scale, 17, 0, 5000, len(src), ts_base=ts))
+    st = step(g, o, b, int(b.ts.max()), "wide node deletes")
+    assert st["n_casc"] > 0
+    ts = int(b.ts.max()) + 1
+    live = g.export()[3]
+    close = [int(x) for x in live[1000:1010]]                   # ten adjacent ids
+    b2 = Batch.of([(NODE_DELETE, v, 0, 0.0, ts + i) for i, v in enumerate(close)])
+    step(g, o, b2, ts + 20, "close node deletes")

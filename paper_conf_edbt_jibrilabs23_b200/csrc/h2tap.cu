@@ -4,7 +4,7 @@
 // replica's stream:
 //   a1 k_partition         validate, number, split pending / node ops / edge ops
 //   a2 node ops            radix sort by (v, ts, seq), k_node_segments, k_node_lists,
-//                          remap tables + k_new_ext + k_place_inserted (ID-map compaction)
+//                          remap tables (k_remap_tables) + k_node_place (ID-map compaction)
 //   a3 edge ops            k_edge_prep (lookup, gating, packed key), onesweep radix
 //                          sort, k_reduce_classify (latest-commit-wins + outcome lists)
 //   a6 k_merge             global merge path into the back buffer
@@ -444,6 +444,9 @@ ExtIndex ext_index(h2tap_replica* r) {
 #ifndef H2TAP_CASC_TMA
 #define H2TAP_CASC_TMA 1  // cascade column pass streamed by TMA, one small CTA per SM
 #endif
+#ifndef H2TAP_CC_CTAS
+#define H2TAP_CC_CTAS 8  // TMA cascade pass: CTAs per 8 SMs (fewer leave HBM headroom to the edge-op kernels)
+#endif
 #ifndef H2TAP_CASC_CTAS
 #define H2TAP_CASC_CTAS 4
 #endif
@@ -723,39 +726,12 @@ h2tap_status apply_core(h2tap_replica* r, const BatchIn& in, uint64_t S, bool cr
         ins_q = r->get<uint32_t>(r->ins_q, n_node);
         ins_oldpos = r->get<uint32_t>(r->ins_oldpos, n_node);
         hd_rows = r->get<uint32_t>(r->hd_rows, n_node);
-        k_node_lists<<<(unsigned)nt, kThreads, 0, st>>>(nv, dropped, ins_q, ins_oldpos, hd_rows, stt, nt, dc,
+        hd_bits = r->get<uint32_t>(r->hd_bits, cdiv(V, 32));  // deleted vertices (set by k_node_lists)
+        CK(cudaMemsetAsync(hd_bits, 0, cdiv(V, 32) * 4, st));
+        k_node_lists<<<(unsigned)nt, kThreads, 0, st>>>(nv, dropped, ins_q, ins_oldpos, hd_rows, hd_bits, stt, nt, dc,
                                                         r->tomb ? 1 : 0);
         CKL();
         TR("node_lists");
-        // ID-map compaction: remap tables (64K-id block shifts, 32-id groups, the
-        // unchanged / uniformly shifted id ranges), then the survivors and the inserted
-        const size_t ext_cap = r->ext[ec ^ 1].cap;  // a regrow (even at the same address) zeroes it
-        new_ext = r->get<uint64_t>(r->ext[ec ^ 1], Vn_ub);
-        idsame = r->get<unsigned long long>(r->idsame, 2);
-        if (r->ext[ec ^ 1].cap != ext_cap) CK(cudaMemsetAsync(idsame, 0, 16, st));  // fresh back buffer
-        const uint64_t nblk = cdiv(V, 1ull << kRemapBlockShift), ng = cdiv(V, 32);
-        int32_t* rs = r->get<int32_t>(r->remap_shift, nblk + 8);  // + lohi (6 entries)
-        uint2* r32 = r->get<uint2>(r->remap32, ng);
-        k_remap_blocks<<<g1(nblk), 256, 0, st>>>(V, dropped, ins_oldpos, dc, rs, rs + nblk);  // also writes c->Vn
-        CKL();
-        if (ng) { k_remap32<<<g1(ng), 256, 0, st>>>(V, dropped, ins_oldpos, dc, rs + nblk, r32); CKL(); }
-        R.shift = rs; R.g32 = r32; R.ins_oldpos = ins_oldpos; R.n_vins = &dc->n_inserted; R.lohi = rs + nblk;
-        TR("remap_tables");
-        // the inserted vertices' ID-map entries now; the survivors' entries are written
-        // by k_rows_fused together with the new row offsets
-        k_place_inserted<<<g1(n_node), 256, 0, st>>>(nv, nv_ext, ins_q, ins_oldpos, dropped, dc, new_ext);
-        CKL();
-        k_nv_newid<<<g1(n_node), 256, 0, st>>>(nv, dc, R);
-        CKL();
-        if (r->sharded) {
-            k_row_range_new<<<1, 1, 0, st>>>(dropped, ins_q, nv_ext, row_lo, row_lo + Vr, r->own, dc);
-            CKL();
-        }
-        // cascade pass (a4, reading A8): one bit per old element removed by a node delete
-        hd_bits = r->get<uint32_t>(r->hd_bits, cdiv(V, 32));
-        CK(cudaMemsetAsync(hd_bits, 0, cdiv(V, 32) * 4, st));
-        k_set_bits<<<g1(n_node), 256, 0, st>>>(hd_rows, dc, hd_bits);
-        CKL();
         const uint64_t nblk_c = cdiv(E, kCascBlock);
         casc_mask = r->get<uint32_t>(r->casc_mask, (nblk_c + 2) * (kCascBlock / 32));
         casc_cnt = r->get<uint64_t>(r->tile_emit, nblk_c + 1);
@@ -765,11 +741,11 @@ h2tap_status apply_core(h2tap_replica* r, const BatchIn& in, uint64_t S, bool cr
         uint64_t* st2s2 = r->get<uint64_t>(r->casc_status, nst);
         CK(cudaMemsetAsync(st2s2, 0, nst * 8, st));
         casc_wrel = r->get<uint16_t>(r->casc_wrel, (nblk_c + 1) * (kCascBlock / 32));
-        TR("nv_newid+bits");
-        // The cascade pass streams the old columns (HBM-bound) and nothing in the edge-op
-        // phase below (latency-bound sort / classify) reads its output, so it runs on the
-        // side stream with a grid of 4 CTAs per SM, leaving most of every SM to the edge-op
-        // kernels; the row pass joins it (casc_join) before reading the cascade tables.
+        // The cascade pass (a4, reading A8: one bit per old element removed by a node delete)
+        // streams the old columns (HBM-bound) and nothing before the row pass reads its
+        // output, so it starts as soon as the deleted vertices are known and runs on the side
+        // stream beside the remap tables and the edge-op phase; the row pass joins it
+        // (casc_join) before reading the cascade tables.
 #ifndef H2TAP_CASC_MAIN
 #define H2TAP_CASC_MAIN 0
 #endif
@@ -780,7 +756,7 @@ h2tap_status apply_core(h2tap_replica* r, const BatchIn& in, uint64_t S, bool cr
             if (H2TAP_CASC_TMA) {
                 static bool attr = false;
                 if (!attr) { CK(cudaFuncSetAttribute(k_casc_cols_tma, cudaFuncAttributeMaxDynamicSharedMemorySize, kCcSmem)); attr = true; }
-                const unsigned gc = (unsigned)std::min<uint64_t>(cdiv(E, kCcChunk), (uint64_t)r->n_sm);
+                const unsigned gc = (unsigned)std::min<uint64_t>(cdiv(E, kCcChunk), (uint64_t)r->n_sm * H2TAP_CC_CTAS / 8);
                 k_casc_cols_tma<<<gc, kCcThreads, kCcSmem, cs>>>(old_cols_nc, E, hd_bits, hd_rows, dc, casc_mask);
             } else {
                 const unsigned gc = (unsigned)std::min<uint64_t>(cdiv(nblk_c, 2), (uint64_t)r->n_sm * kCascCtasPerSm);
@@ -796,6 +772,29 @@ h2tap_status apply_core(h2tap_replica* r, const BatchIn& in, uint64_t S, bool cr
         CKL();
         CK(cudaEventRecord(r->evB, cs));
         casc_pending = true;
+        // ID-map compaction: remap tables (64K-id block shifts, 32-id groups, the
+        // unchanged / uniformly shifted id ranges), then the survivors and the inserted
+        const size_t ext_cap = r->ext[ec ^ 1].cap;  // a regrow (even at the same address) zeroes it
+        new_ext = r->get<uint64_t>(r->ext[ec ^ 1], Vn_ub);
+        idsame = r->get<unsigned long long>(r->idsame, 2);
+        if (r->ext[ec ^ 1].cap != ext_cap) CK(cudaMemsetAsync(idsame, 0, 16, st));  // fresh back buffer
+        const uint64_t nblk = cdiv(V, 1ull << kRemapBlockShift), ng = cdiv(V, 32);
+        int32_t* rs = r->get<int32_t>(r->remap_shift, nblk + 8);  // + lohi (6 entries)
+        uint2* r32 = r->get<uint2>(r->remap32, ng);
+        k_remap_tables<<<g1(std::max(nblk, ng)), 256, 0, st>>>(V, dropped, ins_oldpos, dc, rs, rs + nblk, r32);  // + c->Vn
+        CKL();
+        R.shift = rs; R.g32 = r32; R.ins_oldpos = ins_oldpos; R.n_vins = &dc->n_inserted; R.lohi = rs + nblk;
+        TR("remap_tables");
+        // the inserted vertices' ID-map entries now; the survivors' entries are written
+        // by k_rows_fused together with the new row offsets
+        // (+ the node-op vertices' new ids)
+        k_node_place<<<g1(n_node), 256, 0, st>>>(nv, nv_ext, ins_q, ins_oldpos, dropped, dc, new_ext, R);
+        CKL();
+        TR("nv_newid");
+        if (r->sharded) {
+            k_row_range_new<<<1, 1, 0, st>>>(dropped, ins_q, nv_ext, row_lo, row_lo + Vr, r->own, dc);
+            CKL();
+        }
     }
     CK(cudaEventRecord(r->ev[2], st));
     g_ht.mark("idmap");

@@ -577,7 +577,8 @@ __global__ void __launch_bounds__(kThreads) k_node_segments(
 __global__ void __launch_bounds__(kThreads) k_node_lists(
     const NodeVtx* __restrict__ nv, uint32_t* __restrict__ dropped,
     uint32_t* __restrict__ ins_q, uint32_t* __restrict__ ins_oldpos, uint32_t* __restrict__ hd_rows,
-    uint64_t* __restrict__ status3, uint64_t n_tiles_ub, Counters* __restrict__ c, int tomb) {
+    uint32_t* __restrict__ hd_bits, uint64_t* __restrict__ status3, uint64_t n_tiles_ub, Counters* __restrict__ c,
+    int tomb) {
     __shared__ uint32_t s_tile;
     __shared__ uint64_t s_scan[kThreads / 32 + 1];
     __shared__ uint64_t s_base[3];
@@ -627,7 +628,11 @@ __global__ void __launch_bounds__(kThreads) k_node_lists(
         uint64_t i = i0 + j;
         if (fl[j] & 1) dropped[o0++] = nv[i].oldpos;
         if (fl[j] & 2) { ins_q[o1] = (uint32_t)i; ins_oldpos[o1] = nv[i].oldpos; ++o1; }
-        if (fl[j] & 4) hd_rows[o2++] = nv[i].oldpos;
+        if (fl[j] & 4) {  // + its bit in the deleted-vertex bitmap of the cascade pass
+            const uint32_t v = nv[i].oldpos;
+            hd_rows[o2++] = v;
+            atomicOr(&hd_bits[v >> 5], 1u << (v & 31));
+        }
     }
 }
 
@@ -648,30 +653,32 @@ __device__ __forceinline__ uint64_t gallop_ub(const T* a, uint64_t lo, uint64_t 
 }
 
 // inserted vertex i lands at oldpos_i - (#dropped before oldpos_i) + i
-__global__ void k_place_inserted(NodeVtx* __restrict__ nv, const uint64_t* __restrict__ nv_ext,
-                                 const uint32_t* __restrict__ ins_q, const uint32_t* __restrict__ ins_oldpos,
-                                 const uint32_t* __restrict__ dropped, const Counters* __restrict__ c,
-                                 uint64_t* __restrict__ new_ext) {
-    uint64_t i = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x;
-    const uint64_t n_ins = c->n_inserted, n_dropped = c->n_dropped;
-    if (i >= n_ins) return;
-    uint32_t op = ins_oldpos[i];
-    uint64_t pos = op - lower_bound_dev(dropped, 0, n_dropped, op) + i;
-    new_ext[pos] = nv_ext[ins_q[i]];
-    nv[ins_q[i]].newid = (uint32_t)pos;
-}
 
 // new ids of surviving old vertices that have node ops
-__global__ void k_nv_newid(NodeVtx* __restrict__ nv, const Counters* __restrict__ c, RemapView R) {
-    uint64_t q = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x;
-    if (q >= c->n_unique) return;
-    uint32_t f = nv[q].flags;
-    if ((f & NV_OLD) && (f & NV_FINAL)) nv[q].newid = remap_of(R, nv[q].oldpos);
-}
 
 // tombstone mode: final liveness of the vertices with node ops in the new slots (after
 // k_rows_fused copied the old flags): present vertices keep their slot (remapped only by
 // insertions), inserted ones take their placed id
+// After the node-op lists and the remap tables (a2), one launch, thread i: the ID-map entry
+// and new id of the i-th inserted vertex (insertion point minus the dropped ids before it,
+// plus the inserted ones before it) and the new id of the i-th unique node-op vertex that
+// existed and survives
+__global__ void k_node_place(NodeVtx* __restrict__ nv, const uint64_t* __restrict__ nv_ext,
+                             const uint32_t* __restrict__ ins_q, const uint32_t* __restrict__ ins_oldpos,
+                             const uint32_t* __restrict__ dropped, const Counters* __restrict__ c,
+                             uint64_t* __restrict__ new_ext, RemapView R) {
+    const uint64_t i = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x;
+    if (i < c->n_inserted) {
+        const uint32_t op = ins_oldpos[i];
+        const uint64_t pos = op - lower_bound_dev(dropped, 0, c->n_dropped, op) + i;
+        new_ext[pos] = nv_ext[ins_q[i]];
+        nv[ins_q[i]].newid = (uint32_t)pos;
+    }
+    if (i < c->n_unique) {  // existed and survives (never an inserted vertex: no race with the above)
+        const uint32_t f = nv[i].flags;
+        if ((f & NV_OLD) && (f & NV_FINAL)) nv[i].newid = remap_of(R, nv[i].oldpos);
+    }
+}
 __global__ void k_nv_live(const NodeVtx* __restrict__ nv, const Counters* __restrict__ c, RemapView R,
                           uint8_t* __restrict__ new_live) {
     const uint64_t q = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x;
@@ -679,10 +686,6 @@ __global__ void k_nv_live(const NodeVtx* __restrict__ nv, const Counters* __rest
     const NodeVtx r = nv[q];
     const uint32_t u = (r.flags & NV_OLD) ? remap_of(R, r.oldpos) : r.newid;
     if (u != kNone32) new_live[u] = (r.flags & NV_FINAL) ? 1 : 0;
-}
-__global__ void k_set_bits(const uint32_t* __restrict__ rows, const Counters* __restrict__ c, uint32_t* __restrict__ bits) {
-    uint64_t i = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x;
-    if (i < c->n_hd) atomicOr(&bits[rows[i] >> 5], 1u << (rows[i] & 31));
 }
 
 // ===================================================================== a3 ====
@@ -2018,14 +2021,26 @@ __global__ void __launch_bounds__(kThreads) k_merge3(MergeArgs a_, const TilePar
     if (tid == 0) bulk_wait_all();
 }
 
-// per 64K-id block of old ids: constant new-id shift, or kRemapMixed if a dropped
-// id or an inserted id's insertion point lies strictly inside the block
-// Thread 0 also writes lohi = {lo, hi, shift}: below lo = min(first dropped id, first
-// insertion point) nothing moves; from hi = max(last dropped id + 1, last insertion
-// point) on, every id is shifted by n_ins - n_dropped.
-__global__ void k_remap_blocks(uint64_t V, const uint32_t* __restrict__ dropped, const uint32_t* __restrict__ ins_oldpos,
-                               Counters* __restrict__ c, int32_t* __restrict__ shift, int32_t* __restrict__ lohi) {
+
+
+
+
+
+// Remap tables in one launch (thread t: the 64K-id block t, then the 32-id group t):
+// per 64K-id block of old ids: constant new-id shift, or kRemapMixed if a dropped id or an
+// inserted id's insertion point lies strictly inside the block.  Thread 0 also writes
+// lohi = {lo, hi, shift}: below lo = min(first dropped id, first insertion point) nothing
+// moves; from hi = max(last dropped id + 1, last insertion point) on, every id is shifted by
+// n_ins - n_dropped.
+// Per 32 old ids: {new id of the group's first id (as if it survived) | exact << 31, dropped
+// bitmask}; exact = an insertion point lies strictly inside the group.  Only the groups of the
+// 64K-id blocks overlapping [lo, hi) are written: every reader (k_merge3's table path,
+// remap_of on a mixed 64K block) looks up ids there only.
+__global__ void k_remap_tables(uint64_t V, const uint32_t* __restrict__ dropped, const uint32_t* __restrict__ ins_oldpos,
+                               Counters* __restrict__ c, int32_t* __restrict__ shift, int32_t* __restrict__ lohi,
+                               uint2* __restrict__ out) {
     const uint64_t n_dropped = c->n_dropped, n_ins = c->n_inserted;
+    {
     uint64_t bk = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x;
     uint64_t nb = (V + (1u << kRemapBlockShift) - 1) >> kRemapBlockShift;
     if (bk == 0) {
@@ -2044,47 +2059,28 @@ __global__ void k_remap_blocks(uint64_t V, const uint32_t* __restrict__ dropped,
         lohi[5] = (int32_t)((int64_t)ci - (int64_t)n_dropped);
         c->Vn = V - n_dropped + n_ins;  // vertices of the new ID map
     }
-    if (bk >= nb) return;
-    uint64_t lo = bk << kRemapBlockShift, hi = min(lo + (1u << kRemapBlockShift), V);
-    uint64_t d0 = lower_bound_dev(dropped, 0, n_dropped, (uint32_t)lo);
-    uint64_t d1 = lower_bound_dev(dropped, d0, n_dropped, (uint32_t)hi);
-    uint64_t i0 = upper_bound_dev(ins_oldpos, 0, n_ins, (uint32_t)lo);      // oldpos <= lo
-    uint64_t i1 = upper_bound_dev(ins_oldpos, i0, n_ins, (uint32_t)(hi - 1));  // oldpos <= hi-1
-    shift[bk] = (d1 > d0 || i1 > i0) ? kRemapMixed : (int32_t)((int64_t)i0 - (int64_t)d0);
-}
+    if (bk < nb) {
+        uint64_t lo = bk << kRemapBlockShift, hi = min(lo + (1u << kRemapBlockShift), V);
+        uint64_t d0 = lower_bound_dev(dropped, 0, n_dropped, (uint32_t)lo);
+        uint64_t d1 = lower_bound_dev(dropped, d0, n_dropped, (uint32_t)hi);
+        uint64_t i0 = upper_bound_dev(ins_oldpos, 0, n_ins, (uint32_t)lo);      // oldpos <= lo
+        uint64_t i1 = upper_bound_dev(ins_oldpos, i0, n_ins, (uint32_t)(hi - 1));  // oldpos <= hi-1
+        shift[bk] = (d1 > d0 || i1 > i0) ? kRemapMixed : (int32_t)((int64_t)i0 - (int64_t)d0);
+    }
+    }
 
-
-
-
-
-// rows of inserted (new) vertices: kept old elements before the old position they
-// are inserted at, plus inserted records in rows < their new id
-__global__ void k_offsets_inserted(const NodeVtx* __restrict__ nv, const uint32_t* __restrict__ ins_q,
-                                   RowArgs a_) {
-    const RowArgs a = row_counts(a_);
-    uint64_t i = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x;
-    if (i >= a.n_vins) return;
-    if (!a.own.owns(a.nv_ext[ins_q[i]])) return;  // another shard's row
-    const NodeVtx& r = nv[ins_q[i]];
-    const uint64_t x = (uint64_t)a.old_off[r.oldpos];
-    const uint64_t kept = x - casc_before(a, x) - lower_bound_dev(a.del_pos, 0, a.n_del, x);
-    a.new_off[r.newid - a.row_lo_new] = (int64_t)(kept + lower_bound_dev(a.ins_row, 0, a.n_ins, r.newid));
-}
-
-// per 32 old ids: {new id of the group's first id (as if it survived) | exact << 31,
-// dropped bitmask}; exact = an insertion point lies strictly inside the group.  Only the
-// groups of the 64K-id blocks overlapping [lohi[0], lohi[1]) are written: every reader
-// (k_merge3's table path, remap_of on a mixed 64K block) looks up ids there only
-__global__ void k_remap32(uint64_t V, const uint32_t* __restrict__ dropped, const uint32_t* __restrict__ ins_oldpos,
-                          const Counters* __restrict__ c, const int32_t* __restrict__ lohi, uint2* __restrict__ out) {
     // the CTA's id range narrows both sorted lists once (4 searches), then every group
     // searches only its CTA's slices (empty for most CTAs)
     __shared__ uint64_t s_rng[4];
-    const uint64_t n_dropped = c->n_dropped, n_vins = c->n_inserted, ng = (V + 31) / 32;
+    const uint64_t n_vins = n_ins, ng = (V + 31) / 32;
     const uint64_t gb = (uint64_t)blockIdx.x * blockDim.x;
     // [lo, hi) widened to whole 64K-id blocks: remap_of reads the groups of a mixed block
     constexpr uint64_t B = 1ull << kRemapBlockShift;
-    const uint64_t lo = (uint64_t)(uint32_t)lohi[0] & ~(B - 1), hi = ((uint64_t)(uint32_t)lohi[1] + B - 1) & ~(B - 1);
+    // (lo, hi as thread 0 computes them for lohi[0], lohi[1] above)
+    const uint64_t lo0 = min(n_dropped ? (uint64_t)dropped[0] : V, n_vins ? (uint64_t)ins_oldpos[0] : V);
+    const uint64_t hi0 = max(max(n_dropped ? (uint64_t)dropped[n_dropped - 1] + 1 : (uint64_t)0,
+                                 n_vins ? (uint64_t)ins_oldpos[n_vins - 1] : (uint64_t)0), lo0);
+    const uint64_t lo = lo0 & ~(B - 1), hi = (hi0 + B - 1) & ~(B - 1);
     if ((gb + blockDim.x) * 32 <= lo || gb * 32 >= hi) return;  // CTA-uniform
     if (threadIdx.x < 4) {
         const uint64_t lo = gb * 32, hi = min((gb + blockDim.x) * 32, (uint64_t)0xFFFFFFFFull);
@@ -2104,6 +2100,21 @@ __global__ void k_remap32(uint64_t V, const uint32_t* __restrict__ dropped, cons
     for (uint64_t d = d0; d < s_rng[1] && dropped[d] < c0 + 32; ++d) m |= 1u << (dropped[d] - c0);
     out[g] = make_uint2((uint32_t)(c0 - d0 + i0) | (i1 > i0 ? 0x80000000u : 0u), m);
 }
+
+// rows of inserted (new) vertices: kept old elements before the old position they
+// are inserted at, plus inserted records in rows < their new id
+__global__ void k_offsets_inserted(const NodeVtx* __restrict__ nv, const uint32_t* __restrict__ ins_q,
+                                   RowArgs a_) {
+    const RowArgs a = row_counts(a_);
+    uint64_t i = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x;
+    if (i >= a.n_vins) return;
+    if (!a.own.owns(a.nv_ext[ins_q[i]])) return;  // another shard's row
+    const NodeVtx& r = nv[ins_q[i]];
+    const uint64_t x = (uint64_t)a.old_off[r.oldpos];
+    const uint64_t kept = x - casc_before(a, x) - lower_bound_dev(a.del_pos, 0, a.n_del, x);
+    a.new_off[r.newid - a.row_lo_new] = (int64_t)(kept + lower_bound_dev(a.ins_row, 0, a.n_ins, r.newid));
+}
+
 
 // V == ~0: the vertex count of the new ID map is c->Vn (device-side)
 __global__ void k_row_range(const uint64_t* __restrict__ ext, uint64_t V, OwnRange own, Counters* c) {

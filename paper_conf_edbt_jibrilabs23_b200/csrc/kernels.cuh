@@ -155,7 +155,7 @@ __global__ void __launch_bounds__(kThreads) k_partition(
                 tmin = min(tmin, t); tmax = max(tmax, t);
                 vmin = min(vmin, v); vmax = max(vmax, v);
             } else cat[j] = 2;
-            if (cat[j] < 3) cnt[cat[j]]++;
+            cnt[0] += cat[j] == 0; cnt[1] += cat[j] == 1; cnt[2] += cat[j] == 2;  // no dynamic index
         }
     }
     if (bad) atomicOr(&c->status, (unsigned long long)bad);
@@ -177,21 +177,25 @@ __global__ void __launch_bounds__(kThreads) k_partition(
     for (int q = 0; q < 3; ++q) excl[q] = block_exclusive_scan<kThreads>(cnt[q], s_scan, &tot[q]);
     const int wid = threadIdx.x >> 5;
     if (wid < 3) {
-        uint64_t b = lookback_warp(status3 + (uint64_t)wid * n_tiles, tile, tot[wid]);
+        const uint64_t tw = wid == 0 ? tot[0] : (wid == 1 ? tot[1] : tot[2]);  // register select
+        uint64_t b = lookback_warp(status3 + (uint64_t)wid * n_tiles, tile, tw);
         if (lane_id() == 0) {
             s_base[wid] = b;
             if (tile == n_tiles - 1) {
                 unsigned long long* dst = wid == 0 ? &c->n_pend : (wid == 1 ? &c->n_node : &c->n_edge);
-                *dst = b + tot[wid];
+                *dst = b + tw;
             }
         }
     }
     __syncthreads();
-    uint64_t o[3] = {s_base[0] + excl[0], s_base[1] + excl[1], s_base[2] + excl[2]};
-    uint32_t* outs[3] = {pend_idx, node_idx, edge_idx};
+    // three running output positions in registers (no dynamically indexed local arrays)
+    uint64_t o0 = s_base[0] + excl[0], o1 = s_base[1] + excl[1], o2 = s_base[2] + excl[2];
 #pragma unroll
     for (int j = 0; j < kItems; ++j) {
-        if (cat[j] < 3) outs[cat[j]][o[cat[j]]++] = (uint32_t)(i0 + j);
+        const uint32_t x = (uint32_t)(i0 + j);
+        if (cat[j] == 0) pend_idx[o0++] = x;
+        else if (cat[j] == 1) node_idx[o1++] = x;
+        else if (cat[j] == 2) edge_idx[o2++] = x;
     }
 }
 
@@ -612,12 +616,13 @@ __global__ void __launch_bounds__(kThreads) k_node_lists(
     for (int q = 0; q < 3; ++q) excl[q] = block_exclusive_scan<kThreads>(cnt[q], s_scan, &tot[q]);
     const int wid = threadIdx.x >> 5;
     if (wid < 3) {
-        uint64_t b = lookback_warp(status3 + (uint64_t)wid * n_tiles_ub, tile, tot[wid]);
+        const uint64_t tw = wid == 0 ? tot[0] : (wid == 1 ? tot[1] : tot[2]);  // register select
+        uint64_t b = lookback_warp(status3 + (uint64_t)wid * n_tiles_ub, tile, tw);
         if (lane_id() == 0) {
             s_base[wid] = b;
             if (tile == n_tiles - 1) {
                 unsigned long long* d = wid == 0 ? &c->n_dropped : (wid == 1 ? &c->n_inserted : &c->n_hd);
-                *d = b + tot[wid];
+                *d = b + tw;
             }
         }
     }

@@ -53,6 +53,18 @@ def test_host_only_entry_points(lib):
     assert lib.h2tap_delta_apply(None, None, ctypes.c_uint64(0), None) == -1
 
 
+def test_collective_mode_host_entry_points(lib):
+    """The collective mode's NCCL is loaded at run time: an id can be made on the host (no GPU),
+    a too-small buffer is refused, and the per-replica stats refuse a null handle."""
+    buf = ctypes.create_string_buffer(128)
+    lib.h2tap_nccl_unique_id.restype = ctypes.c_int
+    assert lib.h2tap_nccl_unique_id(buf, 128) == 0
+    assert any(buf.raw)
+    assert lib.h2tap_nccl_unique_id(buf, 16) == -1
+    lib.h2tap_collective_stats.restype = ctypes.c_int
+    assert lib.h2tap_collective_stats(None, None, None) == -1
+
+
 def test_library_is_sm100a_code():
     out = subprocess.check_output(["cuobjdump", "--list-elf", LIB]).decode()
     assert "sm_100a" in out

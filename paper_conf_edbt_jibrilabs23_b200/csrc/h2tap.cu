@@ -979,20 +979,18 @@ h2tap_status apply_core(h2tap_replica* r, const BatchIn& in, uint64_t S, bool cr
         if (V) {
             k_rows_fused<<<(unsigned)ncta, kThreads, 0, st>>>(ra);  // survivors: ID map + row offsets
             CKL();
-            k_idmap_mark<<<1, 1, 0, st>>>(idsame, R.lohi, dc, (r->tomb || !H2TAP_IDMAP_KEEP) ? 1 : 0);
-            CKL();
         } else {
             CK(cudaMemsetAsync(idsame, 0, 16, st));
         }
-        k_offsets_inserted<<<g1(n_node), 256, 0, st>>>(nv, ins_q, ra);
+        // the inserted vertices' rows, the new ID map's fence and the ID-map prefix mark
+        uint64_t* f = r->get<uint64_t>(r->fence[ec ^ 1], n_fence(Vn_ub));
+        k_rows_finish<<<std::max(g1(n_node), g1(n_fence(Vn_ub))), 256, 0, st>>>(
+            nv, ins_q, ra, new_ext, f, idsame, R.lohi, (r->tomb || !H2TAP_IDMAP_KEEP) ? 1 : 0, V ? 1 : 0);
         CKL();
         if (new_live) {  // node-op vertices' final liveness over the carried flags
             k_nv_live<<<g1(n_node), 256, 0, st>>>(nv, dc, R, new_live);
             CKL();
         }
-        uint64_t* f = r->get<uint64_t>(r->fence[ec ^ 1], n_fence(Vn_ub));
-        k_build_fence_dev<<<g1(n_fence(Vn_ub)), 256, 0, st>>>(new_ext, dc, f);
-        CKL();
     }
     // ---- a4/a5 without node ops: row offsets (while the outcome lists are L2-resident)
     if (Vr && !node_mode) {

@@ -1615,15 +1615,8 @@ __global__ void __launch_bounds__(kThreads, H2TAP_ROWS_MINB) k_rows_fused(RowArg
 
 // ID-map prefix bookkeeping (node mode).  *same: the back ID-map buffer equals the front
 // one on [0, *same).  The survivor pass rewrote the back buffer from min(*same, lo) on, so
-// it now equals the front one only below that (what an abort leaves); after the swap the
-// two buffers hold consecutive snapshots, equal below this cycle's lo.
-__global__ void k_idmap_mark(unsigned long long* same, const int32_t* __restrict__ lohi, Counters* c, int tomb) {
-    const unsigned long long lo = (unsigned long long)(uint32_t)lohi[0];
-    c->idmap_lo = lo;
-    c->idmap_keep = tomb ? 0ull : min(same[0], lo);
-    same[0] = min(same[0], lo);
-    same[1] = lo;  // what the swap makes of same[0]
-}
+// it then equals the front one only below that (what an abort leaves; k_rows_finish marks
+// it); after the swap the two buffers hold consecutive snapshots, equal below this cycle's lo.
 __global__ void k_idmap_commit(unsigned long long* same) { same[0] = same[1]; }
 
 // Row offsets without node ops (a4/a5; identity remap, no cascade): the exclusive
@@ -2106,18 +2099,30 @@ __global__ void k_remap_tables(uint64_t V, const uint32_t* __restrict__ dropped,
     out[g] = make_uint2((uint32_t)(c0 - d0 + i0) | (i1 > i0 ? 0x80000000u : 0u), m);
 }
 
-// rows of inserted (new) vertices: kept old elements before the old position they
-// are inserted at, plus inserted records in rows < their new id
-__global__ void k_offsets_inserted(const NodeVtx* __restrict__ nv, const uint32_t* __restrict__ ins_q,
-                                   RowArgs a_) {
+// After the survivor pass (node mode), one launch: the inserted vertices' row offsets (kept
+// old elements before the old position they are inserted at, plus inserted records in rows <
+// their new id), the fence of the new ID map (its size is a device count), and (thread 0,
+// mark) the ID-map prefix bookkeeping
+__global__ void k_rows_finish(const NodeVtx* __restrict__ nv, const uint32_t* __restrict__ ins_q, RowArgs a_,
+                              const uint64_t* __restrict__ new_ext, uint64_t* __restrict__ fence,
+                              unsigned long long* same, const int32_t* __restrict__ lohi, int tomb, int mark) {
     const RowArgs a = row_counts(a_);
-    uint64_t i = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x;
-    if (i >= a.n_vins) return;
-    if (!a.own.owns(a.nv_ext[ins_q[i]])) return;  // another shard's row
-    const NodeVtx& r = nv[ins_q[i]];
-    const uint64_t x = (uint64_t)a.old_off[r.oldpos];
-    const uint64_t kept = x - casc_before(a, x) - lower_bound_dev(a.del_pos, 0, a.n_del, x);
-    a.new_off[r.newid - a.row_lo_new] = (int64_t)(kept + lower_bound_dev(a.ins_row, 0, a.n_ins, r.newid));
+    const uint64_t i = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x;
+    if (mark && i == 0) {
+        const unsigned long long lo = (unsigned long long)(uint32_t)lohi[0];
+        Counters* c = const_cast<Counters*>(a.c);
+        c->idmap_lo = lo;
+        c->idmap_keep = tomb ? 0ull : min(same[0], lo);
+        same[0] = min(same[0], lo);
+        same[1] = lo;  // what the swap makes of same[0]
+    }
+    if (i < a.n_vins && a.own.owns(a.nv_ext[ins_q[i]])) {  // (another shard's row otherwise)
+        const NodeVtx& r = nv[ins_q[i]];
+        const uint64_t x = (uint64_t)a.old_off[r.oldpos];
+        const uint64_t kept = x - casc_before(a, x) - lower_bound_dev(a.del_pos, 0, a.n_del, x);
+        a.new_off[r.newid - a.row_lo_new] = (int64_t)(kept + lower_bound_dev(a.ins_row, 0, a.n_ins, r.newid));
+    }
+    if ((i << kFenceShift) < a.c->Vn) fence[i] = new_ext[i << kFenceShift];
 }
 
 
@@ -2144,12 +2149,6 @@ __global__ void k_finish(Counters* __restrict__ c, uint64_t V, uint64_t Vr, uint
     if (new_off) new_off[Vr_new] = (int64_t)En;
 }
 
-// fence of the new ID map (its size is a device count)
-__global__ void k_build_fence_dev(const uint64_t* __restrict__ ext, const Counters* __restrict__ c,
-                                  uint64_t* __restrict__ fence) {
-    uint64_t i = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x;
-    if ((i << kFenceShift) < c->Vn) fence[i] = ext[i << kFenceShift];
-}
 
 // ================================================================ checks ====
 template <typename T>

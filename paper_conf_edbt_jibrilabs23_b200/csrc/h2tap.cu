@@ -147,6 +147,8 @@ struct h2tap_replica {
     } stg[2];
     int stg_next = 0;
     cudaEvent_t evA = nullptr, evB = nullptr, evC = nullptr, evD = nullptr, evS = nullptr;
+    cudaEvent_t evE0 = nullptr, evE1 = nullptr;  // node mode: early endpoint lookups (side stream)
+    Buf epre;
     uint64_t V = 0, E = 0, snap = 0, next_seq = 0, n_pend = 0;
     // sharding: V = global live vertices (the replicated ID map), the CSR holds the Vr rows
     // of the owned external-ID range starting at global dense id row_lo
@@ -441,6 +443,9 @@ ExtIndex ext_index(h2tap_replica* r) {
 #ifndef H2TAP_IDMAP_KEEP
 #define H2TAP_IDMAP_KEEP 1  // node mode: leave the ID-map prefix both buffers already share
 #endif
+#ifndef H2TAP_EDGE_PRE
+#define H2TAP_EDGE_PRE 1  // node mode: edge endpoints looked up in the old ID map early, on the side stream
+#endif
 #ifndef H2TAP_CASC_TMA
 #define H2TAP_CASC_TMA 1  // cascade column pass streamed by TMA, one small CTA per SM
 #endif
@@ -685,6 +690,20 @@ h2tap_status apply_core(h2tap_replica* r, const BatchIn& in, uint64_t S, bool cr
     uint16_t* casc_wrel = nullptr;
     const int64_t* old_off_nc = static_cast<const int64_t*>(r->off[r->cur].p);
     const uint32_t* old_cols_nc = static_cast<const uint32_t*>(r->cols[r->cur].p);
+    // node mode: the old-map lookups of the edge ops' endpoints, on the side stream beside the
+    // node-op phase (k_edge_prep then reads them instead of searching the ID map while the
+    // cascade pass streams the columns)
+    uint32_t* epre = nullptr;
+    if (node_mode && n_edge && !r->identity && H2TAP_EDGE_PRE) {
+        epre = r->get<uint32_t>(r->epre, 2 * n_edge);
+        if (!r->evE0) CK(cudaEventCreateWithFlags(&r->evE0, cudaEventDisableTiming));
+        if (!r->evE1) CK(cudaEventCreateWithFlags(&r->evE1, cudaEventDisableTiming));
+        CK(cudaEventRecord(r->evE0, st));
+        CK(cudaStreamWaitEvent(r->st2, r->evE0, 0));
+        k_edge_oldpos<<<g1(n_edge), 256, 0, r->st2>>>(ops, idx_e, dc, ext_index(r), epre);
+        CKL();
+        CK(cudaEventRecord(r->evE1, r->st2));
+    }
     if (node_mode) {
         uint64_t* kA = r->get<uint64_t>(r->keyA, n_node);
         uint64_t* kB = r->get<uint64_t>(r->keyB, n_node);
@@ -834,6 +853,10 @@ h2tap_status apply_core(h2tap_replica* r, const BatchIn& in, uint64_t S, bool cr
         pa.keys = kA;
         pa.vals = vA;
         pa.recs = r->get<EdgeRec>(r->op_flags, m);
+        if (epre) {  // the endpoints' old-map lookups (side stream)
+            CK(cudaStreamWaitEvent(st, r->evE1, 0));
+            pa.epre = epre;
+        }
         const bool lookups_direct = r->identity && !node_mode;  // no searches -> 4 ops per thread
 #ifndef H2TAP_EI_DIRECT
 #define H2TAP_EI_DIRECT 4
@@ -1237,7 +1260,7 @@ void free_replica(h2tap_replica* r) {
                    &r->ins_oldpos, &r->hd_rows, &r->hd_bits, &r->op_flags, &r->op_ou, &r->op_ow,
                    &r->ins_pos, &r->ins_row, &r->ins_col, &r->ins_w, &r->del_pos, &r->upd_pos, &r->upd_w,
                    &r->KR, &r->cls_cat, &r->cls_pos, &r->cls_w, &r->misc, &r->nsorted, &r->part, &r->opart, &r->deg, &r->tsum, &r->remap_shift, &r->remap32, &r->casc_wrel, &r->tile_emit, &r->tile_base, &r->del_row, &r->casc_mask, &r->status2, &r->bounds_dev, &r->fence[0], &r->fence[1], &r->bfs_a, &r->bfs_b, &r->pr_a, &r->pr_b, &r->ctr,
-                   &r->xrec, &r->xins, &r->xwts, &r->xdel, &r->xcnt, &r->xoff, &r->xbig, &r->xnbig, &r->live[0], &r->live[1], &r->casc_status, &r->idsame, &r->coll, &r->coll_send, &r->coll_recv};
+                   &r->xrec, &r->xins, &r->xwts, &r->xdel, &r->xcnt, &r->xoff, &r->xbig, &r->xnbig, &r->live[0], &r->live[1], &r->casc_status, &r->idsame, &r->epre, &r->coll, &r->coll_send, &r->coll_recv};
     for (Buf* b : bufs) if (b->p) r->dfree(b->p);
     cudaStreamSynchronize(r->st);
     for (auto& e : r->ev) if (e) cudaEventDestroy(e);
@@ -1246,6 +1269,8 @@ void free_replica(h2tap_replica* r) {
     if (r->evC) cudaEventDestroy(r->evC);
     if (r->evD) cudaEventDestroy(r->evD);
     if (r->evS) cudaEventDestroy(r->evS);
+    if (r->evE0) cudaEventDestroy(r->evE0);
+    if (r->evE1) cudaEventDestroy(r->evE1);
     if (r->st2) { cudaStreamSynchronize(r->st2); cudaStreamDestroy(r->st2); }
     if (r->st_copy) { cudaStreamSynchronize(r->st_copy); cudaStreamDestroy(r->st_copy); }
     for (auto& g : r->stg) {

@@ -734,9 +734,11 @@ struct PrepArgs {
     uint64_t n_tiles;
     Counters* c;
     int count_dev;                // 1: n_edge is an upper bound, the count is c->n_edge (speculative launch)
+    const uint32_t* epre;         // node mode: old-map lookups of the endpoints of edge op i at
+                                  // [2i], [2i+1] (k_edge_oldpos: old dense id | present << 31)
 };
 
-__device__ __forceinline__ Lookup do_lookup(const PrepArgs& a, uint64_t U, uint64_t x) {
+__device__ __forceinline__ Lookup do_lookup(const PrepArgs& a, uint64_t U, uint64_t x, uint32_t pre = kNone32) {
     Lookup L;
     L.q = -1;
     L.hasD = false;
@@ -757,12 +759,29 @@ __device__ __forceinline__ Lookup do_lookup(const PrepArgs& a, uint64_t U, uint6
         }
     }
     bool present;
-    uint64_t k = old_lookup(a.X, x, &present);
+    uint64_t k;
+    if (pre != kNone32) { k = pre & 0x7FFFFFFFu; present = pre >> 31; }  // looked up earlier
+    else k = old_lookup(a.X, x, &present);
     L.oldpos = (uint32_t)k;
     L.old_present = present;
     L.final_live = L.live0 = present && (!a.X.live || a.X.live[k]);
     L.newid = present ? remap_of(a.R, (uint32_t)k) : kNone32;
     return L;
+}
+
+// Node mode: the old-map lookups of every visible edge op's endpoints (old dense id | present
+// << 31), done on the side stream while the node-op phase runs - before the cascade pass
+// saturates HBM, which would multiply the latency of these random ID-map reads inside
+// k_edge_prep
+__global__ void k_edge_oldpos(Ops ops, const uint32_t* __restrict__ edge_idx, const Counters* __restrict__ c,
+                              ExtIndex X, uint32_t* __restrict__ epre) {
+    const uint64_t i = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x;
+    if (i >= c->n_edge) return;
+    const uint32_t o = edge_idx[i];
+    bool p0, p1;
+    const uint64_t k0 = old_lookup(X, ops.src[o], &p0), k1 = old_lookup(X, ops.dst[o], &p1);
+    epre[2 * i] = (uint32_t)k0 | (p0 ? 0x80000000u : 0u);
+    epre[2 * i + 1] = (uint32_t)k1 | (p1 ? 0x80000000u : 0u);
 }
 
 // liveness of a vertex with node ops just before point (ts, seq) (reading A13)
@@ -828,8 +847,8 @@ __global__ void __launch_bounds__(kThreads) k_edge_prep(PrepArgs a) {
         uint32_t o = oj[j];
         uint8_t kind = a.ops.kind[o];
         uint64_t ts = a.ops.ts[o], seq = a.ops.seq[o];
-        Lookup Lu = do_lookup(a, U, sj[j]);
-        Lookup Lw = do_lookup(a, U, dj[j]);
+        Lookup Lu = do_lookup(a, U, sj[j], a.epre ? a.epre[2 * i] : kNone32);
+        Lookup Lw = do_lookup(a, U, dj[j], a.epre ? a.epre[2 * i + 1] : kNone32);
         bool ok = Lu.final_live && Lw.final_live;
         if (a.create && !(Lu.old_present && Lw.old_present)) nbad++;
         // routed to the wrong shard: flagged (the apply fails) and dropped here, so the

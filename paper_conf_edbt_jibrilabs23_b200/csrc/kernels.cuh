@@ -1483,18 +1483,29 @@ __global__ void __launch_bounds__(kThreads) k_casc_scan(const uint32_t* __restri
     __syncthreads();
     const uint64_t blk0 = (uint64_t)s_tile * kThreads;  // one block count per thread
     const int w = threadIdx.x >> 5;
-    for (int i = 0; i < 32; ++i) {  // warp w handles blocks blk0 + w*32 + i (2 words per lane)
-        uint64_t bk = blk0 + w * 32 + i;
-        uint32_t c = 0;
-        if (bk < nblk) {
-            const uint2 v = reinterpret_cast<const uint2*>(mask + bk * (kCascBlock / 32))[lane_id()];
-            const uint32_t c0 = __popc(v.x), c1 = __popc(v.y);
-            const uint32_t inc = warp_inclusive_scan(c0 + c1);
-            reinterpret_cast<ushort2*>(wrel + bk * (kCascBlock / 32))[lane_id()] =
-                make_ushort2((uint16_t)(inc - c0 - c1), (uint16_t)(inc - c1));
-            c = __shfl_sync(0xffffffffu, inc, 31);
+    // warp w handles blocks blk0 + w*32 + i (2 words per lane); the mask loads of 16 blocks are
+    // issued together (one dependent L2 round trip per 16 blocks, not per block)
+    for (int i0 = 0; i0 < 32; i0 += 16) {
+        uint2 vv[16];
+#pragma unroll
+        for (int i = 0; i < 16; ++i) {
+            const uint64_t bk = blk0 + w * 32 + i0 + i;
+            vv[i] = bk < nblk ? reinterpret_cast<const uint2*>(mask + bk * (kCascBlock / 32))[lane_id()]
+                              : make_uint2(0u, 0u);
         }
-        if (lane_id() == 0) s_cnt[w * 32 + i] = c;
+#pragma unroll
+        for (int i = 0; i < 16; ++i) {
+            const uint64_t bk = blk0 + w * 32 + i0 + i;
+            uint32_t c = 0;
+            if (bk < nblk) {
+                const uint32_t c0 = __popc(vv[i].x), c1 = __popc(vv[i].y);
+                const uint32_t inc = warp_inclusive_scan(c0 + c1);
+                reinterpret_cast<ushort2*>(wrel + bk * (kCascBlock / 32))[lane_id()] =
+                    make_ushort2((uint16_t)(inc - c0 - c1), (uint16_t)(inc - c1));
+                c = __shfl_sync(0xffffffffu, inc, 31);
+            }
+            if (lane_id() == 0) s_cnt[w * 32 + i0 + i] = c;
+        }
     }
     __syncthreads();
     uint64_t v = s_cnt[threadIdx.x], tot;
